@@ -1,0 +1,84 @@
+"""fp64 GraphSAGE forward / backward -- ORACLE (test infrastructure only).
+
+Follows Eq. 1: h_v^k = sigma[AGG^k({W^k h_u^{k-1} : u in N(v)})] with
+W^k of shape d' x d, AGG = mean (GraphSAGE), sigma = ReLU on
+hidden layers and identity on the output (reading Z9), bias added once after
+the aggregation (Z10), W applied after the mean (Z8: W*mean = mean(W*) in
+exact arithmetic).  Loss = sum_s CE(h^K_s, y_s) / |global batch| (Z20).
+
+bf16 mode emulates the CUDA path's rounding points (O5): features are exact
+in bf16 (O4), Z -> fp32 -> bf16 RNE, W -> bf16 RNE, everything else fp64.
+"""
+from __future__ import annotations
+
+import numpy as np
+
+from . import aggregate, aggregate_bwd, bf16_round, features
+
+
+def forward(blocks, feat_seed, dim, params, dtype="f32", x0=None):
+    """params: [(W [d_out x d_in], b [d_out])] layer 1 first.  blocks[h], hop 0 at seeds.
+    Returns a dict with per-layer Z, pre, h (fp64) and the logits."""
+    K = len(blocks)
+    assert len(params) == K
+    H = features(feat_seed, blocks[K - 1].src, dim) if x0 is None else np.asarray(x0, np.float64)
+    cache = {"Z": [], "pre": [], "h": [], "W": []}
+    for l in range(1, K + 1):
+        blk = blocks[K - l]
+        W, b = params[l - 1]
+        W = np.asarray(W, np.float64)
+        Z = aggregate(blk.indptr, blk.indices, H)
+        if dtype == "bf16":
+            Z = bf16_round(Z)
+            W = bf16_round(W)
+        pre = Z @ W.T + np.asarray(b, np.float64)
+        H = np.maximum(pre, 0.0) if l < K else pre
+        cache["Z"].append(Z)
+        cache["pre"].append(pre)
+        cache["h"].append(H)
+        cache["W"].append(W)
+    cache["logits"] = H
+    return cache
+
+
+def ce_loss_grad(logits, labels, n_global):
+    """Cross entropy summed over the seeds / n_global (Z20) and d loss / d logits."""
+    m = logits.max(axis=1, keepdims=True)
+    e = np.exp(logits - m)
+    s = e.sum(axis=1, keepdims=True)
+    logp = logits - m - np.log(s)
+    idx = np.arange(len(labels))
+    loss = -logp[idx, labels].sum() / n_global
+    g = e / s
+    g[idx, labels] -= 1.0
+    return loss, g / n_global
+
+
+def backward(blocks, cache, g_logits):
+    """Returns [(dW_l, db_l)] layer 1 first, plus per-layer g (= dL/dpre)."""
+    K = len(blocks)
+    grads = [None] * K
+    gs = [None] * K
+    g = g_logits
+    for l in range(K, 0, -1):
+        Z = cache["Z"][l - 1]
+        W = cache["W"][l - 1]
+        gs[l - 1] = g
+        grads[l - 1] = (g.T @ Z, g.sum(axis=0))
+        if l > 1:
+            blk = blocks[K - l]
+            dZ = g @ W
+            dH = aggregate_bwd(blk.indptr, blk.indices, dZ, blk.n_src)
+            g = dH * (cache["pre"][l - 2] > 0)
+    return grads, gs
+
+
+def train_step(blocks, feat_seed, dim, params, labels_of_seeds, n_global, dtype="f32", lr=None):
+    cache = forward(blocks, feat_seed, dim, params, dtype)
+    loss, g = ce_loss_grad(cache["logits"], labels_of_seeds, n_global)
+    grads, gs = backward(blocks, cache, g)
+    out = {"loss": loss, "cache": cache, "grads": grads, "g": gs}
+    if lr is not None:
+        out["new_params"] = [(np.asarray(W, np.float64) - lr * dW, np.asarray(b, np.float64) - lr * db)
+                             for (W, b), (dW, db) in zip(params, grads)]
+    return out

@@ -1,0 +1,194 @@
+"""Per-rank emulation of APT's four strategies + the Eq. 2 cost model -- ORACLE.
+
+TEST INFRASTRUCTURE ONLY.  Emulates C ranks in one process:
+it builds, for each strategy, exactly what every rank owns, sends and reads for
+the first GNN layer, and counts the paper's quantities N_d, N_vs, N_vd
+ plus the exact bytes of the message formats DESIGN.md §Messages
+fixes.  The numerical result of every strategy is the 1-GPU result (P:59,
+P:279 "semantically equivalent"), so h^1 / dW are compared against
+``oracle.model`` on the same global batch; this module pins the *structures*.
+
+Strategies (Fig. 3; Fig. 5 P:219 tensor partitioning):
+  GDP  seeds split by chunk; each rank aggregates its own blocks; remote rows
+       are read from the owning rank.
+  NFP  features split by column (d/C each); every rank receives every layer-1
+       block (AllBroadcast), computes partial projections of its
+       column slice and sends them to the requester.
+  SNP  edge-cut partition; rank c aggregates the sources it owns for every
+       destination that has >=1 sampled source in partition c, a virtual node
+       on c when c != requester; partial embeddings return to the requester
+       (P:126).
+  DNP  each layer-1 destination goes to its owning rank, which computes the
+       complete h^1 and sends it back.
+"""
+from __future__ import annotations
+
+import numpy as np
+
+STRATEGIES = ("GDP", "NFP", "SNP", "DNP")
+
+# Bandwidth-profile operator slots (DESIGN.md §Cost model; apt.h apt_bw_profile).
+OP_LOCAL_GATHER, OP_PEER_PULL, OP_PEER_PUSH, OP_ALLTOALLV, OP_ALLGATHER, OP_REDUCE_SCATTER, \
+    OP_ALLREDUCE, OP_HOST_GATHER = range(8)
+
+
+def col_range(c, C, d):
+    """NFP column slice of rank c: [floor(c*d/C), floor((c+1)*d/C))."""
+    return (c * d) // C, ((c + 1) * d) // C
+
+
+def assign_seeds(strategy, gbatch, part, C, B):
+    """O1 / Z19: GDP, NFP take contiguous chunk r of the global batch; SNP, DNP take
+    the seeds of their own partition, in permutation order (P:163 last sentence)."""
+    gbatch = np.asarray(gbatch, np.int64)
+    if strategy in ("GDP", "NFP"):
+        return [gbatch[r * B:(r + 1) * B] for r in range(C)]
+    p = part[gbatch]
+    return [gbatch[p == r] for r in range(C)]
+
+
+def msg_bytes_graph(G, n_e):
+    """Packed sub-graph message: header(2) + row_tag[G] + deg[G]
+    + indptr[G+1] + src_gid[n_e], all int32."""
+    return 4 * (2 + G + G + (G + 1) + n_e)
+
+
+def msg_bytes_ids(G):
+    """DNP request message: header(2) + row_tag[G] + dst_gid[G], int32."""
+    return 4 * (2 + 2 * G)
+
+
+def _edges(blk):
+    """(row, src_gid) for every edge of a block."""
+    rows = np.repeat(np.arange(blk.n_dst), np.diff(blk.indptr))
+    return rows, blk.src[blk.indices]
+
+
+def emulate_layer1(strategy, l1_blocks, part, C, d, d_out, feat_bytes=4, hidden_bytes=4):
+    """l1_blocks[r] = rank r's layer-1 Block (dst, src, indptr, indices).
+    Returns per-rank dict of counts and the per-rank structures."""
+    out = []
+    N_d = [b.n_dst for b in l1_blocks]
+    for r in range(C):
+        out.append(dict(n_d=N_d[r], n_vs=0, n_vd=0, rows_local=0, rows_peer=0,
+                        feat_bytes_local=0, feat_bytes_peer=0, graph_bytes=0,
+                        hidden_bytes_fwd=0, hidden_bytes_bwd=0, n_calls=0,
+                        virtual=[], requests=[]))
+    if strategy == "GDP":
+        for r, blk in enumerate(l1_blocks):
+            _, u = _edges(blk)
+            uu = np.unique(u)
+            loc = int((part[uu] == r).sum())
+            out[r]["rows_local"] = loc
+            out[r]["rows_peer"] = len(uu) - loc
+            out[r]["feat_bytes_local"] = loc * d * feat_bytes
+            out[r]["feat_bytes_peer"] = (len(uu) - loc) * d * feat_bytes
+        return out
+    if strategy == "NFP":
+        for c in range(C):
+            lo, hi = col_range(c, C, d)
+            rows = 0
+            for b, blk in enumerate(l1_blocks):
+                _, u = _edges(blk)
+                rows += len(np.unique(u))
+                if b != c:
+                    out[c]["graph_bytes"] += msg_bytes_graph(blk.n_dst, blk.n_edges)
+                    out[c]["hidden_bytes_bwd"] += blk.n_dst * d_out * hidden_bytes
+            out[c]["rows_local"] = rows
+            out[c]["feat_bytes_local"] = rows * (hi - lo) * feat_bytes
+            out[c]["hidden_bytes_fwd"] = (C - 1) * N_d[c] * d_out * hidden_bytes
+            out[c]["n_calls"] = 3 if C > 1 else 0   # graph all-gather, partial reduce, g all-gather
+        return out
+    if strategy == "SNP":
+        # groups[c] = list of (requester r, row v, [src gids in partition c])
+        recv_rows = [set() for _ in range(C)]
+        for r, blk in enumerate(l1_blocks):
+            rows, u = _edges(blk)
+            pu = part[u]
+            for c in range(C):
+                m = pu == c
+                if not m.any():
+                    continue
+                vs = np.unique(rows[m])
+                recv_rows[c].update(u[m].tolist())
+                if c != r:
+                    out[r]["n_vs"] += len(vs)
+                    out[r]["virtual"].append((c, blk.dst[vs]))
+                    out[c]["graph_bytes"] += msg_bytes_graph(len(vs), int(m.sum()))
+                    out[r]["hidden_bytes_fwd"] += len(vs) * d_out * hidden_bytes
+                    out[c]["hidden_bytes_bwd"] += len(vs) * d_out * hidden_bytes
+        for c in range(C):
+            out[c]["rows_local"] = len(recv_rows[c])
+            out[c]["feat_bytes_local"] = len(recv_rows[c]) * d * feat_bytes
+            out[c]["n_calls"] = 3 if C > 1 else 0   # graph all-to-all, partial reduce, g all-to-all
+        return out
+    if strategy == "DNP":
+        owned_rows = [set() for _ in range(C)]   # sources read by owner o
+        for r, blk in enumerate(l1_blocks):
+            rows, u = _edges(blk)
+            owner = part[blk.dst]
+            for o in range(C):
+                vs = np.nonzero(owner == o)[0]
+                if len(vs) == 0:
+                    continue
+                m = np.isin(rows, vs)
+                owned_rows[o].update(u[m].tolist())
+                if o != r:
+                    out[r]["n_vd"] += len(vs)
+                    out[r]["requests"].append((o, blk.dst[vs]))
+                    out[o]["graph_bytes"] += msg_bytes_ids(len(vs))
+                    out[r]["hidden_bytes_fwd"] += len(vs) * d_out * hidden_bytes
+                    out[o]["hidden_bytes_bwd"] += len(vs) * d_out * hidden_bytes
+        for o in range(C):
+            uu = np.fromiter(owned_rows[o], np.int64, len(owned_rows[o]))
+            loc = int((part[uu] == o).sum()) if len(uu) else 0
+            out[o]["rows_local"] = loc
+            out[o]["rows_peer"] = len(uu) - loc
+            out[o]["feat_bytes_local"] = loc * d * feat_bytes
+            out[o]["feat_bytes_peer"] = (len(uu) - loc) * d * feat_bytes
+            out[o]["n_calls"] = 3 if C > 1 else 0   # request all-to-all, h1 return, g return
+        return out
+    raise ValueError(strategy)
+
+
+def paper_volume(strategy, stats, d_out, hidden_bytes=4):
+    """The paper's closed-form T_shuffle volumes, per rank:
+    NFP 2 d' C N_d, SNP 2 d' N_vs, DNP 2 d' N_vd, GDP 0 (elements x bytes, Z14)."""
+    C = len(stats)
+    if strategy == "GDP":
+        return [0] * C
+    if strategy == "NFP":
+        return [2 * d_out * C * s["n_d"] * hidden_bytes for s in stats]
+    if strategy == "SNP":
+        return [2 * d_out * s["n_vs"] * hidden_bytes for s in stats]
+    return [2 * d_out * s["n_vd"] * hidden_bytes for s in stats]
+
+
+def predict(per_strategy_stats, alpha, beta, t_build):
+    """Eq. 2 minus the common T_train: for every strategy and rank
+    T = T_build + T_load + T_shuffle, with T_load = bytes/beta per tier and
+    T_shuffle = sum over ops (alpha * calls + bytes / beta)  (reading Z23 adds alpha).
+    per_strategy_stats[s][r] are counts summed over the dry-run epoch; t_build[s][r]
+    is the measured build time.  Predicted time = max over ranks (Z13).
+    Returns (pred[4], pick index)."""
+    pred = []
+    for si, s in enumerate(STRATEGIES):
+        worst = 0.0
+        for r, st in enumerate(per_strategy_stats[si]):
+            steps = st.get("steps", 1)
+            t = t_build[si][r]
+            t += st["feat_bytes_local"] / beta[OP_LOCAL_GATHER] + steps * alpha[OP_LOCAL_GATHER]
+            if st["feat_bytes_peer"]:
+                t += st["feat_bytes_peer"] / beta[OP_PEER_PULL] + steps * alpha[OP_PEER_PULL]
+            if s == "NFP" and st["n_calls"]:
+                t += 2 * steps * alpha[OP_ALLGATHER] + steps * alpha[OP_REDUCE_SCATTER]
+                t += st["graph_bytes"] / beta[OP_ALLGATHER]
+                t += st["hidden_bytes_fwd"] / beta[OP_REDUCE_SCATTER]
+                t += st["hidden_bytes_bwd"] / beta[OP_ALLGATHER]
+            elif s in ("SNP", "DNP") and st["n_calls"]:
+                t += 3 * steps * alpha[OP_ALLTOALLV]
+                t += (st["graph_bytes"] + st["hidden_bytes_fwd"] + st["hidden_bytes_bwd"]) / beta[OP_ALLTOALLV]
+            worst = max(worst, t)
+        pred.append(worst)
+    pick = int(np.argmin(pred))
+    return pred, pick

@@ -1,0 +1,24 @@
+import os
+import sys
+
+import pytest
+
+ROOT = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
+if ROOT not in sys.path:
+    sys.path.insert(0, ROOT)
+
+
+def pytest_configure(config):
+    config.addinivalue_line("markers", "gpu: needs a B200 (sm_100a) and the built CUDA library")
+
+
+@pytest.fixture(scope="session")
+def tiny_cfg():
+    import aptgen
+    return aptgen.CONFIGS["tiny"]
+
+
+@pytest.fixture(scope="session")
+def tiny_graph(tiny_cfg):
+    import aptgen
+    return aptgen.make_graph(tiny_cfg)

@@ -1,0 +1,153 @@
+"""Pins for the oracle's strategy emulation and cost model (-m "not gpu").
+
+The worked example of Figs. 2-3 pins the virtual-node / remote-row
+logic; closed-form volumes pin the counters; Table 1's text
+ gives directional checks.
+"""
+import numpy as np
+import pytest
+
+import aptgen
+import oracle
+from oracle import strategy as S
+
+# Fig. 2(a)/3 node names -> ids.  GPU 1 manages A,B,E,G,H; GPU 2 manages C,D,F,M,K.
+NAMES = "ABCDEFGHKM"
+ID = {c: i for i, c in enumerate(NAMES)}
+PART = np.array([0 if c in "ABEGH" else 1 for c in NAMES], np.int32)
+
+
+def hand_block(dst, edges):
+    """Hand-built layer-1 block (no sampler): dst list, {dst: [src...]}."""
+    dst_ids = np.array([ID[c] for c in dst], np.int64)
+    new = sorted({ID[u] for v in dst for u in edges.get(v, [])} - set(dst_ids.tolist()))
+    src = np.concatenate([dst_ids, np.array(new, np.int64)])
+    pos = {int(u): i for i, u in enumerate(src)}
+    indptr, indices = [0], []
+    for v in dst:
+        us = sorted(ID[u] for u in edges.get(v, []))
+        indices += [pos[u] for u in us]
+        indptr.append(len(indices))
+    return oracle.Block(1, dst_ids, src, np.array(indptr, np.int64), np.array(indices, np.int32),
+                        None, None, 0)
+
+
+@pytest.fixture
+def fig2():
+    # seed A on GPU 1: layer-1 destinations B, K; B <- G, H and K <- D, A.
+    b0 = hand_block("BK", {"B": "GH", "K": "DA"})
+    b1 = hand_block("", {})
+    return [b0, b1]
+
+
+def test_fig3_snp_one_virtual_node(fig2):
+    st = S.emulate_layer1("SNP", fig2, PART, 2, d=4, d_out=2)
+    assert st[0]["n_vs"] == 1                                  # K' on GPU 2 (source D)
+    (c, vs), = st[0]["virtual"]
+    assert c == 1 and [NAMES[v] for v in vs] == ["K"]
+    assert st[1]["rows_local"] == 1                            # GPU 2 reads only D
+    assert st[0]["rows_peer"] == st[1]["rows_peer"] == 0       # SNP reads are all local
+
+
+def test_fig3_dnp_ships_k_and_reads_a_remotely(fig2):
+    st = S.emulate_layer1("DNP", fig2, PART, 2, d=4, d_out=2)
+    assert st[0]["n_vd"] == 1                                  # K -> GPU 2
+    (o, vs), = st[0]["requests"]
+    assert o == 1 and [NAMES[v] for v in vs] == ["K"]
+    assert st[1]["rows_local"] == 1 and st[1]["rows_peer"] == 1   # D local, A remote
+    assert st[0]["rows_local"] == 2 and st[0]["rows_peer"] == 0   # G, H for B
+
+
+def test_fig3_nfp_gpu2_gets_latter_half_columns(fig2):
+    st = S.emulate_layer1("NFP", fig2, PART, 2, d=4, d_out=2)
+    assert S.col_range(1, 2, 4) == (2, 4)                      # latter-half dims
+    assert st[1]["graph_bytes"] == S.msg_bytes_graph(2, 4)     # GPU 2 receives GPU 1's graph
+    assert st[1]["rows_local"] == 4 and st[1]["feat_bytes_local"] == 4 * 2 * 4
+    assert st[0]["hidden_bytes_fwd"] == 1 * 2 * 2 * 4          # B, K partials from GPU 2
+
+
+def test_fig3_gdp_reads_d_remotely(fig2):
+    st = S.emulate_layer1("GDP", fig2, PART, 2, d=4, d_out=2)
+    assert st[0]["rows_peer"] == 1 and st[0]["rows_local"] == 3   # D remote; G, H, A local
+    assert all(s["hidden_bytes_fwd"] == 0 for s in st)        # GDP T_shuffle = 0
+
+
+def _rank_blocks(graph, cfg, C, strategy, step=0):
+    train = aptgen.train_nodes(graph, cfg)
+    perm = oracle.epoch_perm(train, cfg.sample_seed, 0)
+    gb = oracle.global_batch(perm, step, C, 64)
+    part = aptgen.partition(graph.n, C)
+    seeds = S.assign_seeds(strategy, gb, part, C, 64)
+    blocks = [oracle.sample_blocks(graph, s, cfg.fanouts, cfg.sample_seed, step)[-1] for s in seeds]
+    return blocks, part, gb, seeds
+
+
+@pytest.mark.parametrize("C", [2, 4, 8])
+def test_volumes_equal_paper_formulas(tiny_graph, tiny_cfg, C):
+    d, dd = tiny_cfg.dim, tiny_cfg.hidden
+    for s in S.STRATEGIES:
+        blocks, part, gb, seeds = _rank_blocks(tiny_graph, tiny_cfg, C, s)
+        st = S.emulate_layer1(s, blocks, part, C, d, dd)
+        counted = sum(x["hidden_bytes_fwd"] + x["hidden_bytes_bwd"] for x in st)
+        paper = sum(S.paper_volume(s, st, dd))
+        if s in ("GDP", "SNP", "DNP"):
+            assert counted == paper                             # P:146, 148, 161 exactly
+        else:
+            # P:147 counts 2 d' C N_d including each rank's own partial; the wire
+            # carries the (C-1) remote ones (reading Z15).
+            assert counted * C == paper * (C - 1)
+        assert sum(x["n_d"] for x in st) == sum(len(b.dst) for b in blocks)
+        # seed assignment is a partition of the global batch
+        assert np.array_equal(np.sort(np.concatenate(seeds)), np.sort(gb))
+
+
+@pytest.mark.parametrize("C", [2, 4, 8])
+def test_table1_directional_tradeoffs(tiny_graph, tiny_cfg, C):
+    """NFP ships the most hidden embeddings, DNP at most one per dst;
+    SNP/NFP read all features locally; only GDP and DNP read remote rows."""
+    vol = {}
+    for s in S.STRATEGIES:
+        blocks, part, _, _ = _rank_blocks(tiny_graph, tiny_cfg, C, s)
+        st = S.emulate_layer1(s, blocks, part, C, tiny_cfg.dim, tiny_cfg.hidden)
+        vol[s] = sum(x["hidden_bytes_fwd"] for x in st)
+        if s in ("SNP", "NFP"):
+            assert all(x["rows_peer"] == 0 for x in st)
+        if s == "DNP":
+            assert all(x["n_vd"] <= x["n_d"] for x in st)
+        if s == "SNP":
+            assert all(x["n_vs"] <= (C - 1) * x["n_d"] for x in st)
+    assert vol["GDP"] == 0
+    assert vol["NFP"] >= vol["SNP"] and vol["NFP"] >= vol["DNP"]
+
+
+def test_snp_dnp_degrade_under_random_partition(tiny_graph, tiny_cfg):
+    """Fig. 11: a random partition raises N_vs and N_vd."""
+    C = 4
+    good = {}
+    for part_kind in ("planted", "random"):
+        for s in ("SNP", "DNP"):
+            blocks, part, _, _ = _rank_blocks(tiny_graph, tiny_cfg, C, s)
+            if part_kind == "random":
+                part = np.random.default_rng(0).integers(0, C, tiny_graph.n).astype(np.int32)
+            st = S.emulate_layer1(s, blocks, part, C, tiny_cfg.dim, tiny_cfg.hidden)
+            good[(part_kind, s)] = sum(x["n_vs"] + x["n_vd"] for x in st)
+    assert good[("random", "SNP")] > good[("planted", "SNP")]
+    assert good[("random", "DNP")] > good[("planted", "DNP")]
+
+
+def test_cost_model_picks_argmin_and_gdp_wins_when_shuffle_is_costly():
+    mk = lambda **kw: [dict(dict(feat_bytes_local=0, feat_bytes_peer=0, graph_bytes=0,
+                                 hidden_bytes_fwd=0, hidden_bytes_bwd=0, n_calls=3, steps=1), **kw)]
+    stats = [mk(feat_bytes_local=1e9, feat_bytes_peer=1e9, n_calls=0),
+             mk(feat_bytes_local=1e8, hidden_bytes_fwd=1e10, hidden_bytes_bwd=1e10),
+             mk(feat_bytes_local=1e8, hidden_bytes_fwd=5e9, hidden_bytes_bwd=5e9),
+             mk(feat_bytes_local=1e8, hidden_bytes_fwd=2e9, hidden_bytes_bwd=2e9)]
+    alpha = [1e-5] * 8
+    beta = [1e12] * 8
+    tb = [[0.0]] * 4
+    pred, pick = S.predict(stats, alpha, beta, tb)
+    assert pick == 0 and pred[0] == pytest.approx(2e9 / 1e12 + 2e-5)
+    beta2 = list(beta)
+    beta2[S.OP_PEER_PULL] = 1e9                                # slow peer reads -> DNP
+    pred2, pick2 = S.predict(stats, alpha, beta2, tb)
+    assert pick2 == 3 and pred2[3] < pred2[2] < pred2[1]
