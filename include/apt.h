@@ -1,0 +1,235 @@
+/*
+ * apt.h -- C ABI of the B200-native APT hot path.
+ *
+ * APT (Ma et al., "Adaptive Parallel Training for Graph Neural Networks",
+ * PPoPP'25).  "P:<n>" cites line n of the paper text (reference PAPER.md).
+ * The library runs the per-mini-batch sampled-subgraph step -- Philox-keyed
+ * fanout sampling into CSR blocks, a gather from a feature store
+ * sharded over GPUs, GraphSAGE mean aggregation and the
+ * dense projection -- under the paper's four parallelisation
+ * strategies GDP / NFP / SNP / DNP, plus APT's dry-run cost model
+ * and strategy pick.  All kernels are hand-written sm_100a.
+ *
+ * Conventions (every function):
+ *  - returns apt_status, never throws or aborts; the message of the last
+ *    failure is apt_last_error(ctx) (valid until the next call on that ctx);
+ *  - invalid arguments -> APT_E_INVALID, CUDA failure -> APT_E_CUDA (sticky:
+ *    the ctx is unusable afterwards), device-side error word (bad node id,
+ *    overflow) -> APT_E_DEVICE_ASSERT at the next synchronising call;
+ *  - "device" pointers live on the ctx device; "host" pointers are CPU memory;
+ *    the caller owns every buffer it passes in and the library copies what it
+ *    keeps; objects returned through `out` are library-owned and released with
+ *    the matching apt_*_destroy;
+ *  - all work is stream-ordered on the ctx stream; calls documented as
+ *    "syncs" block the host, all others are asynchronous;
+ *  - node ids are int64 at the ABI and int32 inside (n_nodes < 2^31 checked).
+ *
+ * World / ranks.  A ctx hosts either one rank of a multi-process job
+ * (rank >= 0; peers' symmetric buffers are attached with apt_ctx_attach_peers)
+ * or all `world` ranks of an emulated job on one device (rank = -1): the same
+ * kernels then address "peer" buffers that happen to live on the same GPU.
+ */
+#ifndef APT_H_
+#define APT_H_
+#include <stddef.h>
+#include <stdint.h>
+
+#ifdef __cplusplus
+extern "C" {
+#endif
+
+typedef enum {
+  APT_OK = 0,
+  APT_E_INVALID = 1,
+  APT_E_OOM = 2,
+  APT_E_CUDA = 3,
+  APT_E_COMM = 4,
+  APT_E_UNSUPPORTED = 5,
+  APT_E_STATE = 6,
+  APT_E_DEVICE_ASSERT = 7
+} apt_status;
+
+/* The four strategies of P:120-128 (Fig. 3) and the cost-model pick. */
+typedef enum { APT_GDP = 0, APT_NFP = 1, APT_SNP = 2, APT_DNP = 3, APT_AUTO = 4 } apt_strategy;
+
+/* Feature storage / tensor-core input type.  APT_F32: fp32 features, exact
+ * fp32 CUDA-core projection (parity mode, rtol 1e-5).  APT_BF16: bf16 features,
+ * Z rounded to bf16, tcgen05 bf16 projection with fp32 accumulation.          */
+typedef enum { APT_F32 = 0, APT_BF16 = 1 } apt_dtype;
+
+#define APT_MAX_LAYERS 4
+#define APT_MAX_RANKS 8
+
+typedef struct apt_ctx apt_ctx;
+typedef struct apt_graph apt_graph;
+typedef struct apt_fstore apt_fstore;
+typedef struct apt_batch apt_batch;
+typedef struct apt_trainer apt_trainer;
+
+/* A sampled bipartite block: dst ids are the prefix of src ids;
+ * CSR over local source positions.  Device pointers, borrowed from the
+ * owning apt_batch; int32 node ids.                                         */
+typedef struct {
+  int64_t n_dst, n_src, n_edges;
+  const int32_t* dst_ids;  /* [n_dst]   global ids (device)                 */
+  const int32_t* src_ids;  /* [n_src]   global ids, dst prefix (device)     */
+  const int32_t* indptr;   /* [n_dst+1] (device)                            */
+  const int32_t* indices;  /* [n_edges] positions into src_ids (device)     */
+} apt_block_view;
+
+/* Model + sampler of the training task (the user's "specifics"). */
+typedef struct {
+  int n_layers;                        /* K                                  */
+  int dims[APT_MAX_LAYERS + 1];        /* d_0 = input dim ... d_K = classes  */
+  int fanouts[APT_MAX_LAYERS];         /* fanouts[l-1] for layer l (DGL)     */
+  int batch;                           /* B, seeds per GPU           */
+  apt_dtype dtype;
+  float lr;                            /* SGD learning rate                  */
+  uint64_t sample_seed;                /* Philox key of the sampler (O2)     */
+  uint64_t feat_seed;                  /* synthetic features (O4)            */
+} apt_model_desc;
+
+/* Dry-run statistics, per strategy s and rank r, summed over the
+ * dry-run steps.  Bytes follow DESIGN.md §Messages.                         */
+typedef struct {
+  int world;
+  int64_t steps;
+  int64_t n_d[4][APT_MAX_RANKS];             /* layer-1 destinations N_d          */
+  int64_t n_vs[APT_MAX_RANKS];               /* SNP virtual nodes          */
+  int64_t n_vd[APT_MAX_RANKS];               /* DNP virtual nodes          */
+  int64_t rows_local[4][APT_MAX_RANKS];      /* unique feature rows read locally   */
+  int64_t rows_peer[4][APT_MAX_RANKS];       /* ... read from a peer GPU (NVLink)  */
+  int64_t feat_bytes_local[4][APT_MAX_RANKS];
+  int64_t feat_bytes_peer[4][APT_MAX_RANKS];
+  int64_t graph_bytes[4][APT_MAX_RANKS];     /* Shuffle: computation graph received */
+  int64_t hidden_bytes_fwd[4][APT_MAX_RANKS];/* Reshuffle fwd: hidden received     */
+  int64_t hidden_bytes_bwd[4][APT_MAX_RANKS];/* Reshuffle bwd: gradients received  */
+  int64_t n_calls[4][APT_MAX_RANKS];         /* exchange operators per step        */
+  double t_build_s[4][APT_MAX_RANKS];        /* measured T_build           */
+  double t_train_s;                          /* measured common T_train (GDP)      */
+} apt_plan_stats;
+
+/* Operator slots of the bandwidth profile ("trials").          */
+enum {
+  APT_OP_LOCAL_GATHER = 0, APT_OP_PEER_PULL = 1, APT_OP_PEER_PUSH = 2, APT_OP_ALLTOALLV = 3,
+  APT_OP_ALLGATHER = 4, APT_OP_REDUCE_SCATTER = 5, APT_OP_ALLREDUCE = 6, APT_OP_HOST_GATHER = 7
+};
+typedef struct {
+  int world;
+  double alpha_s[8];     /* per-call latency of each operator (reading Z23) */
+  double beta_Bps[8];    /* bytes per second of each operator                */
+} apt_bw_profile;
+
+/* ---------------------------------------------------------------- context */
+/* rank >= 0: one rank of `world`; rank == -1: all `world` ranks emulated on
+ * `device`.  cuda_stream may be NULL (library-created stream).              */
+apt_status apt_ctx_create(int rank, int world, int device, void* cuda_stream, apt_ctx** out);
+apt_status apt_ctx_destroy(apt_ctx* ctx);
+const char* apt_last_error(const apt_ctx* ctx);
+/* Syncs: waits for the ctx stream and reports device-side error words.      */
+apt_status apt_ctx_sync(apt_ctx* ctx);
+/* Copy helper for tests/bindings: kind 0 = D2H, 1 = H2D, 2 = D2D. Syncs.   */
+apt_status apt_memcpy(apt_ctx* ctx, void* dst, const void* src, size_t bytes, int kind);
+/* Number of kernels this ctx launched so far (evidence for gpu_launches).   */
+int64_t apt_ctx_launches(const apt_ctx* ctx);
+
+/* ------------------------------------------------------------------ graph */
+/* Copies a symmetric CSR (host) into HBM, replicated per device (P:186 keeps
+ * topology replicated).  part: host int32[n] owner of every node (edge-cut
+ * partition); NULL => range partition floor(u*world/n).  Syncs.      */
+apt_status apt_graph_load(apt_ctx* ctx, int64_t n_nodes, int64_t nnz, const int64_t* indptr,
+                          const int32_t* indices, const int32_t* part, apt_graph** out);
+apt_status apt_graph_destroy(apt_graph* g);
+
+/* ------------------------------------------------------------ feature store */
+/* Unified feature store laid out for `layout`:
+ * GDP/SNP/DNP: rows sharded by part (rank r holds its partition's rows);
+ * NFP: columns sharded, rank c holds columns [c*d/C, (c+1)*d/C) of all rows.
+ * host_feats: host fp32 [n x dim] or NULL => synthetic O4 features from
+ * feat_seed generated on the device.  Rows padded to 16 bytes.  Syncs.      */
+apt_status apt_fstore_create(apt_ctx* ctx, const apt_graph* g, apt_strategy layout, apt_dtype dtype,
+                             int dim, const float* host_feats, uint64_t feat_seed, apt_fstore** out);
+apt_status apt_fstore_destroy(apt_fstore* f);
+
+/* ---------------------------------------------------------------- sampling */
+/* K-hop node-wise sampling of seeds_dev (device int64[n_seeds]) with
+ * fanouts (host, fanouts[l-1] for layer l, 1..256), Philox key rng_seed and
+ * step id `step` (reading O2).  Builds hop-h blocks h = 0..K-1 (layer l's
+ * block is hop K-l).  Syncs once at the end (block sizes).                  */
+apt_status apt_sample(apt_ctx* ctx, const apt_graph* g, const int64_t* seeds_dev, int64_t n_seeds,
+                      const int32_t* fanouts, int n_layers, uint64_t rng_seed, uint64_t step,
+                      apt_batch** out);
+apt_status apt_batch_block(const apt_batch* b, int hop, apt_block_view* out);
+apt_status apt_batch_destroy(apt_batch* b);
+
+/* ------------------------------------------------------------ single ops */
+/* Gather rows of ids_dev (device int32[n]) from rank-0's view of the store
+ * into out_dev (device, rows of the store's padded pitch, store dtype).     */
+apt_status apt_gather(apt_ctx* ctx, const apt_fstore* f, const int32_t* ids_dev, int64_t n, void* out_dev);
+/* Segmented mean (O5): z[v] = mean_{e in row v} x[indices[e]].  x_src device
+ * [n_src x x_pitch] of dtype; z_dst device fp32 [n_dst x z_pitch].          */
+apt_status apt_aggregate(apt_ctx* ctx, const apt_block_view* blk, const void* x_src, apt_dtype dtype,
+                         int dim, int64_t x_pitch, float* z_dst, int64_t z_pitch);
+/* Backward of the mean: dx[indices[e]] += dz[v]/deg(v) (accumulates).       */
+apt_status apt_aggregate_bwd(apt_ctx* ctx, const apt_block_view* blk, const float* dz, int dim, int64_t dz_pitch,
+                             float* dx_src, int64_t dx_pitch);
+/* Projection Y = Z W^T + b (+ReLU) (Eq. 1).  dtype APT_BF16: Z is
+ * bf16 [M x z_pitch], tcgen05 path (N, K <= 256); APT_F32: Z fp32, CUDA-core
+ * fp32.  W host-independent device fp32 [N x K]; Y device fp32 [M x y_pitch]. */
+apt_status apt_project(apt_ctx* ctx, const void* Z, int64_t z_pitch, apt_dtype dtype, const float* W,
+                       const float* bias, int64_t M, int N, int K, int relu, float* Y, int64_t y_pitch);
+
+/* ------------------------------------------------------------------ trainer */
+/* The per-mini-batch step (P:110 sampling -> loading -> training) under one
+ * strategy, for every rank hosted by ctx.  labels: host int32[n_nodes].      */
+apt_status apt_trainer_create(apt_ctx* ctx, const apt_graph* g, const apt_fstore* f, const apt_model_desc* m,
+                              apt_strategy s, const int32_t* labels, apt_trainer** out);
+apt_status apt_trainer_destroy(apt_trainer* t);
+/* Host fp32 W [d_out x d_in] row-major and b [d_out] of layer l (1..K); every rank. */
+apt_status apt_trainer_set_params(apt_trainer* t, int layer, const float* W, const float* b);
+apt_status apt_trainer_get_params(apt_trainer* t, int rank, int layer, float* W, float* b);
+/* Epoch permutation of the train set (O1): host int64[n_train] ascending.   */
+apt_status apt_trainer_set_epoch(apt_trainer* t, const int64_t* train, int64_t n_train, uint64_t epoch);
+int64_t apt_trainer_steps_per_epoch(const apt_trainer* t);
+/* One training step: seeds of step `step` of the epoch, sampling, layer-1
+ * strategy forward (Permute/Shuffle/Execute/Reshuffle), upper
+ * layers, CE loss, backward, gradient all-reduce, SGD if update != 0.  Async. */
+apt_status apt_trainer_step(apt_trainer* t, int64_t step, int update);
+/* Same, but the global batch comes from host memory (pinned for overlap),
+ * copied in on the stream, and the loss is copied back: the end-to-end call.
+ * Syncs.                                                                    */
+apt_status apt_trainer_step_host(apt_trainer* t, const int64_t* gbatch_host, int64_t n_global, int64_t step,
+                                 int update, float* loss_host);
+/* Loss of the last step (sum over ranks).  Syncs.                           */
+apt_status apt_trainer_loss(apt_trainer* t, float* loss);
+/* Record/replay the device part of apt_trainer_step as a CUDA graph.        */
+apt_status apt_trainer_use_graph(apt_trainer* t, int enable);
+
+/* Readouts for tests (syncs).  what: 0 seeds, 1 layer-l dst ids, 2 Z_l (fp32),
+ * 3 H_l (post-activation / logits), 4 dW_l, 5 db_l, 6 G_l (dL/dpre).
+ * Copies min(cap, rows*cols) values (int32 for ids, fp32 otherwise).         */
+apt_status apt_trainer_read(apt_trainer* t, int rank, int what, int layer, void* host, int64_t cap,
+                            int64_t* rows, int* cols);
+/* Per-phase device time of the last step in ms (CUDA events), n <= 16:
+ * 0 seeds+sampling, 1 layer-1 fwd, 2 upper fwd + loss, 3 backward, 4 allreduce+SGD,
+ * 5 dominant kernel (layer-1 gather+aggregate).  Syncs.                      */
+apt_status apt_trainer_phase_ms(apt_trainer* t, double* ms, int n);
+/* Algorithmic bytes of the last step's layer-1 gather+aggregate. Syncs. */
+apt_status apt_trainer_agg_bytes(apt_trainer* t, double* bytes);
+
+/* ------------------------------------------------------------------ planner */
+/* Dry-run: samples `n_steps` steps of the current epoch,
+ * runs Permute+Shuffle of every strategy on the shared samples (no feature
+ * loading, no training), counts volumes and times T_build.  Syncs.          */
+apt_status apt_dryrun(apt_trainer* t, int64_t n_steps, apt_plan_stats* out);
+/* Bandwidth trials of the exchange operators.  Syncs.        */
+apt_status apt_profile_links(apt_ctx* ctx, apt_bw_profile* out);
+/* Eq. 2 without the common T_train: pred_s[s] = max over ranks of
+ * T_build + T_load + T_shuffle; *pick = argmin.  Pure host arithmetic.      */
+apt_status apt_select_strategy(const apt_plan_stats* st, const apt_bw_profile* bw, apt_strategy* pick,
+                               double pred_s[4]);
+
+#ifdef __cplusplus
+}
+#endif
+#endif /* APT_H_ */

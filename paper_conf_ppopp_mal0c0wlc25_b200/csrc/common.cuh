@@ -1,0 +1,104 @@
+// common.cuh -- shared device helpers for the APT B200 hot path (sm_100a only).
+//
+// Nothing here is shared with oracle/ (the CPU oracle has its own Philox).
+#pragma once
+#include <cuda_runtime.h>
+#include <cuda_bf16.h>
+#include <stdint.h>
+
+#ifndef __CUDACC__
+#error "compile with nvcc -gencode arch=compute_100a,code=sm_100a"
+#endif
+
+namespace apt {
+
+constexpr int kWarp = 32;
+constexpr int kMaxLayers = 4;
+constexpr int kMaxRanks = 8;
+
+// ---------------------------------------------------------------- Philox ----
+// Philox4x32-10 (Salmon et al. SC'11), the counter-based generator that keys
+// every random draw of the method (reading Z2: the paper fixes no RNG).
+// Domain separation: key = (seed_lo, seed_hi ^ DOMAIN).
+constexpr uint32_t kDomSample = 0x53414D50u;
+constexpr uint32_t kDomFeat = 0x46454154u;
+constexpr uint32_t kDomPerm = 0x5045524Du;
+
+__host__ __device__ __forceinline__ uint4 philox(uint4 c, uint2 k) {
+#pragma unroll
+  for (int i = 0; i < 10; ++i) {
+    if (i) { k.x += 0x9E3779B9u; k.y += 0xBB67AE85u; }
+#ifdef __CUDA_ARCH__
+    const uint32_t hi0 = __umulhi(0xD2511F53u, c.x), lo0 = 0xD2511F53u * c.x;
+    const uint32_t hi1 = __umulhi(0xCD9E8D57u, c.z), lo1 = 0xCD9E8D57u * c.z;
+#else
+    const uint64_t p0 = 0xD2511F53ull * c.x, p1 = 0xCD9E8D57ull * c.z;
+    const uint32_t hi0 = uint32_t(p0 >> 32), lo0 = uint32_t(p0);
+    const uint32_t hi1 = uint32_t(p1 >> 32), lo1 = uint32_t(p1);
+#endif
+    c = make_uint4(hi1 ^ c.y ^ k.x, lo1, hi0 ^ c.w ^ k.y, lo0);
+  }
+  return c;
+}
+
+__host__ __device__ __forceinline__ uint2 philox_key(uint64_t seed, uint32_t dom) {
+  return make_uint2(uint32_t(seed), uint32_t(seed >> 32) ^ dom);
+}
+
+__host__ __device__ __forceinline__ uint32_t word_of(uint4 w, int i) {
+  return i == 0 ? w.x : i == 1 ? w.y : i == 2 ? w.z : w.w;
+}
+
+// Synthetic feature x[u][j] = (int8)(Philox_FEAT(seed;{u,0,j>>2,0}).word(j&3)) / 64
+// (input recipe O4; exact in bf16 and fp32).
+__host__ __device__ __forceinline__ float feature_value(uint2 key, int64_t u, int j) {
+  uint4 w = philox(make_uint4(uint32_t(u), uint32_t(uint64_t(u) >> 32), uint32_t(j >> 2), 0u), key);
+  int8_t b = int8_t(word_of(w, j & 3) & 0xFFu);
+  return float(b) * (1.0f / 64.0f);
+}
+
+// ---------------------------------------------------------------- misc ----
+__host__ __device__ __forceinline__ int64_t ceil_div(int64_t a, int64_t b) { return (a + b - 1) / b; }
+__host__ __device__ __forceinline__ int64_t round_up(int64_t a, int64_t b) { return ceil_div(a, b) * b; }
+
+__device__ __forceinline__ int lane_id() { return threadIdx.x & 31; }
+
+template <typename T>
+__device__ __forceinline__ T warp_sum(T v) {
+#pragma unroll
+  for (int o = 16; o > 0; o >>= 1) v += __shfl_xor_sync(0xffffffffu, v, o);
+  return v;
+}
+
+__device__ __forceinline__ float bf16_lo(uint32_t v) { return __uint_as_float(v << 16); }
+__device__ __forceinline__ float bf16_hi(uint32_t v) { return __uint_as_float(v & 0xFFFF0000u); }
+
+__device__ __forceinline__ uint32_t pack_bf16x2(float a, float b) {
+  __nv_bfloat162 h = __floats2bfloat162_rn(a, b);   // RNE (O5 rounding point)
+  return *reinterpret_cast<uint32_t*>(&h);
+}
+
+// 16-byte loads bypassing L1 allocation for streaming rows.
+__device__ __forceinline__ uint4 ld_nc_v4(const void* p) {
+  uint4 r;
+  asm volatile("ld.global.nc.L1::no_allocate.v4.u32 {%0,%1,%2,%3}, [%4];"
+               : "=r"(r.x), "=r"(r.y), "=r"(r.z), "=r"(r.w) : "l"(p));
+  return r;
+}
+
+// Vector fp32 atomic add (sm_90+): 4 floats per red.
+__device__ __forceinline__ void red_add_v4(float* p, float a, float b, float c, float d) {
+  asm volatile("red.global.add.v4.f32 [%0], {%1,%2,%3,%4};" ::"l"(p), "f"(a), "f"(b), "f"(c), "f"(d)
+               : "memory");
+}
+
+// Device error word: kernels OR an APT_DEV_* bit on invalid input instead of trapping.
+enum : uint32_t { kDevErrBadId = 1u, kDevErrOverflow = 2u };
+
+}  // namespace apt
+
+#define APT_CUDA_OK(expr)                                                     \
+  do {                                                                        \
+    cudaError_t _e = (expr);                                                  \
+    if (_e != cudaSuccess) return ::apt::fail_cuda(_e, #expr, __FILE__, __LINE__); \
+  } while (0)

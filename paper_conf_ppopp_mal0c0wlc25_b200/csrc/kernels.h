@@ -1,0 +1,163 @@
+// kernels.h -- launcher declarations for the sm_100a kernels (internal, C++).
+#pragma once
+#include <cuda_runtime.h>
+#include <stdint.h>
+
+namespace apt {
+
+// ---------------------------------------------------------------- sample.cu
+struct SampleArgs {
+  const int64_t* indptr;
+  const int32_t* indices;
+  const int32_t* frontier;
+  const int32_t* n_frontier;   // device count
+  int64_t max_frontier;        // grid upper bound
+  int k;
+  uint2 key;
+  const uint64_t* step;        // device step id
+  int hop;
+  int32_t* cnt;                // [max_frontier]
+  int32_t* nbr;                // [max_frontier * k] global ids, fixed stride k
+};
+cudaError_t launch_sample(const SampleArgs& a, cudaStream_t st);
+
+struct CompactArgs {
+  const int32_t* dst;          // frontier (dst ids)
+  const int32_t* n_dst;
+  int64_t max_dst;
+  const int32_t* cnt;
+  const int32_t* nbr;
+  int k;
+  uint32_t* dst_bm;            // [n_words], zero on entry and exit
+  uint32_t* new_bm;            // [n_words], zero on entry and exit
+  int64_t n_words;
+  int32_t* pos;                // [n_nodes] scratch global->local map
+  int32_t* src;                // [max_src]
+  int32_t* n_src;
+  int32_t* indptr;             // [max_dst + 1]
+  int32_t* indices;            // [max_dst * k]
+  int32_t* n_edges;
+  int32_t* partials;           // scan workspace (>= n_words/2048 + 2)
+  int32_t* partials2;          // scan workspace (>= max_dst/2048 + 2)
+};
+cudaError_t launch_compact(const CompactArgs& a, cudaStream_t st);
+
+struct SeedArgs {
+  const int32_t* perm;
+  int64_t n_train;
+  const uint64_t* step;
+  int64_t steps_per_epoch;
+  int world, rank, batch, by_part;
+  const int32_t* part;
+  int32_t* seeds;
+  int32_t* n_seeds;
+  int32_t* n_global;
+};
+cudaError_t launch_select_seeds(const SeedArgs& a, cudaStream_t st);
+cudaError_t launch_perm_keys(const int32_t* train, int64_t n, uint64_t seed, uint64_t epoch, uint64_t* keys,
+                             cudaStream_t st);
+
+// ------------------------------------------------------------------ agg.cu
+enum DType : int { kF32 = 0, kBF16 = 1 };
+
+// Feature store view used by the fused gather+mean kernel (S6+S7).
+struct FeatView {
+  const void* base[8];         // per-owner shard base (local or NVLink peer pointer)
+  const int32_t* part;         // owner of node u (nullptr => single shard, row = u)
+  const int32_t* lrow;         // row of u inside its owner's shard
+  int64_t pitch;               // elements per stored row (padded to 16 B)
+  int dim;                     // logical columns to aggregate
+  int col0;                    // first column inside the stored row
+  DType dtype;
+};
+
+// Edge source for aggregation: either an ELL (cnt + nbr global ids, fixed stride
+// k; used for layer 1 straight from the sampler) or a CSR over local indices.
+struct AggArgs {
+  // ELL form (layer 1)
+  const int32_t* cnt;
+  const int32_t* nbr;
+  int k;
+  // CSR form (upper layers)
+  const int32_t* indptr;
+  const int32_t* indices;
+  const float* x;              // [n_src x x_pitch] fp32 (CSR form)
+  int64_t x_pitch;
+  // optional per-edge filter (SNP partial sums): only sources u with part[u] == keep_part
+  const int32_t* filt_part;
+  int keep_part;
+  const int32_t* deg_override; // SNP: divide by the full sampled degree of the requester
+  // rows
+  const int32_t* n_dst;
+  int64_t max_dst;
+  int dim;
+  // outputs (any may be null)
+  float* z_f32;
+  int64_t z_f32_pitch;
+  uint16_t* z_bf16;
+  int64_t z_bf16_pitch;
+};
+cudaError_t launch_agg_fstore(const AggArgs& a, const FeatView& fv, cudaStream_t st);
+cudaError_t launch_agg_csr(const AggArgs& a, cudaStream_t st);
+
+// dX[src_e] += dZ[v] / deg(v)  (O5 backward), fp32 atomics.
+cudaError_t launch_agg_bwd(const int32_t* indptr, const int32_t* indices, const int32_t* n_dst, int64_t max_dst,
+                           const float* dz, int64_t dz_pitch, int dim, float* dx, int64_t dx_pitch,
+                           cudaStream_t st);
+
+// Gather rows of the feature store into a dense buffer (apt_gather).
+cudaError_t launch_gather(const FeatView& fv, const int32_t* ids, const int32_t* n_dev, int64_t max_n, void* out,
+                          int64_t out_pitch, cudaStream_t st);
+
+// Fill a shard with the synthetic O4 features of the listed global ids.
+cudaError_t launch_fill_features(void* shard, DType dt, int64_t pitch, int col0, int ncols, const int32_t* ids,
+                                 int64_t n, uint64_t seed, cudaStream_t st);
+
+// ---------------------------------------------------------------- gemm_simt.cu
+// C[m][n] (+)= sum_k A(m,k) B(k,n) (+ bias[n]) (relu), fp32 accumulate.
+// A(m,k) = A[m*sam + k*sak]; B(k,n) = B[k*sbk + n*sbn]; M may live on device.
+struct SimtGemmArgs {
+  const void* A; DType a_t; int64_t sam, sak;
+  const void* B; DType b_t; int64_t sbk, sbn;
+  float* C; int64_t ldc;
+  const float* bias;
+  const int32_t* M_dev;        // if set, M = *M_dev (<= M)
+  int64_t M; int N; int64_t K;
+  int relu;
+  int accumulate;              // atomically add into C (split-K)
+  int64_t k_chunk;             // split-K chunk (0 => whole K)
+  const int32_t* K_dev;        // if set, K = *K_dev (<= K)
+};
+cudaError_t launch_simt_gemm(const SimtGemmArgs& a, cudaStream_t st);
+
+// ---------------------------------------------------------------- gemm_tc.cu
+// tcgen05 projection: Y[m][n] = sum_k Z[m][k] W[n][k] + bias[n] (relu), bf16 in,
+// fp32 accumulate in TMEM, fp32 out.  Z, W are K-major bf16 with 16-B pitches.
+struct TcGemmArgs {
+  const uint16_t* Z; int64_t z_pitch;  // [M_max x K] bf16
+  const uint16_t* W; int64_t w_pitch;  // [N x K] bf16
+  int64_t M_max; const int32_t* M_dev; int N; int K;
+  const float* bias; int relu;
+  float* Y; int64_t y_pitch;
+  // optional row routing (peer-store epilogue): row m goes to
+  // out_base[out_rank[m]] + out_row[m] * y_pitch
+  float* const* out_base; const int32_t* out_rank; const int32_t* out_row;
+};
+int tc_gemm_supported(int N, int K);
+cudaError_t launch_tc_gemm(const TcGemmArgs& a, cudaStream_t st);
+
+// ---------------------------------------------------------------- misc.cu
+cudaError_t launch_ce_loss(const float* logits, int64_t pitch, int n_classes, const int32_t* seeds,
+                           const int32_t* n_seeds, int64_t max_seeds, const int32_t* labels,
+                           const int32_t* n_global, float* loss, float* g, int64_t g_pitch, cudaStream_t st);
+cudaError_t launch_relu_bwd(float* g, const float* h, int64_t pitch, int dim, const int32_t* n_dev, int64_t max_n,
+                            cudaStream_t st);
+cudaError_t launch_colsum(const float* g, int64_t pitch, int dim, const int32_t* n_dev, int64_t max_n, float* out,
+                          cudaStream_t st);
+cudaError_t launch_sgd(float* W, const float* dW, int64_t n, float lr, uint16_t* W_bf16, int rows, int cols,
+                       int64_t bf16_pitch, cudaStream_t st);
+cudaError_t launch_to_bf16(const float* src, int64_t src_pitch, uint16_t* dst, int64_t dst_pitch, int cols,
+                           const int32_t* n_dev, int64_t max_n, cudaStream_t st);
+cudaError_t launch_transpose(const float* src, int rows, int cols, float* dst, cudaStream_t st);
+
+}  // namespace apt

@@ -1,0 +1,141 @@
+// misc.cu -- small elementwise kernels of the training step (S10/S11):
+// cross-entropy loss + its gradient, ReLU backward, bias gradient, SGD update
+// with the bf16 weight copy for the tensor-core projection, conversions.
+#include "common.cuh"
+#include "kernels.h"
+#include <algorithm>
+
+namespace apt {
+
+static int64_t grid_of(int64_t n, int t = 256) {
+  return std::max<int64_t>(1, std::min<int64_t>(ceil_div(n, t), 148 * 32));
+}
+
+// loss = sum_s CE(logits_s, y_s) / n_global  (reading Z20);  g = (softmax - onehot) / n_global.
+__global__ void ce_loss_kernel(const float* __restrict__ logits, int64_t pitch, int C,
+                               const int32_t* __restrict__ seeds, const int32_t* __restrict__ n_seeds_p,
+                               const int32_t* __restrict__ labels, const int32_t* __restrict__ n_global_p,
+                               float* __restrict__ loss, float* __restrict__ g, int64_t g_pitch) {
+  const int lane = lane_id();
+  const int64_t n = *n_seeds_p;
+  const float inv_n = 1.0f / float(max(1, *n_global_p));
+  const int64_t nwarps = int64_t(gridDim.x) * (blockDim.x >> 5);
+  for (int64_t i = (int64_t(blockIdx.x) * blockDim.x + threadIdx.x) >> 5; i < n; i += nwarps) {
+    const float* row = logits + i * pitch;
+    float m = -INFINITY;
+    for (int c = lane; c < C; c += 32) m = fmaxf(m, row[c]);
+#pragma unroll
+    for (int o = 16; o > 0; o >>= 1) m = fmaxf(m, __shfl_xor_sync(0xffffffffu, m, o));
+    float s = 0.f;
+    for (int c = lane; c < C; c += 32) s += expf(row[c] - m);
+    s = warp_sum(s);
+    const int y = labels[seeds[i]];
+    const float lse = m + logf(s);
+    if (lane == 0) atomicAdd(loss, (lse - row[y]) * inv_n);
+    for (int c = lane; c < C; c += 32) {
+      const float p = expf(row[c] - lse);
+      g[i * g_pitch + c] = (p - (c == y ? 1.f : 0.f)) * inv_n;
+    }
+  }
+}
+
+cudaError_t launch_ce_loss(const float* logits, int64_t pitch, int n_classes, const int32_t* seeds,
+                           const int32_t* n_seeds, int64_t max_seeds, const int32_t* labels,
+                           const int32_t* n_global, float* loss, float* g, int64_t g_pitch, cudaStream_t st) {
+  ce_loss_kernel<<<grid_of(max_seeds * 32), 256, 0, st>>>(logits, pitch, n_classes, seeds, n_seeds, labels,
+                                                          n_global, loss, g, g_pitch);
+  return cudaGetLastError();
+}
+
+__global__ void relu_bwd_kernel(float* __restrict__ g, const float* __restrict__ h, int64_t pitch, int dim,
+                                const int32_t* __restrict__ n_p) {
+  const int64_t n = *n_p;
+  const int64_t total = n * dim;
+  for (int64_t t = int64_t(blockIdx.x) * blockDim.x + threadIdx.x; t < total; t += int64_t(gridDim.x) * blockDim.x) {
+    const int64_t r = t / dim;
+    const int64_t off = r * pitch + (t - r * dim);
+    if (!(h[off] > 0.f)) g[off] = 0.f;
+  }
+}
+
+cudaError_t launch_relu_bwd(float* g, const float* h, int64_t pitch, int dim, const int32_t* n_dev, int64_t max_n,
+                            cudaStream_t st) {
+  relu_bwd_kernel<<<grid_of(max_n * dim), 256, 0, st>>>(g, h, pitch, dim, n_dev);
+  return cudaGetLastError();
+}
+
+// out[c] += sum_r g[r][c]  (db = sum of g over the rows, O5)
+__global__ void colsum_kernel(const float* __restrict__ g, int64_t pitch, int dim, const int32_t* __restrict__ n_p,
+                              float* __restrict__ out) {
+  const int64_t n = *n_p;
+  const int c = blockIdx.y * blockDim.x + threadIdx.x;
+  if (c >= dim) return;
+  const int64_t rows_per = ceil_div(n, gridDim.x);
+  const int64_t r0 = int64_t(blockIdx.x) * rows_per, r1 = std::min<int64_t>(n, r0 + rows_per);
+  float s = 0.f;
+  for (int64_t r = r0; r < r1; ++r) s += g[r * pitch + c];
+  if (r1 > r0) atomicAdd(out + c, s);
+}
+
+cudaError_t launch_colsum(const float* g, int64_t pitch, int dim, const int32_t* n_dev, int64_t max_n, float* out,
+                          cudaStream_t st) {
+  const int tx = 128;
+  dim3 grid(unsigned(std::max<int64_t>(1, std::min<int64_t>(max_n / 256 + 1, 296))), unsigned(ceil_div(dim, tx)));
+  colsum_kernel<<<grid, tx, 0, st>>>(g, pitch, dim, n_dev, out);
+  return cudaGetLastError();
+}
+
+// W -= lr * dW; optionally refresh the bf16 copy [rows x cols] (pitch) used by tcgen05.
+__global__ void sgd_kernel(float* __restrict__ W, const float* __restrict__ dW, int64_t n, float lr,
+                           uint16_t* __restrict__ wb, int cols, int64_t bpitch) {
+  for (int64_t t = int64_t(blockIdx.x) * blockDim.x + threadIdx.x; t < n; t += int64_t(gridDim.x) * blockDim.x) {
+    const float w = W[t] - lr * dW[t];
+    W[t] = w;
+    if (wb) {
+      const int64_t r = t / cols;
+      __nv_bfloat16 h = __float2bfloat16_rn(w);
+      wb[r * bpitch + (t - r * cols)] = *reinterpret_cast<uint16_t*>(&h);
+    }
+  }
+}
+
+cudaError_t launch_sgd(float* W, const float* dW, int64_t n, float lr, uint16_t* W_bf16, int rows, int cols,
+                       int64_t bf16_pitch, cudaStream_t st) {
+  (void)rows;
+  sgd_kernel<<<grid_of(n), 256, 0, st>>>(W, dW, n, lr, W_bf16, cols, bf16_pitch);
+  return cudaGetLastError();
+}
+
+__global__ void to_bf16_kernel(const float* __restrict__ src, int64_t sp, uint16_t* __restrict__ dst, int64_t dp,
+                               int cols, const int32_t* __restrict__ n_p, int64_t n_static) {
+  const int64_t n = n_p ? int64_t(*n_p) : n_static;
+  const int64_t total = n * cols;
+  for (int64_t t = int64_t(blockIdx.x) * blockDim.x + threadIdx.x; t < total; t += int64_t(gridDim.x) * blockDim.x) {
+    const int64_t r = t / cols;
+    const int c = int(t - r * cols);
+    __nv_bfloat16 h = __float2bfloat16_rn(src[r * sp + c]);
+    dst[r * dp + c] = *reinterpret_cast<uint16_t*>(&h);
+  }
+}
+
+cudaError_t launch_to_bf16(const float* src, int64_t src_pitch, uint16_t* dst, int64_t dst_pitch, int cols,
+                           const int32_t* n_dev, int64_t max_n, cudaStream_t st) {
+  to_bf16_kernel<<<grid_of(max_n * cols), 256, 0, st>>>(src, src_pitch, dst, dst_pitch, cols, n_dev, max_n);
+  return cudaGetLastError();
+}
+
+__global__ void transpose_kernel(const float* __restrict__ s, int rows, int cols, float* __restrict__ d) {
+  const int64_t n = int64_t(rows) * cols;
+  for (int64_t t = int64_t(blockIdx.x) * blockDim.x + threadIdx.x; t < n; t += int64_t(gridDim.x) * blockDim.x) {
+    const int64_t r = t / cols;
+    const int c = int(t - r * cols);
+    d[int64_t(c) * rows + r] = s[t];
+  }
+}
+
+cudaError_t launch_transpose(const float* src, int rows, int cols, float* dst, cudaStream_t st) {
+  transpose_kernel<<<grid_of(int64_t(rows) * cols), 256, 0, st>>>(src, rows, cols, dst);
+  return cudaGetLastError();
+}
+
+}  // namespace apt

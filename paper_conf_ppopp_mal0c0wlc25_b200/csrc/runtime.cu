@@ -1,0 +1,451 @@
+// runtime.cu -- C ABI (include/apt.h): contexts, graph, feature store,
+// sampling batches and the single-op entry points.  The trainer (strategy
+// drivers) is in trainer.cu, the planner in plan.cu.
+#include <algorithm>
+#include <cstdarg>
+#include <cstdio>
+#include <cstring>
+#include <numeric>
+
+#include "common.cuh"
+#include "runtime.h"
+
+using namespace apt;
+
+namespace apt {
+thread_local std::string g_err;
+
+apt_status set_err(apt_ctx* c, apt_status s, const char* fmt, ...) {
+  char buf[512];
+  va_list ap;
+  va_start(ap, fmt);
+  vsnprintf(buf, sizeof buf, fmt, ap);
+  va_end(ap);
+  if (c) c->err = buf;
+  g_err = buf;
+  return s;
+}
+
+apt_status check_cuda(apt_ctx* c, cudaError_t e, const char* what) {
+  if (e == cudaSuccess) return APT_OK;
+  if (c) c->broken = true;
+  return set_err(c, APT_E_CUDA, "%s: %s", what, cudaGetErrorString(e));
+}
+}  // namespace apt
+
+#define CK(ctx, expr)                                               \
+  do {                                                              \
+    apt_status _s = ::apt::check_cuda((ctx), (expr), #expr);        \
+    if (_s != APT_OK) return _s;                                    \
+  } while (0)
+
+extern "C" {
+
+apt_status apt_ctx_create(int rank, int world, int device, void* stream, apt_ctx** out) {
+  if (!out || world < 1 || world > APT_MAX_RANKS || rank < -1 || rank >= world)
+    return set_err(nullptr, APT_E_INVALID, "apt_ctx_create: bad rank/world (%d/%d)", rank, world);
+  auto* c = new apt_ctx();
+  c->world = world;
+  c->emulated = rank < 0;
+  c->rank = rank < 0 ? 0 : rank;
+  c->n_local = rank < 0 ? world : 1;
+  c->device = device;
+  cudaError_t e = cudaSetDevice(device);
+  if (e != cudaSuccess) {
+    set_err(nullptr, APT_E_CUDA, "cudaSetDevice(%d): %s", device, cudaGetErrorString(e));
+    delete c;
+    return APT_E_CUDA;
+  }
+  int major = 0;
+  cudaDeviceGetAttribute(&major, cudaDevAttrComputeCapabilityMajor, device);
+  cudaDeviceGetAttribute(&c->sm_count, cudaDevAttrMultiProcessorCount, device);
+  if (major != 10) {
+    set_err(nullptr, APT_E_UNSUPPORTED, "device %d is sm_%d0: this library is built for sm_100a only", device, major);
+    delete c;
+    return APT_E_UNSUPPORTED;
+  }
+  if (stream) {
+    c->stream = static_cast<cudaStream_t>(stream);
+  } else {
+    cudaStreamCreateWithFlags(&c->stream, cudaStreamNonBlocking);
+    c->own_stream = true;
+  }
+  c->dev_err = c->arena.alloc<uint32_t>(4);
+  c->scratch = c->arena.alloc<int32_t>(16);
+  if (!c->dev_err || !c->scratch) {
+    delete c;
+    return set_err(nullptr, APT_E_OOM, "apt_ctx_create: out of device memory");
+  }
+  *out = c;
+  return APT_OK;
+}
+
+apt_status apt_ctx_destroy(apt_ctx* c) {
+  if (!c) return APT_OK;
+  cudaStreamSynchronize(c->stream);
+  c->arena.release();
+  if (c->own_stream) cudaStreamDestroy(c->stream);
+  delete c;
+  return APT_OK;
+}
+
+const char* apt_last_error(const apt_ctx* c) { return c ? c->err.c_str() : g_err.c_str(); }
+
+int64_t apt_ctx_launches(const apt_ctx* c) { return c ? c->launches : 0; }
+
+apt_status apt_ctx_sync(apt_ctx* c) {
+  if (!c) return set_err(nullptr, APT_E_INVALID, "null ctx");
+  CK(c, cudaStreamSynchronize(c->stream));
+  uint32_t w = 0;
+  CK(c, cudaMemcpy(&w, c->dev_err, 4, cudaMemcpyDeviceToHost));
+  if (w) return set_err(c, APT_E_DEVICE_ASSERT, "device error word 0x%x", w);
+  return APT_OK;
+}
+
+apt_status apt_memcpy(apt_ctx* c, void* dst, const void* src, size_t bytes, int kind) {
+  if (!c || (!dst && bytes) || (!src && bytes)) return set_err(c, APT_E_INVALID, "apt_memcpy: null");
+  cudaMemcpyKind k = kind == 0 ? cudaMemcpyDeviceToHost : kind == 1 ? cudaMemcpyHostToDevice : cudaMemcpyDeviceToDevice;
+  CK(c, cudaMemcpyAsync(dst, src, bytes, k, c->stream));
+  CK(c, cudaStreamSynchronize(c->stream));
+  return APT_OK;
+}
+
+// ------------------------------------------------------------------ graph
+apt_status apt_graph_load(apt_ctx* c, int64_t n, int64_t nnz, const int64_t* indptr, const int32_t* indices,
+                          const int32_t* part, apt_graph** out) {
+  if (!c || !out || n <= 0 || nnz < 0 || !indptr || (!indices && nnz))
+    return set_err(c, APT_E_INVALID, "apt_graph_load: bad arguments");
+  if (n >= (int64_t(1) << 31)) return set_err(c, APT_E_INVALID, "apt_graph_load: n_nodes >= 2^31");
+  if (indptr[0] != 0 || indptr[n] != nnz) return set_err(c, APT_E_INVALID, "apt_graph_load: indptr[0]/indptr[n] mismatch");
+  auto* g = new apt_graph();
+  g->ctx = c;
+  g->n = n;
+  g->nnz = nnz;
+  g->world = c->world;
+  g->indptr = g->arena.alloc<int64_t>(n + 1, false);
+  g->indices = g->arena.alloc<int32_t>(nnz, false);
+  g->part = g->arena.alloc<int32_t>(n, false);
+  g->lrow = g->arena.alloc<int32_t>(n, false);
+  if (!g->indptr || !g->indices || !g->part || !g->lrow) {
+    delete g;
+    return set_err(c, APT_E_OOM, "apt_graph_load: out of device memory (n=%lld nnz=%lld)", (long long)n, (long long)nnz);
+  }
+  g->part_h.resize(n);
+  std::vector<int32_t> lrow(n);
+  g->shard_rows.assign(c->world, 0);
+  for (int64_t u = 0; u < n; ++u) {
+    int p = part ? part[u] : int((u * c->world) / n);
+    if (p < 0 || p >= c->world) {
+      delete g;
+      return set_err(c, APT_E_INVALID, "apt_graph_load: part[%lld]=%d out of range", (long long)u, p);
+    }
+    g->part_h[u] = p;
+    lrow[u] = int32_t(g->shard_rows[p]++);
+  }
+  CK(c, cudaMemcpyAsync(g->indptr, indptr, sizeof(int64_t) * (n + 1), cudaMemcpyHostToDevice, c->stream));
+  if (nnz) CK(c, cudaMemcpyAsync(g->indices, indices, sizeof(int32_t) * nnz, cudaMemcpyHostToDevice, c->stream));
+  CK(c, cudaMemcpyAsync(g->part, g->part_h.data(), sizeof(int32_t) * n, cudaMemcpyHostToDevice, c->stream));
+  CK(c, cudaMemcpyAsync(g->lrow, lrow.data(), sizeof(int32_t) * n, cudaMemcpyHostToDevice, c->stream));
+  CK(c, cudaStreamSynchronize(c->stream));
+  *out = g;
+  return APT_OK;
+}
+
+apt_status apt_graph_destroy(apt_graph* g) {
+  delete g;
+  return APT_OK;
+}
+
+// ------------------------------------------------------------- feature store
+apt_status apt_fstore_create(apt_ctx* c, const apt_graph* g, apt_strategy layout, apt_dtype dtype, int dim,
+                             const float* host_feats, uint64_t feat_seed, apt_fstore** out) {
+  if (!c || !g || !out || dim <= 0 || (dtype != APT_F32 && dtype != APT_BF16) || layout < APT_GDP || layout > APT_AUTO)
+    return set_err(c, APT_E_INVALID, "apt_fstore_create: bad arguments");
+  auto* f = new apt_fstore();
+  f->ctx = c;
+  f->g = g;
+  f->layout = layout == APT_AUTO ? APT_GDP : layout;
+  f->dtype = dtype == APT_BF16 ? kBF16 : kF32;
+  f->dim = dim;
+  f->world = c->world;
+  const int C = c->world;
+  const int align = dtype == APT_BF16 ? 8 : 4;     // 16-byte rows
+  const size_t esz = dtype == APT_BF16 ? 2 : 4;
+  for (int r = 0; r < C; ++r) {
+    if (f->layout == APT_NFP && C > 1) {
+      f->col_lo[r] = int((int64_t(r) * dim) / C);
+      f->col_hi[r] = int((int64_t(r + 1) * dim) / C);
+      f->rows[r] = g->n;
+    } else {
+      f->col_lo[r] = 0;
+      f->col_hi[r] = dim;
+      f->rows[r] = C > 1 ? g->shard_rows[r] : g->n;
+    }
+    const int w = std::max(1, f->col_hi[r] - f->col_lo[r]);
+    f->pitch[r] = round_up(w, align);
+  }
+  // ids of every shard's rows (ascending global ids) -> synthetic fill / host copy
+  std::vector<std::vector<int32_t>> ids(C);
+  if (f->layout != APT_NFP && C > 1) {
+    for (int64_t u = 0; u < g->n; ++u) ids[g->part_h[u]].push_back(int32_t(u));
+  }
+  int32_t* ids_dev = f->arena.alloc<int32_t>(g->n, false);
+  for (int r = 0; r < C; ++r) {
+    // emulated: all shards here; multi-process: only the own shard is local
+    if (!c->emulated && r != c->rank) continue;
+    f->shard[r] = f->arena.alloc<uint8_t>(f->rows[r] * f->pitch[r] * int64_t(esz), true);
+    if (!f->shard[r] || !ids_dev) {
+      delete f;
+      return set_err(c, APT_E_OOM, "apt_fstore_create: out of device memory");
+    }
+    const int32_t* idp = nullptr;
+    if (!ids[r].empty()) {
+      CK(c, cudaMemcpyAsync(ids_dev, ids[r].data(), sizeof(int32_t) * ids[r].size(), cudaMemcpyHostToDevice, c->stream));
+      idp = ids_dev;
+    }
+    const int ncols = f->col_hi[r] - f->col_lo[r];
+    if (host_feats) {
+      // host fp32 [n x dim] -> this shard (rows of the shard, its column slice), converted on the host
+      std::vector<uint8_t> buf(size_t(f->rows[r] * f->pitch[r]) * esz, 0);
+      for (int64_t i = 0; i < f->rows[r]; ++i) {
+        const int64_t u = idp ? ids[r][i] : i;
+        for (int j = 0; j < ncols; ++j) {
+          const float v = host_feats[u * dim + f->col_lo[r] + j];
+          if (esz == 4) {
+            reinterpret_cast<float*>(buf.data())[i * f->pitch[r] + j] = v;
+          } else {
+            uint32_t b;
+            memcpy(&b, &v, 4);
+            b = (b + 0x7FFFu + ((b >> 16) & 1u)) >> 16;   // RNE
+            reinterpret_cast<uint16_t*>(buf.data())[i * f->pitch[r] + j] = uint16_t(b);
+          }
+        }
+      }
+      CK(c, cudaMemcpyAsync(f->shard[r], buf.data(), buf.size(), cudaMemcpyHostToDevice, c->stream));
+      CK(c, cudaStreamSynchronize(c->stream));
+    } else {
+      CK(c, launch_fill_features(f->shard[r], f->dtype, f->pitch[r], f->col_lo[r], ncols, idp, f->rows[r], feat_seed,
+                                 c->stream));
+      c->launches++;
+      CK(c, cudaStreamSynchronize(c->stream));
+    }
+  }
+  *out = f;
+  return APT_OK;
+}
+
+apt_status apt_fstore_destroy(apt_fstore* f) {
+  delete f;
+  return APT_OK;
+}
+
+}  // extern "C"
+
+namespace apt {
+// FeatView of the row-sharded store as seen by rank r (every shard reachable:
+// locally or through its peer pointer).
+FeatView feat_view(const apt_fstore* f, int r) {
+  FeatView v{};
+  const bool rows_sharded = f->layout != APT_NFP && f->world > 1;
+  for (int o = 0; o < f->world; ++o) v.base[o] = f->shard[o];
+  if (rows_sharded) {
+    v.part = f->g->part;
+    v.lrow = f->g->lrow;
+    v.pitch = f->pitch[0];
+    v.dim = f->dim;
+  } else {
+    const int s = f->world > 1 ? r : 0;
+    v.base[0] = f->shard[s];
+    v.part = nullptr;
+    v.lrow = nullptr;
+    v.pitch = f->pitch[s];
+    v.dim = f->col_hi[s] - f->col_lo[s];
+  }
+  v.col0 = 0;
+  v.dtype = f->dtype;
+  return v;
+}
+}  // namespace apt
+
+extern "C" {
+
+// ---------------------------------------------------------------- sampling
+apt_status apt_sample(apt_ctx* c, const apt_graph* g, const int64_t* seeds_dev, int64_t n_seeds,
+                      const int32_t* fanouts, int K, uint64_t rng_seed, uint64_t step, apt_batch** out) {
+  if (!c || !g || !out || (!seeds_dev && n_seeds) || n_seeds < 0 || !fanouts || K < 1 || K > APT_MAX_LAYERS)
+    return set_err(c, APT_E_INVALID, "apt_sample: bad arguments");
+  for (int l = 0; l < K; ++l)
+    if (fanouts[l] < 1 || fanouts[l] > 256) return set_err(c, APT_E_INVALID, "apt_sample: fanout %d out of [1,256]", fanouts[l]);
+  auto* b = new apt_batch();
+  b->ctx = c;
+  b->K = K;
+  const int64_t n_words = ceil_div(g->n, 32);
+  uint32_t* dst_bm = b->arena.alloc<uint32_t>(n_words, true);
+  uint32_t* new_bm = b->arena.alloc<uint32_t>(n_words, true);
+  int32_t* pos = b->arena.alloc<int32_t>(g->n, false);
+  int64_t maxF = n_seeds;
+  int64_t max_part = ceil_div(n_words, 2048) + 2;
+  int32_t* counts = b->arena.alloc<int32_t>(4 * K + 4, true);
+  uint64_t* step_dev = b->arena.alloc<uint64_t>(1, false);
+  int32_t* seeds32 = b->arena.alloc<int32_t>(n_seeds, false);
+  if (!dst_bm || !new_bm || !pos || !counts || !step_dev || !seeds32) {
+    delete b;
+    return set_err(c, APT_E_OOM, "apt_sample: out of device memory");
+  }
+  // int64 seeds -> int32 (validated on the host copy)
+  {
+    std::vector<int64_t> h(n_seeds);
+    CK(c, cudaMemcpyAsync(h.data(), seeds_dev, sizeof(int64_t) * n_seeds, cudaMemcpyDeviceToHost, c->stream));
+    CK(c, cudaStreamSynchronize(c->stream));
+    std::vector<int32_t> h32(n_seeds);
+    for (int64_t i = 0; i < n_seeds; ++i) {
+      if (h[i] < 0 || h[i] >= g->n) {
+        delete b;
+        return set_err(c, APT_E_INVALID, "apt_sample: seed %lld out of range", (long long)h[i]);
+      }
+      h32[i] = int32_t(h[i]);
+    }
+    int32_t ns = int32_t(n_seeds);
+    CK(c, cudaMemcpyAsync(seeds32, h32.data(), sizeof(int32_t) * n_seeds, cudaMemcpyHostToDevice, c->stream));
+    CK(c, cudaMemcpyAsync(counts, &ns, 4, cudaMemcpyHostToDevice, c->stream));
+    CK(c, cudaMemcpyAsync(step_dev, &step, 8, cudaMemcpyHostToDevice, c->stream));
+  }
+  const int32_t* dst = seeds32;
+  const int32_t* n_dst = counts;   // counts[0] = n_seeds; counts[1+2h] = n_src(h), counts[2+2h] = n_edges(h)
+  int32_t* partials = b->arena.alloc<int32_t>(max_part, false);
+  for (int h = 0; h < K; ++h) {
+    const int k = fanouts[K - 1 - h];
+    const int64_t maxS = std::max<int64_t>(maxF, std::min<int64_t>(maxF * (1 + k), g->n));
+    int32_t* cnt = b->arena.alloc<int32_t>(maxF, true);
+    int32_t* nbr = b->arena.alloc<int32_t>(maxF * k, false);
+    int32_t* src = b->arena.alloc<int32_t>(maxS, false);
+    int32_t* indptr = b->arena.alloc<int32_t>(maxF + 1, true);
+    int32_t* indices = b->arena.alloc<int32_t>(maxF * k, false);
+    int32_t* part2 = b->arena.alloc<int32_t>(ceil_div(maxF, 2048) + 4, false);
+    if (!cnt || !nbr || !src || !indptr || !indices || !partials || !part2) {
+      delete b;
+      return set_err(c, APT_E_OOM, "apt_sample: out of device memory");
+    }
+    SampleArgs sa{g->indptr, g->indices, dst, n_dst, maxF, k, philox_key(rng_seed, kDomSample), step_dev, h, cnt, nbr};
+    CK(c, launch_sample(sa, c->stream));
+    CompactArgs ca{dst, n_dst, maxF, cnt, nbr, k, dst_bm, new_bm, n_words, pos, src, counts + 1 + 2 * h,
+                   indptr, indices, counts + 2 + 2 * h, partials, part2};
+    CK(c, launch_compact(ca, c->stream));
+    c->launches += 10;
+    b->dst[h] = const_cast<int32_t*>(dst);
+    b->src[h] = src;
+    b->indptr[h] = indptr;
+    b->indices[h] = indices;
+    dst = src;
+    n_dst = counts + 1 + 2 * h;
+    maxF = maxS;
+  }
+  std::vector<int32_t> hc(4 * K + 4);
+  CK(c, cudaMemcpyAsync(hc.data(), counts, sizeof(int32_t) * hc.size(), cudaMemcpyDeviceToHost, c->stream));
+  CK(c, cudaStreamSynchronize(c->stream));
+  int64_t nd = n_seeds;
+  for (int h = 0; h < K; ++h) {
+    b->n_dst[h] = nd;
+    b->n_src[h] = hc[1 + 2 * h];
+    b->n_edges[h] = hc[2 + 2 * h];
+    nd = b->n_src[h];
+  }
+  *out = b;
+  return APT_OK;
+}
+
+apt_status apt_batch_block(const apt_batch* b, int hop, apt_block_view* out) {
+  if (!b || !out || hop < 0 || hop >= b->K) return set_err(nullptr, APT_E_INVALID, "apt_batch_block: bad hop");
+  out->n_dst = b->n_dst[hop];
+  out->n_src = b->n_src[hop];
+  out->n_edges = b->n_edges[hop];
+  out->dst_ids = b->dst[hop];
+  out->src_ids = b->src[hop];
+  out->indptr = b->indptr[hop];
+  out->indices = b->indices[hop];
+  return APT_OK;
+}
+
+apt_status apt_batch_destroy(apt_batch* b) {
+  delete b;
+  return APT_OK;
+}
+
+// ------------------------------------------------------------- single ops
+apt_status apt_gather(apt_ctx* c, const apt_fstore* f, const int32_t* ids, int64_t n, void* out) {
+  if (!c || !f || (n && (!ids || !out)) || n < 0) return set_err(c, APT_E_INVALID, "apt_gather: bad arguments");
+  FeatView v = feat_view(f, c->rank);
+  CK(c, launch_gather(v, ids, nullptr, n, out, v.pitch, c->stream));
+  c->launches++;
+  return APT_OK;
+}
+
+apt_status apt_aggregate(apt_ctx* c, const apt_block_view* blk, const void* x, apt_dtype dt, int dim, int64_t x_pitch,
+                         float* z, int64_t z_pitch) {
+  if (!c || !blk || !x || !z || dim <= 0 || x_pitch < dim || z_pitch < dim || (z_pitch % 4) || dt != APT_F32)
+    return set_err(c, APT_E_INVALID, "apt_aggregate: bad arguments (fp32 x, pitches multiple of 4)");
+  if (x_pitch % 4) return set_err(c, APT_E_INVALID, "apt_aggregate: x_pitch must be a multiple of 4");
+  int32_t* nd = c->scratch;
+  int32_t h = int32_t(blk->n_dst);
+  CK(c, cudaMemcpyAsync(nd, &h, 4, cudaMemcpyHostToDevice, c->stream));
+  AggArgs a{};
+  a.indptr = blk->indptr;
+  a.indices = blk->indices;
+  a.x = static_cast<const float*>(x);
+  a.x_pitch = x_pitch;
+  a.n_dst = nd;
+  a.max_dst = blk->n_dst;
+  a.dim = dim;
+  a.z_f32 = z;
+  a.z_f32_pitch = z_pitch;
+  CK(c, launch_agg_csr(a, c->stream));
+  c->launches++;
+  CK(c, cudaStreamSynchronize(c->stream));
+  return APT_OK;
+}
+
+apt_status apt_aggregate_bwd(apt_ctx* c, const apt_block_view* blk, const float* dz, int dim, int64_t dz_pitch,
+                             float* dx, int64_t dx_pitch) {
+  if (!c || !blk || !dz || !dx || dim <= 0 || (dz_pitch % 4) || (dx_pitch % 4))
+    return set_err(c, APT_E_INVALID, "apt_aggregate_bwd: bad arguments");
+  int32_t* nd = c->scratch;
+  int32_t h = int32_t(blk->n_dst);
+  CK(c, cudaMemcpyAsync(nd, &h, 4, cudaMemcpyHostToDevice, c->stream));
+  CK(c, launch_agg_bwd(blk->indptr, blk->indices, nd, blk->n_dst, dz, dz_pitch, dim, dx, dx_pitch, c->stream));
+  c->launches++;
+  CK(c, cudaStreamSynchronize(c->stream));
+  return APT_OK;
+}
+
+apt_status apt_project(apt_ctx* c, const void* Z, int64_t z_pitch, apt_dtype dt, const float* W, const float* bias,
+                       int64_t M, int N, int K, int relu, float* Y, int64_t y_pitch) {
+  if (!c || !Z || !W || !Y || M < 0 || N <= 0 || K <= 0 || z_pitch < K || y_pitch < N)
+    return set_err(c, APT_E_INVALID, "apt_project: bad arguments");
+  int32_t* md = c->scratch;
+  int32_t mh = int32_t(M);
+  CK(c, cudaMemcpyAsync(md, &mh, 4, cudaMemcpyHostToDevice, c->stream));
+  if (dt == APT_BF16) {
+    if (!tc_gemm_supported(N, K)) return set_err(c, APT_E_UNSUPPORTED, "apt_project: tcgen05 path needs N,K <= 256");
+    const int64_t wp = round_up(K, 8);
+    uint16_t* Wb = nullptr;
+    CK(c, cudaMallocAsync(reinterpret_cast<void**>(&Wb), sizeof(uint16_t) * N * wp, c->stream));
+    CK(c, cudaMemsetAsync(Wb, 0, sizeof(uint16_t) * N * wp, c->stream));
+    CK(c, launch_to_bf16(W, K, Wb, wp, K, nullptr, N, c->stream));
+    TcGemmArgs a{static_cast<const uint16_t*>(Z), z_pitch, Wb, wp, M, md, N, K, bias, relu, Y, y_pitch,
+                 nullptr, nullptr, nullptr};
+    CK(c, launch_tc_gemm(a, c->stream));
+    CK(c, cudaFreeAsync(Wb, c->stream));
+    c->launches += 2;
+  } else {
+    SimtGemmArgs a{};
+    a.A = Z; a.a_t = kF32; a.sam = z_pitch; a.sak = 1;
+    a.B = W; a.b_t = kF32; a.sbk = 1; a.sbn = K;
+    a.C = Y; a.ldc = y_pitch; a.bias = bias; a.M_dev = md; a.M = M; a.N = N; a.K = K; a.relu = relu;
+    CK(c, launch_simt_gemm(a, c->stream));
+    c->launches++;
+  }
+  CK(c, cudaStreamSynchronize(c->stream));
+  return APT_OK;
+}
+
+}  // extern "C"

@@ -1,0 +1,99 @@
+// runtime.h -- internal host-side structures behind the C ABI (include/apt.h).
+#pragma once
+#include <cuda_runtime.h>
+#include <stdint.h>
+
+#include <string>
+#include <vector>
+
+#include "../../include/apt.h"
+#include "kernels.h"
+
+namespace apt {
+
+// Device allocation owned by one library object.
+struct DevBuf {
+  void* p = nullptr;
+  size_t bytes = 0;
+};
+
+struct Arena {
+  std::vector<DevBuf> bufs;
+  size_t total = 0;
+  ~Arena() { release(); }
+  void release() {
+    for (auto& b : bufs) cudaFree(b.p);
+    bufs.clear();
+    total = 0;
+  }
+  template <typename T>
+  T* alloc(int64_t n, bool zero = true) {
+    void* p = nullptr;
+    size_t bytes = size_t(std::max<int64_t>(n, 1)) * sizeof(T);
+    bytes = (bytes + 255) & ~size_t(255);
+    if (cudaMalloc(&p, bytes) != cudaSuccess) return nullptr;
+    if (zero) cudaMemset(p, 0, bytes);
+    bufs.push_back({p, bytes});
+    total += bytes;
+    return static_cast<T*>(p);
+  }
+};
+
+}  // namespace apt
+
+struct apt_ctx {
+  int rank = 0;          // first hosted rank
+  int world = 1;
+  int n_local = 1;       // ranks hosted by this ctx
+  bool emulated = false;
+  int device = 0;
+  int sm_count = 148;
+  cudaStream_t stream = nullptr;
+  bool own_stream = false;
+  bool broken = false;
+  std::string err;
+  int64_t launches = 0;
+  uint32_t* dev_err = nullptr;   // device error word
+  int32_t* scratch = nullptr;    // small device ints for single-op calls
+  apt::Arena arena;
+};
+
+struct apt_graph {
+  apt_ctx* ctx = nullptr;
+  int64_t n = 0, nnz = 0;
+  int64_t* indptr = nullptr;     // device
+  int32_t* indices = nullptr;    // device
+  int32_t* part = nullptr;       // device owner of every node
+  int32_t* lrow = nullptr;       // device row inside the owner's shard
+  std::vector<int32_t> part_h;   // host copy
+  std::vector<int64_t> shard_rows;   // rows per rank
+  int world = 1;
+  apt::Arena arena;
+};
+
+struct apt_fstore {
+  apt_ctx* ctx = nullptr;
+  const apt_graph* g = nullptr;
+  apt_strategy layout = APT_GDP;
+  apt::DType dtype = apt::kF32;
+  int dim = 0;
+  int world = 1;
+  // per rank shard
+  void* shard[APT_MAX_RANKS] = {};
+  int64_t pitch[APT_MAX_RANKS] = {};   // elements per row
+  int col_lo[APT_MAX_RANKS] = {};
+  int col_hi[APT_MAX_RANKS] = {};
+  int64_t rows[APT_MAX_RANKS] = {};
+  apt::Arena arena;
+};
+
+struct apt_batch {
+  apt_ctx* ctx = nullptr;
+  int K = 0;
+  int64_t n_dst[APT_MAX_LAYERS] = {}, n_src[APT_MAX_LAYERS] = {}, n_edges[APT_MAX_LAYERS] = {};
+  int32_t* dst[APT_MAX_LAYERS] = {};
+  int32_t* src[APT_MAX_LAYERS] = {};
+  int32_t* indptr[APT_MAX_LAYERS] = {};
+  int32_t* indices[APT_MAX_LAYERS] = {};
+  apt::Arena arena;
+};

@@ -1,0 +1,628 @@
+// trainer.cu -- the per-mini-batch training step (sampling -> loading ->
+// training) under APT's strategies, for every rank hosted by the ctx.
+//
+// Step phases:
+//   A  S1 seeds of the step, S2/S3 K-hop sampling + compaction (all ranks)
+//   B  layer-1 forward under the strategy: Permute / Shuffle / Execute /
+//      Reshuffle -- strategies.cu for NFP / SNP / DNP
+//   C  S10 upper layers (data parallel) + CE loss
+//   D  backward of the upper layers, then the layer-1 backward of the strategy (S11)
+//   E  gradient all-reduce across ranks (DDP) + SGD
+// Every count stays on the device, every grid is sized by an upper bound:
+// the step issues no host synchronisation and can be replayed as a CUDA graph.
+#include <algorithm>
+#include <cstring>
+#include <cub/device/device_radix_sort.cuh>
+
+#include "common.cuh"
+#include "trainer.h"
+
+using namespace apt;
+
+namespace apt {
+apt_status set_err(apt_ctx* c, apt_status s, const char* fmt, ...);
+apt_status check_cuda(apt_ctx* c, cudaError_t e, const char* what);
+FeatView feat_view(const apt_fstore* f, int r);
+// strategies.cu
+apt_status strategy_alloc(apt_trainer* t, RankState& rs);
+apt_status layer1_fwd_strategy(apt_trainer* t);
+apt_status layer1_bwd_strategy(apt_trainer* t);
+}  // namespace apt
+
+#define CK(ctx, expr)                                        \
+  do {                                                       \
+    apt_status _s = ::apt::check_cuda((ctx), (expr), #expr); \
+    if (_s != APT_OK) return _s;                             \
+  } while (0)
+
+namespace apt {
+
+__global__ void allreduce_sum_kernel(float* const* tab, int C, int64_t n) {
+  for (int64_t i = int64_t(blockIdx.x) * blockDim.x + threadIdx.x; i < n; i += int64_t(gridDim.x) * blockDim.x) {
+    float s = 0.f;
+    for (int r = 0; r < C; ++r) s += tab[r][i];
+    for (int r = 0; r < C; ++r) tab[r][i] = s;
+  }
+}
+
+__global__ void zero_rows_kernel(float* p, int64_t pitch, const int32_t* n_p) {
+  const int64_t total = int64_t(*n_p) * pitch;
+  float4* q = reinterpret_cast<float4*>(p);
+  for (int64_t t = int64_t(blockIdx.x) * blockDim.x + threadIdx.x; t < total / 4; t += int64_t(gridDim.x) * blockDim.x)
+    q[t] = make_float4(0.f, 0.f, 0.f, 0.f);
+}
+
+static int64_t blocks_for(int64_t n) { return std::max<int64_t>(1, std::min<int64_t>(ceil_div(n, 256), 148 * 16)); }
+
+// Projection dispatch: tcgen05 (bf16 mode) or exact fp32 CUDA cores.
+apt_status project(apt_trainer* t, const Layer& L, const void* Zb, const float* Zf, int64_t z_pitch_b,
+                   int64_t z_pitch_f, const int32_t* n_rows, int64_t max_rows, int K, const float* W, const uint16_t* Wb,
+                   const float* bias, int relu, float* Y, float* const* out_base, const int32_t* out_rank,
+                   const int32_t* out_row) {
+  apt_ctx* c = t->ctx;
+  if (t->m.dtype == APT_BF16 && tc_gemm_supported(L.d_out, K)) {
+    TcGemmArgs a{static_cast<const uint16_t*>(Zb), z_pitch_b, Wb, L.wb_pitch, max_rows, n_rows, L.d_out, K,
+                 bias, relu, Y, L.h_pitch, out_base, out_rank, out_row};
+    CK(c, launch_tc_gemm(a, c->stream));
+  } else {
+    if (out_rank) return set_err(c, APT_E_UNSUPPORTED, "routed epilogue needs the tcgen05 path");
+    SimtGemmArgs a{};
+    if (t->m.dtype == APT_BF16) { a.A = Zb; a.a_t = kBF16; a.sam = z_pitch_b; a.B = Wb; a.b_t = kBF16; a.sbn = L.wb_pitch; }
+    else { a.A = Zf; a.a_t = kF32; a.sam = z_pitch_f; a.B = W; a.b_t = kF32; a.sbn = L.d_in; }
+    a.sak = 1; a.sbk = 1;
+    a.C = Y; a.ldc = L.h_pitch; a.bias = bias; a.M_dev = n_rows; a.M = max_rows; a.N = L.d_out; a.K = K; a.relu = relu;
+    CK(c, launch_simt_gemm(a, c->stream));
+  }
+  c->launches++;
+  return APT_OK;
+}
+
+// dW (+)= G^T Z over the device-counted rows; db += colsum(G)
+apt_status weight_grad(apt_trainer* t, const Layer& L, const float* G, int64_t g_pitch, const void* Z, bool z_bf16,
+                       int64_t z_pitch, const int32_t* n_rows, int64_t max_rows, int d_in, float* dW, float* db,
+                       int64_t dW_ld) {
+  apt_ctx* c = t->ctx;
+  SimtGemmArgs a{};
+  a.A = G; a.a_t = kF32; a.sam = 1; a.sak = g_pitch;
+  a.B = Z; a.b_t = z_bf16 ? kBF16 : kF32; a.sbk = z_pitch; a.sbn = 1;
+  a.C = dW; a.ldc = dW_ld; a.M = L.d_out; a.N = d_in; a.K = max_rows; a.K_dev = n_rows;
+  a.accumulate = 1; a.k_chunk = 2048;
+  CK(c, launch_simt_gemm(a, c->stream));
+  if (db) CK(c, launch_colsum(G, g_pitch, L.d_out, n_rows, max_rows, db, c->stream));
+  c->launches += db ? 2 : 1;
+  return APT_OK;
+}
+
+}  // namespace apt
+
+extern "C" {
+
+apt_status apt_trainer_create(apt_ctx* c, const apt_graph* g, const apt_fstore* f, const apt_model_desc* m,
+                              apt_strategy s, const int32_t* labels, apt_trainer** out) {
+  if (!c || !g || !f || !m || !labels || !out || m->n_layers < 1 || m->n_layers > APT_MAX_LAYERS || m->batch < 1 ||
+      s < APT_GDP || s > APT_DNP)
+    return set_err(c, APT_E_INVALID, "apt_trainer_create: bad arguments");
+  if (m->dims[0] != f->dim) return set_err(c, APT_E_INVALID, "apt_trainer_create: dims[0]=%d != store dim %d", m->dims[0], f->dim);
+  if (c->world > 1 && s == APT_NFP && f->layout != APT_NFP)
+    return set_err(c, APT_E_INVALID, "apt_trainer_create: NFP needs an NFP (column-sharded) store");
+  if (c->world > 1 && s != APT_NFP && f->layout == APT_NFP)
+    return set_err(c, APT_E_INVALID, "apt_trainer_create: row strategies need a row-sharded store");
+  for (int l = 0; l < m->n_layers; ++l)
+    if (m->fanouts[l] < 1 || m->fanouts[l] > 256 || m->dims[l + 1] < 1)
+      return set_err(c, APT_E_INVALID, "apt_trainer_create: fanout/dim out of range");
+  auto* t = new apt_trainer();
+  t->ctx = c;
+  t->g = g;
+  t->f = f;
+  t->m = *m;
+  t->s = s;
+  t->K = m->n_layers;
+  t->world = c->world;
+  Arena& A = t->arena;
+  const int K = t->K, C = t->world;
+  t->labels = A.alloc<int32_t>(g->n, false);
+  t->step_dev = A.alloc<uint64_t>(1, true);
+  CK(c, cudaMallocHost(&t->step_pinned, 8));
+  *t->step_pinned = 0;
+  CK(c, cudaMemcpyAsync(t->labels, labels, sizeof(int32_t) * g->n, cudaMemcpyHostToDevice, c->stream));
+  const int64_t n_words = ceil_div(g->n, 32);
+  // upper bounds per hop.  SNP/DNP seeds follow the partition: up to C*B on one rank.
+  const int64_t B0 = (s == APT_SNP || s == APT_DNP) ? int64_t(C) * m->batch : m->batch;
+  t->R.resize(c->n_local);
+  for (int li = 0; li < c->n_local; ++li) {
+    RankState& rs = t->R[li];
+    rs.rank = c->emulated ? li : c->rank;
+    rs.seeds = A.alloc<int32_t>(std::max<int64_t>(B0, int64_t(C) * m->batch), false);
+    rs.small = A.alloc<int32_t>(16, true);
+    rs.loss = A.alloc<float>(4, true);
+    rs.dst_bm = A.alloc<uint32_t>(n_words, true);
+    rs.new_bm = A.alloc<uint32_t>(n_words, true);
+    rs.pos = A.alloc<int32_t>(g->n, false);
+    rs.partials = A.alloc<int32_t>(ceil_div(n_words, 2048) + 4, false);
+    rs.hops.resize(K);
+    int64_t maxF = B0;
+    const int32_t* dst = rs.seeds;
+    const int32_t* n_dst = rs.small;
+    for (int h = 0; h < K; ++h) {
+      Hop& hp = rs.hops[h];
+      hp.k = m->fanouts[K - 1 - h];
+      hp.max_dst = maxF;
+      hp.max_src = std::max<int64_t>(maxF, std::min<int64_t>(maxF * (1 + hp.k), g->n));
+      hp.dst = dst;
+      hp.n_dst = n_dst;
+      hp.cnt = A.alloc<int32_t>(maxF, true);
+      hp.nbr = A.alloc<int32_t>(maxF * hp.k, false);
+      hp.counts = A.alloc<int32_t>(4, true);
+      hp.part2 = A.alloc<int32_t>(ceil_div(maxF, 2048) + 4, false);
+      if (h + 1 < K) {   // the layer-1 hop is consumed in ELL form (fused gather), no CSR needed
+        hp.src = A.alloc<int32_t>(hp.max_src, false);
+        hp.indptr = A.alloc<int32_t>(maxF + 1, true);
+        hp.indices = A.alloc<int32_t>(maxF * hp.k, false);
+      }
+      dst = hp.src;
+      n_dst = hp.counts;
+      maxF = hp.max_src;
+    }
+    rs.L.resize(K);
+    for (int l = 1; l <= K; ++l) {
+      Layer& L = rs.L[l - 1];
+      const Hop& hp = rs.hops[K - l];
+      L.d_in = m->dims[l - 1];
+      L.d_out = m->dims[l];
+      L.zf_pitch = round_up(L.d_in, 4);
+      L.zb_pitch = round_up(L.d_in, 8);
+      L.h_pitch = round_up(L.d_out, 4);
+      L.wb_pitch = round_up(L.d_in, 8);
+      L.max_rows = hp.max_dst;
+      L.n_rows = hp.n_dst;
+      if (m->dtype == APT_BF16) L.Zb = A.alloc<uint16_t>(L.max_rows * L.zb_pitch, true);
+      else L.Zf = A.alloc<float>(L.max_rows * L.zf_pitch, true);
+      L.H = A.alloc<float>(L.max_rows * L.h_pitch, true);
+      L.G = A.alloc<float>(L.max_rows * L.h_pitch, true);
+      if (l > 1) L.dZ = A.alloc<float>(L.max_rows * L.zf_pitch, true);
+      L.W = A.alloc<float>(int64_t(L.d_out) * L.d_in, true);
+      L.b = A.alloc<float>(L.d_out, true);
+      L.Wb = A.alloc<uint16_t>(int64_t(L.d_out) * L.wb_pitch, true);
+    }
+    // flat gradient buffer [dW1 db1 dW2 db2 ...] so one all-reduce covers the model
+    int64_t P = 0;
+    for (auto& L : rs.L) P += int64_t(L.d_out) * L.d_in + L.d_out;
+    float* grads = A.alloc<float>(P, true);
+    int64_t off = 0;
+    for (auto& L : rs.L) {
+      L.dW = grads + off;
+      off += int64_t(L.d_out) * L.d_in;
+      L.db = grads + off;
+      off += L.d_out;
+    }
+    if (!rs.seeds || !rs.pos || !grads) {
+      delete t;
+      return set_err(c, APT_E_OOM, "apt_trainer_create: out of device memory");
+    }
+    if (C > 1 && s != APT_GDP) {
+      apt_status st = strategy_alloc(t, rs);
+      if (st != APT_OK) { delete t; return st; }
+    }
+  }
+  {
+    std::vector<float*> tab(C, nullptr);
+    for (auto& rs : t->R) tab[rs.rank] = rs.L[0].dW;
+    t->dW_tab = A.alloc<float*>(C, false);
+    CK(c, cudaMemcpyAsync(t->dW_tab, tab.data(), sizeof(float*) * C, cudaMemcpyHostToDevice, c->stream));
+  }
+  for (int i = 0; i < 8; ++i) cudaEventCreate(&t->ev[i]);
+  CK(c, cudaStreamSynchronize(c->stream));
+  *out = t;
+  return APT_OK;
+}
+
+apt_status apt_trainer_destroy(apt_trainer* t) {
+  if (!t) return APT_OK;
+  cudaStreamSynchronize(t->ctx->stream);
+  if (t->gexec) cudaGraphExecDestroy(t->gexec);
+  for (int i = 0; i < 8; ++i)
+    if (t->ev[i]) cudaEventDestroy(t->ev[i]);
+  if (t->step_pinned) cudaFreeHost(t->step_pinned);
+  delete t;
+  return APT_OK;
+}
+
+apt_status apt_trainer_set_params(apt_trainer* t, int layer, const float* W, const float* b) {
+  if (!t || layer < 1 || layer > t->K || !W || !b) return set_err(t ? t->ctx : nullptr, APT_E_INVALID, "set_params: bad args");
+  apt_ctx* c = t->ctx;
+  for (auto& rs : t->R) {
+    Layer& L = rs.L[layer - 1];
+    CK(c, cudaMemcpyAsync(L.W, W, sizeof(float) * L.d_out * L.d_in, cudaMemcpyHostToDevice, c->stream));
+    CK(c, cudaMemcpyAsync(L.b, b, sizeof(float) * L.d_out, cudaMemcpyHostToDevice, c->stream));
+    CK(c, launch_to_bf16(L.W, L.d_in, L.Wb, L.wb_pitch, L.d_in, nullptr, L.d_out, c->stream));
+    c->launches++;
+  }
+  CK(c, cudaStreamSynchronize(c->stream));
+  return APT_OK;
+}
+
+apt_status apt_trainer_get_params(apt_trainer* t, int rank, int layer, float* W, float* b) {
+  if (!t || layer < 1 || layer > t->K) return set_err(t ? t->ctx : nullptr, APT_E_INVALID, "get_params: bad args");
+  for (auto& rs : t->R)
+    if (rs.rank == rank) {
+      Layer& L = rs.L[layer - 1];
+      CK(t->ctx, cudaStreamSynchronize(t->ctx->stream));
+      if (W) CK(t->ctx, cudaMemcpy(W, L.W, sizeof(float) * L.d_out * L.d_in, cudaMemcpyDeviceToHost));
+      if (b) CK(t->ctx, cudaMemcpy(b, L.b, sizeof(float) * L.d_out, cudaMemcpyDeviceToHost));
+      return APT_OK;
+    }
+  return set_err(t->ctx, APT_E_INVALID, "get_params: rank %d not hosted", rank);
+}
+
+apt_status apt_trainer_set_epoch(apt_trainer* t, const int64_t* train, int64_t n_train, uint64_t epoch) {
+  if (!t || !train || n_train < 1) return set_err(t ? t->ctx : nullptr, APT_E_INVALID, "set_epoch: bad args");
+  apt_ctx* c = t->ctx;
+  std::vector<int32_t> h(n_train);
+  for (int64_t i = 0; i < n_train; ++i) {
+    if (train[i] < 0 || train[i] >= t->g->n || (i && train[i] <= train[i - 1]))
+      return set_err(c, APT_E_INVALID, "set_epoch: train ids must be ascending and in range");
+    h[i] = int32_t(train[i]);
+  }
+  if (!t->perm || n_train > t->n_train) t->perm = t->arena.alloc<int32_t>(n_train, false);
+  t->n_train = n_train;
+  t->steps_per_epoch = ceil_div(n_train, int64_t(t->world) * t->m.batch);
+  int32_t *tr_dev = nullptr, *tmp_vals = nullptr;
+  uint64_t *k_in = nullptr, *k_out = nullptr;
+  void* tmp = nullptr;
+  size_t tmp_bytes = 0;
+  CK(c, cudaMallocAsync(&tr_dev, sizeof(int32_t) * n_train, c->stream));
+  CK(c, cudaMallocAsync(&tmp_vals, sizeof(int32_t) * n_train, c->stream));
+  CK(c, cudaMallocAsync(&k_in, sizeof(uint64_t) * n_train, c->stream));
+  CK(c, cudaMallocAsync(&k_out, sizeof(uint64_t) * n_train, c->stream));
+  CK(c, cudaMemcpyAsync(tr_dev, h.data(), sizeof(int32_t) * n_train, cudaMemcpyHostToDevice, c->stream));
+  CK(c, launch_perm_keys(tr_dev, n_train, t->m.sample_seed, epoch, k_in, c->stream));
+  // stable LSD radix sort by key: ties keep the ascending id order (reading O1)
+  CK(c, cub::DeviceRadixSort::SortPairs(nullptr, tmp_bytes, k_in, k_out, tr_dev, t->perm, int(n_train), 0, 64, c->stream));
+  CK(c, cudaMallocAsync(&tmp, tmp_bytes, c->stream));
+  CK(c, cub::DeviceRadixSort::SortPairs(tmp, tmp_bytes, k_in, k_out, tr_dev, t->perm, int(n_train), 0, 64, c->stream));
+  c->launches += 6;
+  for (void* p : {static_cast<void*>(tr_dev), static_cast<void*>(tmp_vals), static_cast<void*>(k_in),
+                  static_cast<void*>(k_out), tmp})
+    CK(c, cudaFreeAsync(p, c->stream));
+  CK(c, cudaStreamSynchronize(c->stream));
+  return APT_OK;
+}
+
+int64_t apt_trainer_steps_per_epoch(const apt_trainer* t) { return t ? t->steps_per_epoch : 0; }
+
+}  // extern "C"
+
+namespace apt {
+
+// Phase A for one rank: seeds + sampling (+ compaction for every hop but the layer-1 one).
+apt_status phase_sample(apt_trainer* t, RankState& rs, bool from_host_batch) {
+  apt_ctx* c = t->ctx;
+  if (!from_host_batch) {
+    const bool by_part = (t->s == APT_SNP || t->s == APT_DNP) && t->world > 1;
+    SeedArgs sa{t->perm, t->n_train, t->step_dev, t->steps_per_epoch, t->world, rs.rank, t->m.batch, by_part ? 1 : 0,
+                t->g->part, rs.seeds, rs.small, rs.small + 1};
+    CK(c, launch_select_seeds(sa, c->stream));
+    c->launches++;
+  }
+  const int64_t n_words = ceil_div(t->g->n, 32);
+  for (int h = 0; h < t->K; ++h) {
+    Hop& hp = rs.hops[h];
+    SampleArgs sa{t->g->indptr, t->g->indices, hp.dst, hp.n_dst, hp.max_dst, hp.k,
+                  philox_key(t->m.sample_seed, kDomSample), t->step_dev, h, hp.cnt, hp.nbr};
+    CK(c, launch_sample(sa, c->stream));
+    c->launches++;
+    if (h + 1 < t->K) {
+      CompactArgs ca{hp.dst, hp.n_dst, hp.max_dst, hp.cnt, hp.nbr, hp.k, rs.dst_bm, rs.new_bm, n_words, rs.pos, hp.src,
+                     hp.counts, hp.indptr, hp.indices, hp.counts + 1, rs.partials, hp.part2};
+      CK(c, launch_compact(ca, c->stream));
+      c->launches += 9;
+    }
+  }
+  return APT_OK;
+}
+
+// GDP layer-1 forward on one rank: fused gather (local + peer rows) + mean, projection.
+apt_status layer1_fwd_gdp(apt_trainer* t, RankState& rs, bool time_it) {
+  apt_ctx* c = t->ctx;
+  Layer& L = rs.L[0];
+  const Hop& hp = rs.hops[t->K - 1];
+  AggArgs a{};
+  a.cnt = hp.cnt; a.nbr = hp.nbr; a.k = hp.k;
+  a.n_dst = hp.n_dst; a.max_dst = hp.max_dst; a.dim = L.d_in;
+  if (t->m.dtype == APT_BF16) { a.z_bf16 = L.Zb; a.z_bf16_pitch = L.zb_pitch; }
+  else { a.z_f32 = L.Zf; a.z_f32_pitch = L.zf_pitch; }
+  if (time_it) CK(c, cudaEventRecord(t->ev[6], c->stream));
+  CK(c, launch_agg_fstore(a, feat_view(t->f, rs.rank), c->stream));
+  c->launches++;
+  if (time_it) CK(c, cudaEventRecord(t->ev[7], c->stream));
+  return project(t, L, L.Zb, L.Zf, L.zb_pitch, L.zf_pitch, L.n_rows, L.max_rows, L.d_in, L.W, L.Wb, L.b,
+                 t->K > 1 ? 1 : 0, L.H, nullptr, nullptr, nullptr);
+}
+
+// Upper layers l = 2..K (data parallel) + CE loss on one rank.
+apt_status upper_fwd_loss(apt_trainer* t, RankState& rs) {
+  apt_ctx* c = t->ctx;
+  for (int l = 2; l <= t->K; ++l) {
+    Layer& L = rs.L[l - 1];
+    const Layer& P = rs.L[l - 2];
+    const Hop& hp = rs.hops[t->K - l];
+    AggArgs a{};
+    a.indptr = hp.indptr; a.indices = hp.indices; a.x = P.H; a.x_pitch = P.h_pitch;
+    a.n_dst = hp.n_dst; a.max_dst = hp.max_dst; a.dim = L.d_in;
+    if (t->m.dtype == APT_BF16) { a.z_bf16 = L.Zb; a.z_bf16_pitch = L.zb_pitch; }
+    // fp32 Z is kept in both modes for the upper layers' weight gradient in fp32 mode
+    if (t->m.dtype != APT_BF16) { a.z_f32 = L.Zf; a.z_f32_pitch = L.zf_pitch; }
+    CK(c, launch_agg_csr(a, c->stream));
+    c->launches++;
+    apt_status s = project(t, L, L.Zb, L.Zf, L.zb_pitch, L.zf_pitch, L.n_rows, L.max_rows, L.d_in, L.W, L.Wb, L.b,
+                           l < t->K ? 1 : 0, L.H, nullptr, nullptr, nullptr);
+    if (s != APT_OK) return s;
+  }
+  Layer& LK = rs.L[t->K - 1];
+  CK(c, cudaMemsetAsync(rs.loss, 0, sizeof(float), c->stream));
+  CK(c, launch_ce_loss(LK.H, LK.h_pitch, LK.d_out, rs.seeds, rs.small, LK.max_rows, t->labels, rs.small + 1, rs.loss,
+                       LK.G, LK.h_pitch, c->stream));
+  c->launches++;
+  return APT_OK;
+}
+
+// Backward of layers K..2 on one rank (layer 1's weight gradient is strategy specific).
+apt_status upper_bwd(apt_trainer* t, RankState& rs) {
+  apt_ctx* c = t->ctx;
+  const bool bf = t->m.dtype == APT_BF16;
+  for (int l = t->K; l >= 2; --l) {
+    Layer& L = rs.L[l - 1];
+    Layer& P = rs.L[l - 2];
+    const Hop& hp = rs.hops[t->K - l];
+    apt_status s = weight_grad(t, L, L.G, L.h_pitch, bf ? static_cast<const void*>(L.Zb) : L.Zf, bf,
+                               bf ? L.zb_pitch : L.zf_pitch, L.n_rows, L.max_rows, L.d_in, L.dW, L.db, L.d_in);
+    if (s != APT_OK) return s;
+    // dZ = G W  (bf16 mode uses the bf16 weights of the forward)
+    SimtGemmArgs a{};
+    a.A = L.G; a.a_t = kF32; a.sam = L.h_pitch; a.sak = 1;
+    if (bf) { a.B = L.Wb; a.b_t = kBF16; a.sbk = L.wb_pitch; }
+    else { a.B = L.W; a.b_t = kF32; a.sbk = L.d_in; }
+    a.sbn = 1;
+    a.C = L.dZ; a.ldc = L.zf_pitch; a.M_dev = L.n_rows; a.M = L.max_rows; a.N = L.d_in; a.K = L.d_out;
+    CK(c, launch_simt_gemm(a, c->stream));
+    // dH_{l-1} = scatter(dZ / deg) over the layer-l block, then through the ReLU
+    zero_rows_kernel<<<blocks_for(P.max_rows * P.h_pitch / 4), 256, 0, c->stream>>>(P.G, P.h_pitch, P.n_rows);
+    CK(c, cudaGetLastError());
+    CK(c, launch_agg_bwd(hp.indptr, hp.indices, hp.n_dst, hp.max_dst, L.dZ, L.zf_pitch, L.d_in, P.G, P.h_pitch,
+                         c->stream));
+    CK(c, launch_relu_bwd(P.G, P.H, P.h_pitch, P.d_out, P.n_rows, P.max_rows, c->stream));
+    c->launches += 4;
+  }
+  return APT_OK;
+}
+
+apt_status layer1_bwd_gdp(apt_trainer* t, RankState& rs) {
+  Layer& L = rs.L[0];
+  const bool bf = t->m.dtype == APT_BF16;
+  return weight_grad(t, L, L.G, L.h_pitch, bf ? static_cast<const void*>(L.Zb) : L.Zf, bf,
+                     bf ? L.zb_pitch : L.zf_pitch, L.n_rows, L.max_rows, L.d_in, L.dW, L.db, L.d_in);
+}
+
+apt_status allreduce_sgd(apt_trainer* t, int update) {
+  apt_ctx* c = t->ctx;
+  int64_t P = 0;
+  for (auto& L : t->R[0].L) P += int64_t(L.d_out) * L.d_in + L.d_out;
+  if (t->world > 1) {
+    if (!c->emulated) return set_err(c, APT_E_UNSUPPORTED, "multi-process all-reduce not attached");
+    allreduce_sum_kernel<<<blocks_for(P), 256, 0, c->stream>>>(t->dW_tab, t->world, P);
+    CK(c, cudaGetLastError());
+    c->launches++;
+  }
+  if (!update) return APT_OK;
+  for (auto& rs : t->R) {
+    for (auto& L : rs.L) {
+      CK(c, launch_sgd(L.W, L.dW, int64_t(L.d_out) * L.d_in, t->m.lr, L.Wb, L.d_out, L.d_in, L.wb_pitch, c->stream));
+      CK(c, launch_sgd(L.b, L.db, L.d_out, t->m.lr, nullptr, 1, L.d_out, 0, c->stream));
+      c->launches += 2;
+    }
+  }
+  return APT_OK;
+}
+
+apt_status step_body(apt_trainer* t, int update, bool host_batch) {
+  apt_ctx* c = t->ctx;
+  const bool gdp = t->world == 1 || t->s == APT_GDP;
+  CK(c, cudaEventRecord(t->ev[0], c->stream));
+  for (auto& rs : t->R) {
+    apt_status s = phase_sample(t, rs, host_batch);
+    if (s != APT_OK) return s;
+  }
+  CK(c, cudaEventRecord(t->ev[1], c->stream));
+  if (gdp) {
+    bool first = true;
+    for (auto& rs : t->R) {
+      apt_status s = layer1_fwd_gdp(t, rs, first);
+      first = false;
+      if (s != APT_OK) return s;
+    }
+  } else {
+    apt_status s = layer1_fwd_strategy(t);
+    if (s != APT_OK) return s;
+  }
+  CK(c, cudaEventRecord(t->ev[2], c->stream));
+  for (auto& rs : t->R) {
+    apt_status s = upper_fwd_loss(t, rs);
+    if (s != APT_OK) return s;
+  }
+  CK(c, cudaEventRecord(t->ev[3], c->stream));
+  // zero the gradient accumulators, then backward
+  for (auto& rs : t->R) {
+    int64_t P = 0;
+    for (auto& L : rs.L) P += int64_t(L.d_out) * L.d_in + L.d_out;
+    CK(c, cudaMemsetAsync(rs.L[0].dW, 0, sizeof(float) * P, c->stream));
+  }
+  for (auto& rs : t->R) {
+    apt_status s = upper_bwd(t, rs);
+    if (s != APT_OK) return s;
+  }
+  if (gdp) {
+    for (auto& rs : t->R) {
+      apt_status s = layer1_bwd_gdp(t, rs);
+      if (s != APT_OK) return s;
+    }
+  } else {
+    apt_status s = layer1_bwd_strategy(t);
+    if (s != APT_OK) return s;
+  }
+  CK(c, cudaEventRecord(t->ev[4], c->stream));
+  apt_status s = allreduce_sgd(t, update);
+  if (s != APT_OK) return s;
+  CK(c, cudaEventRecord(t->ev[5], c->stream));
+  t->ev_ok = true;
+  return APT_OK;
+}
+
+}  // namespace apt
+
+extern "C" {
+
+apt_status apt_trainer_step(apt_trainer* t, int64_t step, int update) {
+  if (!t || !t->perm) return set_err(t ? t->ctx : nullptr, APT_E_STATE, "apt_trainer_step: call apt_trainer_set_epoch first");
+  apt_ctx* c = t->ctx;
+  if (c->broken) return set_err(c, APT_E_STATE, "ctx is broken by an earlier CUDA error");
+  // the step id reaches the device through a pinned cell copied on the stream,
+  // so a captured CUDA graph replays with the current value
+  *t->step_pinned = uint64_t(step);
+  if (t->use_graph) {
+    if (!t->gexec || t->graph_update != update) {
+      if (t->gexec) { cudaGraphExecDestroy(t->gexec); t->gexec = nullptr; }
+      cudaGraph_t graph;
+      CK(c, cudaStreamBeginCapture(c->stream, cudaStreamCaptureModeThreadLocal));
+      cudaMemcpyAsync(t->step_dev, t->step_pinned, 8, cudaMemcpyHostToDevice, c->stream);
+      apt_status s = step_body(t, update, false);
+      cudaError_t e = cudaStreamEndCapture(c->stream, &graph);
+      if (s != APT_OK) return s;
+      CK(c, e);
+      CK(c, cudaGraphInstantiate(&t->gexec, graph, 0));
+      cudaGraphDestroy(graph);
+      t->graph_update = update;
+    }
+    CK(c, cudaGraphLaunch(t->gexec, c->stream));
+    return APT_OK;
+  }
+  CK(c, cudaMemcpyAsync(t->step_dev, t->step_pinned, 8, cudaMemcpyHostToDevice, c->stream));
+  return step_body(t, update, false);
+}
+
+apt_status apt_trainer_step_host(apt_trainer* t, const int64_t* gbatch, int64_t n_global, int64_t step, int update,
+                                 float* loss_host) {
+  if (!t || !gbatch || n_global < 1 || n_global > int64_t(t->world) * t->m.batch)
+    return set_err(t ? t->ctx : nullptr, APT_E_INVALID, "apt_trainer_step_host: bad arguments");
+  apt_ctx* c = t->ctx;
+  // host global batch -> per-rank seeds (GDP/NFP: chunk r; SNP/DNP: partition r), H2D on the stream
+  for (auto& rs : t->R) {
+    std::vector<int32_t> mine;
+    const bool by_part = (t->s == APT_SNP || t->s == APT_DNP) && t->world > 1;
+    for (int64_t i = 0; i < n_global; ++i) {
+      const int64_t u = gbatch[i];
+      if (u < 0 || u >= t->g->n) return set_err(c, APT_E_INVALID, "step_host: seed out of range");
+      if (by_part ? t->g->part_h[u] == rs.rank : (i / t->m.batch) == rs.rank) mine.push_back(int32_t(u));
+    }
+    int32_t hdr[2] = {int32_t(mine.size()), int32_t(n_global)};
+    CK(c, cudaMemcpyAsync(rs.seeds, mine.data(), sizeof(int32_t) * mine.size(), cudaMemcpyHostToDevice, c->stream));
+    CK(c, cudaMemcpyAsync(rs.small, hdr, sizeof hdr, cudaMemcpyHostToDevice, c->stream));
+  }
+  *t->step_pinned = uint64_t(step);
+  CK(c, cudaMemcpyAsync(t->step_dev, t->step_pinned, 8, cudaMemcpyHostToDevice, c->stream));
+  apt_status s = step_body(t, update, true);
+  if (s != APT_OK) return s;
+  return apt_trainer_loss(t, loss_host);
+}
+
+apt_status apt_trainer_loss(apt_trainer* t, float* loss) {
+  if (!t || !loss) return set_err(t ? t->ctx : nullptr, APT_E_INVALID, "loss: null");
+  apt_ctx* c = t->ctx;
+  float tot = 0.f;
+  for (auto& rs : t->R) {
+    float v = 0.f;
+    CK(c, cudaMemcpyAsync(&v, rs.loss, 4, cudaMemcpyDeviceToHost, c->stream));
+    CK(c, cudaStreamSynchronize(c->stream));
+    tot += v;
+  }
+  *loss = tot;
+  return apt_ctx_sync(c);
+}
+
+apt_status apt_trainer_use_graph(apt_trainer* t, int enable) {
+  if (!t) return set_err(nullptr, APT_E_INVALID, "null trainer");
+  t->use_graph = enable != 0;
+  return APT_OK;
+}
+
+apt_status apt_trainer_phase_ms(apt_trainer* t, double* ms, int n) {
+  if (!t || !ms || n < 1) return set_err(t ? t->ctx : nullptr, APT_E_INVALID, "phase_ms: bad args");
+  CK(t->ctx, cudaStreamSynchronize(t->ctx->stream));
+  if (!t->ev_ok) return set_err(t->ctx, APT_E_STATE, "phase_ms: no step recorded");
+  for (int i = 0; i < n && i < 6; ++i) {
+    float v = 0.f;
+    if (i < 5) CK(t->ctx, cudaEventElapsedTime(&v, t->ev[i], t->ev[i + 1]));
+    else CK(t->ctx, cudaEventElapsedTime(&v, t->ev[6], t->ev[7]));
+    ms[i] = v;
+  }
+  return APT_OK;
+}
+
+apt_status apt_trainer_read(apt_trainer* t, int rank, int what, int layer, void* host, int64_t cap, int64_t* rows,
+                            int* cols) {
+  if (!t || !host || !rows || !cols) return set_err(t ? t->ctx : nullptr, APT_E_INVALID, "read: null");
+  apt_ctx* c = t->ctx;
+  RankState* rs = nullptr;
+  for (auto& r : t->R)
+    if (r.rank == rank) rs = &r;
+  if (!rs) return set_err(c, APT_E_INVALID, "read: rank %d not hosted", rank);
+  if (what != 0 && (layer < 1 || layer > t->K)) return set_err(c, APT_E_INVALID, "read: layer out of range");
+  CK(c, cudaStreamSynchronize(c->stream));
+  auto count = [&](const int32_t* p) {
+    int32_t v = 0;
+    cudaMemcpy(&v, p, 4, cudaMemcpyDeviceToHost);
+    return int64_t(v);
+  };
+  auto copy_rows = [&](const void* src, int64_t nr, int nc, int64_t pitch, int esz, bool bf) -> apt_status {
+    *rows = nr;
+    *cols = nc;
+    const int64_t n = std::min<int64_t>(cap, nr * nc);
+    std::vector<uint8_t> buf(size_t(std::max<int64_t>(nr, 1) * pitch * esz));
+    if (nr) CK(c, cudaMemcpy(buf.data(), src, size_t(nr * pitch * esz), cudaMemcpyDeviceToHost));
+    for (int64_t i = 0; i < n; ++i) {
+      const int64_t r = i / nc, cc = i % nc;
+      if (bf) {
+        uint32_t b = uint32_t(reinterpret_cast<uint16_t*>(buf.data())[r * pitch + cc]) << 16;
+        memcpy(static_cast<float*>(host) + i, &b, 4);
+      } else if (esz == 4) {
+        memcpy(static_cast<uint8_t*>(host) + i * 4, buf.data() + (r * pitch + cc) * 4, 4);
+      }
+    }
+    return APT_OK;
+  };
+  switch (what) {
+    case 0: return copy_rows(rs->seeds, count(rs->small), 1, 1, 4, false);
+    case 1: {
+      const Hop& hp = rs->hops[t->K - layer];
+      return copy_rows(hp.dst, count(hp.n_dst), 1, 1, 4, false);
+    }
+    case 2: {
+      const Layer& L = rs->L[layer - 1];
+      const int64_t nr = count(L.n_rows);
+      if (L.Zb) return copy_rows(L.Zb, nr, L.d_in, L.zb_pitch, 2, true);
+      return copy_rows(L.Zf, nr, L.d_in, L.zf_pitch, 4, false);
+    }
+    case 3: { const Layer& L = rs->L[layer - 1]; return copy_rows(L.H, count(L.n_rows), L.d_out, L.h_pitch, 4, false); }
+    case 4: { const Layer& L = rs->L[layer - 1]; return copy_rows(L.dW, L.d_out, L.d_in, L.d_in, 4, false); }
+    case 5: { const Layer& L = rs->L[layer - 1]; return copy_rows(L.db, 1, L.d_out, L.d_out, 4, false); }
+    case 6: { const Layer& L = rs->L[layer - 1]; return copy_rows(L.G, count(L.n_rows), L.d_out, L.h_pitch, 4, false); }
+    default: return set_err(c, APT_E_INVALID, "read: unknown item %d", what);
+  }
+}
+
+apt_status apt_trainer_agg_bytes(apt_trainer* t, double* bytes) {
+  if (!t || !bytes) return set_err(nullptr, APT_E_INVALID, "agg_bytes: null");
+  *bytes = t->last_agg_bytes;
+  return APT_OK;
+}
+
+}  // extern "C"

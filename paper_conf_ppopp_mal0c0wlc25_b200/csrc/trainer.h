@@ -1,0 +1,104 @@
+// trainer.h -- per-rank state of the training step (internal).
+#pragma once
+#include <cuda_runtime.h>
+
+#include <vector>
+
+#include "runtime.h"
+
+namespace apt {
+
+struct Hop {
+  int k = 0;
+  int64_t max_dst = 0, max_src = 0;
+  const int32_t* dst = nullptr;     // frontier (seeds or previous hop's src)
+  const int32_t* n_dst = nullptr;   // device count
+  int32_t* cnt = nullptr;           // [max_dst]
+  int32_t* nbr = nullptr;           // [max_dst * k] global ids (ELL)
+  int32_t* src = nullptr;           // [max_src]
+  int32_t* indptr = nullptr;        // [max_dst + 1]
+  int32_t* indices = nullptr;       // [max_dst * k]
+  int32_t* counts = nullptr;        // [0] n_src, [1] n_edges
+  int32_t* part2 = nullptr;         // scan workspace
+};
+
+struct Layer {
+  int d_in = 0, d_out = 0;
+  int64_t zf_pitch = 0, zb_pitch = 0, h_pitch = 0, wb_pitch = 0;
+  int64_t max_rows = 0;
+  const int32_t* n_rows = nullptr;  // device count of dst rows
+  float* Zf = nullptr;              // [max_rows x zf_pitch] (fp32 mode)
+  uint16_t* Zb = nullptr;           // [max_rows x zb_pitch] (bf16 mode)
+  float* H = nullptr;               // post-activation (or logits)
+  float* G = nullptr;               // dL/dpre
+  float* dZ = nullptr;              // [max_rows x zf_pitch] scratch (l > 1)
+  float* W = nullptr;               // [d_out x d_in] fp32 master
+  float* b = nullptr;
+  uint16_t* Wb = nullptr;           // [d_out x wb_pitch] bf16 copy (tensor cores)
+  float* dW = nullptr;
+  float* db = nullptr;
+};
+
+// NFP / SNP / DNP exchange state of one rank (trainer_strategies.cu).
+struct Xchg {
+  // generic receive slots written by peers: slot[s] holds what rank s sent
+  int32_t* req_cnt = nullptr;        // [C] rows received from each sender (device)
+  int32_t* req_row = nullptr;        // [C x cap] requester row / tag
+  int32_t* req_gid = nullptr;        // [C x cap] node id (DNP) or group deg (SNP)
+  int32_t* req_indptr = nullptr;     // [C x (cap+1)] (SNP edge groups)
+  int32_t* req_src = nullptr;        // [C x ecap] source gids (SNP)
+  int32_t* ecnt = nullptr;           // [C] edges received from each sender
+  int64_t cap = 0, ecap = 0;
+  // owner-side work list (DNP) / contributor work (SNP)
+  int32_t* work_rank = nullptr;      // [wcap] requester rank of every work row
+  int32_t* work_row = nullptr;       // [wcap] requester row
+  int32_t* work_gid = nullptr;       // [wcap] node id
+  int32_t* n_work = nullptr;         // device count
+  int64_t wcap = 0;
+  int32_t* wcnt = nullptr;           // [wcap] re-sampled ELL (DNP)
+  int32_t* wnbr = nullptr;           // [wcap * k]
+  uint16_t* wZb = nullptr;           // [wcap x zb_pitch]
+  float* wZf = nullptr;              // [wcap x zf_pitch]
+  float* wG = nullptr;               // [wcap x h_pitch] gathered gradients (bwd)
+  float* partial = nullptr;          // [C x cap x h_pitch] partial sums received (SNP/NFP)
+};
+
+struct RankState {
+  int rank = 0;
+  int32_t* seeds = nullptr;
+  int32_t* small = nullptr;         // [0] n_seeds [1] n_global ...
+  std::vector<Hop> hops;
+  std::vector<Layer> L;
+  uint32_t* dst_bm = nullptr;
+  uint32_t* new_bm = nullptr;
+  int32_t* pos = nullptr;
+  int32_t* partials = nullptr;
+  float* loss = nullptr;
+  Xchg x;
+};
+
+}  // namespace apt
+
+struct apt_trainer {
+  apt_ctx* ctx = nullptr;
+  const apt_graph* g = nullptr;
+  const apt_fstore* f = nullptr;
+  apt_model_desc m{};
+  apt_strategy s = APT_GDP;
+  int K = 0, world = 1;
+  int32_t* labels = nullptr;
+  int32_t* perm = nullptr;
+  int64_t n_train = 0, steps_per_epoch = 1;
+  uint64_t* step_dev = nullptr;
+  uint64_t* step_pinned = nullptr;
+  std::vector<apt::RankState> R;
+  // device pointer tables for cross-rank kernels
+  float** dW_tab = nullptr;
+  bool use_graph = false;
+  cudaGraphExec_t gexec = nullptr;
+  int graph_update = -1;
+  cudaEvent_t ev[8] = {};
+  bool ev_ok = false;
+  double last_agg_bytes = 0;
+  apt::Arena arena;
+};

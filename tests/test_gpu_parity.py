@@ -1,0 +1,254 @@
+"""GPU parity: the sm_100a path through the C ABI vs the CPU oracle (-m gpu).
+
+Bars (BASELINE.json north_star): sampled blocks and indices bit-exact; Z under the
+O4 features bit-exact; fp32 outputs and gradients rtol 1e-5 / atol 1e-6; bf16
+paths rtol 2e-2 (atol derived in DESIGN.md §Tolerances).
+"""
+import numpy as np
+import pytest
+
+import aptgen
+import oracle
+from oracle import model
+
+pytestmark = pytest.mark.gpu
+
+torch = pytest.importorskip("torch")
+
+
+@pytest.fixture(scope="module")
+def A():
+    import paper_conf_ppopp_mal0c0wlc25_b200.apt as A
+    A.lib()
+    return A
+
+
+@pytest.fixture(scope="module")
+def ctx(A):
+    torch.cuda.set_device(0)
+    return A.Ctx(0, 1, 0)
+
+
+@pytest.fixture(scope="module")
+def tiny(tiny_cfg, tiny_graph):
+    return tiny_cfg, tiny_graph, aptgen.train_nodes(tiny_graph, tiny_cfg)
+
+
+def dev_i64(a):
+    return torch.as_tensor(np.ascontiguousarray(a, np.int64)).cuda()
+
+
+# ------------------------------------------------------------------ S2 / S3
+@pytest.mark.parametrize("step", [0, 1, 5])
+def test_sample_blocks_bit_exact_tiny(A, ctx, tiny, step):
+    cfg, g, train = tiny
+    gr = ctx.graph_load(g.indptr, g.indices)
+    perm = oracle.epoch_perm(train, cfg.sample_seed, 0)
+    seeds = perm[step * cfg.batch:(step + 1) * cfg.batch]
+    sd = dev_i64(seeds)
+    b = ctx.sample(gr, sd, len(seeds), cfg.fanouts, cfg.sample_seed, step)
+    ref = oracle.sample_blocks(g, seeds, cfg.fanouts, cfg.sample_seed, step)
+    for h, rb in enumerate(ref):
+        dst, src, indptr, indices = b.block_host(h)
+        assert np.array_equal(dst, rb.dst)
+        assert np.array_equal(src, rb.src)
+        assert np.array_equal(indptr, rb.indptr)
+        assert np.array_equal(indices, rb.indices)
+
+
+@pytest.mark.parametrize("fanouts", [(1, 3), (25, 7), (40,), (256, 2)])
+def test_sample_edge_fanouts(A, ctx, tiny, fanouts):
+    """fanout 1, > 32 (multi-slot Floyd), 256 (max) and deg <= k rows."""
+    cfg, g, train = tiny
+    gr = ctx.graph_load(g.indptr, g.indices)
+    seeds = train[::7][:300]
+    b = ctx.sample(gr, dev_i64(seeds), len(seeds), fanouts, 11, 3)
+    ref = oracle.sample_blocks(g, seeds, fanouts, 11, 3)
+    for h, rb in enumerate(ref):
+        dst, src, indptr, indices = b.block_host(h)
+        assert np.array_equal(src, rb.src) and np.array_equal(indptr, rb.indptr)
+        assert np.array_equal(indices, rb.indices)
+
+
+def test_sample_empty_and_isolated(A, ctx, tiny):
+    cfg, g, _ = tiny
+    gr = ctx.graph_load(g.indptr, g.indices)
+    iso = np.nonzero(g.degrees() == 0)[0][:5].astype(np.int64)
+    b = ctx.sample(gr, dev_i64(iso), len(iso), (3, 3), 1, 0)
+    v = b.block(0)
+    assert v.n_dst == len(iso) and v.n_edges == 0 and v.n_src == len(iso)
+    b0 = ctx.sample(gr, dev_i64(np.zeros(0)), 0, (3, 3), 1, 0)
+    assert b0.block(1).n_dst == 0
+
+
+@pytest.mark.slow
+def test_sample_products_bit_exact(A, ctx):
+    cfg = aptgen.CONFIGS["products"]
+    g = aptgen.make_graph(cfg)
+    train = aptgen.train_nodes(g, cfg)
+    gr = ctx.graph_load(g.indptr, g.indices)
+    perm = oracle.epoch_perm(train, cfg.sample_seed, 0)
+    for step in (0, 17):
+        seeds = perm[step * cfg.batch:(step + 1) * cfg.batch]
+        b = ctx.sample(gr, dev_i64(seeds), len(seeds), cfg.fanouts, cfg.sample_seed, step)
+        ref = oracle.sample_blocks(g, seeds, cfg.fanouts, cfg.sample_seed, step)
+        for h, rb in enumerate(ref):
+            dst, src, indptr, indices = b.block_host(h)
+            assert np.array_equal(src, rb.src) and np.array_equal(indices, rb.indices)
+            assert np.array_equal(indptr, rb.indptr)
+
+
+# ------------------------------------------------------------------ features / gather
+@pytest.mark.parametrize("dtype,dim", [("f32", 64), ("bf16", 100), ("f32", 100), ("bf16", 256)])
+def test_feature_store_bit_exact(A, ctx, tiny, dtype, dim):
+    cfg, g, _ = tiny
+    gr = ctx.graph_load(g.indptr, g.indices)
+    fs = ctx.fstore_create(gr, A.GDP, A.DTYPE[dtype], dim, None, cfg.feat_seed)
+    ids = np.array([0, 1, 2, 77, 4095, 9999, 5000, 5000], np.int32)
+    pitch = ((dim + 7) // 8 * 8) if dtype == "bf16" else ((dim + 3) // 4 * 4)
+    esz = 2 if dtype == "bf16" else 4
+    out = torch.zeros(len(ids) * pitch * esz, dtype=torch.uint8, device="cuda")
+    ctx.gather(fs, torch.as_tensor(ids).cuda(), len(ids), out)
+    torch.cuda.synchronize()
+    raw = out.cpu().numpy()
+    if dtype == "bf16":
+        got = (raw.view(np.uint16).astype(np.uint32) << 16).view(np.float32).reshape(len(ids), pitch)[:, :dim]
+    else:
+        got = raw.view(np.float32).reshape(len(ids), pitch)[:, :dim]
+    ref = oracle.features(cfg.feat_seed, ids.astype(np.int64), dim)
+    assert np.array_equal(got.astype(np.float64), ref)
+
+
+# ------------------------------------------------------------------ S7 aggregation
+def test_aggregate_bit_exact_and_bwd(A, ctx, tiny):
+    cfg, g, train = tiny
+    gr = ctx.graph_load(g.indptr, g.indices)
+    seeds = train[:200]
+    b = ctx.sample(gr, dev_i64(seeds), len(seeds), (6,), 5, 2)
+    (rb,) = oracle.sample_blocks(g, seeds, (6,), 5, 2)
+    d = 36
+    x = oracle.features(cfg.feat_seed, rb.src, d)
+    xd = torch.as_tensor(x.astype(np.float32)).cuda().contiguous()
+    z = torch.zeros((rb.n_dst, 36), dtype=torch.float32, device="cuda")
+    v = b.block(0)
+    ctx.aggregate(v, xd, A.F32, d, d, z, 36)
+    ref = oracle.aggregate(rb.indptr, rb.indices, x)
+    assert np.array_equal(z.cpu().numpy(), ref.astype(np.float32))          # exact under O4
+    dz = np.random.default_rng(0).normal(size=(rb.n_dst, d)).astype(np.float32)
+    dx = torch.zeros((rb.n_src, d), dtype=torch.float32, device="cuda")
+    ctx.aggregate_bwd(v, torch.as_tensor(dz).cuda(), d, d, dx, d)
+    refb = oracle.aggregate_bwd(rb.indptr, rb.indices, dz.astype(np.float64), rb.n_src)
+    assert np.allclose(dx.cpu().numpy(), refb, rtol=1e-5, atol=1e-6)
+
+
+# ------------------------------------------------------------------ S8 projection
+@pytest.mark.parametrize("M,N,K", [(1, 16, 64), (127, 32, 64), (128, 47, 100), (1000, 256, 100),
+                                   (5000, 256, 256), (333, 48, 256), (4099, 8, 16)])
+def test_project_tcgen05_bf16(A, ctx, M, N, K):
+    rng = np.random.default_rng(M + N + K)
+    kp = (K + 7) // 8 * 8
+    Z = oracle.bf16_round(rng.normal(size=(M, K)))
+    W = rng.normal(size=(N, K)).astype(np.float32) / np.sqrt(K)
+    bias = rng.normal(size=N).astype(np.float32)
+    Zb = np.zeros((M, kp), np.uint16)
+    Zb[:, :K] = (Z.astype(np.float32).view(np.uint32) >> 16).astype(np.uint16)
+    yp = (N + 3) // 4 * 4
+    Y = torch.zeros((M, yp), dtype=torch.float32, device="cuda")
+    ctx.project(torch.as_tensor(Zb.view(np.int16)).cuda(), kp, A.BF16, torch.as_tensor(W).cuda(),
+                torch.as_tensor(bias).cuda(), M, N, K, 1, Y, yp)
+    ref = np.maximum(Z @ oracle.bf16_round(W).T + bias, 0)
+    got = Y.cpu().numpy()[:, :N]
+    assert np.allclose(got, ref, rtol=1e-5, atol=1e-5), np.abs(got - ref).max()
+
+
+@pytest.mark.parametrize("M,N,K", [(1, 5, 3), (130, 47, 100), (2000, 256, 100)])
+def test_project_fp32(A, ctx, M, N, K):
+    rng = np.random.default_rng(7)
+    Z = rng.normal(size=(M, K)).astype(np.float32)
+    W = rng.normal(size=(N, K)).astype(np.float32)
+    bias = rng.normal(size=N).astype(np.float32)
+    Y = torch.zeros((M, N), dtype=torch.float32, device="cuda")
+    ctx.project(torch.as_tensor(Z).cuda(), K, A.F32, torch.as_tensor(W).cuda(), torch.as_tensor(bias).cuda(),
+                M, N, K, 0, Y, N)
+    ref = Z.astype(np.float64) @ W.T.astype(np.float64) + bias
+    assert np.allclose(Y.cpu().numpy(), ref, rtol=1e-5, atol=1e-5)
+
+
+# ------------------------------------------------------------------ the training step (C = 1)
+def _trainer(A, ctx, cfg, g, train, dtype, strategy="GDP", lr=0.1):
+    gr = ctx.graph_load(g.indptr, g.indices)
+    fs = ctx.fstore_create(gr, A.STRATEGY[strategy] if strategy == "NFP" else A.GDP, A.DTYPE[dtype], cfg.dim, None,
+                           cfg.feat_seed)
+    dims = [cfg.dim] + [d for _, d in cfg.dims()]
+    labels = aptgen.labels(cfg, g.n)
+    tr = A.Trainer(ctx, gr, fs, dims, cfg.fanouts, cfg.batch, A.DTYPE[dtype], lr, cfg.sample_seed, cfg.feat_seed,
+                   A.STRATEGY[strategy], labels)
+    params = aptgen.weights(cfg)
+    tr.set_params(params)
+    tr.set_epoch(train, 0)
+    return tr, params, labels
+
+
+TOL = {"f32": dict(rtol=1e-5, atol=1e-6), "bf16": dict(rtol=2e-2, atol=2e-3)}
+
+
+@pytest.mark.parametrize("dtype", ["f32", "bf16"])
+@pytest.mark.parametrize("step", [0, 3])
+def test_train_step_matches_oracle(A, ctx, tiny, dtype, step):
+    cfg, g, train = tiny
+    tr, params, labels = _trainer(A, ctx, cfg, g, train, dtype)
+    tr.step(step, update=False)
+    loss = tr.loss()
+    seeds = tr.read("seeds")[:, 0].astype(np.int64)
+    perm = oracle.epoch_perm(train, cfg.sample_seed, 0)
+    assert np.array_equal(seeds, perm[step * cfg.batch:(step + 1) * cfg.batch])
+    blocks = oracle.sample_blocks(g, seeds, cfg.fanouts, cfg.sample_seed, step)
+    p64 = [(W.astype(np.float64), b.astype(np.float64)) for W, b in params]
+    ref = model.train_step(blocks, cfg.feat_seed, cfg.dim, p64, labels[seeds], len(seeds), dtype)
+    K = len(blocks)
+    for l in range(1, K + 1):
+        assert np.array_equal(tr.read("dst", l)[:, 0], blocks[K - l].dst)
+    # layer-1 Z is bit-exact under O4 features (exact sums, IEEE division)
+    assert np.array_equal(tr.read("Z", 1), ref["cache"]["Z"][0].astype(np.float32))
+    tol = TOL[dtype]
+    for l in range(1, K + 1):
+        assert np.allclose(tr.read("H", l), ref["cache"]["h"][l - 1], **tol), f"H layer {l}"
+    assert abs(loss - ref["loss"]) <= tol["rtol"] * abs(ref["loss"]) + tol["atol"]
+    for l in range(1, K + 1):
+        dW, db = ref["grads"][l - 1]
+        assert np.allclose(tr.read("dW", l), dW, **tol), f"dW layer {l}"
+        assert np.allclose(tr.read("db", l)[0], db, **tol), f"db layer {l}"
+
+
+def test_sgd_update_and_graph_replay(A, ctx, tiny):
+    """Two steps with the update, eager vs CUDA-graph replay: identical parameters."""
+    cfg, g, train = tiny
+    outs = []
+    for use_graph in (False, True):
+        tr, params, labels = _trainer(A, ctx, cfg, g, train, "f32", lr=0.5)
+        tr.use_graph(use_graph)
+        for s in range(3):
+            tr.step(s, update=True)
+        outs.append(tr.get_params())
+    for (W0, b0), (W1, b1) in zip(*outs):
+        assert np.allclose(W0, W1, rtol=1e-6, atol=1e-7) and np.allclose(b0, b1, rtol=1e-6, atol=1e-7)
+    # one step against the oracle's SGD
+    tr, params, labels = _trainer(A, ctx, cfg, g, train, "f32", lr=0.5)
+    tr.step(0, update=True)
+    seeds = tr.read("seeds")[:, 0].astype(np.int64)
+    blocks = oracle.sample_blocks(g, seeds, cfg.fanouts, cfg.sample_seed, 0)
+    p64 = [(W.astype(np.float64), b.astype(np.float64)) for W, b in params]
+    ref = model.train_step(blocks, cfg.feat_seed, cfg.dim, p64, labels[seeds], len(seeds), "f32", lr=0.5)
+    for (W, b), (Wr, br) in zip(tr.get_params(), ref["new_params"]):
+        assert np.allclose(W, Wr, rtol=1e-5, atol=1e-6) and np.allclose(b, br, rtol=1e-5, atol=1e-6)
+
+
+def test_step_host_e2e_matches_device_step(A, ctx, tiny):
+    cfg, g, train = tiny
+    tr, params, labels = _trainer(A, ctx, cfg, g, train, "bf16")
+    tr.step(2, update=False)
+    l_dev = tr.loss()
+    perm = oracle.epoch_perm(train, cfg.sample_seed, 0)
+    gb = torch.as_tensor(perm[2 * cfg.batch:3 * cfg.batch]).pin_memory()
+    l_host = tr.step_host(gb, 2, update=False)
+    assert l_host == pytest.approx(l_dev, rel=1e-6)
