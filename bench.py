@@ -1,0 +1,319 @@
+"""bench.py -- seeds/s of APT's per-mini-batch sampled-subgraph step on B200.
+
+Contract (task statement + SURVEY.md §8(d)):
+  python bench.py --gpus N --steps K --warmup W [--impl apt|reference]
+One step = one pass of the whole hot path over one global batch: seed selection
+(S1), 3-hop Philox sampling + compaction (S2/S3), the layer-1 strategy forward
+(S4-S9: fused gather + mean, tcgen05 projection), upper layers + CE loss (S10),
+backward (S10/S11), gradient all-reduce + SGD.  All of it runs in libapt.so's
+sm_100a kernels, replayed as one CUDA graph per step.
+
+Workload (BASELINE.json configs[1]): synthetic ogbn-products shape, R-MAT
+2.4M nodes / 62M undirected edges, d=100 (bf16 rows padded to 104), GraphSAGE
+100->256->256->47, fanout [10,10,10], B=1024 seeds per GPU.
+
+value      = seeds/s of the whole job (C*B seeds per step / max-over-ranks step time)
+e2e        = the same through apt_trainer_step_host (host batch in, host loss out)
+roofline   = the dominant kernel (layer-1 fused gather + mean, HBM bound)
+cpu_baseline = the oracle (oracle/, single thread) on the first steps of the
+               same epoch, rank 0 at N=1 only.
+--impl reference: the oracle itself, timed on the host cores (this tier has no
+installable reference implementation; its reference arm is the oracle).
+"""
+from __future__ import annotations
+
+import argparse
+import json
+import os
+import statistics
+import subprocess
+import sys
+import threading
+import time
+
+ROOT = os.path.dirname(os.path.abspath(__file__))
+sys.path.insert(0, ROOT)
+
+import numpy as np  # noqa: E402
+
+import aptgen  # noqa: E402
+
+METRIC = "seeds/s"
+STRATS = ("GDP", "NFP", "SNP", "DNP")
+
+
+def parse():
+    ap = argparse.ArgumentParser()
+    ap.add_argument("--gpus", type=int, default=1)
+    ap.add_argument("--steps", type=int, default=30)
+    ap.add_argument("--warmup", type=int, default=5)
+    ap.add_argument("--impl", default="apt", choices=["apt", "reference"])
+    ap.add_argument("--config", default="products", choices=sorted(aptgen.CONFIGS))
+    ap.add_argument("--strategy", default="GDP", choices=list(STRATS))
+    ap.add_argument("--dtype", default="bf16", choices=["bf16", "f32"])
+    ap.add_argument("--no-graph", action="store_true", help="eager launches instead of CUDA-graph replay")
+    ap.add_argument("--no-cpu-baseline", action="store_true")
+    ap.add_argument("--cpu-steps", type=int, default=3, help="oracle steps for cpu_baseline")
+    ap.add_argument("--e2e-steps", type=int, default=10)
+    ap.add_argument("--verbose", action="store_true")
+    return ap.parse_args()
+
+
+def dist_env():
+    return int(os.environ.get("RANK", 0)), int(os.environ.get("WORLD_SIZE", 1)), int(os.environ.get("LOCAL_RANK", 0))
+
+
+def workload_config(cfg):
+    return {"workload": f"synthetic ogbn-{cfg.name} shape (R-MAT {cfg.n} nodes / {cfg.m} undirected edges)"
+            if cfg.name != "tiny" else f"tiny R-MAT {cfg.n} nodes / {cfg.m} edges",
+            "model": "GraphSAGE-mean " + "->".join(str(d) for d in [cfg.dim] + [o for _, o in cfg.dims()]),
+            "fanouts": list(cfg.fanouts), "batch_per_gpu": cfg.batch, "feat_dim": cfg.dim}
+
+
+# --------------------------------------------------------------------- clocks
+class ClockSampler:
+    """nvidia-smi clocks + throttle reasons sampled during the timed region."""
+    Q = ("clocks.sm,clocks.max.sm,power.draw,clocks_event_reasons.hw_slowdown,"
+         "clocks_event_reasons.hw_thermal_slowdown,clocks_event_reasons.sw_thermal_slowdown,"
+         "clocks_event_reasons.sw_power_cap")
+
+    def __init__(self, index):
+        self.index, self.rows, self.stop_ev = index, [], threading.Event()
+
+    def _run(self):
+        while not self.stop_ev.is_set():
+            try:
+                out = subprocess.run(["nvidia-smi", "-i", str(self.index), f"--query-gpu={self.Q}",
+                                      "--format=csv,noheader,nounits"], capture_output=True, text=True,
+                                     timeout=5).stdout.strip()
+                if out:
+                    self.rows.append([x.strip() for x in out.split(",")])
+            except Exception:
+                pass
+            self.stop_ev.wait(0.1)
+
+    def __enter__(self):
+        self.th = threading.Thread(target=self._run, daemon=True)
+        self.th.start()
+        return self
+
+    def __exit__(self, *a):
+        self.stop_ev.set()
+        self.th.join(timeout=10)
+
+    def summary(self):
+        if not self.rows:
+            return {"sm_mhz": None, "sm_max_mhz": None, "reasons": ["nvidia-smi unavailable"], "samples": 0}
+        sm = [float(r[0]) for r in self.rows if r[0].replace(".", "").isdigit()]
+        mx = [float(r[1]) for r in self.rows if r[1].replace(".", "").isdigit()]
+        names = ["hw_slowdown", "hw_thermal_slowdown", "sw_thermal_slowdown", "sw_power_cap"]
+        reasons = sorted({names[i] for r in self.rows for i in range(4) if len(r) > 3 + i and r[3 + i] == "Active"})
+        return {"sm_mhz": statistics.median(sm) if sm else None, "sm_max_mhz": max(mx) if mx else None,
+                "reasons": reasons, "samples": len(self.rows)}
+
+
+# --------------------------------------------------------------------- oracle legs
+def oracle_steps(cfg, g, train, labels, n_steps, world=1):
+    """Time the oracle (test infrastructure, single thread) on the first n_steps
+    global steps of epoch 0: sampling + compaction + fp64 SAGE fwd/bwd."""
+    from threadpoolctl import threadpool_limits
+
+    import oracle
+    from oracle import model
+    params = [(W.astype(np.float64), b.astype(np.float64)) for W, b in aptgen.weights(cfg)]
+    perm = oracle.epoch_perm(train, cfg.sample_seed, 0)
+    B = world * cfg.batch
+    times, seeds_done = [], 0
+    with threadpool_limits(limits=1):
+        for t in range(n_steps):
+            seeds = perm[t * B:(t + 1) * B]
+            t0 = time.perf_counter()
+            blocks = oracle.sample_blocks(g, seeds, cfg.fanouts, cfg.sample_seed, t)
+            model.train_step(blocks, cfg.feat_seed, cfg.dim, params, labels[seeds], len(seeds), "bf16")
+            times.append(time.perf_counter() - t0)
+            seeds_done += len(seeds)
+    return times, seeds_done
+
+
+def run_reference(args, cfg):
+    rank, world, _ = dist_env()
+    if rank != 0:
+        return 0
+    g = aptgen.make_graph(cfg)
+    train = aptgen.train_nodes(g, cfg)
+    labels = aptgen.labels(cfg, g.n)
+    n = args.warmup + args.steps
+    times, _ = oracle_steps(cfg, g, train, labels, n, args.gpus)
+    timed = times[args.warmup:]
+    B = args.gpus * cfg.batch
+    ms = 1e3 * sum(timed) / len(timed)
+    value = B / (ms / 1e3)
+    sample = (f"{args.steps} timed global steps of epoch 0 after {args.warmup} warm-up, {B} seeds each, "
+              f"full fanout {list(cfg.fanouts)} sampling + fp64 SAGE fwd/bwd, one host thread")
+    line = {"impl": "reference", "metric": METRIC, "value": value, "unit": "seeds/s", "n_gpus": args.gpus,
+            "steps": args.steps, "warmup": args.warmup, "ms_per_step": ms, "higher_is_better": True,
+            "scaling": "weak", "vs_baseline": None, "dtype": "f64", "data": "synthetic",
+            "config": workload_config(cfg),
+            "cpu_baseline": {"value": value, "unit": "seeds/s", "cores": 1, "kind": "oracle", "sample": sample},
+            "e2e": {"value": value, "unit": "seeds/s", "h2d_bytes_per_step": 0, "d2h_bytes_per_step": 0}}
+    print(json.dumps(line), flush=True)
+    return 0
+
+
+# --------------------------------------------------------------------- product leg
+def run_apt(args, cfg):
+    import torch
+    import torch.distributed as dist
+
+    import paper_conf_ppopp_mal0c0wlc25_b200.apt as A
+
+    rank, world, local = dist_env()
+    if world != args.gpus:
+        raise SystemExit(f"--gpus {args.gpus} but WORLD_SIZE={world}")
+    torch.cuda.set_device(local)
+    if world > 1:
+        dist.init_process_group("nccl", device_id=torch.device("cuda", local))
+    # one non-default stream shared by torch (events, L2 flush) and the library
+    stream = torch.cuda.Stream()
+    torch.cuda.set_stream(stream)
+    A.lib()   # fails loudly if libapt.so is missing: there is no CPU path
+
+    g = aptgen.make_graph(cfg)
+    train = aptgen.train_nodes(g, cfg)
+    labels = aptgen.labels(cfg, g.n)
+    part = aptgen.partition(g.n, world)
+    dt = A.DTYPE[args.dtype]
+    ctx = A.Ctx(rank if world > 1 else 0, world, local, stream.cuda_stream)
+    if world > 1:
+        raise SystemExit("multi-process strategies are not wired into bench.py yet")
+    gr = ctx.graph_load(g.indptr, g.indices, part)
+    strat = A.STRATEGY[args.strategy]
+    fs = ctx.fstore_create(gr, strat if strat == A.NFP else A.GDP, dt, cfg.dim, None, cfg.feat_seed)
+    dims = [cfg.dim] + [d for _, d in cfg.dims()]
+    tr = A.Trainer(ctx, gr, fs, dims, cfg.fanouts, cfg.batch, dt, 0.05, cfg.sample_seed, cfg.feat_seed, strat, labels)
+    tr.set_params(aptgen.weights(cfg))
+    tr.set_epoch(train, 0)
+    tr.use_graph(not args.no_graph)
+    spe = tr.steps_per_epoch()
+
+    flush = torch.empty(256 << 20, dtype=torch.uint8, device="cuda")   # 256 MB > 126 MB L2
+    for i in range(args.warmup):
+        tr.step(i % spe)
+    torch.cuda.synchronize()
+
+    K = args.steps
+    ev = [(torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)) for _ in range(K)]
+    agg_ms, phases, step_ids, agg_bytes = [], [], [], []
+    bf = 2 if args.dtype == "bf16" else 4
+    if world > 1:
+        dist.barrier()
+    torch.cuda.synchronize()
+    l0 = ctx.launches()
+    with ClockSampler(local) as clk:
+        for i in range(K):
+            s = (args.warmup + i) % spe
+            flush.zero_()                      # L2 flushed between timed steps (outside the events)
+            ev[i][0].record(stream)
+            tr.step(s)
+            ev[i][1].record(stream)
+            ph = tr.phase_ms()                 # syncs; device time inside the step comes from events
+            phases.append(ph)
+            agg_ms.append(ph[5])
+            step_ids.append(s)
+            agg_bytes.append(layer1_bytes(ctx, gr, tr, cfg, rank, s, bf))   # outside the events
+        torch.cuda.synchronize()
+    launches = ctx.launches() - l0
+    if world > 1:
+        dist.barrier()
+    step_ms = [a.elapsed_time(b) for a, b in ev]
+    ms_local = sum(step_ms) / K
+    ms = ms_local
+    if world > 1:
+        tt = torch.tensor([ms_local], device="cuda")
+        dist.all_reduce(tt, op=dist.ReduceOp.MAX)
+        ms = float(tt.item())
+    value = world * cfg.batch / (ms / 1e3)
+
+    # ---- e2e: host global batch in (pinned), host loss out, through apt_trainer_step_host
+    rng = np.random.default_rng(1234)
+    host_perm = rng.permutation(train)
+    B = world * cfg.batch
+    e2e_times, h2d = [], 0
+    tr.use_graph(False)
+    for i in range(args.warmup + args.e2e_steps):
+        gb = torch.as_tensor(host_perm[(i * B) % (len(host_perm) - B):][:B].copy()).pin_memory()
+        if world > 1:
+            dist.barrier()
+        torch.cuda.synchronize()
+        t0 = time.perf_counter()
+        tr.step_host(gb, i % spe)
+        t1 = time.perf_counter()
+        if i >= args.warmup:
+            e2e_times.append(t1 - t0)
+            h2d = 4 * len(gb) // world + 8   # int32 seeds of this rank + 8-B header (int64 ids converted on host)
+    e2e_s = sum(e2e_times) / len(e2e_times)
+    if world > 1:
+        tt = torch.tensor([e2e_s], device="cuda")
+        dist.all_reduce(tt, op=dist.ReduceOp.MAX)
+        e2e_s = float(tt.item())
+
+    peaks = json.load(open(os.path.join(ROOT, "MEASURED_PEAKS.json"))) if os.path.exists(
+        os.path.join(ROOT, "MEASURED_PEAKS.json")) else None
+    hbm_peak = peaks["hbm_gbs"] if peaks else 6650.0
+    achieved = sum(agg_bytes) / (sum(agg_ms) * 1e-3) / 1e9
+    mean_agg = sum(agg_ms) / len(agg_ms)
+    phase_mean = [sum(p[j] for p in phases) / len(phases) for j in range(6)]
+
+    out = {
+        "metric": METRIC, "value": value, "unit": "seeds/s", "n_gpus": world, "steps": K, "warmup": args.warmup,
+        "ms_per_step": ms, "higher_is_better": True, "scaling": "weak", "vs_baseline": None,
+        "dtype": args.dtype, "data": "synthetic",
+        "config": dict(workload_config(cfg), strategy=args.strategy, parallelism=f"{args.strategy.lower()}{world}",
+                       global_batch=B, l2="flushed between timed steps (256 MB write); inputs also > L2",
+                       cuda_graph=not args.no_graph),
+        "e2e": {"value": B / e2e_s, "unit": "seeds/s", "h2d_bytes_per_step": h2d, "d2h_bytes_per_step": 4},
+        "gpu_launches": int(launches),
+        "roofline": {"bound": "hbm", "achieved": achieved, "peak": hbm_peak, "unit": "GB/s",
+                     "frac": (achieved / hbm_peak) if achieved else None, "traffic": None,
+                     "kernel": "agg_kernel (layer-1 fused gather+mean)",
+                     "peak_source": "MEASURED_PEAKS.json hbm_gbs" if peaks else "fallback 6.65 TB/s",
+                     "share_of_step": mean_agg / ms_local},
+        "phases_ms": {"sample": phase_mean[0], "layer1_fwd": phase_mean[1], "upper_fwd_loss": phase_mean[2],
+                      "backward": phase_mean[3], "allreduce_sgd": phase_mean[4], "agg_kernel": phase_mean[5]},
+        "clocks": clk.summary(),
+    }
+    if rank == 0 and world == 1 and not args.no_cpu_baseline:
+        times, nseeds = oracle_steps(cfg, g, train, labels, args.cpu_steps, 1)
+        out["cpu_baseline"] = {"value": nseeds / sum(times), "unit": "seeds/s", "cores": 1, "kind": "oracle",
+                               "sample": f"first {args.cpu_steps} steps of epoch 0 ({cfg.batch} seeds each, "
+                                         f"full step: sampling + fp64 SAGE fwd/bwd), one host thread"}
+    if rank == 0:
+        print(json.dumps(out), flush=True)
+    if world > 1:
+        dist.destroy_process_group()
+    return 0
+
+
+def layer1_bytes(ctx, gr, tr, cfg, rank, step, bf):
+    """Algorithmic bytes of the layer-1 fused gather+mean launch of `step`:
+    cnt N_d*4 + neighbour ids E_1*4 + unique source rows U*d*b_f + Z write N_d*d*b_z, with
+    N_d, E_1, U from apt_sample on the same seeds and step (bit-identical blocks by O2/O3)."""
+    import torch
+    seeds = torch.as_tensor(tr.read("seeds", rank=rank)[:, 0].astype(np.int64)).cuda()
+    b = ctx.sample(gr, seeds, len(seeds), cfg.fanouts, cfg.sample_seed, step)
+    v = b.block(len(cfg.fanouts) - 1)
+    n = v.n_dst * 4 + v.n_edges * 4 + v.n_src * cfg.dim * bf + v.n_dst * cfg.dim * bf
+    b.close()
+    return n
+
+
+def main():
+    args = parse()
+    cfg = aptgen.CONFIGS[args.config]
+    if args.impl == "reference":
+        return run_reference(args, cfg)
+    return run_apt(args, cfg)
+
+
+if __name__ == "__main__":
+    sys.exit(main())

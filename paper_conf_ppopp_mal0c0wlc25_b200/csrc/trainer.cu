@@ -11,6 +11,7 @@
 // Every count stays on the device, every grid is sized by an upper bound:
 // the step issues no host synchronisation and can be replayed as a CUDA graph.
 #include <algorithm>
+#include <vector>
 #include <cstring>
 #include <cub/device/device_radix_sort.cuh>
 
@@ -44,6 +45,17 @@ __global__ void allreduce_sum_kernel(float* const* tab, int C, int64_t n) {
     for (int r = 0; r < C; ++r) tab[r][i] = s;
   }
 }
+
+// Phase events: inside a stream capture they must become external event-record
+// nodes (so replays time the phases); outside a capture a plain record.
+static cudaError_t record_ev(apt_trainer* t, int i) {
+  return t->capturing ? cudaEventRecordWithFlags(t->ev[i], t->ctx->stream, cudaEventRecordExternal)
+                      : cudaEventRecord(t->ev[i], t->ctx->stream);
+}
+
+// The step id enters the device as a kernel argument (no host cell that a later
+// call could overwrite before the copy runs); graph replays patch the argument.
+__global__ void set_step_kernel(uint64_t* step_dev, uint64_t step) { *step_dev = step; }
 
 __global__ void zero_rows_kernel(float* p, int64_t pitch, const int32_t* n_p) {
   const int64_t total = int64_t(*n_p) * pitch;
@@ -122,8 +134,6 @@ apt_status apt_trainer_create(apt_ctx* c, const apt_graph* g, const apt_fstore* 
   const int K = t->K, C = t->world;
   t->labels = A.alloc<int32_t>(g->n, false);
   t->step_dev = A.alloc<uint64_t>(1, true);
-  CK(c, cudaMallocHost(&t->step_pinned, 8));
-  *t->step_pinned = 0;
   CK(c, cudaMemcpyAsync(t->labels, labels, sizeof(int32_t) * g->n, cudaMemcpyHostToDevice, c->stream));
   const int64_t n_words = ceil_div(g->n, 32);
   // upper bounds per hop.  SNP/DNP seeds follow the partition: up to C*B on one rank.
@@ -220,9 +230,9 @@ apt_status apt_trainer_destroy(apt_trainer* t) {
   if (!t) return APT_OK;
   cudaStreamSynchronize(t->ctx->stream);
   if (t->gexec) cudaGraphExecDestroy(t->gexec);
+  if (t->graph) cudaGraphDestroy(t->graph);
   for (int i = 0; i < 8; ++i)
     if (t->ev[i]) cudaEventDestroy(t->ev[i]);
-  if (t->step_pinned) cudaFreeHost(t->step_pinned);
   delete t;
   return APT_OK;
 }
@@ -331,10 +341,10 @@ apt_status layer1_fwd_gdp(apt_trainer* t, RankState& rs, bool time_it) {
   a.n_dst = hp.n_dst; a.max_dst = hp.max_dst; a.dim = L.d_in;
   if (t->m.dtype == APT_BF16) { a.z_bf16 = L.Zb; a.z_bf16_pitch = L.zb_pitch; }
   else { a.z_f32 = L.Zf; a.z_f32_pitch = L.zf_pitch; }
-  if (time_it) CK(c, cudaEventRecord(t->ev[6], c->stream));
+  if (time_it) CK(c, record_ev(t, 6));
   CK(c, launch_agg_fstore(a, feat_view(t->f, rs.rank), c->stream));
   c->launches++;
-  if (time_it) CK(c, cudaEventRecord(t->ev[7], c->stream));
+  if (time_it) CK(c, record_ev(t, 7));
   return project(t, L, L.Zb, L.Zf, L.zb_pitch, L.zf_pitch, L.n_rows, L.max_rows, L.d_in, L.W, L.Wb, L.b,
                  t->K > 1 ? 1 : 0, L.H, nullptr, nullptr, nullptr);
 }
@@ -427,12 +437,12 @@ apt_status allreduce_sgd(apt_trainer* t, int update) {
 apt_status step_body(apt_trainer* t, int update, bool host_batch) {
   apt_ctx* c = t->ctx;
   const bool gdp = t->world == 1 || t->s == APT_GDP;
-  CK(c, cudaEventRecord(t->ev[0], c->stream));
+  CK(c, record_ev(t, 0));
   for (auto& rs : t->R) {
     apt_status s = phase_sample(t, rs, host_batch);
     if (s != APT_OK) return s;
   }
-  CK(c, cudaEventRecord(t->ev[1], c->stream));
+  CK(c, record_ev(t, 1));
   if (gdp) {
     bool first = true;
     for (auto& rs : t->R) {
@@ -444,12 +454,12 @@ apt_status step_body(apt_trainer* t, int update, bool host_batch) {
     apt_status s = layer1_fwd_strategy(t);
     if (s != APT_OK) return s;
   }
-  CK(c, cudaEventRecord(t->ev[2], c->stream));
+  CK(c, record_ev(t, 2));
   for (auto& rs : t->R) {
     apt_status s = upper_fwd_loss(t, rs);
     if (s != APT_OK) return s;
   }
-  CK(c, cudaEventRecord(t->ev[3], c->stream));
+  CK(c, record_ev(t, 3));
   // zero the gradient accumulators, then backward
   for (auto& rs : t->R) {
     int64_t P = 0;
@@ -469,10 +479,10 @@ apt_status step_body(apt_trainer* t, int update, bool host_batch) {
     apt_status s = layer1_bwd_strategy(t);
     if (s != APT_OK) return s;
   }
-  CK(c, cudaEventRecord(t->ev[4], c->stream));
+  CK(c, record_ev(t, 4));
   apt_status s = allreduce_sgd(t, update);
   if (s != APT_OK) return s;
-  CK(c, cudaEventRecord(t->ev[5], c->stream));
+  CK(c, record_ev(t, 5));
   t->ev_ok = true;
   return APT_OK;
 }
@@ -485,28 +495,62 @@ apt_status apt_trainer_step(apt_trainer* t, int64_t step, int update) {
   if (!t || !t->perm) return set_err(t ? t->ctx : nullptr, APT_E_STATE, "apt_trainer_step: call apt_trainer_set_epoch first");
   apt_ctx* c = t->ctx;
   if (c->broken) return set_err(c, APT_E_STATE, "ctx is broken by an earlier CUDA error");
-  // the step id reaches the device through a pinned cell copied on the stream,
-  // so a captured CUDA graph replays with the current value
-  *t->step_pinned = uint64_t(step);
   if (t->use_graph) {
     if (!t->gexec || t->graph_update != update) {
       if (t->gexec) { cudaGraphExecDestroy(t->gexec); t->gexec = nullptr; }
+      if (t->graph) { cudaGraphDestroy(t->graph); t->graph = nullptr; }
       cudaGraph_t graph;
       CK(c, cudaStreamBeginCapture(c->stream, cudaStreamCaptureModeThreadLocal));
-      cudaMemcpyAsync(t->step_dev, t->step_pinned, 8, cudaMemcpyHostToDevice, c->stream);
+      set_step_kernel<<<1, 1, 0, c->stream>>>(t->step_dev, uint64_t(step));
+      const int64_t l0 = c->launches;
+      t->capturing = true;
       apt_status s = step_body(t, update, false);
+      t->capturing = false;
       cudaError_t e = cudaStreamEndCapture(c->stream, &graph);
+      t->launches_per_step = c->launches - l0 + 1;   // counted at replay, not at capture
+      c->launches = l0;
       if (s != APT_OK) return s;
       CK(c, e);
+      // find the set_step node so replays can patch the step id
+      size_t n = 0;
+      CK(c, cudaGraphGetNodes(graph, nullptr, &n));
+      std::vector<cudaGraphNode_t> nodes(n);
+      CK(c, cudaGraphGetNodes(graph, nodes.data(), &n));
+      t->step_node = nullptr;
+      for (auto nd : nodes) {
+        cudaGraphNodeType ty;
+        if (cudaGraphNodeGetType(nd, &ty) != cudaSuccess || ty != cudaGraphNodeTypeKernel) continue;
+        cudaKernelNodeParams kp;
+        if (cudaGraphKernelNodeGetParams(nd, &kp) == cudaSuccess && kp.func == (void*)set_step_kernel) {
+          t->step_node = nd;
+          break;
+        }
+      }
+      if (!t->step_node) { cudaGraphDestroy(graph); return set_err(c, APT_E_CUDA, "step node not found in graph"); }
       CK(c, cudaGraphInstantiate(&t->gexec, graph, 0));
-      cudaGraphDestroy(graph);
+      t->graph = graph;
       t->graph_update = update;
     }
+    uint64_t* sd = t->step_dev;
+    uint64_t sv = uint64_t(step);
+    void* args[2] = {&sd, &sv};
+    cudaKernelNodeParams kp{};
+    kp.func = (void*)set_step_kernel;
+    kp.gridDim = dim3(1);
+    kp.blockDim = dim3(1);
+    kp.kernelParams = args;
+    CK(c, cudaGraphExecKernelNodeSetParams(t->gexec, t->step_node, &kp));
     CK(c, cudaGraphLaunch(t->gexec, c->stream));
+    c->launches += t->launches_per_step;
     return APT_OK;
   }
-  CK(c, cudaMemcpyAsync(t->step_dev, t->step_pinned, 8, cudaMemcpyHostToDevice, c->stream));
-  return step_body(t, update, false);
+  set_step_kernel<<<1, 1, 0, c->stream>>>(t->step_dev, uint64_t(step));
+  CK(c, cudaGetLastError());
+  const int64_t l0 = c->launches;
+  c->launches++;
+  apt_status s = step_body(t, update, false);
+  t->launches_per_step = c->launches - l0;
+  return s;
 }
 
 apt_status apt_trainer_step_host(apt_trainer* t, const int64_t* gbatch, int64_t n_global, int64_t step, int update,
@@ -527,8 +571,9 @@ apt_status apt_trainer_step_host(apt_trainer* t, const int64_t* gbatch, int64_t 
     CK(c, cudaMemcpyAsync(rs.seeds, mine.data(), sizeof(int32_t) * mine.size(), cudaMemcpyHostToDevice, c->stream));
     CK(c, cudaMemcpyAsync(rs.small, hdr, sizeof hdr, cudaMemcpyHostToDevice, c->stream));
   }
-  *t->step_pinned = uint64_t(step);
-  CK(c, cudaMemcpyAsync(t->step_dev, t->step_pinned, 8, cudaMemcpyHostToDevice, c->stream));
+  set_step_kernel<<<1, 1, 0, c->stream>>>(t->step_dev, uint64_t(step));
+  CK(c, cudaGetLastError());
+  c->launches++;
   apt_status s = step_body(t, update, true);
   if (s != APT_OK) return s;
   return apt_trainer_loss(t, loss_host);

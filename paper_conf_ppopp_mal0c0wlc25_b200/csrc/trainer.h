@@ -90,12 +90,15 @@ struct apt_trainer {
   int32_t* perm = nullptr;
   int64_t n_train = 0, steps_per_epoch = 1;
   uint64_t* step_dev = nullptr;
-  uint64_t* step_pinned = nullptr;
   std::vector<apt::RankState> R;
   // device pointer tables for cross-rank kernels
   float** dW_tab = nullptr;
   bool use_graph = false;
+  bool capturing = false;
   cudaGraphExec_t gexec = nullptr;
+  cudaGraph_t graph = nullptr;
+  cudaGraphNode_t step_node = nullptr;
+  int64_t launches_per_step = 0;
   int graph_update = -1;
   cudaEvent_t ev[8] = {};
   bool ev_ok = false;

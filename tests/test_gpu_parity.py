@@ -148,7 +148,7 @@ def test_project_tcgen05_bf16(A, ctx, M, N, K):
     rng = np.random.default_rng(M + N + K)
     kp = (K + 7) // 8 * 8
     Z = oracle.bf16_round(rng.normal(size=(M, K)))
-    W = rng.normal(size=(N, K)).astype(np.float32) / np.sqrt(K)
+    W = (rng.normal(size=(N, K)) / np.sqrt(K)).astype(np.float32)
     bias = rng.normal(size=N).astype(np.float32)
     Zb = np.zeros((M, kp), np.uint16)
     Zb[:, :K] = (Z.astype(np.float32).view(np.uint32) >> 16).astype(np.uint16)
@@ -231,7 +231,8 @@ def test_sgd_update_and_graph_replay(A, ctx, tiny):
             tr.step(s, update=True)
         outs.append(tr.get_params())
     for (W0, b0), (W1, b1) in zip(*outs):
-        assert np.allclose(W0, W1, rtol=1e-6, atol=1e-7) and np.allclose(b0, b1, rtol=1e-6, atol=1e-7)
+        assert np.allclose(W0, W1, rtol=1e-6, atol=1e-7), np.abs(W0 - W1).max()
+        assert np.allclose(b0, b1, rtol=1e-6, atol=1e-7), np.abs(b0 - b1).max()
     # one step against the oracle's SGD
     tr, params, labels = _trainer(A, ctx, cfg, g, train, "f32", lr=0.5)
     tr.step(0, update=True)
