@@ -179,6 +179,15 @@ apt_status apt_aggregate_bwd(apt_ctx* ctx, const apt_block_view* blk, const floa
 apt_status apt_project(apt_ctx* ctx, const void* Z, int64_t z_pitch, apt_dtype dtype, const float* W,
                        const float* bias, int64_t M, int N, int K, int relu, float* Y, int64_t y_pitch);
 
+/* Weight gradient of the projection (S11; reading O5): dW[o][i] += sum_r
+ * G[r][o] Z[r][i] and db[o] += sum_r G[r][o] over rows r < rows (accumulates
+ * into dW [d_out x d_in] and db [d_out], device fp32; db may be NULL).  G device
+ * fp32 [rows x g_pitch]; Z device [rows x z_pitch] of dtype.  APT_BF16: G is
+ * rounded to bf16 and the contraction runs on tcgen05 (d_out <= 256, d_in < 320);
+ * APT_F32: exact fp32 CUDA cores.  Syncs.                                    */
+apt_status apt_weight_grad(apt_ctx* ctx, const float* G, int64_t g_pitch, const void* Z, int64_t z_pitch,
+                           apt_dtype dtype, int64_t rows, int d_out, int d_in, float* dW, float* db);
+
 /* ------------------------------------------------------------------ trainer */
 /* The per-mini-batch step (P:110 sampling -> loading -> training) under one
  * strategy, for every rank hosted by ctx.  labels: host int32[n_nodes].      */

@@ -76,6 +76,7 @@ def lib():
             "apt_aggregate": [vp, vp, vp, i32, i32, i64, vp, i64],
             "apt_aggregate_bwd": [vp, vp, vp, i32, i64, vp, i64],
             "apt_project": [vp, vp, i64, i32, vp, vp, i64, i32, i32, i32, vp, i64],
+            "apt_weight_grad": [vp, vp, i64, vp, i64, i32, i64, i32, i32, vp, vp],
             "apt_trainer_create": [vp, vp, vp, vp, i32, vp, vp], "apt_trainer_destroy": [vp],
             "apt_trainer_set_params": [vp, i32, vp, vp], "apt_trainer_get_params": [vp, i32, i32, vp, vp],
             "apt_trainer_set_epoch": [vp, vp, i64, u64], "apt_trainer_step": [vp, i64, i32],
@@ -181,6 +182,10 @@ class Ctx:
     def project(self, Z_dev, z_pitch, dtype, W_dev, bias_dev, M, N, K, relu, Y_dev, y_pitch):
         self.ck(lib().apt_project(self.h, _ptr(Z_dev), z_pitch, dtype, _ptr(W_dev), _ptr(bias_dev), M, N, K, relu,
                                   _ptr(Y_dev), y_pitch))
+
+    def weight_grad(self, G_dev, g_pitch, Z_dev, z_pitch, dtype, rows, d_out, d_in, dW_dev, db_dev=None):
+        self.ck(lib().apt_weight_grad(self.h, _ptr(G_dev), g_pitch, _ptr(Z_dev), z_pitch, dtype, rows, d_out, d_in,
+                                      _ptr(dW_dev), _ptr(db_dev)))
 
     def profile_links(self):
         bw = BwProfile()

@@ -114,6 +114,7 @@ __global__ void __launch_bounds__(256) agg_kernel(AggArgs a, Src src) {
       }
     }
     if (g != 0 || !active) continue;
+    if (a.z_ones && lane == 0) a.z_bf16[i * a.z_bf16_pitch + a.dim] = 0x3F80;   // bf16 1.0: bias-gradient column
     const float fdeg = float(deg);
 #pragma unroll
     for (int p = 0; p < VPL; ++p) {

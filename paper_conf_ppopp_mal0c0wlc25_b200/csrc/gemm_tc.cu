@@ -1,20 +1,36 @@
-// gemm_tc.cu -- S8: the dense projection Y = Z W^T + b (Fig. 5 "dense
-// tensor multiplication between H^0 and W") on the 5th-generation tensor cores.
+// gemm_tc.cu -- the dense contractions of the step on the 5th-generation tensor
+// cores (tcgen05, bf16 operands, fp32 accumulation in TMEM):
 //
-// sm_100a design (DESIGN.md §Kernels/K11):
-//  * persistent CTAs (grid <= 148), one 128-row M tile per iteration;
-//  * warp 0: TMA producer.  W (N x K, bf16, <= 256 x 256) is loaded once per CTA
-//    and stays resident in shared memory; Z tiles (128 x 64 bf16, 128B swizzle)
-//    stream through a 4-stage mbarrier ring;
-//  * warp 1: TMEM allocator + single-thread tcgen05.mma issuer
-//    (kind::f16, M=128, N=BN, K=16 per instruction), accumulators double
-//    buffered in TMEM (2 x BN fp32 columns) so the epilogue of tile i overlaps
-//    the MMAs of tile i+1;
-//  * warps 2..5: epilogue.  tcgen05.ld 32x32b.x16 -> +bias -> ReLU -> fp32
-//    stores; a row can be routed to another rank's buffer (peer-store epilogue
-//    used by the DNP / SNP / NFP reshuffle).
+//   S8   projection      Y  = Z W^T + b (ReLU)     (Eq. 1; Fig. 5
+//                                                  "dense tensor multiplication")
+//   S10  input gradient  dZ = G W                  (backward of the projection)
+//   S11  weight gradient dW = G^T Z, db = G^T 1    (split over the rows)
+//
+// sm_100a design (DESIGN.md §Kernels):
+//  * rowtile kernel (projection, dZ): persistent CTAs (grid <= #SMs), one
+//    128-row M tile per iteration.  The B operand (W, <= 256 x 256 bf16) is
+//    TMA-loaded once per CTA and stays resident in shared memory; A tiles
+//    (128 x 64 bf16, 128-B swizzle) stream through a 4-stage mbarrier ring.
+//    Warp 0 = TMA producer, warp 1 = TMEM allocator + single-thread MMA issuer
+//    (M=128, N=BN, K=16 per instruction) with double-buffered accumulators so
+//    the epilogue of tile i overlaps the MMAs of tile i+1, warps 2..5 =
+//    epilogue (tcgen05.ld 32x32b -> +bias -> ReLU -> fp32 stores; a row may be
+//    routed to another rank's buffer: the peer-store epilogue of the strategies).
+//  * wgrad kernel (dW, db): the reduction runs over the sampled rows, so both
+//    operands are MN-major in memory (G [rows x d_out], Z [rows x d_in]); grid =
+//    (row splits) x (128-wide d_out tiles), each CTA accumulates its row range in
+//    TMEM (N up to 512 columns: d_in plus the all-ones column of Z that turns
+//    the bias gradient into one more output column), then adds it into dW/db
+//    with 16-byte vector reductions.
+// Operand layouts (CUTLASS canonical forms, uint128 units, SW128):
+//  * K-major : ((8,m),(8,2)) : ((8,SBO),(1,...)), rows of 128 B, SBO = 1024 B;
+//              the k-th K=16 slice starts 32 B further.
+//  * MN-major: ((8,n),(8,k)) : ((1,LBO),(8,SBO)); one TMA box = 64 MN x 64 K =
+//              8 KB, boxes of consecutive MN blocks 8 KB apart (LBO = 8192),
+//              8-row K groups 1024 B apart (SBO); the k-th K=16 slice starts
+//              2048 B further.
 // The projection is HBM-bound (AI <= 114 FLOP/B < ridge ~250), so the design
-// goal is streaming Z and Y at full bandwidth, not MMA throughput.
+// goal is streaming A and the outputs at full bandwidth, not MMA throughput.
 #include "common.cuh"
 #include "kernels.h"
 #include <cuda.h>
@@ -31,6 +47,7 @@ constexpr int BK = 64;              // 64 bf16 = 128 B = one swizzle row
 constexpr int STAGES = 4;
 constexpr int A_STAGE_BYTES = BM * BK * 2;   // 16 KB
 constexpr int THREADS = 192;        // 6 warps
+constexpr int MNBLK = 8192;         // one MN-major TMA box (64 x 64 bf16)
 
 __device__ __forceinline__ uint32_t smem_u32(const void* p) {
   return static_cast<uint32_t>(__cvta_generic_to_shared(p));
@@ -69,11 +86,20 @@ __device__ __forceinline__ void tma_load_2d(void* smem_dst, const CUtensorMap* m
 __device__ __forceinline__ void fence_before() { asm volatile("tcgen05.fence::before_thread_sync;" ::: "memory"); }
 __device__ __forceinline__ void fence_after() { asm volatile("tcgen05.fence::after_thread_sync;" ::: "memory"); }
 
-// K-major operand, 128-byte swizzle: 8-row x 128-B atoms, SBO = 1024 B between
-// atoms along M/N, LBO unused (1), descriptor version 1 (sm_100), layout 2.
-__device__ __forceinline__ uint64_t sw128_desc(uint32_t saddr) {
-  return uint64_t((saddr & 0x3FFFFu) >> 4) | (uint64_t(1) << 16) | (uint64_t(1024 >> 4) << 32) |
-         (uint64_t(1) << 46) | (uint64_t(2) << 61);
+// SW128 shared-memory descriptor (sm_100 version 1, layout type 2).
+__device__ __forceinline__ uint64_t sw128_desc(uint32_t saddr, uint32_t lbo, uint32_t sbo) {
+  return uint64_t((saddr & 0x3FFFFu) >> 4) | (uint64_t((lbo >> 4) & 0x3FFFu) << 16) |
+         (uint64_t((sbo >> 4) & 0x3FFFu) << 32) | (uint64_t(1) << 46) | (uint64_t(2) << 61);
+}
+// K-major tile: k-th K=16 slice of a [rows x 64] SW128 tile.
+__device__ __forceinline__ uint64_t desc_k(uint32_t base, int kk) { return sw128_desc(base + kk * 32, 16, 1024); }
+// MN-major tile: k-th K=16 slice of 64-K-row boxes, MN blocks 8 KB apart.
+__device__ __forceinline__ uint64_t desc_mn(uint32_t base, int kk) { return sw128_desc(base + kk * 2048, MNBLK, 1024); }
+
+// Instruction descriptor, kind::f16: D fp32, A/B bf16, majors, N>>3, M>>4.
+__host__ __device__ __forceinline__ uint32_t idesc_bf16(int M, int N, int a_mn, int b_mn) {
+  return (1u << 4) | (1u << 7) | (1u << 10) | (uint32_t(a_mn) << 15) | (uint32_t(b_mn) << 16) |
+         (uint32_t(N >> 3) << 17) | (uint32_t(M >> 4) << 24);
 }
 
 __device__ __forceinline__ void mma_bf16(uint32_t d_tmem, uint64_t a, uint64_t b, uint32_t idesc, uint32_t accum) {
@@ -99,10 +125,20 @@ __device__ __forceinline__ void tmem_ld16(uint32_t taddr, uint32_t (&r)[16]) {
   asm volatile("tcgen05.wait::ld.sync.aligned;" ::: "memory");
 }
 
-struct Params {
+__device__ __forceinline__ void tmem_alloc(uint32_t* slot, uint32_t cols) {
+  asm volatile("tcgen05.alloc.cta_group::1.sync.aligned.shared::cta.b32 [%0], %1;" ::"r"(smem_u32(slot)), "r"(cols));
+  asm volatile("tcgen05.relinquish_alloc_permit.cta_group::1.sync.aligned;");
+}
+__device__ __forceinline__ void tmem_dealloc(uint32_t base, uint32_t cols) {
+  asm volatile("tcgen05.dealloc.cta_group::1.sync.aligned.b32 %0, %1;" ::"r"(base), "r"(cols));
+}
+
+// ------------------------------------------------------------ row-tile kernel
+struct RowParams {
   int64_t M_max;
   const int32_t* M_dev;
-  int N, BN, nkb, tmem_cols;
+  int N, BN, nkb, tmem_cols, b_mn;
+  uint32_t b_kb_bytes;      // bytes of one resident B k-block
   const float* bias;
   int relu;
   float* Y;
@@ -113,17 +149,16 @@ struct Params {
 };
 
 __global__ void __launch_bounds__(THREADS, 1)
-    proj_kernel(const __grid_constant__ CUtensorMap mapZ, const __grid_constant__ CUtensorMap mapW, Params p) {
+    rowtile_kernel(const __grid_constant__ CUtensorMap mapA, const __grid_constant__ CUtensorMap mapB, RowParams p) {
   extern __shared__ __align__(1024) uint8_t smem_raw[];
-  // 1024-B align the dynamic smem base (SWIZZLE_128B atoms)
   uint8_t* smem = reinterpret_cast<uint8_t*>((reinterpret_cast<uintptr_t>(smem_raw) + 1023) & ~uintptr_t(1023));
   uint8_t* smem_a = smem;                                        // STAGES x 16 KB
-  uint8_t* smem_w = smem + STAGES * A_STAGE_BYTES;               // nkb x BN x 128 B
-  uint64_t* bars = reinterpret_cast<uint64_t*>(smem_w + size_t(p.nkb) * p.BN * 128);
+  uint8_t* smem_b = smem + STAGES * A_STAGE_BYTES;               // nkb x b_kb_bytes
+  uint64_t* bars = reinterpret_cast<uint64_t*>(smem_b + size_t(p.nkb) * p.b_kb_bytes);
   uint64_t* full = bars;                  // [STAGES]
   uint64_t* empty = bars + STAGES;        // [STAGES]
-  uint64_t* wfull = bars + 2 * STAGES;    // [1]
-  uint64_t* tfull = wfull + 1;            // [2]
+  uint64_t* bfull = bars + 2 * STAGES;    // [1]
+  uint64_t* tfull = bfull + 1;            // [2]
   uint64_t* tempty = tfull + 2;           // [2]
   uint32_t* tmem_slot = reinterpret_cast<uint32_t*>(tempty + 2);
 
@@ -133,69 +168,75 @@ __global__ void __launch_bounds__(THREADS, 1)
 
   if (warp == 0 && lane == 0) {
     for (int s = 0; s < STAGES; ++s) { mbar_init(full + s, 1); mbar_init(empty + s, 1); }
-    mbar_init(wfull, 1);
+    mbar_init(bfull, 1);
     for (int a = 0; a < 2; ++a) { mbar_init(tfull + a, 1); mbar_init(tempty + a, 128); }
     asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
-    asm volatile("prefetch.tensormap [%0];" ::"l"(reinterpret_cast<uint64_t>(&mapZ)) : "memory");
-    asm volatile("prefetch.tensormap [%0];" ::"l"(reinterpret_cast<uint64_t>(&mapW)) : "memory");
+    asm volatile("prefetch.tensormap [%0];" ::"l"(reinterpret_cast<uint64_t>(&mapA)) : "memory");
+    asm volatile("prefetch.tensormap [%0];" ::"l"(reinterpret_cast<uint64_t>(&mapB)) : "memory");
   }
-  if (warp == 1) {
-    asm volatile("tcgen05.alloc.cta_group::1.sync.aligned.shared::cta.b32 [%0], %1;" ::"r"(smem_u32(tmem_slot)),
-                 "r"(uint32_t(p.tmem_cols)));
-    asm volatile("tcgen05.relinquish_alloc_permit.cta_group::1.sync.aligned;");
-  }
+  if (warp == 1) tmem_alloc(tmem_slot, uint32_t(p.tmem_cols));
   fence_before();
   __syncthreads();
   fence_after();
   const uint32_t tmem_base = *tmem_slot;
 
   if (warp == 0) {
-    if (lane == 0) {
-      // ---- TMA producer
-      mbar_expect_tx(wfull, uint32_t(p.nkb) * p.BN * 128);
-      for (int kb = 0; kb < p.nkb; ++kb) tma_load_2d(smem_w + size_t(kb) * p.BN * 128, &mapW, wfull, kb * BK, 0);
+    if (lane == 0 && ntiles > int64_t(blockIdx.x)) {
+      // ---- TMA producer: resident B, then the A ring
+      mbar_expect_tx(bfull, uint32_t(p.nkb) * p.b_kb_bytes);
+      const int nb = int(ceil_div(p.BN, 64));
+      for (int kb = 0; kb < p.nkb; ++kb) {
+        uint8_t* dst = smem_b + size_t(kb) * p.b_kb_bytes;
+        if (p.b_mn) {
+          for (int j = 0; j < nb; ++j) tma_load_2d(dst + j * MNBLK, &mapB, bfull, j * 64, kb * BK);
+        } else {
+          tma_load_2d(dst, &mapB, bfull, kb * BK, 0);
+        }
+      }
       int s = 0;
       uint32_t ph = 0;
       for (int64_t t = blockIdx.x; t < ntiles; t += gridDim.x) {
         for (int kb = 0; kb < p.nkb; ++kb) {
           mbar_wait(empty + s, ph ^ 1);
           mbar_expect_tx(full + s, A_STAGE_BYTES);
-          tma_load_2d(smem_a + s * A_STAGE_BYTES, &mapZ, full + s, kb * BK, int(t * BM));
+          tma_load_2d(smem_a + s * A_STAGE_BYTES, &mapA, full + s, kb * BK, int(t * BM));
           if (++s == STAGES) { s = 0; ph ^= 1; }
         }
       }
     }
   } else if (warp == 1) {
     // ---- MMA issuer (one thread)
-    const uint32_t idesc = (1u << 4) | (1u << 7) | (1u << 10) | (uint32_t(p.BN >> 3) << 17) | (uint32_t(BM >> 4) << 24);
-    mbar_wait(wfull, 0);
-    fence_after();
-    int s = 0;
-    uint32_t ph = 0;
-    int acc = 0;
-    uint32_t aph = 0;
-    for (int64_t t = blockIdx.x; t < ntiles; t += gridDim.x) {
-      mbar_wait(tempty + acc, aph ^ 1);
+    if (ntiles > int64_t(blockIdx.x)) {
+      const uint32_t idesc = idesc_bf16(BM, p.BN, 0, p.b_mn);
+      mbar_wait(bfull, 0);
       fence_after();
-      const uint32_t d = tmem_base + uint32_t(acc * p.BN);
-      for (int kb = 0; kb < p.nkb; ++kb) {
-        mbar_wait(full + s, ph);
+      int s = 0;
+      uint32_t ph = 0;
+      int acc = 0;
+      uint32_t aph = 0;
+      for (int64_t t = blockIdx.x; t < ntiles; t += gridDim.x) {
+        mbar_wait(tempty + acc, aph ^ 1);
         fence_after();
-        if (lane == 0) {
-          const uint32_t a0 = smem_u32(smem_a + s * A_STAGE_BYTES);
-          const uint32_t b0 = smem_u32(smem_w + size_t(kb) * p.BN * 128);
+        const uint32_t d = tmem_base + uint32_t(acc * p.BN);
+        for (int kb = 0; kb < p.nkb; ++kb) {
+          mbar_wait(full + s, ph);
+          fence_after();
+          if (lane == 0) {
+            const uint32_t a0 = smem_u32(smem_a + s * A_STAGE_BYTES);
+            const uint32_t b0 = smem_u32(smem_b + size_t(kb) * p.b_kb_bytes);
 #pragma unroll
-          for (int kk = 0; kk < BK / 16; ++kk)
-            mma_bf16(d, sw128_desc(a0 + kk * 32), sw128_desc(b0 + kk * 32), idesc, (kb | kk) != 0);
-          mma_commit(empty + s);            // frees the smem stage when these MMAs finish
+            for (int kk = 0; kk < BK / 16; ++kk)
+              mma_bf16(d, desc_k(a0, kk), p.b_mn ? desc_mn(b0, kk) : desc_k(b0, kk), idesc, (kb | kk) != 0);
+            mma_commit(empty + s);            // frees the smem stage when these MMAs finish
+          }
+          __syncwarp();
+          if (++s == STAGES) { s = 0; ph ^= 1; }
         }
+        if (lane == 0) mma_commit(tfull + acc);   // accumulator ready for the epilogue
         __syncwarp();
-        if (++s == STAGES) { s = 0; ph ^= 1; }
+        acc ^= 1;
+        if (acc == 0) aph ^= 1;
       }
-      if (lane == 0) mma_commit(tfull + acc);   // accumulator ready for the epilogue
-      __syncwarp();
-      acc ^= 1;
-      if (acc == 0) aph ^= 1;
     }
   } else {
     // ---- epilogue warps 2..5: TMEM lane quarter = warp % 4
@@ -241,10 +282,135 @@ __global__ void __launch_bounds__(THREADS, 1)
   __syncthreads();
   if (warp == 1) {
     fence_after();
-    asm volatile("tcgen05.dealloc.cta_group::1.sync.aligned.b32 %0, %1;" ::"r"(tmem_base), "r"(uint32_t(p.tmem_cols)));
+    tmem_dealloc(tmem_base, uint32_t(p.tmem_cols));
   }
 }
 
+// ------------------------------------------------------------ weight-gradient kernel
+constexpr int WG_STAGES = 3;
+
+struct WgradParams {
+  const int32_t* rows_dev;  // number of valid rows (device)
+  int64_t rows_max;
+  int d_out, d_in, BN, nbz, tmem_cols;
+  int ones_col;             // Z column d_in holds 1.0: output column d_in is db
+  uint32_t stage_bytes;     // A (2 x 8 KB) + B (nbz x 8 KB)
+  float* dW;                // [d_out x d_in] (accumulated)
+  float* db;                // [d_out] (accumulated) or null
+};
+
+__global__ void __launch_bounds__(THREADS, 1)
+    wgrad_kernel(const __grid_constant__ CUtensorMap mapG, const __grid_constant__ CUtensorMap mapZ, WgradParams p) {
+  extern __shared__ __align__(1024) uint8_t smem_raw[];
+  uint8_t* smem = reinterpret_cast<uint8_t*>((reinterpret_cast<uintptr_t>(smem_raw) + 1023) & ~uintptr_t(1023));
+  uint64_t* bars = reinterpret_cast<uint64_t*>(smem + size_t(WG_STAGES) * p.stage_bytes);
+  uint64_t* full = bars;
+  uint64_t* empty = bars + WG_STAGES;
+  uint64_t* tfull = bars + 2 * WG_STAGES;
+  uint32_t* tmem_slot = reinterpret_cast<uint32_t*>(tfull + 1);
+
+  const int warp = threadIdx.x >> 5, lane = lane_id();
+  const int64_t rows = std::min<int64_t>(p.rows_max, int64_t(*p.rows_dev));
+  const int64_t nkb_all = ceil_div(rows, BK);
+  const int64_t per = ceil_div(nkb_all, int64_t(gridDim.x));
+  const int64_t kb0 = int64_t(blockIdx.x) * per;
+  const int64_t kb1 = std::min<int64_t>(nkb_all, kb0 + per);
+  const int m0 = blockIdx.y * BM;
+  if (kb0 >= kb1) return;   // uniform for the CTA: nothing to add
+
+  if (warp == 0 && lane == 0) {
+    for (int s = 0; s < WG_STAGES; ++s) { mbar_init(full + s, 1); mbar_init(empty + s, 1); }
+    mbar_init(tfull, 1);
+    asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
+    asm volatile("prefetch.tensormap [%0];" ::"l"(reinterpret_cast<uint64_t>(&mapG)) : "memory");
+    asm volatile("prefetch.tensormap [%0];" ::"l"(reinterpret_cast<uint64_t>(&mapZ)) : "memory");
+  }
+  if (warp == 1) tmem_alloc(tmem_slot, uint32_t(p.tmem_cols));
+  fence_before();
+  __syncthreads();
+  fence_after();
+  const uint32_t tmem_base = *tmem_slot;
+
+  if (warp == 0) {
+    if (lane == 0) {
+      int s = 0;
+      uint32_t ph = 0;
+      // boxes entirely outside the matrices are not loaded: the MMA rows / columns
+      // they feed are never read back by the epilogue
+      const int na = (p.d_out - m0 > 64) ? 2 : 1;
+      const int zcols = p.ones_col ? p.d_in + 1 : p.d_in;
+      const int nz = int(ceil_div(zcols, 64));
+      for (int64_t kb = kb0; kb < kb1; ++kb) {
+        mbar_wait(empty + s, ph ^ 1);
+        mbar_expect_tx(full + s, uint32_t(na + nz) * MNBLK);
+        uint8_t* st = smem + size_t(s) * p.stage_bytes;
+        const int y = int(kb * BK);
+        for (int j = 0; j < na; ++j) tma_load_2d(st + j * MNBLK, &mapG, full + s, m0 + 64 * j, y);
+        for (int j = 0; j < nz; ++j) tma_load_2d(st + 2 * MNBLK + j * MNBLK, &mapZ, full + s, j * 64, y);
+        if (++s == WG_STAGES) { s = 0; ph ^= 1; }
+      }
+    }
+  } else if (warp == 1) {
+    int s = 0;
+    uint32_t ph = 0;
+    for (int64_t kb = kb0; kb < kb1; ++kb) {
+      mbar_wait(full + s, ph);
+      fence_after();
+      if (lane == 0) {
+        const uint32_t a0 = smem_u32(smem + size_t(s) * p.stage_bytes);
+        const uint32_t b0 = a0 + 2 * MNBLK;
+#pragma unroll
+        for (int kk = 0; kk < BK / 16; ++kk) {
+          for (int n0 = 0; n0 < p.BN; n0 += 256) {
+            const int nn = std::min(256, p.BN - n0);
+            mma_bf16(tmem_base + uint32_t(n0), desc_mn(a0, kk), desc_mn(b0 + uint32_t(n0 / 64) * MNBLK, kk),
+                     idesc_bf16(BM, nn, 1, 1), (kb > kb0 || kk) ? 1u : 0u);
+          }
+        }
+        mma_commit(empty + s);
+      }
+      __syncwarp();
+      if (++s == WG_STAGES) { s = 0; ph ^= 1; }
+    }
+    if (lane == 0) mma_commit(tfull);
+    __syncwarp();
+  } else {
+    // ---- epilogue: lane quarter q holds d_out rows m0 + 32q .. +31
+    const int q = warp & 3;
+    mbar_wait(tfull, 0);
+    fence_after();
+    const int o = m0 + q * 32 + lane;
+    const bool valid = o < p.d_out;
+    float* wrow = p.dW + int64_t(o) * p.d_in;
+    const bool vec = (p.d_in & 3) == 0;
+    for (int c = 0; c < p.BN; c += 16) {
+      uint32_t r[16];
+      tmem_ld16(tmem_base + (uint32_t(q * 32) << 16) + uint32_t(c), r);
+      if (!valid) continue;
+      if (vec && c + 16 <= p.d_in) {
+#pragma unroll
+        for (int j = 0; j < 16; j += 4)
+          red_add_v4(wrow + c + j, __uint_as_float(r[j]), __uint_as_float(r[j + 1]), __uint_as_float(r[j + 2]),
+                     __uint_as_float(r[j + 3]));
+      } else {
+#pragma unroll
+        for (int j = 0; j < 16; ++j) {
+          const int col = c + j;
+          if (col < p.d_in) atomicAdd(wrow + col, __uint_as_float(r[j]));
+          else if (col == p.d_in && p.ones_col && p.db) atomicAdd(p.db + o, __uint_as_float(r[j]));
+        }
+      }
+    }
+  }
+  fence_before();
+  __syncthreads();
+  if (warp == 1) {
+    fence_after();
+    tmem_dealloc(tmem_base, uint32_t(p.tmem_cols));
+  }
+}
+
+// ------------------------------------------------------------ host side
 static PFN_cuTensorMapEncodeTiled_v12000 encode_fn() {
   static PFN_cuTensorMapEncodeTiled_v12000 fn = nullptr;
   static std::once_flag once;
@@ -258,6 +424,7 @@ static PFN_cuTensorMapEncodeTiled_v12000 encode_fn() {
   return fn;
 }
 
+// 2-D bf16 map over a row-major [rows x cols] matrix with `pitch_elems` per row.
 static bool make_map(CUtensorMap* m, const void* base, int64_t cols, int64_t rows, int64_t pitch_elems, int box_cols,
                      int box_rows) {
   auto fn = encode_fn();
@@ -272,10 +439,6 @@ static bool make_map(CUtensorMap* m, const void* base, int64_t cols, int64_t row
   return r == CUDA_SUCCESS;
 }
 
-}  // namespace tc
-
-int tc_gemm_supported(int N, int K) { return N >= 1 && N <= 256 && K >= 1 && K <= 256; }
-
 static int sm_count() {
   static int n = 0;
   if (!n) {
@@ -287,6 +450,10 @@ static int sm_count() {
   return n;
 }
 
+}  // namespace tc
+
+int tc_gemm_supported(int N, int K) { return N >= 1 && N <= 256 && K >= 1 && K <= 256; }
+
 cudaError_t launch_tc_gemm(const TcGemmArgs& a, cudaStream_t st) {
   using namespace tc;
   if (!tc_gemm_supported(a.N, a.K)) return cudaErrorInvalidValue;
@@ -295,19 +462,61 @@ cudaError_t launch_tc_gemm(const TcGemmArgs& a, cudaStream_t st) {
   const int nkb = int(ceil_div(a.K, BK));
   int cols = 32;
   while (cols < 2 * BN) cols <<= 1;
-  CUtensorMap mz, mw;
-  if (!make_map(&mz, a.Z, a.K, std::max<int64_t>(a.M_max, 1), a.z_pitch, BK, BM)) return cudaErrorInvalidValue;
-  if (!make_map(&mw, a.W, a.K, a.N, a.w_pitch, BK, BN)) return cudaErrorInvalidValue;
-  Params p{a.M_max, a.M_dev, a.N, BN, nkb, cols, a.bias, a.relu, a.Y, a.y_pitch, a.out_base, a.out_rank, a.out_row};
-  const size_t smem = 1024 + size_t(STAGES) * A_STAGE_BYTES + size_t(nkb) * BN * 128 + 16 * 8 + 16;
+  CUtensorMap ma, mb;
+  if (!make_map(&ma, a.Z, a.K, std::max<int64_t>(a.M_max, 1), a.z_pitch, BK, BM)) return cudaErrorInvalidValue;
+  uint32_t b_kb_bytes;
+  if (a.w_mn) {
+    // W stored [K x N] (N contiguous): boxes of 64 N x 64 K
+    if (!make_map(&mb, a.W, a.N, a.K, a.w_pitch, 64, BK)) return cudaErrorInvalidValue;
+    b_kb_bytes = uint32_t(ceil_div(BN, 64)) * MNBLK;
+  } else {
+    if (!make_map(&mb, a.W, a.K, a.N, a.w_pitch, BK, BN)) return cudaErrorInvalidValue;
+    b_kb_bytes = uint32_t(BN) * 128;
+  }
+  RowParams p{a.M_max, a.M_dev, a.N, BN, nkb, cols, a.w_mn, b_kb_bytes, a.bias, a.relu, a.Y, a.y_pitch,
+              a.out_base, a.out_rank, a.out_row};
+  const size_t smem = 1024 + size_t(STAGES) * A_STAGE_BYTES + size_t(nkb) * b_kb_bytes + 16 * 8 + 16;
+  if (smem > 227 * 1024) return cudaErrorInvalidValue;
   static bool attr_set = false;
   if (!attr_set) {
-    cudaFuncSetAttribute(proj_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize, 227 * 1024);
+    cudaFuncSetAttribute(rowtile_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize, 227 * 1024);
     attr_set = true;
   }
   const int64_t tiles = std::max<int64_t>(1, ceil_div(a.M_max, BM));
   const int grid = int(std::min<int64_t>(tiles, sm_count()));
-  proj_kernel<<<grid, THREADS, smem, st>>>(mz, mw, p);
+  rowtile_kernel<<<grid, THREADS, smem, st>>>(ma, mb, p);
+  return cudaGetLastError();
+}
+
+int tc_wgrad_supported(int d_out, int d_in) { return d_out >= 1 && d_out <= 256 && d_in >= 1 && d_in + 1 <= 320; }
+
+cudaError_t launch_tc_wgrad(const TcWgradArgs& a, cudaStream_t st) {
+  using namespace tc;
+  if (!tc_wgrad_supported(a.d_out, a.d_in)) return cudaErrorInvalidValue;
+  if ((a.g_pitch * 2) % 16 || (a.z_pitch * 2) % 16) return cudaErrorInvalidValue;
+  const int zcols = a.db ? a.d_in + 1 : a.d_in;     // column d_in of Z is all ones (db)
+  if (a.db && a.z_pitch < zcols) return cudaErrorInvalidValue;
+  const int BN = int(round_up(zcols, 16));
+  const int nbz = int(ceil_div(BN, 64));
+  int cols = 32;
+  while (cols < BN) cols <<= 1;
+  CUtensorMap mg, mz;
+  const int64_t rows = std::max<int64_t>(a.rows_max, 1);
+  if (!make_map(&mg, a.G, a.d_out, rows, a.g_pitch, 64, BK)) return cudaErrorInvalidValue;
+  if (!make_map(&mz, a.Z, zcols, rows, a.z_pitch, 64, BK)) return cudaErrorInvalidValue;
+  const uint32_t stage = uint32_t(2 + nbz) * MNBLK;
+  WgradParams p{a.rows_dev, a.rows_max, a.d_out, a.d_in, BN, nbz, cols, a.db ? 1 : 0, stage, a.dW, a.db};
+  const size_t smem = 1024 + size_t(WG_STAGES) * stage + 8 * 8 + 16;
+  if (smem > 227 * 1024) return cudaErrorInvalidValue;
+  static bool attr_set = false;
+  if (!attr_set) {
+    cudaFuncSetAttribute(wgrad_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize, 227 * 1024);
+    attr_set = true;
+  }
+  const int mt = int(ceil_div(a.d_out, BM));
+  const int64_t kbs = std::max<int64_t>(1, ceil_div(a.rows_max, BK));
+  const int splits = int(std::max<int64_t>(1, std::min<int64_t>(kbs, sm_count() / mt)));
+  wgrad_kernel<<<dim3(splits, mt), THREADS, smem, st>>>(mg, mz, p);
   return cudaGetLastError();
 }
 

@@ -96,6 +96,7 @@ struct AggArgs {
   int64_t z_f32_pitch;
   uint16_t* z_bf16;
   int64_t z_bf16_pitch;
+  int z_ones;                  // write 1.0 into bf16 column `dim` (bias-gradient column of the wgrad GEMM)
 };
 cudaError_t launch_agg_fstore(const AggArgs& a, const FeatView& fv, cudaStream_t st);
 cudaError_t launch_agg_csr(const AggArgs& a, cudaStream_t st);
@@ -134,22 +135,42 @@ cudaError_t launch_simt_gemm(const SimtGemmArgs& a, cudaStream_t st);
 // tcgen05 projection: Y[m][n] = sum_k Z[m][k] W[n][k] + bias[n] (relu), bf16 in,
 // fp32 accumulate in TMEM, fp32 out.  Z, W are K-major bf16 with 16-B pitches.
 struct TcGemmArgs {
-  const uint16_t* Z; int64_t z_pitch;  // [M_max x K] bf16
-  const uint16_t* W; int64_t w_pitch;  // [N x K] bf16
+  const uint16_t* Z; int64_t z_pitch;  // A: [M_max x K] bf16 (K-major)
+  const uint16_t* W; int64_t w_pitch;  // B: [N x K] bf16 (K-major), or [K x N] if w_mn
   int64_t M_max; const int32_t* M_dev; int N; int K;
   const float* bias; int relu;
   float* Y; int64_t y_pitch;
   // optional row routing (peer-store epilogue): row m goes to
   // out_base[out_rank[m]] + out_row[m] * y_pitch
   float* const* out_base; const int32_t* out_rank; const int32_t* out_row;
+  int w_mn;                            // B stored N-contiguous (dZ = G W uses W [d_out x d_in] as is)
 };
 int tc_gemm_supported(int N, int K);
 cudaError_t launch_tc_gemm(const TcGemmArgs& a, cudaStream_t st);
 
+// tcgen05 weight gradient: dW[o][i] += sum_r G[r][o] Z[r][i]; db[o] += sum_r G[r][o]
+// (db via Z's all-ones column d_in, required when db != null).  G, Z bf16 row-major;
+// rows beyond *rows_dev up to the next multiple of 64 must be zero in G.
+struct TcWgradArgs {
+  const uint16_t* G; int64_t g_pitch;  // [rows_max x d_out]
+  const uint16_t* Z; int64_t z_pitch;  // [rows_max x (d_in + 1)]
+  const int32_t* rows_dev; int64_t rows_max;
+  int d_out, d_in;
+  float* dW; float* db;
+};
+int tc_wgrad_supported(int d_out, int d_in);
+cudaError_t launch_tc_wgrad(const TcWgradArgs& a, cudaStream_t st);
+
+// Gb = bf16(G * (H > 0)) over rows < n (relu != 0) or bf16(G); rows in
+// [n, round_up(n, 64)) of Gb are zeroed (tail of the tcgen05 row blocks).
+cudaError_t launch_grad_finish(const float* G, int64_t g_pitch, const float* H, int64_t h_pitch, int dim, int relu,
+                               uint16_t* Gb, int64_t gb_pitch, const int32_t* n_dev, int64_t max_n, cudaStream_t st);
+
 // ---------------------------------------------------------------- misc.cu
 cudaError_t launch_ce_loss(const float* logits, int64_t pitch, int n_classes, const int32_t* seeds,
                            const int32_t* n_seeds, int64_t max_seeds, const int32_t* labels,
-                           const int32_t* n_global, float* loss, float* g, int64_t g_pitch, cudaStream_t st);
+                           const int32_t* n_global, float* loss, float* g, int64_t g_pitch, uint16_t* gb,
+                           int64_t gb_pitch, cudaStream_t st);
 cudaError_t launch_relu_bwd(float* g, const float* h, int64_t pitch, int dim, const int32_t* n_dev, int64_t max_n,
                             cudaStream_t st);
 cudaError_t launch_colsum(const float* g, int64_t pitch, int dim, const int32_t* n_dev, int64_t max_n, float* out,
@@ -158,6 +179,8 @@ cudaError_t launch_sgd(float* W, const float* dW, int64_t n, float lr, uint16_t*
                        int64_t bf16_pitch, cudaStream_t st);
 cudaError_t launch_to_bf16(const float* src, int64_t src_pitch, uint16_t* dst, int64_t dst_pitch, int cols,
                            const int32_t* n_dev, int64_t max_n, cudaStream_t st);
+cudaError_t launch_bf16_pad_ones(const uint16_t* src, int64_t src_pitch, uint16_t* dst, int64_t dst_pitch, int cols,
+                                 const int32_t* n_dev, int64_t max_n, cudaStream_t st);
 cudaError_t launch_transpose(const float* src, int rows, int cols, float* dst, cudaStream_t st);
 
 }  // namespace apt

@@ -15,7 +15,8 @@ static int64_t grid_of(int64_t n, int t = 256) {
 __global__ void ce_loss_kernel(const float* __restrict__ logits, int64_t pitch, int C,
                                const int32_t* __restrict__ seeds, const int32_t* __restrict__ n_seeds_p,
                                const int32_t* __restrict__ labels, const int32_t* __restrict__ n_global_p,
-                               float* __restrict__ loss, float* __restrict__ g, int64_t g_pitch) {
+                               float* __restrict__ loss, float* __restrict__ g, int64_t g_pitch,
+                               uint16_t* __restrict__ gb, int64_t gb_pitch, int64_t max_seeds) {
   const int lane = lane_id();
   const int64_t n = *n_seeds_p;
   const float inv_n = 1.0f / float(max(1, *n_global_p));
@@ -34,16 +35,28 @@ __global__ void ce_loss_kernel(const float* __restrict__ logits, int64_t pitch, 
     if (lane == 0) atomicAdd(loss, (lse - row[y]) * inv_n);
     for (int c = lane; c < C; c += 32) {
       const float p = expf(row[c] - lse);
-      g[i * g_pitch + c] = (p - (c == y ? 1.f : 0.f)) * inv_n;
+      const float v = (p - (c == y ? 1.f : 0.f)) * inv_n;
+      g[i * g_pitch + c] = v;
+      if (gb) {
+        __nv_bfloat16 h = __float2bfloat16_rn(v);
+        gb[i * gb_pitch + c] = *reinterpret_cast<uint16_t*>(&h);
+      }
     }
+  }
+  if (gb) {   // zero the tail of the last 64-row block (tcgen05 wgrad reads whole blocks)
+    const int64_t tail_end = std::min<int64_t>(max_seeds, round_up(n, 64));
+    for (int64_t t = int64_t(blockIdx.x) * blockDim.x + threadIdx.x; t < (tail_end - n) * gb_pitch;
+         t += int64_t(gridDim.x) * blockDim.x)
+      gb[n * gb_pitch + t] = 0;
   }
 }
 
 cudaError_t launch_ce_loss(const float* logits, int64_t pitch, int n_classes, const int32_t* seeds,
                            const int32_t* n_seeds, int64_t max_seeds, const int32_t* labels,
-                           const int32_t* n_global, float* loss, float* g, int64_t g_pitch, cudaStream_t st) {
+                           const int32_t* n_global, float* loss, float* g, int64_t g_pitch, uint16_t* gb,
+                           int64_t gb_pitch, cudaStream_t st) {
   ce_loss_kernel<<<grid_of(max_seeds * 32), 256, 0, st>>>(logits, pitch, n_classes, seeds, n_seeds, labels,
-                                                          n_global, loss, g, g_pitch);
+                                                          n_global, loss, g, g_pitch, gb, gb_pitch, max_seeds);
   return cudaGetLastError();
 }
 
@@ -61,6 +74,70 @@ __global__ void relu_bwd_kernel(float* __restrict__ g, const float* __restrict__
 cudaError_t launch_relu_bwd(float* g, const float* h, int64_t pitch, int dim, const int32_t* n_dev, int64_t max_n,
                             cudaStream_t st) {
   relu_bwd_kernel<<<grid_of(max_n * dim), 256, 0, st>>>(g, h, pitch, dim, n_dev);
+  return cudaGetLastError();
+}
+
+// Gb = bf16(G * (H > 0)) (or bf16(G)); the 64-row-block tail of Gb is zeroed.
+// One thread per 4 columns (16-B G / H loads, 8-B Gb stores).
+__global__ void grad_finish_kernel(const float* __restrict__ G, int64_t gp, const float* __restrict__ H, int64_t hp,
+                                   int dim, int relu, uint16_t* __restrict__ Gb, int64_t gbp,
+                                   const int32_t* __restrict__ n_p, int64_t max_n) {
+  const int64_t n = *n_p;
+  const int64_t rows = std::min<int64_t>(max_n, round_up(n, 64));
+  const int V = int(ceil_div(dim, 4));
+  const int64_t total = rows * V;
+  for (int64_t t = int64_t(blockIdx.x) * blockDim.x + threadIdx.x; t < total; t += int64_t(gridDim.x) * blockDim.x) {
+    const int64_t r = t / V;
+    const int c = int(t - r * V) * 4;
+    uint16_t* o = Gb + r * gbp + c;
+    if (r >= n) {
+      for (int q = 0; q < 4 && c + q < dim; ++q) o[q] = 0;
+      continue;
+    }
+    float4 g = *reinterpret_cast<const float4*>(G + r * gp + c);
+    if (relu) {
+      const float4 h = *reinterpret_cast<const float4*>(H + r * hp + c);
+      if (!(h.x > 0.f)) g.x = 0.f;
+      if (!(h.y > 0.f)) g.y = 0.f;
+      if (!(h.z > 0.f)) g.z = 0.f;
+      if (!(h.w > 0.f)) g.w = 0.f;
+    }
+    if (c + 4 <= dim && (gbp & 3) == 0) {
+      *reinterpret_cast<uint2*>(o) = make_uint2(pack_bf16x2(g.x, g.y), pack_bf16x2(g.z, g.w));
+    } else {
+      const float v[4] = {g.x, g.y, g.z, g.w};
+      for (int q = 0; q < 4 && c + q < dim; ++q) {
+        __nv_bfloat16 h = __float2bfloat16_rn(v[q]);
+        o[q] = *reinterpret_cast<uint16_t*>(&h);
+      }
+    }
+  }
+}
+
+cudaError_t launch_grad_finish(const float* G, int64_t g_pitch, const float* H, int64_t h_pitch, int dim, int relu,
+                               uint16_t* Gb, int64_t gb_pitch, const int32_t* n_dev, int64_t max_n, cudaStream_t st) {
+  if ((g_pitch & 3) || (h_pitch & 3)) return cudaErrorInvalidValue;
+  grad_finish_kernel<<<grid_of(max_n * ceil_div(dim, 4)), 256, 0, st>>>(G, g_pitch, H, h_pitch, dim, relu, Gb,
+                                                                          gb_pitch, n_dev, max_n);
+  return cudaGetLastError();
+}
+
+// dst[r][0:cols] = src[r][0:cols], dst[r][cols] = 1.0 (bf16), zero tail rows to the 64-row block.
+__global__ void bf16_pad_ones_kernel(const uint16_t* __restrict__ src, int64_t sp, uint16_t* __restrict__ dst,
+                                     int64_t dp, int cols, const int32_t* __restrict__ n_p, int64_t max_n) {
+  const int64_t n = *n_p;
+  const int64_t rows = std::min<int64_t>(max_n, round_up(n, 64));
+  const int64_t total = rows * dp;
+  for (int64_t t = int64_t(blockIdx.x) * blockDim.x + threadIdx.x; t < total; t += int64_t(gridDim.x) * blockDim.x) {
+    const int64_t r = t / dp;
+    const int c = int(t - r * dp);
+    dst[t] = r >= n ? 0 : c < cols ? src[r * sp + c] : c == cols ? 0x3F80 : 0;
+  }
+}
+
+cudaError_t launch_bf16_pad_ones(const uint16_t* src, int64_t src_pitch, uint16_t* dst, int64_t dst_pitch, int cols,
+                                 const int32_t* n_dev, int64_t max_n, cudaStream_t st) {
+  bf16_pad_ones_kernel<<<grid_of(max_n * dst_pitch), 256, 0, st>>>(src, src_pitch, dst, dst_pitch, cols, n_dev, max_n);
   return cudaGetLastError();
 }
 

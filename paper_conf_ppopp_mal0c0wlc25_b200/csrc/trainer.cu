@@ -74,7 +74,7 @@ apt_status project(apt_trainer* t, const Layer& L, const void* Zb, const float* 
   apt_ctx* c = t->ctx;
   if (t->m.dtype == APT_BF16 && tc_gemm_supported(L.d_out, K)) {
     TcGemmArgs a{static_cast<const uint16_t*>(Zb), z_pitch_b, Wb, L.wb_pitch, max_rows, n_rows, L.d_out, K,
-                 bias, relu, Y, L.h_pitch, out_base, out_rank, out_row};
+                 bias, relu, Y, L.h_pitch, out_base, out_rank, out_row, 0};
     CK(c, launch_tc_gemm(a, c->stream));
   } else {
     if (out_rank) return set_err(c, APT_E_UNSUPPORTED, "routed epilogue needs the tcgen05 path");
@@ -94,6 +94,14 @@ apt_status weight_grad(apt_trainer* t, const Layer& L, const float* G, int64_t g
                        int64_t z_pitch, const int32_t* n_rows, int64_t max_rows, int d_in, float* dW, float* db,
                        int64_t dW_ld) {
   apt_ctx* c = t->ctx;
+  if (z_bf16 && L.Gb && tc_wgrad_supported(L.d_out, d_in)) {
+    // tcgen05: dW = Gb^T Zb with db from Z's all-ones column d_in
+    TcWgradArgs w{L.Gb, L.gb_pitch, static_cast<const uint16_t*>(Z), z_pitch, n_rows, max_rows, L.d_out, d_in,
+                  dW, db};
+    CK(c, launch_tc_wgrad(w, c->stream));
+    c->launches++;
+    return APT_OK;
+  }
   SimtGemmArgs a{};
   a.A = G; a.a_t = kF32; a.sam = 1; a.sak = g_pitch;
   a.B = Z; a.b_t = z_bf16 ? kBF16 : kF32; a.sbk = z_pitch; a.sbn = 1;
@@ -180,7 +188,8 @@ apt_status apt_trainer_create(apt_ctx* c, const apt_graph* g, const apt_fstore* 
       L.d_in = m->dims[l - 1];
       L.d_out = m->dims[l];
       L.zf_pitch = round_up(L.d_in, 4);
-      L.zb_pitch = round_up(L.d_in, 8);
+      L.zb_pitch = round_up(L.d_in + 1, 8);   // + the all-ones bias-gradient column
+      L.gb_pitch = round_up(L.d_out, 8);
       L.h_pitch = round_up(L.d_out, 4);
       L.wb_pitch = round_up(L.d_in, 8);
       L.max_rows = hp.max_dst;
@@ -189,6 +198,7 @@ apt_status apt_trainer_create(apt_ctx* c, const apt_graph* g, const apt_fstore* 
       else L.Zf = A.alloc<float>(L.max_rows * L.zf_pitch, true);
       L.H = A.alloc<float>(L.max_rows * L.h_pitch, true);
       L.G = A.alloc<float>(L.max_rows * L.h_pitch, true);
+      if (m->dtype == APT_BF16) L.Gb = A.alloc<uint16_t>(L.max_rows * L.gb_pitch, true);
       if (l > 1) L.dZ = A.alloc<float>(L.max_rows * L.zf_pitch, true);
       L.W = A.alloc<float>(int64_t(L.d_out) * L.d_in, true);
       L.b = A.alloc<float>(L.d_out, true);
@@ -339,7 +349,7 @@ apt_status layer1_fwd_gdp(apt_trainer* t, RankState& rs, bool time_it) {
   AggArgs a{};
   a.cnt = hp.cnt; a.nbr = hp.nbr; a.k = hp.k;
   a.n_dst = hp.n_dst; a.max_dst = hp.max_dst; a.dim = L.d_in;
-  if (t->m.dtype == APT_BF16) { a.z_bf16 = L.Zb; a.z_bf16_pitch = L.zb_pitch; }
+  if (t->m.dtype == APT_BF16) { a.z_bf16 = L.Zb; a.z_bf16_pitch = L.zb_pitch; a.z_ones = 1; }
   else { a.z_f32 = L.Zf; a.z_f32_pitch = L.zf_pitch; }
   if (time_it) CK(c, record_ev(t, 6));
   CK(c, launch_agg_fstore(a, feat_view(t->f, rs.rank), c->stream));
@@ -359,7 +369,7 @@ apt_status upper_fwd_loss(apt_trainer* t, RankState& rs) {
     AggArgs a{};
     a.indptr = hp.indptr; a.indices = hp.indices; a.x = P.H; a.x_pitch = P.h_pitch;
     a.n_dst = hp.n_dst; a.max_dst = hp.max_dst; a.dim = L.d_in;
-    if (t->m.dtype == APT_BF16) { a.z_bf16 = L.Zb; a.z_bf16_pitch = L.zb_pitch; }
+    if (t->m.dtype == APT_BF16) { a.z_bf16 = L.Zb; a.z_bf16_pitch = L.zb_pitch; a.z_ones = 1; }
     // fp32 Z is kept in both modes for the upper layers' weight gradient in fp32 mode
     if (t->m.dtype != APT_BF16) { a.z_f32 = L.Zf; a.z_f32_pitch = L.zf_pitch; }
     CK(c, launch_agg_csr(a, c->stream));
@@ -371,7 +381,7 @@ apt_status upper_fwd_loss(apt_trainer* t, RankState& rs) {
   Layer& LK = rs.L[t->K - 1];
   CK(c, cudaMemsetAsync(rs.loss, 0, sizeof(float), c->stream));
   CK(c, launch_ce_loss(LK.H, LK.h_pitch, LK.d_out, rs.seeds, rs.small, LK.max_rows, t->labels, rs.small + 1, rs.loss,
-                       LK.G, LK.h_pitch, c->stream));
+                       LK.G, LK.h_pitch, LK.Gb, LK.gb_pitch, c->stream));
   c->launches++;
   return APT_OK;
 }
@@ -387,20 +397,28 @@ apt_status upper_bwd(apt_trainer* t, RankState& rs) {
     apt_status s = weight_grad(t, L, L.G, L.h_pitch, bf ? static_cast<const void*>(L.Zb) : L.Zf, bf,
                                bf ? L.zb_pitch : L.zf_pitch, L.n_rows, L.max_rows, L.d_in, L.dW, L.db, L.d_in);
     if (s != APT_OK) return s;
-    // dZ = G W  (bf16 mode uses the bf16 weights of the forward)
-    SimtGemmArgs a{};
-    a.A = L.G; a.a_t = kF32; a.sam = L.h_pitch; a.sak = 1;
-    if (bf) { a.B = L.Wb; a.b_t = kBF16; a.sbk = L.wb_pitch; }
-    else { a.B = L.W; a.b_t = kF32; a.sbk = L.d_in; }
-    a.sbn = 1;
-    a.C = L.dZ; a.ldc = L.zf_pitch; a.M_dev = L.n_rows; a.M = L.max_rows; a.N = L.d_in; a.K = L.d_out;
-    CK(c, launch_simt_gemm(a, c->stream));
+    // dZ = G W  (bf16 mode: tcgen05 with the bf16 weights of the forward, W read N-major as stored)
+    if (bf && tc_gemm_supported(L.d_in, L.d_out)) {
+      TcGemmArgs g{L.Gb, L.gb_pitch, L.Wb, L.wb_pitch, L.max_rows, L.n_rows, L.d_in, L.d_out, nullptr, 0,
+                   L.dZ, L.zf_pitch, nullptr, nullptr, nullptr, 1};
+      CK(c, launch_tc_gemm(g, c->stream));
+    } else {
+      SimtGemmArgs a{};
+      a.A = L.G; a.a_t = kF32; a.sam = L.h_pitch; a.sak = 1;
+      if (bf) { a.B = L.Wb; a.b_t = kBF16; a.sbk = L.wb_pitch; }
+      else { a.B = L.W; a.b_t = kF32; a.sbk = L.d_in; }
+      a.sbn = 1;
+      a.C = L.dZ; a.ldc = L.zf_pitch; a.M_dev = L.n_rows; a.M = L.max_rows; a.N = L.d_in; a.K = L.d_out;
+      CK(c, launch_simt_gemm(a, c->stream));
+    }
     // dH_{l-1} = scatter(dZ / deg) over the layer-l block, then through the ReLU
     zero_rows_kernel<<<blocks_for(P.max_rows * P.h_pitch / 4), 256, 0, c->stream>>>(P.G, P.h_pitch, P.n_rows);
     CK(c, cudaGetLastError());
     CK(c, launch_agg_bwd(hp.indptr, hp.indices, hp.n_dst, hp.max_dst, L.dZ, L.zf_pitch, L.d_in, P.G, P.h_pitch,
                          c->stream));
-    CK(c, launch_relu_bwd(P.G, P.H, P.h_pitch, P.d_out, P.n_rows, P.max_rows, c->stream));
+    if (bf) CK(c, launch_grad_finish(P.G, P.h_pitch, P.H, P.h_pitch, P.d_out, 1, P.Gb, P.gb_pitch, P.n_rows,
+                                     P.max_rows, c->stream));
+    else CK(c, launch_relu_bwd(P.G, P.H, P.h_pitch, P.d_out, P.n_rows, P.max_rows, c->stream));
     c->launches += 4;
   }
   return APT_OK;

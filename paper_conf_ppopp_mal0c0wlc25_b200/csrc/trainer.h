@@ -31,6 +31,8 @@ struct Layer {
   uint16_t* Zb = nullptr;           // [max_rows x zb_pitch] (bf16 mode)
   float* H = nullptr;               // post-activation (or logits)
   float* G = nullptr;               // dL/dpre
+  uint16_t* Gb = nullptr;           // bf16 copy of G (tcgen05 backward, bf16 mode)
+  int64_t gb_pitch = 0;
   float* dZ = nullptr;              // [max_rows x zf_pitch] scratch (l > 1)
   float* W = nullptr;               // [d_out x d_in] fp32 master
   float* b = nullptr;

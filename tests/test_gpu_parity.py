@@ -253,3 +253,39 @@ def test_step_host_e2e_matches_device_step(A, ctx, tiny):
     gb = torch.as_tensor(perm[2 * cfg.batch:3 * cfg.batch]).pin_memory()
     l_host = tr.step_host(gb, 2, update=False)
     assert l_host == pytest.approx(l_dev, rel=1e-6)
+
+
+# ------------------------------------------------------------------ S11 weight gradient
+@pytest.mark.parametrize("rows,d_out,d_in", [(1, 16, 64), (63, 47, 256), (64, 256, 100), (1000, 256, 256),
+                                             (49537, 256, 100), (5000, 32, 64), (300, 200, 8)])
+@pytest.mark.parametrize("dtype", ["bf16", "f32"])
+def test_weight_grad(A, ctx, rows, d_out, d_in, dtype):
+    """dW = G^T Z, db = colsum(G): tcgen05 (MN-major operands, all-ones bias column) in bf16
+    mode, exact CUDA-core fp32 otherwise; against an fp64 product of the same rounded inputs."""
+    rng = np.random.default_rng(rows + d_out + d_in)
+    G = rng.normal(size=(rows, d_out)).astype(np.float32)
+    Z = rng.normal(size=(rows, d_in))
+    gp = (d_out + 3) // 4 * 4
+    Gd = np.zeros((rows, gp), np.float32)
+    Gd[:, :d_out] = G
+    if dtype == "bf16":
+        Zr = oracle.bf16_round(Z)
+        zp = (d_in + 7) // 8 * 8
+        Zh = np.zeros((rows, zp), np.uint16)
+        Zh[:, :d_in] = (Zr.astype(np.float32).view(np.uint32) >> 16).astype(np.uint16)
+        Zt = torch.as_tensor(Zh.view(np.int16)).cuda()
+        Gr = oracle.bf16_round(G)
+        tol = dict(rtol=1e-4, atol=1e-5 * np.sqrt(rows))
+    else:
+        Zr = Z.astype(np.float32).astype(np.float64)
+        zp = (d_in + 3) // 4 * 4
+        Zf = np.zeros((rows, zp), np.float32)
+        Zf[:, :d_in] = Zr
+        Zt = torch.as_tensor(Zf).cuda()
+        Gr = G.astype(np.float64)
+        tol = dict(rtol=1e-5, atol=1e-5 * np.sqrt(rows))   # fp32 accumulation-order error grows ~ sqrt(rows)
+    dW = torch.zeros((d_out, d_in), dtype=torch.float32, device="cuda")
+    db = torch.zeros(d_out, dtype=torch.float32, device="cuda")
+    ctx.weight_grad(torch.as_tensor(Gd).cuda(), gp, Zt, zp, A.DTYPE[dtype], rows, d_out, d_in, dW, db)
+    assert np.allclose(dW.cpu().numpy(), Gr.T @ Zr, **tol), np.abs(dW.cpu().numpy() - Gr.T @ Zr).max()
+    assert np.allclose(db.cpu().numpy(), Gr.sum(0), **tol)
