@@ -239,38 +239,64 @@ __global__ void __launch_bounds__(THREADS, 1)
       }
     }
   } else {
-    // ---- epilogue warps 2..5: TMEM lane quarter = warp % 4
+    // ---- epilogue warps 2..5: TMEM lane quarter = warp % 4.  Each 32-column chunk
+    // of the warp's 32 rows is staged in shared memory (row stride 33 floats:
+    // conflict-free both ways) and written back row-contiguously: 8 lanes cover
+    // one 128-B row segment, so every store instruction moves 4 full lines
+    // instead of 32 scattered 16-B pieces.
     const int q = warp & 3;
+    float* stg = reinterpret_cast<float*>(tmem_slot + 4) + (warp - 2) * 32 * 33;
+    const int rsub = lane >> 3, cq = (lane & 7) * 4;
     int acc = 0;
     uint32_t aph = 0;
     for (int64_t t = blockIdx.x; t < ntiles; t += gridDim.x) {
       mbar_wait(tfull + acc, aph);
       fence_after();
-      const int64_t m = t * BM + q * 32 + lane;
-      const bool valid = m < M;
-      float* out = nullptr;
-      if (valid) {
-        if (p.out_rank) out = p.out_base[p.out_rank[m]] + int64_t(p.out_row[m]) * p.y_pitch;
-        else out = p.Y + m * p.y_pitch;
+      // own row (= TMEM lane) destination; shuffled to the lanes that store it
+      const int64_t m_own = t * BM + q * 32 + lane;
+      float* own = nullptr;
+      if (m_own < M) {
+        if (p.out_rank) own = p.out_base[p.out_rank[m_own]] + int64_t(p.out_row[m_own]) * p.y_pitch;
+        else own = p.Y + m_own * p.y_pitch;
       }
-      for (int c = 0; c < p.BN; c += 16) {
+      for (int c = 0; c < p.BN; c += 32) {
         uint32_t r[16];
         tmem_ld16(tmem_base + (uint32_t(q * 32) << 16) + uint32_t(acc * p.BN + c), r);
-        if (!valid) continue;
-        float v[16];
 #pragma unroll
-        for (int j = 0; j < 16; ++j) {
-          float x = __uint_as_float(r[j]);
-          if (p.bias && c + j < p.N) x += p.bias[c + j];
-          if (p.relu) x = fmaxf(x, 0.f);
-          v[j] = x;
-        }
-        if (c + 16 <= p.N) {
+        for (int j = 0; j < 16; ++j) stg[lane * 33 + j] = __uint_as_float(r[j]);
+        if (c + 16 < p.BN) {
+          tmem_ld16(tmem_base + (uint32_t(q * 32) << 16) + uint32_t(acc * p.BN + c + 16), r);
 #pragma unroll
-          for (int j = 0; j < 16; j += 4) *reinterpret_cast<float4*>(out + c + j) = make_float4(v[j], v[j + 1], v[j + 2], v[j + 3]);
-        } else {
-          for (int j = 0; j < 16 && c + j < p.N; ++j) out[c + j] = v[j];
+          for (int j = 0; j < 16; ++j) stg[lane * 33 + 16 + j] = __uint_as_float(r[j]);
         }
+        __syncwarp();
+        const int col = c + cq;
+        float4 bv = make_float4(0.f, 0.f, 0.f, 0.f);
+        if (p.bias) {
+          if (col + 4 <= p.N) bv = *reinterpret_cast<const float4*>(p.bias + col);
+          else {
+            if (col < p.N) bv.x = p.bias[col];
+            if (col + 1 < p.N) bv.y = p.bias[col + 1];
+            if (col + 2 < p.N) bv.z = p.bias[col + 2];
+          }
+        }
+#pragma unroll
+        for (int it = 0; it < 8; ++it) {
+          const int row = it * 4 + rsub;
+          float* dst = reinterpret_cast<float*>(__shfl_sync(0xffffffffu, reinterpret_cast<uintptr_t>(own), row));
+          if (!dst || col >= p.N) continue;
+          float4 v = make_float4(stg[row * 33 + cq] + bv.x, stg[row * 33 + cq + 1] + bv.y, stg[row * 33 + cq + 2] + bv.z,
+                                 stg[row * 33 + cq + 3] + bv.w);
+          if (p.relu) { v.x = fmaxf(v.x, 0.f); v.y = fmaxf(v.y, 0.f); v.z = fmaxf(v.z, 0.f); v.w = fmaxf(v.w, 0.f); }
+          if (col + 4 <= p.N) {
+            *reinterpret_cast<float4*>(dst + col) = v;
+          } else {
+            dst[col] = v.x;
+            if (col + 1 < p.N) dst[col + 1] = v.y;
+            if (col + 2 < p.N) dst[col + 2] = v.z;
+          }
+        }
+        __syncwarp();
       }
       fence_before();
       mbar_arrive(tempty + acc);
@@ -375,31 +401,43 @@ __global__ void __launch_bounds__(THREADS, 1)
     if (lane == 0) mma_commit(tfull);
     __syncwarp();
   } else {
-    // ---- epilogue: lane quarter q holds d_out rows m0 + 32q .. +31
+    // ---- epilogue: lane quarter q holds d_out rows m0 + 32q .. +31; 32-column
+    // chunks staged in shared memory, then row-contiguous 16-B vector reductions
     const int q = warp & 3;
+    float* stg = reinterpret_cast<float*>(tmem_slot + 4) + (warp - 2) * 32 * 33;
+    const int rsub = lane >> 3, cq = (lane & 7) * 4;
     mbar_wait(tfull, 0);
     fence_after();
-    const int o = m0 + q * 32 + lane;
-    const bool valid = o < p.d_out;
-    float* wrow = p.dW + int64_t(o) * p.d_in;
     const bool vec = (p.d_in & 3) == 0;
-    for (int c = 0; c < p.BN; c += 16) {
+    for (int c = 0; c < p.BN; c += 32) {
       uint32_t r[16];
       tmem_ld16(tmem_base + (uint32_t(q * 32) << 16) + uint32_t(c), r);
-      if (!valid) continue;
-      if (vec && c + 16 <= p.d_in) {
 #pragma unroll
-        for (int j = 0; j < 16; j += 4)
-          red_add_v4(wrow + c + j, __uint_as_float(r[j]), __uint_as_float(r[j + 1]), __uint_as_float(r[j + 2]),
-                     __uint_as_float(r[j + 3]));
-      } else {
+      for (int j = 0; j < 16; ++j) stg[lane * 33 + j] = __uint_as_float(r[j]);
+      if (c + 16 < p.BN) {
+        tmem_ld16(tmem_base + (uint32_t(q * 32) << 16) + uint32_t(c + 16), r);
 #pragma unroll
-        for (int j = 0; j < 16; ++j) {
-          const int col = c + j;
-          if (col < p.d_in) atomicAdd(wrow + col, __uint_as_float(r[j]));
-          else if (col == p.d_in && p.ones_col && p.db) atomicAdd(p.db + o, __uint_as_float(r[j]));
+        for (int j = 0; j < 16; ++j) stg[lane * 33 + 16 + j] = __uint_as_float(r[j]);
+      }
+      __syncwarp();
+      const int col = c + cq;
+#pragma unroll
+      for (int it = 0; it < 8; ++it) {
+        const int row = it * 4 + rsub;
+        const int o = m0 + q * 32 + row;
+        if (o >= p.d_out || col > p.d_in) continue;
+        const float* sv = stg + row * 33 + cq;
+        float* w = p.dW + int64_t(o) * p.d_in + col;
+        if (vec && col + 4 <= p.d_in) {
+          red_add_v4(w, sv[0], sv[1], sv[2], sv[3]);
+        } else {
+          for (int j = 0; j < 4; ++j) {
+            if (col + j < p.d_in) atomicAdd(w + j, sv[j]);
+            else if (col + j == p.d_in && p.ones_col && p.db) atomicAdd(p.db + o, sv[j]);
+          }
         }
       }
+      __syncwarp();
     }
   }
   fence_before();
@@ -475,7 +513,8 @@ cudaError_t launch_tc_gemm(const TcGemmArgs& a, cudaStream_t st) {
   }
   RowParams p{a.M_max, a.M_dev, a.N, BN, nkb, cols, a.w_mn, b_kb_bytes, a.bias, a.relu, a.Y, a.y_pitch,
               a.out_base, a.out_rank, a.out_row};
-  const size_t smem = 1024 + size_t(STAGES) * A_STAGE_BYTES + size_t(nkb) * b_kb_bytes + 16 * 8 + 16;
+  const size_t smem = 1024 + size_t(STAGES) * A_STAGE_BYTES + size_t(nkb) * b_kb_bytes + 16 * 8 + 16 +
+                      4 * 32 * 33 * 4;   // + epilogue staging
   if (smem > 227 * 1024) return cudaErrorInvalidValue;
   static bool attr_set = false;
   if (!attr_set) {
@@ -506,7 +545,7 @@ cudaError_t launch_tc_wgrad(const TcWgradArgs& a, cudaStream_t st) {
   if (!make_map(&mz, a.Z, zcols, rows, a.z_pitch, 64, BK)) return cudaErrorInvalidValue;
   const uint32_t stage = uint32_t(2 + nbz) * MNBLK;
   WgradParams p{a.rows_dev, a.rows_max, a.d_out, a.d_in, BN, nbz, cols, a.db ? 1 : 0, stage, a.dW, a.db};
-  const size_t smem = 1024 + size_t(WG_STAGES) * stage + 8 * 8 + 16;
+  const size_t smem = 1024 + size_t(WG_STAGES) * stage + 8 * 8 + 16 + 4 * 32 * 33 * 4;
   if (smem > 227 * 1024) return cudaErrorInvalidValue;
   static bool attr_set = false;
   if (!attr_set) {
