@@ -16,22 +16,49 @@ import numpy as np
 from . import aggregate, aggregate_bwd, bf16_round, features
 
 
-def forward(blocks, feat_seed, dim, params, dtype="f32", x0=None):
+def snp_partials(blk, x_src, part, C):
+    """SNP's partial aggregates of layer 1:
+    P~_c[v] = (1/deg_s(v)) * sum over sampled sources u of v with part(u) = c of x_u,
+    one [n_dst x d] array per partition c.  sum_c P~_c = the mean (exact arithmetic)."""
+    deg = np.diff(blk.indptr)
+    rows = np.repeat(np.arange(blk.n_dst), deg)
+    owner = np.asarray(part)[blk.src[blk.indices]]
+    out = []
+    for c in range(C):
+        m = owner == c
+        acc = np.zeros((blk.n_dst, x_src.shape[1]), np.float64)
+        np.add.at(acc, rows[m], x_src[blk.indices[m]])
+        out.append(np.where(deg[:, None] > 0, acc / np.maximum(deg, 1)[:, None], 0.0))
+    return out
+
+
+def forward(blocks, feat_seed, dim, params, dtype="f32", x0=None, snp=None):
     """params: [(W [d_out x d_in], b [d_out])] layer 1 first.  blocks[h], hop 0 at seeds.
+    snp = (part, C): layer 1 is computed as SNP does -- partial aggregates P~_c, each
+    rounded at the bf16 rounding point and projected, summed before bias/ReLU (Z10).
     Returns a dict with per-layer Z, pre, h (fp64) and the logits."""
     K = len(blocks)
     assert len(params) == K
     H = features(feat_seed, blocks[K - 1].src, dim) if x0 is None else np.asarray(x0, np.float64)
-    cache = {"Z": [], "pre": [], "h": [], "W": []}
+    cache = {"Z": [], "pre": [], "h": [], "W": [], "Zparts": None}
     for l in range(1, K + 1):
         blk = blocks[K - l]
         W, b = params[l - 1]
         W = np.asarray(W, np.float64)
-        Z = aggregate(blk.indptr, blk.indices, H)
         if dtype == "bf16":
-            Z = bf16_round(Z)
             W = bf16_round(W)
-        pre = Z @ W.T + np.asarray(b, np.float64)
+        if l == 1 and snp is not None:
+            parts = snp_partials(blk, H, snp[0], snp[1])
+            if dtype == "bf16":
+                parts = [bf16_round(P) for P in parts]
+            cache["Zparts"] = parts
+            Z = sum(parts)
+            pre = sum(P @ W.T for P in parts) + np.asarray(b, np.float64)
+        else:
+            Z = aggregate(blk.indptr, blk.indices, H)
+            if dtype == "bf16":
+                Z = bf16_round(Z)
+            pre = Z @ W.T + np.asarray(b, np.float64)
         H = np.maximum(pre, 0.0) if l < K else pre
         cache["Z"].append(Z)
         cache["pre"].append(pre)
@@ -64,7 +91,10 @@ def backward(blocks, cache, g_logits):
         Z = cache["Z"][l - 1]
         W = cache["W"][l - 1]
         gs[l - 1] = g
-        grads[l - 1] = (g.T @ Z, g.sum(axis=0))
+        if l == 1 and cache.get("Zparts") is not None:
+            grads[l - 1] = (sum(g.T @ P for P in cache["Zparts"]), g.sum(axis=0))
+        else:
+            grads[l - 1] = (g.T @ Z, g.sum(axis=0))
         if l > 1:
             blk = blocks[K - l]
             dZ = g @ W
@@ -73,8 +103,8 @@ def backward(blocks, cache, g_logits):
     return grads, gs
 
 
-def train_step(blocks, feat_seed, dim, params, labels_of_seeds, n_global, dtype="f32", lr=None):
-    cache = forward(blocks, feat_seed, dim, params, dtype)
+def train_step(blocks, feat_seed, dim, params, labels_of_seeds, n_global, dtype="f32", lr=None, snp=None):
+    cache = forward(blocks, feat_seed, dim, params, dtype, snp=snp)
     loss, g = ce_loss_grad(cache["logits"], labels_of_seeds, n_global)
     grads, gs = backward(blocks, cache, g)
     out = {"loss": loss, "cache": cache, "grads": grads, "g": gs}

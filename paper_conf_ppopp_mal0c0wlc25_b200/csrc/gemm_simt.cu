@@ -76,6 +76,7 @@ __global__ void __launch_bounds__(256) simt_gemm_kernel(SimtGemmArgs a) {
   for (int i = 0; i < 4; ++i) {
     const int64_t gm = m0 + tm + i;
     if (gm >= M) continue;
+    float* crow = a.out_rank ? a.out_base[a.out_rank[gm]] + int64_t(a.out_row[gm]) * a.ldc : a.C + gm * a.ldc;
 #pragma unroll
     for (int j = 0; j < 4; ++j) {
       const int gn = n0 + tn + j;
@@ -83,10 +84,10 @@ __global__ void __launch_bounds__(256) simt_gemm_kernel(SimtGemmArgs a) {
       float v = acc[i][j];
       if (a.bias && blockIdx.z == 0) v += a.bias[gn];
       if (a.accumulate) {
-        atomicAdd(a.C + gm * a.ldc + gn, v);
+        atomicAdd(crow + gn, v);
       } else {
         if (a.relu) v = fmaxf(v, 0.f);
-        a.C[gm * a.ldc + gn] = v;
+        crow[gn] = v;
       }
     }
   }

@@ -146,6 +146,7 @@ struct RowParams {
   float* const* out_base;
   const int32_t* out_rank;
   const int32_t* out_row;
+  int accumulate;
 };
 
 __global__ void __launch_bounds__(THREADS, 1)
@@ -288,7 +289,15 @@ __global__ void __launch_bounds__(THREADS, 1)
           float4 v = make_float4(stg[row * 33 + cq] + bv.x, stg[row * 33 + cq + 1] + bv.y, stg[row * 33 + cq + 2] + bv.z,
                                  stg[row * 33 + cq + 3] + bv.w);
           if (p.relu) { v.x = fmaxf(v.x, 0.f); v.y = fmaxf(v.y, 0.f); v.z = fmaxf(v.z, 0.f); v.w = fmaxf(v.w, 0.f); }
-          if (col + 4 <= p.N) {
+          if (p.accumulate) {
+            if (col + 4 <= p.N) {
+              red_add_v4(dst + col, v.x, v.y, v.z, v.w);
+            } else {
+              atomicAdd(dst + col, v.x);
+              if (col + 1 < p.N) atomicAdd(dst + col + 1, v.y);
+              if (col + 2 < p.N) atomicAdd(dst + col + 2, v.z);
+            }
+          } else if (col + 4 <= p.N) {
             *reinterpret_cast<float4*>(dst + col) = v;
           } else {
             dst[col] = v.x;
@@ -321,8 +330,9 @@ struct WgradParams {
   int d_out, d_in, BN, nbz, tmem_cols;
   int ones_col;             // Z column d_in holds 1.0: output column d_in is db
   uint32_t stage_bytes;     // A (2 x 8 KB) + B (nbz x 8 KB)
-  float* dW;                // [d_out x d_in] (accumulated)
+  float* dW;                // [d_out x ldw] (accumulated)
   float* db;                // [d_out] (accumulated) or null
+  int64_t ldw;
 };
 
 __global__ void __launch_bounds__(THREADS, 1)
@@ -408,7 +418,7 @@ __global__ void __launch_bounds__(THREADS, 1)
     const int rsub = lane >> 3, cq = (lane & 7) * 4;
     mbar_wait(tfull, 0);
     fence_after();
-    const bool vec = (p.d_in & 3) == 0;
+    const bool vec = (p.d_in & 3) == 0 && (p.ldw & 3) == 0 && (reinterpret_cast<uintptr_t>(p.dW) & 15) == 0;
     for (int c = 0; c < p.BN; c += 32) {
       uint32_t r[16];
       tmem_ld16(tmem_base + (uint32_t(q * 32) << 16) + uint32_t(c), r);
@@ -427,7 +437,7 @@ __global__ void __launch_bounds__(THREADS, 1)
         const int o = m0 + q * 32 + row;
         if (o >= p.d_out || col > p.d_in) continue;
         const float* sv = stg + row * 33 + cq;
-        float* w = p.dW + int64_t(o) * p.d_in + col;
+        float* w = p.dW + int64_t(o) * p.ldw + col;
         if (vec && col + 4 <= p.d_in) {
           red_add_v4(w, sv[0], sv[1], sv[2], sv[3]);
         } else {
@@ -512,7 +522,7 @@ cudaError_t launch_tc_gemm(const TcGemmArgs& a, cudaStream_t st) {
     b_kb_bytes = uint32_t(BN) * 128;
   }
   RowParams p{a.M_max, a.M_dev, a.N, BN, nkb, cols, a.w_mn, b_kb_bytes, a.bias, a.relu, a.Y, a.y_pitch,
-              a.out_base, a.out_rank, a.out_row};
+              a.out_base, a.out_rank, a.out_row, a.accumulate};
   const size_t smem = 1024 + size_t(STAGES) * A_STAGE_BYTES + size_t(nkb) * b_kb_bytes + 16 * 8 + 16 +
                       4 * 32 * 33 * 4;   // + epilogue staging
   if (smem > 227 * 1024) return cudaErrorInvalidValue;
@@ -544,7 +554,8 @@ cudaError_t launch_tc_wgrad(const TcWgradArgs& a, cudaStream_t st) {
   if (!make_map(&mg, a.G, a.d_out, rows, a.g_pitch, 64, BK)) return cudaErrorInvalidValue;
   if (!make_map(&mz, a.Z, zcols, rows, a.z_pitch, 64, BK)) return cudaErrorInvalidValue;
   const uint32_t stage = uint32_t(2 + nbz) * MNBLK;
-  WgradParams p{a.rows_dev, a.rows_max, a.d_out, a.d_in, BN, nbz, cols, a.db ? 1 : 0, stage, a.dW, a.db};
+  WgradParams p{a.rows_dev, a.rows_max, a.d_out, a.d_in, BN, nbz, cols, a.db ? 1 : 0, stage, a.dW, a.db,
+                a.ldw > 0 ? a.ldw : a.d_in};
   const size_t smem = 1024 + size_t(WG_STAGES) * stage + 8 * 8 + 16 + 4 * 32 * 33 * 4;
   if (smem > 227 * 1024) return cudaErrorInvalidValue;
   static bool attr_set = false;

@@ -128,6 +128,8 @@ struct SimtGemmArgs {
   int accumulate;              // atomically add into C (split-K)
   int64_t k_chunk;             // split-K chunk (0 => whole K)
   const int32_t* K_dev;        // if set, K = *K_dev (<= K)
+  // optional row routing: row m goes to out_base[out_rank[m]] + out_row[m] * ldc
+  float* const* out_base; const int32_t* out_rank; const int32_t* out_row;
 };
 cudaError_t launch_simt_gemm(const SimtGemmArgs& a, cudaStream_t st);
 
@@ -144,6 +146,7 @@ struct TcGemmArgs {
   // out_base[out_rank[m]] + out_row[m] * y_pitch
   float* const* out_base; const int32_t* out_rank; const int32_t* out_row;
   int w_mn;                            // B stored N-contiguous (dZ = G W uses W [d_out x d_in] as is)
+  int accumulate;                      // add into Y with vector reductions (partial sums of SNP / NFP)
 };
 int tc_gemm_supported(int N, int K);
 cudaError_t launch_tc_gemm(const TcGemmArgs& a, cudaStream_t st);
@@ -157,6 +160,7 @@ struct TcWgradArgs {
   const int32_t* rows_dev; int64_t rows_max;
   int d_out, d_in;
   float* dW; float* db;
+  int64_t ldw;                         // row stride of dW (0 => d_in)
 };
 int tc_wgrad_supported(int d_out, int d_in);
 cudaError_t launch_tc_wgrad(const TcWgradArgs& a, cudaStream_t st);

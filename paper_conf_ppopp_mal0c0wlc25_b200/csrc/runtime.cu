@@ -26,6 +26,17 @@ apt_status set_err(apt_ctx* c, apt_status s, const char* fmt, ...) {
   return s;
 }
 
+static void ctx_free(apt_ctx* c) {
+  cudaStreamSynchronize(c->stream);
+  c->arena.release();
+  if (c->own_stream) cudaStreamDestroy(c->stream);
+  delete c;
+}
+void ctx_retain(apt_ctx* c) { if (c) ++c->children; }
+void ctx_release(apt_ctx* c) {
+  if (c && --c->children == 0 && c->zombie) ctx_free(c);
+}
+
 apt_status check_cuda(apt_ctx* c, cudaError_t e, const char* what) {
   if (e == cudaSuccess) return APT_OK;
   if (c) c->broken = true;
@@ -82,10 +93,11 @@ apt_status apt_ctx_create(int rank, int world, int device, void* stream, apt_ctx
 
 apt_status apt_ctx_destroy(apt_ctx* c) {
   if (!c) return APT_OK;
-  cudaStreamSynchronize(c->stream);
-  c->arena.release();
-  if (c->own_stream) cudaStreamDestroy(c->stream);
-  delete c;
+  if (c->children > 0) {
+    c->zombie = true;   // released with its last child
+    return APT_OK;
+  }
+  apt::ctx_free(c);
   return APT_OK;
 }
 
@@ -119,6 +131,7 @@ apt_status apt_graph_load(apt_ctx* c, int64_t n, int64_t nnz, const int64_t* ind
   if (indptr[0] != 0 || indptr[n] != nnz) return set_err(c, APT_E_INVALID, "apt_graph_load: indptr[0]/indptr[n] mismatch");
   auto* g = new apt_graph();
   g->ctx = c;
+  ctx_retain(c);
   g->n = n;
   g->nnz = nnz;
   g->world = c->world;
@@ -127,7 +140,7 @@ apt_status apt_graph_load(apt_ctx* c, int64_t n, int64_t nnz, const int64_t* ind
   g->part = g->arena.alloc<int32_t>(n, false);
   g->lrow = g->arena.alloc<int32_t>(n, false);
   if (!g->indptr || !g->indices || !g->part || !g->lrow) {
-    delete g;
+    apt_graph_destroy(g);
     return set_err(c, APT_E_OOM, "apt_graph_load: out of device memory (n=%lld nnz=%lld)", (long long)n, (long long)nnz);
   }
   g->part_h.resize(n);
@@ -136,7 +149,7 @@ apt_status apt_graph_load(apt_ctx* c, int64_t n, int64_t nnz, const int64_t* ind
   for (int64_t u = 0; u < n; ++u) {
     int p = part ? part[u] : int((u * c->world) / n);
     if (p < 0 || p >= c->world) {
-      delete g;
+      apt_graph_destroy(g);
       return set_err(c, APT_E_INVALID, "apt_graph_load: part[%lld]=%d out of range", (long long)u, p);
     }
     g->part_h[u] = p;
@@ -152,7 +165,10 @@ apt_status apt_graph_load(apt_ctx* c, int64_t n, int64_t nnz, const int64_t* ind
 }
 
 apt_status apt_graph_destroy(apt_graph* g) {
+  if (!g) return APT_OK;
+  apt_ctx* c = g->ctx;
   delete g;
+  ctx_release(c);
   return APT_OK;
 }
 
@@ -163,6 +179,7 @@ apt_status apt_fstore_create(apt_ctx* c, const apt_graph* g, apt_strategy layout
     return set_err(c, APT_E_INVALID, "apt_fstore_create: bad arguments");
   auto* f = new apt_fstore();
   f->ctx = c;
+  ctx_retain(c);
   f->g = g;
   f->layout = layout == APT_AUTO ? APT_GDP : layout;
   f->dtype = dtype == APT_BF16 ? kBF16 : kF32;
@@ -195,7 +212,7 @@ apt_status apt_fstore_create(apt_ctx* c, const apt_graph* g, apt_strategy layout
     if (!c->emulated && r != c->rank) continue;
     f->shard[r] = f->arena.alloc<uint8_t>(f->rows[r] * f->pitch[r] * int64_t(esz), true);
     if (!f->shard[r] || !ids_dev) {
-      delete f;
+      apt_fstore_destroy(f);
       return set_err(c, APT_E_OOM, "apt_fstore_create: out of device memory");
     }
     const int32_t* idp = nullptr;
@@ -235,7 +252,10 @@ apt_status apt_fstore_create(apt_ctx* c, const apt_graph* g, apt_strategy layout
 }
 
 apt_status apt_fstore_destroy(apt_fstore* f) {
+  if (!f) return APT_OK;
+  apt_ctx* c = f->ctx;
   delete f;
+  ctx_release(c);
   return APT_OK;
 }
 
@@ -278,6 +298,7 @@ apt_status apt_sample(apt_ctx* c, const apt_graph* g, const int64_t* seeds_dev, 
     if (fanouts[l] < 1 || fanouts[l] > 256) return set_err(c, APT_E_INVALID, "apt_sample: fanout %d out of [1,256]", fanouts[l]);
   auto* b = new apt_batch();
   b->ctx = c;
+  ctx_retain(c);
   b->K = K;
   const int64_t n_words = ceil_div(g->n, 32);
   uint32_t* dst_bm = b->arena.alloc<uint32_t>(n_words, true);
@@ -289,7 +310,7 @@ apt_status apt_sample(apt_ctx* c, const apt_graph* g, const int64_t* seeds_dev, 
   uint64_t* step_dev = b->arena.alloc<uint64_t>(1, false);
   int32_t* seeds32 = b->arena.alloc<int32_t>(n_seeds, false);
   if (!dst_bm || !new_bm || !pos || !counts || !step_dev || !seeds32) {
-    delete b;
+    apt_batch_destroy(b);
     return set_err(c, APT_E_OOM, "apt_sample: out of device memory");
   }
   // int64 seeds -> int32 (validated on the host copy)
@@ -300,7 +321,7 @@ apt_status apt_sample(apt_ctx* c, const apt_graph* g, const int64_t* seeds_dev, 
     std::vector<int32_t> h32(n_seeds);
     for (int64_t i = 0; i < n_seeds; ++i) {
       if (h[i] < 0 || h[i] >= g->n) {
-        delete b;
+        apt_batch_destroy(b);
         return set_err(c, APT_E_INVALID, "apt_sample: seed %lld out of range", (long long)h[i]);
       }
       h32[i] = int32_t(h[i]);
@@ -323,7 +344,7 @@ apt_status apt_sample(apt_ctx* c, const apt_graph* g, const int64_t* seeds_dev, 
     int32_t* indices = b->arena.alloc<int32_t>(maxF * k, false);
     int32_t* part2 = b->arena.alloc<int32_t>(ceil_div(maxF, 2048) + 4, false);
     if (!cnt || !nbr || !src || !indptr || !indices || !partials || !part2) {
-      delete b;
+      apt_batch_destroy(b);
       return set_err(c, APT_E_OOM, "apt_sample: out of device memory");
     }
     SampleArgs sa{g->indptr, g->indices, dst, n_dst, maxF, k, philox_key(rng_seed, kDomSample), step_dev, h, cnt, nbr};
@@ -367,7 +388,10 @@ apt_status apt_batch_block(const apt_batch* b, int hop, apt_block_view* out) {
 }
 
 apt_status apt_batch_destroy(apt_batch* b) {
+  if (!b) return APT_OK;
+  apt_ctx* c = b->ctx;
   delete b;
+  ctx_release(c);
   return APT_OK;
 }
 

@@ -39,6 +39,11 @@ struct Arena {
   }
 };
 
+// Child objects keep their ctx alive: a ctx destroyed before them is released by
+// the last child (any destruction order is safe, e.g. at interpreter exit).
+void ctx_retain(apt_ctx* c);
+void ctx_release(apt_ctx* c);
+
 }  // namespace apt
 
 struct apt_ctx {
@@ -53,6 +58,8 @@ struct apt_ctx {
   bool broken = false;
   std::string err;
   int64_t launches = 0;
+  int children = 0;      // live graphs / stores / batches / trainers created on this ctx
+  bool zombie = false;   // apt_ctx_destroy called while children were alive
   uint32_t* dev_err = nullptr;   // device error word
   int32_t* scratch = nullptr;    // small device ints for single-op calls
   apt::Arena arena;

@@ -26,6 +26,7 @@ apt_status check_cuda(apt_ctx* c, cudaError_t e, const char* what);
 FeatView feat_view(const apt_fstore* f, int r);
 // strategies.cu
 apt_status strategy_alloc(apt_trainer* t, RankState& rs);
+apt_status strategy_tables(apt_trainer* t);
 apt_status layer1_fwd_strategy(apt_trainer* t);
 apt_status layer1_bwd_strategy(apt_trainer* t);
 }  // namespace apt
@@ -117,6 +118,8 @@ apt_status weight_grad(apt_trainer* t, const Layer& L, const float* G, int64_t g
 
 extern "C" {
 
+apt_status apt_trainer_destroy(apt_trainer* t);
+
 apt_status apt_trainer_create(apt_ctx* c, const apt_graph* g, const apt_fstore* f, const apt_model_desc* m,
                               apt_strategy s, const int32_t* labels, apt_trainer** out) {
   if (!c || !g || !f || !m || !labels || !out || m->n_layers < 1 || m->n_layers > APT_MAX_LAYERS || m->batch < 1 ||
@@ -132,6 +135,7 @@ apt_status apt_trainer_create(apt_ctx* c, const apt_graph* g, const apt_fstore* 
       return set_err(c, APT_E_INVALID, "apt_trainer_create: fanout/dim out of range");
   auto* t = new apt_trainer();
   t->ctx = c;
+  ctx_retain(c);
   t->g = g;
   t->f = f;
   t->m = *m;
@@ -216,13 +220,17 @@ apt_status apt_trainer_create(apt_ctx* c, const apt_graph* g, const apt_fstore* 
       off += L.d_out;
     }
     if (!rs.seeds || !rs.pos || !grads) {
-      delete t;
+      apt_trainer_destroy(t);
       return set_err(c, APT_E_OOM, "apt_trainer_create: out of device memory");
     }
     if (C > 1 && s != APT_GDP) {
       apt_status st = strategy_alloc(t, rs);
-      if (st != APT_OK) { delete t; return st; }
+      if (st != APT_OK) { apt_trainer_destroy(t); return st; }
     }
+  }
+  if (C > 1 && s != APT_GDP) {
+    apt_status st = strategy_tables(t);
+    if (st != APT_OK) { apt_trainer_destroy(t); return st; }
   }
   {
     std::vector<float*> tab(C, nullptr);
@@ -243,7 +251,9 @@ apt_status apt_trainer_destroy(apt_trainer* t) {
   if (t->graph) cudaGraphDestroy(t->graph);
   for (int i = 0; i < 8; ++i)
     if (t->ev[i]) cudaEventDestroy(t->ev[i]);
+  apt_ctx* c = t->ctx;
   delete t;
+  ctx_release(c);
   return APT_OK;
 }
 
@@ -256,6 +266,15 @@ apt_status apt_trainer_set_params(apt_trainer* t, int layer, const float* W, con
     CK(c, cudaMemcpyAsync(L.b, b, sizeof(float) * L.d_out, cudaMemcpyHostToDevice, c->stream));
     CK(c, launch_to_bf16(L.W, L.d_in, L.Wb, L.wb_pitch, L.d_in, nullptr, L.d_out, c->stream));
     c->launches++;
+    if (layer == 1 && rs.x.W1s) {   // NFP: the rank's column slice of W^1 (column-owned)
+      const int w = rs.x.w_cols;
+      if (w > 0) {
+        CK(c, cudaMemcpy2DAsync(rs.x.W1s, sizeof(float) * w, W + rs.x.col_lo, sizeof(float) * L.d_in, sizeof(float) * w,
+                                L.d_out, cudaMemcpyHostToDevice, c->stream));
+        CK(c, launch_to_bf16(rs.x.W1s, w, rs.x.Wb1s, rs.x.ws_pitch, w, nullptr, L.d_out, c->stream));
+        c->launches++;
+      }
+    }
   }
   CK(c, cudaStreamSynchronize(c->stream));
   return APT_OK;
@@ -268,6 +287,13 @@ apt_status apt_trainer_get_params(apt_trainer* t, int rank, int layer, float* W,
       Layer& L = rs.L[layer - 1];
       CK(t->ctx, cudaStreamSynchronize(t->ctx->stream));
       if (W) CK(t->ctx, cudaMemcpy(W, L.W, sizeof(float) * L.d_out * L.d_in, cudaMemcpyDeviceToHost));
+      if (W && layer == 1 && rs.x.W1s) {   // NFP: W^1 is column-owned; assemble the hosted slices
+        for (auto& o : t->R) {
+          if (o.x.w_cols <= 0) continue;
+          CK(t->ctx, cudaMemcpy2D(W + o.x.col_lo, sizeof(float) * L.d_in, o.x.W1s, sizeof(float) * o.x.w_cols,
+                                  sizeof(float) * o.x.w_cols, L.d_out, cudaMemcpyDeviceToHost));
+        }
+      }
       if (b) CK(t->ctx, cudaMemcpy(b, L.b, sizeof(float) * L.d_out, cudaMemcpyDeviceToHost));
       return APT_OK;
     }
@@ -443,7 +469,18 @@ apt_status allreduce_sgd(apt_trainer* t, int update) {
   }
   if (!update) return APT_OK;
   for (auto& rs : t->R) {
+    if (rs.x.W1s && rs.x.w_cols > 0) {   // NFP: each rank updates only its column slice of W^1
+      const Layer& L = rs.L[0];
+      CK(c, launch_sgd(rs.x.W1s, rs.x.dW1s, int64_t(L.d_out) * rs.x.w_cols, t->m.lr, rs.x.Wb1s, L.d_out, rs.x.w_cols,
+                       rs.x.ws_pitch, c->stream));
+      c->launches++;
+    }
     for (auto& L : rs.L) {
+      if (&L == &rs.L[0] && rs.x.W1s) {
+        CK(c, launch_sgd(L.b, L.db, L.d_out, t->m.lr, nullptr, 1, L.d_out, 0, c->stream));
+        c->launches++;
+        continue;
+      }
       CK(c, launch_sgd(L.W, L.dW, int64_t(L.d_out) * L.d_in, t->m.lr, L.Wb, L.d_out, L.d_in, L.wb_pitch, c->stream));
       CK(c, launch_sgd(L.b, L.db, L.d_out, t->m.lr, nullptr, 1, L.d_out, 0, c->stream));
       c->launches += 2;
@@ -675,7 +712,22 @@ apt_status apt_trainer_read(apt_trainer* t, int rank, int what, int layer, void*
       return copy_rows(L.Zf, nr, L.d_in, L.zf_pitch, 4, false);
     }
     case 3: { const Layer& L = rs->L[layer - 1]; return copy_rows(L.H, count(L.n_rows), L.d_out, L.h_pitch, 4, false); }
-    case 4: { const Layer& L = rs->L[layer - 1]; return copy_rows(L.dW, L.d_out, L.d_in, L.d_in, 4, false); }
+    case 4: {
+      const Layer& L = rs->L[layer - 1];
+      if (layer == 1 && rs->x.dW1s) {   // NFP: concatenate the column-owned slices of the hosted ranks
+        *rows = L.d_out;
+        *cols = L.d_in;
+        std::vector<float> full(size_t(L.d_out) * L.d_in, 0.f);
+        for (auto& o : t->R) {
+          if (o.x.w_cols <= 0) continue;
+          CK(c, cudaMemcpy2D(full.data() + o.x.col_lo, sizeof(float) * L.d_in, o.x.dW1s, sizeof(float) * o.x.w_cols,
+                             sizeof(float) * o.x.w_cols, L.d_out, cudaMemcpyDeviceToHost));
+        }
+        memcpy(host, full.data(), sizeof(float) * std::min<int64_t>(cap, int64_t(full.size())));
+        return APT_OK;
+      }
+      return copy_rows(L.dW, L.d_out, L.d_in, L.d_in, 4, false);
+    }
     case 5: { const Layer& L = rs->L[layer - 1]; return copy_rows(L.db, 1, L.d_out, L.d_out, 4, false); }
     case 6: { const Layer& L = rs->L[layer - 1]; return copy_rows(L.G, count(L.n_rows), L.d_out, L.h_pitch, 4, false); }
     default: return set_err(c, APT_E_INVALID, "read: unknown item %d", what);

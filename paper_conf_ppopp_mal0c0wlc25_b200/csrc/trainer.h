@@ -41,28 +41,29 @@ struct Layer {
   float* db = nullptr;
 };
 
-// NFP / SNP / DNP exchange state of one rank (trainer_strategies.cu).
+// NFP / SNP / DNP state of one rank (strategies.cu).  The rank is both a
+// requester (its own layer-1 rows, whose h^1 it needs) and an owner (work items
+// other ranks -- and itself -- send it: Permute/Shuffle).
 struct Xchg {
-  // generic receive slots written by peers: slot[s] holds what rank s sent
-  int32_t* req_cnt = nullptr;        // [C] rows received from each sender (device)
-  int32_t* req_row = nullptr;        // [C x cap] requester row / tag
-  int32_t* req_gid = nullptr;        // [C x cap] node id (DNP) or group deg (SNP)
-  int32_t* req_indptr = nullptr;     // [C x (cap+1)] (SNP edge groups)
-  int32_t* req_src = nullptr;        // [C x ecap] source gids (SNP)
-  int32_t* ecnt = nullptr;           // [C] edges received from each sender
-  int64_t cap = 0, ecap = 0;
-  // owner-side work list (DNP) / contributor work (SNP)
-  int32_t* work_rank = nullptr;      // [wcap] requester rank of every work row
-  int32_t* work_row = nullptr;       // [wcap] requester row
-  int32_t* work_gid = nullptr;       // [wcap] node id
-  int32_t* n_work = nullptr;         // device count
-  int64_t wcap = 0;
-  int32_t* wcnt = nullptr;           // [wcap] re-sampled ELL (DNP)
+  int64_t wcap = 0;                  // work-item capacity (sum of all requesters' layer-1 rows)
+  int32_t* n_work = nullptr;         // [1] device count of items owned
+  int32_t* work_rank = nullptr;      // [wcap] requester rank
+  int32_t* work_row = nullptr;       // [wcap] requester layer-1 row
+  int32_t* work_gid = nullptr;       // [wcap] destination node id
+  int32_t* wcnt = nullptr;           // [wcap] re-sampled ELL count (same Philox key: identical sample)
   int32_t* wnbr = nullptr;           // [wcap * k]
-  uint16_t* wZb = nullptr;           // [wcap x zb_pitch]
-  float* wZf = nullptr;              // [wcap x zf_pitch]
-  float* wG = nullptr;               // [wcap x h_pitch] gathered gradients (bwd)
-  float* partial = nullptr;          // [C x cap x h_pitch] partial sums received (SNP/NFP)
+  int w_cols = 0;                    // aggregated columns: d, or the NFP column slice width
+  int64_t wzb_pitch = 0, wzf_pitch = 0;
+  uint16_t* wZb = nullptr;           // [wcap x wzb_pitch] bf16 (full mean or SNP partial)
+  float* wZf = nullptr;              // [wcap x wzf_pitch] fp32 mode
+  uint16_t* wGb = nullptr;           // [wcap x gb_pitch] gathered dL/dpre (bf16 mode)
+  float* wGf = nullptr;              // [wcap x h_pitch] (fp32 mode)
+  // NFP: the rank's column slice [col_lo, col_hi) of W^1 (column-owned, no all-reduce)
+  int col_lo = 0, col_hi = 0;
+  int64_t ws_pitch = 0;
+  float* W1s = nullptr;              // [d_out x w_cols]
+  uint16_t* Wb1s = nullptr;          // [d_out x ws_pitch]
+  float* dW1s = nullptr;             // [d_out x w_cols]
 };
 
 struct RankState {
@@ -93,8 +94,15 @@ struct apt_trainer {
   int64_t n_train = 0, steps_per_epoch = 1;
   uint64_t* step_dev = nullptr;
   std::vector<apt::RankState> R;
-  // device pointer tables for cross-rank kernels
+  // device pointer tables for cross-rank kernels (peer pointers in a multi-GPU job)
   float** dW_tab = nullptr;
+  float** H1_tab = nullptr;          // requesters' layer-1 outputs
+  float** G1_tab = nullptr;          // requesters' layer-1 dL/dpre (fp32)
+  uint16_t** Gb1_tab = nullptr;      // ... bf16
+  int32_t** wn_tab = nullptr;        // owners' work counters / lists
+  int32_t** wrank_tab = nullptr;
+  int32_t** wrow_tab = nullptr;
+  int32_t** wgid_tab = nullptr;
   bool use_graph = false;
   bool capturing = false;
   cudaGraphExec_t gexec = nullptr;

@@ -289,3 +289,56 @@ def test_weight_grad(A, ctx, rows, d_out, d_in, dtype):
     ctx.weight_grad(torch.as_tensor(Gd).cuda(), gp, Zt, zp, A.DTYPE[dtype], rows, d_out, d_in, dW, db)
     assert np.allclose(dW.cpu().numpy(), Gr.T @ Zr, **tol), np.abs(dW.cpu().numpy() - Gr.T @ Zr).max()
     assert np.allclose(db.cpu().numpy(), Gr.sum(0), **tol)
+
+
+# ------------------------------------------------------------------ strategies (C ranks emulated on one B200)
+def _strategy_ref(cfg, g, train, labels, params, strategy, C, step, dtype):
+    """Oracle: every rank's own blocks through the fp64 model, loss over the global batch (Z20);
+    the strategies must reproduce it (P:59, P:279 'semantically equivalent')."""
+    from oracle import strategy as S
+    perm = oracle.epoch_perm(train, cfg.sample_seed, 0)
+    gb = oracle.global_batch(perm, step, C, cfg.batch)
+    part = aptgen.partition(g.n, C)
+    seeds = S.assign_seeds(strategy, gb, part, C, cfg.batch)
+    p64 = [(W.astype(np.float64), b.astype(np.float64)) for W, b in params]
+    refs = []
+    for r in range(C):
+        blocks = oracle.sample_blocks(g, seeds[r], cfg.fanouts, cfg.sample_seed, step)
+        snp = (part, C) if strategy == "SNP" else None     # SNP's own rounding points (partials)
+        refs.append(model.train_step(blocks, cfg.feat_seed, cfg.dim, p64, labels[seeds[r]], len(gb), dtype, snp=snp))
+    return seeds, refs
+
+
+@pytest.mark.parametrize("dtype", ["f32", "bf16"])
+@pytest.mark.parametrize("C", [2, 4])
+@pytest.mark.parametrize("strategy", ["GDP", "NFP", "SNP", "DNP"])
+def test_strategy_step_matches_oracle(A, tiny, strategy, C, dtype):
+    cfg, g, train = tiny
+    ctx = A.Ctx(-1, C, 0)                      # all C ranks on this device
+    gr = ctx.graph_load(g.indptr, g.indices, aptgen.partition(g.n, C))
+    dt = A.DTYPE[dtype]
+    fs = ctx.fstore_create(gr, A.NFP if strategy == "NFP" else A.GDP, dt, cfg.dim, None, cfg.feat_seed)
+    dims = [cfg.dim] + [d for _, d in cfg.dims()]
+    labels = aptgen.labels(cfg, g.n)
+    tr = A.Trainer(ctx, gr, fs, dims, cfg.fanouts, cfg.batch, dt, 0.1, cfg.sample_seed, cfg.feat_seed,
+                   A.STRATEGY[strategy], labels)
+    params = aptgen.weights(cfg)
+    tr.set_params(params)
+    tr.set_epoch(train, 0)
+    tr.step(0, update=False)
+    seeds, refs = _strategy_ref(cfg, g, train, labels, params, strategy, C, 0, dtype)
+    tol = TOL[dtype]
+    K = len(cfg.fanouts)
+    for r in range(C):
+        assert np.array_equal(tr.read("seeds", rank=r)[:, 0], seeds[r])
+        assert np.allclose(tr.read("H", 1, rank=r), refs[r]["cache"]["h"][0], **tol), f"h1 rank {r}"
+        assert np.allclose(tr.read("H", K, rank=r), refs[r]["cache"]["h"][K - 1], **tol), f"logits rank {r}"
+    loss = tr.loss()
+    ref_loss = sum(x["loss"] for x in refs)
+    assert abs(loss - ref_loss) <= tol["rtol"] * abs(ref_loss) + tol["atol"]
+    for l in range(1, K + 1):
+        dW = sum(x["grads"][l - 1][0] for x in refs)
+        db = sum(x["grads"][l - 1][1] for x in refs)
+        for r in (0, C - 1):
+            assert np.allclose(tr.read("dW", l, rank=r), dW, **tol), f"dW layer {l} rank {r}"
+            assert np.allclose(tr.read("db", l, rank=r)[0], db, **tol), f"db layer {l} rank {r}"

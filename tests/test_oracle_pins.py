@@ -247,3 +247,20 @@ def test_epoch_perm_is_permutation_and_epoch_dependent():
     # positions are uniform-ish: mean rank of the first half of train ~ n/2
     rank = np.empty(len(train)); rank[np.searchsorted(train, p0)] = np.arange(len(train))
     assert abs(rank[: len(train) // 2].mean() / len(train) - 0.5) < 0.05
+
+
+def test_snp_partials_sum_to_mean_and_split_by_partition(tiny_graph, tiny_cfg):
+    """SNP partial aggregates: sum over partitions = the full mean (linearity),
+    and P~_c only draws on sources owned by c."""
+    from oracle import model
+    seeds = aptgen.train_nodes(tiny_graph, tiny_cfg)[:64]
+    blk = oracle.sample_blocks(tiny_graph, seeds, (6,), 9, 1)[0]
+    x = oracle.features(tiny_cfg.feat_seed, blk.src, 16)
+    part = aptgen.partition(tiny_graph.n, 4)
+    parts = model.snp_partials(blk, x, part, 4)
+    assert np.allclose(sum(parts), oracle.aggregate(blk.indptr, blk.indices, x), rtol=0, atol=1e-12)
+    # zeroing the features of partition 1 leaves every other partial unchanged
+    x2 = x.copy()
+    x2[part[blk.src] == 1] = 0.0
+    p2 = model.snp_partials(blk, x2, part, 4)
+    assert np.array_equal(p2[0], parts[0]) and np.array_equal(p2[2], parts[2]) and not p2[1].any()
