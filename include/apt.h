@@ -238,6 +238,12 @@ apt_status apt_profile_links(apt_ctx* ctx, apt_bw_profile* out);
 apt_status apt_select_strategy(const apt_plan_stats* st, const apt_bw_profile* bw, apt_strategy* pick,
                                double pred_s[4]);
 
+/* Self-test of the mean's division (reading O5): the number of operands for which
+ * the reciprocal-based correctly-rounded division differs bitwise from IEEE
+ * x / d over every O4 mean (x = m/64, |m| <= 2^17, d = 1..256) and random normal
+ * numerators; 0 expected, < 0 on a CUDA failure.  Uses the current device.      */
+int64_t apt_selftest_div(void);
+
 #ifdef __cplusplus
 }
 #endif

@@ -93,6 +93,8 @@ def lib():
         L.apt_last_error.restype = C.c_char_p
         L.apt_ctx_launches.argtypes = [vp]
         L.apt_ctx_launches.restype = C.c_int64
+        L.apt_selftest_div.argtypes = []
+        L.apt_selftest_div.restype = C.c_int64
         L.apt_trainer_steps_per_epoch.argtypes = [vp]
         L.apt_trainer_steps_per_epoch.restype = C.c_int64
         _lib = L

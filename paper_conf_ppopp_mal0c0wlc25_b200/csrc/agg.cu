@@ -30,100 +30,100 @@ __device__ __forceinline__ void accumulate_vec(float* acc, uint4 raw) {
   }
 }
 
-struct EllFstoreSrc {
+// Edge sources.  row_ptr(u) is the 16-B aligned start of source u's stored row.
+struct EllFstoreSrc {            // layer 1: sampler ELL + the feature store (local / peer shards)
   const int32_t* cnt; const int32_t* nbr; int k;
-  FeatView fv;
-  __device__ int64_t begin(int64_t i) const { return i * k; }
-  __device__ int64_t end(int64_t i) const { return i * k + cnt[i]; }
-  __device__ int node(int64_t e) const { return nbr[e]; }
-  __device__ const char* row(int u) const {
-    if (fv.part) {
-      const int o = fv.part[u];
-      return reinterpret_cast<const char*>(fv.base[o]) + int64_t(fv.lrow[u]) * fv.pitch * (fv.dtype == kBF16 ? 2 : 4);
-    }
-    return reinterpret_cast<const char*>(fv.base[0]) + int64_t(u) * fv.pitch * (fv.dtype == kBF16 ? 2 : 4);
+  FeatView fv; int64_t row_bytes;
+  __device__ __forceinline__ int64_t begin(int64_t i) const { return i * k; }
+  __device__ __forceinline__ int count(int64_t i) const { return cnt[i]; }
+  // ids can be read before the count arrives: the ELL row has k slots
+  __device__ __forceinline__ int cap(int c) const { return k; }
+  __device__ __forceinline__ int node(int64_t e) const { return nbr[e]; }
+  __device__ __forceinline__ const char* row_ptr(int u) const {
+    if (fv.part) return reinterpret_cast<const char*>(fv.base[fv.part[u]]) + int64_t(fv.lrow[u]) * row_bytes;
+    return reinterpret_cast<const char*>(fv.base[0]) + int64_t(u) * row_bytes;
   }
 };
 
-struct CsrSrc {
-  const int32_t* indptr; const int32_t* indices; const float* x; int64_t pitch;
-  __device__ int64_t begin(int64_t i) const { return indptr[i]; }
-  __device__ int64_t end(int64_t i) const { return indptr[i + 1]; }
-  __device__ int node(int64_t e) const { return indices[e]; }
-  __device__ const char* row(int u) const { return reinterpret_cast<const char*>(x + int64_t(u) * pitch); }
+struct CsrSrc {                  // upper layers: block CSR over the previous layer's rows
+  const int32_t* indptr; const int32_t* indices; const float* x; int64_t row_bytes;
+  __device__ __forceinline__ int64_t begin(int64_t i) const { return indptr[i]; }
+  __device__ __forceinline__ int count(int64_t i) const { return indptr[i + 1] - indptr[i]; }
+  __device__ __forceinline__ int cap(int c) const { return c; }
+  __device__ __forceinline__ int node(int64_t e) const { return indices[e]; }
+  __device__ __forceinline__ const char* row_ptr(int u) const {
+    return reinterpret_cast<const char*>(x) + int64_t(u) * row_bytes;
+  }
 };
 
-// EPV: elements per 16-B vector (8 = bf16 input, 4 = fp32 input); VPL: vectors per lane.
-template <int EPV, int VPL, class Src>
+// Segmented mean with the gather fused in (S6+S7).  A row of V 16-byte vectors
+// is owned by a lane group of LG lanes (LG = 16: two destination rows per warp
+// when V <= 16; LG = 32 otherwise, VPL = ceil(V/32) vectors per lane).  Per chunk
+// of LG edges, every lane resolves ONE edge's row pointer (and, for SNP, its
+// partition filter) with coalesced loads; the pointers are then broadcast by
+// shuffles and each lane streams its vector of 4 edges at a time (4 independent
+// 16-B loads in flight per lane, no dependent index load on the critical path).
+// Sum in fp32 (exact under O4), IEEE RN division by the sampled degree (O5).
+template <int EPV, int VPL, int LG, class Src>
 __global__ void __launch_bounds__(256) agg_kernel(AggArgs a, Src src) {
   const int lane = lane_id();
+  const int sub = LG == 16 ? (lane >> 4) : 0;
+  const int l = LG == 16 ? (lane & 15) : lane;
+  constexpr int RPW = 32 / LG;                                 // destination rows per warp
   const int64_t n_dst = *a.n_dst;
   const int V = int(ceil_div(a.dim, EPV));
-  const int G = (VPL == 1 && V <= 16) ? (32 / V) : 1;      // lane groups (edges in flight)
-  const int g = (VPL == 1) ? lane / V : 0;
-  const int jv = (VPL == 1) ? lane - g * V : lane;          // first vector of this lane
-  const bool active = (VPL == 1) ? (g < G) : true;
   const int64_t nwarps = int64_t(gridDim.x) * (blockDim.x >> 5);
-  for (int64_t i = (int64_t(blockIdx.x) * blockDim.x + threadIdx.x) >> 5; i < n_dst; i += nwarps) {
+  for (int64_t w = (int64_t(blockIdx.x) * blockDim.x + threadIdx.x) >> 5; w * RPW < n_dst; w += nwarps) {
+    const int64_t i = w * RPW + sub;
+    const bool valid = i < n_dst;
+    const int cnt = valid ? src.count(i) : 0;
+    const int64_t e_base = valid ? src.begin(i) : 0;
+    int cmax = cnt;
+    if (LG == 16) cmax = max(cmax, __shfl_xor_sync(0xffffffffu, cmax, 16));
     float acc[VPL][EPV];
 #pragma unroll
     for (int p = 0; p < VPL; ++p)
 #pragma unroll
       for (int q = 0; q < EPV; ++q) acc[p][q] = 0.f;
-    const int64_t e0 = src.begin(i), e1 = src.end(i);
-    int deg = int(e1 - e0);
-    if (a.deg_override) deg = a.deg_override[i];
-    if (active) {
-      int64_t e = e0 + g;
-      // two edges per group per iteration: 2*G*V independent 16-B loads per warp
-      for (; e + G < e1; e += 2 * G) {
-        const int u0 = src.node(e), u1 = src.node(e + G);
-        const bool k0 = !a.filt_part || a.filt_part[u0] == a.keep_part;
-        const bool k1 = !a.filt_part || a.filt_part[u1] == a.keep_part;
-        const char* r0 = src.row(u0);
-        const char* r1 = src.row(u1);
-        uint4 v0[VPL], v1[VPL];
+    constexpr int NB = 4;                                      // 16-B loads in flight per lane (8: more registers, slower)
+    for (int e0 = 0; e0 < cmax; e0 += LG) {
+      // resolve one edge per lane (ELL: the id load does not wait for the count)
+      int u = -1;
+      if (valid && e0 + l < src.cap(cnt)) u = src.node(e_base + e0 + l);
+      const char* rp = nullptr;
+      if (e0 + l < cnt && (!a.filt_part || a.filt_part[u] == a.keep_part)) rp = src.row_ptr(u);
+      const int m = min(LG, cmax - e0);
+      for (int j = 0; j < m; j += NB) {
+        uint4 v[NB][VPL];
 #pragma unroll
-        for (int p = 0; p < VPL; ++p) {
-          const int j = jv + p * 32;
-          v0[p] = (k0 && j < V) ? ld_nc_v4(r0 + int64_t(j) * 16) : make_uint4(0, 0, 0, 0);
-          v1[p] = (k1 && j < V) ? ld_nc_v4(r1 + int64_t(j) * 16) : make_uint4(0, 0, 0, 0);
-        }
-#pragma unroll
-        for (int p = 0; p < VPL; ++p) { accumulate_vec<EPV>(acc[p], v0[p]); accumulate_vec<EPV>(acc[p], v1[p]); }
-      }
-      if (e < e1) {
-        const int u0 = src.node(e);
-        if (!a.filt_part || a.filt_part[u0] == a.keep_part) {
-          const char* r0 = src.row(u0);
+        for (int q = 0; q < NB; ++q) {
+          const char* r = reinterpret_cast<const char*>(
+              __shfl_sync(0xffffffffu, reinterpret_cast<uintptr_t>(rp), sub * LG + ((j + q) & (LG - 1))));
+          const bool on = (j + q < m) && r != nullptr;
 #pragma unroll
           for (int p = 0; p < VPL; ++p) {
-            const int j = jv + p * 32;
-            if (j < V) accumulate_vec<EPV>(acc[p], ld_nc_v4(r0 + int64_t(j) * 16));
+            const int jv = l + p * LG;
+            v[q][p] = (on && jv < V) ? ld_nc_v4(r + int64_t(jv) * 16) : make_uint4(0, 0, 0, 0);
           }
         }
-      }
-    }
-    if (VPL == 1) {   // fold the G lane groups into group 0 (fixed order: deterministic)
-      for (int s = 1; s < G; ++s) {
 #pragma unroll
-        for (int q = 0; q < EPV; ++q) {
-          const float o = __shfl_sync(0xffffffffu, acc[0][q], (lane + s * V) & 31);
-          if (g == 0 && lane + s * V < 32) acc[0][q] += o;
-        }
+        for (int q = 0; q < NB; ++q)
+#pragma unroll
+          for (int p = 0; p < VPL; ++p) accumulate_vec<EPV>(acc[p], v[q][p]);
       }
     }
-    if (g != 0 || !active) continue;
-    if (a.z_ones && lane == 0) a.z_bf16[i * a.z_bf16_pitch + a.dim] = 0x3F80;   // bf16 1.0: bias-gradient column
-    const float fdeg = float(deg);
+    if (!valid) continue;
+    if (a.z_ones && l == 0) a.z_bf16[i * a.z_bf16_pitch + a.dim] = 0x3F80;   // bf16 1.0: bias-gradient column
+    const float fdeg = float(a.deg_override ? a.deg_override[i] : cnt);
+    const float rdeg = fdeg > 0.f ? __frcp_rn(fdeg) : 0.f;   // one reciprocal per row (O5 division below)
 #pragma unroll
     for (int p = 0; p < VPL; ++p) {
-      const int j = jv + p * 32;
-      if (j >= V) continue;
+      const int jv = l + p * LG;
+      if (jv >= V) continue;
       float z[EPV];
 #pragma unroll
-      for (int q = 0; q < EPV; ++q) z[q] = deg > 0 ? __fdiv_rn(acc[p][q], fdeg) : 0.f;
-      const int c0 = j * EPV;
+      for (int q = 0; q < EPV; ++q) z[q] = fdeg > 0.f ? div_rn_rcp(acc[p][q], fdeg, rdeg) : 0.f;
+      const int c0 = jv * EPV;
       const bool full = c0 + EPV <= a.dim;
       if (a.z_f32) {
         float* o = a.z_f32 + i * a.z_f32_pitch + c0;
@@ -131,7 +131,9 @@ __global__ void __launch_bounds__(256) agg_kernel(AggArgs a, Src src) {
 #pragma unroll
           for (int q = 0; q < EPV; q += 4) *reinterpret_cast<float4*>(o + q) = make_float4(z[q], z[q + 1], z[q + 2], z[q + 3]);
         } else {
-          for (int q = 0; q < EPV && c0 + q < a.dim; ++q) o[q] = z[q];
+#pragma unroll
+          for (int q = 0; q < EPV; ++q)
+            if (c0 + q < a.dim) o[q] = z[q];
         }
       }
       if (a.z_bf16) {
@@ -144,9 +146,12 @@ __global__ void __launch_bounds__(256) agg_kernel(AggArgs a, Src src) {
             *reinterpret_cast<uint2*>(o) = make_uint2(pack_bf16x2(z[0], z[1]), pack_bf16x2(z[2], z[3]));
           }
         } else {
-          for (int q = 0; q < EPV && c0 + q < a.dim; ++q) {
-            __nv_bfloat16 h = __float2bfloat16_rn(z[q]);
-            o[q] = *reinterpret_cast<uint16_t*>(&h);
+#pragma unroll
+          for (int q = 0; q < EPV; ++q) {
+            if (c0 + q < a.dim) {
+              __nv_bfloat16 h = __float2bfloat16_rn(z[q]);
+              o[q] = *reinterpret_cast<uint16_t*>(&h);
+            }
           }
         }
       }
@@ -158,24 +163,26 @@ template <int EPV, class Src>
 static cudaError_t dispatch_agg(const AggArgs& a, const Src& s, cudaStream_t st) {
   const int V = int(ceil_div(a.dim, EPV));
   const int threads = 256;
-  int64_t blocks = ceil_div(a.max_dst * 32, threads);
+  const int rpw = V <= 16 ? 2 : 1;
+  int64_t blocks = ceil_div(ceil_div(a.max_dst, rpw) * 32, threads);
   blocks = std::max<int64_t>(1, std::min<int64_t>(blocks, 148 * 16));
-  if (V <= 32) agg_kernel<EPV, 1, Src><<<blocks, threads, 0, st>>>(a, s);
-  else if (V <= 64) agg_kernel<EPV, 2, Src><<<blocks, threads, 0, st>>>(a, s);
-  else if (V <= 128) agg_kernel<EPV, 4, Src><<<blocks, threads, 0, st>>>(a, s);
+  if (V <= 16) agg_kernel<EPV, 1, 16, Src><<<blocks, threads, 0, st>>>(a, s);
+  else if (V <= 32) agg_kernel<EPV, 1, 32, Src><<<blocks, threads, 0, st>>>(a, s);
+  else if (V <= 64) agg_kernel<EPV, 2, 32, Src><<<blocks, threads, 0, st>>>(a, s);
+  else if (V <= 128) agg_kernel<EPV, 4, 32, Src><<<blocks, threads, 0, st>>>(a, s);
   else return cudaErrorInvalidValue;
   return cudaGetLastError();
 }
 
 cudaError_t launch_agg_fstore(const AggArgs& a, const FeatView& fv, cudaStream_t st) {
-  EllFstoreSrc s{a.cnt, a.nbr, a.k, fv};
+  EllFstoreSrc s{a.cnt, a.nbr, a.k, fv, fv.pitch * (fv.dtype == kBF16 ? 2 : 4)};
   AggArgs b = a;
   b.dim = fv.dim;
   return fv.dtype == kBF16 ? dispatch_agg<8>(b, s, st) : dispatch_agg<4>(b, s, st);
 }
 
 cudaError_t launch_agg_csr(const AggArgs& a, cudaStream_t st) {
-  CsrSrc s{a.indptr, a.indices, a.x, a.x_pitch};
+  CsrSrc s{a.indptr, a.indices, a.x, a.x_pitch * 4};
   return dispatch_agg<4>(a, s, st);
 }
 
@@ -197,7 +204,7 @@ __global__ void __launch_bounds__(256) agg_bwd_kernel(const int32_t* __restrict_
     const float fdeg = float(e1 - e0);
     for (int j = lane; j < V; j += 32) {
       const float4 g = *reinterpret_cast<const float4*>(dz + i * dz_pitch + j * 4);
-      const float a = __fdiv_rn(g.x, fdeg), b = __fdiv_rn(g.y, fdeg), c = __fdiv_rn(g.z, fdeg), d = __fdiv_rn(g.w, fdeg);
+      const float a = div_rn(g.x, fdeg), b = div_rn(g.y, fdeg), c = div_rn(g.z, fdeg), d = div_rn(g.w, fdeg);
       for (int e = e0; e < e1; ++e) red_add_v4(dx + int64_t(indices[e]) * dx_pitch + j * 4, a, b, c, d);
     }
   }
@@ -261,3 +268,40 @@ cudaError_t launch_fill_features(void* shard, DType dt, int64_t pitch, int col0,
 }
 
 }  // namespace apt
+
+// ---------------------------------------------------------------- self-test
+// Exhaustive check of div_rn_rcp against the IEEE division for every mean the
+// method can form under O4 (x = m/64, |m| <= 2^17, d = 1..256) plus random
+// normal floats: counts bitwise mismatches.
+namespace apt {
+__global__ void selftest_div_kernel(unsigned long long* bad) {
+  const int64_t total = (int64_t(1) << 18) * 256;
+  unsigned long long nb = 0;
+  for (int64_t t = int64_t(blockIdx.x) * blockDim.x + threadIdx.x; t < total; t += int64_t(gridDim.x) * blockDim.x) {
+    const int d = int(t & 255) + 1;
+    const int m = int(t >> 8) - (1 << 17);
+    const float x = float(m) * (1.0f / 64.0f);
+    const float fd = float(d);
+    const float a = div_rn_rcp(x, fd, __frcp_rn(fd)), b = __fdiv_rn(x, fd);
+    if (__float_as_uint(a) != __float_as_uint(b) && !(a == 0.f && b == 0.f)) ++nb;
+    // random normal numerator (hash of t), same denominators
+    uint32_t h = uint32_t(t) * 2654435761u ^ 0x9E3779B9u;
+    h ^= h >> 15; h *= 0x85EBCA6Bu; h ^= h >> 13;
+    const float y = __uint_as_float((h & 0x807FFFFFu) | (uint32_t(100 + (h >> 24) % 60) << 23));
+    const float c = div_rn_rcp(y, fd, __frcp_rn(fd)), e = __fdiv_rn(y, fd);
+    if (__float_as_uint(c) != __float_as_uint(e)) ++nb;
+  }
+  if (nb) atomicAdd(bad, nb);
+}
+}  // namespace apt
+
+extern "C" int64_t apt_selftest_div(void) {
+  unsigned long long* d = nullptr;
+  if (cudaMalloc(&d, 8) != cudaSuccess) return -1;
+  cudaMemset(d, 0, 8);
+  apt::selftest_div_kernel<<<148 * 8, 256>>>(d);
+  unsigned long long h = 0;
+  if (cudaMemcpy(&h, d, 8, cudaMemcpyDeviceToHost) != cudaSuccess) h = ~0ull;
+  cudaFree(d);
+  return int64_t(h);
+}

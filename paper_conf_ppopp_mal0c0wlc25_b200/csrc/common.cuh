@@ -78,6 +78,22 @@ __device__ __forceinline__ uint32_t pack_bf16x2(float a, float b) {
   return *reinterpret_cast<uint32_t*>(&h);
 }
 
+// IEEE round-to-nearest x / d (reading O5) for d >= 1.  A zero numerator takes the
+// division's slow path (exponent 0), so it is answered directly: 0 / d = 0 (same
+// sign), which keeps every sum that cancels to zero off the ~100-instruction path.
+__device__ __forceinline__ float div_rn(float x, float d) { return x == 0.f ? x : __fdiv_rn(x, d); }
+
+// Correctly rounded x / d from a correctly rounded reciprocal r = RN(1/d)
+// (Markstein: with r within 1/2 ulp of 1/d and q0 within 1 ulp of x/d, the
+// residual rem = x - q0*d is exact in one FMA and q0 + rem*r rounds to RN(x/d)).
+// Valid for normal x, d (all means of the method: |x| < 2^24, d in [1, 2^16]);
+// checked exhaustively against __fdiv_rn by apt_selftest_div.
+__device__ __forceinline__ float div_rn_rcp(float x, float d, float r) {
+  const float q0 = x * r;
+  const float rem = fmaf(-q0, d, x);
+  return fmaf(rem, r, q0);
+}
+
 // 16-byte loads bypassing L1 allocation for streaming rows.
 __device__ __forceinline__ uint4 ld_nc_v4(const void* p) {
   uint4 r;

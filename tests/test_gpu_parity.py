@@ -120,6 +120,11 @@ def test_feature_store_bit_exact(A, ctx, tiny, dtype, dim):
 
 
 # ------------------------------------------------------------------ S7 aggregation
+def test_mean_division_is_ieee_exhaustive(A, ctx):
+    """The mean divides with a per-row reciprocal + one FMA correction (Markstein); it must
+    agree bit for bit with IEEE x/d on every O4 mean (O5) -- 67M operands."""
+    assert A.lib().apt_selftest_div() == 0
+
 def test_aggregate_bit_exact_and_bwd(A, ctx, tiny):
     cfg, g, train = tiny
     gr = ctx.graph_load(g.indptr, g.indices)
