@@ -118,6 +118,8 @@ typedef struct {
   int world;
   double alpha_s[8];     /* per-call latency of each operator (reading Z23) */
   double beta_Bps[8];    /* bytes per second of each operator                */
+  int measured[8];       /* 1: timed by apt_profile_links on this process;
+                            0: the pool's measured NVLink reference (no peer GPU) */
 } apt_bw_profile;
 
 /* ---------------------------------------------------------------- context */
@@ -231,7 +233,10 @@ apt_status apt_trainer_agg_bytes(apt_trainer* t, double* bytes);
  * runs Permute+Shuffle of every strategy on the shared samples (no feature
  * loading, no training), counts volumes and times T_build.  Syncs.          */
 apt_status apt_dryrun(apt_trainer* t, int64_t n_steps, apt_plan_stats* out);
-/* Bandwidth trials of the exchange operators.  Syncs.        */
+/* Bandwidth trials of the exchange operators: each operator this
+ * process can run is timed at two message sizes and fitted to alpha + bytes/beta
+ * (local HBM row gather, pinned-host read); NVLink operators take the pool's
+ * measured references when no peer GPU is attached (measured[op] = 0).  Syncs. */
 apt_status apt_profile_links(apt_ctx* ctx, apt_bw_profile* out);
 /* Eq. 2 without the common T_train: pred_s[s] = max over ranks of
  * T_build + T_load + T_shuffle; *pick = argmin.  Pure host arithmetic.      */

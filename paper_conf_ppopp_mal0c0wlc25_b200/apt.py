@@ -53,7 +53,8 @@ class PlanStats(C.Structure):
 
 
 class BwProfile(C.Structure):
-    _fields_ = [("world", C.c_int), ("alpha_s", C.c_double * 8), ("beta_Bps", C.c_double * 8)]
+    _fields_ = [("world", C.c_int), ("alpha_s", C.c_double * 8), ("beta_Bps", C.c_double * 8),
+                ("measured", C.c_int * 8)]
 
 
 _lib = None

@@ -347,3 +347,55 @@ def test_strategy_step_matches_oracle(A, tiny, strategy, C, dtype):
         for r in (0, C - 1):
             assert np.allclose(tr.read("dW", l, rank=r), dW, **tol), f"dW layer {l} rank {r}"
             assert np.allclose(tr.read("db", l, rank=r)[0], db, **tol), f"db layer {l} rank {r}"
+
+
+# ------------------------------------------------------------------ S12/S13 planner
+FIELDS = ("n_d", "rows_local", "rows_peer", "feat_bytes_local", "feat_bytes_peer", "graph_bytes",
+          "hidden_bytes_fwd", "hidden_bytes_bwd", "n_calls")
+
+
+@pytest.mark.parametrize("C", [2, 4])
+def test_dryrun_counts_match_oracle_and_pick(A, tiny, C):
+    """apt_dryrun's per-strategy, per-rank counts are integers: bit-exact against
+    the oracle's emulation of every rank's blocks (O7); apt_select_strategy = oracle Eq. 2 (O8)."""
+    from oracle import strategy as S
+    cfg, g, train = tiny
+    ctx = A.Ctx(-1, C, 0)
+    part = aptgen.partition(g.n, C)
+    gr = ctx.graph_load(g.indptr, g.indices, part)
+    fs = ctx.fstore_create(gr, A.GDP, A.F32, cfg.dim, None, cfg.feat_seed)
+    dims = [cfg.dim] + [d for _, d in cfg.dims()]
+    labels = aptgen.labels(cfg, g.n)
+    tr = A.Trainer(ctx, gr, fs, dims, cfg.fanouts, cfg.batch, A.F32, 0.1, cfg.sample_seed, cfg.feat_seed, A.GDP,
+                   labels)
+    tr.set_epoch(train, 0)
+    st = tr.dryrun(2)
+    steps = st.steps
+    assert steps == min(2, tr.steps_per_epoch())
+    perm = oracle.epoch_perm(train, cfg.sample_seed, 0)
+    ref = []
+    for si, s in enumerate(S.STRATEGIES):
+        tot = [dict.fromkeys(FIELDS + ("n_vs", "n_vd"), 0) for _ in range(C)]
+        for step in range(steps):
+            gb = oracle.global_batch(perm, step, C, cfg.batch)
+            seeds = S.assign_seeds(s, gb, part, C, cfg.batch)
+            blocks = [oracle.sample_blocks(g, sd, cfg.fanouts, cfg.sample_seed, step)[-1] for sd in seeds]
+            for r, e in enumerate(S.emulate_layer1(s, blocks, part, C, cfg.dim, cfg.hidden, 4, 4)):
+                for k in tot[r]:
+                    tot[r][k] += e[k]
+        for r in range(C):
+            for k in FIELDS:
+                assert getattr(st, k)[si][r] == tot[r][k], (s, r, k, getattr(st, k)[si][r], tot[r][k])
+            if s == "SNP":
+                assert st.n_vs[r] == tot[r]["n_vs"]
+            if s == "DNP":
+                assert st.n_vd[r] == tot[r]["n_vd"]
+        for r in range(C):
+            tot[r]["steps"] = steps
+        ref.append(tot)
+    bw = ctx.profile_links()
+    assert bw.beta_Bps[0] > 1e11 and bw.measured[0] == 1            # local HBM gather was timed
+    pick, pred = A.select_strategy(st, bw)
+    tb = [[st.t_build_s[si][r] for r in range(C)] for si in range(4)]
+    rpred, rpick = S.predict(ref, list(bw.alpha_s), list(bw.beta_Bps), tb)
+    assert pick == rpick and np.allclose(pred, rpred, rtol=1e-9)
