@@ -216,6 +216,18 @@ apt_status apt_trainer_loss(apt_trainer* t, float* loss);
 /* Record/replay the device part of apt_trainer_step as a CUDA graph.        */
 apt_status apt_trainer_use_graph(apt_trainer* t, int enable);
 
+/* The first GNN layer alone under the trainer's strategy -- the layer APT
+ * parallelises (upper layers are data parallel and may be the
+ * caller's own).  apt_layer_fwd: seeds of `step`, K-hop sampling and the layer-1
+ * Permute/Shuffle/Execute/Reshuffle for every hosted rank; h^1 is read
+ * with apt_trainer_read(H, layer 1).  Async.
+ * apt_layer_bwd: dh1[i] = device fp32 dL/dh^1 of hosted rank i (rows = its layer-1
+ * destinations, `pitch` floats apart); computes dL/dpre^1 (ReLU mask when K > 1)
+ * and dW^1, db^1 of the strategy (owners' g^T Z, requester db), all-reduced over
+ * the ranks (NFP: column-owned slices, read back concatenated).  Async.        */
+apt_status apt_layer_fwd(apt_trainer* t, int64_t step);
+apt_status apt_layer_bwd(apt_trainer* t, const float* const* dh1, int64_t pitch);
+
 /* Readouts for tests (syncs).  what: 0 seeds, 1 layer-l dst ids, 2 Z_l (fp32),
  * 3 H_l (post-activation / logits), 4 dW_l, 5 db_l, 6 G_l (dL/dpre).
  * Copies min(cap, rows*cols) values (int32 for ids, fp32 otherwise).         */

@@ -84,7 +84,7 @@ def lib():
             "apt_trainer_step_host": [vp, vp, i64, i64, i32, vp], "apt_trainer_loss": [vp, vp],
             "apt_trainer_use_graph": [vp, i32], "apt_trainer_read": [vp, i32, i32, i32, vp, i64, vp, vp],
             "apt_trainer_phase_ms": [vp, vp, i32], "apt_trainer_agg_bytes": [vp, vp],
-            "apt_dryrun": [vp, i64, vp], "apt_profile_links": [vp, vp], "apt_select_strategy": [vp, vp, vp, vp],
+            "apt_dryrun": [vp, i64, vp], "apt_layer_fwd": [vp, i64], "apt_layer_bwd": [vp, vp, i64], "apt_profile_links": [vp, vp], "apt_select_strategy": [vp, vp, vp, vp],
         }
         for name, args in sig.items():
             f = getattr(L, name)
@@ -308,6 +308,14 @@ class Trainer(Handle):
         ms = (C.c_double * 6)()
         self.ctx.ck(lib().apt_trainer_phase_ms(self.h, ms, 6))
         return list(ms)
+
+    def layer_fwd(self, step):
+        self.ctx.ck(lib().apt_layer_fwd(self.h, step))
+
+    def layer_bwd(self, dh1_list, pitch):
+        """dh1_list: one device tensor per hosted rank (fp32 [rows x pitch])."""
+        arr = (C.c_void_p * len(dh1_list))(*[_ptr(x) for x in dh1_list])
+        self.ctx.ck(lib().apt_layer_bwd(self.h, arr, pitch))
 
     def dryrun(self, n_steps):
         st = PlanStats()

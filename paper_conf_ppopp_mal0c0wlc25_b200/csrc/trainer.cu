@@ -58,6 +58,17 @@ static cudaError_t record_ev(apt_trainer* t, int i) {
 // call could overwrite before the copy runs); graph replays patch the argument.
 __global__ void set_step_kernel(uint64_t* step_dev, uint64_t step) { *step_dev = step; }
 
+// dst[r][0:cols] = src[r][0:cols] for r < *n (device count)
+__global__ void copy_rows_kernel(float* __restrict__ dst, int64_t dp, const float* __restrict__ src, int64_t sp, int cols,
+                                 const int32_t* __restrict__ n_p) {
+  const int64_t total = int64_t(*n_p) * cols;
+  for (int64_t t = int64_t(blockIdx.x) * blockDim.x + threadIdx.x; t < total; t += int64_t(gridDim.x) * blockDim.x) {
+    const int64_t r = t / cols;
+    const int c = int(t - r * cols);
+    dst[r * dp + c] = src[r * sp + c];
+  }
+}
+
 __global__ void zero_rows_kernel(float* p, int64_t pitch, const int32_t* n_p) {
   const int64_t total = int64_t(*n_p) * pitch;
   float4* q = reinterpret_cast<float4*>(p);
@@ -545,6 +556,72 @@ apt_status step_body(apt_trainer* t, int update, bool host_batch) {
 }  // namespace apt
 
 extern "C" {
+
+// ---- the first layer alone (the part APT parallelises): forward ...
+apt_status apt_layer_fwd(apt_trainer* t, int64_t step) {
+  if (!t || !t->perm) return set_err(t ? t->ctx : nullptr, APT_E_STATE, "apt_layer_fwd: call apt_trainer_set_epoch first");
+  apt_ctx* c = t->ctx;
+  if (c->broken) return set_err(c, APT_E_STATE, "ctx is broken by an earlier CUDA error");
+  set_step_kernel<<<1, 1, 0, c->stream>>>(t->step_dev, uint64_t(step));
+  CK(c, cudaGetLastError());
+  c->launches++;
+  for (auto& rs : t->R) {
+    apt_status s = phase_sample(t, rs, false);
+    if (s != APT_OK) return s;
+  }
+  if (t->world == 1 || t->s == APT_GDP) {
+    bool first = true;
+    for (auto& rs : t->R) {
+      apt_status s = layer1_fwd_gdp(t, rs, first);
+      first = false;
+      if (s != APT_OK) return s;
+    }
+    return APT_OK;
+  }
+  return layer1_fwd_strategy(t);
+}
+
+// ... and backward from dL/dh1 (one device pointer per hosted rank, rows of the
+// rank's layer-1 destinations, fp32, `pitch` floats apart): dW1/db1 of the
+// strategy, all-reduced over the ranks (NFP: column-owned slices).
+apt_status apt_layer_bwd(apt_trainer* t, const float* const* dh1, int64_t pitch) {
+  if (!t || !dh1 || pitch < t->m.dims[1]) return set_err(t ? t->ctx : nullptr, APT_E_INVALID, "apt_layer_bwd: bad arguments");
+  apt_ctx* c = t->ctx;
+  const bool bf = t->m.dtype == APT_BF16;
+  const int relu = t->K > 1 ? 1 : 0;
+  for (size_t li = 0; li < t->R.size(); ++li) {
+    RankState& rs = t->R[li];
+    Layer& L = rs.L[0];
+    if (!dh1[li]) return set_err(c, APT_E_INVALID, "apt_layer_bwd: dh1[%zu] is null", li);
+    // G = dh1 (copied over the rows the step produced; the count stays on the device)
+    copy_rows_kernel<<<blocks_for(L.max_rows * L.d_out), 256, 0, c->stream>>>(L.G, L.h_pitch, dh1[li], pitch, L.d_out,
+                                                                             L.n_rows);
+    CK(c, cudaGetLastError());
+    if (bf) CK(c, launch_grad_finish(L.G, L.h_pitch, L.H, L.h_pitch, L.d_out, relu, L.Gb, L.gb_pitch, L.n_rows,
+                                     L.max_rows, c->stream));
+    else if (relu) CK(c, launch_relu_bwd(L.G, L.H, L.h_pitch, L.d_out, L.n_rows, L.max_rows, c->stream));
+    CK(c, cudaMemsetAsync(L.dW, 0, sizeof(float) * (int64_t(L.d_out) * L.d_in + L.d_out), c->stream));
+    c->launches++;
+  }
+  if (t->world == 1 || t->s == APT_GDP) {
+    for (auto& rs : t->R) {
+      apt_status s = layer1_bwd_gdp(t, rs);
+      if (s != APT_OK) return s;
+    }
+  } else {
+    apt_status s = layer1_bwd_strategy(t);
+    if (s != APT_OK) return s;
+  }
+  if (t->world > 1) {
+    if (!c->emulated) return set_err(c, APT_E_UNSUPPORTED, "multi-process all-reduce not attached");
+    const Layer& L = t->R[0].L[0];
+    allreduce_sum_kernel<<<blocks_for(int64_t(L.d_out) * L.d_in + L.d_out), 256, 0, c->stream>>>(
+        t->dW_tab, t->world, int64_t(L.d_out) * L.d_in + L.d_out);
+    CK(c, cudaGetLastError());
+    c->launches++;
+  }
+  return APT_OK;
+}
 
 apt_status apt_trainer_step(apt_trainer* t, int64_t step, int update) {
   if (!t || !t->perm) return set_err(t ? t->ctx : nullptr, APT_E_STATE, "apt_trainer_step: call apt_trainer_set_epoch first");

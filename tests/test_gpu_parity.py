@@ -399,3 +399,53 @@ def test_dryrun_counts_match_oracle_and_pick(A, tiny, C):
     tb = [[st.t_build_s[si][r] for r in range(C)] for si in range(4)]
     rpred, rpick = S.predict(ref, list(bw.alpha_s), list(bw.beta_Bps), tb)
     assert pick == rpick and np.allclose(pred, rpred, rtol=1e-9)
+
+
+@pytest.mark.parametrize("dtype", ["f32", "bf16"])
+@pytest.mark.parametrize("strategy,C", [("GDP", 1), ("GDP", 2), ("NFP", 2), ("SNP", 4), ("DNP", 4)])
+def test_layer_fwd_bwd_api(A, tiny, strategy, C, dtype):
+    """apt_layer_fwd / apt_layer_bwd: the first layer alone under each strategy, with the
+    upstream gradient supplied by the caller (upper layers may be the user's own)."""
+    cfg, g, train = tiny
+    ctx = A.Ctx(-1, C, 0) if C > 1 else A.Ctx(0, 1, 0)
+    part = aptgen.partition(g.n, C)
+    gr = ctx.graph_load(g.indptr, g.indices, part)
+    dt = A.DTYPE[dtype]
+    fs = ctx.fstore_create(gr, A.NFP if strategy == "NFP" else A.GDP, dt, cfg.dim, None, cfg.feat_seed)
+    dims = [cfg.dim] + [d for _, d in cfg.dims()]
+    labels = aptgen.labels(cfg, g.n)
+    tr = A.Trainer(ctx, gr, fs, dims, cfg.fanouts, cfg.batch, dt, 0.1, cfg.sample_seed, cfg.feat_seed,
+                   A.STRATEGY[strategy], labels)
+    params = aptgen.weights(cfg)
+    tr.set_params(params)
+    tr.set_epoch(train, 0)
+    tr.layer_fwd(0)
+    from oracle import strategy as S
+    perm = oracle.epoch_perm(train, cfg.sample_seed, 0)
+    gb = oracle.global_batch(perm, 0, C, cfg.batch)
+    seeds = S.assign_seeds(strategy, gb, part, C, cfg.batch)
+    p64 = [(W.astype(np.float64), b.astype(np.float64)) for W, b in params]
+    rng = np.random.default_rng(C)
+    dW = 0.0
+    db = 0.0
+    dh_dev = []
+    tol = TOL[dtype]
+    for r in range(C):
+        blocks = oracle.sample_blocks(g, seeds[r], cfg.fanouts, cfg.sample_seed, 0)
+        cache = model.forward(blocks, cfg.feat_seed, cfg.dim, p64, dtype,
+                              snp=(part, C) if strategy == "SNP" else None)
+        assert np.allclose(tr.read("H", 1, rank=r), cache["h"][0], **tol)
+        n1, d1 = cache["h"][0].shape
+        dh = rng.normal(size=(n1, d1)).astype(np.float32)
+        gpre = dh.astype(np.float64) * (cache["pre"][0] > 0)
+        if dtype == "bf16":
+            gpre = oracle.bf16_round(gpre)                     # reading R4: g rounded for tcgen05
+        Zs = cache["Zparts"] if cache["Zparts"] is not None else [cache["Z"][0]]
+        dW = dW + sum(gpre.T @ Z for Z in Zs)
+        db = db + gpre.sum(0)
+        dh_dev.append(torch.as_tensor(dh).cuda())
+    tr.layer_bwd(dh_dev, d1)
+    atol = tol["atol"] * 100                                   # unit-scale g: sums of ~1e4 products
+    for r in (0, C - 1):
+        assert np.allclose(tr.read("dW", 1, rank=r), dW, rtol=tol["rtol"], atol=atol)
+        assert np.allclose(tr.read("db", 1, rank=r)[0], db, rtol=tol["rtol"], atol=atol)
