@@ -55,6 +55,8 @@ def parse():
     ap.add_argument("--no-cpu-baseline", action="store_true")
     ap.add_argument("--cpu-steps", type=int, default=3, help="oracle steps for cpu_baseline")
     ap.add_argument("--e2e-steps", type=int, default=10)
+    ap.add_argument("--no-planner", action="store_true")
+    ap.add_argument("--dryrun-steps", type=int, default=8)
     ap.add_argument("--verbose", action="store_true")
     return ap.parse_args()
 
@@ -282,6 +284,8 @@ def run_apt(args, cfg):
                       "backward": phase_mean[3], "allreduce_sgd": phase_mean[4], "agg_kernel": phase_mean[5]},
         "clocks": clk.summary(),
     }
+    if rank == 0 and world == 1 and not args.no_planner:
+        out["planner"] = planner_report(A, g, cfg, train, labels, args, stream, ms_local)
     if rank == 0 and world == 1 and not args.no_cpu_baseline:
         times, nseeds = oracle_steps(cfg, g, train, labels, args.cpu_steps, 1)
         out["cpu_baseline"] = {"value": nseeds / sum(times), "unit": "seeds/s", "cores": 1, "kind": "oracle",
@@ -292,6 +296,42 @@ def run_apt(args, cfg):
     if world > 1:
         dist.destroy_process_group()
     return 0
+
+
+def planner_report(A, g, cfg, train, labels, args, stream, gdp_ms):
+    """APT's Planner on this workload: link trials, then for C = 2, 4, 8 a dry-run
+    of every strategy over the first steps of the epoch (all C ranks' blocks counted on this
+    GPU: sampling is a pure function of (seed, node, hop, step)) and Eq. 2's prediction per
+    strategy + the pick.  Predictions only for C > 1: this run has one GPU, so no C > 1 step
+    is measured; at C = 1 every strategy is the measured GDP step."""
+    dt = A.DTYPE[args.dtype]
+    rep = {"note": "pred = T_build + T_load + T_shuffle per step (max over ranks), common T_train excluded; "
+                   "NVLink betas are the pool's measured references (no peer GPU in this run)"}
+    for C in (2, 4, 8):
+        ctx = A.Ctx(-1, C, 0, stream.cuda_stream)
+        gr = ctx.graph_load(g.indptr, g.indices, aptgen.partition(g.n, C))
+        fs = ctx.fstore_create(gr, A.GDP, dt, cfg.dim, None, cfg.feat_seed)
+        dims = [cfg.dim] + [d for _, d in cfg.dims()]
+        tr = A.Trainer(ctx, gr, fs, dims, cfg.fanouts, cfg.batch, dt, 0.05, cfg.sample_seed, cfg.feat_seed, A.GDP,
+                       labels)
+        tr.set_epoch(train, 0)
+        st = tr.dryrun(args.dryrun_steps)
+        bw = ctx.profile_links()
+        pick, pred = A.select_strategy(st, bw)
+        steps = max(1, st.steps)
+        rep[f"C{C}"] = {"dryrun_steps": st.steps, "pred_ms_per_step": {s: 1e3 * p / steps for s, p in zip(STRATS, pred)},
+                        "pick": STRATS[pick],
+                        "n_vs_per_step": sum(st.n_vs[r] for r in range(C)) / steps,
+                        "n_vd_per_step": sum(st.n_vd[r] for r in range(C)) / steps}
+        if C == 2:
+            rep["bw_profile"] = {"local_gather_GBps": bw.beta_Bps[0] / 1e9, "local_gather_alpha_us": bw.alpha_s[0] * 1e6,
+                                 "host_read_GBps": bw.beta_Bps[7] / 1e9, "measured": list(bw.measured)}
+        for h in (tr, fs, gr):
+            h.close()
+        ctx.close()
+    rep["C1"] = {"measured_ms_per_step": {s: gdp_ms for s in STRATS}, "pick": "GDP",
+                 "note": "at C = 1 every strategy degenerates to GDP (SURVEY §8(d))"}
+    return rep
 
 
 def layer1_bytes(ctx, gr, tr, cfg, rank, step, bf):
