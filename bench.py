@@ -187,7 +187,7 @@ def run_apt(args, cfg):
     dt = A.DTYPE[args.dtype]
     ctx = A.Ctx(rank if world > 1 else 0, world, local, stream.cuda_stream)
     if world > 1:
-        raise SystemExit("multi-process strategies are not wired into bench.py yet")
+        ctx.set_exchange(dist)   # CUDA-IPC peer mappings + device barrier (bootstrap only)
     gr = ctx.graph_load(g.indptr, g.indices, part)
     strat = A.STRATEGY[args.strategy]
     fs = ctx.fstore_create(gr, strat if strat == A.NFP else A.GDP, dt, cfg.dim, None, cfg.feat_seed)

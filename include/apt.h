@@ -122,12 +122,25 @@ typedef struct {
                             0: the pool's measured NVLink reference (no peer GPU) */
 } apt_bw_profile;
 
+/* All-gather used to bootstrap a job of one process per GPU: every rank passes
+ * `bytes` bytes in `send`; on return `recv` holds world*bytes bytes, rank p's
+ * block at offset p*bytes.  Returns 0 on success.  (The Python binding supplies
+ * one built on torch.distributed.)  Used only while creating objects, never on
+ * the step path.                                                            */
+typedef int (*apt_allgather_fn)(const void* send, void* recv, size_t bytes, void* user);
+
 /* ---------------------------------------------------------------- context */
 /* rank >= 0: one rank of `world`; rank == -1: all `world` ranks emulated on
  * `device`.  cuda_stream may be NULL (library-created stream).              */
 apt_status apt_ctx_create(int rank, int world, int device, void* cuda_stream, apt_ctx** out);
 apt_status apt_ctx_destroy(apt_ctx* ctx);
 const char* apt_last_error(const apt_ctx* ctx);
+/* Multi-process job (rank >= 0, world > 1): install the bootstrap all-gather.
+ * Collective.  Sets up the device barrier (peer-mapped flag arrays); objects
+ * created afterwards map their peers' buffers through CUDA IPC.              */
+apt_status apt_ctx_set_exchange(apt_ctx* ctx, apt_allgather_fn fn, void* user);
+/* Host-only check of an exchange function's protocol (no GPU used). Collective. */
+apt_status apt_exchange_selftest(int rank, int world, apt_allgather_fn fn, void* user);
 /* Syncs: waits for the ctx stream and reports device-side error words.      */
 apt_status apt_ctx_sync(apt_ctx* ctx);
 /* Copy helper for tests/bindings: kind 0 = D2H, 1 = H2D, 2 = D2D. Syncs.   */

@@ -59,6 +59,30 @@ class BwProfile(C.Structure):
 
 _lib = None
 
+# int (*apt_allgather_fn)(const void* send, void* recv, size_t bytes, void* user)
+ALLGATHER_FN = C.CFUNCTYPE(C.c_int, C.c_void_p, C.c_void_p, C.c_size_t, C.c_void_p)
+
+
+def make_exchange(dist, group=None):
+    """Bootstrap all-gather for a job of one process per GPU, on torch.distributed
+    (any backend).  Plumbing only: the library calls it while creating objects to
+    swap CUDA-IPC handles, never on the step path."""
+    world = dist.get_world_size(group)
+
+    @ALLGATHER_FN
+    def fn(send, recv, nbytes, user):
+        try:
+            out = [None] * world
+            dist.all_gather_object(out, C.string_at(send, nbytes), group=group)
+            blob = b"".join(out)
+            if len(blob) != nbytes * world:
+                return 2
+            C.memmove(recv, blob, len(blob))
+            return 0
+        except Exception:
+            return 1
+    return fn
+
 
 def lib():
     global _lib
@@ -94,6 +118,10 @@ def lib():
         L.apt_last_error.restype = C.c_char_p
         L.apt_ctx_launches.argtypes = [vp]
         L.apt_ctx_launches.restype = C.c_int64
+        L.apt_ctx_set_exchange.argtypes = [vp, ALLGATHER_FN, vp]
+        L.apt_ctx_set_exchange.restype = st
+        L.apt_exchange_selftest.argtypes = [i32, i32, ALLGATHER_FN, vp]
+        L.apt_exchange_selftest.restype = st
         L.apt_selftest_div.argtypes = []
         L.apt_selftest_div.restype = C.c_int64
         L.apt_trainer_steps_per_epoch.argtypes = [vp]
@@ -139,6 +167,11 @@ class Ctx:
 
     def ck(self, s):
         check(s, self.h)
+
+    def set_exchange(self, dist, group=None):
+        """Multi-process job: install the torch.distributed bootstrap all-gather (collective)."""
+        self._xfn = make_exchange(dist, group)
+        self.ck(lib().apt_ctx_set_exchange(self.h, self._xfn, None))
 
     def sync(self):
         self.ck(lib().apt_ctx_sync(self.h))
@@ -321,6 +354,12 @@ class Trainer(Handle):
         st = PlanStats()
         self.ctx.ck(lib().apt_dryrun(self.h, n_steps, C.byref(st)))
         return st
+
+
+def exchange_selftest(rank, world, dist, group=None):
+    """Host-only check of the bootstrap all-gather protocol (no GPU)."""
+    fn = make_exchange(dist, group)
+    check(lib().apt_exchange_selftest(rank, world, fn, None))
 
 
 def select_strategy(stats: PlanStats, bw: BwProfile):

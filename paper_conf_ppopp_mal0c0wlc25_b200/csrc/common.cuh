@@ -109,7 +109,7 @@ __device__ __forceinline__ void red_add_v4(float* p, float a, float b, float c, 
 }
 
 // Device error word: kernels OR an APT_DEV_* bit on invalid input instead of trapping.
-enum : uint32_t { kDevErrBadId = 1u, kDevErrOverflow = 2u };
+enum : uint32_t { kDevErrBadId = 1u, kDevErrOverflow = 2u, kDevErrTimeout = 4u };
 
 }  // namespace apt
 

@@ -26,8 +26,11 @@ apt_status set_err(apt_ctx* c, apt_status s, const char* fmt, ...) {
   return s;
 }
 
+void release_exported(apt_ctx* c);
+
 static void ctx_free(apt_ctx* c) {
   cudaStreamSynchronize(c->stream);
+  release_exported(c);
   c->arena.release();
   if (c->own_stream) cudaStreamDestroy(c->stream);
   delete c;
@@ -246,6 +249,13 @@ apt_status apt_fstore_create(apt_ctx* c, const apt_graph* g, apt_strategy layout
       c->launches++;
       CK(c, cudaStreamSynchronize(c->stream));
     }
+  }
+  if (multiprocess(c) && f->layout != APT_NFP) {
+    // row-sharded store: every rank maps every peer's shard (GDP / DNP halo reads over NVLink)
+    void* tab[APT_MAX_RANKS] = {};
+    apt_status s = share_ptr(c, f->shard[c->rank], tab, &f->peer_opened);
+    if (s != APT_OK) { apt_fstore_destroy(f); return s; }
+    for (int r = 0; r < C; ++r) f->shard[r] = tab[r];
   }
   *out = f;
   return APT_OK;

@@ -32,7 +32,12 @@ struct Arena {
     size_t bytes = size_t(std::max<int64_t>(n, 1)) * sizeof(T);
     bytes = (bytes + 255) & ~size_t(255);
     if (cudaMalloc(&p, bytes) != cudaSuccess) return nullptr;
-    if (zero) cudaMemset(p, 0, bytes);
+    // cudaMemset runs on the legacy stream, which does not order against the ctx's
+    // non-blocking stream: wait for it, or a later kernel's output could be zeroed
+    if (zero && (cudaMemset(p, 0, bytes) != cudaSuccess || cudaStreamSynchronize(cudaStreamLegacy) != cudaSuccess)) {
+      cudaFree(p);
+      return nullptr;
+    }
     bufs.push_back({p, bytes});
     total += bytes;
     return static_cast<T*>(p);
@@ -43,6 +48,17 @@ struct Arena {
 // the last child (any destruction order is safe, e.g. at interpreter exit).
 void ctx_retain(apt_ctx* c);
 void ctx_release(apt_ctx* c);
+
+// comm.cu: one process per GPU
+bool multiprocess(const apt_ctx* c);
+apt_status allgather(apt_ctx* c, const void* send, void* recv, size_t bytes);
+apt_status share_ptr(apt_ctx* c, void* local, void** tab, std::vector<void*>* opened);
+void close_peers(std::vector<void*>& opened);
+apt_status device_barrier(apt_ctx* c);
+// Multi-process: an exporter may free a buffer only after every importer closed its
+// mapping (CUDA IPC rule), so objects hand their buffers to the ctx, which frees them
+// at its (collective) destruction behind a host barrier.
+void defer_exported(apt_ctx* c, Arena& a);
 
 }  // namespace apt
 
@@ -59,6 +75,13 @@ struct apt_ctx {
   std::string err;
   int64_t launches = 0;
   int children = 0;      // live graphs / stores / batches / trainers created on this ctx
+  apt_allgather_fn exchange = nullptr;   // multi-process bootstrap (apt_ctx_set_exchange)
+  void* exchange_user = nullptr;
+  uint64_t* bar_flags = nullptr;         // [APT_MAX_RANKS] arrival slots + epoch (device barrier)
+  uint64_t** bar_tab = nullptr;          // every rank's bar_flags (peer-mapped)
+  std::vector<void*> peer_opened;        // IPC mappings to close
+  std::vector<apt::DevBuf> deferred;     // exported buffers of destroyed objects: freed only at
+                                         // ctx destroy, after every peer has closed its mapping
   bool zombie = false;   // apt_ctx_destroy called while children were alive
   uint32_t* dev_err = nullptr;   // device error word
   int32_t* scratch = nullptr;    // small device ints for single-op calls
@@ -91,7 +114,9 @@ struct apt_fstore {
   int col_lo[APT_MAX_RANKS] = {};
   int col_hi[APT_MAX_RANKS] = {};
   int64_t rows[APT_MAX_RANKS] = {};
+  std::vector<void*> peer_opened;   // IPC-mapped peer shards (multi-process)
   apt::Arena arena;
+  ~apt_fstore() { apt::close_peers(peer_opened); apt::defer_exported(ctx, arena); }
 };
 
 struct apt_batch {

@@ -29,6 +29,7 @@
 // compute dW^1 += g^T Z on tcgen05 (or exact fp32), the requester adds db^1;
 // dW^1 is all-reduced for DNP/SNP, column-owned (never reduced) for NFP.
 #include <algorithm>
+#include <type_traits>
 #include <vector>
 
 #include "common.cuh"
@@ -231,20 +232,39 @@ apt_status strategy_alloc(apt_trainer* t, RankState& rs) {
   return APT_OK;
 }
 
-// Pointer tables over all ranks (after every hosted rank is allocated).
+// Pointer tables over all ranks (after every hosted rank is allocated): the
+// hosted ranks' own buffers in an emulated job, CUDA-IPC-mapped peer buffers in a
+// job of one process per GPU.
 apt_status strategy_tables(apt_trainer* t) {
   const int C = t->world;
   std::vector<float*> h1(C), g1(C);
   std::vector<uint16_t*> gb1(C);
   std::vector<int32_t*> wn(C), wr(C), wrow(C), wg(C);
-  for (auto& rs : t->R) {
-    h1[rs.rank] = rs.L[0].H;
-    g1[rs.rank] = rs.L[0].G;
-    gb1[rs.rank] = rs.L[0].Gb;
-    wn[rs.rank] = rs.x.n_work;
-    wr[rs.rank] = rs.x.work_rank;
-    wrow[rs.rank] = rs.x.work_row;
-    wg[rs.rank] = rs.x.work_gid;
+  if (multiprocess(t->ctx)) {
+    RankState& rs = t->R[0];
+    auto share = [&](auto& tab, auto* mine) -> apt_status {
+      if (!mine) return APT_OK;
+      std::vector<void*> v(C, nullptr);
+      apt_status s = share_ptr(t->ctx, mine, v.data(), &t->peer_opened);
+      for (int p = 0; p < C; ++p) tab[p] = static_cast<std::remove_reference_t<decltype(tab[0])>>(v[p]);
+      return s;
+    };
+    apt_status s;
+    if ((s = share(h1, rs.L[0].H)) != APT_OK || (s = share(g1, rs.L[0].G)) != APT_OK ||
+        (s = share(gb1, rs.L[0].Gb)) != APT_OK || (s = share(wn, rs.x.n_work)) != APT_OK ||
+        (s = share(wr, rs.x.work_rank)) != APT_OK || (s = share(wrow, rs.x.work_row)) != APT_OK ||
+        (s = share(wg, rs.x.work_gid)) != APT_OK)
+      return s;
+  } else {
+    for (auto& rs : t->R) {
+      h1[rs.rank] = rs.L[0].H;
+      g1[rs.rank] = rs.L[0].G;
+      gb1[rs.rank] = rs.L[0].Gb;
+      wn[rs.rank] = rs.x.n_work;
+      wr[rs.rank] = rs.x.work_rank;
+      wrow[rs.rank] = rs.x.work_row;
+      wg[rs.rank] = rs.x.work_gid;
+    }
   }
   t->H1_tab = upload_tab(t, h1);
   t->G1_tab = upload_tab(t, g1);
@@ -330,6 +350,7 @@ apt_status layer1_fwd_strategy(apt_trainer* t) {
       CK(c, cudaMemsetAsync(L.H, 0, sizeof(float) * L.max_rows * L.h_pitch, c->stream));
     }
   }
+  { apt_status s = device_barrier(c); if (s != APT_OK) return s; }   // lists cleared everywhere
   for (auto& rs : t->R) {
     const Hop& hp = rs.hops[t->K - 1];
     permute_kernel<<<grid_n(hp.max_dst), 256, 0, c->stream>>>(mode, rs.rank, t->world, hp.dst, hp.n_dst, hp.cnt,
@@ -337,6 +358,7 @@ apt_status layer1_fwd_strategy(apt_trainer* t) {
     CK(c, cudaGetLastError());
     c->launches++;
   }
+  { apt_status s = device_barrier(c); if (s != APT_OK) return s; }   // every list complete
   // Execute + Reshuffle on every owner
   bool first = true;
   for (auto& rs : t->R) {
@@ -344,6 +366,7 @@ apt_status layer1_fwd_strategy(apt_trainer* t) {
     first = false;
     if (s != APT_OK) return s;
   }
+  { apt_status s = device_barrier(c); if (s != APT_OK) return s; }   // every h^1 row delivered
   // requesters finish the partial sums: bias once, then the activation (Z10)
   if (partial) {
     for (auto& rs : t->R) {
@@ -368,6 +391,7 @@ apt_status layer1_bwd_strategy(apt_trainer* t) {
                       : launch_colsum2(c, L.G, false, L.h_pitch, L.d_out, L.n_rows, L.db);
     if (s != APT_OK) return s;
   }
+  { apt_status s = device_barrier(c); if (s != APT_OK) return s; }   // every requester's g ready
   // owners: gather g of their items, dW^1 (+)= g^T Z
   for (auto& rs : t->R) {
     Xchg& x = rs.x;

@@ -39,6 +39,17 @@ apt_status layer1_bwd_strategy(apt_trainer* t);
 
 namespace apt {
 
+// One process per GPU: out[i] = sum over ranks of tab[r][i] (peer loads over NVLink);
+// the caller fences with device barriers before (peers' gradients complete) and
+// after (everyone has read them) and copies out -> own buffer.
+__global__ void allreduce_gather_kernel(float* const* tab, int C, int64_t n, float* __restrict__ out) {
+  for (int64_t i = int64_t(blockIdx.x) * blockDim.x + threadIdx.x; i < n; i += int64_t(gridDim.x) * blockDim.x) {
+    float s = 0.f;
+    for (int r = 0; r < C; ++r) s += tab[r][i];   // fixed rank order: every rank gets identical sums
+    out[i] = s;
+  }
+}
+
 __global__ void allreduce_sum_kernel(float* const* tab, int C, int64_t n) {
   for (int64_t i = int64_t(blockIdx.x) * blockDim.x + threadIdx.x; i < n; i += int64_t(gridDim.x) * blockDim.x) {
     float s = 0.f;
@@ -243,7 +254,17 @@ apt_status apt_trainer_create(apt_ctx* c, const apt_graph* g, const apt_fstore* 
     apt_status st = strategy_tables(t);
     if (st != APT_OK) { apt_trainer_destroy(t); return st; }
   }
-  {
+  if (multiprocess(c)) {
+    // every rank reads every peer's flat gradient buffer in the all-reduce
+    std::vector<void*> v(C, nullptr);
+    apt_status st = share_ptr(c, t->R[0].L[0].dW, v.data(), &t->peer_opened);
+    if (st != APT_OK) { apt_trainer_destroy(t); return st; }
+    int64_t P = 0;
+    for (auto& L : t->R[0].L) P += int64_t(L.d_out) * L.d_in + L.d_out;
+    t->ar_scratch = A.alloc<float>(P, false);
+    t->dW_tab = A.alloc<float*>(C, false);
+    CK(c, cudaMemcpyAsync(t->dW_tab, v.data(), sizeof(float*) * C, cudaMemcpyHostToDevice, c->stream));
+  } else {
     std::vector<float*> tab(C, nullptr);
     for (auto& rs : t->R) tab[rs.rank] = rs.L[0].dW;
     t->dW_tab = A.alloc<float*>(C, false);
@@ -468,15 +489,33 @@ apt_status layer1_bwd_gdp(apt_trainer* t, RankState& rs) {
                      bf ? L.zb_pitch : L.zf_pitch, L.n_rows, L.max_rows, L.d_in, L.dW, L.db, L.d_in);
 }
 
+// Gradient all-reduce over the ranks (DDP) of the first P floats of the
+// flat gradient buffer [dW1 db1 dW2 ...].
+apt_status allreduce_grads(apt_trainer* t, int64_t P) {
+  apt_ctx* c = t->ctx;
+  if (c->emulated) {
+    allreduce_sum_kernel<<<blocks_for(P), 256, 0, c->stream>>>(t->dW_tab, t->world, P);
+    CK(c, cudaGetLastError());
+    c->launches++;
+    return APT_OK;
+  }
+  apt_status s = device_barrier(c);
+  if (s != APT_OK) return s;
+  allreduce_gather_kernel<<<blocks_for(P), 256, 0, c->stream>>>(t->dW_tab, t->world, P, t->ar_scratch);
+  CK(c, cudaGetLastError());
+  if ((s = device_barrier(c)) != APT_OK) return s;
+  CK(c, cudaMemcpyAsync(t->R[0].L[0].dW, t->ar_scratch, sizeof(float) * P, cudaMemcpyDeviceToDevice, c->stream));
+  c->launches++;
+  return APT_OK;
+}
+
 apt_status allreduce_sgd(apt_trainer* t, int update) {
   apt_ctx* c = t->ctx;
   int64_t P = 0;
   for (auto& L : t->R[0].L) P += int64_t(L.d_out) * L.d_in + L.d_out;
   if (t->world > 1) {
-    if (!c->emulated) return set_err(c, APT_E_UNSUPPORTED, "multi-process all-reduce not attached");
-    allreduce_sum_kernel<<<blocks_for(P), 256, 0, c->stream>>>(t->dW_tab, t->world, P);
-    CK(c, cudaGetLastError());
-    c->launches++;
+    apt_status s = allreduce_grads(t, P);
+    if (s != APT_OK) return s;
   }
   if (!update) return APT_OK;
   for (auto& rs : t->R) {
@@ -613,12 +652,8 @@ apt_status apt_layer_bwd(apt_trainer* t, const float* const* dh1, int64_t pitch)
     if (s != APT_OK) return s;
   }
   if (t->world > 1) {
-    if (!c->emulated) return set_err(c, APT_E_UNSUPPORTED, "multi-process all-reduce not attached");
     const Layer& L = t->R[0].L[0];
-    allreduce_sum_kernel<<<blocks_for(int64_t(L.d_out) * L.d_in + L.d_out), 256, 0, c->stream>>>(
-        t->dW_tab, t->world, int64_t(L.d_out) * L.d_in + L.d_out);
-    CK(c, cudaGetLastError());
-    c->launches++;
+    return allreduce_grads(t, int64_t(L.d_out) * L.d_in + L.d_out);
   }
   return APT_OK;
 }

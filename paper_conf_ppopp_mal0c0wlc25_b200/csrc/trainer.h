@@ -109,9 +109,12 @@ struct apt_trainer {
   cudaGraph_t graph = nullptr;
   cudaGraphNode_t step_node = nullptr;
   int64_t launches_per_step = 0;
+  float* ar_scratch = nullptr;       // multi-process all-reduce: sum of the peers' gradients
+  std::vector<void*> peer_opened;    // IPC mappings of peer buffers
   int graph_update = -1;
   cudaEvent_t ev[8] = {};
   bool ev_ok = false;
   double last_agg_bytes = 0;
   apt::Arena arena;
+  ~apt_trainer() { apt::close_peers(peer_opened); apt::defer_exported(ctx, arena); }
 };

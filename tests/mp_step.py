@@ -1,0 +1,118 @@
+"""One process per rank, all on one B200 (CUDA IPC within the device stands in for
+NVLink): a training step of every strategy through the multi-process path
+(peer-mapped buffers, device barriers, peer all-reduce) against the oracle.
+Launched by tests/test_gpu_multiprocess.py under torchrun; rank 0 prints RESULT."""
+import os
+import sys
+
+ROOT = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
+sys.path.insert(0, ROOT)
+
+import numpy as np  # noqa: E402
+import torch  # noqa: E402
+import torch.distributed as dist  # noqa: E402
+
+import aptgen  # noqa: E402
+import oracle  # noqa: E402
+from oracle import model  # noqa: E402
+from oracle import strategy as S  # noqa: E402
+import paper_conf_ppopp_mal0c0wlc25_b200.apt as A  # noqa: E402
+
+TOL = {"f32": dict(rtol=1e-5, atol=1e-6), "bf16": dict(rtol=2e-2, atol=2e-3)}
+
+
+def main():
+    rank, world = int(os.environ["RANK"]), int(os.environ["WORLD_SIZE"])
+    dev = int(os.environ.get("APT_TEST_DEVICE", os.environ.get("LOCAL_RANK", 0)))
+    dist.init_process_group("gloo")
+    torch.cuda.set_device(dev)
+    cfg = aptgen.CONFIGS["tiny"]
+    g = aptgen.make_graph(cfg)
+    train = aptgen.train_nodes(g, cfg)
+    labels = aptgen.labels(cfg, g.n)
+    part = aptgen.partition(g.n, world)
+    params = aptgen.weights(cfg)
+    p64 = [(W.astype(np.float64), b.astype(np.float64)) for W, b in params]
+    perm = oracle.epoch_perm(train, cfg.sample_seed, 0)
+    errors = []
+    for dtype in sys.argv[1].split(","):
+        for strategy in sys.argv[2].split(","):
+            ctx = A.Ctx(rank, world, dev)
+            ctx.set_exchange(dist)
+            gr = ctx.graph_load(g.indptr, g.indices, part)
+            dt = A.DTYPE[dtype]
+            fs = ctx.fstore_create(gr, A.NFP if strategy == "NFP" else A.GDP, dt, cfg.dim, None, cfg.feat_seed)
+            if strategy != "NFP":   # every row through this rank's view of the sharded store (peer shards via IPC)
+                ids = np.arange(0, g.n, 7, dtype=np.int32)
+                esz = 2 if dtype == "bf16" else 4
+                pitch = (cfg.dim + 7) // 8 * 8 if dtype == "bf16" else (cfg.dim + 3) // 4 * 4
+                buf = torch.zeros(len(ids) * pitch * esz, dtype=torch.uint8, device="cuda")
+                torch.cuda.synchronize()            # torch's zero-fill runs on another stream than the library's
+                ctx.gather(fs, torch.as_tensor(ids).cuda(), len(ids), buf)
+                torch.cuda.synchronize()
+                raw = buf.cpu().numpy()
+                if dtype == "bf16":
+                    got = (raw.view(np.uint16).astype(np.uint32) << 16).view(np.float32).reshape(len(ids), pitch)
+                else:
+                    got = raw.view(np.float32).reshape(len(ids), pitch)
+                ref = oracle.features(cfg.feat_seed, ids.astype(np.int64), cfg.dim)
+                bad = ~(got[:, :cfg.dim] == ref).all(1)
+                if bad.any():
+                    errors.append(f"{strategy}/{dtype}/rank{rank}: store rows wrong: {int(bad.sum())} of {len(ids)}, "
+                                  f"owners {np.bincount(part[ids[bad]], minlength=world).tolist()}")
+            dims = [cfg.dim] + [d for _, d in cfg.dims()]
+            tr = A.Trainer(ctx, gr, fs, dims, cfg.fanouts, cfg.batch, dt, 0.1, cfg.sample_seed, cfg.feat_seed,
+                           A.STRATEGY[strategy], labels)
+            tr.set_params(params)
+            tr.set_epoch(train, 0)
+            tr.use_graph(True)
+            steps = min(2, tr.steps_per_epoch())
+            for step in range(steps):
+                tr.step(step, update=False)
+                try:
+                    ctx.sync()                      # device error word: a barrier timeout would show here
+                except Exception as e:
+                    errors.append(f"{strategy}/{dtype}/step{step}/rank{rank}: {e}")
+                gb = oracle.global_batch(perm, step, world, cfg.batch)
+                seeds = S.assign_seeds(strategy, gb, part, world, cfg.batch)
+                refs = [model.train_step(oracle.sample_blocks(g, seeds[r], cfg.fanouts, cfg.sample_seed, step),
+                                         cfg.feat_seed, cfg.dim, p64, labels[seeds[r]], len(gb), dtype,
+                                         snp=(part, world) if strategy == "SNP" else None) for r in range(world)]
+                tol = TOL[dtype]
+                tag = f"{strategy}/{dtype}/step{step}/rank{rank}"
+                if not np.array_equal(tr.read("seeds", rank=rank)[:, 0], seeds[rank]):
+                    errors.append(f"{tag}: seeds")
+                h1 = tr.read("H", 1, rank=rank)
+                if not np.allclose(h1, refs[rank]["cache"]["h"][0], **tol):
+                    bad = ~np.isclose(h1, refs[rank]["cache"]["h"][0], **tol)
+                    rows = np.nonzero(bad.any(1))[0]
+                    errors.append(f"{tag}: h1 ({len(rows)} of {len(h1)} rows, first {rows[:5].tolist()}, "
+                                  f"max err {np.abs(h1 - refs[rank]['cache']['h'][0]).max():.3g})")
+                for l in range(1, len(cfg.fanouts) + 1):
+                    if strategy == "NFP" and l == 1:
+                        continue   # column-owned: checked on the assembled slices below
+                    ref = sum(x["grads"][l - 1][0] for x in refs)
+                    if not np.allclose(tr.read("dW", l, rank=rank), ref, **tol):
+                        errors.append(f"{tag}: dW{l} max err {np.abs(tr.read('dW', l, rank=rank) - ref).max():.3g}")
+                    refb = sum(x["grads"][l - 1][1] for x in refs)
+                    if not np.allclose(tr.read("db", l, rank=rank)[0], refb, **tol):
+                        errors.append(f"{tag}: db{l}")
+                if strategy == "NFP":
+                    lo, hi = S.col_range(rank, world, cfg.dim)
+                    ref = sum(x["grads"][0][0] for x in refs)[:, lo:hi]
+                    mine = tr.read("dW", 1, rank=rank)[:, lo:hi]
+                    if not np.allclose(mine, ref, **tol):
+                        errors.append(f"{tag}: dW1 slice")
+            for h in (tr, fs, gr):
+                h.close()
+            ctx.close()
+    allerr = [None] * world
+    dist.all_gather_object(allerr, errors)
+    if rank == 0:
+        flat = [e for x in allerr for e in x]
+        print("RESULT", "OK" if not flat else "FAIL " + "; ".join(flat[:20]), flush=True)
+    dist.destroy_process_group()
+
+
+if __name__ == "__main__":
+    main()
