@@ -172,9 +172,14 @@ def run_apt(args, cfg):
     rank, world, local = dist_env()
     if world != args.gpus:
         raise SystemExit(f"--gpus {args.gpus} but WORLD_SIZE={world}")
+    # APT_DEVICE_OVERRIDE: plumbing test with several ranks on one GPU (numbers then meaningless)
+    local = int(os.environ.get("APT_DEVICE_OVERRIDE", local))
     torch.cuda.set_device(local)
     if world > 1:
-        dist.init_process_group("nccl", device_id=torch.device("cuda", local))
+        if "APT_DEVICE_OVERRIDE" in os.environ:   # NCCL refuses two ranks on one GPU
+            dist.init_process_group("gloo")
+        else:
+            dist.init_process_group("nccl", device_id=torch.device("cuda", local))
     # one non-default stream shared by torch (events, L2 flush) and the library
     stream = torch.cuda.Stream()
     torch.cuda.set_stream(stream)
