@@ -46,7 +46,8 @@ constexpr int BM = 128;
 constexpr int BK = 64;              // 64 bf16 = 128 B = one swizzle row
 constexpr int STAGES = 4;
 constexpr int A_STAGE_BYTES = BM * BK * 2;   // 16 KB
-constexpr int THREADS = 192;        // 6 warps
+constexpr int THREADS = 192;        // 6 warps (wgrad)
+constexpr int ROW_THREADS = 320;    // 10 warps: TMA, MMA, 8 epilogue
 constexpr int MNBLK = 8192;         // one MN-major TMA box (64 x 64 bf16)
 
 __device__ __forceinline__ uint32_t smem_u32(const void* p) {
@@ -149,10 +150,10 @@ struct RowParams {
   int accumulate;
 };
 
-__global__ void __launch_bounds__(THREADS, 1)
+__global__ void __launch_bounds__(ROW_THREADS, 1)
     rowtile_kernel(const __grid_constant__ CUtensorMap mapA, const __grid_constant__ CUtensorMap mapB, RowParams p) {
   extern __shared__ __align__(1024) uint8_t smem_raw[];
-  uint8_t* smem = reinterpret_cast<uint8_t*>((reinterpret_cast<uintptr_t>(smem_raw) + 1023) & ~uintptr_t(1023));
+  uint8_t* smem = smem_raw + ((1024u - (smem_u32(smem_raw) & 1023u)) & 1023u);   // 1 KB aligned, still __shared__
   uint8_t* smem_a = smem;                                        // STAGES x 16 KB
   uint8_t* smem_b = smem + STAGES * A_STAGE_BYTES;               // nkb x b_kb_bytes
   uint64_t* bars = reinterpret_cast<uint64_t*>(smem_b + size_t(p.nkb) * p.b_kb_bytes);
@@ -170,7 +171,7 @@ __global__ void __launch_bounds__(THREADS, 1)
   if (warp == 0 && lane == 0) {
     for (int s = 0; s < STAGES; ++s) { mbar_init(full + s, 1); mbar_init(empty + s, 1); }
     mbar_init(bfull, 1);
-    for (int a = 0; a < 2; ++a) { mbar_init(tfull + a, 1); mbar_init(tempty + a, 128); }
+    for (int a = 0; a < 2; ++a) { mbar_init(tfull + a, 1); mbar_init(tempty + a, 256); }
     asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
     asm volatile("prefetch.tensormap [%0];" ::"l"(reinterpret_cast<uint64_t>(&mapA)) : "memory");
     asm volatile("prefetch.tensormap [%0];" ::"l"(reinterpret_cast<uint64_t>(&mapB)) : "memory");
@@ -240,14 +241,15 @@ __global__ void __launch_bounds__(THREADS, 1)
       }
     }
   } else {
-    // ---- epilogue warps 2..5: TMEM lane quarter = warp % 4.  Each 32-column chunk
-    // of the warp's 32 rows is staged in shared memory (row stride 33 floats:
-    // conflict-free both ways) and written back row-contiguously: 8 lanes cover
-    // one 128-B row segment, so every store instruction moves 4 full lines
-    // instead of 32 scattered 16-B pieces.
-    const int q = warp & 3;
-    float* stg = reinterpret_cast<float*>(tmem_slot + 4) + (warp - 2) * 32 * 33;
-    const int rsub = lane >> 3, cq = (lane & 7) * 4;
+    // ---- epilogue warps 2..9: TMEM lane quarter q = warp % 4 (hardware rule), column
+    // half h: the warp takes every other 16-column chunk.  A chunk of the warp's 32
+    // rows is staged in shared memory (row stride 17 floats: conflict-free writes) and
+    // written back row-contiguously: 4 lanes cover one 64-B row segment, so a store
+    // instruction moves 8 segments instead of 32 scattered 16-B pieces.  Eight
+    // warps keep twice the independent TMEM-load -> store chains in flight.
+    const int q = warp & 3, h = (warp - 2) >> 2;
+    float* stg = reinterpret_cast<float*>(tmem_slot + 4) + (warp - 2) * 32 * 17;
+    const int rsub = lane >> 2, cq = (lane & 3) * 4;
     int acc = 0;
     uint32_t aph = 0;
     for (int64_t t = blockIdx.x; t < ntiles; t += gridDim.x) {
@@ -260,16 +262,11 @@ __global__ void __launch_bounds__(THREADS, 1)
         if (p.out_rank) own = p.out_base[p.out_rank[m_own]] + int64_t(p.out_row[m_own]) * p.y_pitch;
         else own = p.Y + m_own * p.y_pitch;
       }
-      for (int c = 0; c < p.BN; c += 32) {
+      for (int c = 16 * h; c < p.BN; c += 32) {
         uint32_t r[16];
         tmem_ld16(tmem_base + (uint32_t(q * 32) << 16) + uint32_t(acc * p.BN + c), r);
 #pragma unroll
-        for (int j = 0; j < 16; ++j) stg[lane * 33 + j] = __uint_as_float(r[j]);
-        if (c + 16 < p.BN) {
-          tmem_ld16(tmem_base + (uint32_t(q * 32) << 16) + uint32_t(acc * p.BN + c + 16), r);
-#pragma unroll
-          for (int j = 0; j < 16; ++j) stg[lane * 33 + 16 + j] = __uint_as_float(r[j]);
-        }
+        for (int j = 0; j < 16; ++j) stg[lane * 17 + j] = __uint_as_float(r[j]);
         __syncwarp();
         const int col = c + cq;
         float4 bv = make_float4(0.f, 0.f, 0.f, 0.f);
@@ -282,12 +279,12 @@ __global__ void __launch_bounds__(THREADS, 1)
           }
         }
 #pragma unroll
-        for (int it = 0; it < 8; ++it) {
-          const int row = it * 4 + rsub;
+        for (int it = 0; it < 4; ++it) {
+          const int row = it * 8 + rsub;
           float* dst = reinterpret_cast<float*>(__shfl_sync(0xffffffffu, reinterpret_cast<uintptr_t>(own), row));
           if (!dst || col >= p.N) continue;
-          float4 v = make_float4(stg[row * 33 + cq] + bv.x, stg[row * 33 + cq + 1] + bv.y, stg[row * 33 + cq + 2] + bv.z,
-                                 stg[row * 33 + cq + 3] + bv.w);
+          const float* sv = stg + row * 17 + cq;
+          float4 v = make_float4(sv[0] + bv.x, sv[1] + bv.y, sv[2] + bv.z, sv[3] + bv.w);
           if (p.relu) { v.x = fmaxf(v.x, 0.f); v.y = fmaxf(v.y, 0.f); v.z = fmaxf(v.z, 0.f); v.w = fmaxf(v.w, 0.f); }
           if (p.accumulate) {
             if (col + 4 <= p.N) {
@@ -338,7 +335,7 @@ struct WgradParams {
 __global__ void __launch_bounds__(THREADS, 1)
     wgrad_kernel(const __grid_constant__ CUtensorMap mapG, const __grid_constant__ CUtensorMap mapZ, WgradParams p) {
   extern __shared__ __align__(1024) uint8_t smem_raw[];
-  uint8_t* smem = reinterpret_cast<uint8_t*>((reinterpret_cast<uintptr_t>(smem_raw) + 1023) & ~uintptr_t(1023));
+  uint8_t* smem = smem_raw + ((1024u - (smem_u32(smem_raw) & 1023u)) & 1023u);   // 1 KB aligned, still __shared__
   uint64_t* bars = reinterpret_cast<uint64_t*>(smem + size_t(WG_STAGES) * p.stage_bytes);
   uint64_t* full = bars;
   uint64_t* empty = bars + WG_STAGES;
@@ -524,7 +521,7 @@ cudaError_t launch_tc_gemm(const TcGemmArgs& a, cudaStream_t st) {
   RowParams p{a.M_max, a.M_dev, a.N, BN, nkb, cols, a.w_mn, b_kb_bytes, a.bias, a.relu, a.Y, a.y_pitch,
               a.out_base, a.out_rank, a.out_row, a.accumulate};
   const size_t smem = 1024 + size_t(STAGES) * A_STAGE_BYTES + size_t(nkb) * b_kb_bytes + 16 * 8 + 16 +
-                      4 * 32 * 33 * 4;   // + epilogue staging
+                      8 * 32 * 17 * 4;   // + epilogue staging
   if (smem > 227 * 1024) return cudaErrorInvalidValue;
   static bool attr_set = false;
   if (!attr_set) {
@@ -533,7 +530,7 @@ cudaError_t launch_tc_gemm(const TcGemmArgs& a, cudaStream_t st) {
   }
   const int64_t tiles = std::max<int64_t>(1, ceil_div(a.M_max, BM));
   const int grid = int(std::min<int64_t>(tiles, sm_count()));
-  rowtile_kernel<<<grid, THREADS, smem, st>>>(ma, mb, p);
+  rowtile_kernel<<<grid, ROW_THREADS, smem, st>>>(ma, mb, p);
   return cudaGetLastError();
 }
 
