@@ -147,7 +147,7 @@ extern "C" apt_status apt_dryrun(apt_trainer* t, int64_t n_steps, apt_plan_stats
   uint32_t* dst_bm = A.alloc<uint32_t>(n_words, true);
   uint32_t* new_bm = A.alloc<uint32_t>(n_words, true);
   int32_t* pos = A.alloc<int32_t>(g->n, false);
-  int32_t* partials = A.alloc<int32_t>(ceil_div(n_words, 2048) + 4, false);
+  int32_t* partials = A.alloc<int32_t>(2 * ceil_div(n_words, 2048) + 8, false);
   uint64_t* step_dev = A.alloc<uint64_t>(1, true);
   uint32_t* own_bm = A.alloc<uint32_t>(n_words * C, true);        // one bitmap per owner / block
   DryCounters* dc = A.alloc<DryCounters>(4, true);                 // per strategy
@@ -166,7 +166,7 @@ extern "C" apt_status apt_dryrun(apt_trainer* t, int64_t n_steps, apt_plan_stats
       hp.cnt = A.alloc<int32_t>(maxF, true);
       hp.nbr = A.alloc<int32_t>(maxF * hp.k, false);
       hp.counts = A.alloc<int32_t>(4, true);
-      hp.part2 = A.alloc<int32_t>(ceil_div(maxF, 2048) + 4, false);
+      hp.part2 = A.alloc<int32_t>(2 * ceil_div(maxF, 2048) + 8, false);
       if (h + 1 < K) {
         hp.src = A.alloc<int32_t>(hp.max_src, false);
         hp.indptr = A.alloc<int32_t>(maxF + 1, true);
@@ -216,7 +216,7 @@ extern "C" apt_status apt_dryrun(apt_trainer* t, int64_t n_steps, apt_plan_stats
         dry_count_kernel<<<blocks, 256, 0, c->stream>>>(S, r, C, l1.dst, l1.n_dst, l1.cnt, l1.nbr, l1.k, g->part,
                                                         own_bm, n_words, dc + S);
         CK(c, cudaGetLastError());
-        c->launches += 4 + 10 * K;
+        c->launches += 4 + 4 * K;
       }
       dry_fold_kernel<<<1, 64, 0, c->stream>>>(C, dc + S);
       CK(c, cudaGetLastError());

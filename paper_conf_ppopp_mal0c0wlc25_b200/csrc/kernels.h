@@ -181,6 +181,9 @@ cudaError_t launch_colsum(const float* g, int64_t pitch, int dim, const int32_t*
                           cudaStream_t st);
 cudaError_t launch_sgd(float* W, const float* dW, int64_t n, float lr, uint16_t* W_bf16, int rows, int cols,
                        int64_t bf16_pitch, cudaStream_t st);
+struct SgdSeg { float* W; const float* dW; int64_t n; uint16_t* Wb; int cols; int64_t bpitch; };
+struct SgdBatch { SgdSeg seg[16]; int n; };
+cudaError_t launch_sgd_multi(const SgdBatch& b, float lr, cudaStream_t st);
 cudaError_t launch_to_bf16(const float* src, int64_t src_pitch, uint16_t* dst, int64_t dst_pitch, int cols,
                            const int32_t* n_dev, int64_t max_n, cudaStream_t st);
 cudaError_t launch_bf16_pad_ones(const uint16_t* src, int64_t src_pitch, uint16_t* dst, int64_t dst_pitch, int cols,

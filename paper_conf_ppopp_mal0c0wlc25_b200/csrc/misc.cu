@@ -176,6 +176,29 @@ __global__ void sgd_kernel(float* __restrict__ W, const float* __restrict__ dW, 
   }
 }
 
+// All parameter tensors of a step in one launch: blockIdx.y = tensor.
+__global__ void sgd_multi_kernel(SgdBatch b, float lr) {
+  const SgdSeg& g = b.seg[blockIdx.y];
+  for (int64_t t = int64_t(blockIdx.x) * blockDim.x + threadIdx.x; t < g.n; t += int64_t(gridDim.x) * blockDim.x) {
+    const float w = g.W[t] - lr * g.dW[t];
+    g.W[t] = w;
+    if (g.Wb) {
+      const int64_t r = t / g.cols;
+      __nv_bfloat16 h = __float2bfloat16_rn(w);
+      g.Wb[r * g.bpitch + (t - r * g.cols)] = *reinterpret_cast<uint16_t*>(&h);
+    }
+  }
+}
+
+cudaError_t launch_sgd_multi(const SgdBatch& b, float lr, cudaStream_t st) {
+  if (b.n <= 0) return cudaSuccess;
+  int64_t mx = 1;
+  for (int i = 0; i < b.n; ++i) mx = std::max<int64_t>(mx, b.seg[i].n);
+  dim3 grid(unsigned(std::min<int64_t>(ceil_div(mx, 256), 148 * 4)), unsigned(b.n));
+  sgd_multi_kernel<<<grid, 256, 0, st>>>(b, lr);
+  return cudaGetLastError();
+}
+
 cudaError_t launch_sgd(float* W, const float* dW, int64_t n, float lr, uint16_t* W_bf16, int rows, int cols,
                        int64_t bf16_pitch, cudaStream_t st) {
   (void)rows;

@@ -150,140 +150,9 @@ __device__ __forceinline__ T block_exclusive_scan(T v, T* total) {
   return r;
 }
 
-template <class Op>
-__global__ void __launch_bounds__(kScanThreads) scan_partials(Op op, int32_t* partials) {
-  const int64_t n = op.size();
-  const int64_t base = int64_t(blockIdx.x) * kScanTile + int64_t(threadIdx.x) * kScanItems;
-  int32_t s = 0;
-#pragma unroll
-  for (int j = 0; j < kScanItems; ++j)
-    if (base + j < n) s += op.value(base + j);
-  __shared__ int32_t tot;
-  block_exclusive_scan<int32_t>(s, &tot);
-  if (threadIdx.x == 0) partials[blockIdx.x] = tot;
-}
-
-__global__ void __launch_bounds__(1024) scan_spine(int32_t* partials, int nb) {
-  __shared__ int32_t carry_s;
-  __shared__ int32_t wsum[32];
-  if (threadIdx.x == 0) carry_s = 0;
-  __syncthreads();
-  for (int off = 0; off < nb; off += 1024) {
-    const int i = off + threadIdx.x;
-    const int32_t v = i < nb ? partials[i] : 0;
-    const int lane = lane_id(), wid = threadIdx.x >> 5;
-    int32_t incl = v;
-#pragma unroll
-    for (int o = 1; o < 32; o <<= 1) {
-      int32_t n = __shfl_up_sync(0xffffffffu, incl, o);
-      if (lane >= o) incl += n;
-    }
-    if (lane == 31) wsum[wid] = incl;
-    __syncthreads();
-    if (wid == 0) {
-      int32_t w = wsum[lane], wi = w;
-#pragma unroll
-      for (int o = 1; o < 32; o <<= 1) {
-        int32_t n = __shfl_up_sync(0xffffffffu, wi, o);
-        if (lane >= o) wi += n;
-      }
-      wsum[lane] = wi - w;
-    }
-    __syncthreads();
-    const int32_t carry = carry_s;
-    const int32_t excl = carry + wsum[wid] + incl - v;
-    if (i < nb) partials[i] = excl;
-    __syncthreads();
-    if (threadIdx.x == 1023) carry_s = excl + v;
-    __syncthreads();
-  }
-  if (threadIdx.x == 0) partials[nb] = carry_s;   // grand total
-}
-
-template <class Op>
-__global__ void __launch_bounds__(kScanThreads) scan_emit(Op op, const int32_t* partials, int nb) {
-  const int64_t n = op.size();
-  const int64_t base = int64_t(blockIdx.x) * kScanTile + int64_t(threadIdx.x) * kScanItems;
-  int32_t vals[kScanItems];
-  int32_t s = 0;
-#pragma unroll
-  for (int j = 0; j < kScanItems; ++j) {
-    vals[j] = (base + j < n) ? op.value(base + j) : 0;
-    s += vals[j];
-  }
-  __shared__ int32_t tot;
-  int32_t excl = block_exclusive_scan<int32_t>(s, &tot) + partials[blockIdx.x];
-#pragma unroll
-  for (int j = 0; j < kScanItems; ++j) {
-    if (base + j < n) op.emit(base + j, excl, vals[j]);
-    excl += vals[j];
-  }
-  if (blockIdx.x == 0 && threadIdx.x == 0) op.finish(partials[nb]);
-}
-
-template <class Op>
-static cudaError_t run_scan(const Op& op, int64_t max_n, int32_t* partials, cudaStream_t st) {
-  const int nb = int(std::max<int64_t>(1, ceil_div(max_n, kScanTile)));
-  scan_partials<Op><<<nb, kScanThreads, 0, st>>>(op, partials);
-  scan_spine<<<1, 1024, 0, st>>>(partials, nb);
-  scan_emit<Op><<<nb, kScanThreads, 0, st>>>(op, partials, nb);
-  return cudaGetLastError();
-}
-
 // --------------------------------------------------------- compaction ----
 // S3 / reading O3: src = dst ++ ascending(unique(nbrs) \ dst); indptr = scan(cnt);
 // indices[e] = position of nbr[e] in src.
-
-__global__ void mark_dst_kernel(const int32_t* __restrict__ dst, const int32_t* __restrict__ n_dst,
-                                uint32_t* __restrict__ dst_bm, int32_t* __restrict__ pos) {
-  const int64_t F = *n_dst;
-  for (int64_t i = int64_t(blockIdx.x) * blockDim.x + threadIdx.x; i < F; i += int64_t(gridDim.x) * blockDim.x) {
-    const int v = dst[i];
-    atomicOr(dst_bm + (v >> 5), 1u << (v & 31));
-    pos[v] = int32_t(i);
-  }
-}
-
-__global__ void mark_new_kernel(const int32_t* __restrict__ cnt, const int32_t* __restrict__ nbr,
-                                const int32_t* __restrict__ n_dst, int k,
-                                const uint32_t* __restrict__ dst_bm, uint32_t* __restrict__ new_bm) {
-  const int64_t slots = int64_t(*n_dst) * k;
-  for (int64_t s = int64_t(blockIdx.x) * blockDim.x + threadIdx.x; s < slots; s += int64_t(gridDim.x) * blockDim.x) {
-    const int64_t i = s / k;
-    const int q = int(s - i * k);
-    if (q >= cnt[i]) continue;
-    const int u = nbr[s];
-    const uint32_t bit = 1u << (u & 31);
-    if (dst_bm[u >> 5] & bit) continue;
-    if (!(__ldcg(new_bm + (u >> 5)) & bit)) atomicOr(new_bm + (u >> 5), bit);
-  }
-}
-
-struct BitmapScanOp {
-  uint32_t* new_bm;
-  int64_t n_words;
-  const int32_t* n_dst;
-  int32_t* src;
-  int32_t* pos;
-  int32_t* n_src;
-  __device__ int64_t size() const { return n_words; }
-  __device__ int32_t value(int64_t w) const { return __popc(new_bm[w]); }
-  __device__ void emit(int64_t w, int32_t excl, int32_t val) const {
-    if (!val) return;
-    uint32_t word = new_bm[w];
-    int32_t idx = *n_dst + excl;
-    while (word) {
-      const int b = __ffs(word) - 1;
-      word &= word - 1;
-      const int u = int(w * 32 + b);
-      src[idx] = u;
-      pos[u] = idx;
-      ++idx;
-    }
-    new_bm[w] = 0u;   // leave the bitmap clean for the next hop
-  }
-  __device__ void finish(int32_t total) const { *n_src = *n_dst + total; }
-};
 
 struct CntScanOp {
   const int32_t* cnt;
@@ -321,20 +190,150 @@ static int64_t grid_for(int64_t n, int threads) {
   return std::max<int64_t>(1, std::min<int64_t>(ceil_div(n, threads), 148 * 32));
 }
 
+// Fused compaction, three launches per hop:
+//  1. mark: dst bits + pos[dst] + the dst prefix of src, every sampled neighbour's bit
+//     (no exclusion yet: a block cannot know the dst bitmap is complete), clears the
+//     scan state of step 2;
+//  2. one single-pass scan (decoupled look-back; tickets give blocks their order) over
+//     two domains at once: the words of (new & ~dst) -> ascending new ids, their
+//     positions and n_src; the counts -> indptr and n_edges;
+//  3. map_indices (above): indices[e] = pos[nbr[e]], and the dst bits are cleared.
+__global__ void compact_mark_kernel(const int32_t* __restrict__ dst, const int32_t* __restrict__ n_dst,
+                                    const int32_t* __restrict__ cnt, const int32_t* __restrict__ nbr, int k,
+                                    uint32_t* __restrict__ dst_bm, uint32_t* __restrict__ new_bm,
+                                    int32_t* __restrict__ pos, int32_t* __restrict__ src, uint64_t* __restrict__ stA,
+                                    int nbA, uint64_t* __restrict__ stB, int nbB, int32_t* __restrict__ ticket) {
+  const int64_t F = *n_dst;
+  const int64_t tid = int64_t(blockIdx.x) * blockDim.x + threadIdx.x, nth = int64_t(gridDim.x) * blockDim.x;
+  for (int64_t i = tid; i < nbA + nbB + 1; i += nth) {
+    if (i < nbA) stA[i] = 0;
+    else if (i < nbA + nbB) stB[i - nbA] = 0;
+    else *ticket = 0;
+  }
+  for (int64_t i = tid; i < F; i += nth) {
+    const int v = dst[i];
+    atomicOr(dst_bm + (v >> 5), 1u << (v & 31));
+    pos[v] = int32_t(i);
+    src[i] = v;
+  }
+  const int64_t slots = F * k;
+  for (int64_t s = tid; s < slots; s += nth) {
+    const int64_t i = s / k;
+    const int q = int(s - i * k);
+    if (q >= cnt[i]) continue;
+    const int u = nbr[s];
+    const uint32_t bit = 1u << (u & 31);
+    if (!(__ldcg(new_bm + (u >> 5)) & bit)) atomicOr(new_bm + (u >> 5), bit);
+  }
+}
+
+__device__ __forceinline__ void st_release_gpu(uint64_t* p, uint64_t v) {
+  asm volatile("st.release.gpu.global.u64 [%0], %1;" ::"l"(p), "l"(v) : "memory");
+}
+__device__ __forceinline__ uint64_t ld_acquire_gpu(const uint64_t* p) {
+  uint64_t v;
+  asm volatile("ld.acquire.gpu.global.u64 %0, [%1];" : "=l"(v) : "l"(p) : "memory");
+  return v;
+}
+
+// Decoupled look-back for block `b` of a chain: publishes the block aggregate, walks
+// predecessors until an inclusive prefix, publishes its own.  Thread 0 only.
+__device__ int32_t chain_prefix(uint64_t* st, int b, int32_t agg) {
+  constexpr uint64_t kAgg = 1ull << 32, kIncl = 2ull << 32;
+  if (b == 0) {
+    st_release_gpu(st, kIncl | uint32_t(agg));
+    return 0;
+  }
+  st_release_gpu(st + b, kAgg | uint32_t(agg));
+  int32_t excl = 0;
+  for (int j = b - 1;;) {
+    const uint64_t w = ld_acquire_gpu(st + j);
+    const uint64_t flag = w & (3ull << 32);
+    if (!flag) continue;
+    excl += int32_t(uint32_t(w));
+    if (flag == kIncl) break;
+    --j;
+  }
+  st_release_gpu(st + b, kIncl | uint32_t(excl + agg));
+  return excl;
+}
+
+template <class Op>
+__device__ void scan_tile(const Op& op, uint64_t* st, int b, int nb) {
+  const int64_t n = op.size();
+  const int64_t base = int64_t(b) * kScanTile + int64_t(threadIdx.x) * kScanItems;
+  int32_t vals[kScanItems];
+  int32_t s = 0;
+#pragma unroll
+  for (int j = 0; j < kScanItems; ++j) {
+    vals[j] = (base + j < n) ? op.value(base + j) : 0;
+    s += vals[j];
+  }
+  __shared__ int32_t tot, prefix;
+  int32_t excl = block_exclusive_scan<int32_t>(s, &tot);
+  if (threadIdx.x == 0) {
+    prefix = chain_prefix(st, b, tot);
+    if (b == nb - 1) op.finish(prefix + tot);
+  }
+  __syncthreads();
+  excl += prefix;
+#pragma unroll
+  for (int j = 0; j < kScanItems; ++j) {
+    if (base + j < n) op.emit(base + j, excl, vals[j]);
+    excl += vals[j];
+  }
+}
+
+struct NewBitsOp {   // words of (new & ~dst): ascending new source ids
+  uint32_t* new_bm;
+  const uint32_t* dst_bm;
+  int64_t n_words;
+  const int32_t* n_dst;
+  int32_t* src;
+  int32_t* pos;
+  int32_t* n_src;
+  __device__ int64_t size() const { return n_words; }
+  __device__ int32_t value(int64_t w) const { return __popc(new_bm[w] & ~dst_bm[w]); }
+  __device__ void emit(int64_t w, int32_t excl, int32_t val) const {
+    uint32_t word = new_bm[w];
+    if (!word) return;
+    new_bm[w] = 0u;   // leave the bitmap clean for the next hop
+    word &= ~dst_bm[w];
+    int32_t idx = *n_dst + excl;
+    while (word) {
+      const int b = __ffs(word) - 1;
+      word &= word - 1;
+      const int u = int(w * 32 + b);
+      src[idx] = u;
+      pos[u] = idx;
+      ++idx;
+    }
+  }
+  __device__ void finish(int32_t total) const { *n_src = *n_dst + total; }
+};
+
+__global__ void __launch_bounds__(kScanThreads) compact_scan_kernel(NewBitsOp a, uint64_t* stA, int nbA, CntScanOp c,
+                                                                    uint64_t* stB, int nbB, int32_t* ticket) {
+  __shared__ int32_t tk;
+  if (threadIdx.x == 0) tk = atomicAdd(ticket, 1);
+  __syncthreads();
+  const int t = tk;
+  if (t < nbA) scan_tile(a, stA, t, nbA);
+  else scan_tile(c, stB, t - nbA, nbB);
+}
+
 cudaError_t launch_compact(const CompactArgs& a, cudaStream_t st) {
   const int T = 256;
-  mark_dst_kernel<<<grid_for(a.max_dst, T), T, 0, st>>>(a.dst, a.n_dst, a.dst_bm, a.pos);
-  mark_new_kernel<<<grid_for(a.max_dst * a.k, T), T, 0, st>>>(a.cnt, a.nbr, a.n_dst, a.k, a.dst_bm, a.new_bm);
-  // src ids are written after the dst prefix by the bitmap scan; the prefix
-  // itself is a copy of dst (the frontier).
-  cudaError_t e = cudaMemcpyAsync(a.src, a.dst, sizeof(int32_t) * size_t(a.max_dst), cudaMemcpyDeviceToDevice, st);
-  if (e != cudaSuccess) return e;
-  BitmapScanOp bop{a.new_bm, a.n_words, a.n_dst, a.src, a.pos, a.n_src};
-  e = run_scan(bop, a.n_words, a.partials, st);
-  if (e != cudaSuccess) return e;
+  const int nbA = int(std::max<int64_t>(1, ceil_div(a.n_words, kScanTile)));
+  const int nbB = int(std::max<int64_t>(1, ceil_div(a.max_dst, kScanTile)));
+  uint64_t* stA = reinterpret_cast<uint64_t*>(a.partials);            // >= 2*nbA + 8 int32
+  int32_t* ticket = a.partials + 2 * nbA + 2;
+  uint64_t* stB = reinterpret_cast<uint64_t*>(a.partials2);           // >= 2*nbB + 8 int32
+  compact_mark_kernel<<<grid_for(a.max_dst * a.k, T), T, 0, st>>>(a.dst, a.n_dst, a.cnt, a.nbr, a.k, a.dst_bm,
+                                                                   a.new_bm, a.pos, a.src, stA, nbA, stB, nbB, ticket);
+  NewBitsOp bop{a.new_bm, a.dst_bm, a.n_words, a.n_dst, a.src, a.pos, a.n_src};
   CntScanOp cop{a.cnt, a.n_dst, a.indptr, a.n_edges};
-  e = run_scan(cop, a.max_dst, a.partials2, st);
-  if (e != cudaSuccess) return e;
+  compact_scan_kernel<<<nbA + nbB, kScanThreads, 0, st>>>(bop, stA, nbA, cop, stB, nbB, ticket);
   map_indices_kernel<<<grid_for(a.max_dst * a.k, T), T, 0, st>>>(a.dst, a.cnt, a.nbr, a.n_dst, a.k, a.indptr,
                                                                   a.pos, a.indices, a.dst_bm);
   return cudaGetLastError();

@@ -182,7 +182,7 @@ apt_status apt_trainer_create(apt_ctx* c, const apt_graph* g, const apt_fstore* 
     rs.dst_bm = A.alloc<uint32_t>(n_words, true);
     rs.new_bm = A.alloc<uint32_t>(n_words, true);
     rs.pos = A.alloc<int32_t>(g->n, false);
-    rs.partials = A.alloc<int32_t>(ceil_div(n_words, 2048) + 4, false);
+    rs.partials = A.alloc<int32_t>(2 * ceil_div(n_words, 2048) + 8, false);
     rs.hops.resize(K);
     int64_t maxF = B0;
     const int32_t* dst = rs.seeds;
@@ -197,7 +197,7 @@ apt_status apt_trainer_create(apt_ctx* c, const apt_graph* g, const apt_fstore* 
       hp.cnt = A.alloc<int32_t>(maxF, true);
       hp.nbr = A.alloc<int32_t>(maxF * hp.k, false);
       hp.counts = A.alloc<int32_t>(4, true);
-      hp.part2 = A.alloc<int32_t>(ceil_div(maxF, 2048) + 4, false);
+      hp.part2 = A.alloc<int32_t>(2 * ceil_div(maxF, 2048) + 8, false);
       if (h + 1 < K) {   // the layer-1 hop is consumed in ELL form (fused gather), no CSR needed
         hp.src = A.alloc<int32_t>(hp.max_src, false);
         hp.indptr = A.alloc<int32_t>(maxF + 1, true);
@@ -393,7 +393,7 @@ apt_status phase_sample(apt_trainer* t, RankState& rs, bool from_host_batch) {
       CompactArgs ca{hp.dst, hp.n_dst, hp.max_dst, hp.cnt, hp.nbr, hp.k, rs.dst_bm, rs.new_bm, n_words, rs.pos, hp.src,
                      hp.counts, hp.indptr, hp.indices, hp.counts + 1, rs.partials, hp.part2};
       CK(c, launch_compact(ca, c->stream));
-      c->launches += 9;
+      c->launches += 3;
     }
   }
   return APT_OK;
@@ -518,23 +518,33 @@ apt_status allreduce_sgd(apt_trainer* t, int update) {
     if (s != APT_OK) return s;
   }
   if (!update) return APT_OK;
-  for (auto& rs : t->R) {
-    if (rs.x.W1s && rs.x.w_cols > 0) {   // NFP: each rank updates only its column slice of W^1
-      const Layer& L = rs.L[0];
-      CK(c, launch_sgd(rs.x.W1s, rs.x.dW1s, int64_t(L.d_out) * rs.x.w_cols, t->m.lr, rs.x.Wb1s, L.d_out, rs.x.w_cols,
-                       rs.x.ws_pitch, c->stream));
+  // one launch per 16 parameter tensors (all layers, all hosted ranks)
+  SgdBatch bt{};
+  auto add = [&](float* W, const float* dW, int64_t n, uint16_t* Wb, int cols, int64_t bp) -> apt_status {
+    bt.seg[bt.n++] = SgdSeg{W, dW, n, Wb, cols, bp};
+    if (bt.n == 16) {
+      CK(c, launch_sgd_multi(bt, t->m.lr, c->stream));
       c->launches++;
+      bt.n = 0;
     }
+    return APT_OK;
+  };
+  for (auto& rs : t->R) {
     for (auto& L : rs.L) {
-      if (&L == &rs.L[0] && rs.x.W1s) {
-        CK(c, launch_sgd(L.b, L.db, L.d_out, t->m.lr, nullptr, 1, L.d_out, 0, c->stream));
-        c->launches++;
-        continue;
+      apt_status st;
+      if (&L == &rs.L[0] && rs.x.W1s) {   // NFP: each rank updates only its column slice of W^1
+        if (rs.x.w_cols > 0 && (st = add(rs.x.W1s, rs.x.dW1s, int64_t(L.d_out) * rs.x.w_cols, rs.x.Wb1s, rs.x.w_cols,
+                                         rs.x.ws_pitch)) != APT_OK)
+          return st;
+      } else if ((st = add(L.W, L.dW, int64_t(L.d_out) * L.d_in, L.Wb, L.d_in, L.wb_pitch)) != APT_OK) {
+        return st;
       }
-      CK(c, launch_sgd(L.W, L.dW, int64_t(L.d_out) * L.d_in, t->m.lr, L.Wb, L.d_out, L.d_in, L.wb_pitch, c->stream));
-      CK(c, launch_sgd(L.b, L.db, L.d_out, t->m.lr, nullptr, 1, L.d_out, 0, c->stream));
-      c->launches += 2;
+      if ((st = add(L.b, L.db, L.d_out, nullptr, 1, 0)) != APT_OK) return st;
     }
+  }
+  if (bt.n) {
+    CK(c, launch_sgd_multi(bt, t->m.lr, c->stream));
+    c->launches++;
   }
   return APT_OK;
 }
