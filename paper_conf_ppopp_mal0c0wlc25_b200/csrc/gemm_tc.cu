@@ -148,6 +148,7 @@ struct RowParams {
   const int32_t* out_rank;
   const int32_t* out_row;
   int accumulate;
+  int n_split;              // CTAs share an M tile: CTA b computes columns [(b % n_split) * BN, +BN)
 };
 
 __global__ void __launch_bounds__(ROW_THREADS, 1)
@@ -167,6 +168,8 @@ __global__ void __launch_bounds__(ROW_THREADS, 1)
   const int warp = threadIdx.x >> 5, lane = lane_id();
   const int64_t M = std::min<int64_t>(p.M_max, int64_t(*p.M_dev));
   const int64_t ntiles = ceil_div(M, BM);
+  const int n0 = int(blockIdx.x % p.n_split) * p.BN;              // this CTA's column slice
+  const int64_t t0 = blockIdx.x / p.n_split, tstride = gridDim.x / p.n_split;
 
   if (warp == 0 && lane == 0) {
     for (int s = 0; s < STAGES; ++s) { mbar_init(full + s, 1); mbar_init(empty + s, 1); }
@@ -183,21 +186,21 @@ __global__ void __launch_bounds__(ROW_THREADS, 1)
   const uint32_t tmem_base = *tmem_slot;
 
   if (warp == 0) {
-    if (lane == 0 && ntiles > int64_t(blockIdx.x)) {
-      // ---- TMA producer: resident B, then the A ring
+    if (lane == 0 && ntiles > t0) {
+      // ---- TMA producer: resident B (this CTA's column slice), then the A ring
       mbar_expect_tx(bfull, uint32_t(p.nkb) * p.b_kb_bytes);
       const int nb = int(ceil_div(p.BN, 64));
       for (int kb = 0; kb < p.nkb; ++kb) {
         uint8_t* dst = smem_b + size_t(kb) * p.b_kb_bytes;
         if (p.b_mn) {
-          for (int j = 0; j < nb; ++j) tma_load_2d(dst + j * MNBLK, &mapB, bfull, j * 64, kb * BK);
+          for (int j = 0; j < nb; ++j) tma_load_2d(dst + j * MNBLK, &mapB, bfull, n0 + j * 64, kb * BK);
         } else {
-          tma_load_2d(dst, &mapB, bfull, kb * BK, 0);
+          tma_load_2d(dst, &mapB, bfull, kb * BK, n0);
         }
       }
       int s = 0;
       uint32_t ph = 0;
-      for (int64_t t = blockIdx.x; t < ntiles; t += gridDim.x) {
+      for (int64_t t = t0; t < ntiles; t += tstride) {
         for (int kb = 0; kb < p.nkb; ++kb) {
           mbar_wait(empty + s, ph ^ 1);
           mbar_expect_tx(full + s, A_STAGE_BYTES);
@@ -208,7 +211,7 @@ __global__ void __launch_bounds__(ROW_THREADS, 1)
     }
   } else if (warp == 1) {
     // ---- MMA issuer (one thread)
-    if (ntiles > int64_t(blockIdx.x)) {
+    if (ntiles > t0) {
       const uint32_t idesc = idesc_bf16(BM, p.BN, 0, p.b_mn);
       mbar_wait(bfull, 0);
       fence_after();
@@ -216,7 +219,7 @@ __global__ void __launch_bounds__(ROW_THREADS, 1)
       uint32_t ph = 0;
       int acc = 0;
       uint32_t aph = 0;
-      for (int64_t t = blockIdx.x; t < ntiles; t += gridDim.x) {
+      for (int64_t t = t0; t < ntiles; t += tstride) {
         mbar_wait(tempty + acc, aph ^ 1);
         fence_after();
         const uint32_t d = tmem_base + uint32_t(acc * p.BN);
@@ -252,7 +255,7 @@ __global__ void __launch_bounds__(ROW_THREADS, 1)
     const int rsub = lane >> 2, cq = (lane & 3) * 4;
     int acc = 0;
     uint32_t aph = 0;
-    for (int64_t t = blockIdx.x; t < ntiles; t += gridDim.x) {
+    for (int64_t t = t0; t < ntiles; t += tstride) {
       mbar_wait(tfull + acc, aph);
       fence_after();
       // own row (= TMEM lane) destination; shuffled to the lanes that store it
@@ -268,7 +271,7 @@ __global__ void __launch_bounds__(ROW_THREADS, 1)
 #pragma unroll
         for (int j = 0; j < 16; ++j) stg[lane * 17 + j] = __uint_as_float(r[j]);
         __syncwarp();
-        const int col = c + cq;
+        const int col = n0 + c + cq;
         float4 bv = make_float4(0.f, 0.f, 0.f, 0.f);
         if (p.bias) {
           if (col + 4 <= p.N) bv = *reinterpret_cast<const float4*>(p.bias + col);
@@ -503,8 +506,14 @@ cudaError_t launch_tc_gemm(const TcGemmArgs& a, cudaStream_t st) {
   using namespace tc;
   if (!tc_gemm_supported(a.N, a.K)) return cudaErrorInvalidValue;
   if ((a.z_pitch * 2) % 16 || (a.w_pitch * 2) % 16 || (a.y_pitch * 4) % 16) return cudaErrorInvalidValue;
-  const int BN = int(round_up(a.N, 16));
+  const int BN_all = int(round_up(a.N, 16));
   const int nkb = int(ceil_div(a.K, BK));
+  // few M tiles (small blocks, a requester's own rows): split the columns over CTAs so
+  // that more SMs share the tile's epilogue; slices stay multiples of 64 columns
+  const int64_t tiles = std::max<int64_t>(1, ceil_div(a.M_max, BM));
+  int n_split = 1;
+  while (n_split < 4 && tiles * n_split * 2 <= sm_count() && BN_all % (64 * n_split * 2) == 0) n_split *= 2;
+  const int BN = BN_all / n_split;
   int cols = 32;
   while (cols < 2 * BN) cols <<= 1;
   CUtensorMap ma, mb;
@@ -519,7 +528,7 @@ cudaError_t launch_tc_gemm(const TcGemmArgs& a, cudaStream_t st) {
     b_kb_bytes = uint32_t(BN) * 128;
   }
   RowParams p{a.M_max, a.M_dev, a.N, BN, nkb, cols, a.w_mn, b_kb_bytes, a.bias, a.relu, a.Y, a.y_pitch,
-              a.out_base, a.out_rank, a.out_row, a.accumulate};
+              a.out_base, a.out_rank, a.out_row, a.accumulate, n_split};
   const size_t smem = 1024 + size_t(STAGES) * A_STAGE_BYTES + size_t(nkb) * b_kb_bytes + 16 * 8 + 16 +
                       8 * 32 * 17 * 4;   // + epilogue staging
   if (smem > 227 * 1024) return cudaErrorInvalidValue;
@@ -528,8 +537,7 @@ cudaError_t launch_tc_gemm(const TcGemmArgs& a, cudaStream_t st) {
     cudaFuncSetAttribute(rowtile_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize, 227 * 1024);
     attr_set = true;
   }
-  const int64_t tiles = std::max<int64_t>(1, ceil_div(a.M_max, BM));
-  const int grid = int(std::min<int64_t>(tiles, sm_count()));
+  const int grid = int(std::min<int64_t>(tiles * n_split, (sm_count() / n_split) * n_split));
   rowtile_kernel<<<grid, ROW_THREADS, smem, st>>>(ma, mb, p);
   return cudaGetLastError();
 }

@@ -31,6 +31,9 @@ void release_exported(apt_ctx* c);
 static void ctx_free(apt_ctx* c) {
   cudaStreamSynchronize(c->stream);
   release_exported(c);
+  if (c->side) { cudaStreamSynchronize(c->side); cudaStreamDestroy(c->side); }
+  if (c->ev_fork) cudaEventDestroy(c->ev_fork);
+  if (c->ev_join) cudaEventDestroy(c->ev_join);
   c->arena.release();
   if (c->own_stream) cudaStreamDestroy(c->stream);
   delete c;
@@ -84,6 +87,9 @@ apt_status apt_ctx_create(int rank, int world, int device, void* stream, apt_ctx
     cudaStreamCreateWithFlags(&c->stream, cudaStreamNonBlocking);
     c->own_stream = true;
   }
+  cudaStreamCreateWithFlags(&c->side, cudaStreamNonBlocking);
+  cudaEventCreateWithFlags(&c->ev_fork, cudaEventDisableTiming);
+  cudaEventCreateWithFlags(&c->ev_join, cudaEventDisableTiming);
   c->dev_err = c->arena.alloc<uint32_t>(4);
   c->scratch = c->arena.alloc<int32_t>(16);
   if (!c->dev_err || !c->scratch) {

@@ -71,6 +71,8 @@ struct apt_ctx {
   int sm_count = 148;
   cudaStream_t stream = nullptr;
   bool own_stream = false;
+  cudaStream_t side = nullptr;           // forked branch of a step (weight gradients off the critical path)
+  cudaEvent_t ev_fork = nullptr, ev_join = nullptr;
   bool broken = false;
   std::string err;
   int64_t launches = 0;

@@ -115,13 +115,14 @@ apt_status project(apt_trainer* t, const Layer& L, const void* Zb, const float* 
 // dW (+)= G^T Z over the device-counted rows; db += colsum(G)
 apt_status weight_grad(apt_trainer* t, const Layer& L, const float* G, int64_t g_pitch, const void* Z, bool z_bf16,
                        int64_t z_pitch, const int32_t* n_rows, int64_t max_rows, int d_in, float* dW, float* db,
-                       int64_t dW_ld) {
+                       int64_t dW_ld, cudaStream_t st = nullptr) {
   apt_ctx* c = t->ctx;
+  if (!st) st = c->stream;
   if (z_bf16 && L.Gb && tc_wgrad_supported(L.d_out, d_in)) {
     // tcgen05: dW = Gb^T Zb with db from Z's all-ones column d_in
     TcWgradArgs w{L.Gb, L.gb_pitch, static_cast<const uint16_t*>(Z), z_pitch, n_rows, max_rows, L.d_out, d_in,
                   dW, db};
-    CK(c, launch_tc_wgrad(w, c->stream));
+    CK(c, launch_tc_wgrad(w, st));
     c->launches++;
     return APT_OK;
   }
@@ -130,8 +131,8 @@ apt_status weight_grad(apt_trainer* t, const Layer& L, const float* G, int64_t g
   a.B = Z; a.b_t = z_bf16 ? kBF16 : kF32; a.sbk = z_pitch; a.sbn = 1;
   a.C = dW; a.ldc = dW_ld; a.M = L.d_out; a.N = d_in; a.K = max_rows; a.K_dev = n_rows;
   a.accumulate = 1; a.k_chunk = 2048;
-  CK(c, launch_simt_gemm(a, c->stream));
-  if (db) CK(c, launch_colsum(G, g_pitch, L.d_out, n_rows, max_rows, db, c->stream));
+  CK(c, launch_simt_gemm(a, st));
+  if (db) CK(c, launch_colsum(G, g_pitch, L.d_out, n_rows, max_rows, db, st));
   c->launches += db ? 2 : 1;
   return APT_OK;
 }
@@ -452,8 +453,12 @@ apt_status upper_bwd(apt_trainer* t, RankState& rs) {
     Layer& L = rs.L[l - 1];
     Layer& P = rs.L[l - 2];
     const Hop& hp = rs.hops[t->K - l];
+    // dW_l = G_l^T Z_l is independent of the input-gradient chain: fork it onto the
+    // side stream (a parallel branch of the step's graph), joined before the all-reduce
+    CK(c, cudaEventRecord(c->ev_fork, c->stream));
+    CK(c, cudaStreamWaitEvent(c->side, c->ev_fork, 0));
     apt_status s = weight_grad(t, L, L.G, L.h_pitch, bf ? static_cast<const void*>(L.Zb) : L.Zf, bf,
-                               bf ? L.zb_pitch : L.zf_pitch, L.n_rows, L.max_rows, L.d_in, L.dW, L.db, L.d_in);
+                               bf ? L.zb_pitch : L.zf_pitch, L.n_rows, L.max_rows, L.d_in, L.dW, L.db, L.d_in, c->side);
     if (s != APT_OK) return s;
     // dZ = G W  (bf16 mode: tcgen05 with the bf16 weights of the forward, W read N-major as stored)
     if (bf && tc_gemm_supported(L.d_in, L.d_out)) {
@@ -593,6 +598,10 @@ apt_status step_body(apt_trainer* t, int update, bool host_batch) {
   } else {
     apt_status s = layer1_bwd_strategy(t);
     if (s != APT_OK) return s;
+  }
+  if (t->K > 1) {   // join the weight-gradient branch forked in upper_bwd
+    CK(c, cudaEventRecord(c->ev_join, c->side));
+    CK(c, cudaStreamWaitEvent(c->stream, c->ev_join, 0));
   }
   CK(c, record_ev(t, 4));
   apt_status s = allreduce_sgd(t, update);
