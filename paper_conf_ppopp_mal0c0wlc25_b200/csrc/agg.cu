@@ -66,6 +66,7 @@ struct CsrSrc {                  // upper layers: block CSR over the previous la
 // Sum in fp32 (exact under O4), IEEE RN division by the sampled degree (O5).
 template <int EPV, int VPL, int LG, class Src>
 __global__ void __launch_bounds__(256) agg_kernel(AggArgs a, Src src) {
+  APT_PDL_PROLOGUE();
   const int lane = lane_id();
   const int sub = LG == 16 ? (lane >> 4) : 0;
   const int l = LG == 16 ? (lane & 15) : lane;
@@ -166,10 +167,10 @@ static cudaError_t dispatch_agg(const AggArgs& a, const Src& s, cudaStream_t st)
   const int rpw = V <= 16 ? 2 : 1;
   int64_t blocks = ceil_div(ceil_div(a.max_dst, rpw) * 32, threads);
   blocks = std::max<int64_t>(1, std::min<int64_t>(blocks, 148 * 16));
-  if (V <= 16) agg_kernel<EPV, 1, 16, Src><<<blocks, threads, 0, st>>>(a, s);
-  else if (V <= 32) agg_kernel<EPV, 1, 32, Src><<<blocks, threads, 0, st>>>(a, s);
-  else if (V <= 64) agg_kernel<EPV, 2, 32, Src><<<blocks, threads, 0, st>>>(a, s);
-  else if (V <= 128) agg_kernel<EPV, 4, 32, Src><<<blocks, threads, 0, st>>>(a, s);
+  if (V <= 16) launch_pdl(agg_kernel<EPV, 1, 16, Src>, dim3(blocks), dim3(threads), 0, st, a, s);
+  else if (V <= 32) launch_pdl(agg_kernel<EPV, 1, 32, Src>, dim3(blocks), dim3(threads), 0, st, a, s);
+  else if (V <= 64) launch_pdl(agg_kernel<EPV, 2, 32, Src>, dim3(blocks), dim3(threads), 0, st, a, s);
+  else if (V <= 128) launch_pdl(agg_kernel<EPV, 4, 32, Src>, dim3(blocks), dim3(threads), 0, st, a, s);
   else return cudaErrorInvalidValue;
   return cudaGetLastError();
 }
@@ -194,6 +195,7 @@ __global__ void __launch_bounds__(256) agg_bwd_kernel(const int32_t* __restrict_
                                                       const int32_t* __restrict__ n_dst_p, const float* __restrict__ dz,
                                                       int64_t dz_pitch, int dim, float* __restrict__ dx,
                                                       int64_t dx_pitch) {
+  APT_PDL_PROLOGUE();
   const int lane = lane_id();
   const int64_t n_dst = *n_dst_p;
   const int V = int(ceil_div(dim, 4));
@@ -213,13 +215,14 @@ __global__ void __launch_bounds__(256) agg_bwd_kernel(const int32_t* __restrict_
 cudaError_t launch_agg_bwd(const int32_t* indptr, const int32_t* indices, const int32_t* n_dst, int64_t max_dst,
                            const float* dz, int64_t dz_pitch, int dim, float* dx, int64_t dx_pitch, cudaStream_t st) {
   int64_t blocks = std::max<int64_t>(1, std::min<int64_t>(ceil_div(max_dst * 32, 256), 148 * 16));
-  agg_bwd_kernel<<<blocks, 256, 0, st>>>(indptr, indices, n_dst, dz, dz_pitch, dim, dx, dx_pitch);
+  launch_pdl(agg_bwd_kernel, dim3(blocks), dim3(256), 0, st, indptr, indices, n_dst, dz, dz_pitch, dim, dx, dx_pitch);
   return cudaGetLastError();
 }
 
 // ---------------------------------------------------------------- gather
 __global__ void gather_kernel(FeatView fv, const int32_t* __restrict__ ids, const int32_t* __restrict__ n_p,
                               int64_t n_static, char* __restrict__ out, int64_t out_pitch_bytes) {
+  APT_PDL_PROLOGUE();
   const int64_t n = n_p ? int64_t(*n_p) : n_static;
   const int esz = fv.dtype == kBF16 ? 2 : 4;
   const int V = int(ceil_div(int64_t(fv.dim) * esz, 16));
@@ -238,7 +241,7 @@ cudaError_t launch_gather(const FeatView& fv, const int32_t* ids, const int32_t*
                           int64_t out_pitch, cudaStream_t st) {
   int64_t blocks = std::max<int64_t>(1, std::min<int64_t>(ceil_div(max_n * 32, 256), 148 * 16));
   const int esz = fv.dtype == kBF16 ? 2 : 4;
-  gather_kernel<<<blocks, 256, 0, st>>>(fv, ids, n_dev, max_n, reinterpret_cast<char*>(out), out_pitch * esz);
+  launch_pdl(gather_kernel, dim3(blocks), dim3(256), 0, st, fv, ids, n_dev, max_n, reinterpret_cast<char*>(out), out_pitch * esz);
   return cudaGetLastError();
 }
 

@@ -95,6 +95,7 @@ __device__ __forceinline__ uint64_t globaltimer() {
 
 __global__ void barrier_kernel(uint64_t* const* flags, uint64_t* my_flags, uint64_t* epoch, int rank, int C,
                                uint32_t* err) {
+  APT_PDL_PROLOGUE();
   if (threadIdx.x != 0) return;
   const uint64_t e = *epoch + 1;
   *epoch = e;
@@ -132,7 +133,7 @@ apt_status barrier_setup(apt_ctx* c) {
 apt_status device_barrier(apt_ctx* c) {
   if (!multiprocess(c)) return APT_OK;
   if (!c->bar_tab) return set_err(c, APT_E_STATE, "device_barrier: barrier not set up");
-  barrier_kernel<<<1, 32, 0, c->stream>>>(c->bar_tab, c->bar_flags, c->bar_flags + APT_MAX_RANKS, c->rank, c->world,
+  launch_pdl(barrier_kernel, dim3(1), dim3(32), 0, c->stream, c->bar_tab, c->bar_flags, c->bar_flags + APT_MAX_RANKS, c->rank, c->world,
                                           c->dev_err);
   c->launches++;
   return check_cuda(c, cudaGetLastError(), "barrier_kernel");

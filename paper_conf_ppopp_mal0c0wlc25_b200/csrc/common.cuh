@@ -57,6 +57,33 @@ __host__ __device__ __forceinline__ float feature_value(uint2 key, int64_t u, in
   return float(b) * (1.0f / 64.0f);
 }
 
+// ------------------------------------------------- programmatic launches ----
+// Every kernel of the step is launched with programmatic stream serialization:
+// the next kernel's CTAs are scheduled while the previous kernel drains, and each
+// kernel waits (griddepcontrol.wait = all predecessor grids complete and their
+// memory visible) before touching anything, then immediately allows its own
+// dependents to launch.  In a CUDA graph these become programmatic edges, which
+// hides most of the per-kernel launch latency of a ~40-kernel step.
+__device__ __forceinline__ void pdl_wait() { asm volatile("griddepcontrol.wait;" ::: "memory"); }
+__device__ __forceinline__ void pdl_launch() { asm volatile("griddepcontrol.launch_dependents;" :::); }
+#define APT_PDL_PROLOGUE() do { ::apt::pdl_wait(); ::apt::pdl_launch(); } while (0)
+
+template <typename... KArgs, typename... Args>
+inline cudaError_t launch_pdl(void (*kern)(KArgs...), dim3 grid, dim3 block, size_t smem, cudaStream_t st,
+                              Args... args) {
+  cudaLaunchConfig_t cfg = {};
+  cfg.gridDim = grid;
+  cfg.blockDim = block;
+  cfg.dynamicSmemBytes = smem;
+  cfg.stream = st;
+  cudaLaunchAttribute at[1];
+  at[0].id = cudaLaunchAttributeProgrammaticStreamSerialization;
+  at[0].val.programmaticStreamSerializationAllowed = 1;
+  cfg.attrs = at;
+  cfg.numAttrs = 1;
+  return cudaLaunchKernelEx(&cfg, kern, static_cast<KArgs>(args)...);
+}
+
 // ---------------------------------------------------------------- misc ----
 __host__ __device__ __forceinline__ int64_t ceil_div(int64_t a, int64_t b) { return (a + b - 1) / b; }
 __host__ __device__ __forceinline__ int64_t round_up(int64_t a, int64_t b) { return ceil_div(a, b) * b; }

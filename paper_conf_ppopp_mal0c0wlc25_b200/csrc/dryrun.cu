@@ -59,6 +59,7 @@ __device__ __forceinline__ bool test_and_set(uint32_t* bm, int u) {
 __global__ void dry_count_kernel(int S, int r, int C, const int32_t* __restrict__ dst, const int32_t* __restrict__ n_p,
                                  const int32_t* __restrict__ cnt, const int32_t* __restrict__ nbr, int k,
                                  const int32_t* __restrict__ part, uint32_t* bm, int64_t n_words, DryCounters* dc) {
+  APT_PDL_PROLOGUE();
   const int64_t n = *n_p;
   for (int64_t i = int64_t(blockIdx.x) * blockDim.x + threadIdx.x; i < n; i += int64_t(gridDim.x) * blockDim.x) {
     const int v = dst[i];
@@ -109,10 +110,12 @@ __global__ void dry_count_kernel(int S, int r, int C, const int32_t* __restrict_
 }
 
 __global__ void dry_nd_kernel(int r, const int32_t* __restrict__ n_p, DryCounters* dc) {
+  APT_PDL_PROLOGUE();
   if (threadIdx.x == 0) dc->n_d[r] += *n_p;
 }
 
 __global__ void dry_fold_kernel(int C, DryCounters* dc) {
+  APT_PDL_PROLOGUE();
   const int t = threadIdx.x;
   if (t < C * C) {
     const int r = t / C, c = t % C;
@@ -125,7 +128,8 @@ __global__ void dry_fold_kernel(int C, DryCounters* dc) {
   }
 }
 
-__global__ void dry_set_step_kernel(uint64_t* p, uint64_t v) { *p = v; }
+__global__ void dry_set_step_kernel(uint64_t* p, uint64_t v) {
+  APT_PDL_PROLOGUE(); *p = v; }
 
 }  // namespace apt
 
@@ -211,14 +215,14 @@ extern "C" apt_status apt_dryrun(apt_trainer* t, int64_t n_steps, apt_plan_stats
         CK(c, cudaEventRecord(new_event(), c->stream));
         marks.push_back({S, r});
         const Hop& l1 = hops[K - 1];
-        dry_nd_kernel<<<1, 32, 0, c->stream>>>(r, l1.n_dst, dc + S);
+        launch_pdl(dry_nd_kernel, dim3(1), dim3(32), 0, c->stream, r, l1.n_dst, dc + S);
         const int64_t blocks = std::max<int64_t>(1, std::min<int64_t>(ceil_div(l1.max_dst, 256), 148 * 8));
-        dry_count_kernel<<<blocks, 256, 0, c->stream>>>(S, r, C, l1.dst, l1.n_dst, l1.cnt, l1.nbr, l1.k, g->part,
+        launch_pdl(dry_count_kernel, dim3(blocks), dim3(256), 0, c->stream, S, r, C, l1.dst, l1.n_dst, l1.cnt, l1.nbr, l1.k, g->part,
                                                         own_bm, n_words, dc + S);
         CK(c, cudaGetLastError());
         c->launches += 4 + 4 * K;
       }
-      dry_fold_kernel<<<1, 64, 0, c->stream>>>(C, dc + S);
+      launch_pdl(dry_fold_kernel, dim3(1), dim3(64), 0, c->stream, C, dc + S);
       CK(c, cudaGetLastError());
     }
   }

@@ -25,6 +25,7 @@ __device__ __forceinline__ float ldf<uint16_t>(const uint16_t* p, int64_t i) {
 
 template <typename TA, typename TB>
 __global__ void __launch_bounds__(256) simt_gemm_kernel(SimtGemmArgs a) {
+  APT_PDL_PROLOGUE();
   __shared__ float As[BK][BM + 4];
   __shared__ float Bs[BK][BN + 4];
   const int64_t M = a.M_dev ? std::min<int64_t>(a.M, *a.M_dev) : a.M;
@@ -98,10 +99,10 @@ cudaError_t launch_simt_gemm(const SimtGemmArgs& a, cudaStream_t st) {
   const int64_t kc = a.k_chunk > 0 ? a.k_chunk : a.K;
   dim3 grid(unsigned(std::max<int64_t>(1, ceil_div(a.M, BM))), unsigned(ceil_div(a.N, BN)),
             unsigned(std::max<int64_t>(1, ceil_div(a.K, kc))));
-  if (a.a_t == kF32 && a.b_t == kF32) simt_gemm_kernel<float, float><<<grid, 256, 0, st>>>(a);
-  else if (a.a_t == kF32 && a.b_t == kBF16) simt_gemm_kernel<float, uint16_t><<<grid, 256, 0, st>>>(a);
-  else if (a.a_t == kBF16 && a.b_t == kF32) simt_gemm_kernel<uint16_t, float><<<grid, 256, 0, st>>>(a);
-  else simt_gemm_kernel<uint16_t, uint16_t><<<grid, 256, 0, st>>>(a);
+  if (a.a_t == kF32 && a.b_t == kF32) launch_pdl(simt_gemm_kernel<float, float>, dim3(grid), dim3(256), 0, st, a);
+  else if (a.a_t == kF32 && a.b_t == kBF16) launch_pdl(simt_gemm_kernel<float, uint16_t>, dim3(grid), dim3(256), 0, st, a);
+  else if (a.a_t == kBF16 && a.b_t == kF32) launch_pdl(simt_gemm_kernel<uint16_t, float>, dim3(grid), dim3(256), 0, st, a);
+  else launch_pdl(simt_gemm_kernel<uint16_t, uint16_t>, dim3(grid), dim3(256), 0, st, a);
   return cudaGetLastError();
 }
 

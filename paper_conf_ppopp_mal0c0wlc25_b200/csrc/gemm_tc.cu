@@ -153,6 +153,7 @@ struct RowParams {
 
 __global__ void __launch_bounds__(ROW_THREADS, 1)
     rowtile_kernel(const __grid_constant__ CUtensorMap mapA, const __grid_constant__ CUtensorMap mapB, RowParams p) {
+  APT_PDL_PROLOGUE();
   extern __shared__ __align__(1024) uint8_t smem_raw[];
   uint8_t* smem = smem_raw + ((1024u - (smem_u32(smem_raw) & 1023u)) & 1023u);   // 1 KB aligned, still __shared__
   uint8_t* smem_a = smem;                                        // STAGES x 16 KB
@@ -337,6 +338,7 @@ struct WgradParams {
 
 __global__ void __launch_bounds__(THREADS, 1)
     wgrad_kernel(const __grid_constant__ CUtensorMap mapG, const __grid_constant__ CUtensorMap mapZ, WgradParams p) {
+  APT_PDL_PROLOGUE();
   extern __shared__ __align__(1024) uint8_t smem_raw[];
   uint8_t* smem = smem_raw + ((1024u - (smem_u32(smem_raw) & 1023u)) & 1023u);   // 1 KB aligned, still __shared__
   uint64_t* bars = reinterpret_cast<uint64_t*>(smem + size_t(WG_STAGES) * p.stage_bytes);
@@ -538,7 +540,7 @@ cudaError_t launch_tc_gemm(const TcGemmArgs& a, cudaStream_t st) {
     attr_set = true;
   }
   const int grid = int(std::min<int64_t>(tiles * n_split, (sm_count() / n_split) * n_split));
-  rowtile_kernel<<<grid, ROW_THREADS, smem, st>>>(ma, mb, p);
+  launch_pdl(rowtile_kernel, dim3(grid), dim3(ROW_THREADS), smem, st, ma, mb, p);
   return cudaGetLastError();
 }
 
@@ -571,7 +573,7 @@ cudaError_t launch_tc_wgrad(const TcWgradArgs& a, cudaStream_t st) {
   const int mt = int(ceil_div(a.d_out, BM));
   const int64_t kbs = std::max<int64_t>(1, ceil_div(a.rows_max, BK));
   const int splits = int(std::max<int64_t>(1, std::min<int64_t>(kbs, sm_count() / mt)));
-  wgrad_kernel<<<dim3(splits, mt), THREADS, smem, st>>>(mg, mz, p);
+  launch_pdl(wgrad_kernel, dim3(dim3(splits, mt)), dim3(THREADS), smem, st, mg, mz, p);
   return cudaGetLastError();
 }
 

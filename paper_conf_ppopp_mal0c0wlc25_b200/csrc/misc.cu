@@ -17,6 +17,7 @@ __global__ void ce_loss_kernel(const float* __restrict__ logits, int64_t pitch, 
                                const int32_t* __restrict__ labels, const int32_t* __restrict__ n_global_p,
                                float* __restrict__ loss, float* __restrict__ g, int64_t g_pitch,
                                uint16_t* __restrict__ gb, int64_t gb_pitch, int64_t max_seeds) {
+  APT_PDL_PROLOGUE();
   const int lane = lane_id();
   const int64_t n = *n_seeds_p;
   const float inv_n = 1.0f / float(max(1, *n_global_p));
@@ -55,13 +56,14 @@ cudaError_t launch_ce_loss(const float* logits, int64_t pitch, int n_classes, co
                            const int32_t* n_seeds, int64_t max_seeds, const int32_t* labels,
                            const int32_t* n_global, float* loss, float* g, int64_t g_pitch, uint16_t* gb,
                            int64_t gb_pitch, cudaStream_t st) {
-  ce_loss_kernel<<<grid_of(max_seeds * 32), 256, 0, st>>>(logits, pitch, n_classes, seeds, n_seeds, labels,
+  launch_pdl(ce_loss_kernel, dim3(grid_of(max_seeds * 32)), dim3(256), 0, st, logits, pitch, n_classes, seeds, n_seeds, labels,
                                                           n_global, loss, g, g_pitch, gb, gb_pitch, max_seeds);
   return cudaGetLastError();
 }
 
 __global__ void relu_bwd_kernel(float* __restrict__ g, const float* __restrict__ h, int64_t pitch, int dim,
                                 const int32_t* __restrict__ n_p) {
+  APT_PDL_PROLOGUE();
   const int64_t n = *n_p;
   const int64_t total = n * dim;
   for (int64_t t = int64_t(blockIdx.x) * blockDim.x + threadIdx.x; t < total; t += int64_t(gridDim.x) * blockDim.x) {
@@ -73,7 +75,7 @@ __global__ void relu_bwd_kernel(float* __restrict__ g, const float* __restrict__
 
 cudaError_t launch_relu_bwd(float* g, const float* h, int64_t pitch, int dim, const int32_t* n_dev, int64_t max_n,
                             cudaStream_t st) {
-  relu_bwd_kernel<<<grid_of(max_n * dim), 256, 0, st>>>(g, h, pitch, dim, n_dev);
+  launch_pdl(relu_bwd_kernel, dim3(grid_of(max_n * dim)), dim3(256), 0, st, g, h, pitch, dim, n_dev);
   return cudaGetLastError();
 }
 
@@ -82,6 +84,7 @@ cudaError_t launch_relu_bwd(float* g, const float* h, int64_t pitch, int dim, co
 __global__ void grad_finish_kernel(const float* __restrict__ G, int64_t gp, const float* __restrict__ H, int64_t hp,
                                    int dim, int relu, uint16_t* __restrict__ Gb, int64_t gbp,
                                    const int32_t* __restrict__ n_p, int64_t max_n) {
+  APT_PDL_PROLOGUE();
   const int64_t n = *n_p;
   const int64_t rows = std::min<int64_t>(max_n, round_up(n, 64));
   const int V = int(ceil_div(dim, 4));
@@ -117,7 +120,7 @@ __global__ void grad_finish_kernel(const float* __restrict__ G, int64_t gp, cons
 cudaError_t launch_grad_finish(const float* G, int64_t g_pitch, const float* H, int64_t h_pitch, int dim, int relu,
                                uint16_t* Gb, int64_t gb_pitch, const int32_t* n_dev, int64_t max_n, cudaStream_t st) {
   if ((g_pitch & 3) || (h_pitch & 3)) return cudaErrorInvalidValue;
-  grad_finish_kernel<<<grid_of(max_n * ceil_div(dim, 4)), 256, 0, st>>>(G, g_pitch, H, h_pitch, dim, relu, Gb,
+  launch_pdl(grad_finish_kernel, dim3(grid_of(max_n * ceil_div(dim, 4))), dim3(256), 0, st, G, g_pitch, H, h_pitch, dim, relu, Gb,
                                                                           gb_pitch, n_dev, max_n);
   return cudaGetLastError();
 }
@@ -125,6 +128,7 @@ cudaError_t launch_grad_finish(const float* G, int64_t g_pitch, const float* H, 
 // dst[r][0:cols] = src[r][0:cols], dst[r][cols] = 1.0 (bf16), zero tail rows to the 64-row block.
 __global__ void bf16_pad_ones_kernel(const uint16_t* __restrict__ src, int64_t sp, uint16_t* __restrict__ dst,
                                      int64_t dp, int cols, const int32_t* __restrict__ n_p, int64_t max_n) {
+  APT_PDL_PROLOGUE();
   const int64_t n = *n_p;
   const int64_t rows = std::min<int64_t>(max_n, round_up(n, 64));
   const int64_t total = rows * dp;
@@ -137,13 +141,14 @@ __global__ void bf16_pad_ones_kernel(const uint16_t* __restrict__ src, int64_t s
 
 cudaError_t launch_bf16_pad_ones(const uint16_t* src, int64_t src_pitch, uint16_t* dst, int64_t dst_pitch, int cols,
                                  const int32_t* n_dev, int64_t max_n, cudaStream_t st) {
-  bf16_pad_ones_kernel<<<grid_of(max_n * dst_pitch), 256, 0, st>>>(src, src_pitch, dst, dst_pitch, cols, n_dev, max_n);
+  launch_pdl(bf16_pad_ones_kernel, dim3(grid_of(max_n * dst_pitch)), dim3(256), 0, st, src, src_pitch, dst, dst_pitch, cols, n_dev, max_n);
   return cudaGetLastError();
 }
 
 // out[c] += sum_r g[r][c]  (db = sum of g over the rows, O5)
 __global__ void colsum_kernel(const float* __restrict__ g, int64_t pitch, int dim, const int32_t* __restrict__ n_p,
                               float* __restrict__ out) {
+  APT_PDL_PROLOGUE();
   const int64_t n = *n_p;
   const int c = blockIdx.y * blockDim.x + threadIdx.x;
   if (c >= dim) return;
@@ -158,13 +163,14 @@ cudaError_t launch_colsum(const float* g, int64_t pitch, int dim, const int32_t*
                           cudaStream_t st) {
   const int tx = 128;
   dim3 grid(unsigned(std::max<int64_t>(1, std::min<int64_t>(max_n / 256 + 1, 296))), unsigned(ceil_div(dim, tx)));
-  colsum_kernel<<<grid, tx, 0, st>>>(g, pitch, dim, n_dev, out);
+  launch_pdl(colsum_kernel, dim3(grid), dim3(tx), 0, st, g, pitch, dim, n_dev, out);
   return cudaGetLastError();
 }
 
 // W -= lr * dW; optionally refresh the bf16 copy [rows x cols] (pitch) used by tcgen05.
 __global__ void sgd_kernel(float* __restrict__ W, const float* __restrict__ dW, int64_t n, float lr,
                            uint16_t* __restrict__ wb, int cols, int64_t bpitch) {
+  APT_PDL_PROLOGUE();
   for (int64_t t = int64_t(blockIdx.x) * blockDim.x + threadIdx.x; t < n; t += int64_t(gridDim.x) * blockDim.x) {
     const float w = W[t] - lr * dW[t];
     W[t] = w;
@@ -178,6 +184,7 @@ __global__ void sgd_kernel(float* __restrict__ W, const float* __restrict__ dW, 
 
 // All parameter tensors of a step in one launch: blockIdx.y = tensor.
 __global__ void sgd_multi_kernel(SgdBatch b, float lr) {
+  APT_PDL_PROLOGUE();
   const SgdSeg& g = b.seg[blockIdx.y];
   for (int64_t t = int64_t(blockIdx.x) * blockDim.x + threadIdx.x; t < g.n; t += int64_t(gridDim.x) * blockDim.x) {
     const float w = g.W[t] - lr * g.dW[t];
@@ -195,19 +202,20 @@ cudaError_t launch_sgd_multi(const SgdBatch& b, float lr, cudaStream_t st) {
   int64_t mx = 1;
   for (int i = 0; i < b.n; ++i) mx = std::max<int64_t>(mx, b.seg[i].n);
   dim3 grid(unsigned(std::min<int64_t>(ceil_div(mx, 256), 148 * 4)), unsigned(b.n));
-  sgd_multi_kernel<<<grid, 256, 0, st>>>(b, lr);
+  launch_pdl(sgd_multi_kernel, dim3(grid), dim3(256), 0, st, b, lr);
   return cudaGetLastError();
 }
 
 cudaError_t launch_sgd(float* W, const float* dW, int64_t n, float lr, uint16_t* W_bf16, int rows, int cols,
                        int64_t bf16_pitch, cudaStream_t st) {
   (void)rows;
-  sgd_kernel<<<grid_of(n), 256, 0, st>>>(W, dW, n, lr, W_bf16, cols, bf16_pitch);
+  launch_pdl(sgd_kernel, dim3(grid_of(n)), dim3(256), 0, st, W, dW, n, lr, W_bf16, cols, bf16_pitch);
   return cudaGetLastError();
 }
 
 __global__ void to_bf16_kernel(const float* __restrict__ src, int64_t sp, uint16_t* __restrict__ dst, int64_t dp,
                                int cols, const int32_t* __restrict__ n_p, int64_t n_static) {
+  APT_PDL_PROLOGUE();
   const int64_t n = n_p ? int64_t(*n_p) : n_static;
   const int64_t total = n * cols;
   for (int64_t t = int64_t(blockIdx.x) * blockDim.x + threadIdx.x; t < total; t += int64_t(gridDim.x) * blockDim.x) {
@@ -220,7 +228,7 @@ __global__ void to_bf16_kernel(const float* __restrict__ src, int64_t sp, uint16
 
 cudaError_t launch_to_bf16(const float* src, int64_t src_pitch, uint16_t* dst, int64_t dst_pitch, int cols,
                            const int32_t* n_dev, int64_t max_n, cudaStream_t st) {
-  to_bf16_kernel<<<grid_of(max_n * cols), 256, 0, st>>>(src, src_pitch, dst, dst_pitch, cols, n_dev, max_n);
+  launch_pdl(to_bf16_kernel, dim3(grid_of(max_n * cols)), dim3(256), 0, st, src, src_pitch, dst, dst_pitch, cols, n_dev, max_n);
   return cudaGetLastError();
 }
 

@@ -32,6 +32,7 @@ __global__ void __launch_bounds__(256) sample_kernel(const int64_t* __restrict__
                                                      uint2 key, const uint64_t* __restrict__ step_ptr,
                                                      int hop, int32_t* __restrict__ cnt,
                                                      int32_t* __restrict__ nbr) {
+  APT_PDL_PROLOGUE();
   const int lane = lane_id();
   const int64_t F = *n_frontier;
   const uint32_t step = uint32_t(*step_ptr);
@@ -95,7 +96,7 @@ cudaError_t launch_sample(const SampleArgs& a, cudaStream_t st) {
   const int ks = int(ceil_div(a.k, 32));
 #define APT_SAMPLE_CASE(KS)                                                                      \
   case KS:                                                                                       \
-    sample_kernel<KS><<<blocks, threads, 0, st>>>(a.indptr, a.indices, a.frontier, a.n_frontier, \
+    launch_pdl(sample_kernel<KS>, dim3(blocks), dim3(threads), 0, st, a.indptr, a.indices, a.frontier, a.n_frontier, \
                                                   a.k, a.key, a.step, a.hop, a.cnt, a.nbr);      \
     break;
   switch (ks) {
@@ -104,11 +105,11 @@ cudaError_t launch_sample(const SampleArgs& a, cudaStream_t st) {
     APT_SAMPLE_CASE(4)
     APT_SAMPLE_CASE(8)
     case 3:
-      sample_kernel<4><<<blocks, threads, 0, st>>>(a.indptr, a.indices, a.frontier, a.n_frontier,
+      launch_pdl(sample_kernel<4>, dim3(blocks), dim3(threads), 0, st, a.indptr, a.indices, a.frontier, a.n_frontier,
                                                    a.k, a.key, a.step, a.hop, a.cnt, a.nbr);
       break;
     default:
-      sample_kernel<8><<<blocks, threads, 0, st>>>(a.indptr, a.indices, a.frontier, a.n_frontier,
+      launch_pdl(sample_kernel<8>, dim3(blocks), dim3(threads), 0, st, a.indptr, a.indices, a.frontier, a.n_frontier,
                                                    a.k, a.key, a.step, a.hop, a.cnt, a.nbr);
   }
 #undef APT_SAMPLE_CASE
@@ -173,6 +174,7 @@ __global__ void map_indices_kernel(const int32_t* __restrict__ dst, const int32_
                                    int k, const int32_t* __restrict__ indptr,
                                    const int32_t* __restrict__ pos, int32_t* __restrict__ indices,
                                    uint32_t* __restrict__ dst_bm) {
+  APT_PDL_PROLOGUE();
   const int64_t slots = int64_t(*n_dst) * k;
   for (int64_t s = int64_t(blockIdx.x) * blockDim.x + threadIdx.x; s < slots; s += int64_t(gridDim.x) * blockDim.x) {
     const int64_t i = s / k;
@@ -203,6 +205,7 @@ __global__ void compact_mark_kernel(const int32_t* __restrict__ dst, const int32
                                     uint32_t* __restrict__ dst_bm, uint32_t* __restrict__ new_bm,
                                     int32_t* __restrict__ pos, int32_t* __restrict__ src, uint64_t* __restrict__ stA,
                                     int nbA, uint64_t* __restrict__ stB, int nbB, int32_t* __restrict__ ticket) {
+  APT_PDL_PROLOGUE();
   const int64_t F = *n_dst;
   const int64_t tid = int64_t(blockIdx.x) * blockDim.x + threadIdx.x, nth = int64_t(gridDim.x) * blockDim.x;
   for (int64_t i = tid; i < nbA + nbB + 1; i += nth) {
@@ -314,6 +317,7 @@ struct NewBitsOp {   // words of (new & ~dst): ascending new source ids
 
 __global__ void __launch_bounds__(kScanThreads) compact_scan_kernel(NewBitsOp a, uint64_t* stA, int nbA, CntScanOp c,
                                                                     uint64_t* stB, int nbB, int32_t* ticket) {
+  APT_PDL_PROLOGUE();
   __shared__ int32_t tk;
   if (threadIdx.x == 0) tk = atomicAdd(ticket, 1);
   __syncthreads();
@@ -329,12 +333,12 @@ cudaError_t launch_compact(const CompactArgs& a, cudaStream_t st) {
   uint64_t* stA = reinterpret_cast<uint64_t*>(a.partials);            // >= 2*nbA + 8 int32
   int32_t* ticket = a.partials + 2 * nbA + 2;
   uint64_t* stB = reinterpret_cast<uint64_t*>(a.partials2);           // >= 2*nbB + 8 int32
-  compact_mark_kernel<<<grid_for(a.max_dst * a.k, T), T, 0, st>>>(a.dst, a.n_dst, a.cnt, a.nbr, a.k, a.dst_bm,
+  launch_pdl(compact_mark_kernel, dim3(grid_for(a.max_dst * a.k, T)), dim3(T), 0, st, a.dst, a.n_dst, a.cnt, a.nbr, a.k, a.dst_bm,
                                                                    a.new_bm, a.pos, a.src, stA, nbA, stB, nbB, ticket);
   NewBitsOp bop{a.new_bm, a.dst_bm, a.n_words, a.n_dst, a.src, a.pos, a.n_src};
   CntScanOp cop{a.cnt, a.n_dst, a.indptr, a.n_edges};
-  compact_scan_kernel<<<nbA + nbB, kScanThreads, 0, st>>>(bop, stA, nbA, cop, stB, nbB, ticket);
-  map_indices_kernel<<<grid_for(a.max_dst * a.k, T), T, 0, st>>>(a.dst, a.cnt, a.nbr, a.n_dst, a.k, a.indptr,
+  launch_pdl(compact_scan_kernel, dim3(nbA + nbB), dim3(kScanThreads), 0, st, bop, stA, nbA, cop, stB, nbB, ticket);
+  launch_pdl(map_indices_kernel, dim3(grid_for(a.max_dst * a.k, T)), dim3(T), 0, st, a.dst, a.cnt, a.nbr, a.n_dst, a.k, a.indptr,
                                                                   a.pos, a.indices, a.dst_bm);
   return cudaGetLastError();
 }
@@ -349,6 +353,7 @@ __global__ void __launch_bounds__(1024) select_seeds_kernel(const int32_t* __res
                                                             const int32_t* __restrict__ part,
                                                             int32_t* __restrict__ seeds, int32_t* __restrict__ n_seeds,
                                                             int32_t* __restrict__ n_global) {
+  APT_PDL_PROLOGUE();
   const int64_t t = int64_t(*step_ptr % uint64_t(steps_per_epoch));
   const int64_t g0 = t * int64_t(world) * batch;
   int64_t gn = n_train - g0;
@@ -388,7 +393,7 @@ __global__ void __launch_bounds__(1024) select_seeds_kernel(const int32_t* __res
 }
 
 cudaError_t launch_select_seeds(const SeedArgs& a, cudaStream_t st) {
-  select_seeds_kernel<<<1, 1024, 0, st>>>(a.perm, a.n_train, a.step, a.steps_per_epoch, a.world, a.rank,
+  launch_pdl(select_seeds_kernel, dim3(1), dim3(1024), 0, st, a.perm, a.n_train, a.step, a.steps_per_epoch, a.world, a.rank,
                                           a.batch, a.by_part, a.part, a.seeds, a.n_seeds, a.n_global);
   return cudaGetLastError();
 }

@@ -63,6 +63,7 @@ struct WorkTab {
 __global__ void permute_kernel(int mode, int req, int C, const int32_t* __restrict__ dst,
                                const int32_t* __restrict__ n_dst, const int32_t* __restrict__ cnt,
                                const int32_t* __restrict__ nbr, int k, const int32_t* __restrict__ part, WorkTab w) {
+  APT_PDL_PROLOGUE();
   const int64_t n = *n_dst;
   for (int64_t i = int64_t(blockIdx.x) * blockDim.x + threadIdx.x; i < n; i += int64_t(gridDim.x) * blockDim.x) {
     const int v = dst[i];
@@ -92,6 +93,7 @@ __global__ void permute_kernel(int mode, int req, int C, const int32_t* __restri
 __global__ void gather_g_bf16_kernel(uint16_t* const* __restrict__ src, int64_t pitch, const int32_t* __restrict__ rank,
                                      const int32_t* __restrict__ row, const int32_t* __restrict__ n_p, int64_t max_n,
                                      uint16_t* __restrict__ out) {
+  APT_PDL_PROLOGUE();
   const int64_t n = *n_p;
   const int64_t rows = std::min<int64_t>(max_n, round_up(n, 64));
   const int V = int(pitch / 8);
@@ -108,6 +110,7 @@ __global__ void gather_g_bf16_kernel(uint16_t* const* __restrict__ src, int64_t 
 __global__ void gather_g_f32_kernel(float* const* __restrict__ src, int64_t pitch, const int32_t* __restrict__ rank,
                                     const int32_t* __restrict__ row, const int32_t* __restrict__ n_p,
                                     float* __restrict__ out) {
+  APT_PDL_PROLOGUE();
   const int64_t n = *n_p;
   const int V = int(pitch / 4);
   const int64_t total = n * V;
@@ -122,6 +125,7 @@ __global__ void gather_g_f32_kernel(float* const* __restrict__ src, int64_t pitc
 // Requester (SNP / NFP): h = act(sum of partial pre-activations + b), in place (Z10).
 __global__ void bias_act_kernel(float* __restrict__ H, int64_t pitch, int dim, const float* __restrict__ b, int relu,
                                 const int32_t* __restrict__ n_p) {
+  APT_PDL_PROLOGUE();
   const int64_t n = *n_p;
   const int64_t total = n * dim;
   for (int64_t t = int64_t(blockIdx.x) * blockDim.x + threadIdx.x; t < total; t += int64_t(gridDim.x) * blockDim.x) {
@@ -138,6 +142,7 @@ __global__ void bias_act_kernel(float* __restrict__ H, int64_t pitch, int dim, c
 template <typename T>
 __global__ void __launch_bounds__(256) colsum_kernel2(const T* __restrict__ g, int64_t pitch, int dim,
                                                       const int32_t* __restrict__ n_p, float* __restrict__ out) {
+  APT_PDL_PROLOGUE();
   __shared__ float red[256 * 4];
   const int64_t n = *n_p;
   const int V = int(ceil_div(dim, 4));
@@ -174,8 +179,8 @@ static apt_status launch_colsum2(apt_ctx* c, const void* g, bool bf16, int64_t p
                                  float* out) {
   if (dim > 1024) return set_err(c, APT_E_UNSUPPORTED, "colsum: dim > 1024");
   const int blocks = 296;
-  if (bf16) colsum_kernel2<uint16_t><<<blocks, 256, 0, c->stream>>>(static_cast<const uint16_t*>(g), pitch, dim, n_dev, out);
-  else colsum_kernel2<float><<<blocks, 256, 0, c->stream>>>(static_cast<const float*>(g), pitch, dim, n_dev, out);
+  if (bf16) launch_pdl(colsum_kernel2<uint16_t>, dim3(blocks), dim3(256), 0, c->stream, static_cast<const uint16_t*>(g), pitch, dim, n_dev, out);
+  else launch_pdl(colsum_kernel2<float>, dim3(blocks), dim3(256), 0, c->stream, static_cast<const float*>(g), pitch, dim, n_dev, out);
   CK(c, cudaGetLastError());
   c->launches++;
   return APT_OK;
@@ -353,7 +358,7 @@ apt_status layer1_fwd_strategy(apt_trainer* t) {
   { apt_status s = device_barrier(c); if (s != APT_OK) return s; }   // lists cleared everywhere
   for (auto& rs : t->R) {
     const Hop& hp = rs.hops[t->K - 1];
-    permute_kernel<<<grid_n(hp.max_dst), 256, 0, c->stream>>>(mode, rs.rank, t->world, hp.dst, hp.n_dst, hp.cnt,
+    launch_pdl(permute_kernel, dim3(grid_n(hp.max_dst)), dim3(256), 0, c->stream, mode, rs.rank, t->world, hp.dst, hp.n_dst, hp.cnt,
                                                                hp.nbr, hp.k, t->g->part, w);
     CK(c, cudaGetLastError());
     c->launches++;
@@ -371,7 +376,7 @@ apt_status layer1_fwd_strategy(apt_trainer* t) {
   if (partial) {
     for (auto& rs : t->R) {
       Layer& L = rs.L[0];
-      bias_act_kernel<<<grid_n(L.max_rows * L.d_out), 256, 0, c->stream>>>(L.H, L.h_pitch, L.d_out, L.b,
+      launch_pdl(bias_act_kernel, dim3(grid_n(L.max_rows * L.d_out)), dim3(256), 0, c->stream, L.H, L.h_pitch, L.d_out, L.b,
                                                                               t->K > 1 ? 1 : 0, L.n_rows);
       CK(c, cudaGetLastError());
       c->launches++;
@@ -401,7 +406,7 @@ apt_status layer1_bwd_strategy(apt_trainer* t) {
     if (t->s == APT_NFP) CK(c, cudaMemsetAsync(x.dW1s, 0, sizeof(float) * L.d_out * std::max(x.w_cols, 1), c->stream));
     if (x.w_cols == 0) continue;
     if (bf) {
-      gather_g_bf16_kernel<<<grid_n(x.wcap * (L.gb_pitch / 8)), 256, 0, c->stream>>>(
+      launch_pdl(gather_g_bf16_kernel, dim3(grid_n(x.wcap * (L.gb_pitch / 8))), dim3(256), 0, c->stream, 
           t->Gb1_tab, L.gb_pitch, x.work_rank, x.work_row, x.n_work, x.wcap, x.wGb);
       CK(c, cudaGetLastError());
       if (tc_wgrad_supported(L.d_out, x.w_cols)) {
@@ -412,7 +417,7 @@ apt_status layer1_bwd_strategy(apt_trainer* t) {
                        L.d_out, x.w_cols);
       }
     } else {
-      gather_g_f32_kernel<<<grid_n(x.wcap * (L.h_pitch / 4)), 256, 0, c->stream>>>(
+      launch_pdl(gather_g_f32_kernel, dim3(grid_n(x.wcap * (L.h_pitch / 4))), dim3(256), 0, c->stream, 
           t->G1_tab, L.h_pitch, x.work_rank, x.work_row, x.n_work, x.wGf);
       CK(c, cudaGetLastError());
       SimtGemmArgs a{};

@@ -43,6 +43,7 @@ namespace apt {
 // the caller fences with device barriers before (peers' gradients complete) and
 // after (everyone has read them) and copies out -> own buffer.
 __global__ void allreduce_gather_kernel(float* const* tab, int C, int64_t n, float* __restrict__ out) {
+  APT_PDL_PROLOGUE();
   for (int64_t i = int64_t(blockIdx.x) * blockDim.x + threadIdx.x; i < n; i += int64_t(gridDim.x) * blockDim.x) {
     float s = 0.f;
     for (int r = 0; r < C; ++r) s += tab[r][i];   // fixed rank order: every rank gets identical sums
@@ -51,6 +52,7 @@ __global__ void allreduce_gather_kernel(float* const* tab, int C, int64_t n, flo
 }
 
 __global__ void allreduce_sum_kernel(float* const* tab, int C, int64_t n) {
+  APT_PDL_PROLOGUE();
   for (int64_t i = int64_t(blockIdx.x) * blockDim.x + threadIdx.x; i < n; i += int64_t(gridDim.x) * blockDim.x) {
     float s = 0.f;
     for (int r = 0; r < C; ++r) s += tab[r][i];
@@ -67,11 +69,13 @@ static cudaError_t record_ev(apt_trainer* t, int i) {
 
 // The step id enters the device as a kernel argument (no host cell that a later
 // call could overwrite before the copy runs); graph replays patch the argument.
-__global__ void set_step_kernel(uint64_t* step_dev, uint64_t step) { *step_dev = step; }
+__global__ void set_step_kernel(uint64_t* step_dev, uint64_t step) {
+  APT_PDL_PROLOGUE(); *step_dev = step; }
 
 // dst[r][0:cols] = src[r][0:cols] for r < *n (device count)
 __global__ void copy_rows_kernel(float* __restrict__ dst, int64_t dp, const float* __restrict__ src, int64_t sp, int cols,
                                  const int32_t* __restrict__ n_p) {
+  APT_PDL_PROLOGUE();
   const int64_t total = int64_t(*n_p) * cols;
   for (int64_t t = int64_t(blockIdx.x) * blockDim.x + threadIdx.x; t < total; t += int64_t(gridDim.x) * blockDim.x) {
     const int64_t r = t / cols;
@@ -81,6 +85,7 @@ __global__ void copy_rows_kernel(float* __restrict__ dst, int64_t dp, const floa
 }
 
 __global__ void zero_rows_kernel(float* p, int64_t pitch, const int32_t* n_p) {
+  APT_PDL_PROLOGUE();
   const int64_t total = int64_t(*n_p) * pitch;
   float4* q = reinterpret_cast<float4*>(p);
   for (int64_t t = int64_t(blockIdx.x) * blockDim.x + threadIdx.x; t < total / 4; t += int64_t(gridDim.x) * blockDim.x)
@@ -475,7 +480,7 @@ apt_status upper_bwd(apt_trainer* t, RankState& rs) {
       CK(c, launch_simt_gemm(a, c->stream));
     }
     // dH_{l-1} = scatter(dZ / deg) over the layer-l block, then through the ReLU
-    zero_rows_kernel<<<blocks_for(P.max_rows * P.h_pitch / 4), 256, 0, c->stream>>>(P.G, P.h_pitch, P.n_rows);
+    launch_pdl(zero_rows_kernel, dim3(blocks_for(P.max_rows * P.h_pitch / 4)), dim3(256), 0, c->stream, P.G, P.h_pitch, P.n_rows);
     CK(c, cudaGetLastError());
     CK(c, launch_agg_bwd(hp.indptr, hp.indices, hp.n_dst, hp.max_dst, L.dZ, L.zf_pitch, L.d_in, P.G, P.h_pitch,
                          c->stream));
@@ -499,14 +504,14 @@ apt_status layer1_bwd_gdp(apt_trainer* t, RankState& rs) {
 apt_status allreduce_grads(apt_trainer* t, int64_t P) {
   apt_ctx* c = t->ctx;
   if (c->emulated) {
-    allreduce_sum_kernel<<<blocks_for(P), 256, 0, c->stream>>>(t->dW_tab, t->world, P);
+    launch_pdl(allreduce_sum_kernel, dim3(blocks_for(P)), dim3(256), 0, c->stream, t->dW_tab, t->world, P);
     CK(c, cudaGetLastError());
     c->launches++;
     return APT_OK;
   }
   apt_status s = device_barrier(c);
   if (s != APT_OK) return s;
-  allreduce_gather_kernel<<<blocks_for(P), 256, 0, c->stream>>>(t->dW_tab, t->world, P, t->ar_scratch);
+  launch_pdl(allreduce_gather_kernel, dim3(blocks_for(P)), dim3(256), 0, c->stream, t->dW_tab, t->world, P, t->ar_scratch);
   CK(c, cudaGetLastError());
   if ((s = device_barrier(c)) != APT_OK) return s;
   CK(c, cudaMemcpyAsync(t->R[0].L[0].dW, t->ar_scratch, sizeof(float) * P, cudaMemcpyDeviceToDevice, c->stream));
@@ -652,7 +657,7 @@ apt_status apt_layer_bwd(apt_trainer* t, const float* const* dh1, int64_t pitch)
     Layer& L = rs.L[0];
     if (!dh1[li]) return set_err(c, APT_E_INVALID, "apt_layer_bwd: dh1[%zu] is null", li);
     // G = dh1 (copied over the rows the step produced; the count stays on the device)
-    copy_rows_kernel<<<blocks_for(L.max_rows * L.d_out), 256, 0, c->stream>>>(L.G, L.h_pitch, dh1[li], pitch, L.d_out,
+    launch_pdl(copy_rows_kernel, dim3(blocks_for(L.max_rows * L.d_out)), dim3(256), 0, c->stream, L.G, L.h_pitch, dh1[li], pitch, L.d_out,
                                                                              L.n_rows);
     CK(c, cudaGetLastError());
     if (bf) CK(c, launch_grad_finish(L.G, L.h_pitch, L.H, L.h_pitch, L.d_out, relu, L.Gb, L.gb_pitch, L.n_rows,
