@@ -52,6 +52,7 @@ struct SeedArgs {
   int32_t* seeds;
   int32_t* n_seeds;
   int32_t* n_global;
+  const int32_t* n_dev;        // if set: perm is one global batch of *n_dev ids (host-batch path)
 };
 cudaError_t launch_select_seeds(const SeedArgs& a, cudaStream_t st);
 cudaError_t launch_perm_keys(const int32_t* train, int64_t n, uint64_t seed, uint64_t epoch, uint64_t* keys,

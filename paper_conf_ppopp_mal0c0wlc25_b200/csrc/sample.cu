@@ -352,9 +352,11 @@ __global__ void __launch_bounds__(1024) select_seeds_kernel(const int32_t* __res
                                                             int world, int rank, int batch, int by_part,
                                                             const int32_t* __restrict__ part,
                                                             int32_t* __restrict__ seeds, int32_t* __restrict__ n_seeds,
-                                                            int32_t* __restrict__ n_global) {
+                                                            int32_t* __restrict__ n_global,
+                                                            const int32_t* __restrict__ n_dev) {
   APT_PDL_PROLOGUE();
-  const int64_t t = int64_t(*step_ptr % uint64_t(steps_per_epoch));
+  if (n_dev) n_train = *n_dev;   // host-batch path: perm holds exactly one global batch
+  const int64_t t = n_dev ? 0 : int64_t(*step_ptr % uint64_t(steps_per_epoch));
   const int64_t g0 = t * int64_t(world) * batch;
   int64_t gn = n_train - g0;
   if (gn > int64_t(world) * batch) gn = int64_t(world) * batch;
@@ -394,7 +396,7 @@ __global__ void __launch_bounds__(1024) select_seeds_kernel(const int32_t* __res
 
 cudaError_t launch_select_seeds(const SeedArgs& a, cudaStream_t st) {
   launch_pdl(select_seeds_kernel, dim3(1), dim3(1024), 0, st, a.perm, a.n_train, a.step, a.steps_per_epoch, a.world, a.rank,
-                                          a.batch, a.by_part, a.part, a.seeds, a.n_seeds, a.n_global);
+                                          a.batch, a.by_part, a.part, a.seeds, a.n_seeds, a.n_global, a.n_dev);
   return cudaGetLastError();
 }
 

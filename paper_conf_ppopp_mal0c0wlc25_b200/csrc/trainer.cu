@@ -84,6 +84,31 @@ __global__ void copy_rows_kernel(float* __restrict__ dst, int64_t dp, const floa
   }
 }
 
+// The set_step node of a captured step graph, and its per-replay patch.
+static cudaGraphNode_t find_step_node(cudaGraph_t graph) {
+  size_t n = 0;
+  if (cudaGraphGetNodes(graph, nullptr, &n) != cudaSuccess) return nullptr;
+  std::vector<cudaGraphNode_t> nodes(n);
+  if (cudaGraphGetNodes(graph, nodes.data(), &n) != cudaSuccess) return nullptr;
+  for (auto nd : nodes) {
+    cudaGraphNodeType ty;
+    if (cudaGraphNodeGetType(nd, &ty) != cudaSuccess || ty != cudaGraphNodeTypeKernel) continue;
+    cudaKernelNodeParams kp;
+    if (cudaGraphKernelNodeGetParams(nd, &kp) == cudaSuccess && kp.func == (void*)set_step_kernel) return nd;
+  }
+  return nullptr;
+}
+
+static cudaError_t patch_step_node(cudaGraphExec_t exec, cudaGraphNode_t node, uint64_t* step_dev, uint64_t step) {
+  void* args[2] = {&step_dev, &step};
+  cudaKernelNodeParams kp{};
+  kp.func = (void*)set_step_kernel;
+  kp.gridDim = dim3(1);
+  kp.blockDim = dim3(1);
+  kp.kernelParams = args;
+  return cudaGraphExecKernelNodeSetParams(exec, node, &kp);
+}
+
 __global__ void zero_rows_kernel(float* p, int64_t pitch, const int32_t* n_p) {
   APT_PDL_PROLOGUE();
   const int64_t total = int64_t(*n_p) * pitch;
@@ -174,6 +199,9 @@ apt_status apt_trainer_create(apt_ctx* c, const apt_graph* g, const apt_fstore* 
   const int K = t->K, C = t->world;
   t->labels = A.alloc<int32_t>(g->n, false);
   t->step_dev = A.alloc<uint64_t>(1, true);
+  t->hb_dev = A.alloc<int32_t>(1 + int64_t(C) * m->batch, true);
+  CK(c, cudaMallocHost(reinterpret_cast<void**>(&t->hb_pinned), sizeof(int32_t) * (1 + int64_t(C) * m->batch)));
+  CK(c, cudaMallocHost(reinterpret_cast<void**>(&t->loss_pinned), sizeof(float) * APT_MAX_RANKS));
   CK(c, cudaMemcpyAsync(t->labels, labels, sizeof(int32_t) * g->n, cudaMemcpyHostToDevice, c->stream));
   const int64_t n_words = ceil_div(g->n, 32);
   // upper bounds per hop.  SNP/DNP seeds follow the partition: up to C*B on one rank.
@@ -287,6 +315,10 @@ apt_status apt_trainer_destroy(apt_trainer* t) {
   cudaStreamSynchronize(t->ctx->stream);
   if (t->gexec) cudaGraphExecDestroy(t->gexec);
   if (t->graph) cudaGraphDestroy(t->graph);
+  if (t->gexec_host) cudaGraphExecDestroy(t->gexec_host);
+  if (t->graph_host) cudaGraphDestroy(t->graph_host);
+  if (t->hb_pinned) cudaFreeHost(t->hb_pinned);
+  if (t->loss_pinned) cudaFreeHost(t->loss_pinned);
   for (int i = 0; i < 8; ++i)
     if (t->ev[i]) cudaEventDestroy(t->ev[i]);
   apt_ctx* c = t->ctx;
@@ -381,10 +413,13 @@ namespace apt {
 // Phase A for one rank: seeds + sampling (+ compaction for every hop but the layer-1 one).
 apt_status phase_sample(apt_trainer* t, RankState& rs, bool from_host_batch) {
   apt_ctx* c = t->ctx;
-  if (!from_host_batch) {
+  {
+    // seeds of the step: from the epoch permutation, or from the global batch the host
+    // copied in (hb_dev = [n, ids...]); chunk r for GDP/NFP, partition r for SNP/DNP
     const bool by_part = (t->s == APT_SNP || t->s == APT_DNP) && t->world > 1;
-    SeedArgs sa{t->perm, t->n_train, t->step_dev, t->steps_per_epoch, t->world, rs.rank, t->m.batch, by_part ? 1 : 0,
-                t->g->part, rs.seeds, rs.small, rs.small + 1};
+    SeedArgs sa{from_host_batch ? t->hb_dev + 1 : t->perm, t->n_train, t->step_dev, t->steps_per_epoch, t->world,
+                rs.rank, t->m.batch, by_part ? 1 : 0, t->g->part, rs.seeds, rs.small, rs.small + 1,
+                from_host_batch ? t->hb_dev : nullptr};
     CK(c, launch_select_seeds(sa, c->stream));
     c->launches++;
   }
@@ -703,34 +738,13 @@ apt_status apt_trainer_step(apt_trainer* t, int64_t step, int update) {
       if (s != APT_OK) return s;
       CK(c, e);
       // find the set_step node so replays can patch the step id
-      size_t n = 0;
-      CK(c, cudaGraphGetNodes(graph, nullptr, &n));
-      std::vector<cudaGraphNode_t> nodes(n);
-      CK(c, cudaGraphGetNodes(graph, nodes.data(), &n));
-      t->step_node = nullptr;
-      for (auto nd : nodes) {
-        cudaGraphNodeType ty;
-        if (cudaGraphNodeGetType(nd, &ty) != cudaSuccess || ty != cudaGraphNodeTypeKernel) continue;
-        cudaKernelNodeParams kp;
-        if (cudaGraphKernelNodeGetParams(nd, &kp) == cudaSuccess && kp.func == (void*)set_step_kernel) {
-          t->step_node = nd;
-          break;
-        }
-      }
+      t->step_node = find_step_node(graph);
       if (!t->step_node) { cudaGraphDestroy(graph); return set_err(c, APT_E_CUDA, "step node not found in graph"); }
       CK(c, cudaGraphInstantiate(&t->gexec, graph, 0));
       t->graph = graph;
       t->graph_update = update;
     }
-    uint64_t* sd = t->step_dev;
-    uint64_t sv = uint64_t(step);
-    void* args[2] = {&sd, &sv};
-    cudaKernelNodeParams kp{};
-    kp.func = (void*)set_step_kernel;
-    kp.gridDim = dim3(1);
-    kp.blockDim = dim3(1);
-    kp.kernelParams = args;
-    CK(c, cudaGraphExecKernelNodeSetParams(t->gexec, t->step_node, &kp));
+    CK(c, patch_step_node(t->gexec, t->step_node, t->step_dev, uint64_t(step)));
     CK(c, cudaGraphLaunch(t->gexec, c->stream));
     c->launches += t->launches_per_step;
     return APT_OK;
@@ -746,28 +760,65 @@ apt_status apt_trainer_step(apt_trainer* t, int64_t step, int update) {
 
 apt_status apt_trainer_step_host(apt_trainer* t, const int64_t* gbatch, int64_t n_global, int64_t step, int update,
                                  float* loss_host) {
-  if (!t || !gbatch || n_global < 1 || n_global > int64_t(t->world) * t->m.batch)
+  if (!t || !gbatch || !loss_host || n_global < 1 || n_global > int64_t(t->world) * t->m.batch)
     return set_err(t ? t->ctx : nullptr, APT_E_INVALID, "apt_trainer_step_host: bad arguments");
   apt_ctx* c = t->ctx;
-  // host global batch -> per-rank seeds (GDP/NFP: chunk r; SNP/DNP: partition r), H2D on the stream
-  for (auto& rs : t->R) {
-    std::vector<int32_t> mine;
-    const bool by_part = (t->s == APT_SNP || t->s == APT_DNP) && t->world > 1;
-    for (int64_t i = 0; i < n_global; ++i) {
-      const int64_t u = gbatch[i];
-      if (u < 0 || u >= t->g->n) return set_err(c, APT_E_INVALID, "step_host: seed out of range");
-      if (by_part ? t->g->part_h[u] == rs.rank : (i / t->m.batch) == rs.rank) mine.push_back(int32_t(u));
-    }
-    int32_t hdr[2] = {int32_t(mine.size()), int32_t(n_global)};
-    CK(c, cudaMemcpyAsync(rs.seeds, mine.data(), sizeof(int32_t) * mine.size(), cudaMemcpyHostToDevice, c->stream));
-    CK(c, cudaMemcpyAsync(rs.small, hdr, sizeof hdr, cudaMemcpyHostToDevice, c->stream));
+  if (c->broken) return set_err(c, APT_E_STATE, "ctx is broken by an earlier CUDA error");
+  // the global batch into pinned staging ([n, ids...], int32); ranks pick their seeds on
+  // the device.  The previous call ended with a sync, so the staging is free.
+  t->hb_pinned[0] = int32_t(n_global);
+  for (int64_t i = 0; i < n_global; ++i) {
+    const int64_t u = gbatch[i];
+    if (u < 0 || u >= t->g->n) return set_err(c, APT_E_INVALID, "step_host: seed %lld out of range", (long long)u);
+    t->hb_pinned[1 + i] = int32_t(u);
   }
-  set_step_kernel<<<1, 1, 0, c->stream>>>(t->step_dev, uint64_t(step));
-  CK(c, cudaGetLastError());
-  c->launches++;
-  apt_status s = step_body(t, update, true);
-  if (s != APT_OK) return s;
-  return apt_trainer_loss(t, loss_host);
+  const size_t hb_bytes = sizeof(int32_t) * (1 + size_t(t->world) * t->m.batch);
+  // H2D batch -> step -> D2H per-rank losses, one stream-ordered sequence (one graph replay)
+  auto body = [&]() -> apt_status {
+    CK(c, cudaMemcpyAsync(t->hb_dev, t->hb_pinned, hb_bytes, cudaMemcpyHostToDevice, c->stream));
+    set_step_kernel<<<1, 1, 0, c->stream>>>(t->step_dev, uint64_t(step));
+    CK(c, cudaGetLastError());
+    apt_status s = step_body(t, update, true);
+    if (s != APT_OK) return s;
+    for (size_t i = 0; i < t->R.size(); ++i)
+      CK(c, cudaMemcpyAsync(t->loss_pinned + i, t->R[i].loss, sizeof(float), cudaMemcpyDeviceToHost, c->stream));
+    return APT_OK;
+  };
+  if (t->use_graph) {
+    if (!t->gexec_host || t->graph_host_update != update) {
+      if (t->gexec_host) { cudaGraphExecDestroy(t->gexec_host); t->gexec_host = nullptr; }
+      if (t->graph_host) { cudaGraphDestroy(t->graph_host); t->graph_host = nullptr; }
+      cudaGraph_t graph;
+      CK(c, cudaStreamBeginCapture(c->stream, cudaStreamCaptureModeThreadLocal));
+      const int64_t l0 = c->launches;
+      t->capturing = true;
+      apt_status s = body();
+      t->capturing = false;
+      cudaError_t e = cudaStreamEndCapture(c->stream, &graph);
+      const int64_t per = c->launches - l0 + 1;
+      c->launches = l0;
+      if (s != APT_OK) return s;
+      CK(c, e);
+      t->step_node_host = find_step_node(graph);
+      if (!t->step_node_host) { cudaGraphDestroy(graph); return set_err(c, APT_E_CUDA, "step node not found in graph"); }
+      CK(c, cudaGraphInstantiate(&t->gexec_host, graph, 0));
+      t->graph_host = graph;
+      t->graph_host_update = update;
+      t->launches_per_step_host = per;
+    }
+    CK(c, patch_step_node(t->gexec_host, t->step_node_host, t->step_dev, uint64_t(step)));
+    CK(c, cudaGraphLaunch(t->gexec_host, c->stream));
+    c->launches += t->launches_per_step_host;
+  } else {
+    apt_status s = body();
+    if (s != APT_OK) return s;
+    c->launches++;
+  }
+  CK(c, cudaStreamSynchronize(c->stream));
+  float tot = 0.f;
+  for (size_t i = 0; i < t->R.size(); ++i) tot += t->loss_pinned[i];
+  *loss_host = tot;
+  return apt_ctx_sync(c);
 }
 
 apt_status apt_trainer_loss(apt_trainer* t, float* loss) {

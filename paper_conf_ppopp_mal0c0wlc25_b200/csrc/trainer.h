@@ -106,6 +106,14 @@ struct apt_trainer {
   bool use_graph = false;
   bool capturing = false;
   cudaGraphExec_t gexec = nullptr;
+  cudaGraphExec_t gexec_host = nullptr;   // the end-to-end step: H2D batch, step, D2H loss
+  cudaGraph_t graph_host = nullptr;
+  cudaGraphNode_t step_node_host = nullptr;
+  int graph_host_update = -1;
+  int64_t launches_per_step_host = 0;
+  int32_t* hb_pinned = nullptr;       // [1 + C*B] host staging: n, ids (pinned)
+  int32_t* hb_dev = nullptr;          // device copy
+  float* loss_pinned = nullptr;       // [APT_MAX_RANKS] per hosted rank
   cudaGraph_t graph = nullptr;
   cudaGraphNode_t step_node = nullptr;
   int64_t launches_per_step = 0;

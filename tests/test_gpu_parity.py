@@ -249,15 +249,21 @@ def test_sgd_update_and_graph_replay(A, ctx, tiny):
         assert np.allclose(W, Wr, rtol=1e-5, atol=1e-6) and np.allclose(b, br, rtol=1e-5, atol=1e-6)
 
 
-def test_step_host_e2e_matches_device_step(A, ctx, tiny):
+@pytest.mark.parametrize("use_graph", [False, True])
+def test_step_host_e2e_matches_device_step(A, ctx, tiny, use_graph):
+    """The end-to-end call (host global batch in, loss out; H2D -> step -> D2H replayed as
+    one graph) reproduces the device-resident step on the same seeds."""
     cfg, g, train = tiny
     tr, params, labels = _trainer(A, ctx, cfg, g, train, "bf16")
-    tr.step(2, update=False)
-    l_dev = tr.loss()
+    tr.use_graph(use_graph)
     perm = oracle.epoch_perm(train, cfg.sample_seed, 0)
-    gb = torch.as_tensor(perm[2 * cfg.batch:3 * cfg.batch]).pin_memory()
-    l_host = tr.step_host(gb, 2, update=False)
-    assert l_host == pytest.approx(l_dev, rel=1e-6)
+    for step in (2, 1, 2):
+        tr.step(step, update=False)
+        l_dev = tr.loss()
+        gb = torch.as_tensor(perm[step * cfg.batch:(step + 1) * cfg.batch]).pin_memory()
+        l_host = tr.step_host(gb, step, update=False)
+        assert l_host == pytest.approx(l_dev, rel=1e-6)
+        assert np.array_equal(tr.read("seeds")[:, 0], perm[step * cfg.batch:(step + 1) * cfg.batch])
 
 
 # ------------------------------------------------------------------ S11 weight gradient
