@@ -115,6 +115,34 @@ cudaError_t launch_gather(const FeatView& fv, const int32_t* ids, const int32_t*
 cudaError_t launch_fill_features(void* shard, DType dt, int64_t pitch, int col0, int ncols, const int32_t* ids,
                                  int64_t n, uint64_t seed, cudaStream_t st);
 
+// ---------------------------------------------------------------- bwd.cu
+// Transpose of a sampled block (counting sort): csc_ptr [n_src+1], csc_dst [E].
+struct CscArgs {
+  const int32_t* indptr; const int32_t* indices;
+  const int32_t* n_dst; int64_t max_dst;
+  const int32_t* n_edges; int64_t max_edges;
+  const int32_t* n_src; int64_t max_src;
+  int32_t* cnt;        // [max_src], zero on entry and exit
+  int32_t* csc_ptr;    // [max_src + 1]
+  int32_t* csc_total;  // [1]
+  int32_t* csc_dst;    // [max_edges]
+  int32_t* ws;         // scan workspace, >= 2*ceil(max_src/2048) + 8
+};
+cudaError_t launch_csc_build(const CscArgs& a, cudaStream_t st);
+
+// G[u] = mask(H[u] > 0) * sum_{(v,u)} dZ[v] / deg(v) over rows u < *n_src; fp32 G and/or
+// bf16 Gb (whose 64-row-block tail is zeroed).
+struct PullArgs {
+  const int32_t* csc_ptr; const int32_t* csc_dst; const int32_t* indptr;
+  const float* dz; int64_t dz_pitch;
+  const float* h; int64_t h_pitch;        // null: no mask
+  float* g; int64_t g_pitch;               // may be null
+  uint16_t* gb; int64_t gb_pitch;          // may be null
+  const int32_t* n_src; int64_t max_src;
+  int dim;
+};
+cudaError_t launch_pull_bwd(const PullArgs& a, cudaStream_t st);
+
 // ---------------------------------------------------------------- gemm_simt.cu
 // C[m][n] (+)= sum_k A(m,k) B(k,n) (+ bias[n]) (relu), fp32 accumulate.
 // A(m,k) = A[m*sam + k*sak]; B(k,n) = B[k*sbk + n*sbn]; M may live on device.

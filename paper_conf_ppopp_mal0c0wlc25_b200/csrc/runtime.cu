@@ -34,6 +34,7 @@ static void ctx_free(apt_ctx* c) {
   if (c->side) { cudaStreamSynchronize(c->side); cudaStreamDestroy(c->side); }
   if (c->ev_fork) cudaEventDestroy(c->ev_fork);
   if (c->ev_join) cudaEventDestroy(c->ev_join);
+  if (c->ev_csc) cudaEventDestroy(c->ev_csc);
   c->arena.release();
   if (c->own_stream) cudaStreamDestroy(c->stream);
   delete c;
@@ -90,6 +91,7 @@ apt_status apt_ctx_create(int rank, int world, int device, void* stream, apt_ctx
   cudaStreamCreateWithFlags(&c->side, cudaStreamNonBlocking);
   cudaEventCreateWithFlags(&c->ev_fork, cudaEventDisableTiming);
   cudaEventCreateWithFlags(&c->ev_join, cudaEventDisableTiming);
+  cudaEventCreateWithFlags(&c->ev_csc, cudaEventDisableTiming);
   c->dev_err = c->arena.alloc<uint32_t>(4);
   c->scratch = c->arena.alloc<int32_t>(16);
   if (!c->dev_err || !c->scratch) {

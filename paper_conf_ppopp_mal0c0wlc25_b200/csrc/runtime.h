@@ -72,7 +72,7 @@ struct apt_ctx {
   cudaStream_t stream = nullptr;
   bool own_stream = false;
   cudaStream_t side = nullptr;           // forked branch of a step (weight gradients off the critical path)
-  cudaEvent_t ev_fork = nullptr, ev_join = nullptr;
+  cudaEvent_t ev_fork = nullptr, ev_join = nullptr, ev_csc = nullptr;
   bool broken = false;
   std::string err;
   int64_t launches = 0;

@@ -326,6 +326,33 @@ __global__ void __launch_bounds__(kScanThreads) compact_scan_kernel(NewBitsOp a,
   else scan_tile(c, stB, t - nbA, nbB);
 }
 
+// Exclusive scan of device-counted int32 values (one launch after a tiny reset):
+// out[i] = sum_{j<i} cnt[j], out[n] = *total = the sum.
+__global__ void scan_reset_kernel(uint64_t* st, int nb, int32_t* ticket) {
+  APT_PDL_PROLOGUE();
+  for (int i = threadIdx.x; i < nb; i += blockDim.x) st[i] = 0;
+  if (threadIdx.x == 0) *ticket = 0;
+}
+
+__global__ void __launch_bounds__(kScanThreads) count_scan_kernel(CntScanOp c, uint64_t* st, int nb, int32_t* ticket) {
+  APT_PDL_PROLOGUE();
+  __shared__ int32_t tk;
+  if (threadIdx.x == 0) tk = atomicAdd(ticket, 1);
+  __syncthreads();
+  scan_tile(c, st, tk, nb);
+}
+
+cudaError_t launch_scan_counts(const int32_t* cnt, const int32_t* n_dev, int64_t max_n, int32_t* out, int32_t* total,
+                               int32_t* ws, cudaStream_t st) {
+  const int nb = int(std::max<int64_t>(1, ceil_div(max_n, kScanTile)));
+  uint64_t* status = reinterpret_cast<uint64_t*>(ws);     // ws >= 2*nb + 8 int32
+  int32_t* ticket = ws + 2 * nb + 2;
+  launch_pdl(scan_reset_kernel, dim3(1), dim3(256), 0, st, status, nb, ticket);
+  CntScanOp cop{cnt, n_dev, out, total};
+  launch_pdl(count_scan_kernel, dim3(nb), dim3(kScanThreads), 0, st, cop, status, nb, ticket);
+  return cudaGetLastError();
+}
+
 cudaError_t launch_compact(const CompactArgs& a, cudaStream_t st) {
   const int T = 256;
   const int nbA = int(std::max<int64_t>(1, ceil_div(a.n_words, kScanTile)));

@@ -236,6 +236,10 @@ apt_status apt_trainer_create(apt_ctx* c, const apt_graph* g, const apt_fstore* 
         hp.src = A.alloc<int32_t>(hp.max_src, false);
         hp.indptr = A.alloc<int32_t>(maxF + 1, true);
         hp.indices = A.alloc<int32_t>(maxF * hp.k, false);
+        hp.csc_cnt = A.alloc<int32_t>(hp.max_src, true);
+        hp.csc_ptr = A.alloc<int32_t>(hp.max_src + 1, true);
+        hp.csc_dst = A.alloc<int32_t>(maxF * hp.k, false);
+        hp.csc_ws = A.alloc<int32_t>(2 * ceil_div(hp.max_src, 2048) + 8, false);
       }
       dst = hp.src;
       n_dst = hp.counts;
@@ -435,8 +439,17 @@ apt_status phase_sample(apt_trainer* t, RankState& rs, bool from_host_batch) {
                      hp.counts, hp.indptr, hp.indices, hp.counts + 1, rs.partials, hp.part2};
       CK(c, launch_compact(ca, c->stream));
       c->launches += 3;
+      // transpose of this block for the pull-form mean backward: a side branch that
+      // overlaps the rest of the forward (joined before the backward, ev_csc)
+      CK(c, cudaEventRecord(c->ev_fork, c->stream));
+      CK(c, cudaStreamWaitEvent(c->side, c->ev_fork, 0));
+      CscArgs cs{hp.indptr, hp.indices, hp.n_dst, hp.max_dst, hp.counts + 1, hp.max_dst * hp.k, hp.counts,
+                 hp.max_src, hp.csc_cnt, hp.csc_ptr, hp.counts + 2, hp.csc_dst, hp.csc_ws};
+      CK(c, launch_csc_build(cs, c->side));
+      c->launches += 4;
     }
   }
+  if (t->K > 1) CK(c, cudaEventRecord(c->ev_csc, c->side));
   return APT_OK;
 }
 
@@ -514,15 +527,14 @@ apt_status upper_bwd(apt_trainer* t, RankState& rs) {
       a.C = L.dZ; a.ldc = L.zf_pitch; a.M_dev = L.n_rows; a.M = L.max_rows; a.N = L.d_in; a.K = L.d_out;
       CK(c, launch_simt_gemm(a, c->stream));
     }
-    // dH_{l-1} = scatter(dZ / deg) over the layer-l block, then through the ReLU
-    launch_pdl(zero_rows_kernel, dim3(blocks_for(P.max_rows * P.h_pitch / 4)), dim3(256), 0, c->stream, P.G, P.h_pitch, P.n_rows);
-    CK(c, cudaGetLastError());
-    CK(c, launch_agg_bwd(hp.indptr, hp.indices, hp.n_dst, hp.max_dst, L.dZ, L.zf_pitch, L.d_in, P.G, P.h_pitch,
-                         c->stream));
-    if (bf) CK(c, launch_grad_finish(P.G, P.h_pitch, P.H, P.h_pitch, P.d_out, 1, P.Gb, P.gb_pitch, P.n_rows,
-                                     P.max_rows, c->stream));
-    else CK(c, launch_relu_bwd(P.G, P.H, P.h_pitch, P.d_out, P.n_rows, P.max_rows, c->stream));
-    c->launches += 4;
+    // dH_{l-1}: every source row of the layer-l block pulls its in-edges' dZ / deg
+    // (transpose built on the side branch), through the ReLU, straight to G (fp32 mode)
+    // or its bf16 copy (bf16 mode)
+    if (l == t->K) CK(c, cudaStreamWaitEvent(c->stream, c->ev_csc, 0));
+    PullArgs pa{hp.csc_ptr, hp.csc_dst, hp.indptr, L.dZ, L.zf_pitch, P.H, P.h_pitch, bf ? nullptr : P.G, P.h_pitch,
+                bf ? P.Gb : nullptr, P.gb_pitch, hp.counts, P.max_rows, L.d_in};
+    CK(c, launch_pull_bwd(pa, c->stream));
+    c->launches += 2;
   }
   return APT_OK;
 }
@@ -667,16 +679,20 @@ apt_status apt_layer_fwd(apt_trainer* t, int64_t step) {
     apt_status s = phase_sample(t, rs, false);
     if (s != APT_OK) return s;
   }
+  apt_status s = APT_OK;
   if (t->world == 1 || t->s == APT_GDP) {
     bool first = true;
     for (auto& rs : t->R) {
-      apt_status s = layer1_fwd_gdp(t, rs, first);
+      s = layer1_fwd_gdp(t, rs, first);
       first = false;
       if (s != APT_OK) return s;
     }
-    return APT_OK;
+  } else {
+    s = layer1_fwd_strategy(t);
+    if (s != APT_OK) return s;
   }
-  return layer1_fwd_strategy(t);
+  if (t->K > 1) CK(c, cudaStreamWaitEvent(c->stream, c->ev_csc, 0));   // join the side branch
+  return APT_OK;
 }
 
 // ... and backward from dL/dh1 (one device pointer per hosted rank, rows of the

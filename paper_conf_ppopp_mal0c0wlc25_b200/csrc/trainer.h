@@ -18,8 +18,13 @@ struct Hop {
   int32_t* src = nullptr;           // [max_src]
   int32_t* indptr = nullptr;        // [max_dst + 1]
   int32_t* indices = nullptr;       // [max_dst * k]
-  int32_t* counts = nullptr;        // [0] n_src, [1] n_edges
+  int32_t* counts = nullptr;        // [0] n_src, [1] n_edges, [2] csc total
   int32_t* part2 = nullptr;         // scan workspace
+  // transpose of the block (upper hops only): in-edges of every local source
+  int32_t* csc_cnt = nullptr;       // [max_src] (zero between uses)
+  int32_t* csc_ptr = nullptr;       // [max_src + 1]
+  int32_t* csc_dst = nullptr;       // [max_dst * k]
+  int32_t* csc_ws = nullptr;        // scan workspace
 };
 
 struct Layer {
