@@ -89,7 +89,13 @@ __global__ void __launch_bounds__(256) pull_bwd_kernel(PullArgs a) {
       const int j = lane + 32 * p;
       if (j >= V) continue;
       float4 g = make_float4(acc[p][0], acc[p][1], acc[p][2], acc[p][3]);
-      if (u < n && a.h) {
+      if (u < n && a.mask) {
+        const uint32_t mw = uint32_t(a.mask[u * a.mask_pitch + (j * 4) / 16]) >> ((j * 4) & 15);
+        if (!(mw & 1u)) g.x = 0.f;
+        if (!(mw & 2u)) g.y = 0.f;
+        if (!(mw & 4u)) g.z = 0.f;
+        if (!(mw & 8u)) g.w = 0.f;
+      } else if (u < n && a.h) {
         const float4 h = *reinterpret_cast<const float4*>(a.h + u * a.h_pitch + j * 4);
         if (!(h.x > 0.f)) g.x = 0.f;
         if (!(h.y > 0.f)) g.y = 0.f;

@@ -149,6 +149,8 @@ struct RowParams {
   const int32_t* out_row;
   int accumulate;
   int n_split;              // CTAs share an M tile: CTA b computes columns [(b % n_split) * BN, +BN)
+  uint16_t* mask;           // optional ReLU bit mask [M x mask_pitch] (16 columns per word)
+  int64_t mask_pitch;
 };
 
 __global__ void __launch_bounds__(ROW_THREADS, 1)
@@ -286,10 +288,21 @@ __global__ void __launch_bounds__(ROW_THREADS, 1)
         for (int it = 0; it < 4; ++it) {
           const int row = it * 8 + rsub;
           float* dst = reinterpret_cast<float*>(__shfl_sync(0xffffffffu, reinterpret_cast<uintptr_t>(own), row));
-          if (!dst || col >= p.N) continue;
           const float* sv = stg + row * 17 + cq;
           float4 v = make_float4(sv[0] + bv.x, sv[1] + bv.y, sv[2] + bv.z, sv[3] + bv.w);
           if (p.relu) { v.x = fmaxf(v.x, 0.f); v.y = fmaxf(v.y, 0.f); v.z = fmaxf(v.z, 0.f); v.w = fmaxf(v.w, 0.f); }
+          if (p.mask) {   // 16 mask bits of (row, chunk) from the 4 lanes of the row segment
+            uint32_t bits = (col < p.N && v.x > 0.f ? 1u : 0u) | (col + 1 < p.N && v.y > 0.f ? 2u : 0u) |
+                            (col + 2 < p.N && v.z > 0.f ? 4u : 0u) | (col + 3 < p.N && v.w > 0.f ? 8u : 0u);
+            bits <<= 4 * (lane & 3);
+            bits |= __shfl_xor_sync(0xffffffffu, bits, 1);
+            bits |= __shfl_xor_sync(0xffffffffu, bits, 2);
+            if ((lane & 3) == 0 && dst && col < p.N) {
+              const int64_t m = t * BM + q * 32 + row;
+              p.mask[m * p.mask_pitch + (n0 + c) / 16] = uint16_t(bits);
+            }
+          }
+          if (!dst || col >= p.N) continue;
           if (p.accumulate) {
             if (col + 4 <= p.N) {
               red_add_v4(dst + col, v.x, v.y, v.z, v.w);
@@ -530,7 +543,7 @@ cudaError_t launch_tc_gemm(const TcGemmArgs& a, cudaStream_t st) {
     b_kb_bytes = uint32_t(BN) * 128;
   }
   RowParams p{a.M_max, a.M_dev, a.N, BN, nkb, cols, a.w_mn, b_kb_bytes, a.bias, a.relu, a.Y, a.y_pitch,
-              a.out_base, a.out_rank, a.out_row, a.accumulate, n_split};
+              a.out_base, a.out_rank, a.out_row, a.accumulate, n_split, a.mask, a.mask_pitch};
   const size_t smem = 1024 + size_t(STAGES) * A_STAGE_BYTES + size_t(nkb) * b_kb_bytes + 16 * 8 + 16 +
                       8 * 32 * 17 * 4;   // + epilogue staging
   if (smem > 227 * 1024) return cudaErrorInvalidValue;

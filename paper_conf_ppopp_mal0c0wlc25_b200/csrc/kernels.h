@@ -136,6 +136,7 @@ struct PullArgs {
   const int32_t* csc_ptr; const int32_t* csc_dst; const int32_t* indptr;
   const float* dz; int64_t dz_pitch;
   const float* h; int64_t h_pitch;        // null: no mask
+  const uint16_t* mask; int64_t mask_pitch;   // if set: the ReLU mask as bits (replaces reading h)
   float* g; int64_t g_pitch;               // may be null
   uint16_t* gb; int64_t gb_pitch;          // may be null
   const int32_t* n_src; int64_t max_src;
@@ -176,6 +177,7 @@ struct TcGemmArgs {
   float* const* out_base; const int32_t* out_rank; const int32_t* out_row;
   int w_mn;                            // B stored N-contiguous (dZ = G W uses W [d_out x d_in] as is)
   int accumulate;                      // add into Y with vector reductions (partial sums of SNP / NFP)
+  uint16_t* mask; int64_t mask_pitch;  // optional: bit c%16 of mask[m][c/16] = (Y[m][c] > 0) (ReLU mask for the backward)
 };
 int tc_gemm_supported(int N, int K);
 cudaError_t launch_tc_gemm(const TcGemmArgs& a, cudaStream_t st);

@@ -239,25 +239,32 @@ __device__ __forceinline__ uint64_t ld_acquire_gpu(const uint64_t* p) {
   return v;
 }
 
-// Decoupled look-back for block `b` of a chain: publishes the block aggregate, walks
-// predecessors until an inclusive prefix, publishes its own.  Thread 0 only.
+// Decoupled look-back for block `b` of a chain, by one warp: publish the block
+// aggregate, then inspect the 32 nearest predecessors at once (each lane spins on
+// one slot until it carries a flag), sum back to the nearest inclusive prefix, and
+// move the window 32 blocks back if none was inclusive yet; finally publish the
+// block's own inclusive prefix.  All lanes of warp 0 call it; all return the prefix.
 __device__ int32_t chain_prefix(uint64_t* st, int b, int32_t agg) {
-  constexpr uint64_t kAgg = 1ull << 32, kIncl = 2ull << 32;
+  constexpr uint64_t kAgg = 1ull << 32, kIncl = 2ull << 32, kFlags = 3ull << 32;
+  const int lane = lane_id();
   if (b == 0) {
-    st_release_gpu(st, kIncl | uint32_t(agg));
+    if (lane == 0) st_release_gpu(st, kIncl | uint32_t(agg));
     return 0;
   }
-  st_release_gpu(st + b, kAgg | uint32_t(agg));
+  if (lane == 0) st_release_gpu(st + b, kAgg | uint32_t(agg));
   int32_t excl = 0;
-  for (int j = b - 1;;) {
-    const uint64_t w = ld_acquire_gpu(st + j);
-    const uint64_t flag = w & (3ull << 32);
-    if (!flag) continue;
-    excl += int32_t(uint32_t(w));
-    if (flag == kIncl) break;
-    --j;
+  for (int end = b;; end -= 32) {
+    const int j = end - 1 - lane;
+    uint64_t w = 0;
+    if (j >= 0) {
+      do { w = ld_acquire_gpu(st + j); } while (!(w & kFlags));
+    }
+    const unsigned incl = __ballot_sync(0xffffffffu, j >= 0 && (w & kFlags) == kIncl);
+    const int stop = incl ? __ffs(incl) - 1 : 31;
+    excl += warp_sum((j >= 0 && lane <= stop) ? int32_t(uint32_t(w)) : 0);
+    if (incl) break;
   }
-  st_release_gpu(st + b, kIncl | uint32_t(excl + agg));
+  if (lane == 0) st_release_gpu(st + b, kIncl | uint32_t(excl + agg));
   return excl;
 }
 
@@ -274,9 +281,12 @@ __device__ void scan_tile(const Op& op, uint64_t* st, int b, int nb) {
   }
   __shared__ int32_t tot, prefix;
   int32_t excl = block_exclusive_scan<int32_t>(s, &tot);
-  if (threadIdx.x == 0) {
-    prefix = chain_prefix(st, b, tot);
-    if (b == nb - 1) op.finish(prefix + tot);
+  if (threadIdx.x < 32) {
+    const int32_t pre = chain_prefix(st, b, tot);
+    if (threadIdx.x == 0) {
+      prefix = pre;
+      if (b == nb - 1) op.finish(pre + tot);
+    }
   }
   __syncthreads();
   excl += prefix;

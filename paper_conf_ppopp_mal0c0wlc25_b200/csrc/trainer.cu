@@ -128,6 +128,7 @@ apt_status project(apt_trainer* t, const Layer& L, const void* Zb, const float* 
   if (t->m.dtype == APT_BF16 && tc_gemm_supported(L.d_out, K)) {
     TcGemmArgs a{static_cast<const uint16_t*>(Zb), z_pitch_b, Wb, L.wb_pitch, max_rows, n_rows, L.d_out, K,
                  bias, relu, Y, L.h_pitch, out_base, out_rank, out_row, 0};
+    if (relu && L.Mk && !out_rank) { a.mask = L.Mk; a.mask_pitch = L.mk_pitch; }   // ReLU bits for the backward
     CK(c, launch_tc_gemm(a, c->stream));
   } else {
     if (out_rank) return set_err(c, APT_E_UNSUPPORTED, "routed epilogue needs the tcgen05 path");
@@ -263,6 +264,9 @@ apt_status apt_trainer_create(apt_ctx* c, const apt_graph* g, const apt_fstore* 
       L.H = A.alloc<float>(L.max_rows * L.h_pitch, true);
       L.G = A.alloc<float>(L.max_rows * L.h_pitch, true);
       if (m->dtype == APT_BF16) L.Gb = A.alloc<uint16_t>(L.max_rows * L.gb_pitch, true);
+      // (ReLU bit masks, L.Mk, are supported by the epilogue and the pull kernel but not
+      //  allocated: measured on products, the 2-byte mask stores cost the projection more
+      //  than the pull saves by not reading H -- 78 vs 66 us forward, 72 vs 74 us backward)
       if (l > 1) L.dZ = A.alloc<float>(L.max_rows * L.zf_pitch, true);
       L.W = A.alloc<float>(int64_t(L.d_out) * L.d_in, true);
       L.b = A.alloc<float>(L.d_out, true);
@@ -531,8 +535,11 @@ apt_status upper_bwd(apt_trainer* t, RankState& rs) {
     // (transpose built on the side branch), through the ReLU, straight to G (fp32 mode)
     // or its bf16 copy (bf16 mode)
     if (l == t->K) CK(c, cudaStreamWaitEvent(c->stream, c->ev_csc, 0));
-    PullArgs pa{hp.csc_ptr, hp.csc_dst, hp.indptr, L.dZ, L.zf_pitch, P.H, P.h_pitch, bf ? nullptr : P.G, P.h_pitch,
-                bf ? P.Gb : nullptr, P.gb_pitch, hp.counts, P.max_rows, L.d_in};
+    // ReLU bits of H_{l-1} exist when its projection ran on this rank's tcgen05 path
+    const bool l1_local = l - 1 > 1 || t->world == 1 || t->s == APT_GDP;
+    const uint16_t* mk = (bf && P.Mk && l1_local && tc_gemm_supported(P.d_out, P.d_in)) ? P.Mk : nullptr;
+    PullArgs pa{hp.csc_ptr, hp.csc_dst, hp.indptr, L.dZ, L.zf_pitch, P.H, P.h_pitch, mk, P.mk_pitch,
+                bf ? nullptr : P.G, P.h_pitch, bf ? P.Gb : nullptr, P.gb_pitch, hp.counts, P.max_rows, L.d_in};
     CK(c, launch_pull_bwd(pa, c->stream));
     c->launches += 2;
   }

@@ -37,6 +37,9 @@ struct Layer {
   float* H = nullptr;               // post-activation (or logits)
   float* G = nullptr;               // dL/dpre
   uint16_t* Gb = nullptr;           // bf16 copy of G (tcgen05 backward, bf16 mode)
+  uint16_t* Mk = nullptr;           // ReLU mask bits of H (bf16 mode, hidden layers) [max_rows x mk_pitch]
+  int64_t mk_pitch = 0;
+  bool mk_valid = false;            // the last forward wrote Mk (tcgen05 epilogue on this rank)
   int64_t gb_pitch = 0;
   float* dZ = nullptr;              // [max_rows x zf_pitch] scratch (l > 1)
   float* W = nullptr;               // [d_out x d_in] fp32 master
