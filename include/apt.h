@@ -228,6 +228,10 @@ apt_status apt_trainer_step_host(apt_trainer* t, const int64_t* gbatch_host, int
 apt_status apt_trainer_loss(apt_trainer* t, float* loss);
 /* Record/replay the device part of apt_trainer_step as a CUDA graph.        */
 apt_status apt_trainer_use_graph(apt_trainer* t, int enable);
+/* Pipelining (default on): while step t computes, step t+1's mini-batch is
+ * sampled into a second buffer set on a separate stream (SURVEY §8(f) NEXT #4,
+ * P:299 "sampling" overlapped).  Results are identical with it off.          */
+apt_status apt_trainer_set_pipeline(apt_trainer* t, int enable);
 
 /* The first GNN layer alone under the trainer's strategy -- the layer APT
  * parallelises (upper layers are data parallel and may be the

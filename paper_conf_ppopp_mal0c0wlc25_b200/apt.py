@@ -106,7 +106,7 @@ def lib():
             "apt_trainer_set_params": [vp, i32, vp, vp], "apt_trainer_get_params": [vp, i32, i32, vp, vp],
             "apt_trainer_set_epoch": [vp, vp, i64, u64], "apt_trainer_step": [vp, i64, i32],
             "apt_trainer_step_host": [vp, vp, i64, i64, i32, vp], "apt_trainer_loss": [vp, vp],
-            "apt_trainer_use_graph": [vp, i32], "apt_trainer_read": [vp, i32, i32, i32, vp, i64, vp, vp],
+            "apt_trainer_use_graph": [vp, i32], "apt_trainer_set_pipeline": [vp, i32], "apt_trainer_read": [vp, i32, i32, i32, vp, i64, vp, vp],
             "apt_trainer_phase_ms": [vp, vp, i32], "apt_trainer_agg_bytes": [vp, vp],
             "apt_dryrun": [vp, i64, vp], "apt_layer_fwd": [vp, i64], "apt_layer_bwd": [vp, vp, i64], "apt_profile_links": [vp, vp], "apt_select_strategy": [vp, vp, vp, vp],
         }
@@ -324,6 +324,9 @@ class Trainer(Handle):
 
     def use_graph(self, on=True):
         self.ctx.ck(lib().apt_trainer_use_graph(self.h, 1 if on else 0))
+
+    def set_pipeline(self, on=True):
+        self.ctx.ck(lib().apt_trainer_set_pipeline(self.h, 1 if on else 0))
 
     def read(self, what, layer=0, rank=0, cap=1 << 28):
         rows, cols = C.c_int64(0), C.c_int(0)

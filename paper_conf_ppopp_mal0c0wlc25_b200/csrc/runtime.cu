@@ -32,6 +32,9 @@ static void ctx_free(apt_ctx* c) {
   cudaStreamSynchronize(c->stream);
   release_exported(c);
   if (c->side) { cudaStreamSynchronize(c->side); cudaStreamDestroy(c->side); }
+  if (c->samp) { cudaStreamSynchronize(c->samp); cudaStreamDestroy(c->samp); }
+  if (c->ev_pfork) cudaEventDestroy(c->ev_pfork);
+  if (c->ev_pjoin) cudaEventDestroy(c->ev_pjoin);
   if (c->ev_fork) cudaEventDestroy(c->ev_fork);
   if (c->ev_join) cudaEventDestroy(c->ev_join);
   if (c->ev_csc) cudaEventDestroy(c->ev_csc);
@@ -89,6 +92,9 @@ apt_status apt_ctx_create(int rank, int world, int device, void* stream, apt_ctx
     c->own_stream = true;
   }
   cudaStreamCreateWithFlags(&c->side, cudaStreamNonBlocking);
+  cudaStreamCreateWithFlags(&c->samp, cudaStreamNonBlocking);
+  cudaEventCreateWithFlags(&c->ev_pfork, cudaEventDisableTiming);
+  cudaEventCreateWithFlags(&c->ev_pjoin, cudaEventDisableTiming);
   cudaEventCreateWithFlags(&c->ev_fork, cudaEventDisableTiming);
   cudaEventCreateWithFlags(&c->ev_join, cudaEventDisableTiming);
   cudaEventCreateWithFlags(&c->ev_csc, cudaEventDisableTiming);

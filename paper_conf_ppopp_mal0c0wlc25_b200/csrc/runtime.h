@@ -72,6 +72,8 @@ struct apt_ctx {
   cudaStream_t stream = nullptr;
   bool own_stream = false;
   cudaStream_t side = nullptr;           // forked branch of a step (weight gradients off the critical path)
+  cudaStream_t samp = nullptr;           // sampling of the next step (pipelined trainer)
+  cudaEvent_t ev_pfork = nullptr, ev_pjoin = nullptr;
   cudaEvent_t ev_fork = nullptr, ev_join = nullptr, ev_csc = nullptr;
   bool broken = false;
   std::string err;

@@ -199,7 +199,8 @@ apt_status apt_trainer_create(apt_ctx* c, const apt_graph* g, const apt_fstore* 
   Arena& A = t->arena;
   const int K = t->K, C = t->world;
   t->labels = A.alloc<int32_t>(g->n, false);
-  t->step_dev = A.alloc<uint64_t>(1, true);
+  t->step_cells = A.alloc<uint64_t>(2, true);   // step id of sample set 0 / 1
+  t->step_dev = t->step_cells;
   t->hb_dev = A.alloc<int32_t>(1 + int64_t(C) * m->batch, true);
   CK(c, cudaMallocHost(reinterpret_cast<void**>(&t->hb_pinned), sizeof(int32_t) * (1 + int64_t(C) * m->batch)));
   CK(c, cudaMallocHost(reinterpret_cast<void**>(&t->loss_pinned), sizeof(float) * APT_MAX_RANKS));
@@ -211,41 +212,48 @@ apt_status apt_trainer_create(apt_ctx* c, const apt_graph* g, const apt_fstore* 
   for (int li = 0; li < c->n_local; ++li) {
     RankState& rs = t->R[li];
     rs.rank = c->emulated ? li : c->rank;
-    rs.seeds = A.alloc<int32_t>(std::max<int64_t>(B0, int64_t(C) * m->batch), false);
-    rs.small = A.alloc<int32_t>(16, true);
     rs.loss = A.alloc<float>(4, true);
     rs.dst_bm = A.alloc<uint32_t>(n_words, true);
     rs.new_bm = A.alloc<uint32_t>(n_words, true);
     rs.pos = A.alloc<int32_t>(g->n, false);
     rs.partials = A.alloc<int32_t>(2 * ceil_div(n_words, 2048) + 8, false);
-    rs.hops.resize(K);
-    int64_t maxF = B0;
-    const int32_t* dst = rs.seeds;
-    const int32_t* n_dst = rs.small;
-    for (int h = 0; h < K; ++h) {
-      Hop& hp = rs.hops[h];
-      hp.k = m->fanouts[K - 1 - h];
-      hp.max_dst = maxF;
-      hp.max_src = std::max<int64_t>(maxF, std::min<int64_t>(maxF * (1 + hp.k), g->n));
-      hp.dst = dst;
-      hp.n_dst = n_dst;
-      hp.cnt = A.alloc<int32_t>(maxF, true);
-      hp.nbr = A.alloc<int32_t>(maxF * hp.k, false);
-      hp.counts = A.alloc<int32_t>(4, true);
-      hp.part2 = A.alloc<int32_t>(2 * ceil_div(maxF, 2048) + 8, false);
-      if (h + 1 < K) {   // the layer-1 hop is consumed in ELL form (fused gather), no CSR needed
-        hp.src = A.alloc<int32_t>(hp.max_src, false);
-        hp.indptr = A.alloc<int32_t>(maxF + 1, true);
-        hp.indices = A.alloc<int32_t>(maxF * hp.k, false);
-        hp.csc_cnt = A.alloc<int32_t>(hp.max_src, true);
-        hp.csc_ptr = A.alloc<int32_t>(hp.max_src + 1, true);
-        hp.csc_dst = A.alloc<int32_t>(maxF * hp.k, false);
-        hp.csc_ws = A.alloc<int32_t>(2 * ceil_div(hp.max_src, 2048) + 8, false);
+    for (int q = 0; q < 2; ++q) {
+      SampleSet& ss = rs.sset[q];
+      ss.seeds = A.alloc<int32_t>(std::max<int64_t>(B0, int64_t(C) * m->batch), false);
+      ss.small = A.alloc<int32_t>(16, true);
+      ss.step_cell = t->step_cells + q;
+      ss.hops.resize(K);
+      int64_t maxF = B0;
+      const int32_t* dst = ss.seeds;
+      const int32_t* n_dst = ss.small;
+      for (int h = 0; h < K; ++h) {
+        Hop& hp = ss.hops[h];
+        hp.k = m->fanouts[K - 1 - h];
+        hp.max_dst = maxF;
+        hp.max_src = std::max<int64_t>(maxF, std::min<int64_t>(maxF * (1 + hp.k), g->n));
+        hp.dst = dst;
+        hp.n_dst = n_dst;
+        hp.cnt = A.alloc<int32_t>(maxF, true);
+        hp.nbr = A.alloc<int32_t>(maxF * hp.k, false);
+        hp.counts = A.alloc<int32_t>(4, true);
+        hp.part2 = A.alloc<int32_t>(2 * ceil_div(maxF, 2048) + 8, false);
+        if (h + 1 < K) {   // the layer-1 hop is consumed in ELL form (fused gather), no CSR needed
+          hp.src = A.alloc<int32_t>(hp.max_src, false);
+          hp.indptr = A.alloc<int32_t>(maxF + 1, true);
+          hp.indices = A.alloc<int32_t>(maxF * hp.k, false);
+          hp.csc_cnt = A.alloc<int32_t>(hp.max_src, true);
+          hp.csc_ptr = A.alloc<int32_t>(hp.max_src + 1, true);
+          hp.csc_dst = A.alloc<int32_t>(maxF * hp.k, false);
+          hp.csc_ws = A.alloc<int32_t>(2 * ceil_div(hp.max_src, 2048) + 8, false);
+        }
+        dst = hp.src;
+        n_dst = hp.counts;
+        maxF = hp.max_src;
       }
-      dst = hp.src;
-      n_dst = hp.counts;
-      maxF = hp.max_src;
     }
+    rs.seeds = rs.sset[0].seeds;
+    rs.small = rs.sset[0].small;
+    rs.hops = rs.sset[0].hops;
     rs.L.resize(K);
     for (int l = 1; l <= K; ++l) {
       Layer& L = rs.L[l - 1];
@@ -323,6 +331,11 @@ apt_status apt_trainer_destroy(apt_trainer* t) {
   cudaStreamSynchronize(t->ctx->stream);
   if (t->gexec) cudaGraphExecDestroy(t->gexec);
   if (t->graph) cudaGraphDestroy(t->graph);
+  for (int p = 0; p < 2; ++p)
+    for (int u = 0; u < 2; ++u) {
+      if (t->gexec_p[p][u]) cudaGraphExecDestroy(t->gexec_p[p][u]);
+      if (t->graph_p[p][u]) cudaGraphDestroy(t->graph_p[p][u]);
+    }
   if (t->gexec_host) cudaGraphExecDestroy(t->gexec_host);
   if (t->graph_host) cudaGraphDestroy(t->graph_host);
   if (t->hb_pinned) cudaFreeHost(t->hb_pinned);
@@ -390,6 +403,7 @@ apt_status apt_trainer_set_epoch(apt_trainer* t, const int64_t* train, int64_t n
   if (!t->perm || n_train > t->n_train) t->perm = t->arena.alloc<int32_t>(n_train, false);
   t->n_train = n_train;
   t->steps_per_epoch = ceil_div(n_train, int64_t(t->world) * t->m.batch);
+  t->primed = -1;   // a prefetched batch belongs to the previous permutation
   int32_t *tr_dev = nullptr, *tmp_vals = nullptr;
   uint64_t *k_in = nullptr, *k_out = nullptr;
   void* tmp = nullptr;
@@ -418,43 +432,74 @@ int64_t apt_trainer_steps_per_epoch(const apt_trainer* t) { return t ? t->steps_
 
 namespace apt {
 
-// Phase A for one rank: seeds + sampling (+ compaction for every hop but the layer-1 one).
-apt_status phase_sample(apt_trainer* t, RankState& rs, bool from_host_batch) {
+// Phase A for one rank: seeds + sampling (+ compaction for every hop but the layer-1
+// one) into sample set `ss`, on stream `st`.  fork_csc: the block transposes run on the
+// side branch (joined before the backward through ev_csc) instead of on `st`.
+apt_status phase_sample(apt_trainer* t, RankState& rs, SampleSet& ss, bool from_host_batch, cudaStream_t st,
+                        bool fork_csc) {
   apt_ctx* c = t->ctx;
   {
     // seeds of the step: from the epoch permutation, or from the global batch the host
     // copied in (hb_dev = [n, ids...]); chunk r for GDP/NFP, partition r for SNP/DNP
     const bool by_part = (t->s == APT_SNP || t->s == APT_DNP) && t->world > 1;
-    SeedArgs sa{from_host_batch ? t->hb_dev + 1 : t->perm, t->n_train, t->step_dev, t->steps_per_epoch, t->world,
-                rs.rank, t->m.batch, by_part ? 1 : 0, t->g->part, rs.seeds, rs.small, rs.small + 1,
+    SeedArgs sa{from_host_batch ? t->hb_dev + 1 : t->perm, t->n_train, ss.step_cell, t->steps_per_epoch, t->world,
+                rs.rank, t->m.batch, by_part ? 1 : 0, t->g->part, ss.seeds, ss.small, ss.small + 1,
                 from_host_batch ? t->hb_dev : nullptr};
-    CK(c, launch_select_seeds(sa, c->stream));
+    CK(c, launch_select_seeds(sa, st));
     c->launches++;
   }
   const int64_t n_words = ceil_div(t->g->n, 32);
   for (int h = 0; h < t->K; ++h) {
-    Hop& hp = rs.hops[h];
+    Hop& hp = ss.hops[h];
     SampleArgs sa{t->g->indptr, t->g->indices, hp.dst, hp.n_dst, hp.max_dst, hp.k,
-                  philox_key(t->m.sample_seed, kDomSample), t->step_dev, h, hp.cnt, hp.nbr};
-    CK(c, launch_sample(sa, c->stream));
+                  philox_key(t->m.sample_seed, kDomSample), ss.step_cell, h, hp.cnt, hp.nbr};
+    CK(c, launch_sample(sa, st));
     c->launches++;
     if (h + 1 < t->K) {
       CompactArgs ca{hp.dst, hp.n_dst, hp.max_dst, hp.cnt, hp.nbr, hp.k, rs.dst_bm, rs.new_bm, n_words, rs.pos, hp.src,
                      hp.counts, hp.indptr, hp.indices, hp.counts + 1, rs.partials, hp.part2};
-      CK(c, launch_compact(ca, c->stream));
+      CK(c, launch_compact(ca, st));
       c->launches += 3;
-      // transpose of this block for the pull-form mean backward: a side branch that
-      // overlaps the rest of the forward (joined before the backward, ev_csc)
-      CK(c, cudaEventRecord(c->ev_fork, c->stream));
-      CK(c, cudaStreamWaitEvent(c->side, c->ev_fork, 0));
+      // transpose of this block for the pull-form mean backward
+      cudaStream_t cs_st = st;
+      if (fork_csc) {
+        CK(c, cudaEventRecord(c->ev_fork, st));
+        CK(c, cudaStreamWaitEvent(c->side, c->ev_fork, 0));
+        cs_st = c->side;
+      }
       CscArgs cs{hp.indptr, hp.indices, hp.n_dst, hp.max_dst, hp.counts + 1, hp.max_dst * hp.k, hp.counts,
                  hp.max_src, hp.csc_cnt, hp.csc_ptr, hp.counts + 2, hp.csc_dst, hp.csc_ws};
-      CK(c, launch_csc_build(cs, c->side));
+      CK(c, launch_csc_build(cs, cs_st));
       c->launches += 4;
     }
   }
-  if (t->K > 1) CK(c, cudaEventRecord(c->ev_csc, c->side));
+  if (fork_csc && t->K > 1) {
+    CK(c, cudaEventRecord(c->ev_csc, c->side));
+    t->csc_forked = true;
+  }
   return APT_OK;
+}
+
+apt_status sample_all(apt_trainer* t, int q, bool host_batch, cudaStream_t st, bool fork_csc) {
+  for (auto& rs : t->R) {
+    apt_status s = phase_sample(t, rs, rs.sset[q], host_batch, st, fork_csc);
+    if (s != APT_OK) return s;
+  }
+  return APT_OK;
+}
+
+// Make sample set q the one the compute phases read (host-side pointer switch; a
+// captured graph keeps the pointers of its parity).
+void activate(apt_trainer* t, int q) {
+  for (auto& rs : t->R) {
+    SampleSet& ss = rs.sset[q];
+    rs.seeds = ss.seeds;
+    rs.small = ss.small;
+    rs.hops = ss.hops;
+    for (int l = 1; l <= t->K; ++l) rs.L[l - 1].n_rows = ss.hops[t->K - l].n_dst;
+  }
+  t->step_dev = t->step_cells + q;
+  t->parity = q;
 }
 
 // GDP layer-1 forward on one rank: fused gather (local + peer rows) + mean, projection.
@@ -534,7 +579,7 @@ apt_status upper_bwd(apt_trainer* t, RankState& rs) {
     // dH_{l-1}: every source row of the layer-l block pulls its in-edges' dZ / deg
     // (transpose built on the side branch), through the ReLU, straight to G (fp32 mode)
     // or its bf16 copy (bf16 mode)
-    if (l == t->K) CK(c, cudaStreamWaitEvent(c->stream, c->ev_csc, 0));
+    if (l == t->K && t->csc_forked) CK(c, cudaStreamWaitEvent(c->stream, c->ev_csc, 0));
     // ReLU bits of H_{l-1} exist when its projection ran on this rank's tcgen05 path
     const bool l1_local = l - 1 > 1 || t->world == 1 || t->s == APT_GDP;
     const uint16_t* mk = (bf && P.Mk && l1_local && tc_gemm_supported(P.d_out, P.d_in)) ? P.Mk : nullptr;
@@ -613,14 +658,44 @@ apt_status allreduce_sgd(apt_trainer* t, int update) {
   return APT_OK;
 }
 
-apt_status step_body(apt_trainer* t, int update, bool host_batch) {
+apt_status compute_body(apt_trainer* t, int update);
+
+// Unpipelined step on sample set q: sampling on the main stream (transposes forked),
+// then the compute phases.
+apt_status step_body(apt_trainer* t, int update, bool host_batch, int q = 0) {
+  apt_ctx* c = t->ctx;
+  CK(c, record_ev(t, 0));
+  t->csc_forked = false;
+  apt_status s = sample_all(t, q, host_batch, c->stream, true);
+  if (s != APT_OK) return s;
+  activate(t, q);
+  return compute_body(t, update);
+}
+
+// Pipelined step: compute on set p while the next step (id `next` is the value of the
+// set_step node, patched per replay) is sampled into set p^1 on the sampling stream.
+apt_status pipelined_body(apt_trainer* t, int p, int update, uint64_t next) {
+  apt_ctx* c = t->ctx;
+  CK(c, record_ev(t, 0));
+  CK(c, cudaEventRecord(c->ev_pfork, c->stream));
+  CK(c, cudaStreamWaitEvent(c->samp, c->ev_pfork, 0));
+  set_step_kernel<<<1, 1, 0, c->samp>>>(t->step_cells + (p ^ 1), next);
+  CK(c, cudaGetLastError());
+  c->launches++;
+  apt_status s = sample_all(t, p ^ 1, false, c->samp, false);
+  if (s != APT_OK) return s;
+  CK(c, cudaEventRecord(c->ev_pjoin, c->samp));
+  t->csc_forked = false;
+  activate(t, p);
+  s = compute_body(t, update);
+  if (s != APT_OK) return s;
+  CK(c, cudaStreamWaitEvent(c->stream, c->ev_pjoin, 0));   // next step's batch complete
+  return APT_OK;
+}
+
+apt_status compute_body(apt_trainer* t, int update) {
   apt_ctx* c = t->ctx;
   const bool gdp = t->world == 1 || t->s == APT_GDP;
-  CK(c, record_ev(t, 0));
-  for (auto& rs : t->R) {
-    apt_status s = phase_sample(t, rs, host_batch);
-    if (s != APT_OK) return s;
-  }
   CK(c, record_ev(t, 1));
   if (gdp) {
     bool first = true;
@@ -679,13 +754,16 @@ apt_status apt_layer_fwd(apt_trainer* t, int64_t step) {
   if (!t || !t->perm) return set_err(t ? t->ctx : nullptr, APT_E_STATE, "apt_layer_fwd: call apt_trainer_set_epoch first");
   apt_ctx* c = t->ctx;
   if (c->broken) return set_err(c, APT_E_STATE, "ctx is broken by an earlier CUDA error");
-  set_step_kernel<<<1, 1, 0, c->stream>>>(t->step_dev, uint64_t(step));
+  t->primed = -1;   // sample set 0 is overwritten
+  set_step_kernel<<<1, 1, 0, c->stream>>>(t->step_cells, uint64_t(step));
   CK(c, cudaGetLastError());
   c->launches++;
-  for (auto& rs : t->R) {
-    apt_status s = phase_sample(t, rs, false);
+  t->csc_forked = false;
+  {
+    apt_status s = sample_all(t, 0, false, c->stream, false);
     if (s != APT_OK) return s;
   }
+  activate(t, 0);
   apt_status s = APT_OK;
   if (t->world == 1 || t->s == APT_GDP) {
     bool first = true;
@@ -698,7 +776,6 @@ apt_status apt_layer_fwd(apt_trainer* t, int64_t step) {
     s = layer1_fwd_strategy(t);
     if (s != APT_OK) return s;
   }
-  if (t->K > 1) CK(c, cudaStreamWaitEvent(c->stream, c->ev_csc, 0));   // join the side branch
   return APT_OK;
 }
 
@@ -744,41 +821,92 @@ apt_status apt_trainer_step(apt_trainer* t, int64_t step, int update) {
   if (!t || !t->perm) return set_err(t ? t->ctx : nullptr, APT_E_STATE, "apt_trainer_step: call apt_trainer_set_epoch first");
   apt_ctx* c = t->ctx;
   if (c->broken) return set_err(c, APT_E_STATE, "ctx is broken by an earlier CUDA error");
+  update = update ? 1 : 0;
+  if (!t->pipeline) {
+    // one stream: sampling, then compute, on sample set 0
+    t->primed = -1;
+    if (t->use_graph) {
+      if (!t->gexec || t->graph_update != update) {
+        if (t->gexec) { cudaGraphExecDestroy(t->gexec); t->gexec = nullptr; }
+        if (t->graph) { cudaGraphDestroy(t->graph); t->graph = nullptr; }
+        cudaGraph_t graph;
+        CK(c, cudaStreamBeginCapture(c->stream, cudaStreamCaptureModeThreadLocal));
+        set_step_kernel<<<1, 1, 0, c->stream>>>(t->step_cells, uint64_t(step));
+        const int64_t l0 = c->launches;
+        t->capturing = true;
+        apt_status s = step_body(t, update, false, 0);
+        t->capturing = false;
+        cudaError_t e = cudaStreamEndCapture(c->stream, &graph);
+        t->launches_per_step = c->launches - l0 + 1;   // counted at replay, not at capture
+        c->launches = l0;
+        if (s != APT_OK) return s;
+        CK(c, e);
+        t->step_node = find_step_node(graph);
+        if (!t->step_node) { cudaGraphDestroy(graph); return set_err(c, APT_E_CUDA, "step node not found in graph"); }
+        CK(c, cudaGraphInstantiate(&t->gexec, graph, 0));
+        t->graph = graph;
+        t->graph_update = update;
+      }
+      CK(c, patch_step_node(t->gexec, t->step_node, t->step_cells, uint64_t(step)));
+      CK(c, cudaGraphLaunch(t->gexec, c->stream));
+      c->launches += t->launches_per_step;
+      return APT_OK;
+    }
+    set_step_kernel<<<1, 1, 0, c->stream>>>(t->step_cells, uint64_t(step));
+    CK(c, cudaGetLastError());
+    c->launches++;
+    return step_body(t, update, false, 0);
+  }
+  // pipelined: this step's batch was sampled during the previous step (else sample it now)
+  int p;
+  if (t->primed == step) {
+    p = t->primed_parity;
+  } else {
+    p = t->parity ^ 1;
+    set_step_kernel<<<1, 1, 0, c->stream>>>(t->step_cells + p, uint64_t(step));
+    CK(c, cudaGetLastError());
+    c->launches++;
+    t->csc_forked = false;
+    apt_status s = sample_all(t, p, false, c->stream, false);
+    if (s != APT_OK) return s;
+  }
+  const uint64_t next = uint64_t(step + 1);
   if (t->use_graph) {
-    if (!t->gexec || t->graph_update != update) {
-      if (t->gexec) { cudaGraphExecDestroy(t->gexec); t->gexec = nullptr; }
-      if (t->graph) { cudaGraphDestroy(t->graph); t->graph = nullptr; }
+    if (!t->gexec_p[p][update]) {
       cudaGraph_t graph;
       CK(c, cudaStreamBeginCapture(c->stream, cudaStreamCaptureModeThreadLocal));
-      set_step_kernel<<<1, 1, 0, c->stream>>>(t->step_dev, uint64_t(step));
       const int64_t l0 = c->launches;
       t->capturing = true;
-      apt_status s = step_body(t, update, false);
+      apt_status s = pipelined_body(t, p, update, next);
       t->capturing = false;
       cudaError_t e = cudaStreamEndCapture(c->stream, &graph);
-      t->launches_per_step = c->launches - l0 + 1;   // counted at replay, not at capture
+      t->launches_p[p][update] = c->launches - l0;
       c->launches = l0;
       if (s != APT_OK) return s;
       CK(c, e);
-      // find the set_step node so replays can patch the step id
-      t->step_node = find_step_node(graph);
-      if (!t->step_node) { cudaGraphDestroy(graph); return set_err(c, APT_E_CUDA, "step node not found in graph"); }
-      CK(c, cudaGraphInstantiate(&t->gexec, graph, 0));
-      t->graph = graph;
-      t->graph_update = update;
+      t->step_node_p[p][update] = find_step_node(graph);
+      if (!t->step_node_p[p][update]) { cudaGraphDestroy(graph); return set_err(c, APT_E_CUDA, "step node not found in graph"); }
+      CK(c, cudaGraphInstantiate(&t->gexec_p[p][update], graph, 0));
+      t->graph_p[p][update] = graph;
     }
-    CK(c, patch_step_node(t->gexec, t->step_node, t->step_dev, uint64_t(step)));
-    CK(c, cudaGraphLaunch(t->gexec, c->stream));
-    c->launches += t->launches_per_step;
-    return APT_OK;
+    activate(t, p);   // readouts after the step see the computed set
+    CK(c, patch_step_node(t->gexec_p[p][update], t->step_node_p[p][update], t->step_cells + (p ^ 1), next));
+    CK(c, cudaGraphLaunch(t->gexec_p[p][update], c->stream));
+    c->launches += t->launches_p[p][update];
+  } else {
+    apt_status s = pipelined_body(t, p, update, next);
+    if (s != APT_OK) return s;
   }
-  set_step_kernel<<<1, 1, 0, c->stream>>>(t->step_dev, uint64_t(step));
-  CK(c, cudaGetLastError());
-  const int64_t l0 = c->launches;
-  c->launches++;
-  apt_status s = step_body(t, update, false);
-  t->launches_per_step = c->launches - l0;
-  return s;
+  t->primed = step + 1;
+  t->primed_parity = p ^ 1;
+  return APT_OK;
+}
+
+apt_status apt_trainer_set_pipeline(apt_trainer* t, int enable) {
+  if (!t) return set_err(nullptr, APT_E_INVALID, "null trainer");
+  t->pipeline = enable != 0;
+  t->primed = -1;
+  return APT_OK;
 }
 
 apt_status apt_trainer_step_host(apt_trainer* t, const int64_t* gbatch, int64_t n_global, int64_t step, int update,
@@ -796,10 +924,11 @@ apt_status apt_trainer_step_host(apt_trainer* t, const int64_t* gbatch, int64_t 
     t->hb_pinned[1 + i] = int32_t(u);
   }
   const size_t hb_bytes = sizeof(int32_t) * (1 + size_t(t->world) * t->m.batch);
+  t->primed = -1;   // sample set 0 is overwritten
   // H2D batch -> step -> D2H per-rank losses, one stream-ordered sequence (one graph replay)
   auto body = [&]() -> apt_status {
     CK(c, cudaMemcpyAsync(t->hb_dev, t->hb_pinned, hb_bytes, cudaMemcpyHostToDevice, c->stream));
-    set_step_kernel<<<1, 1, 0, c->stream>>>(t->step_dev, uint64_t(step));
+    set_step_kernel<<<1, 1, 0, c->stream>>>(t->step_cells, uint64_t(step));
     CK(c, cudaGetLastError());
     apt_status s = step_body(t, update, true);
     if (s != APT_OK) return s;
@@ -829,7 +958,7 @@ apt_status apt_trainer_step_host(apt_trainer* t, const int64_t* gbatch, int64_t 
       t->graph_host_update = update;
       t->launches_per_step_host = per;
     }
-    CK(c, patch_step_node(t->gexec_host, t->step_node_host, t->step_dev, uint64_t(step)));
+    CK(c, patch_step_node(t->gexec_host, t->step_node_host, t->step_cells, uint64_t(step)));
     CK(c, cudaGraphLaunch(t->gexec_host, c->stream));
     c->launches += t->launches_per_step_host;
   } else {

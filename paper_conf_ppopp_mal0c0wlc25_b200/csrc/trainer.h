@@ -74,10 +74,21 @@ struct Xchg {
   float* dW1s = nullptr;             // [d_out x w_cols]
 };
 
+// The sampled mini-batch of one step (seeds, K hops, block transposes).  Two per
+// rank: step t+1 is sampled into one while step t computes on the other.
+struct SampleSet {
+  int32_t* seeds = nullptr;
+  int32_t* small = nullptr;         // [0] n_seeds [1] n_global
+  uint64_t* step_cell = nullptr;    // step id of the batch held here (Philox key of its samples)
+  std::vector<Hop> hops;
+};
+
 struct RankState {
   int rank = 0;
+  SampleSet sset[2];
+  // the set the current step computes on (copies of sset[active]'s fields)
   int32_t* seeds = nullptr;
-  int32_t* small = nullptr;         // [0] n_seeds [1] n_global ...
+  int32_t* small = nullptr;
   std::vector<Hop> hops;
   std::vector<Layer> L;
   uint32_t* dst_bm = nullptr;
@@ -100,7 +111,8 @@ struct apt_trainer {
   int32_t* labels = nullptr;
   int32_t* perm = nullptr;
   int64_t n_train = 0, steps_per_epoch = 1;
-  uint64_t* step_dev = nullptr;
+  uint64_t* step_cells = nullptr;    // [2] step id of the batch in sample set 0 / 1
+  uint64_t* step_dev = nullptr;      // step cell of the set being computed (sset[parity].step_cell)
   std::vector<apt::RankState> R;
   // device pointer tables for cross-rank kernels (peer pointers in a multi-GPU job)
   float** dW_tab = nullptr;
@@ -113,6 +125,16 @@ struct apt_trainer {
   int32_t** wgid_tab = nullptr;
   bool use_graph = false;
   bool capturing = false;
+  // pipelining: step t+1 is sampled on ctx->samp while step t computes
+  bool pipeline = true;
+  int parity = 0;                    // sample set the last step computed on
+  int64_t primed = -1;               // step id already sampled into sset[primed_parity]
+  int primed_parity = 0;
+  bool csc_forked = false;           // this step's block transposes run on the side branch (wait ev_csc)
+  cudaGraphExec_t gexec_p[2][2] = {};   // [parity][update] pipelined step graphs
+  cudaGraph_t graph_p[2][2] = {};
+  cudaGraphNode_t step_node_p[2][2] = {};
+  int64_t launches_p[2][2] = {};
   cudaGraphExec_t gexec = nullptr;
   cudaGraphExec_t gexec_host = nullptr;   // the end-to-end step: H2D batch, step, D2H loss
   cudaGraph_t graph_host = nullptr;

@@ -225,6 +225,34 @@ def test_train_step_matches_oracle(A, ctx, tiny, dtype, step):
         assert np.allclose(tr.read("db", l)[0], db, **tol), f"db layer {l}"
 
 
+@pytest.mark.parametrize("strategy,C", [("GDP", 1), ("SNP", 2), ("NFP", 2), ("DNP", 2)])
+def test_pipelined_steps_equal_unpipelined(A, tiny, strategy, C):
+    """Sampling step t+1 during step t (two sample sets, second stream) changes nothing:
+    eager/graph x pipelined/unpipelined give the same parameters after 4 updates, with a
+    non-sequential step id in the middle (the prefetch is discarded and redone)."""
+    cfg, g, train = tiny
+    outs = []
+    for use_graph, pipe in ((False, False), (True, False), (False, True), (True, True)):
+        ctx = A.Ctx(-1, C, 0) if C > 1 else A.Ctx(0, 1, 0)
+        gr = ctx.graph_load(g.indptr, g.indices, aptgen.partition(g.n, C))
+        fs = ctx.fstore_create(gr, A.NFP if strategy == "NFP" else A.GDP, A.F32, cfg.dim, None, cfg.feat_seed)
+        dims = [cfg.dim] + [d for _, d in cfg.dims()]
+        tr = A.Trainer(ctx, gr, fs, dims, cfg.fanouts, cfg.batch, A.F32, 0.3, cfg.sample_seed, cfg.feat_seed,
+                       A.STRATEGY[strategy], aptgen.labels(cfg, g.n))
+        tr.set_params(aptgen.weights(cfg))
+        tr.set_epoch(train, 0)
+        tr.use_graph(use_graph)
+        tr.set_pipeline(pipe)
+        spe = tr.steps_per_epoch()
+        for s in (0, 1, 0, 1 % spe):
+            tr.step(s % spe, update=True)
+        outs.append((tr.get_params(), tr.read("seeds")[:, 0]))
+    for params, seeds in outs[1:]:
+        assert np.array_equal(seeds, outs[0][1])
+        for (W0, b0), (W1, b1) in zip(outs[0][0], params):
+            assert np.allclose(W0, W1, rtol=1e-5, atol=1e-6) and np.allclose(b0, b1, rtol=1e-5, atol=1e-6)
+
+
 def test_sgd_update_and_graph_replay(A, ctx, tiny):
     """Two steps with the update, eager vs CUDA-graph replay: identical parameters."""
     cfg, g, train = tiny
