@@ -181,7 +181,9 @@ def run_apt(args, cfg):
         else:
             dist.init_process_group("nccl", device_id=torch.device("cuda", local))
     # one non-default stream shared by torch (events, L2 flush) and the library
-    stream = torch.cuda.Stream()
+    # high priority: the library's sampling stream (next step's batch) runs at default
+    # priority and fills the gaps the compute chain leaves
+    stream = torch.cuda.Stream(priority=-1)
     torch.cuda.set_stream(stream)
     A.lib()   # fails loudly if libapt.so is missing: there is no CPU path
 
@@ -275,6 +277,7 @@ def run_apt(args, cfg):
         "metric": METRIC, "value": value, "unit": "seeds/s", "n_gpus": world, "steps": K, "warmup": args.warmup,
         "ms_per_step": ms, "higher_is_better": True, "scaling": "weak", "vs_baseline": None,
         "dtype": args.dtype, "data": "synthetic",
+        "epoch_s": spe * ms / 1e3, "steps_per_epoch": spe,
         "config": dict(workload_config(cfg), strategy=args.strategy, parallelism=f"{args.strategy.lower()}{world}",
                        global_batch=B, l2="flushed between timed steps (256 MB write); inputs also > L2",
                        cuda_graph=not args.no_graph),

@@ -85,14 +85,18 @@ apt_status apt_ctx_create(int rank, int world, int device, void* stream, apt_ctx
     delete c;
     return APT_E_UNSUPPORTED;
   }
+  // priorities: the step's chain and its side branch high, the next step's sampling
+  // (pipelined trainer) at the lowest priority so it only fills idle SM slots
+  int prio_lo = 0, prio_hi = 0;
+  cudaDeviceGetStreamPriorityRange(&prio_lo, &prio_hi);
   if (stream) {
     c->stream = static_cast<cudaStream_t>(stream);
   } else {
-    cudaStreamCreateWithFlags(&c->stream, cudaStreamNonBlocking);
+    cudaStreamCreateWithPriority(&c->stream, cudaStreamNonBlocking, prio_hi);
     c->own_stream = true;
   }
-  cudaStreamCreateWithFlags(&c->side, cudaStreamNonBlocking);
-  cudaStreamCreateWithFlags(&c->samp, cudaStreamNonBlocking);
+  cudaStreamCreateWithPriority(&c->side, cudaStreamNonBlocking, prio_hi);
+  cudaStreamCreateWithPriority(&c->samp, cudaStreamNonBlocking, prio_lo);
   cudaEventCreateWithFlags(&c->ev_pfork, cudaEventDisableTiming);
   cudaEventCreateWithFlags(&c->ev_pjoin, cudaEventDisableTiming);
   cudaEventCreateWithFlags(&c->ev_fork, cudaEventDisableTiming);
