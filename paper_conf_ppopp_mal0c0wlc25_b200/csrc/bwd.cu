@@ -41,11 +41,12 @@ __global__ void csc_fill_kernel(const int32_t* __restrict__ indptr, const int32_
 
 cudaError_t launch_csc_build(const CscArgs& a, cudaStream_t st) {
   const int64_t T = 256;
-  const int64_t ge = std::max<int64_t>(1, std::min<int64_t>(ceil_div(a.max_edges, T), 148 * 16));
+  const int64_t cap = a.grid_cap > 0 ? a.grid_cap : 148 * 16;
+  const int64_t ge = std::max<int64_t>(1, std::min<int64_t>(ceil_div(a.max_edges, T), cap));
   launch_pdl(csc_count_kernel, dim3(ge), dim3(T), 0, st, a.indptr, a.indices, a.n_edges, a.cnt);
   cudaError_t e = launch_scan_counts(a.cnt, a.n_src, a.max_src, a.csc_ptr, a.csc_total, a.ws, st);
   if (e != cudaSuccess) return e;
-  const int64_t gd = std::max<int64_t>(1, std::min<int64_t>(ceil_div(a.max_dst, T), 148 * 16));
+  const int64_t gd = std::max<int64_t>(1, std::min<int64_t>(ceil_div(a.max_dst, T), cap));
   launch_pdl(csc_fill_kernel, dim3(gd), dim3(T), 0, st, a.indptr, a.indices, a.n_dst, a.csc_ptr, a.cnt, a.csc_dst);
   return cudaGetLastError();
 }

@@ -18,6 +18,7 @@ struct SampleArgs {
   int hop;
   int32_t* cnt;                // [max_frontier]
   int32_t* nbr;                // [max_frontier * k] global ids, fixed stride k
+  int64_t grid_cap;            // max blocks (0: default) -- background sampling uses few SMs
 };
 cudaError_t launch_sample(const SampleArgs& a, cudaStream_t st);
 
@@ -39,6 +40,7 @@ struct CompactArgs {
   int32_t* n_edges;
   int32_t* partials;           // scan workspace (>= n_words/2048 + 2)
   int32_t* partials2;          // scan workspace (>= max_dst/2048 + 2)
+  int64_t grid_cap;            // max blocks of the grid-stride kernels (0: default)
 };
 cudaError_t launch_compact(const CompactArgs& a, cudaStream_t st);
 
@@ -127,6 +129,7 @@ struct CscArgs {
   int32_t* csc_total;  // [1]
   int32_t* csc_dst;    // [max_edges]
   int32_t* ws;         // scan workspace, >= 2*ceil(max_src/2048) + 8
+  int64_t grid_cap;    // max blocks of the grid-stride kernels (0: default)
 };
 cudaError_t launch_csc_build(const CscArgs& a, cudaStream_t st);
 

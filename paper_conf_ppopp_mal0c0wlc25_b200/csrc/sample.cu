@@ -92,7 +92,7 @@ cudaError_t launch_sample(const SampleArgs& a, cudaStream_t st) {
   const int threads = 256;
   const int64_t warps = a.max_frontier;
   int64_t blocks = ceil_div(warps * 32, threads);
-  blocks = std::max<int64_t>(1, std::min<int64_t>(blocks, 148 * 16));
+  blocks = std::max<int64_t>(1, std::min<int64_t>(blocks, a.grid_cap > 0 ? a.grid_cap : 148 * 16));
   const int ks = int(ceil_div(a.k, 32));
 #define APT_SAMPLE_CASE(KS)                                                                      \
   case KS:                                                                                       \
@@ -370,12 +370,13 @@ cudaError_t launch_compact(const CompactArgs& a, cudaStream_t st) {
   uint64_t* stA = reinterpret_cast<uint64_t*>(a.partials);            // >= 2*nbA + 8 int32
   int32_t* ticket = a.partials + 2 * nbA + 2;
   uint64_t* stB = reinterpret_cast<uint64_t*>(a.partials2);           // >= 2*nbB + 8 int32
-  launch_pdl(compact_mark_kernel, dim3(grid_for(a.max_dst * a.k, T)), dim3(T), 0, st, a.dst, a.n_dst, a.cnt, a.nbr, a.k, a.dst_bm,
+  const int64_t gm = a.grid_cap > 0 ? std::min<int64_t>(a.grid_cap, grid_for(a.max_dst * a.k, T)) : grid_for(a.max_dst * a.k, T);
+  launch_pdl(compact_mark_kernel, dim3(gm), dim3(T), 0, st, a.dst, a.n_dst, a.cnt, a.nbr, a.k, a.dst_bm,
                                                                    a.new_bm, a.pos, a.src, stA, nbA, stB, nbB, ticket);
   NewBitsOp bop{a.new_bm, a.dst_bm, a.n_words, a.n_dst, a.src, a.pos, a.n_src};
   CntScanOp cop{a.cnt, a.n_dst, a.indptr, a.n_edges};
   launch_pdl(compact_scan_kernel, dim3(nbA + nbB), dim3(kScanThreads), 0, st, bop, stA, nbA, cop, stB, nbB, ticket);
-  launch_pdl(map_indices_kernel, dim3(grid_for(a.max_dst * a.k, T)), dim3(T), 0, st, a.dst, a.cnt, a.nbr, a.n_dst, a.k, a.indptr,
+  launch_pdl(map_indices_kernel, dim3(gm), dim3(T), 0, st, a.dst, a.cnt, a.nbr, a.n_dst, a.k, a.indptr,
                                                                   a.pos, a.indices, a.dst_bm);
   return cudaGetLastError();
 }

@@ -11,6 +11,7 @@
 // Every count stays on the device, every grid is sized by an upper bound:
 // the step issues no host synchronisation and can be replayed as a CUDA graph.
 #include <algorithm>
+#include <cstdlib>
 #include <vector>
 #include <cstring>
 #include <cub/device/device_radix_sort.cuh>
@@ -438,6 +439,13 @@ namespace apt {
 apt_status phase_sample(apt_trainer* t, RankState& rs, SampleSet& ss, bool from_host_batch, cudaStream_t st,
                         bool fork_csc) {
   apt_ctx* c = t->ctx;
+  // background sampling (the next step, pipelined) is confined to a few blocks per SM so
+  // that it fills gaps instead of competing with the step's chain for every SM
+  static const int64_t bg_cap = [] {
+    const char* v = std::getenv("APT_BG_BLOCKS_PER_SM");
+    return int64_t(148) * (v ? std::max(1, atoi(v)) : 4);
+  }();
+  const int64_t cap = st == c->samp ? bg_cap : 0;
   {
     // seeds of the step: from the epoch permutation, or from the global batch the host
     // copied in (hb_dev = [n, ids...]); chunk r for GDP/NFP, partition r for SNP/DNP
@@ -452,12 +460,12 @@ apt_status phase_sample(apt_trainer* t, RankState& rs, SampleSet& ss, bool from_
   for (int h = 0; h < t->K; ++h) {
     Hop& hp = ss.hops[h];
     SampleArgs sa{t->g->indptr, t->g->indices, hp.dst, hp.n_dst, hp.max_dst, hp.k,
-                  philox_key(t->m.sample_seed, kDomSample), ss.step_cell, h, hp.cnt, hp.nbr};
+                  philox_key(t->m.sample_seed, kDomSample), ss.step_cell, h, hp.cnt, hp.nbr, cap};
     CK(c, launch_sample(sa, st));
     c->launches++;
     if (h + 1 < t->K) {
       CompactArgs ca{hp.dst, hp.n_dst, hp.max_dst, hp.cnt, hp.nbr, hp.k, rs.dst_bm, rs.new_bm, n_words, rs.pos, hp.src,
-                     hp.counts, hp.indptr, hp.indices, hp.counts + 1, rs.partials, hp.part2};
+                     hp.counts, hp.indptr, hp.indices, hp.counts + 1, rs.partials, hp.part2, cap};
       CK(c, launch_compact(ca, st));
       c->launches += 3;
       // transpose of this block for the pull-form mean backward
@@ -468,7 +476,7 @@ apt_status phase_sample(apt_trainer* t, RankState& rs, SampleSet& ss, bool from_
         cs_st = c->side;
       }
       CscArgs cs{hp.indptr, hp.indices, hp.n_dst, hp.max_dst, hp.counts + 1, hp.max_dst * hp.k, hp.counts,
-                 hp.max_src, hp.csc_cnt, hp.csc_ptr, hp.counts + 2, hp.csc_dst, hp.csc_ws};
+                 hp.max_src, hp.csc_cnt, hp.csc_ptr, hp.counts + 2, hp.csc_dst, hp.csc_ws, cap};
       CK(c, launch_csc_build(cs, cs_st));
       c->launches += 4;
     }
