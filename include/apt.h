@@ -224,6 +224,13 @@ apt_status apt_trainer_step(apt_trainer* t, int64_t step, int update);
  * Syncs.                                                                    */
 apt_status apt_trainer_step_host(apt_trainer* t, const int64_t* gbatch_host, int64_t n_global, int64_t step,
                                  int update, float* loss_host);
+/* Pipelined end-to-end call: submit the NEXT global batch (host int64 ids, step id
+ * next_step) and run the step of the batch the previous call submitted, returning
+ * its loss in *loss_prev (*had_step = 1).  The next batch's H2D copy and sampling
+ * overlap the step (second sample set, sampling stream).  The first call only
+ * primes (*had_step = 0).  Syncs.                                           */
+apt_status apt_trainer_step_host_pipelined(apt_trainer* t, const int64_t* next_batch, int64_t n_next,
+                                           int64_t next_step, int update, float* loss_prev, int* had_step);
 /* Loss of the last step (sum over ranks).  Syncs.                           */
 apt_status apt_trainer_loss(apt_trainer* t, float* loss);
 /* Record/replay the device part of apt_trainer_step as a CUDA graph.        */

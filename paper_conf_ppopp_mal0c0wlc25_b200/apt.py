@@ -106,6 +106,7 @@ def lib():
             "apt_trainer_set_params": [vp, i32, vp, vp], "apt_trainer_get_params": [vp, i32, i32, vp, vp],
             "apt_trainer_set_epoch": [vp, vp, i64, u64], "apt_trainer_step": [vp, i64, i32],
             "apt_trainer_step_host": [vp, vp, i64, i64, i32, vp], "apt_trainer_loss": [vp, vp],
+            "apt_trainer_step_host_pipelined": [vp, vp, i64, i64, i32, vp, vp],
             "apt_trainer_use_graph": [vp, i32], "apt_trainer_set_pipeline": [vp, i32], "apt_trainer_read": [vp, i32, i32, i32, vp, i64, vp, vp],
             "apt_trainer_phase_ms": [vp, vp, i32], "apt_trainer_agg_bytes": [vp, vp],
             "apt_dryrun": [vp, i64, vp], "apt_layer_fwd": [vp, i64], "apt_layer_bwd": [vp, vp, i64], "apt_profile_links": [vp, vp], "apt_select_strategy": [vp, vp, vp, vp],
@@ -316,6 +317,15 @@ class Trainer(Handle):
         self.ctx.ck(lib().apt_trainer_step_host(self.h, _ptr(gbatch_host), len(gbatch_host), step,
                                                 1 if update else 0, C.byref(loss)))
         return loss.value
+
+    def step_host_pipelined(self, next_batch_host, next_step, update=True):
+        """Submit the next host batch, run the previously submitted one; returns its loss
+        (None for the priming call)."""
+        loss, had = C.c_float(0), C.c_int(0)
+        self.ctx.ck(lib().apt_trainer_step_host_pipelined(self.h, _ptr(next_batch_host), len(next_batch_host),
+                                                          next_step, 1 if update else 0, C.byref(loss),
+                                                          C.byref(had)))
+        return loss.value if had.value else None
 
     def loss(self):
         v = C.c_float(0)

@@ -11,6 +11,7 @@
 // Every count stays on the device, every grid is sized by an upper bound:
 // the step issues no host synchronisation and can be replayed as a CUDA graph.
 #include <algorithm>
+#include <cmath>
 #include <cstdlib>
 #include <vector>
 #include <cstring>
@@ -202,8 +203,9 @@ apt_status apt_trainer_create(apt_ctx* c, const apt_graph* g, const apt_fstore* 
   t->labels = A.alloc<int32_t>(g->n, false);
   t->step_cells = A.alloc<uint64_t>(2, true);   // step id of sample set 0 / 1
   t->step_dev = t->step_cells;
-  t->hb_dev = A.alloc<int32_t>(1 + int64_t(C) * m->batch, true);
-  CK(c, cudaMallocHost(reinterpret_cast<void**>(&t->hb_pinned), sizeof(int32_t) * (1 + int64_t(C) * m->batch)));
+  t->hb_len = 1 + int64_t(C) * m->batch;
+  t->hb_dev = A.alloc<int32_t>(2 * t->hb_len, true);
+  CK(c, cudaMallocHost(reinterpret_cast<void**>(&t->hb_pinned), sizeof(int32_t) * 2 * t->hb_len));
   CK(c, cudaMallocHost(reinterpret_cast<void**>(&t->loss_pinned), sizeof(float) * APT_MAX_RANKS));
   CK(c, cudaMemcpyAsync(t->labels, labels, sizeof(int32_t) * g->n, cudaMemcpyHostToDevice, c->stream));
   const int64_t n_words = ceil_div(g->n, 32);
@@ -336,6 +338,8 @@ apt_status apt_trainer_destroy(apt_trainer* t) {
     for (int u = 0; u < 2; ++u) {
       if (t->gexec_p[p][u]) cudaGraphExecDestroy(t->gexec_p[p][u]);
       if (t->graph_p[p][u]) cudaGraphDestroy(t->graph_p[p][u]);
+      if (t->gexec_hp[p][u]) cudaGraphExecDestroy(t->gexec_hp[p][u]);
+      if (t->graph_hp[p][u]) cudaGraphDestroy(t->graph_hp[p][u]);
     }
   if (t->gexec_host) cudaGraphExecDestroy(t->gexec_host);
   if (t->graph_host) cudaGraphDestroy(t->graph_host);
@@ -405,6 +409,7 @@ apt_status apt_trainer_set_epoch(apt_trainer* t, const int64_t* train, int64_t n
   t->n_train = n_train;
   t->steps_per_epoch = ceil_div(n_train, int64_t(t->world) * t->m.batch);
   t->primed = -1;   // a prefetched batch belongs to the previous permutation
+  t->host_primed = false;
   int32_t *tr_dev = nullptr, *tmp_vals = nullptr;
   uint64_t *k_in = nullptr, *k_out = nullptr;
   void* tmp = nullptr;
@@ -450,9 +455,10 @@ apt_status phase_sample(apt_trainer* t, RankState& rs, SampleSet& ss, bool from_
     // seeds of the step: from the epoch permutation, or from the global batch the host
     // copied in (hb_dev = [n, ids...]); chunk r for GDP/NFP, partition r for SNP/DNP
     const bool by_part = (t->s == APT_SNP || t->s == APT_DNP) && t->world > 1;
-    SeedArgs sa{from_host_batch ? t->hb_dev + 1 : t->perm, t->n_train, ss.step_cell, t->steps_per_epoch, t->world,
+    const int32_t* hb = t->hb_dev + (&ss == &rs.sset[1] ? t->hb_len : 0);   // this set's host-batch staging
+    SeedArgs sa{from_host_batch ? hb + 1 : t->perm, t->n_train, ss.step_cell, t->steps_per_epoch, t->world,
                 rs.rank, t->m.batch, by_part ? 1 : 0, t->g->part, ss.seeds, ss.small, ss.small + 1,
-                from_host_batch ? t->hb_dev : nullptr};
+                from_host_batch ? hb : nullptr};
     CK(c, launch_select_seeds(sa, st));
     c->launches++;
   }
@@ -763,6 +769,7 @@ apt_status apt_layer_fwd(apt_trainer* t, int64_t step) {
   apt_ctx* c = t->ctx;
   if (c->broken) return set_err(c, APT_E_STATE, "ctx is broken by an earlier CUDA error");
   t->primed = -1;   // sample set 0 is overwritten
+  t->host_primed = false;
   set_step_kernel<<<1, 1, 0, c->stream>>>(t->step_cells, uint64_t(step));
   CK(c, cudaGetLastError());
   c->launches++;
@@ -830,6 +837,7 @@ apt_status apt_trainer_step(apt_trainer* t, int64_t step, int update) {
   apt_ctx* c = t->ctx;
   if (c->broken) return set_err(c, APT_E_STATE, "ctx is broken by an earlier CUDA error");
   update = update ? 1 : 0;
+  t->host_primed = false;   // the host-batch pipeline's prefetched set may be overwritten
   if (!t->pipeline) {
     // one stream: sampling, then compute, on sample set 0
     t->primed = -1;
@@ -931,8 +939,9 @@ apt_status apt_trainer_step_host(apt_trainer* t, const int64_t* gbatch, int64_t 
     if (u < 0 || u >= t->g->n) return set_err(c, APT_E_INVALID, "step_host: seed %lld out of range", (long long)u);
     t->hb_pinned[1 + i] = int32_t(u);
   }
-  const size_t hb_bytes = sizeof(int32_t) * (1 + size_t(t->world) * t->m.batch);
+  const size_t hb_bytes = sizeof(int32_t) * size_t(t->hb_len);
   t->primed = -1;   // sample set 0 is overwritten
+  t->host_primed = false;
   // H2D batch -> step -> D2H per-rank losses, one stream-ordered sequence (one graph replay)
   auto body = [&]() -> apt_status {
     CK(c, cudaMemcpyAsync(t->hb_dev, t->hb_pinned, hb_bytes, cudaMemcpyHostToDevice, c->stream));
@@ -978,6 +987,98 @@ apt_status apt_trainer_step_host(apt_trainer* t, const int64_t* gbatch, int64_t 
   float tot = 0.f;
   for (size_t i = 0; i < t->R.size(); ++i) tot += t->loss_pinned[i];
   *loss_host = tot;
+  return apt_ctx_sync(c);
+}
+
+// Pipelined end-to-end call: submit the NEXT global batch (host, copied to pinned
+// staging) and run the step of the batch submitted by the previous call; returns that
+// step's loss.  While the step computes, the next batch is copied in and sampled on
+// the sampling stream (one graph replay per call).  The first call only primes (loss
+// NaN, *had_step = 0).
+apt_status apt_trainer_step_host_pipelined(apt_trainer* t, const int64_t* next_batch, int64_t n_next, int64_t next_step,
+                                           int update, float* loss_prev, int* had_step) {
+  if (!t || !next_batch || !loss_prev || !had_step || n_next < 1 || n_next > int64_t(t->world) * t->m.batch)
+    return set_err(t ? t->ctx : nullptr, APT_E_INVALID, "apt_trainer_step_host_pipelined: bad arguments");
+  apt_ctx* c = t->ctx;
+  if (c->broken) return set_err(c, APT_E_STATE, "ctx is broken by an earlier CUDA error");
+  update = update ? 1 : 0;
+  t->primed = -1;
+  const int p = t->host_primed ? t->host_parity : 0;   // set holding the batch to compute
+  const int q = t->host_primed ? p ^ 1 : 0;            // set receiving the next batch
+  int32_t* stage = t->hb_pinned + q * t->hb_len;
+  stage[0] = int32_t(n_next);
+  for (int64_t i = 0; i < n_next; ++i) {
+    const int64_t u = next_batch[i];
+    if (u < 0 || u >= t->g->n) return set_err(c, APT_E_INVALID, "step_host: seed %lld out of range", (long long)u);
+    stage[1 + i] = int32_t(u);
+  }
+  const size_t hb_bytes = sizeof(int32_t) * size_t(t->hb_len);
+  if (!t->host_primed) {   // prime: copy in and sample the first batch into set 0
+    CK(c, cudaMemcpyAsync(t->hb_dev, stage, hb_bytes, cudaMemcpyHostToDevice, c->stream));
+    set_step_kernel<<<1, 1, 0, c->stream>>>(t->step_cells, uint64_t(next_step));
+    CK(c, cudaGetLastError());
+    t->csc_forked = false;
+    apt_status s = sample_all(t, 0, true, c->stream, false);
+    if (s != APT_OK) return s;
+    CK(c, cudaStreamSynchronize(c->stream));
+    t->host_primed = true;
+    t->host_parity = 0;
+    *loss_prev = std::nanf("");
+    *had_step = 0;
+    return apt_ctx_sync(c);
+  }
+  auto body = [&](uint64_t nstep) -> apt_status {
+    CK(c, record_ev(t, 0));
+    CK(c, cudaEventRecord(c->ev_pfork, c->stream));
+    CK(c, cudaStreamWaitEvent(c->samp, c->ev_pfork, 0));
+    CK(c, cudaMemcpyAsync(t->hb_dev + q * t->hb_len, stage, hb_bytes, cudaMemcpyHostToDevice, c->samp));
+    set_step_kernel<<<1, 1, 0, c->samp>>>(t->step_cells + q, nstep);
+    CK(c, cudaGetLastError());
+    apt_status s = sample_all(t, q, true, c->samp, false);
+    if (s != APT_OK) return s;
+    CK(c, cudaEventRecord(c->ev_pjoin, c->samp));
+    t->csc_forked = false;
+    activate(t, p);
+    s = compute_body(t, update);
+    if (s != APT_OK) return s;
+    for (size_t i = 0; i < t->R.size(); ++i)
+      CK(c, cudaMemcpyAsync(t->loss_pinned + i, t->R[i].loss, sizeof(float), cudaMemcpyDeviceToHost, c->stream));
+    CK(c, cudaStreamWaitEvent(c->stream, c->ev_pjoin, 0));
+    return APT_OK;
+  };
+  if (t->use_graph) {
+    if (!t->gexec_hp[p][update]) {
+      cudaGraph_t graph;
+      CK(c, cudaStreamBeginCapture(c->stream, cudaStreamCaptureModeThreadLocal));
+      const int64_t l0 = c->launches;
+      t->capturing = true;
+      apt_status s = body(uint64_t(next_step));
+      t->capturing = false;
+      cudaError_t e = cudaStreamEndCapture(c->stream, &graph);
+      t->launches_hp[p][update] = c->launches - l0 + 1;
+      c->launches = l0;
+      if (s != APT_OK) return s;
+      CK(c, e);
+      t->step_node_hp[p][update] = find_step_node(graph);
+      if (!t->step_node_hp[p][update]) { cudaGraphDestroy(graph); return set_err(c, APT_E_CUDA, "step node not found"); }
+      CK(c, cudaGraphInstantiate(&t->gexec_hp[p][update], graph, 0));
+      t->graph_hp[p][update] = graph;
+    }
+    activate(t, p);
+    CK(c, patch_step_node(t->gexec_hp[p][update], t->step_node_hp[p][update], t->step_cells + q, uint64_t(next_step)));
+    CK(c, cudaGraphLaunch(t->gexec_hp[p][update], c->stream));
+    c->launches += t->launches_hp[p][update];
+  } else {
+    apt_status s = body(uint64_t(next_step));
+    if (s != APT_OK) return s;
+    c->launches++;
+  }
+  CK(c, cudaStreamSynchronize(c->stream));
+  float tot = 0.f;
+  for (size_t i = 0; i < t->R.size(); ++i) tot += t->loss_pinned[i];
+  *loss_prev = tot;
+  *had_step = 1;
+  t->host_parity = q;
   return apt_ctx_sync(c);
 }
 

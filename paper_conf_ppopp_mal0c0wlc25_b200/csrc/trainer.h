@@ -141,8 +141,16 @@ struct apt_trainer {
   cudaGraphNode_t step_node_host = nullptr;
   int graph_host_update = -1;
   int64_t launches_per_step_host = 0;
-  int32_t* hb_pinned = nullptr;       // [1 + C*B] host staging: n, ids (pinned)
-  int32_t* hb_dev = nullptr;          // device copy
+  int32_t* hb_pinned = nullptr;       // [2][1 + C*B] host staging per sample set: n, ids (pinned)
+  int32_t* hb_dev = nullptr;          // [2][1 + C*B] device copies
+  int64_t hb_len = 0;                 // 1 + C*B
+  // pipelined end-to-end calls: batch submitted by the previous call, sampled into set
+  bool host_primed = false;
+  int host_parity = 0;
+  cudaGraphExec_t gexec_hp[2][2] = {};
+  cudaGraph_t graph_hp[2][2] = {};
+  cudaGraphNode_t step_node_hp[2][2] = {};
+  int64_t launches_hp[2][2] = {};
   float* loss_pinned = nullptr;       // [APT_MAX_RANKS] per hosted rank
   cudaGraph_t graph = nullptr;
   cudaGraphNode_t step_node = nullptr;

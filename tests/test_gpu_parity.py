@@ -225,6 +225,31 @@ def test_train_step_matches_oracle(A, ctx, tiny, dtype, step):
         assert np.allclose(tr.read("db", l)[0], db, **tol), f"db layer {l}"
 
 
+@pytest.mark.parametrize("use_graph", [False, True])
+def test_step_host_pipelined_matches_device_steps(A, ctx, tiny, use_graph):
+    """The pipelined end-to-end call (submit batch t+1, run batch t) returns, call by call,
+    the losses of the device-resident steps on the same batches."""
+    cfg, g, train = tiny
+    perm = oracle.epoch_perm(train, cfg.sample_seed, 0)
+    tr, params, labels = _trainer(A, ctx, cfg, g, train, "bf16")
+    tr.use_graph(use_graph)
+    ref = []
+    for step in range(3):
+        tr.step(step, update=False)
+        ref.append(tr.loss())
+    tr2, _, _ = _trainer(A, ctx, cfg, g, train, "bf16")
+    tr2.use_graph(use_graph)
+    got = []
+    for step in range(4):
+        nxt = torch.as_tensor(perm[(step % 3) * cfg.batch:((step % 3) + 1) * cfg.batch]).pin_memory()
+        loss = tr2.step_host_pipelined(nxt, step % 3, update=False)
+        if step == 0:
+            assert loss is None
+        else:
+            got.append(loss)
+    assert np.allclose(got, ref, rtol=1e-6)
+
+
 @pytest.mark.parametrize("strategy,C", [("GDP", 1), ("SNP", 2), ("NFP", 2), ("DNP", 2)])
 def test_pipelined_steps_equal_unpipelined(A, tiny, strategy, C):
     """Sampling step t+1 during step t (two sample sets, second stream) changes nothing:
