@@ -508,3 +508,46 @@ def test_layer_fwd_bwd_api(A, tiny, strategy, C, dtype):
     for r in (0, C - 1):
         assert np.allclose(tr.read("dW", 1, rank=r), dW, rtol=tol["rtol"], atol=atol)
         assert np.allclose(tr.read("db", 1, rank=r)[0], db, rtol=tol["rtol"], atol=atol)
+
+
+@pytest.mark.slow
+def test_products_full_size_layer1_rows_vs_oracle(A, ctx):
+    """BASELINE configs[1] at full size, in the bench's launch configuration (bf16, CUDA graph,
+    pipelined GDP step): layer-1 Z of 300 sampled destinations recomputed one by one by the
+    oracle (Floyd positions -> neighbour rows -> fp64 mean -> bf16) -- bit-exact under O4 -- and their
+    h1 = ReLU(bf16(Z) bf16(W)^T + b) within the bf16 bar."""
+    cfg = aptgen.CONFIGS["products"]
+    g = aptgen.make_graph(cfg)
+    train = aptgen.train_nodes(g, cfg)
+    labels = aptgen.labels(cfg, g.n)
+    gr = ctx.graph_load(g.indptr, g.indices)
+    fs = ctx.fstore_create(gr, A.GDP, A.BF16, cfg.dim, None, cfg.feat_seed)
+    dims = [cfg.dim] + [d for _, d in cfg.dims()]
+    tr = A.Trainer(ctx, gr, fs, dims, cfg.fanouts, cfg.batch, A.BF16, 0.05, cfg.sample_seed, cfg.feat_seed, A.GDP,
+                   labels)
+    params = aptgen.weights(cfg)
+    tr.set_params(params)
+    tr.set_epoch(train, 0)
+    tr.use_graph(True)
+    for step in range(3):
+        tr.step(step, update=False)
+    step = 2
+    dst = tr.read("dst", 1)[:, 0].astype(np.int64)
+    Z = tr.read("Z", 1)
+    H = tr.read("H", 1)
+    rng = np.random.default_rng(0)
+    rows = rng.choice(len(dst), size=300, replace=False)
+    K = len(cfg.fanouts)
+    W1 = oracle.bf16_round(params[0][0].astype(np.float64))
+    b1 = params[0][1].astype(np.float64)
+    for i in rows:
+        v = int(dst[i])
+        deg = int(g.indptr[v + 1] - g.indptr[v])
+        pos = oracle.sample_positions(v, deg, cfg.fanouts[0], cfg.sample_seed, step, K - 1)
+        nbrs = g.indices[g.indptr[v] + pos].astype(np.int64)
+        x = oracle.features(cfg.feat_seed, nbrs, cfg.dim)
+        z = x.mean(axis=0) if len(nbrs) else np.zeros(cfg.dim)
+        zb = oracle.bf16_round(z)                   # bf16 mode stores Z at its bf16 rounding point (O5)
+        assert np.array_equal(Z[i], zb.astype(np.float32)), v
+        h = np.maximum(zb @ W1.T + b1, 0)
+        assert np.allclose(H[i], h, rtol=2e-2, atol=2e-3), v
