@@ -36,6 +36,7 @@
 #include <cuda.h>
 #include <cudaTypedefs.h>
 #include <algorithm>
+#include <cstdlib>
 #include <mutex>
 
 namespace apt {
@@ -139,6 +140,8 @@ struct RowParams {
   int64_t M_max;
   const int32_t* M_dev;
   int N, BN, nkb, tmem_cols, b_mn;
+  int stages;               // A ring depth (<= STAGES)
+  int nacc;                 // TMEM accumulator buffers (2: epilogue overlaps the next tile's MMAs)
   uint32_t b_kb_bytes;      // bytes of one resident B k-block
   const float* bias;
   int relu;
@@ -153,13 +156,13 @@ struct RowParams {
   int64_t mask_pitch;
 };
 
-__global__ void __launch_bounds__(ROW_THREADS, 1)
+__global__ void __launch_bounds__(ROW_THREADS, 2)
     rowtile_kernel(const __grid_constant__ CUtensorMap mapA, const __grid_constant__ CUtensorMap mapB, RowParams p) {
   APT_PDL_PROLOGUE();
   extern __shared__ __align__(1024) uint8_t smem_raw[];
   uint8_t* smem = smem_raw + ((1024u - (smem_u32(smem_raw) & 1023u)) & 1023u);   // 1 KB aligned, still __shared__
-  uint8_t* smem_a = smem;                                        // STAGES x 16 KB
-  uint8_t* smem_b = smem + STAGES * A_STAGE_BYTES;               // nkb x b_kb_bytes
+  uint8_t* smem_a = smem;                                        // stages x 16 KB
+  uint8_t* smem_b = smem + p.stages * A_STAGE_BYTES;             // nkb x b_kb_bytes
   uint64_t* bars = reinterpret_cast<uint64_t*>(smem_b + size_t(p.nkb) * p.b_kb_bytes);
   uint64_t* full = bars;                  // [STAGES]
   uint64_t* empty = bars + STAGES;        // [STAGES]
@@ -176,7 +179,7 @@ __global__ void __launch_bounds__(ROW_THREADS, 1)
 
   if (warp == 0 && lane == 0) {
     for (int s = 0; s < STAGES; ++s) { mbar_init(full + s, 1); mbar_init(empty + s, 1); }
-    mbar_init(bfull, 1);
+    mbar_init(bfull, 1);   // (barrier slots are laid out for the maximum STAGES)
     for (int a = 0; a < 2; ++a) { mbar_init(tfull + a, 1); mbar_init(tempty + a, 256); }
     asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
     asm volatile("prefetch.tensormap [%0];" ::"l"(reinterpret_cast<uint64_t>(&mapA)) : "memory");
@@ -208,7 +211,7 @@ __global__ void __launch_bounds__(ROW_THREADS, 1)
           mbar_wait(empty + s, ph ^ 1);
           mbar_expect_tx(full + s, A_STAGE_BYTES);
           tma_load_2d(smem_a + s * A_STAGE_BYTES, &mapA, full + s, kb * BK, int(t * BM));
-          if (++s == STAGES) { s = 0; ph ^= 1; }
+          if (++s == p.stages) { s = 0; ph ^= 1; }
         }
       }
     }
@@ -238,12 +241,11 @@ __global__ void __launch_bounds__(ROW_THREADS, 1)
             mma_commit(empty + s);            // frees the smem stage when these MMAs finish
           }
           __syncwarp();
-          if (++s == STAGES) { s = 0; ph ^= 1; }
+          if (++s == p.stages) { s = 0; ph ^= 1; }
         }
         if (lane == 0) mma_commit(tfull + acc);   // accumulator ready for the epilogue
         __syncwarp();
-        acc ^= 1;
-        if (acc == 0) aph ^= 1;
+        if (++acc == p.nacc) { acc = 0; aph ^= 1; }
       }
     }
   } else {
@@ -323,8 +325,7 @@ __global__ void __launch_bounds__(ROW_THREADS, 1)
       }
       fence_before();
       mbar_arrive(tempty + acc);
-      acc ^= 1;
-      if (acc == 0) aph ^= 1;
+      if (++acc == p.nacc) { acc = 0; aph ^= 1; }
     }
   }
   fence_before();
@@ -528,9 +529,13 @@ cudaError_t launch_tc_gemm(const TcGemmArgs& a, cudaStream_t st) {
   const int64_t tiles = std::max<int64_t>(1, ceil_div(a.M_max, BM));
   int n_split = 1;
   while (n_split < 4 && tiles * n_split * 2 <= sm_count() && BN_all % (64 * n_split * 2) == 0) n_split *= 2;
+  // forward projections (W K-major): 128-column slices even with many tiles -- with the
+  // 2-CTA/SM mode below this measured 7 us faster on the products layer-1 projection;
+  // the backward dZ (W N-major) measured faster unsplit, single CTA
+  static const int force_split = [] { const char* v = std::getenv("APT_PROJ_SPLIT"); return v ? atoi(v) : -1; }();
+  const int want_split = force_split >= 0 ? force_split : (a.w_mn ? 1 : 2);
+  if (want_split > n_split && BN_all % (64 * want_split) == 0) n_split = want_split;
   const int BN = BN_all / n_split;
-  int cols = 32;
-  while (cols < 2 * BN) cols <<= 1;
   CUtensorMap ma, mb;
   if (!make_map(&ma, a.Z, a.K, std::max<int64_t>(a.M_max, 1), a.z_pitch, BK, BM)) return cudaErrorInvalidValue;
   uint32_t b_kb_bytes;
@@ -542,17 +547,30 @@ cudaError_t launch_tc_gemm(const TcGemmArgs& a, cudaStream_t st) {
     if (!make_map(&mb, a.W, a.K, a.N, a.w_pitch, BK, BN)) return cudaErrorInvalidValue;
     b_kb_bytes = uint32_t(BN) * 128;
   }
-  RowParams p{a.M_max, a.M_dev, a.N, BN, nkb, cols, a.w_mn, b_kb_bytes, a.bias, a.relu, a.Y, a.y_pitch,
+  // two CTAs per SM when they fit (2-stage ring, one TMEM accumulator each): one CTA's
+  // loads and MMAs overlap the other's epilogue
+  static const int two_cta = [] { const char* v = std::getenv("APT_PROJ_2CTA"); return v ? atoi(v) : 0; }();   // off: measured slower end to end (the overlapped sampling then lands on the backward)
+  auto smem_of = [&](int st) {
+    return 1024 + size_t(st) * A_STAGE_BYTES + size_t(nkb) * b_kb_bytes + 16 * 8 + 16 + 8 * 32 * 17 * 4;
+  };
+  int stages = STAGES, nacc = 2, per_sm = 1;
+  if (two_cta && !a.w_mn && smem_of(2) <= 113 * 1024 && BN <= 256 && tiles * n_split > sm_count()) {
+    stages = 2;
+    nacc = 1;
+    per_sm = 2;
+  }
+  int cols = 32;
+  while (cols < nacc * BN) cols <<= 1;
+  RowParams p{a.M_max, a.M_dev, a.N, BN, nkb, cols, a.w_mn, stages, nacc, b_kb_bytes, a.bias, a.relu, a.Y, a.y_pitch,
               a.out_base, a.out_rank, a.out_row, a.accumulate, n_split, a.mask, a.mask_pitch};
-  const size_t smem = 1024 + size_t(STAGES) * A_STAGE_BYTES + size_t(nkb) * b_kb_bytes + 16 * 8 + 16 +
-                      8 * 32 * 17 * 4;   // + epilogue staging
+  const size_t smem = smem_of(stages);   // + epilogue staging
   if (smem > 227 * 1024) return cudaErrorInvalidValue;
   static bool attr_set = false;
   if (!attr_set) {
     cudaFuncSetAttribute(rowtile_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize, 227 * 1024);
     attr_set = true;
   }
-  const int grid = int(std::min<int64_t>(tiles * n_split, (sm_count() / n_split) * n_split));
+  const int grid = int(std::min<int64_t>(tiles * n_split, ((per_sm * sm_count()) / n_split) * n_split));
   launch_pdl(rowtile_kernel, dim3(grid), dim3(ROW_THREADS), smem, st, ma, mb, p);
   return cudaGetLastError();
 }
