@@ -57,6 +57,8 @@ def parse():
     ap.add_argument("--e2e-steps", type=int, default=10)
     ap.add_argument("--no-planner", action="store_true")
     ap.add_argument("--dryrun-steps", type=int, default=8)
+    ap.add_argument("--emulate-max-c", type=int, default=4,
+                    help="also time every strategy with C ranks emulated on the GPU, for C up to this")
     ap.add_argument("--verbose", action="store_true")
     return ap.parse_args()
 
@@ -336,6 +338,8 @@ def planner_report(A, g, cfg, train, labels, args, stream, gdp_ms):
                         "pick": STRATS[pick],
                         "n_vs_per_step": sum(st.n_vs[r] for r in range(C)) / steps,
                         "n_vd_per_step": sum(st.n_vd[r] for r in range(C)) / steps}
+        if C <= args.emulate_max_c:
+            rep[f"C{C}"]["emulated_ms_per_step"] = emulated_strategy_times(A, g, cfg, train, labels, C, dt, stream)
         if C == 2:
             rep["bw_profile"] = {"local_gather_GBps": bw.beta_Bps[0] / 1e9, "local_gather_alpha_us": bw.alpha_s[0] * 1e6,
                                  "host_read_GBps": bw.beta_Bps[7] / 1e9, "measured": list(bw.measured)}
@@ -345,6 +349,39 @@ def planner_report(A, g, cfg, train, labels, args, stream, gdp_ms):
     rep["C1"] = {"measured_ms_per_step": {s: gdp_ms for s in STRATS}, "pick": "GDP",
                  "note": "at C = 1 every strategy degenerates to GDP (SURVEY §8(d))"}
     return rep
+
+
+def emulated_strategy_times(A, g, cfg, train, labels, C, dt, stream, steps=5):
+    """Every strategy's full step with all C ranks emulated on this one GPU (rank = -1: the
+    same kernels, "peer" buffers local): evidence that all four strategies run on device at
+    this scale.  The C ranks time-share one GPU and no byte crosses NVLink, so these are not
+    C-GPU step times (the Planner's predictions above are)."""
+    import torch
+    out = {}
+    for s in STRATS:
+        ctx = A.Ctx(-1, C, 0, stream.cuda_stream)
+        gr = ctx.graph_load(g.indptr, g.indices, aptgen.partition(g.n, C))
+        fs = ctx.fstore_create(gr, A.NFP if s == "NFP" else A.GDP, dt, cfg.dim, None, cfg.feat_seed)
+        dims = [cfg.dim] + [d for _, d in cfg.dims()]
+        tr = A.Trainer(ctx, gr, fs, dims, cfg.fanouts, cfg.batch, dt, 0.05, cfg.sample_seed, cfg.feat_seed,
+                       A.STRATEGY[s], labels)
+        tr.set_params(aptgen.weights(cfg))
+        tr.set_epoch(train, 0)
+        tr.use_graph(True)
+        for i in range(3):
+            tr.step(i)
+        torch.cuda.synchronize()
+        e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+        e0.record(stream)
+        for i in range(3, 3 + steps):
+            tr.step(i)
+        e1.record(stream)
+        torch.cuda.synchronize()
+        out[s] = e0.elapsed_time(e1) / steps
+        for h in (tr, fs, gr):
+            h.close()
+        ctx.close()
+    return out
 
 
 def layer1_bytes(ctx, gr, tr, cfg, rank, step, bf):

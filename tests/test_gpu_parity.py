@@ -374,7 +374,7 @@ def _strategy_ref(cfg, g, train, labels, params, strategy, C, step, dtype):
 
 
 @pytest.mark.parametrize("dtype", ["f32", "bf16"])
-@pytest.mark.parametrize("C", [2, 4])
+@pytest.mark.parametrize("C", [2, 4, 8])
 @pytest.mark.parametrize("strategy", ["GDP", "NFP", "SNP", "DNP"])
 def test_strategy_step_matches_oracle(A, tiny, strategy, C, dtype):
     cfg, g, train = tiny
