@@ -117,6 +117,21 @@ cudaError_t launch_gather(const FeatView& fv, const int32_t* ids, const int32_t*
 cudaError_t launch_fill_features(void* shard, DType dt, int64_t pitch, int col0, int ncols, const int32_t* ids,
                                  int64_t n, uint64_t seed, cudaStream_t st);
 
+// ---------------------------------------------------------------- fused.cu
+// Layer-1 forward in one kernel: TMA gather4 of the sampled rows, mean, tcgen05
+// projection, bias + ReLU.  Single-shard bf16 store; cudaErrorNotSupported otherwise.
+struct FusedL1Args {
+  const int32_t* cnt; const int32_t* nbr; int k;        // sampler ELL
+  const int32_t* n_dev; int64_t M_max;                  // destination rows
+  const uint16_t* feat; int64_t n_rows_table; int row_elems;   // bf16 store [rows x row_elems]
+  int d;                                                // features aggregated
+  const uint16_t* Wb; int64_t w_pitch; int N;           // bf16 W [N x w_pitch]
+  const float* bias; int relu;
+  float* Y; int64_t y_pitch;                            // fp32 h1
+  uint16_t* Z; int64_t z_pitch; int z_ones;             // bf16 Z (weight gradient)
+};
+cudaError_t launch_sage_l1(const FusedL1Args& a, cudaStream_t st);
+
 // ---------------------------------------------------------------- bwd.cu
 // Transpose of a sampled block (counting sort): csc_ptr [n_src+1], csc_dst [E].
 struct CscArgs {

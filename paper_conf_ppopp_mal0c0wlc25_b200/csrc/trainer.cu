@@ -516,18 +516,42 @@ void activate(apt_trainer* t, int q) {
   t->parity = q;
 }
 
-// GDP layer-1 forward on one rank: fused gather (local + peer rows) + mean, projection.
+// GDP layer-1 forward on one rank: the fused gather+mean (local + peer rows), then the
+// projection.  APT_FUSED_L1=1 selects the single-kernel layer (fused.cu: gather warps ->
+// UMMA tile in shared memory -> tcgen05 -> epilogue) for a single-shard bf16 store --
+// correct (tested) but measured slower on products (78 us vs 34 + 30 us): the gather
+// needs the parallelism of thousands of short-lived warps more than it gains from not
+// writing and re-reading the 10 MB Z.
 apt_status layer1_fwd_gdp(apt_trainer* t, RankState& rs, bool time_it) {
   apt_ctx* c = t->ctx;
   Layer& L = rs.L[0];
   const Hop& hp = rs.hops[t->K - 1];
+  const FeatView fv = feat_view(t->f, rs.rank);
+  const char* fz = std::getenv("APT_FUSED_L1");
+  const bool want_fused = fz && *fz == '1';
+  if (t->m.dtype == APT_BF16 && !fv.part && want_fused && tc_gemm_supported(L.d_out, L.d_in)) {
+    FusedL1Args fa{hp.cnt, hp.nbr, hp.k, hp.n_dst, hp.max_dst, static_cast<const uint16_t*>(fv.base[0]),
+                   t->g->n, int(fv.pitch), fv.dim, L.Wb, L.wb_pitch, L.d_out, L.b, t->K > 1 ? 1 : 0,
+                   L.H, L.h_pitch, L.Zb, L.zb_pitch, 1};
+    if (time_it) CK(c, record_ev(t, 6));
+    cudaError_t e = launch_sage_l1(fa, c->stream);
+    if (e == cudaSuccess) {
+      if (time_it) CK(c, record_ev(t, 7));
+      c->launches++;
+      t->fused_l1 = true;
+      return APT_OK;
+    }
+    if (e != cudaErrorNotSupported) return check_cuda(c, e, "launch_sage_l1");
+    cudaGetLastError();   // clear the sticky not-supported status; take the two-kernel path
+  }
+  t->fused_l1 = false;
   AggArgs a{};
   a.cnt = hp.cnt; a.nbr = hp.nbr; a.k = hp.k;
   a.n_dst = hp.n_dst; a.max_dst = hp.max_dst; a.dim = L.d_in;
   if (t->m.dtype == APT_BF16) { a.z_bf16 = L.Zb; a.z_bf16_pitch = L.zb_pitch; a.z_ones = 1; }
   else { a.z_f32 = L.Zf; a.z_f32_pitch = L.zf_pitch; }
   if (time_it) CK(c, record_ev(t, 6));
-  CK(c, launch_agg_fstore(a, feat_view(t->f, rs.rank), c->stream));
+  CK(c, launch_agg_fstore(a, fv, c->stream));
   c->launches++;
   if (time_it) CK(c, record_ev(t, 7));
   return project(t, L, L.Zb, L.Zf, L.zb_pitch, L.zf_pitch, L.n_rows, L.max_rows, L.d_in, L.W, L.Wb, L.b,

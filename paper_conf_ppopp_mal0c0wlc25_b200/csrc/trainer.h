@@ -130,7 +130,8 @@ struct apt_trainer {
   int parity = 0;                    // sample set the last step computed on
   int64_t primed = -1;               // step id already sampled into sset[primed_parity]
   int primed_parity = 0;
-  bool csc_forked = false;           // this step's block transposes run on the side branch (wait ev_csc)
+  bool csc_forked = false;
+  bool fused_l1 = false;             // the last layer-1 forward ran as the single fused kernel           // this step's block transposes run on the side branch (wait ev_csc)
   cudaGraphExec_t gexec_p[2][2] = {};   // [parity][update] pipelined step graphs
   cudaGraph_t graph_p[2][2] = {};
   cudaGraphNode_t step_node_p[2][2] = {};

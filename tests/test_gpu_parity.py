@@ -278,6 +278,25 @@ def test_pipelined_steps_equal_unpipelined(A, tiny, strategy, C):
             assert np.allclose(W0, W1, rtol=1e-5, atol=1e-6) and np.allclose(b0, b1, rtol=1e-5, atol=1e-6)
 
 
+@pytest.mark.parametrize("dtype", ["bf16"])
+def test_fused_layer1_kernel_matches_oracle(A, ctx, tiny, dtype, monkeypatch):
+    """The opt-in single-kernel layer 1 (gather -> UMMA tile in smem -> tcgen05 -> epilogue):
+    Z bit-exact, h1 / logits / gradients against the oracle, like the two-kernel path."""
+    monkeypatch.setenv("APT_FUSED_L1", "1")
+    cfg, g, train = tiny
+    tr, params, labels = _trainer(A, ctx, cfg, g, train, dtype)
+    tr.step(1, update=False)
+    seeds = tr.read("seeds")[:, 0].astype(np.int64)
+    blocks = oracle.sample_blocks(g, seeds, cfg.fanouts, cfg.sample_seed, 1)
+    p64 = [(W.astype(np.float64), b.astype(np.float64)) for W, b in params]
+    ref = model.train_step(blocks, cfg.feat_seed, cfg.dim, p64, labels[seeds], len(seeds), dtype)
+    assert np.array_equal(tr.read("Z", 1), ref["cache"]["Z"][0].astype(np.float32))
+    tol = TOL[dtype]
+    assert np.allclose(tr.read("H", 1), ref["cache"]["h"][0], **tol)
+    for l in range(1, len(blocks) + 1):
+        assert np.allclose(tr.read("dW", l), ref["grads"][l - 1][0], **tol)
+
+
 def test_sgd_update_and_graph_replay(A, ctx, tiny):
     """Two steps with the update, eager vs CUDA-graph replay: identical parameters."""
     cfg, g, train = tiny
