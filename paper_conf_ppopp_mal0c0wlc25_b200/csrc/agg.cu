@@ -65,7 +65,7 @@ struct CsrSrc {                  // upper layers: block CSR over the previous la
 // 16-B loads in flight per lane, no dependent index load on the critical path).
 // Sum in fp32 (exact under O4), IEEE RN division by the sampled degree (O5).
 template <int EPV, int VPL, int LG, class Src>
-__global__ void __launch_bounds__(256, (VPL == 1 ? 8 : 4)) agg_kernel(AggArgs a, Src src) {
+__global__ void __launch_bounds__(256, (VPL == 1 ? 6 : 4)) agg_kernel(AggArgs a, Src src) {
   APT_PDL_PROLOGUE();
   const int lane = lane_id();
   const int sub = LG == 16 ? (lane >> 4) : 0;
