@@ -339,7 +339,12 @@ def planner_report(A, g, cfg, train, labels, args, stream, gdp_ms):
                         "n_vs_per_step": sum(st.n_vs[r] for r in range(C)) / steps,
                         "n_vd_per_step": sum(st.n_vd[r] for r in range(C)) / steps}
         if C <= args.emulate_max_c:
-            rep[f"C{C}"]["emulated_ms_per_step"] = emulated_strategy_times(A, g, cfg, train, labels, C, dt, stream)
+            em = emulated_strategy_times(A, g, cfg, train, labels, C, dt, stream)
+            fastest = min(em, key=em.get)
+            rep[f"C{C}"]["emulated_ms_per_step"] = em
+            rep[f"C{C}"]["emulated_fastest"] = fastest
+            # the pick's slowdown vs the measured fastest, on the emulated job (target <= 1.10)
+            rep[f"C{C}"]["pick_slowdown_vs_fastest_emulated"] = em[STRATS[pick]] / em[fastest]
         if C == 2:
             rep["bw_profile"] = {"local_gather_GBps": bw.beta_Bps[0] / 1e9, "local_gather_alpha_us": bw.alpha_s[0] * 1e6,
                                  "host_read_GBps": bw.beta_Bps[7] / 1e9, "measured": list(bw.measured)}
