@@ -166,6 +166,20 @@ apt_status apt_fstore_create(apt_ctx* ctx, const apt_graph* g, apt_strategy layo
                              int dim, const float* host_feats, uint64_t feat_seed, apt_fstore** out);
 apt_status apt_fstore_destroy(apt_fstore* f);
 
+/* Tiers of the unified feature store. */
+typedef struct {
+  double hbm_frac;          /* fraction of every partition's rows kept in its owner's HBM (1.0: all); the
+                               rest form the host tier (pinned, mapped; read over PCIe / C2C)          */
+  int64_t cache_rows;       /* excess cache: rows replicated into every GPU's spare HBM */
+  const int64_t* hot_ids;   /* host, >= cache_rows candidate ids, hottest first (apt_hot_rows)        */
+} apt_fstore_opts;
+/* apt_fstore_create with tiers (opts NULL: everything in HBM).  Row-sharded
+ * layouts only (NFP: APT_E_UNSUPPORTED).  Kernels see one view per rank: own
+ * HBM rows, NVLink peer rows, host rows, own cached rows.  Syncs.            */
+apt_status apt_fstore_create_tiered(apt_ctx* ctx, const apt_graph* g, apt_strategy layout, apt_dtype dtype,
+                                    int dim, const float* host_feats, uint64_t feat_seed, const apt_fstore_opts* opts,
+                                    apt_fstore** out);
+
 /* ---------------------------------------------------------------- sampling */
 /* K-hop node-wise sampling of seeds_dev (device int64[n_seeds]) with
  * fanouts (host, fanouts[l-1] for layer l, 1..256), Philox key rng_seed and

@@ -52,6 +52,10 @@ class PlanStats(C.Structure):
                 ("t_build_s", _D4), ("t_train_s", C.c_double)]
 
 
+class FstoreOpts(C.Structure):
+    _fields_ = [("hbm_frac", C.c_double), ("cache_rows", C.c_int64), ("hot_ids", C.c_void_p)]
+
+
 class BwProfile(C.Structure):
     _fields_ = [("world", C.c_int), ("alpha_s", C.c_double * 8), ("beta_Bps", C.c_double * 8),
                 ("measured", C.c_int * 8)]
@@ -96,6 +100,7 @@ def lib():
             "apt_memcpy": [vp, vp, vp, C.c_size_t, i32],
             "apt_graph_load": [vp, i64, i64, vp, vp, vp, vp], "apt_graph_destroy": [vp],
             "apt_fstore_create": [vp, vp, i32, i32, i32, vp, u64, vp], "apt_fstore_destroy": [vp],
+            "apt_fstore_create_tiered": [vp, vp, i32, i32, i32, vp, u64, vp, vp],
             "apt_sample": [vp, vp, vp, i64, vp, i32, u64, u64, vp], "apt_batch_block": [vp, i32, vp],
             "apt_batch_destroy": [vp], "apt_gather": [vp, vp, vp, i64, vp],
             "apt_aggregate": [vp, vp, vp, i32, i32, i64, vp, i64],
@@ -194,11 +199,19 @@ class Ctx:
                                      indices.ctypes.data, _ptr(part), C.byref(h)))
         return Handle(h, lib().apt_graph_destroy, keep=(self,))
 
-    def fstore_create(self, graph, layout, dtype, dim, host_feats=None, feat_seed=0):
+    def fstore_create(self, graph, layout, dtype, dim, host_feats=None, feat_seed=0, hbm_frac=1.0, hot_ids=None):
+        """hbm_frac < 1: the rows beyond every shard's HBM budget form the pinned host tier;
+        hot_ids: rows replicated into every GPU's spare HBM (excess cache), hottest first."""
         h = C.c_void_p()
         hf = None if host_feats is None else np.ascontiguousarray(host_feats, np.float32)
-        self.ck(lib().apt_fstore_create(self.h, graph.h, layout, dtype, dim, _ptr(hf), feat_seed, C.byref(h)))
-        return Handle(h, lib().apt_fstore_destroy, keep=(self, graph))
+        if hbm_frac == 1.0 and hot_ids is None:
+            self.ck(lib().apt_fstore_create(self.h, graph.h, layout, dtype, dim, _ptr(hf), feat_seed, C.byref(h)))
+            return Handle(h, lib().apt_fstore_destroy, keep=(self, graph))
+        hot = None if hot_ids is None else np.ascontiguousarray(hot_ids, np.int64)
+        o = FstoreOpts(hbm_frac, 0 if hot is None else len(hot), None if hot is None else hot.ctypes.data)
+        self.ck(lib().apt_fstore_create_tiered(self.h, graph.h, layout, dtype, dim, _ptr(hf), feat_seed, C.byref(o),
+                                               C.byref(h)))
+        return Handle(h, lib().apt_fstore_destroy, keep=(self, graph, hot))
 
     def sample(self, graph, seeds_dev, n_seeds, fanouts, rng_seed, step):
         f = np.ascontiguousarray(fanouts, np.int32)

@@ -64,10 +64,13 @@ cudaError_t launch_perm_keys(const int32_t* train, int64_t n, uint64_t seed, uin
 enum DType : int { kF32 = 0, kBF16 = 1 };
 
 // Feature store view used by the fused gather+mean kernel (S6+S7).
+// Unified feature store as seen by one rank: tier t of node u is
+// part[u]: 0..C-1 = that rank's HBM shard (local or NVLink peer), C = the host tier
+// (pinned, mapped), C+1 = this rank's cache of replicated hot rows.
 struct FeatView {
-  const void* base[8];         // per-owner shard base (local or NVLink peer pointer)
-  const int32_t* part;         // owner of node u (nullptr => single shard, row = u)
-  const int32_t* lrow;         // row of u inside its owner's shard
+  const void* base[10];        // per-tier base (local / NVLink peer / mapped host / own cache)
+  const int32_t* part;         // tier of node u (nullptr => single shard, row = u)
+  const int32_t* lrow;         // row of u inside its tier
   int64_t pitch;               // elements per stored row (padded to 16 B)
   int dim;                     // logical columns to aggregate
   int col0;                    // first column inside the stored row

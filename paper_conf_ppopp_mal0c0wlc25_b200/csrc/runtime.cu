@@ -5,6 +5,7 @@
 #include <cstdarg>
 #include <cstdio>
 #include <cstring>
+#include <cmath>
 #include <numeric>
 
 #include "common.cuh"
@@ -196,8 +197,18 @@ apt_status apt_graph_destroy(apt_graph* g) {
 // ------------------------------------------------------------- feature store
 apt_status apt_fstore_create(apt_ctx* c, const apt_graph* g, apt_strategy layout, apt_dtype dtype, int dim,
                              const float* host_feats, uint64_t feat_seed, apt_fstore** out) {
+  return apt_fstore_create_tiered(c, g, layout, dtype, dim, host_feats, feat_seed, nullptr, out);
+}
+
+apt_status apt_fstore_create_tiered(apt_ctx* c, const apt_graph* g, apt_strategy layout, apt_dtype dtype, int dim,
+                                    const float* host_feats, uint64_t feat_seed, const apt_fstore_opts* opts,
+                                    apt_fstore** out) {
   if (!c || !g || !out || dim <= 0 || (dtype != APT_F32 && dtype != APT_BF16) || layout < APT_GDP || layout > APT_AUTO)
     return set_err(c, APT_E_INVALID, "apt_fstore_create: bad arguments");
+  const double frac = opts ? opts->hbm_frac : 1.0;
+  const int64_t want_cache = opts ? opts->cache_rows : 0;
+  if (!(frac > 0.0 && frac <= 1.0) || want_cache < 0 || (want_cache > 0 && !opts->hot_ids))
+    return set_err(c, APT_E_INVALID, "apt_fstore_create: hbm_frac in (0,1], cache_rows >= 0 with hot_ids");
   auto* f = new apt_fstore();
   f->ctx = c;
   ctx_retain(c);
@@ -207,68 +218,140 @@ apt_status apt_fstore_create(apt_ctx* c, const apt_graph* g, apt_strategy layout
   f->dim = dim;
   f->world = c->world;
   const int C = c->world;
+  const bool col_sharded = f->layout == APT_NFP && C > 1;
+  f->tiered = !col_sharded && (frac < 1.0 || want_cache > 0);
+  f->hbm_frac = frac;
+  if (col_sharded && (frac < 1.0 || want_cache > 0)) {
+    apt_fstore_destroy(f);
+    return set_err(c, APT_E_UNSUPPORTED, "apt_fstore_create: tiers apply to row-sharded stores (NFP reads only its "
+                                         "column slice and has no excess cache, P:175-178)");
+  }
   const int align = dtype == APT_BF16 ? 8 : 4;     // 16-byte rows
   const size_t esz = dtype == APT_BF16 ? 2 : 4;
+  // ids of every shard's rows, ascending (a single shard holds every node)
+  std::vector<std::vector<int32_t>> ids(C);
+  if (!col_sharded) {
+    if (C > 1) {
+      for (int64_t u = 0; u < g->n; ++u) ids[g->part_h[u]].push_back(int32_t(u));
+    } else {
+      ids[0].resize(g->n);
+      for (int64_t u = 0; u < g->n; ++u) ids[0][u] = int32_t(u);
+    }
+  }
   for (int r = 0; r < C; ++r) {
-    if (f->layout == APT_NFP && C > 1) {
+    if (col_sharded) {
       f->col_lo[r] = int((int64_t(r) * dim) / C);
       f->col_hi[r] = int((int64_t(r + 1) * dim) / C);
       f->rows[r] = g->n;
     } else {
       f->col_lo[r] = 0;
       f->col_hi[r] = dim;
-      f->rows[r] = C > 1 ? g->shard_rows[r] : g->n;
+      const int64_t all = int64_t(ids[r].size());
+      f->rows[r] = std::min<int64_t>(all, int64_t(std::ceil(frac * double(all))));   // rows kept in HBM
     }
     const int w = std::max(1, f->col_hi[r] - f->col_lo[r]);
     f->pitch[r] = round_up(w, align);
   }
-  // ids of every shard's rows (ascending global ids) -> synthetic fill / host copy
-  std::vector<std::vector<int32_t>> ids(C);
-  if (f->layout != APT_NFP && C > 1) {
-    for (int64_t u = 0; u < g->n; ++u) ids[g->part_h[u]].push_back(int32_t(u));
-  }
-  int32_t* ids_dev = f->arena.alloc<int32_t>(g->n, false);
+  const int64_t pitch = f->pitch[0];
+  int32_t* ids_dev = f->arena.alloc<int32_t>(std::max<int64_t>(g->n, 1), false);
+  auto fill_rows = [&](void* dst, const int32_t* ids_h, int64_t n_rows, int col0, int ncols, int64_t pch) -> apt_status {
+    if (n_rows <= 0) return APT_OK;
+    if (host_feats) {
+      std::vector<uint8_t> buf(size_t(n_rows * pch) * esz, 0);
+      for (int64_t i = 0; i < n_rows; ++i) {
+        const int64_t u = ids_h ? ids_h[i] : i;
+        for (int j = 0; j < ncols; ++j) {
+          const float v = host_feats[u * dim + col0 + j];
+          if (esz == 4) {
+            reinterpret_cast<float*>(buf.data())[i * pch + j] = v;
+          } else {
+            uint32_t bits;
+            memcpy(&bits, &v, 4);
+            bits = (bits + 0x7FFFu + ((bits >> 16) & 1u)) >> 16;   // RNE
+            reinterpret_cast<uint16_t*>(buf.data())[i * pch + j] = uint16_t(bits);
+          }
+        }
+      }
+      CK(c, cudaMemcpyAsync(dst, buf.data(), buf.size(), cudaMemcpyDefault, c->stream));
+    } else {
+      const int32_t* idp = nullptr;
+      if (ids_h) {
+        CK(c, cudaMemcpyAsync(ids_dev, ids_h, sizeof(int32_t) * n_rows, cudaMemcpyHostToDevice, c->stream));
+        idp = ids_dev;
+      }
+      CK(c, launch_fill_features(dst, f->dtype, pch, col0, ncols, idp, n_rows, feat_seed, c->stream));
+      c->launches++;
+    }
+    CK(c, cudaStreamSynchronize(c->stream));
+    return APT_OK;
+  };
   for (int r = 0; r < C; ++r) {
     // emulated: all shards here; multi-process: only the own shard is local
     if (!c->emulated && r != c->rank) continue;
-    f->shard[r] = f->arena.alloc<uint8_t>(f->rows[r] * f->pitch[r] * int64_t(esz), true);
+    f->shard[r] = f->arena.alloc<uint8_t>(std::max<int64_t>(f->rows[r], 1) * f->pitch[r] * int64_t(esz), true);
     if (!f->shard[r] || !ids_dev) {
       apt_fstore_destroy(f);
       return set_err(c, APT_E_OOM, "apt_fstore_create: out of device memory");
     }
-    const int32_t* idp = nullptr;
-    if (!ids[r].empty()) {
-      CK(c, cudaMemcpyAsync(ids_dev, ids[r].data(), sizeof(int32_t) * ids[r].size(), cudaMemcpyHostToDevice, c->stream));
-      idp = ids_dev;
-    }
     const int ncols = f->col_hi[r] - f->col_lo[r];
-    if (host_feats) {
-      // host fp32 [n x dim] -> this shard (rows of the shard, its column slice), converted on the host
-      std::vector<uint8_t> buf(size_t(f->rows[r] * f->pitch[r]) * esz, 0);
-      for (int64_t i = 0; i < f->rows[r]; ++i) {
-        const int64_t u = idp ? ids[r][i] : i;
-        for (int j = 0; j < ncols; ++j) {
-          const float v = host_feats[u * dim + f->col_lo[r] + j];
-          if (esz == 4) {
-            reinterpret_cast<float*>(buf.data())[i * f->pitch[r] + j] = v;
-          } else {
-            uint32_t b;
-            memcpy(&b, &v, 4);
-            b = (b + 0x7FFFu + ((b >> 16) & 1u)) >> 16;   // RNE
-            reinterpret_cast<uint16_t*>(buf.data())[i * f->pitch[r] + j] = uint16_t(b);
-          }
-        }
+    apt_status st = col_sharded ? fill_rows(f->shard[r], nullptr, f->rows[r], f->col_lo[r], ncols, f->pitch[r])
+                                : fill_rows(f->shard[r], C > 1 ? ids[r].data() : nullptr, f->rows[r], 0, ncols,
+                                            f->pitch[r]);
+    if (st != APT_OK) { apt_fstore_destroy(f); return st; }
+  }
+  if (f->tiered) {
+    // host tier: every shard's rows beyond its HBM budget, in (owner, row) order; each
+    // process keeps the whole tier in its pinned host memory (like the topology)
+    std::vector<int32_t> host_ids;
+    for (int r = 0; r < C; ++r)
+      for (size_t i = size_t(f->rows[r]); i < ids[r].size(); ++i) host_ids.push_back(ids[r][i]);
+    f->host_rows = int64_t(host_ids.size());
+    if (f->host_rows > 0) {
+      if (cudaHostAlloc(&f->host, size_t(f->host_rows * pitch) * esz, cudaHostAllocMapped | cudaHostAllocPortable) !=
+          cudaSuccess) {
+        apt_fstore_destroy(f);
+        return set_err(c, APT_E_OOM, "apt_fstore_create: pinned host tier of %lld rows", (long long)f->host_rows);
       }
-      CK(c, cudaMemcpyAsync(f->shard[r], buf.data(), buf.size(), cudaMemcpyHostToDevice, c->stream));
+      apt_status st = fill_rows(f->host, host_ids.data(), f->host_rows, 0, dim, pitch);
+      if (st != APT_OK) { apt_fstore_destroy(f); return st; }
+    }
+    std::vector<int32_t> base_tier(g->n), base_row(g->n);
+    for (int r = 0; r < C; ++r)
+      for (size_t i = 0; i < ids[r].size(); ++i) {
+        const int32_t u = ids[r][i];
+        if (int64_t(i) < f->rows[r]) { base_tier[u] = r; base_row[u] = int32_t(i); }
+        else { base_tier[u] = C; base_row[u] = -1; }
+      }
+    for (int64_t i = 0, h = 0; i < int64_t(host_ids.size()); ++i, ++h) base_row[host_ids[i]] = int32_t(h);
+    // per hosted rank: its view, with its cache of hot rows (those it does not hold in HBM)
+    for (int r = 0; r < C; ++r) {
+      if (!c->emulated && r != c->rank) continue;
+      std::vector<int32_t> tier = base_tier, trow = base_row, cached;
+      for (int64_t j = 0; j < want_cache && int64_t(cached.size()) < want_cache; ++j) {
+        const int64_t u = opts->hot_ids[j];
+        if (u < 0 || u >= g->n) { apt_fstore_destroy(f); return set_err(c, APT_E_INVALID, "hot id out of range"); }
+        if (tier[u] == r || tier[u] == C + 1) continue;          // already local
+        tier[u] = C + 1;
+        trow[u] = int32_t(cached.size());
+        cached.push_back(int32_t(u));
+      }
+      f->cache_rows[r] = int64_t(cached.size());
+      if (!cached.empty()) {
+        f->cache[r] = f->arena.alloc<uint8_t>(f->cache_rows[r] * pitch * int64_t(esz), false);
+        if (!f->cache[r]) { apt_fstore_destroy(f); return set_err(c, APT_E_OOM, "apt_fstore_create: cache"); }
+        apt_status st = fill_rows(f->cache[r], cached.data(), f->cache_rows[r], 0, dim, pitch);
+        if (st != APT_OK) { apt_fstore_destroy(f); return st; }
+      }
+      f->tier_map[r] = f->arena.alloc<int32_t>(g->n, false);
+      f->trow_map[r] = f->arena.alloc<int32_t>(g->n, false);
+      if (!f->tier_map[r] || !f->trow_map[r]) { apt_fstore_destroy(f); return set_err(c, APT_E_OOM, "feature map"); }
+      CK(c, cudaMemcpyAsync(f->tier_map[r], tier.data(), sizeof(int32_t) * g->n, cudaMemcpyHostToDevice, c->stream));
+      CK(c, cudaMemcpyAsync(f->trow_map[r], trow.data(), sizeof(int32_t) * g->n, cudaMemcpyHostToDevice, c->stream));
       CK(c, cudaStreamSynchronize(c->stream));
-    } else {
-      CK(c, launch_fill_features(f->shard[r], f->dtype, f->pitch[r], f->col_lo[r], ncols, idp, f->rows[r], feat_seed,
-                                 c->stream));
-      c->launches++;
-      CK(c, cudaStreamSynchronize(c->stream));
+      f->tier_h[r] = std::move(tier);
     }
   }
-  if (multiprocess(c) && f->layout != APT_NFP) {
+  if (multiprocess(c) && !col_sharded) {
     // row-sharded store: every rank maps every peer's shard (GDP / DNP halo reads over NVLink)
     void* tab[APT_MAX_RANKS] = {};
     apt_status s = share_ptr(c, f->shard[c->rank], tab, &f->peer_opened);
@@ -296,7 +379,15 @@ FeatView feat_view(const apt_fstore* f, int r) {
   FeatView v{};
   const bool rows_sharded = f->layout != APT_NFP && f->world > 1;
   for (int o = 0; o < f->world; ++o) v.base[o] = f->shard[o];
-  if (rows_sharded) {
+  if (f->tiered) {
+    const int rr = f->world > 1 ? r : 0;
+    v.base[f->world] = f->host;
+    v.base[f->world + 1] = f->cache[rr];
+    v.part = f->tier_map[rr];
+    v.lrow = f->trow_map[rr];
+    v.pitch = f->pitch[0];
+    v.dim = f->dim;
+  } else if (rows_sharded) {
     v.part = f->g->part;
     v.lrow = f->g->lrow;
     v.pitch = f->pitch[0];

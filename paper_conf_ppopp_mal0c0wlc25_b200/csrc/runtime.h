@@ -117,10 +117,24 @@ struct apt_fstore {
   int64_t pitch[APT_MAX_RANKS] = {};   // elements per row
   int col_lo[APT_MAX_RANKS] = {};
   int col_hi[APT_MAX_RANKS] = {};
-  int64_t rows[APT_MAX_RANKS] = {};
+  int64_t rows[APT_MAX_RANKS] = {};      // rows of each shard held in HBM
+  // tiers (apt_fstore_opts): host tier + per-rank hot-row caches, and the per-rank maps
+  bool tiered = false;
+  double hbm_frac = 1.0;
+  int64_t host_rows = 0;
+  void* host = nullptr;                  // pinned, mapped: rows beyond every shard's HBM budget
+  int64_t cache_rows[APT_MAX_RANKS] = {};
+  void* cache[APT_MAX_RANKS] = {};       // replicated hot rows (hosted ranks)
+  int32_t* tier_map[APT_MAX_RANKS] = {}; // device [n] per hosted rank
+  int32_t* trow_map[APT_MAX_RANKS] = {};
+  std::vector<int32_t> tier_h[APT_MAX_RANKS];   // host copies (dry-run counters, tests)
   std::vector<void*> peer_opened;   // IPC-mapped peer shards (multi-process)
   apt::Arena arena;
-  ~apt_fstore() { apt::close_peers(peer_opened); apt::defer_exported(ctx, arena); }
+  ~apt_fstore() {
+    apt::close_peers(peer_opened);
+    apt::defer_exported(ctx, arena);
+    if (host) cudaFreeHost(host);
+  }
 };
 
 struct apt_batch {

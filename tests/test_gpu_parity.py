@@ -570,3 +570,45 @@ def test_products_full_size_layer1_rows_vs_oracle(A, ctx):
         assert np.array_equal(Z[i], zb.astype(np.float32)), v
         h = np.maximum(zb @ W1.T + b1, 0)
         assert np.allclose(H[i], h, rtol=2e-2, atol=2e-3), v
+
+
+# ------------------------------------------------------------------ unified feature store tiers (NEXT #2)
+@pytest.mark.parametrize("dtype", ["f32", "bf16"])
+@pytest.mark.parametrize("frac,n_hot", [(0.5, 0), (0.3, 400), (1.0, 400)])
+def test_tiered_store_rows_and_step(A, tiny, dtype, frac, n_hot):
+    """HBM budget + pinned host tier + replicated hot rows: every row reads back bit-exact
+    through each rank's view, and GDP / DNP / SNP steps at C = 2 still match the oracle."""
+    cfg, g, train = tiny
+    rng = np.random.default_rng(3)
+    hot = rng.choice(g.n, size=n_hot, replace=False) if n_hot else None
+    for strategy, C in (("GDP", 1), ("GDP", 2), ("DNP", 2), ("SNP", 2)):
+        ctx = A.Ctx(-1, C, 0) if C > 1 else A.Ctx(0, 1, 0)
+        part = aptgen.partition(g.n, C)
+        gr = ctx.graph_load(g.indptr, g.indices, part)
+        fs = ctx.fstore_create(gr, A.GDP, A.DTYPE[dtype], cfg.dim, None, cfg.feat_seed, hbm_frac=frac, hot_ids=hot)
+        if strategy == "GDP":
+            ids = np.arange(g.n, dtype=np.int32)
+            pitch = ((cfg.dim + 7) // 8 * 8) if dtype == "bf16" else ((cfg.dim + 3) // 4 * 4)
+            esz = 2 if dtype == "bf16" else 4
+            out = torch.zeros(g.n * pitch * esz, dtype=torch.uint8, device="cuda")
+            torch.cuda.synchronize()
+            ctx.gather(fs, torch.as_tensor(ids).cuda(), g.n, out)
+            torch.cuda.synchronize()
+            raw = out.cpu().numpy()
+            got = ((raw.view(np.uint16).astype(np.uint32) << 16).view(np.float32) if dtype == "bf16"
+                   else raw.view(np.float32)).reshape(g.n, pitch)[:, :cfg.dim]
+            assert np.array_equal(got.astype(np.float64), oracle.features(cfg.feat_seed, ids.astype(np.int64), cfg.dim))
+        dims = [cfg.dim] + [d for _, d in cfg.dims()]
+        labels = aptgen.labels(cfg, g.n)
+        tr = A.Trainer(ctx, gr, fs, dims, cfg.fanouts, cfg.batch, A.DTYPE[dtype], 0.1, cfg.sample_seed, cfg.feat_seed,
+                       A.STRATEGY[strategy], labels)
+        params = aptgen.weights(cfg)
+        tr.set_params(params)
+        tr.set_epoch(train, 0)
+        tr.step(0, update=False)
+        seeds, refs = _strategy_ref(cfg, g, train, labels, params, strategy, C, 0, dtype)
+        tol = TOL[dtype]
+        for r in range(C):
+            assert np.allclose(tr.read("H", 1, rank=r), refs[r]["cache"]["h"][0], **tol), (strategy, C, r)
+        dW = sum(x["grads"][0][0] for x in refs)
+        assert np.allclose(tr.read("dW", 1, rank=0), dW, **tol), (strategy, C)
