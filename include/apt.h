@@ -107,6 +107,8 @@ typedef struct {
   int64_t n_calls[4][APT_MAX_RANKS];         /* exchange operators per step        */
   double t_build_s[4][APT_MAX_RANKS];        /* measured T_build           */
   double t_train_s;                          /* measured common T_train (GDP)      */
+  int64_t rows_host[4][APT_MAX_RANKS];       /* unique rows read from the host tier */
+  int64_t feat_bytes_host[4][APT_MAX_RANKS];
 } apt_plan_stats;
 
 /* Operator slots of the bandwidth profile ("trials").          */

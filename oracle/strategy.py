@@ -64,25 +64,64 @@ def _edges(blk):
     return rows, blk.src[blk.indices]
 
 
-def emulate_layer1(strategy, l1_blocks, part, C, d, d_out, feat_bytes=4, hidden_bytes=4):
-    """l1_blocks[r] = rank r's layer-1 Block (dst, src, indptr, indices).
-    Returns per-rank dict of counts and the per-rank structures."""
+def tiered_store(part, C, hbm_frac, hot_ids=None, cache_rows=0):
+    """The unified feature store's tiers (apt_fstore_create_tiered):
+    every partition keeps its first ceil(hbm_frac * size) rows (ascending id) in its
+    owner's HBM, the rest in the host tier; rank r replicates the first cache_rows hot
+    ids it does not hold in its own HBM (excess cache).
+    Returns tier(r, ids) -> array of 0 local, 1 NVLink peer, 2 host."""
+    part = np.asarray(part)
+    n = len(part)
+    host = np.zeros(n, bool)
+    for o in range(C):
+        ids = np.nonzero(part == o)[0]
+        keep = min(len(ids), int(np.ceil(hbm_frac * len(ids))))
+        host[ids[keep:]] = True
+    cached = [np.zeros(n, bool) for _ in range(C)]
+    if hot_ids is not None and cache_rows:
+        for r in range(C):
+            taken = 0
+            for u in hot_ids[:cache_rows]:
+                if taken >= cache_rows:
+                    break
+                if (part[u] == r and not host[u]) or cached[r][u]:
+                    continue
+                cached[r][u] = True
+                taken += 1
+
+    def tier(r, ids):
+        ids = np.asarray(ids, np.int64)
+        t = np.where(part[ids] == r, 0, 1)
+        t = np.where(host[ids], 2, t)
+        return np.where(cached[r][ids], 0, t)
+    return tier
+
+
+def emulate_layer1(strategy, l1_blocks, part, C, d, d_out, feat_bytes=4, hidden_bytes=4, tier=None):
+    """l1_blocks[r] = rank r's layer-1 Block (dst, src, indptr, indices).  tier(r, ids):
+    where rank r reads each row (0 local HBM, 1 NVLink peer, 2 host; default: own
+    partition local, others peer).  Returns per-rank dict of counts and structures."""
+    if tier is None:
+        def tier(r, ids):
+            return np.where(np.asarray(part)[np.asarray(ids, np.int64)] == r, 0, 1)
     out = []
     N_d = [b.n_dst for b in l1_blocks]
     for r in range(C):
-        out.append(dict(n_d=N_d[r], n_vs=0, n_vd=0, rows_local=0, rows_peer=0,
-                        feat_bytes_local=0, feat_bytes_peer=0, graph_bytes=0,
+        out.append(dict(n_d=N_d[r], n_vs=0, n_vd=0, rows_local=0, rows_peer=0, rows_host=0,
+                        feat_bytes_local=0, feat_bytes_peer=0, feat_bytes_host=0, graph_bytes=0,
                         hidden_bytes_fwd=0, hidden_bytes_bwd=0, n_calls=0,
                         virtual=[], requests=[]))
+
+    def count(o, uu, rec):
+        t = tier(o, uu) if len(uu) else np.zeros(0, int)
+        for key, code in (("local", 0), ("peer", 1), ("host", 2)):
+            rec["rows_" + key] = int((t == code).sum())
+            rec["feat_bytes_" + key] = rec["rows_" + key] * d * feat_bytes
+
     if strategy == "GDP":
         for r, blk in enumerate(l1_blocks):
             _, u = _edges(blk)
-            uu = np.unique(u)
-            loc = int((part[uu] == r).sum())
-            out[r]["rows_local"] = loc
-            out[r]["rows_peer"] = len(uu) - loc
-            out[r]["feat_bytes_local"] = loc * d * feat_bytes
-            out[r]["feat_bytes_peer"] = (len(uu) - loc) * d * feat_bytes
+            count(r, np.unique(u), out[r])
         return out
     if strategy == "NFP":
         for c in range(C):
@@ -118,8 +157,7 @@ def emulate_layer1(strategy, l1_blocks, part, C, d, d_out, feat_bytes=4, hidden_
                     out[r]["hidden_bytes_fwd"] += len(vs) * d_out * hidden_bytes
                     out[c]["hidden_bytes_bwd"] += len(vs) * d_out * hidden_bytes
         for c in range(C):
-            out[c]["rows_local"] = len(recv_rows[c])
-            out[c]["feat_bytes_local"] = len(recv_rows[c]) * d * feat_bytes
+            count(c, np.fromiter(recv_rows[c], np.int64, len(recv_rows[c])), out[c])   # own partition: HBM or host
             out[c]["n_calls"] = 3 if C > 1 else 0   # graph all-to-all, partial reduce, g all-to-all
         return out
     if strategy == "DNP":
@@ -140,12 +178,7 @@ def emulate_layer1(strategy, l1_blocks, part, C, d, d_out, feat_bytes=4, hidden_
                     out[r]["hidden_bytes_fwd"] += len(vs) * d_out * hidden_bytes
                     out[o]["hidden_bytes_bwd"] += len(vs) * d_out * hidden_bytes
         for o in range(C):
-            uu = np.fromiter(owned_rows[o], np.int64, len(owned_rows[o]))
-            loc = int((part[uu] == o).sum()) if len(uu) else 0
-            out[o]["rows_local"] = loc
-            out[o]["rows_peer"] = len(uu) - loc
-            out[o]["feat_bytes_local"] = loc * d * feat_bytes
-            out[o]["feat_bytes_peer"] = (len(uu) - loc) * d * feat_bytes
+            count(o, np.fromiter(owned_rows[o], np.int64, len(owned_rows[o])), out[o])
             out[o]["n_calls"] = 3 if C > 1 else 0   # request all-to-all, h1 return, g return
         return out
     raise ValueError(strategy)
@@ -180,6 +213,8 @@ def predict(per_strategy_stats, alpha, beta, t_build):
             t += st["feat_bytes_local"] / beta[OP_LOCAL_GATHER] + steps * alpha[OP_LOCAL_GATHER]
             if st["feat_bytes_peer"]:
                 t += st["feat_bytes_peer"] / beta[OP_PEER_PULL] + steps * alpha[OP_PEER_PULL]
+            if st.get("feat_bytes_host"):   # host tier of the unified store
+                t += st["feat_bytes_host"] / beta[OP_HOST_GATHER] + steps * alpha[OP_HOST_GATHER]
             if s == "NFP" and st["n_calls"]:
                 t += 2 * steps * alpha[OP_ALLGATHER] + steps * alpha[OP_REDUCE_SCATTER]
                 t += st["graph_bytes"] / beta[OP_ALLGATHER]

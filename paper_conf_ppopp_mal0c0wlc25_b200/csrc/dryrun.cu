@@ -43,11 +43,24 @@ struct DryCounters {
   unsigned long long uniq[APT_MAX_RANKS];                     // GDP/NFP: unique sources of block r
   unsigned long long rows_local[APT_MAX_RANKS];               // per owner
   unsigned long long rows_peer[APT_MAX_RANKS];
+  unsigned long long rows_host[APT_MAX_RANKS];
   unsigned long long pair_rows[APT_MAX_RANKS][APT_MAX_RANKS]; // this step: rows of requester r sent to owner c
   unsigned long long pair_edges[APT_MAX_RANKS][APT_MAX_RANKS];
   unsigned long long tot_rows[APT_MAX_RANKS][APT_MAX_RANKS];
   unsigned long long tot_edges[APT_MAX_RANKS][APT_MAX_RANKS];
   unsigned long long tot_msgs[APT_MAX_RANKS][APT_MAX_RANKS];  // steps in which the (r, c) message was non-empty
+};
+
+// Where rank r reads node u from (the unified store's tiers): 0 local HBM (own shard or
+// own cache), 1 NVLink peer, 2 host tier.
+struct TierInfo {
+  const int32_t* part; const int32_t* lrow; const int64_t* rows; const uint32_t* cache_bm; int64_t n_words;
+  __device__ __forceinline__ int of(int u, int r) const {
+    if (cache_bm && (cache_bm[int64_t(r) * n_words + (u >> 5)] >> (u & 31) & 1u)) return 0;
+    const int o = part[u];
+    if (rows && lrow[u] >= rows[o]) return 2;
+    return o == r ? 0 : 1;
+  }
 };
 
 __device__ __forceinline__ bool test_and_set(uint32_t* bm, int u) {
@@ -58,7 +71,8 @@ __device__ __forceinline__ bool test_and_set(uint32_t* bm, int u) {
 // One thread per layer-1 row of requester r (ELL cnt/nbr of the layer-1 hop).
 __global__ void dry_count_kernel(int S, int r, int C, const int32_t* __restrict__ dst, const int32_t* __restrict__ n_p,
                                  const int32_t* __restrict__ cnt, const int32_t* __restrict__ nbr, int k,
-                                 const int32_t* __restrict__ part, uint32_t* bm, int64_t n_words, DryCounters* dc) {
+                                 const int32_t* __restrict__ part, uint32_t* bm, int64_t n_words, DryCounters* dc,
+                                 TierInfo ti) {
   APT_PDL_PROLOGUE();
   const int64_t n = *n_p;
   for (int64_t i = int64_t(blockIdx.x) * blockDim.x + threadIdx.x; i < n; i += int64_t(gridDim.x) * blockDim.x) {
@@ -73,8 +87,8 @@ __global__ void dry_count_kernel(int S, int r, int C, const int32_t* __restrict_
         if (test_and_set(b, u)) {
           atomicAdd(&dc->uniq[r], 1ull);
           if (S == APT_GDP) {
-            if (part[u] == r) atomicAdd(&dc->rows_local[r], 1ull);
-            else atomicAdd(&dc->rows_peer[r], 1ull);
+            const int tr = ti.of(u, r);
+            atomicAdd(tr == 0 ? &dc->rows_local[r] : tr == 1 ? &dc->rows_peer[r] : &dc->rows_host[r], 1ull);
           }
         }
       }
@@ -86,7 +100,8 @@ __global__ void dry_count_kernel(int S, int r, int C, const int32_t* __restrict_
         const int u = row[e];
         const int c = part[u];
         ++ec[c];
-        if (test_and_set(bm + int64_t(c) * n_words, u)) atomicAdd(&dc->rows_local[c], 1ull);   // SNP reads are local
+        if (test_and_set(bm + int64_t(c) * n_words, u))   // SNP reads its own partition: HBM or host tier
+          atomicAdd(ti.of(u, c) == 2 ? &dc->rows_host[c] : &dc->rows_local[c], 1ull);
       }
 #pragma unroll
       for (int c = 0; c < APT_MAX_RANKS; ++c)
@@ -101,8 +116,8 @@ __global__ void dry_count_kernel(int S, int r, int C, const int32_t* __restrict_
       for (int e = 0; e < c_i; ++e) {
         const int u = row[e];
         if (test_and_set(bm + int64_t(o) * n_words, u)) {
-          if (part[u] == o) atomicAdd(&dc->rows_local[o], 1ull);
-          else atomicAdd(&dc->rows_peer[o], 1ull);
+          const int to = ti.of(u, o);
+          atomicAdd(to == 0 ? &dc->rows_local[o] : to == 1 ? &dc->rows_peer[o] : &dc->rows_host[o], 1ull);
         }
       }
     }
@@ -182,6 +197,8 @@ extern "C" apt_status apt_dryrun(apt_trainer* t, int64_t n_steps, apt_plan_stats
     }
   }
   if (!own_bm || !dc || !hops[K - 1].nbr) return set_err(c, APT_E_OOM, "apt_dryrun: out of device memory");
+  // tiers of the unified store (rows beyond the HBM budgets, replicated hot rows)
+  const TierInfo ti{g->part, g->lrow, t->f->tiered ? t->f->rows_dev : nullptr, t->f->cache_bm, n_words};
   std::vector<cudaEvent_t> ev;
   struct Mark { int s, r; };
   std::vector<Mark> marks;
@@ -218,7 +235,7 @@ extern "C" apt_status apt_dryrun(apt_trainer* t, int64_t n_steps, apt_plan_stats
         launch_pdl(dry_nd_kernel, dim3(1), dim3(32), 0, c->stream, r, l1.n_dst, dc + S);
         const int64_t blocks = std::max<int64_t>(1, std::min<int64_t>(ceil_div(l1.max_dst, 256), 148 * 8));
         launch_pdl(dry_count_kernel, dim3(blocks), dim3(256), 0, c->stream, S, r, C, l1.dst, l1.n_dst, l1.cnt, l1.nbr, l1.k, g->part,
-                                                        own_bm, n_words, dc + S);
+                                                        own_bm, n_words, dc + S, ti);
         CK(c, cudaGetLastError());
         c->launches += 4 + 4 * K;
       }
@@ -250,10 +267,11 @@ extern "C" apt_status apt_dryrun(apt_trainer* t, int64_t n_steps, apt_plan_stats
       out->n_d[S][r] = h[S].n_d[r];
       out->t_build_s[S][r] = tb[S][r];
     }
-  // GDP: local / peer rows of each requester's own block
+  // GDP: local / peer / host rows of each requester's own block
   for (int r = 0; r < C; ++r) {
     out->rows_local[APT_GDP][r] = h[APT_GDP].rows_local[r];
     out->rows_peer[APT_GDP][r] = h[APT_GDP].rows_peer[r];
+    out->rows_host[APT_GDP][r] = h[APT_GDP].rows_host[r];
   }
   // NFP: every rank reads the unique sources of every block, its column slice only;
   // receives every other block (AllBroadcast), sends (C-1) partials per own row
@@ -277,7 +295,10 @@ extern "C" apt_status apt_dryrun(apt_trainer* t, int64_t n_steps, apt_plan_stats
   // SNP: virtual nodes (r -> c != r), local reads only
   {
     const DryCounters& q = h[APT_SNP];
-    for (int cc = 0; cc < C; ++cc) out->rows_local[APT_SNP][cc] = q.rows_local[cc];
+    for (int cc = 0; cc < C; ++cc) {
+      out->rows_local[APT_SNP][cc] = q.rows_local[cc];
+      out->rows_host[APT_SNP][cc] = q.rows_host[cc];
+    }
     for (int r = 0; r < C; ++r)
       for (int cc = 0; cc < C; ++cc) {
         if (r == cc) continue;
@@ -294,6 +315,7 @@ extern "C" apt_status apt_dryrun(apt_trainer* t, int64_t n_steps, apt_plan_stats
     for (int o = 0; o < C; ++o) {
       out->rows_local[APT_DNP][o] = q.rows_local[o];
       out->rows_peer[APT_DNP][o] = q.rows_peer[o];
+      out->rows_host[APT_DNP][o] = q.rows_host[o];
     }
     for (int r = 0; r < C; ++r)
       for (int o = 0; o < C; ++o) {
@@ -309,6 +331,7 @@ extern "C" apt_status apt_dryrun(apt_trainer* t, int64_t n_steps, apt_plan_stats
     for (int r = 0; r < C; ++r) {
       if (S != APT_NFP) out->feat_bytes_local[S][r] = out->rows_local[S][r] * d * bf;
       out->feat_bytes_peer[S][r] = out->rows_peer[S][r] * d * bf;
+      out->feat_bytes_host[S][r] = out->rows_host[S][r] * d * bf;
     }
   return APT_OK;
 }

@@ -36,6 +36,8 @@ extern "C" apt_status apt_select_strategy(const apt_plan_stats* st, const apt_bw
       t += double(st->feat_bytes_local[s][r]) / b[APT_OP_LOCAL_GATHER] + steps * a[APT_OP_LOCAL_GATHER];
       if (st->feat_bytes_peer[s][r] > 0)
         t += double(st->feat_bytes_peer[s][r]) / b[APT_OP_PEER_PULL] + steps * a[APT_OP_PEER_PULL];
+      if (st->feat_bytes_host[s][r] > 0)   // host tier of the unified store
+        t += double(st->feat_bytes_host[s][r]) / b[APT_OP_HOST_GATHER] + steps * a[APT_OP_HOST_GATHER];
       // T_shuffle (+ the graph shuffle, counted in T_build by the paper but
       // modelled here too since the dry-run does not move it over NVLink)
       if (st->n_calls[s][r] > 0) {

@@ -323,6 +323,28 @@ apt_status apt_fstore_create_tiered(apt_ctx* c, const apt_graph* g, apt_strategy
         else { base_tier[u] = C; base_row[u] = -1; }
       }
     for (int64_t i = 0, h = 0; i < int64_t(host_ids.size()); ++i, ++h) base_row[host_ids[i]] = int32_t(h);
+    // HBM rows per shard + every rank's cache membership (dry-run classification)
+    f->rows_dev = f->arena.alloc<int64_t>(C, false);
+    CK(c, cudaMemcpyAsync(f->rows_dev, f->rows, sizeof(int64_t) * C, cudaMemcpyHostToDevice, c->stream));
+    const int64_t n_words = ceil_div(g->n, 32);
+    if (want_cache > 0) {
+      std::vector<uint32_t> bm(size_t(C) * n_words, 0u);
+      for (int r = 0; r < C; ++r) {
+        int64_t taken = 0;
+        for (int64_t j = 0; j < want_cache && taken < want_cache; ++j) {
+          const int64_t u = opts->hot_ids[j];
+          if (u < 0 || u >= g->n) { apt_fstore_destroy(f); return set_err(c, APT_E_INVALID, "hot id out of range"); }
+          uint32_t& w = bm[size_t(r) * n_words + (u >> 5)];
+          if (base_tier[u] == r || (w >> (u & 31) & 1u)) continue;
+          w |= 1u << (u & 31);
+          ++taken;
+        }
+      }
+      f->cache_bm = f->arena.alloc<uint32_t>(int64_t(C) * n_words, false);
+      if (!f->cache_bm) { apt_fstore_destroy(f); return set_err(c, APT_E_OOM, "cache bitmaps"); }
+      CK(c, cudaMemcpyAsync(f->cache_bm, bm.data(), sizeof(uint32_t) * bm.size(), cudaMemcpyHostToDevice, c->stream));
+    }
+    CK(c, cudaStreamSynchronize(c->stream));
     // per hosted rank: its view, with its cache of hot rows (those it does not hold in HBM)
     for (int r = 0; r < C; ++r) {
       if (!c->emulated && r != c->rank) continue;

@@ -127,7 +127,12 @@ struct apt_fstore {
   void* cache[APT_MAX_RANKS] = {};       // replicated hot rows (hosted ranks)
   int32_t* tier_map[APT_MAX_RANKS] = {}; // device [n] per hosted rank
   int32_t* trow_map[APT_MAX_RANKS] = {};
-  std::vector<int32_t> tier_h[APT_MAX_RANKS];   // host copies (dry-run counters, tests)
+  std::vector<int32_t> tier_h[APT_MAX_RANKS];   // host copies (tests)
+  // for the dry-run's tier classification of every rank's reads (all ranks, any process):
+  // u is local to r iff cached by r or (part[u] == r and lrow[u] < rows[r]); host iff
+  // lrow[u] >= rows[part[u]] and not cached by r
+  int64_t* rows_dev = nullptr;           // [C] HBM rows per shard
+  uint32_t* cache_bm = nullptr;          // [C x ceil(n/32)] cached-by-rank bitmaps (null: no caches)
   std::vector<void*> peer_opened;   // IPC-mapped peer shards (multi-process)
   apt::Arena arena;
   ~apt_fstore() {

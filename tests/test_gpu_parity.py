@@ -428,12 +428,12 @@ def test_strategy_step_matches_oracle(A, tiny, strategy, C, dtype):
 
 
 # ------------------------------------------------------------------ S12/S13 planner
-FIELDS = ("n_d", "rows_local", "rows_peer", "feat_bytes_local", "feat_bytes_peer", "graph_bytes",
-          "hidden_bytes_fwd", "hidden_bytes_bwd", "n_calls")
+FIELDS = ("n_d", "rows_local", "rows_peer", "rows_host", "feat_bytes_local", "feat_bytes_peer", "feat_bytes_host",
+          "graph_bytes", "hidden_bytes_fwd", "hidden_bytes_bwd", "n_calls")
 
 
-@pytest.mark.parametrize("C", [2, 4])
-def test_dryrun_counts_match_oracle_and_pick(A, tiny, C):
+@pytest.mark.parametrize("C,frac,n_hot", [(2, 1.0, 0), (4, 1.0, 0), (4, 0.4, 300)])
+def test_dryrun_counts_match_oracle_and_pick(A, tiny, C, frac, n_hot):
     """apt_dryrun's per-strategy, per-rank counts are integers: bit-exact against
     the oracle's emulation of every rank's blocks (O7); apt_select_strategy = oracle Eq. 2 (O8)."""
     from oracle import strategy as S
@@ -441,7 +441,9 @@ def test_dryrun_counts_match_oracle_and_pick(A, tiny, C):
     ctx = A.Ctx(-1, C, 0)
     part = aptgen.partition(g.n, C)
     gr = ctx.graph_load(g.indptr, g.indices, part)
-    fs = ctx.fstore_create(gr, A.GDP, A.F32, cfg.dim, None, cfg.feat_seed)
+    hot = np.random.default_rng(5).choice(g.n, size=n_hot, replace=False) if n_hot else None
+    fs = ctx.fstore_create(gr, A.GDP, A.F32, cfg.dim, None, cfg.feat_seed, hbm_frac=frac, hot_ids=hot)
+    tier = S.tiered_store(part, C, frac, hot, n_hot) if (frac < 1.0 or n_hot) else None
     dims = [cfg.dim] + [d for _, d in cfg.dims()]
     labels = aptgen.labels(cfg, g.n)
     tr = A.Trainer(ctx, gr, fs, dims, cfg.fanouts, cfg.batch, A.F32, 0.1, cfg.sample_seed, cfg.feat_seed, A.GDP,
@@ -458,7 +460,7 @@ def test_dryrun_counts_match_oracle_and_pick(A, tiny, C):
             gb = oracle.global_batch(perm, step, C, cfg.batch)
             seeds = S.assign_seeds(s, gb, part, C, cfg.batch)
             blocks = [oracle.sample_blocks(g, sd, cfg.fanouts, cfg.sample_seed, step)[-1] for sd in seeds]
-            for r, e in enumerate(S.emulate_layer1(s, blocks, part, C, cfg.dim, cfg.hidden, 4, 4)):
+            for r, e in enumerate(S.emulate_layer1(s, blocks, part, C, cfg.dim, cfg.hidden, 4, 4, tier=tier)):
                 for k in tot[r]:
                     tot[r][k] += e[k]
         for r in range(C):

@@ -151,3 +151,26 @@ def test_cost_model_picks_argmin_and_gdp_wins_when_shuffle_is_costly():
     beta2[S.OP_PEER_PULL] = 1e9                                # slow peer reads -> DNP
     pred2, pick2 = S.predict(stats, alpha, beta2, tb)
     assert pick2 == 3 and pred2[3] < pred2[2] < pred2[1]
+
+
+def test_tiered_store_classification_invariants(tiny_graph):
+    """Tiers of the unified store: with everything in HBM and no cache the
+    classification is the plain partition one; the host tier holds exactly the rows past
+    each partition's HBM budget; a cached row is local for its rank only."""
+    C, n = 4, tiny_graph.n
+    part = aptgen.partition(n, C)
+    ids = np.arange(n)
+    plain = S.tiered_store(part, C, 1.0)
+    for r in range(C):
+        assert np.array_equal(plain(r, ids), np.where(part == r, 0, 1))
+    t = S.tiered_store(part, C, 0.25)
+    n_host = sum(len(np.nonzero(part == o)[0]) - int(np.ceil(0.25 * (part == o).sum())) for o in range(C))
+    assert (t(0, ids) == 2).sum() == n_host
+    hot = np.arange(0, n, 97)[:50]                          # spread over all partitions
+    tc = S.tiered_store(part, C, 0.25, hot, 50)
+    for r in range(C):
+        newly_local = (tc(r, ids) == 0) & (t(r, ids) != 0)
+        # every candidate not already in r's HBM is replicated on r, nothing else changes
+        assert newly_local.sum() == int((t(r, hot) != 0).sum()) > 0
+        assert np.all(np.isin(ids[newly_local], hot))
+        assert np.array_equal(tc(r, ids)[~newly_local], t(r, ids)[~newly_local])
