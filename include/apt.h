@@ -87,6 +87,9 @@ typedef struct {
   float lr;                            /* SGD learning rate                  */
   uint64_t sample_seed;                /* Philox key of the sampler (O2)     */
   uint64_t feat_seed;                  /* synthetic features (O4)            */
+  int gat_heads;                       /* 0: GraphSAGE-mean layer 1; H in {1,2,4,8}: a GAT
+                                          layer 1 with H heads of dims[1]/H columns, concatenated
+                                          ("GAT uses attention", [45]; G1-G4)    */
 } apt_model_desc;
 
 /* Dry-run statistics, per strategy s and rank r, summed over the
@@ -228,6 +231,12 @@ apt_status apt_trainer_destroy(apt_trainer* t);
 /* Host fp32 W [d_out x d_in] row-major and b [d_out] of layer l (1..K); every rank. */
 apt_status apt_trainer_set_params(apt_trainer* t, int layer, const float* W, const float* b);
 apt_status apt_trainer_get_params(apt_trainer* t, int rank, int layer, float* W, float* b);
+/* GAT layer 1 (gat_heads > 0) attention vectors, host fp32 [dims[1]] each, head h at
+ * [h*F, (h+1)*F): e_vu^h = LeakyReLU_0.2(a_src^h . (W x_u)^h + a_dst^h . (W x_v)^h)
+ * (GAT [45]; reading G1).  Replicated on every rank; updated by SGD.
+ * APT_E_STATE on a SAGE layer 1.  Syncs.                                     */
+apt_status apt_trainer_set_attention(apt_trainer* t, const float* a_src, const float* a_dst);
+apt_status apt_trainer_get_attention(apt_trainer* t, int rank, float* a_src, float* a_dst);
 /* Epoch permutation of the train set (O1): host int64[n_train] ascending.   */
 apt_status apt_trainer_set_epoch(apt_trainer* t, const int64_t* train, int64_t n_train, uint64_t epoch);
 int64_t apt_trainer_steps_per_epoch(const apt_trainer* t);
@@ -269,7 +278,8 @@ apt_status apt_layer_fwd(apt_trainer* t, int64_t step);
 apt_status apt_layer_bwd(apt_trainer* t, const float* const* dh1, int64_t pitch);
 
 /* Readouts for tests (syncs).  what: 0 seeds, 1 layer-l dst ids, 2 Z_l (fp32),
- * 3 H_l (post-activation / logits), 4 dW_l, 5 db_l, 6 G_l (dL/dpre).
+ * 3 H_l (post-activation / logits), 4 dW_l, 5 db_l, 6 G_l (dL/dpre),
+ * 7 (GAT layer 1) the attention gradients [da_src | da_dst] (1 x 2*dims[1]).
  * Copies min(cap, rows*cols) values (int32 for ids, fp32 otherwise).         */
 apt_status apt_trainer_read(apt_trainer* t, int rank, int what, int layer, void* host, int64_t cap,
                             int64_t* rows, int* cols);

@@ -18,6 +18,9 @@ DESIGN.md §3 (G1-G6):
   G2  bias once after the aggregation, ReLU on hidden layers (Z9, Z10).
   G3  a destination with no sampled neighbour gets pre_v = b.
   G4  heads are concatenated; no attention dropout, no residual.
+  G5  SNP partial attention: per source partition, the softmax
+      state (max, sum) and the normalised partial sum travel with the partial
+      projection; the requester merges them (online-softmax combine).
 
 ``forward`` / ``backward`` follow the definition step by step (project, score,
 softmax, weighted sum; then the chain rule in reverse).  ``forward_aggfirst``
@@ -113,11 +116,18 @@ def backward(indptr, indices, x_src, n_dst, W, a_src, a_dst, cache, g, heads):
     return dW, da_src, da_dst, db
 
 
-def forward_aggfirst(indptr, indices, x_src, n_dst, W, a_src, a_dst, b, heads, relu=True, dtype="f32"):
+def forward_aggfirst(indptr, indices, x_src, n_dst, W, a_src, a_dst, b, heads, relu=True, dtype="f32", snp=None):
     """The same layer re-associated: w~_src^h = W^hT a_src^h, el_u = x_u . w~_src^h
     (and er likewise), Z_v^h = sum_u alpha_vu^h x_u, pre_v^h = W^h Z_v^h + b^h.
     dtype "bf16" rounds Z^h and W to bf16 (the CUDA path's rounding points); the
-    scores use the fp32 master W.  Returns pre, alpha, Z [n_dst x H x d]."""
+    scores use the fp32 master W.  Returns pre, alpha, Z [n_dst x H x d].
+
+    snp = (part_of_src, C): the layer as SNP computes it (P:126 -- each source
+    partition c aggregates only its own sources of v; reading G5): partition c's
+    softmax over its edges (max m_c, sum S_c), its normalised partial
+    Z_c^h = sum_{u in c} e^{e_vu - m_c} x_u / S_c (rounded in bf16 mode), projected,
+    and the partials merged with weights w_c = S_c e^{m_c - m} / sum_c' S_c' e^{m_c' - m}
+    (m = max_c m_c).  In exact arithmetic this equals the plain layer (tested)."""
     W = np.asarray(W, np.float64)
     H = heads
     dp, d = W.shape
@@ -131,12 +141,40 @@ def forward_aggfirst(indptr, indices, x_src, n_dst, W, a_src, a_dst, b, heads, r
     rows, _ = _rows(indptr)
     s = el[indices] + er[rows]
     alpha = edge_softmax(indptr, _leaky(s))
+    Wp = bf16_round(Wh) if dtype == "bf16" else Wh
+    if snp is not None:
+        part, C = snp
+        e = _leaky(s)
+        owner = np.asarray(part)[indices]
+        parts_m = np.full((C, n_dst, H), -np.inf)
+        for c in range(C):
+            sel = owner == c
+            np.maximum.at(parts_m[c], rows[sel], e[sel])
+        m = parts_m.max(axis=0)
+        Q = np.zeros((n_dst, H, F))
+        wsum = np.zeros((n_dst, H))
+        for c in range(C):
+            sel = owner == c
+            mc = parts_m[c]
+            p = np.exp(e[sel] - mc[rows[sel]])
+            Sc = np.zeros((n_dst, H))
+            np.add.at(Sc, rows[sel], p)
+            Zc = np.zeros((n_dst, H, d))
+            np.add.at(Zc, rows[sel], p[:, :, None] * x[indices[sel]][:, None, :])
+            Zc = np.where(Sc[:, :, None] > 0, Zc / np.where(Sc > 0, Sc, 1.0)[:, :, None], 0.0)
+            if dtype == "bf16":
+                Zc = bf16_round(Zc)
+            wc = np.where(Sc > 0, Sc * np.exp(np.where(Sc > 0, mc - m, 0.0)), 0.0)
+            Q += wc[:, :, None] * np.einsum("vhd,hfd->vhf", Zc, Wp)
+            wsum += wc
+        Q = np.where(wsum[:, :, None] > 0, Q / np.where(wsum > 0, wsum, 1.0)[:, :, None], 0.0)
+        pre = Q.reshape(n_dst, dp) + np.asarray(b, np.float64)
+        h = np.maximum(pre, 0.0) if relu else pre
+        return {"pre": pre, "h": h, "alpha": alpha, "Z": None, "s": s}
     Z = np.zeros((n_dst, H, d))
     np.add.at(Z, rows, alpha[:, :, None] * x[indices][:, None, :])
-    Wp = Wh
     if dtype == "bf16":
         Z = bf16_round(Z)
-        Wp = bf16_round(Wh)
     pre = np.einsum("vhd,hfd->vhf", Z, Wp).reshape(n_dst, dp) + np.asarray(b, np.float64)
     h = np.maximum(pre, 0.0) if relu else pre
     return {"pre": pre, "h": h, "alpha": alpha, "Z": Z, "s": s}

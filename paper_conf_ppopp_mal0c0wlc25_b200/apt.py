@@ -20,7 +20,7 @@ STRATEGY = {"GDP": GDP, "NFP": NFP, "SNP": SNP, "DNP": DNP, "AUTO": AUTO}
 F32, BF16 = 0, 1
 DTYPE = {"f32": F32, "bf16": BF16}
 MAX_LAYERS, MAX_RANKS = 4, 8
-READ = {"seeds": 0, "dst": 1, "Z": 2, "H": 3, "dW": 4, "db": 5, "G": 6}
+READ = {"seeds": 0, "dst": 1, "Z": 2, "H": 3, "dW": 4, "db": 5, "G": 6, "dA": 7}
 
 
 class AptError(RuntimeError):
@@ -37,7 +37,7 @@ class BlockView(C.Structure):
 class ModelDesc(C.Structure):
     _fields_ = [("n_layers", C.c_int), ("dims", C.c_int * (MAX_LAYERS + 1)), ("fanouts", C.c_int * MAX_LAYERS),
                 ("batch", C.c_int), ("dtype", C.c_int), ("lr", C.c_float), ("sample_seed", C.c_uint64),
-                ("feat_seed", C.c_uint64)]
+                ("feat_seed", C.c_uint64), ("gat_heads", C.c_int)]
 
 
 _A4 = (C.c_int64 * MAX_RANKS) * 4
@@ -109,6 +109,7 @@ def lib():
             "apt_weight_grad": [vp, vp, i64, vp, i64, i32, i64, i32, i32, vp, vp],
             "apt_trainer_create": [vp, vp, vp, vp, i32, vp, vp], "apt_trainer_destroy": [vp],
             "apt_trainer_set_params": [vp, i32, vp, vp], "apt_trainer_get_params": [vp, i32, i32, vp, vp],
+            "apt_trainer_set_attention": [vp, vp, vp], "apt_trainer_get_attention": [vp, i32, vp, vp],
             "apt_trainer_set_epoch": [vp, vp, i64, u64], "apt_trainer_step": [vp, i64, i32],
             "apt_trainer_step_host": [vp, vp, i64, i64, i32, vp], "apt_trainer_loss": [vp, vp],
             "apt_trainer_step_host_pipelined": [vp, vp, i64, i64, i32, vp, vp],
@@ -285,8 +286,9 @@ class Trainer(Handle):
     """apt_trainer: the per-mini-batch step under one strategy."""
 
     def __init__(self, ctx, graph, fstore, cfg_dims, fanouts, batch, dtype, lr, sample_seed, feat_seed, strategy,
-                 labels):
+                 labels, gat_heads=0):
         m = ModelDesc()
+        m.gat_heads = gat_heads
         m.n_layers = len(fanouts)
         for i, d in enumerate(cfg_dims):
             m.dims[i] = d
@@ -314,6 +316,18 @@ class Trainer(Handle):
             self.ctx.ck(lib().apt_trainer_get_params(self.h, rank, l, W.ctypes.data, b.ctypes.data))
             out.append((W, b))
         return out
+
+    def set_attention(self, a_src, a_dst):
+        """GAT layer 1: attention vectors [dims[1]] each (head h at [h*F, (h+1)*F))."""
+        a_src = np.ascontiguousarray(a_src, np.float32).reshape(-1)
+        a_dst = np.ascontiguousarray(a_dst, np.float32).reshape(-1)
+        self.ctx.ck(lib().apt_trainer_set_attention(self.h, a_src.ctypes.data, a_dst.ctypes.data))
+
+    def get_attention(self, rank=0):
+        a_src = np.empty(self.dims[1], np.float32)
+        a_dst = np.empty(self.dims[1], np.float32)
+        self.ctx.ck(lib().apt_trainer_get_attention(self.h, rank, a_src.ctypes.data, a_dst.ctypes.data))
+        return a_src, a_dst
 
     def set_epoch(self, train, epoch):
         train = np.ascontiguousarray(train, np.int64)

@@ -175,7 +175,7 @@ __global__ void __launch_bounds__(256) colsum_kernel2(const T* __restrict__ g, i
   }
 }
 
-static apt_status launch_colsum2(apt_ctx* c, const void* g, bool bf16, int64_t pitch, int dim, const int32_t* n_dev,
+apt_status launch_colsum2(apt_ctx* c, const void* g, bool bf16, int64_t pitch, int dim, const int32_t* n_dev,
                                  float* out) {
   if (dim > 1024) return set_err(c, APT_E_UNSUPPORTED, "colsum: dim > 1024");
   const int blocks = 296;
@@ -272,6 +272,7 @@ apt_status strategy_tables(apt_trainer* t) {
     }
   }
   t->H1_tab = upload_tab(t, h1);
+  t->h1_host = h1;
   t->G1_tab = upload_tab(t, g1);
   t->Gb1_tab = upload_tab(t, gb1);
   t->wn_tab = upload_tab(t, wn);
@@ -283,17 +284,26 @@ apt_status strategy_tables(apt_trainer* t) {
 }
 
 // ------------------------------------------------------------------ forward
+// Owner: re-sample the items' nodes -- the same (seed, node, hop, step) key gives the
+// requester's sample bit for bit (readings Z2 / Z18).
+apt_status resample_items(apt_trainer* t, RankState& rs) {
+  apt_ctx* c = t->ctx;
+  Xchg& x = rs.x;
+  const Hop& hp = rs.hops[t->K - 1];
+  SampleArgs sa{t->g->indptr, t->g->indices, x.work_gid, x.n_work, x.wcap, hp.k,
+                philox_key(t->m.sample_seed, kDomSample), t->step_dev, t->K - 1, x.wcnt, x.wnbr};
+  CK(c, launch_sample(sa, c->stream));
+  c->launches++;
+  return APT_OK;
+}
+
 static apt_status owner_execute(apt_trainer* t, RankState& rs, bool time_it) {
   apt_ctx* c = t->ctx;
   Xchg& x = rs.x;
   Layer& L = rs.L[0];
   const Hop& hp = rs.hops[t->K - 1];
   const bool bf = t->m.dtype == APT_BF16;
-  const int hop = t->K - 1;
-  // re-sample the items' nodes: same (seed, node, hop, step) key => the requester's sample
-  SampleArgs sa{t->g->indptr, t->g->indices, x.work_gid, x.n_work, x.wcap, hp.k,
-                philox_key(t->m.sample_seed, kDomSample), t->step_dev, hop, x.wcnt, x.wnbr};
-  CK(c, launch_sample(sa, c->stream));
+  { apt_status s = resample_items(t, rs); if (s != APT_OK) return s; }
   // Execute (S6+S7): fused gather + mean over the items (SNP: own sources only)
   AggArgs a{};
   a.cnt = x.wcnt; a.nbr = x.wnbr; a.k = hp.k;
@@ -306,7 +316,7 @@ static apt_status owner_execute(apt_trainer* t, RankState& rs, bool time_it) {
   CK(c, launch_agg_fstore(a, feat_view(t->f, rs.rank), c->stream));
   if (time_it) CK(c, t->capturing ? cudaEventRecordWithFlags(t->ev[7], c->stream, cudaEventRecordExternal)
                                   : cudaEventRecord(t->ev[7], c->stream));
-  c->launches += 2;
+  c->launches++;
   // Projection with the Reshuffle fused into its epilogue (S8+S9): rows routed to the
   // requesters' h^1 buffers; DNP stores act(Y + b), SNP/NFP add partial Y.
   const bool partial = t->s != APT_DNP;
@@ -341,10 +351,13 @@ static apt_status owner_execute(apt_trainer* t, RankState& rs, bool time_it) {
   return APT_OK;
 }
 
-apt_status layer1_fwd_strategy(apt_trainer* t) {
+// Permute + Shuffle (S4/S5) of the layer-1 rows into the owners' work lists (shared
+// by the SAGE and the GAT first layer).  zero_h: also clear the requesters' h^1
+// (the partial strategies accumulate into it).
+apt_status shuffle_items(apt_trainer* t, bool zero_h) {
   apt_ctx* c = t->ctx;
   const int mode = t->s == APT_DNP ? 0 : t->s == APT_SNP ? 1 : 2;
-  const bool partial = t->s != APT_DNP;
+  const bool partial = zero_h;
   WorkTab w{t->wn_tab, t->wrank_tab, t->wrow_tab, t->wgid_tab};
   // Permute + Shuffle: clear owners' lists (and the requesters' partial-sum buffers),
   // then every requester pushes its layer-1 rows
@@ -363,7 +376,13 @@ apt_status layer1_fwd_strategy(apt_trainer* t) {
     CK(c, cudaGetLastError());
     c->launches++;
   }
-  { apt_status s = device_barrier(c); if (s != APT_OK) return s; }   // every list complete
+  return device_barrier(c);   // every list complete
+}
+
+apt_status layer1_fwd_strategy(apt_trainer* t) {
+  apt_ctx* c = t->ctx;
+  const bool partial = t->s != APT_DNP;
+  { apt_status s = shuffle_items(t, partial); if (s != APT_OK) return s; }
   // Execute + Reshuffle on every owner
   bool first = true;
   for (auto& rs : t->R) {

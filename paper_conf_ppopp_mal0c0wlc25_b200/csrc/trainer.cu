@@ -31,6 +31,23 @@ apt_status strategy_alloc(apt_trainer* t, RankState& rs);
 apt_status strategy_tables(apt_trainer* t);
 apt_status layer1_fwd_strategy(apt_trainer* t);
 apt_status layer1_bwd_strategy(apt_trainer* t);
+apt_status gat_alloc(apt_trainer* t, RankState& rs);
+apt_status gat_tables(apt_trainer* t);
+apt_status gat_layer1_fwd(apt_trainer* t, bool time_it);
+apt_status gat_layer1_bwd(apt_trainer* t);
+
+// Floats of the flat gradient buffer [dW1 db1 (da_src1 da_dst1 for a GAT layer 1) dW2 db2 ...].
+int64_t grad_floats(const apt_trainer* t, const RankState& rs) {
+  int64_t P = 0;
+  for (auto& L : rs.L) P += int64_t(L.d_out) * L.d_in + L.d_out;
+  if (t->gat_heads) P += 2 * int64_t(rs.L[0].d_out);
+  return P;
+}
+// ... of its layer-1 part
+static int64_t grad_floats_l1(const apt_trainer* t) {
+  const Layer& L = t->R[0].L[0];
+  return int64_t(L.d_out) * L.d_in + L.d_out + (t->gat_heads ? 2 * int64_t(L.d_out) : 0);
+}
 }  // namespace apt
 
 #define CK(ctx, expr)                                        \
@@ -189,8 +206,12 @@ apt_status apt_trainer_create(apt_ctx* c, const apt_graph* g, const apt_fstore* 
   for (int l = 0; l < m->n_layers; ++l)
     if (m->fanouts[l] < 1 || m->fanouts[l] > 256 || m->dims[l + 1] < 1)
       return set_err(c, APT_E_INVALID, "apt_trainer_create: fanout/dim out of range");
+  if (m->gat_heads < 0 || m->gat_heads > 8 || (m->gat_heads & (m->gat_heads - 1)) ||
+      (m->gat_heads && m->dims[1] % m->gat_heads))
+    return set_err(c, APT_E_INVALID, "apt_trainer_create: gat_heads must be 0, 1, 2, 4 or 8 and divide dims[1]");
   auto* t = new apt_trainer();
   t->ctx = c;
+  t->gat_heads = m->gat_heads;
   ctx_retain(c);
   t->g = g;
   t->f = f;
@@ -284,8 +305,7 @@ apt_status apt_trainer_create(apt_ctx* c, const apt_graph* g, const apt_fstore* 
       L.Wb = A.alloc<uint16_t>(int64_t(L.d_out) * L.wb_pitch, true);
     }
     // flat gradient buffer [dW1 db1 dW2 db2 ...] so one all-reduce covers the model
-    int64_t P = 0;
-    for (auto& L : rs.L) P += int64_t(L.d_out) * L.d_in + L.d_out;
+    const int64_t P = grad_floats(t, rs);
     float* grads = A.alloc<float>(P, true);
     int64_t off = 0;
     for (auto& L : rs.L) {
@@ -293,6 +313,11 @@ apt_status apt_trainer_create(apt_ctx* c, const apt_graph* g, const apt_fstore* 
       off += int64_t(L.d_out) * L.d_in;
       L.db = grads + off;
       off += L.d_out;
+      if (&L == &rs.L[0] && t->gat_heads) {
+        rs.ga.da_src = grads + off;
+        rs.ga.da_dst = grads + off + L.d_out;
+        off += 2 * int64_t(L.d_out);
+      }
     }
     if (!rs.seeds || !rs.pos || !grads) {
       apt_trainer_destroy(t);
@@ -302,9 +327,17 @@ apt_status apt_trainer_create(apt_ctx* c, const apt_graph* g, const apt_fstore* 
       apt_status st = strategy_alloc(t, rs);
       if (st != APT_OK) { apt_trainer_destroy(t); return st; }
     }
+    if (t->gat_heads) {
+      apt_status st = gat_alloc(t, rs);
+      if (st != APT_OK) { apt_trainer_destroy(t); return st; }
+    }
   }
   if (C > 1 && s != APT_GDP) {
     apt_status st = strategy_tables(t);
+    if (st != APT_OK) { apt_trainer_destroy(t); return st; }
+  }
+  if (t->gat_heads) {
+    apt_status st = gat_tables(t);
     if (st != APT_OK) { apt_trainer_destroy(t); return st; }
   }
   if (multiprocess(c)) {
@@ -312,8 +345,7 @@ apt_status apt_trainer_create(apt_ctx* c, const apt_graph* g, const apt_fstore* 
     std::vector<void*> v(C, nullptr);
     apt_status st = share_ptr(c, t->R[0].L[0].dW, v.data(), &t->peer_opened);
     if (st != APT_OK) { apt_trainer_destroy(t); return st; }
-    int64_t P = 0;
-    for (auto& L : t->R[0].L) P += int64_t(L.d_out) * L.d_in + L.d_out;
+    const int64_t P = grad_floats(t, t->R[0]);
     t->ar_scratch = A.alloc<float>(P, false);
     t->dW_tab = A.alloc<float*>(C, false);
     CK(c, cudaMemcpyAsync(t->dW_tab, v.data(), sizeof(float*) * C, cudaMemcpyHostToDevice, c->stream));
@@ -394,6 +426,31 @@ apt_status apt_trainer_get_params(apt_trainer* t, int rank, int layer, float* W,
       return APT_OK;
     }
   return set_err(t->ctx, APT_E_INVALID, "get_params: rank %d not hosted", rank);
+}
+
+apt_status apt_trainer_set_attention(apt_trainer* t, const float* a_src, const float* a_dst) {
+  if (!t || !a_src || !a_dst) return set_err(t ? t->ctx : nullptr, APT_E_INVALID, "set_attention: bad args");
+  if (!t->gat_heads) return set_err(t->ctx, APT_E_STATE, "set_attention: layer 1 is not a GAT layer");
+  apt_ctx* c = t->ctx;
+  for (auto& rs : t->R) {
+    CK(c, cudaMemcpyAsync(rs.ga.a_src, a_src, sizeof(float) * rs.L[0].d_out, cudaMemcpyHostToDevice, c->stream));
+    CK(c, cudaMemcpyAsync(rs.ga.a_dst, a_dst, sizeof(float) * rs.L[0].d_out, cudaMemcpyHostToDevice, c->stream));
+  }
+  CK(c, cudaStreamSynchronize(c->stream));
+  return APT_OK;
+}
+
+apt_status apt_trainer_get_attention(apt_trainer* t, int rank, float* a_src, float* a_dst) {
+  if (!t || !a_src || !a_dst) return set_err(t ? t->ctx : nullptr, APT_E_INVALID, "get_attention: bad args");
+  if (!t->gat_heads) return set_err(t->ctx, APT_E_STATE, "get_attention: layer 1 is not a GAT layer");
+  for (auto& rs : t->R)
+    if (rs.rank == rank) {
+      CK(t->ctx, cudaStreamSynchronize(t->ctx->stream));
+      CK(t->ctx, cudaMemcpy(a_src, rs.ga.a_src, sizeof(float) * rs.L[0].d_out, cudaMemcpyDeviceToHost));
+      CK(t->ctx, cudaMemcpy(a_dst, rs.ga.a_dst, sizeof(float) * rs.L[0].d_out, cudaMemcpyDeviceToHost));
+      return APT_OK;
+    }
+  return set_err(t->ctx, APT_E_INVALID, "get_attention: rank %d not hosted", rank);
 }
 
 apt_status apt_trainer_set_epoch(apt_trainer* t, const int64_t* train, int64_t n_train, uint64_t epoch) {
@@ -658,8 +715,7 @@ apt_status allreduce_grads(apt_trainer* t, int64_t P) {
 
 apt_status allreduce_sgd(apt_trainer* t, int update) {
   apt_ctx* c = t->ctx;
-  int64_t P = 0;
-  for (auto& L : t->R[0].L) P += int64_t(L.d_out) * L.d_in + L.d_out;
+  const int64_t P = grad_floats(t, t->R[0]);
   if (t->world > 1) {
     apt_status s = allreduce_grads(t, P);
     if (s != APT_OK) return s;
@@ -687,6 +743,10 @@ apt_status allreduce_sgd(apt_trainer* t, int update) {
         return st;
       }
       if ((st = add(L.b, L.db, L.d_out, nullptr, 1, 0)) != APT_OK) return st;
+      if (&L == &rs.L[0] && t->gat_heads &&
+          ((st = add(rs.ga.a_src, rs.ga.da_src, L.d_out, nullptr, 1, 0)) != APT_OK ||
+           (st = add(rs.ga.a_dst, rs.ga.da_dst, L.d_out, nullptr, 1, 0)) != APT_OK))
+        return st;
     }
   }
   if (bt.n) {
@@ -735,7 +795,10 @@ apt_status compute_body(apt_trainer* t, int update) {
   apt_ctx* c = t->ctx;
   const bool gdp = t->world == 1 || t->s == APT_GDP;
   CK(c, record_ev(t, 1));
-  if (gdp) {
+  if (t->gat_heads) {
+    apt_status s = gat_layer1_fwd(t, true);
+    if (s != APT_OK) return s;
+  } else if (gdp) {
     bool first = true;
     for (auto& rs : t->R) {
       apt_status s = layer1_fwd_gdp(t, rs, first);
@@ -753,16 +816,15 @@ apt_status compute_body(apt_trainer* t, int update) {
   }
   CK(c, record_ev(t, 3));
   // zero the gradient accumulators, then backward
-  for (auto& rs : t->R) {
-    int64_t P = 0;
-    for (auto& L : rs.L) P += int64_t(L.d_out) * L.d_in + L.d_out;
-    CK(c, cudaMemsetAsync(rs.L[0].dW, 0, sizeof(float) * P, c->stream));
-  }
+  for (auto& rs : t->R) CK(c, cudaMemsetAsync(rs.L[0].dW, 0, sizeof(float) * grad_floats(t, rs), c->stream));
   for (auto& rs : t->R) {
     apt_status s = upper_bwd(t, rs);
     if (s != APT_OK) return s;
   }
-  if (gdp) {
+  if (t->gat_heads) {
+    apt_status s = gat_layer1_bwd(t);
+    if (s != APT_OK) return s;
+  } else if (gdp) {
     for (auto& rs : t->R) {
       apt_status s = layer1_bwd_gdp(t, rs);
       if (s != APT_OK) return s;
@@ -804,7 +866,9 @@ apt_status apt_layer_fwd(apt_trainer* t, int64_t step) {
   }
   activate(t, 0);
   apt_status s = APT_OK;
-  if (t->world == 1 || t->s == APT_GDP) {
+  if (t->gat_heads) {
+    return gat_layer1_fwd(t, false);
+  } else if (t->world == 1 || t->s == APT_GDP) {
     bool first = true;
     for (auto& rs : t->R) {
       s = layer1_fwd_gdp(t, rs, first);
@@ -837,10 +901,13 @@ apt_status apt_layer_bwd(apt_trainer* t, const float* const* dh1, int64_t pitch)
     if (bf) CK(c, launch_grad_finish(L.G, L.h_pitch, L.H, L.h_pitch, L.d_out, relu, L.Gb, L.gb_pitch, L.n_rows,
                                      L.max_rows, c->stream));
     else if (relu) CK(c, launch_relu_bwd(L.G, L.H, L.h_pitch, L.d_out, L.n_rows, L.max_rows, c->stream));
-    CK(c, cudaMemsetAsync(L.dW, 0, sizeof(float) * (int64_t(L.d_out) * L.d_in + L.d_out), c->stream));
+    CK(c, cudaMemsetAsync(L.dW, 0, sizeof(float) * grad_floats_l1(t), c->stream));
     c->launches++;
   }
-  if (t->world == 1 || t->s == APT_GDP) {
+  if (t->gat_heads) {
+    apt_status s = gat_layer1_bwd(t);
+    if (s != APT_OK) return s;
+  } else if (t->world == 1 || t->s == APT_GDP) {
     for (auto& rs : t->R) {
       apt_status s = layer1_bwd_gdp(t, rs);
       if (s != APT_OK) return s;
@@ -849,10 +916,7 @@ apt_status apt_layer_bwd(apt_trainer* t, const float* const* dh1, int64_t pitch)
     apt_status s = layer1_bwd_strategy(t);
     if (s != APT_OK) return s;
   }
-  if (t->world > 1) {
-    const Layer& L = t->R[0].L[0];
-    return allreduce_grads(t, int64_t(L.d_out) * L.d_in + L.d_out);
-  }
+  if (t->world > 1) return allreduce_grads(t, grad_floats_l1(t));
   return APT_OK;
 }
 
@@ -1202,6 +1266,10 @@ apt_status apt_trainer_read(apt_trainer* t, int rank, int what, int layer, void*
     }
     case 5: { const Layer& L = rs->L[layer - 1]; return copy_rows(L.db, 1, L.d_out, L.d_out, 4, false); }
     case 6: { const Layer& L = rs->L[layer - 1]; return copy_rows(L.G, count(L.n_rows), L.d_out, L.h_pitch, 4, false); }
+    case 7: {   // GAT layer 1: [da_src | da_dst]
+      if (!t->gat_heads || layer != 1) return set_err(c, APT_E_INVALID, "read: no attention gradients (GAT layer 1 only)");
+      return copy_rows(rs->ga.da_src, 1, 2 * rs->L[0].d_out, 2 * rs->L[0].d_out, 4, false);
+    }
     default: return set_err(c, APT_E_INVALID, "read: unknown item %d", what);
   }
 }

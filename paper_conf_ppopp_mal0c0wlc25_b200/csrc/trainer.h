@@ -74,6 +74,40 @@ struct Xchg {
   float* dW1s = nullptr;             // [d_out x w_cols]
 };
 
+// GAT first layer (gat.cu).  Every strategy runs as owners
+// processing work items (GDP: the rank's own rows); per item the owner keeps the
+// per-head aggregate Z^h = sum_u alpha_vu^h x_u, the LeakyReLU scores and the
+// softmax statistics for the backward.
+struct GatState {
+  int H = 0, F = 0;                  // heads, per-head width (d_out = H*F)
+  int cols = 0;                      // aggregated feature columns (d, or the NFP slice)
+  int64_t zp = 0;                    // per-head pitch of Z (elements); an item's Z row is H*zp
+  int64_t icap = 0;                  // item capacity
+  float* a_src = nullptr;            // [d_out] attention vectors (replicated)
+  float* a_dst = nullptr;
+  float* da_src = nullptr;           // [d_out] in the flat gradient buffer (after db^1)
+  float* da_dst = nullptr;
+  float* wt = nullptr;               // [2][H][cols] w~ = W^hT a^h (src, dst)
+  float* dwt = nullptr;              // [2][H][cols] dL/dw~ accumulators
+  void* Z = nullptr;                 // [icap][H][zp] bf16 or fp32
+  float* esc = nullptr;              // [icap*k][H] LeakyReLU scores
+  float* Lm = nullptr;               // [icap][H] log-sum-exp (SNP: the partial max m_c)
+  float* Ss = nullptr;               // [icap][H] SNP: partial sum S_c
+  float* Lb = nullptr;               // [icap][H] backward: the (global) log-sum-exp of the item
+  float* tb = nullptr;               // [icap][H] backward: t = g . (pre - b) of the item
+  float* wG = nullptr;               // [icap][d_out] gathered g (fp32)
+  float* wGs = nullptr;              // [icap][d_out] g scaled by the SNP merge weight (else == wG)
+  float* Gam = nullptr;              // [icap][H][cols] gamma^h = W^hT g^h
+  float** otab = nullptr;            // [H][C] routed projection targets per head
+  // requester side
+  float* t = nullptr;                // [max_rows][H]
+  float* Lr = nullptr;               // [max_rows][H] SNP: merged log-sum-exp
+  float* slot = nullptr;             // SNP: [max_rows][C][slot_pitch] partial (Q, m_c, S_c)
+  int64_t slot_pitch = 0;
+  float* ssum = nullptr;             // NFP: [max_rows][k][H] summed partial scores
+  float* dsum = nullptr;             // NFP: [max_rows][k][H] summed partial dalpha
+};
+
 // The sampled mini-batch of one step (seeds, K hops, block transposes).  Two per
 // rank: step t+1 is sampled into one while step t computes on the other.
 struct SampleSet {
@@ -97,6 +131,7 @@ struct RankState {
   int32_t* partials = nullptr;
   float* loss = nullptr;
   Xchg x;
+  GatState ga;
 };
 
 }  // namespace apt
@@ -117,12 +152,22 @@ struct apt_trainer {
   // device pointer tables for cross-rank kernels (peer pointers in a multi-GPU job)
   float** dW_tab = nullptr;
   float** H1_tab = nullptr;          // requesters' layer-1 outputs
+  std::vector<float*> h1_host;       // ... the same pointers on the host
   float** G1_tab = nullptr;          // requesters' layer-1 dL/dpre (fp32)
   uint16_t** Gb1_tab = nullptr;      // ... bf16
   int32_t** wn_tab = nullptr;        // owners' work counters / lists
   int32_t** wrank_tab = nullptr;
   int32_t** wrow_tab = nullptr;
   int32_t** wgid_tab = nullptr;
+  // GAT first layer (gat_heads > 0): requesters' buffers seen by every rank
+  int gat_heads = 0;
+  float** gt_tab = nullptr;          // t
+  float** gL_tab = nullptr;          // SNP merged log-sum-exp
+  float** slot_tab = nullptr;        // SNP partial slots
+  float** ssum_tab = nullptr;        // NFP score sums
+  float** dsum_tab = nullptr;        // NFP dalpha sums
+  float** gG_tab = nullptr;          // requesters' G (fp32)
+  uint16_t** gGb_tab = nullptr;      // requesters' Gb (bf16)
   bool use_graph = false;
   bool capturing = false;
   // pipelining: step t+1 is sampled on ctx->samp while step t computes

@@ -143,3 +143,17 @@ def test_bf16_emulation_rounds_only_z_and_w():
     assert np.allclose(oracle.bf16_round(f["Z"]), h["Z"], rtol=0, atol=0)
     bound = np.abs(f["Z"]).reshape(len(f["Z"]), -1).sum(1).max() * np.abs(W).max() * 2.0 ** -8
     assert np.abs(f["pre"] - h["pre"]).max() <= bound
+
+
+@pytest.mark.parametrize("C", [2, 3])
+def test_snp_partial_merge_equals_definition(C):
+    # SNP's per-partition softmax state + merge (reading G5) re-associates the same sums
+    rng = np.random.default_rng(10 + C)
+    indptr, indices, n_src = _rand_block(rng, 12, 20, 6)
+    d, H, F = 6, 4, 2
+    x = rng.normal(size=(n_src, d))
+    P = _params(rng, d, H, F)
+    part = rng.integers(0, C, n_src)
+    a = gat.forward(indptr, indices, x, len(indptr) - 1, *P, H)
+    b = gat.forward_aggfirst(indptr, indices, x, len(indptr) - 1, *P, H, snp=(part, C))
+    assert np.allclose(a["pre"], b["pre"], rtol=1e-12, atol=1e-12)
