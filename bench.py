@@ -60,6 +60,11 @@ def parse():
     ap.add_argument("--emulate-max-c", type=int, default=4,
                     help="also time every strategy with C ranks emulated on the GPU, for C up to this")
     ap.add_argument("--verbose", action="store_true")
+    ap.add_argument("--gat-heads", type=int, default=0,
+                    help="layer 1 as a GAT layer with this many heads (BASELINE config 5; 0: GraphSAGE-mean)")
+    ap.add_argument("--feat-dim", type=int, default=0, help="override the config's input dim d (sweeps)")
+    ap.add_argument("--hidden", type=int, default=0, help="override the config's hidden dim d' (sweeps)")
+    ap.add_argument("--fanouts", default="", help="override the fanouts, e.g. 15,10 (layer 1 first; NEXT #4 sweep)")
     return ap.parse_args()
 
 
@@ -67,10 +72,15 @@ def dist_env():
     return int(os.environ.get("RANK", 0)), int(os.environ.get("WORLD_SIZE", 1)), int(os.environ.get("LOCAL_RANK", 0))
 
 
+GAT_HEADS = 0   # set from --gat-heads
+
+
 def workload_config(cfg):
+    dims = "->".join(str(d) for d in [cfg.dim] + [o for _, o in cfg.dims()])
     return {"workload": f"synthetic ogbn-{cfg.name} shape (R-MAT {cfg.n} nodes / {cfg.m} undirected edges)"
             if cfg.name != "tiny" else f"tiny R-MAT {cfg.n} nodes / {cfg.m} edges",
-            "model": "GraphSAGE-mean " + "->".join(str(d) for d in [cfg.dim] + [o for _, o in cfg.dims()]),
+            "model": (f"GAT layer 1 ({GAT_HEADS} heads) + GraphSAGE-mean upper layers " + dims) if GAT_HEADS
+            else "GraphSAGE-mean " + dims,
             "fanouts": list(cfg.fanouts), "batch_per_gpu": cfg.batch, "feat_dim": cfg.dim}
 
 
@@ -133,10 +143,43 @@ def oracle_steps(cfg, g, train, labels, n_steps, world=1):
             seeds = perm[t * B:(t + 1) * B]
             t0 = time.perf_counter()
             blocks = oracle.sample_blocks(g, seeds, cfg.fanouts, cfg.sample_seed, t)
-            model.train_step(blocks, cfg.feat_seed, cfg.dim, params, labels[seeds], len(seeds), "bf16")
+            if GAT_HEADS:
+                gat_oracle_step(cfg, blocks, params, labels[seeds], len(seeds))
+            else:
+                model.train_step(blocks, cfg.feat_seed, cfg.dim, params, labels[seeds], len(seeds), "bf16")
             times.append(time.perf_counter() - t0)
             seeds_done += len(seeds)
     return times, seeds_done
+
+
+def gat_oracle_step(cfg, blocks, params, labels_s, n_global):
+    """The oracle's step with a GAT first layer (oracle/gat.py, fp64) and SAGE-mean upper
+    layers: forward, CE loss, backward of every layer (test infrastructure timed as a baseline)."""
+    import oracle
+    from oracle import gat, model
+    K = len(blocks)
+    blk = blocks[K - 1]
+    x = oracle.features(cfg.feat_seed, blk.src, cfg.dim)
+    W1, b1 = params[0]
+    F = W1.shape[0] // GAT_HEADS
+    rng = np.random.default_rng(cfg.weight_seed + 100)
+    a_s = (rng.normal(size=W1.shape[0]) * 0.3).reshape(GAT_HEADS, F)
+    a_d = (rng.normal(size=W1.shape[0]) * 0.3).reshape(GAT_HEADS, F)
+    c = gat.forward(blk.indptr, blk.indices, x, blk.n_dst, W1, a_s, a_d, b1, GAT_HEADS, relu=K > 1)
+    Hs, pres = [c["h"]], [c["pre"]]
+    for l in range(2, K + 1):
+        b2 = blocks[K - l]
+        W, b = params[l - 1]
+        pre = oracle.aggregate(b2.indptr, b2.indices, Hs[-1]) @ W.T + b
+        pres.append(pre)
+        Hs.append(np.maximum(pre, 0.0) if l < K else pre)
+    _, gl = model.ce_loss_grad(Hs[-1], labels_s, n_global)
+    for l in range(K, 1, -1):
+        b2 = blocks[K - l]
+        W, _ = params[l - 1]
+        dH = oracle.aggregate_bwd(b2.indptr, b2.indices, gl @ W, b2.n_src)
+        gl = dH * (pres[l - 2] > 0)
+    gat.backward(blk.indptr, blk.indices, x, blk.n_dst, W1, a_s, a_d, c, gl, GAT_HEADS)
 
 
 def run_reference(args, cfg):
@@ -200,8 +243,7 @@ def run_apt(args, cfg):
     gr = ctx.graph_load(g.indptr, g.indices, part)
     strat = A.STRATEGY[args.strategy]
     fs = ctx.fstore_create(gr, strat if strat == A.NFP else A.GDP, dt, cfg.dim, None, cfg.feat_seed)
-    dims = [cfg.dim] + [d for _, d in cfg.dims()]
-    tr = A.Trainer(ctx, gr, fs, dims, cfg.fanouts, cfg.batch, dt, 0.05, cfg.sample_seed, cfg.feat_seed, strat, labels)
+    tr = make_trainer(A, ctx, gr, fs, cfg, dt, strat, labels)
     tr.set_params(aptgen.weights(cfg))
     tr.set_epoch(train, 0)
     tr.use_graph(not args.no_graph)
@@ -292,7 +334,8 @@ def run_apt(args, cfg):
         "gpu_launches": int(launches),
         "roofline": {"bound": "hbm", "achieved": achieved, "peak": hbm_peak, "unit": "GB/s",
                      "frac": (achieved / hbm_peak) if achieved else None, "traffic": None,
-                     "kernel": "agg_kernel (layer-1 fused gather+mean)",
+                     "kernel": "gat_fwd_kernel (layer-1 fused gather+attention+weighted sums)" if GAT_HEADS
+                     else "agg_kernel (layer-1 fused gather+mean)",
                      "peak_source": "MEASURED_PEAKS.json hbm_gbs" if peaks else "fallback 6.65 TB/s",
                      "share_of_step": mean_agg / ms_local},
         "phases_ms": {"sample": phase_mean[0], "layer1_fwd": phase_mean[1], "upper_fwd_loss": phase_mean[2],
@@ -305,7 +348,8 @@ def run_apt(args, cfg):
         times, nseeds = oracle_steps(cfg, g, train, labels, args.cpu_steps, 1)
         out["cpu_baseline"] = {"value": nseeds / sum(times), "unit": "seeds/s", "cores": 1, "kind": "oracle",
                                "sample": f"first {args.cpu_steps} steps of epoch 0 ({cfg.batch} seeds each, "
-                                         f"full step: sampling + fp64 SAGE fwd/bwd), one host thread"}
+                                         f"full step: sampling + fp64 {'GAT layer 1 + ' if GAT_HEADS else ''}SAGE "
+                                         f"fwd/bwd), one host thread"}
     if rank == 0:
         print(json.dumps(out), flush=True)
     if world > 1:
@@ -326,9 +370,7 @@ def planner_report(A, g, cfg, train, labels, args, stream, gdp_ms):
         ctx = A.Ctx(-1, C, 0, stream.cuda_stream)
         gr = ctx.graph_load(g.indptr, g.indices, aptgen.partition(g.n, C))
         fs = ctx.fstore_create(gr, A.GDP, dt, cfg.dim, None, cfg.feat_seed)
-        dims = [cfg.dim] + [d for _, d in cfg.dims()]
-        tr = A.Trainer(ctx, gr, fs, dims, cfg.fanouts, cfg.batch, dt, 0.05, cfg.sample_seed, cfg.feat_seed, A.GDP,
-                       labels)
+        tr = make_trainer(A, ctx, gr, fs, cfg, dt, A.GDP, labels)
         tr.set_epoch(train, 0)
         st = tr.dryrun(args.dryrun_steps)
         bw = ctx.profile_links()
@@ -367,9 +409,7 @@ def emulated_strategy_times(A, g, cfg, train, labels, C, dt, stream, steps=5):
         ctx = A.Ctx(-1, C, 0, stream.cuda_stream)
         gr = ctx.graph_load(g.indptr, g.indices, aptgen.partition(g.n, C))
         fs = ctx.fstore_create(gr, A.NFP if s == "NFP" else A.GDP, dt, cfg.dim, None, cfg.feat_seed)
-        dims = [cfg.dim] + [d for _, d in cfg.dims()]
-        tr = A.Trainer(ctx, gr, fs, dims, cfg.fanouts, cfg.batch, dt, 0.05, cfg.sample_seed, cfg.feat_seed,
-                       A.STRATEGY[s], labels)
+        tr = make_trainer(A, ctx, gr, fs, cfg, dt, A.STRATEGY[s], labels)
         tr.set_params(aptgen.weights(cfg))
         tr.set_epoch(train, 0)
         tr.use_graph(True)
@@ -398,13 +438,38 @@ def layer1_bytes(ctx, gr, tr, cfg, rank, step, bf):
     b = ctx.sample(gr, seeds, len(seeds), cfg.fanouts, cfg.sample_seed, step)
     v = b.block(len(cfg.fanouts) - 1)
     n = v.n_dst * 4 + v.n_edges * 4 + v.n_src * cfg.dim * bf + v.n_dst * cfg.dim * bf
+    if GAT_HEADS:   # GAT: per-head Z rows and the per-edge scores kept for the backward
+        n += v.n_dst * cfg.dim * bf * (GAT_HEADS - 1) + v.n_edges * GAT_HEADS * 4
     b.close()
     return n
 
 
+def make_trainer(A, ctx, gr, fs, cfg, dt, strat, labels, lr=0.05):
+    """The product's trainer for this workload (GAT layer 1 when --gat-heads > 0)."""
+    dims = [cfg.dim] + [d for _, d in cfg.dims()]
+    tr = A.Trainer(ctx, gr, fs, dims, cfg.fanouts, cfg.batch, dt, lr, cfg.sample_seed, cfg.feat_seed, strat, labels,
+                   gat_heads=GAT_HEADS)
+    if GAT_HEADS:
+        rng = np.random.default_rng(cfg.weight_seed + 100)
+        tr.set_attention((rng.normal(size=dims[1]) * 0.3).astype(np.float32),
+                         (rng.normal(size=dims[1]) * 0.3).astype(np.float32))
+    return tr
+
+
 def main():
+    global GAT_HEADS
     args = parse()
     cfg = aptgen.CONFIGS[args.config]
+    GAT_HEADS = args.gat_heads
+    over = {}
+    if args.feat_dim:
+        over["dim"] = args.feat_dim
+    if args.hidden:
+        over["hidden"] = args.hidden
+    if args.fanouts:
+        over["fanouts"] = tuple(int(x) for x in args.fanouts.split(","))
+    if over:
+        cfg = cfg.replace(**over)
     if args.impl == "reference":
         return run_reference(args, cfg)
     return run_apt(args, cfg)

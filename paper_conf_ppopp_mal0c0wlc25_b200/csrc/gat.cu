@@ -90,7 +90,8 @@ struct GatKArgs {
   void* Z; int z_bf16; int64_t zp;
   float* const* slot_tab; int64_t slot_pitch; int d_out; int C;
   // backward
-  const float* gam;       // [icap][H][cols]
+  const float* gam;       // [icap][H][gp]
+  int64_t gp;
   const float* tb;        // [icap][H]
   const float* Lb;        // [icap][H]
   float* dwt;             // [2][H][cols]
@@ -219,13 +220,17 @@ __global__ void __launch_bounds__(256) gat_fwd_kernel(GatKArgs a) {
           for (int h = 0; h < H; ++h) {
             const float ev = s[h] > 0.f ? s[h] : kSlope * s[h];
             if (l == 0) a.esc[(i * k + e) * H + h] = ev;
-            const float mn = fmaxf(m[h], ev);
-            const float sc = expf(m[h] - mn);
-            const float p = expf(ev - mn);
-            S[h] = fmaf(S[h], sc, p);
+            if (ev > m[h]) {            // new running max (uniform in the lane group): rescale once
+              const float sc = __expf(m[h] - ev);
+              S[h] *= sc;
 #pragma unroll
-            for (int qq = 0; qq < EPV; ++qq) acc[h][qq] = fmaf(acc[h][qq], sc, p * xu[qq]);
-            m[h] = mn;
+              for (int qq = 0; qq < EPV; ++qq) acc[h][qq] *= sc;
+              m[h] = ev;
+            }
+            const float p = __expf(ev - m[h]);
+            S[h] += p;
+#pragma unroll
+            for (int qq = 0; qq < EPV; ++qq) acc[h][qq] = fmaf(p, xu[qq], acc[h][qq]);
           }
         }
       }
@@ -295,7 +300,7 @@ __global__ void __launch_bounds__(256) gat_bwd_kernel(GatKArgs a) {
 #pragma unroll
       for (int q = 0; q < EPV; ++q) {
         const int c = l * EPV + q;
-        gm[h][q] = (valid && a.mode != 2 && l < V && c < a.cols) ? a.gam[(i * H + h) * a.cols + c] : 0.f;
+        gm[h][q] = (valid && a.mode != 2 && l < V && c < a.cols) ? a.gam[(i * H + h) * a.gp + c] : 0.f;
         dws[h][q] = 0.f;
       }
       t[h] = valid ? a.tb[i * H + h] : 0.f;
@@ -350,7 +355,7 @@ __global__ void __launch_bounds__(256) gat_bwd_kernel(GatKArgs a) {
 #pragma unroll
           for (int h = 0; h < H; ++h) {
             const float ev = a.esc[(i * k + e) * H + h];
-            const float al = expf(ev - Lv[h]);
+            const float al = __expf(ev - Lv[h]);
             const float ds = al * (da[h] - t[h]) * (ev > 0.f ? 1.f : kSlope);
             der[h] += ds;
 #pragma unroll
@@ -439,44 +444,66 @@ __global__ void gat_t_kernel(const T* __restrict__ g, int64_t gp, const float* _
                              float* __restrict__ t) {
   APT_PDL_PROLOGUE();
   const int64_t n = *n_p;
-  for (int64_t x = int64_t(blockIdx.x) * blockDim.x + threadIdx.x; x < n * H; x += int64_t(gridDim.x) * blockDim.x) {
-    const int64_t r = x / H;
-    const int h = int(x - r * H);
-    float s = 0.f;
-    for (int f = 0; f < F; ++f) {
-      const int c = h * F + f;
-      float gv;
-      if constexpr (sizeof(T) == 2) gv = __uint_as_float(uint32_t(g[r * gp + c]) << 16);
-      else gv = float(g[r * gp + c]);
-      s = fmaf(gv, h1[r * hp + c] - b[c], s);
+  const int lane = lane_id();
+  const int64_t nw = int64_t(gridDim.x) * (blockDim.x >> 5);
+  for (int64_t r = (int64_t(blockIdx.x) * blockDim.x + threadIdx.x) >> 5; r < n; r += nw) {   // warp per row
+    for (int h = 0; h < H; ++h) {
+      float s = 0.f;
+      for (int f = lane; f < F; f += 32) {
+        const int c = h * F + f;
+        float gv;
+        if constexpr (sizeof(T) == 2) gv = __uint_as_float(uint32_t(g[r * gp + c]) << 16);
+        else gv = float(g[r * gp + c]);
+        s = fmaf(gv, h1[r * hp + c] - b[c], s);
+      }
+      s = warp_sum(s);
+      if (lane == 0) t[r * H + h] = s;
     }
-    t[x] = s;
   }
 }
 
 // Owner: g rows (fp32), t and the global log-sum-exp of its items from the
 // requesters; SNP scales g by the merge weight omega_c = S_c e^{m_c - L}.
+// bf16 mode (T = uint16_t) writes the bf16 operands of the tcgen05 contractions and zeroes
+// their rows [n, round_up(n, 64)) (the weight-gradient kernel's row-block tail).
 template <typename T>
 __global__ void gat_gather_kernel(T* const* __restrict__ gtab, int64_t gp, float* const* __restrict__ ttab,
                                   float* const* __restrict__ Ltab, GatItems it, int H, int F,
                                   const float* __restrict__ Lm, const float* __restrict__ Ss, int snp,
-                                  float* __restrict__ wG, float* __restrict__ wGs, int64_t wp, float* __restrict__ tb,
-                                  float* __restrict__ Lb) {
+                                  float* __restrict__ wG, float* __restrict__ wGs, int64_t wp,
+                                  uint16_t* __restrict__ wGb, uint16_t* __restrict__ wGsb, int64_t wpb, int64_t icap,
+                                  float* __restrict__ tb, float* __restrict__ Lb) {
   APT_PDL_PROLOGUE();
   const int64_t n = *it.n;
+  const int64_t rows = sizeof(T) == 2 ? std::min<int64_t>(icap, round_up(n, 64)) : n;
   const int d_out = H * F;
-  for (int64_t x = int64_t(blockIdx.x) * blockDim.x + threadIdx.x; x < n * d_out; x += int64_t(gridDim.x) * blockDim.x) {
+  for (int64_t x = int64_t(blockIdx.x) * blockDim.x + threadIdx.x; x < rows * d_out; x += int64_t(gridDim.x) * blockDim.x) {
     const int64_t i = x / d_out;
     const int c = int(x - i * d_out);
+    if (i >= n) {
+      wGb[i * wpb + c] = 0;
+      if (snp) wGsb[i * wpb + c] = 0;
+      continue;
+    }
     const int h = c / F;
     const int rk = it.rank ? it.rank[i] : it.self;
     const int row = it.row ? it.row[i] : int(i);
+    const T graw = gtab[rk][int64_t(row) * gp + c];
     float gv;
-    if constexpr (sizeof(T) == 2) gv = __uint_as_float(uint32_t(gtab[rk][int64_t(row) * gp + c]) << 16);
-    else gv = float(gtab[rk][int64_t(row) * gp + c]);
-    wG[i * wp + c] = gv;
+    if constexpr (sizeof(T) == 2) gv = __uint_as_float(uint32_t(graw) << 16);
+    else gv = float(graw);
     const float L = snp ? Ltab[rk][int64_t(row) * H + h] : Lm[i * H + h];
-    if (snp) wGs[i * wp + c] = gv * (Ss[i * H + h] > 0.f ? Ss[i * H + h] * expf(Lm[i * H + h] - L) : 0.f);
+    const float om = snp ? (Ss[i * H + h] > 0.f ? Ss[i * H + h] * expf(Lm[i * H + h] - L) : 0.f) : 1.f;
+    if constexpr (sizeof(T) == 2) {
+      wGb[i * wpb + c] = graw;
+      if (snp) {
+        __nv_bfloat16 q = __float2bfloat16_rn(gv * om);
+        wGsb[i * wpb + c] = *reinterpret_cast<uint16_t*>(&q);
+      }
+    } else {
+      wG[i * wp + c] = gv;
+      if (snp) wGs[i * wp + c] = gv * om;
+    }
     if (c % F == 0) {
       tb[i * H + h] = ttab[rk][int64_t(row) * H + h];
       Lb[i * H + h] = L;
@@ -578,6 +605,7 @@ static GatKArgs kargs(apt_trainer* t, RankState& rs) {
   a.d_out = rs.L[0].d_out;
   a.C = t->world;
   a.gam = ga.Gam;
+  a.gp = ga.gp;
   a.tb = ga.tb;
   a.Lb = ga.Lb;
   a.dwt = ga.dwt;
@@ -650,9 +678,18 @@ apt_status gat_alloc(apt_trainer* t, RankState& rs) {
   ga.Ss = A.alloc<float>(ic * H, true);
   ga.Lb = A.alloc<float>(ic * H, true);
   ga.tb = A.alloc<float>(ic * H, true);
-  ga.wG = A.alloc<float>(ic * wp, true);
-  ga.wGs = (t->s == APT_SNP && !gdp) ? A.alloc<float>(ic * wp, true) : ga.wG;
-  ga.Gam = A.alloc<float>(ic * H * std::max(ga.cols, 1), true);
+  const bool snp = t->s == APT_SNP && !gdp;
+  if (esz == 2) {
+    ga.wpb = round_up(L.d_out, 8);
+    ga.wGb = A.alloc<uint16_t>(ic * ga.wpb, true);
+    ga.wGsb = snp ? A.alloc<uint16_t>(ic * ga.wpb, true) : ga.wGb;
+    ga.wG = ga.wGs = reinterpret_cast<float*>(ga.wGb);   // (unused in bf16 mode; non-null marker)
+  } else {
+    ga.wG = A.alloc<float>(ic * wp, true);
+    ga.wGs = snp ? A.alloc<float>(ic * wp, true) : ga.wG;
+  }
+  ga.gp = round_up(std::max(ga.cols, 1), 4);
+  ga.Gam = A.alloc<float>(ic * H * ga.gp, true);
   ga.t = A.alloc<float>(L.max_rows * H, true);
   if (!gdp && t->s == APT_SNP) {
     ga.slot_pitch = round_up(L.d_out + 2 * H, 4);
@@ -777,7 +814,31 @@ apt_status gat_layer1_fwd(apt_trainer* t, bool time_it) {
     Layer& L = rs.L[0];
     const WView wv = wview(t, rs);
     const GatItems it = items_of(t, rs);
-    for (int h = 0; h < H; ++h) {
+    const bool tc = bf && ga.F % 4 == 0 && ga.cols > 0 && tc_gemm_supported(ga.F, ga.cols);
+    for (int h = 0; h < H && tc; ++h) {   // tcgen05: A = Z^h (K-major, pitch H*zp), B = W^h
+      TcGemmArgs g{};
+      g.Z = static_cast<const uint16_t*>(ga.Z) + size_t(h) * ga.zp;
+      g.z_pitch = int64_t(H) * ga.zp;
+      g.W = static_cast<const uint16_t*>(wv.Wp) + size_t(h) * ga.F * wv.ldp;
+      g.w_pitch = wv.ldp;
+      g.M_max = ga.icap; g.M_dev = it.n; g.N = ga.F; g.K = ga.cols;
+      if (gdp) {
+        g.Y = L.H + h * ga.F; g.y_pitch = L.h_pitch;
+        g.bias = L.b + h * ga.F; g.relu = t->K > 1 ? 1 : 0;
+      } else {
+        g.out_base = ga.otab + size_t(h) * t->world; g.out_rank = it.rank; g.out_row = it.row;
+        if (t->s == APT_SNP) {
+          g.y_pitch = int64_t(t->world) * ga.slot_pitch;
+        } else {
+          g.y_pitch = L.h_pitch;
+          if (t->s == APT_DNP) { g.bias = L.b + h * ga.F; g.relu = t->K > 1 ? 1 : 0; }
+          else g.accumulate = 1;
+        }
+      }
+      CK(c, launch_tc_gemm(g, c->stream));
+      c->launches++;
+    }
+    for (int h = 0; h < H && !tc; ++h) {
       SimtGemmArgs g{};
       g.A = static_cast<const uint8_t*>(ga.Z) + size_t(h) * ga.zp * (bf ? 2 : 4);
       g.a_t = bf ? kBF16 : kF32;
@@ -844,10 +905,10 @@ apt_status gat_layer1_bwd(apt_trainer* t) {
   for (auto& rs : t->R) {    // requesters: t = g . (pre - b), db = sum g
     Layer& L = rs.L[0];
     GatState& ga = rs.ga;
-    if (bf) launch_pdl(gat_t_kernel<uint16_t>, dim3(gridn(L.max_rows * H)), dim3(256), 0, c->stream,
+    if (bf) launch_pdl(gat_t_kernel<uint16_t>, dim3(gridn(L.max_rows * 32)), dim3(256), 0, c->stream,
                        static_cast<const uint16_t*>(L.Gb), L.gb_pitch, static_cast<const float*>(L.H), L.h_pitch,
                        static_cast<const float*>(L.b), H, ga.F, L.n_rows, ga.t);
-    else launch_pdl(gat_t_kernel<float>, dim3(gridn(L.max_rows * H)), dim3(256), 0, c->stream,
+    else launch_pdl(gat_t_kernel<float>, dim3(gridn(L.max_rows * 32)), dim3(256), 0, c->stream,
                     static_cast<const float*>(L.G), L.h_pitch, static_cast<const float*>(L.H), L.h_pitch,
                     static_cast<const float*>(L.b), H, ga.F, L.n_rows, ga.t);
     CK(c, cudaGetLastError());
@@ -870,20 +931,36 @@ apt_status gat_layer1_bwd(apt_trainer* t) {
     const int snp = (!gdp && t->s == APT_SNP) ? 1 : 0;
     if (bf) launch_pdl(gat_gather_kernel<uint16_t>, dim3(gridn(ga.icap * L.d_out)), dim3(256), 0, c->stream,
                        t->gGb_tab, L.gb_pitch, t->gt_tab, t->gL_tab, it, H, ga.F,
-                       static_cast<const float*>(ga.Lm), static_cast<const float*>(ga.Ss), snp, ga.wG, ga.wGs, wp, ga.tb, ga.Lb);
+                       static_cast<const float*>(ga.Lm), static_cast<const float*>(ga.Ss), snp,
+                       static_cast<float*>(nullptr), static_cast<float*>(nullptr), wp, ga.wGb, ga.wGsb, ga.wpb, ga.icap,
+                       ga.tb, ga.Lb);
     else launch_pdl(gat_gather_kernel<float>, dim3(gridn(ga.icap * L.d_out)), dim3(256), 0, c->stream,
                     t->gG_tab, L.h_pitch, t->gt_tab, t->gL_tab, it, H, ga.F,
-                    static_cast<const float*>(ga.Lm), static_cast<const float*>(ga.Ss), snp, ga.wG, ga.wGs, wp, ga.tb, ga.Lb);
+                    static_cast<const float*>(ga.Lm), static_cast<const float*>(ga.Ss), snp, ga.wG, ga.wGs, wp,
+                    static_cast<uint16_t*>(nullptr), static_cast<uint16_t*>(nullptr), int64_t(0), ga.icap, ga.tb, ga.Lb);
     CK(c, cudaGetLastError());
     c->launches++;
+    // gamma^h = W^hT g^h: tcgen05 with W read N-major as stored (bf16 mode), else fp32 CUDA cores
+    const bool tcg = bf && ga.F % 16 == 0 && ga.cols > 0 && tc_gemm_supported(ga.cols, ga.F);
     for (int h = 0; h < H; ++h) {
-      SimtGemmArgs g{};
-      g.A = ga.wG + h * ga.F; g.a_t = kF32; g.sam = wp; g.sak = 1;
-      g.B = static_cast<const uint8_t*>(wv.Wp) + size_t(h) * ga.F * wv.ldp * (bf ? 2 : 4);
-      g.b_t = wv.wt; g.sbk = wv.ldp; g.sbn = 1;
-      g.C = ga.Gam + int64_t(h) * ga.cols; g.ldc = int64_t(H) * ga.cols;
-      g.M_dev = it.n; g.M = ga.icap; g.N = ga.cols; g.K = ga.F;
-      if (ga.cols > 0) CK(c, launch_simt_gemm(g, c->stream));
+      if (tcg) {
+        TcGemmArgs g{};
+        g.Z = ga.wGb + h * ga.F; g.z_pitch = ga.wpb;
+        g.W = static_cast<const uint16_t*>(wv.Wp) + size_t(h) * ga.F * wv.ldp; g.w_pitch = wv.ldp; g.w_mn = 1;
+        g.M_max = ga.icap; g.M_dev = it.n; g.N = ga.cols; g.K = ga.F;
+        g.Y = ga.Gam + int64_t(h) * ga.gp; g.y_pitch = int64_t(H) * ga.gp;
+        CK(c, launch_tc_gemm(g, c->stream));
+      } else {
+        SimtGemmArgs g{};
+        if (bf) { g.A = ga.wGb + h * ga.F; g.a_t = kBF16; g.sam = ga.wpb; }
+        else { g.A = ga.wG + h * ga.F; g.a_t = kF32; g.sam = wp; }
+        g.sak = 1;
+        g.B = static_cast<const uint8_t*>(wv.Wp) + size_t(h) * ga.F * wv.ldp * (bf ? 2 : 4);
+        g.b_t = wv.wt; g.sbk = wv.ldp; g.sbn = 1;
+        g.C = ga.Gam + int64_t(h) * ga.gp; g.ldc = int64_t(H) * ga.gp;
+        g.M_dev = it.n; g.M = ga.icap; g.N = ga.cols; g.K = ga.F;
+        if (ga.cols > 0) CK(c, launch_simt_gemm(g, c->stream));
+      }
       c->launches++;
     }
     if (!gdp && t->s == APT_NFP) {
@@ -905,15 +982,26 @@ apt_status gat_layer1_bwd(apt_trainer* t) {
     a.tab = t->dsum_tab;
     apt_status s = launch_gat(t, a, true, ga.icap);
     if (s != APT_OK) return s;
+    // dW^h += (omega g^h)^T Z^h: tcgen05 weight-gradient kernel (bf16), else fp32 split-K
+    const bool tcw = bf && ga.F % 8 == 0 && ga.cols > 0 && tc_wgrad_supported(ga.F, ga.cols);
     for (int h = 0; h < H; ++h) {
-      SimtGemmArgs g{};
-      g.A = ga.wGs + h * ga.F; g.a_t = kF32; g.sam = 1; g.sak = wp;
-      g.B = static_cast<const uint8_t*>(ga.Z) + size_t(h) * ga.zp * (bf ? 2 : 4);
-      g.b_t = bf ? kBF16 : kF32; g.sbk = int64_t(H) * ga.zp; g.sbn = 1;
-      g.C = wv.dW + int64_t(h) * ga.F * wv.lddw; g.ldc = wv.lddw;
-      g.M = ga.F; g.N = ga.cols; g.K = ga.icap; g.K_dev = it.n;
-      g.accumulate = 1; g.k_chunk = 2048;
-      if (ga.cols > 0) CK(c, launch_simt_gemm(g, c->stream));
+      if (tcw) {
+        TcWgradArgs w{ga.wGsb + h * ga.F, ga.wpb, static_cast<const uint16_t*>(ga.Z) + size_t(h) * ga.zp,
+                      int64_t(H) * ga.zp, it.n, ga.icap, ga.F, ga.cols, wv.dW + int64_t(h) * ga.F * wv.lddw, nullptr,
+                      wv.lddw};
+        CK(c, launch_tc_wgrad(w, c->stream));
+      } else {
+        SimtGemmArgs g{};
+        if (bf) { g.A = ga.wGsb + h * ga.F; g.a_t = kBF16; g.sak = ga.wpb; }
+        else { g.A = ga.wGs + h * ga.F; g.a_t = kF32; g.sak = wp; }
+        g.sam = 1;
+        g.B = static_cast<const uint8_t*>(ga.Z) + size_t(h) * ga.zp * (bf ? 2 : 4);
+        g.b_t = bf ? kBF16 : kF32; g.sbk = int64_t(H) * ga.zp; g.sbn = 1;
+        g.C = wv.dW + int64_t(h) * ga.F * wv.lddw; g.ldc = wv.lddw;
+        g.M = ga.F; g.N = ga.cols; g.K = ga.icap; g.K_dev = it.n;
+        g.accumulate = 1; g.k_chunk = 256;    // short k-chunks: the loop is latency bound
+        if (ga.cols > 0) CK(c, launch_simt_gemm(g, c->stream));
+      }
       c->launches++;
     }
     if (ga.cols > 0) {

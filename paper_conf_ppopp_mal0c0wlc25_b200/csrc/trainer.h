@@ -97,7 +97,11 @@ struct GatState {
   float* tb = nullptr;               // [icap][H] backward: t = g . (pre - b) of the item
   float* wG = nullptr;               // [icap][d_out] gathered g (fp32)
   float* wGs = nullptr;              // [icap][d_out] g scaled by the SNP merge weight (else == wG)
-  float* Gam = nullptr;              // [icap][H][cols] gamma^h = W^hT g^h
+  uint16_t* wGb = nullptr;           // bf16 mode: [icap][wpb] gathered g (tcgen05 operands; tail rows zero)
+  uint16_t* wGsb = nullptr;          // bf16 mode: ... scaled by the SNP merge weight (else == wGb)
+  int64_t wpb = 0;
+  float* Gam = nullptr;              // [icap][H][gp] gamma^h = W^hT g^h
+  int64_t gp = 0;                    // per-head pitch of Gam (floats, multiple of 4)
   float** otab = nullptr;            // [H][C] routed projection targets per head
   // requester side
   float* t = nullptr;                // [max_rows][H]
