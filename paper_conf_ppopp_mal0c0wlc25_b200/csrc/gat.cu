@@ -122,7 +122,7 @@ __device__ __forceinline__ float gsum(float v) {
 // Fused gather + attention + per-head weighted sums over the owner's items.  A lane
 // group of LG lanes owns an item; lane l holds the l-th 16-byte vector of each row.
 template <int EPV, int LG, int H>
-__global__ void __launch_bounds__(256) gat_fwd_kernel(GatKArgs a) {
+__global__ void __launch_bounds__(256, 2) gat_fwd_kernel(GatKArgs a) {
   APT_PDL_PROLOGUE();
   extern __shared__ float swt[];                     // [2][H][cpad], zero past cols
   for (int t = threadIdx.x; t < 2 * H * a.cpad; t += blockDim.x) {
@@ -188,24 +188,47 @@ __global__ void __launch_bounds__(256) gat_fwd_kernel(GatKArgs a) {
           kp[q] = __shfl_sync(0xffffffffu, int(keep), src_lane) && (j + q < mloc);
           raw[q] = ld_nc_v4(r + lv * 16);
         }
+        // phase 1: the NB edges' scores (independent reductions: the shuffles overlap)
+        float sc[NB][H];
+#pragma unroll
+        for (int q = 0; q < NB; ++q) {
+          const int e = e0 + j + q;
+          if (a.mode == 2) {
+#pragma unroll
+            for (int h = 0; h < H; ++h) sc[q][h] = kp[q] ? a.tab[rk][(int64_t(row) * k + e) * H + h] : 0.f;
+          } else {
+            float xu[EPV];
+            unpack<EPV>(raw[q], xu);
+#pragma unroll
+            for (int h = 0; h < H; ++h) {
+              float p = 0.f;
+#pragma unroll
+              for (int qq = 0; qq < EPV; ++qq) p = fmaf(xu[qq], ws[h * a.cpad + qq], p);
+              sc[q][h] = l < V ? p : 0.f;
+            }
+          }
+        }
+        if (a.mode != 2) {
+#pragma unroll
+          for (int o = LG / 2; o > 0; o >>= 1)
+#pragma unroll
+            for (int q = 0; q < NB; ++q)
+#pragma unroll
+              for (int h = 0; h < H; ++h) sc[q][h] += __shfl_xor_sync(0xffffffffu, sc[q][h], o);
+#pragma unroll
+          for (int q = 0; q < NB; ++q)
+#pragma unroll
+            for (int h = 0; h < H; ++h) sc[q][h] += er[h];
+        }
+        // phase 2: the online-softmax updates, in edge order
 #pragma unroll
         for (int q = 0; q < NB; ++q) {
           const int e = e0 + j + q;
           float xu[EPV];
           unpack<EPV>(raw[q], xu);
           float s[H];
-          if (a.mode == 2) {
 #pragma unroll
-            for (int h = 0; h < H; ++h) s[h] = kp[q] ? a.tab[rk][(int64_t(row) * k + e) * H + h] : 0.f;
-          } else {
-#pragma unroll
-            for (int h = 0; h < H; ++h) {
-              float p = 0.f;
-#pragma unroll
-              for (int qq = 0; qq < EPV; ++qq) p = fmaf(xu[qq], ws[h * a.cpad + qq], p);
-              s[h] = gsum<LG>(l < V ? p : 0.f) + er[h];
-            }
-          }
+          for (int h = 0; h < H; ++h) s[h] = sc[q][h];
           if (a.mode == 1) {
             if (kp[q] && l < H) {
               float sv = s[0];
@@ -271,7 +294,7 @@ __global__ void __launch_bounds__(256) gat_fwd_kernel(GatKArgs a) {
 // Backward over the owner's items: dalpha, softmax and LeakyReLU backward, and the
 // gradients of the two score vectors w~ (accumulated in shared memory per block).
 template <int EPV, int LG, int H>
-__global__ void __launch_bounds__(256) gat_bwd_kernel(GatKArgs a) {
+__global__ void __launch_bounds__(256, 2) gat_bwd_kernel(GatKArgs a) {
   APT_PDL_PROLOGUE();
   extern __shared__ float sdw[];                     // [2][H][cpad]
   for (int t = threadIdx.x; t < 2 * H * a.cpad; t += blockDim.x) sdw[t] = 0.f;
@@ -313,7 +336,7 @@ __global__ void __launch_bounds__(256) gat_bwd_kernel(GatKArgs a) {
       const bool keep = u >= 0 && (a.snp_rank < 0 || a.part[u] == a.snp_rank);
       const char* rp = keep ? gat_row(a, u) : reinterpret_cast<const char*>(g_gat_zero_row);
       const int mloc = min(LG, cmax - e0);
-      constexpr int NB = 4;
+      constexpr int NB = 2;             // (4: register spills at 2 blocks/SM)
       for (int j = 0; j < mloc; j += NB) {
         uint4 raw[NB];
         int kp[NB];
@@ -324,24 +347,41 @@ __global__ void __launch_bounds__(256) gat_bwd_kernel(GatKArgs a) {
           kp[q] = __shfl_sync(0xffffffffu, int(keep), src_lane) && (j + q < mloc);
           raw[q] = ld_nc_v4(r + lv * 16);
         }
+        float dq[NB][H];     // phase 1: the NB edges' dalpha (independent reductions)
+#pragma unroll
+        for (int q = 0; q < NB; ++q) {
+          const int e = e0 + j + q;
+          if (a.mode == 2) {
+#pragma unroll
+            for (int h = 0; h < H; ++h) dq[q][h] = kp[q] ? a.tab[rk][(int64_t(row) * k + e) * H + h] : 0.f;
+          } else {
+            float xu[EPV];
+            unpack<EPV>(raw[q], xu);
+#pragma unroll
+            for (int h = 0; h < H; ++h) {
+              float p = 0.f;
+#pragma unroll
+              for (int qq = 0; qq < EPV; ++qq) p = fmaf(xu[qq], gm[h][qq], p);
+              dq[q][h] = p;
+            }
+          }
+        }
+        if (a.mode != 2) {
+#pragma unroll
+          for (int o = LG / 2; o > 0; o >>= 1)
+#pragma unroll
+            for (int q = 0; q < NB; ++q)
+#pragma unroll
+              for (int h = 0; h < H; ++h) dq[q][h] += __shfl_xor_sync(0xffffffffu, dq[q][h], o);
+        }
 #pragma unroll
         for (int q = 0; q < NB; ++q) {
           const int e = e0 + j + q;
           float xu[EPV];
           unpack<EPV>(raw[q], xu);
           float da[H];
-          if (a.mode == 2) {
 #pragma unroll
-            for (int h = 0; h < H; ++h) da[h] = kp[q] ? a.tab[rk][(int64_t(row) * k + e) * H + h] : 0.f;
-          } else {
-#pragma unroll
-            for (int h = 0; h < H; ++h) {
-              float p = 0.f;
-#pragma unroll
-              for (int qq = 0; qq < EPV; ++qq) p = fmaf(xu[qq], gm[h][qq], p);
-              da[h] = gsum<LG>(p);
-            }
-          }
+          for (int h = 0; h < H; ++h) da[h] = dq[q][h];
           if (a.mode == 1) {
             if (kp[q] && l < H) {
               float dv = da[0];
