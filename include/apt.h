@@ -112,6 +112,16 @@ typedef struct {
   double t_train_s;                          /* measured common T_train (GDP)      */
   int64_t rows_host[4][APT_MAX_RANKS];       /* unique rows read from the host tier */
   int64_t feat_bytes_host[4][APT_MAX_RANKS];
+  /* GAT layer 1 (gat_heads > 0): the extra exchange attention costs NFP and SNP
+   * (Fig. 10 / P:344).  NFP: the partial score and dalpha sums,
+   * reduced into and read back from every other requester (4 passes x H x 4 B per
+   * edge); SNP: the softmax state (m, S) with every partial and (t, L) with every
+   * gradient (2H x 4 B each way per virtual node) and, per item an owner
+   * computes, the destination's own feature row (attn_feat_bytes, NVLink).
+   * GDP and DNP: 0 ("each destination node has a complete view").      */
+  int gat_heads;
+  int64_t attn_bytes[4][APT_MAX_RANKS];
+  int64_t attn_feat_bytes[4][APT_MAX_RANKS];
 } apt_plan_stats;
 
 /* Operator slots of the bandwidth profile ("trials").          */

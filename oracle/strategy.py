@@ -97,10 +97,16 @@ def tiered_store(part, C, hbm_frac, hot_ids=None, cache_rows=0):
     return tier
 
 
-def emulate_layer1(strategy, l1_blocks, part, C, d, d_out, feat_bytes=4, hidden_bytes=4, tier=None):
+def emulate_layer1(strategy, l1_blocks, part, C, d, d_out, feat_bytes=4, hidden_bytes=4, tier=None, heads=0):
     """l1_blocks[r] = rank r's layer-1 Block (dst, src, indptr, indices).  tier(r, ids):
     where rank r reads each row (0 local HBM, 1 NVLink peer, 2 host; default: own
-    partition local, others peer).  Returns per-rank dict of counts and structures."""
+    partition local, others peer).  heads > 0: a GAT first layer, whose attention
+    adds exchanges for NFP and SNP (reading G6): NFP reduces and
+    reads back the partial score and dalpha of every edge of every other block
+    (attn_bytes = 4 passes x H x 4 B per edge); SNP ships (m, S) with each virtual
+    node's partial and (t, L) with its gradient (2H x 4 B each way), and every owner
+    reads the destination's own feature row of each item it computes
+    (attn_feat_bytes).  Returns per-rank dict of counts and structures."""
     if tier is None:
         def tier(r, ids):
             return np.where(np.asarray(part)[np.asarray(ids, np.int64)] == r, 0, 1)
@@ -109,7 +115,7 @@ def emulate_layer1(strategy, l1_blocks, part, C, d, d_out, feat_bytes=4, hidden_
     for r in range(C):
         out.append(dict(n_d=N_d[r], n_vs=0, n_vd=0, rows_local=0, rows_peer=0, rows_host=0,
                         feat_bytes_local=0, feat_bytes_peer=0, feat_bytes_host=0, graph_bytes=0,
-                        hidden_bytes_fwd=0, hidden_bytes_bwd=0, n_calls=0,
+                        hidden_bytes_fwd=0, hidden_bytes_bwd=0, n_calls=0, attn_bytes=0, attn_feat_bytes=0,
                         virtual=[], requests=[]))
 
     def count(o, uu, rec):
@@ -133,6 +139,8 @@ def emulate_layer1(strategy, l1_blocks, part, C, d, d_out, feat_bytes=4, hidden_
                 if b != c:
                     out[c]["graph_bytes"] += msg_bytes_graph(blk.n_dst, blk.n_edges)
                     out[c]["hidden_bytes_bwd"] += blk.n_dst * d_out * hidden_bytes
+                    if heads and C > 1:
+                        out[c]["attn_bytes"] += 4 * heads * 4 * blk.n_edges
             out[c]["rows_local"] = rows
             out[c]["feat_bytes_local"] = rows * (hi - lo) * feat_bytes
             out[c]["hidden_bytes_fwd"] = (C - 1) * N_d[c] * d_out * hidden_bytes
@@ -150,7 +158,12 @@ def emulate_layer1(strategy, l1_blocks, part, C, d, d_out, feat_bytes=4, hidden_
                     continue
                 vs = np.unique(rows[m])
                 recv_rows[c].update(u[m].tolist())
+                if heads and C > 1:
+                    out[c]["attn_feat_bytes"] += len(vs) * d * feat_bytes
                 if c != r:
+                    if heads:
+                        out[r]["attn_bytes"] += len(vs) * 2 * heads * 4
+                        out[c]["attn_bytes"] += len(vs) * 2 * heads * 4
                     out[r]["n_vs"] += len(vs)
                     out[r]["virtual"].append((c, blk.dst[vs]))
                     out[c]["graph_bytes"] += msg_bytes_graph(len(vs), int(m.sum()))
@@ -220,9 +233,14 @@ def predict(per_strategy_stats, alpha, beta, t_build):
                 t += st["graph_bytes"] / beta[OP_ALLGATHER]
                 t += st["hidden_bytes_fwd"] / beta[OP_REDUCE_SCATTER]
                 t += st["hidden_bytes_bwd"] / beta[OP_ALLGATHER]
+                if st.get("attn_bytes", 0) > 0:    # GAT: partial scores / dalpha all-reduced
+                    t += 2 * steps * alpha[OP_ALLREDUCE] + st["attn_bytes"] / beta[OP_ALLREDUCE]
             elif s in ("SNP", "DNP") and st["n_calls"]:
                 t += 3 * steps * alpha[OP_ALLTOALLV]
-                t += (st["graph_bytes"] + st["hidden_bytes_fwd"] + st["hidden_bytes_bwd"]) / beta[OP_ALLTOALLV]
+                t += (st["graph_bytes"] + st["hidden_bytes_fwd"] + st["hidden_bytes_bwd"]
+                      + st.get("attn_bytes", 0)) / beta[OP_ALLTOALLV]
+            if st.get("attn_feat_bytes"):   # SNP-GAT: destinations' own rows
+                t += st["attn_feat_bytes"] / beta[OP_PEER_PULL]
             worst = max(worst, t)
         pred.append(worst)
     pick = int(np.argmin(pred))

@@ -49,7 +49,8 @@ class PlanStats(C.Structure):
                 ("n_vd", C.c_int64 * MAX_RANKS), ("rows_local", _A4), ("rows_peer", _A4),
                 ("feat_bytes_local", _A4), ("feat_bytes_peer", _A4), ("graph_bytes", _A4),
                 ("hidden_bytes_fwd", _A4), ("hidden_bytes_bwd", _A4), ("n_calls", _A4),
-                ("t_build_s", _D4), ("t_train_s", C.c_double), ("rows_host", _A4), ("feat_bytes_host", _A4)]
+                ("t_build_s", _D4), ("t_train_s", C.c_double), ("rows_host", _A4), ("feat_bytes_host", _A4),
+                ("gat_heads", C.c_int), ("attn_bytes", _A4), ("attn_feat_bytes", _A4)]
 
 
 class FstoreOpts(C.Structure):

@@ -333,6 +333,23 @@ extern "C" apt_status apt_dryrun(apt_trainer* t, int64_t n_steps, apt_plan_stats
       out->feat_bytes_peer[S][r] = out->rows_peer[S][r] * d * bf;
       out->feat_bytes_host[S][r] = out->rows_host[S][r] * d * bf;
     }
+  // GAT layer 1: attention's extra exchanges (apt.h; oracle/strategy.py emulate_layer1)
+  const int64_t H = t->gat_heads;
+  out->gat_heads = int(H);
+  if (H > 0 && C > 1) {
+    const DryCounters& qn = h[APT_NFP];
+    for (int cc = 0; cc < C; ++cc)
+      for (int b = 0; b < C; ++b)
+        if (b != cc) out->attn_bytes[APT_NFP][cc] += 4 * H * 4 * int64_t(qn.edges[b]);
+    const DryCounters& qs = h[APT_SNP];
+    for (int r = 0; r < C; ++r)
+      for (int cc = 0; cc < C; ++cc) {
+        out->attn_feat_bytes[APT_SNP][cc] += int64_t(qs.tot_rows[r][cc]) * d * bf;
+        if (r == cc) continue;
+        out->attn_bytes[APT_SNP][r] += int64_t(qs.tot_rows[r][cc]) * 2 * H * 4;
+        out->attn_bytes[APT_SNP][cc] += int64_t(qs.tot_rows[r][cc]) * 2 * H * 4;
+      }
+  }
   return APT_OK;
 }
 

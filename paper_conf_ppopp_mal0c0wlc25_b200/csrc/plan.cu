@@ -46,12 +46,16 @@ extern "C" apt_status apt_select_strategy(const apt_plan_stats* st, const apt_bw
           t += double(st->graph_bytes[s][r]) / b[APT_OP_ALLGATHER];
           t += double(st->hidden_bytes_fwd[s][r]) / b[APT_OP_REDUCE_SCATTER];
           t += double(st->hidden_bytes_bwd[s][r]) / b[APT_OP_ALLGATHER];
+          if (st->attn_bytes[s][r] > 0)   // GAT: partial scores and dalpha, two all-reduces per step
+            t += 2.0 * steps * a[APT_OP_ALLREDUCE] + double(st->attn_bytes[s][r]) / b[APT_OP_ALLREDUCE];
         } else if (s == APT_SNP || s == APT_DNP) {
           t += 3.0 * steps * a[APT_OP_ALLTOALLV];
-          t += double(st->graph_bytes[s][r] + st->hidden_bytes_fwd[s][r] + st->hidden_bytes_bwd[s][r]) /
-               b[APT_OP_ALLTOALLV];
+          t += double(st->graph_bytes[s][r] + st->hidden_bytes_fwd[s][r] + st->hidden_bytes_bwd[s][r] +
+                      st->attn_bytes[s][r]) / b[APT_OP_ALLTOALLV];
         }
       }
+      if (st->attn_feat_bytes[s][r] > 0)   // SNP-GAT: destinations' own rows for the scores
+        t += double(st->attn_feat_bytes[s][r]) / b[APT_OP_PEER_PULL];
       worst = std::fmax(worst, t);
     }
     pred_s[s] = worst;

@@ -432,8 +432,9 @@ FIELDS = ("n_d", "rows_local", "rows_peer", "rows_host", "feat_bytes_local", "fe
           "graph_bytes", "hidden_bytes_fwd", "hidden_bytes_bwd", "n_calls")
 
 
-@pytest.mark.parametrize("C,frac,n_hot", [(2, 1.0, 0), (4, 1.0, 0), (4, 0.4, 300)])
-def test_dryrun_counts_match_oracle_and_pick(A, tiny, C, frac, n_hot):
+@pytest.mark.parametrize("C,frac,n_hot,heads", [(2, 1.0, 0, 0), (4, 1.0, 0, 0), (4, 0.4, 300, 0), (2, 1.0, 0, 4),
+                                                (4, 1.0, 0, 4)])
+def test_dryrun_counts_match_oracle_and_pick(A, tiny, C, frac, n_hot, heads):
     """apt_dryrun's per-strategy, per-rank counts are integers: bit-exact against
     the oracle's emulation of every rank's blocks (O7); apt_select_strategy = oracle Eq. 2 (O8)."""
     from oracle import strategy as S
@@ -447,24 +448,26 @@ def test_dryrun_counts_match_oracle_and_pick(A, tiny, C, frac, n_hot):
     dims = [cfg.dim] + [d for _, d in cfg.dims()]
     labels = aptgen.labels(cfg, g.n)
     tr = A.Trainer(ctx, gr, fs, dims, cfg.fanouts, cfg.batch, A.F32, 0.1, cfg.sample_seed, cfg.feat_seed, A.GDP,
-                   labels)
+                   labels, gat_heads=heads)
     tr.set_epoch(train, 0)
     st = tr.dryrun(2)
+    assert st.gat_heads == heads
     steps = st.steps
     assert steps == min(2, tr.steps_per_epoch())
     perm = oracle.epoch_perm(train, cfg.sample_seed, 0)
     ref = []
     for si, s in enumerate(S.STRATEGIES):
-        tot = [dict.fromkeys(FIELDS + ("n_vs", "n_vd"), 0) for _ in range(C)]
+        tot = [dict.fromkeys(FIELDS + ("n_vs", "n_vd", "attn_bytes", "attn_feat_bytes"), 0) for _ in range(C)]
         for step in range(steps):
             gb = oracle.global_batch(perm, step, C, cfg.batch)
             seeds = S.assign_seeds(s, gb, part, C, cfg.batch)
             blocks = [oracle.sample_blocks(g, sd, cfg.fanouts, cfg.sample_seed, step)[-1] for sd in seeds]
-            for r, e in enumerate(S.emulate_layer1(s, blocks, part, C, cfg.dim, cfg.hidden, 4, 4, tier=tier)):
+            for r, e in enumerate(S.emulate_layer1(s, blocks, part, C, cfg.dim, cfg.hidden, 4, 4, tier=tier,
+                                                   heads=heads)):
                 for k in tot[r]:
                     tot[r][k] += e[k]
         for r in range(C):
-            for k in FIELDS:
+            for k in FIELDS + ("attn_bytes", "attn_feat_bytes"):
                 assert getattr(st, k)[si][r] == tot[r][k], (s, r, k, getattr(st, k)[si][r], tot[r][k])
             if s == "SNP":
                 assert st.n_vs[r] == tot[r]["n_vs"]

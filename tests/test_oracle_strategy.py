@@ -72,6 +72,24 @@ def test_fig3_gdp_reads_d_remotely(fig2):
     assert all(s["hidden_bytes_fwd"] == 0 for s in st)        # GDP T_shuffle = 0
 
 
+def test_fig3_gat_attention_costs(fig2):
+    # P:344 / P:173-178: attention costs GDP and DNP nothing extra; SNP ships the softmax
+    # state with K' (1 virtual node: (m, S) out, (t, L) back) and GPU 2 reads K's own row
+    # for the score; NFP sums partial scores of GPU 1's 4 edges (2 passes fwd, 2 bwd)
+    H = 4
+    for s in ("GDP", "DNP"):
+        assert all(r["attn_bytes"] == 0 and r["attn_feat_bytes"] == 0
+                   for r in S.emulate_layer1(s, fig2, PART, 2, d=4, d_out=8, heads=H))
+    snp = S.emulate_layer1("SNP", fig2, PART, 2, d=4, d_out=8, heads=H)
+    assert snp[0]["attn_bytes"] == snp[1]["attn_bytes"] == 1 * 2 * H * 4
+    # GPU 1 computes B (G, H) and K (A) locally, GPU 2 computes K' (D): one dst row each item
+    assert snp[0]["attn_feat_bytes"] == 2 * 4 * 4 and snp[1]["attn_feat_bytes"] == 1 * 4 * 4
+    nfp = S.emulate_layer1("NFP", fig2, PART, 2, d=4, d_out=8, heads=H)
+    assert nfp[1]["attn_bytes"] == 4 * H * 4 * 4 and nfp[0]["attn_bytes"] == 0
+    sage = S.emulate_layer1("SNP", fig2, PART, 2, d=4, d_out=8)
+    assert sage[0]["attn_bytes"] == 0 and sage[0]["hidden_bytes_fwd"] == snp[0]["hidden_bytes_fwd"]
+
+
 def _rank_blocks(graph, cfg, C, strategy, step=0):
     train = aptgen.train_nodes(graph, cfg)
     perm = oracle.epoch_perm(train, cfg.sample_seed, 0)
