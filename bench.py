@@ -65,6 +65,8 @@ def parse():
     ap.add_argument("--feat-dim", type=int, default=0, help="override the config's input dim d (sweeps)")
     ap.add_argument("--hidden", type=int, default=0, help="override the config's hidden dim d' (sweeps)")
     ap.add_argument("--fanouts", default="", help="override the fanouts, e.g. 15,10 (layer 1 first; NEXT #4 sweep)")
+    ap.add_argument("--partition", default="range", choices=["range", "random", "ldg"],
+                    help="edge-cut partition for SNP/DNP and the store's row sharding (apt_partition; NEXT #3)")
     return ap.parse_args()
 
 
@@ -73,6 +75,22 @@ def dist_env():
 
 
 GAT_HEADS = 0   # set from --gat-heads
+PARTITION = "range"   # set from --partition
+_PART_CACHE = {}
+
+
+def partition(A, g, C):
+    """The job's edge-cut partition into C parts (apt_partition, the library's host
+    partitioner; "range" is the generator's planted partition)."""
+    return _partition(A, g, C)[0]
+
+
+def _partition(A, g, C):
+    key = (id(g), C, PARTITION)
+    if key not in _PART_CACHE:
+        _PART_CACHE[key] = A.partition(g.indptr, g.indices, C, PARTITION, seed=7) if C > 1 else \
+            (np.zeros(g.n, np.int32), 0)
+    return _PART_CACHE[key]
 
 
 def workload_config(cfg):
@@ -235,7 +253,7 @@ def run_apt(args, cfg):
     g = aptgen.make_graph(cfg)
     train = aptgen.train_nodes(g, cfg)
     labels = aptgen.labels(cfg, g.n)
-    part = aptgen.partition(g.n, world)
+    part = partition(A, g, world)
     dt = A.DTYPE[args.dtype]
     ctx = A.Ctx(rank if world > 1 else 0, world, local, stream.cuda_stream)
     if world > 1:
@@ -368,7 +386,7 @@ def planner_report(A, g, cfg, train, labels, args, stream, gdp_ms):
                    "NVLink betas are the pool's measured references (no peer GPU in this run)"}
     for C in (2, 4, 8):
         ctx = A.Ctx(-1, C, 0, stream.cuda_stream)
-        gr = ctx.graph_load(g.indptr, g.indices, aptgen.partition(g.n, C))
+        gr = ctx.graph_load(g.indptr, g.indices, partition(A, g, C))
         fs = ctx.fstore_create(gr, A.GDP, dt, cfg.dim, None, cfg.feat_seed)
         tr = make_trainer(A, ctx, gr, fs, cfg, dt, A.GDP, labels)
         tr.set_epoch(train, 0)
@@ -377,6 +395,7 @@ def planner_report(A, g, cfg, train, labels, args, stream, gdp_ms):
         pick, pred = A.select_strategy(st, bw)
         steps = max(1, st.steps)
         rep[f"C{C}"] = {"dryrun_steps": st.steps, "pred_ms_per_step": {s: 1e3 * p / steps for s, p in zip(STRATS, pred)},
+                        "partition": PARTITION, "edge_cut_frac": _partition(A, g, C)[1] / max(1, g.nnz),
                         "pick": STRATS[pick],
                         "n_vs_per_step": sum(st.n_vs[r] for r in range(C)) / steps,
                         "n_vd_per_step": sum(st.n_vd[r] for r in range(C)) / steps}
@@ -407,7 +426,7 @@ def emulated_strategy_times(A, g, cfg, train, labels, C, dt, stream, steps=5):
     out = {}
     for s in STRATS:
         ctx = A.Ctx(-1, C, 0, stream.cuda_stream)
-        gr = ctx.graph_load(g.indptr, g.indices, aptgen.partition(g.n, C))
+        gr = ctx.graph_load(g.indptr, g.indices, partition(A, g, C))
         fs = ctx.fstore_create(gr, A.NFP if s == "NFP" else A.GDP, dt, cfg.dim, None, cfg.feat_seed)
         tr = make_trainer(A, ctx, gr, fs, cfg, dt, A.STRATEGY[s], labels)
         tr.set_params(aptgen.weights(cfg))
@@ -461,6 +480,8 @@ def main():
     args = parse()
     cfg = aptgen.CONFIGS[args.config]
     GAT_HEADS = args.gat_heads
+    global PARTITION
+    PARTITION = args.partition
     over = {}
     if args.feat_dim:
         over["dim"] = args.feat_dim

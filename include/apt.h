@@ -195,6 +195,21 @@ apt_status apt_fstore_create_tiered(apt_ctx* ctx, const apt_graph* g, apt_strate
                                     int dim, const float* host_feats, uint64_t feat_seed, const apt_fstore_opts* opts,
                                     apt_fstore** out);
 
+/* -------------------------------------------------------------- partition */
+/* Edge-cut partitioners of APT's Prepare stage for SNP / DNP ("edge-cut (e.g.,
+ * METIS)"; Fig. 11 / P:346 quality ablation):
+ *   APT_PART_RANGE   floor(u C / n)       (the generator's planted partition);
+ *   APT_PART_RANDOM  Philox(seed; u) mod C (Fig. 11's random partition);
+ *   APT_PART_LDG     linear deterministic greedy streaming (reading R10): nodes in
+ *                    ascending id, u -> argmax over p with size_p < cap of
+ *                    |N(u) in P_p| * (cap - size_p), ties to the smaller size_p then
+ *                    the smaller p, cap = ceil(1.05 n / C).
+ * Host CSR (symmetric), writes part[n] (host int32); *cut_edges (may be NULL) = CSR
+ * entries (u, v) with part[u] != part[v].  Host only, no ctx.                   */
+enum { APT_PART_RANGE = 0, APT_PART_RANDOM = 1, APT_PART_LDG = 2 };
+apt_status apt_partition(int64_t n, int64_t nnz, const int64_t* indptr, const int32_t* indices, int C, int method,
+                         uint64_t seed, int32_t* part, int64_t* cut_edges);
+
 /* ---------------------------------------------------------------- sampling */
 /* K-hop node-wise sampling of seeds_dev (device int64[n_seeds]) with
  * fanouts (host, fanouts[l-1] for layer l, 1..256), Philox key rng_seed and

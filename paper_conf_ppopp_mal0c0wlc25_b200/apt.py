@@ -116,6 +116,7 @@ def lib():
             "apt_trainer_step_host_pipelined": [vp, vp, i64, i64, i32, vp, vp],
             "apt_trainer_use_graph": [vp, i32], "apt_trainer_set_pipeline": [vp, i32], "apt_trainer_read": [vp, i32, i32, i32, vp, i64, vp, vp],
             "apt_trainer_phase_ms": [vp, vp, i32], "apt_trainer_agg_bytes": [vp, vp],
+            "apt_partition": [i64, i64, vp, vp, i32, i32, u64, vp, vp],
             "apt_dryrun": [vp, i64, vp], "apt_layer_fwd": [vp, i64], "apt_layer_bwd": [vp, vp, i64], "apt_profile_links": [vp, vp], "apt_select_strategy": [vp, vp, vp, vp],
         }
         for name, args in sig.items():
@@ -401,6 +402,22 @@ def exchange_selftest(rank, world, dist, group=None):
     """Host-only check of the bootstrap all-gather protocol (no GPU)."""
     fn = make_exchange(dist, group)
     check(lib().apt_exchange_selftest(rank, world, fn, None))
+
+
+PARTITION = {"range": 0, "random": 1, "ldg": 2}
+
+
+def partition(indptr, indices, n_parts, method="ldg", seed=0):
+    """apt_partition: edge-cut partition of a host CSR into n_parts parts (range /
+    random / ldg).  Returns (part int32[n], cut_edges)."""
+    indptr = np.ascontiguousarray(indptr, np.int64)
+    indices = np.ascontiguousarray(indices, np.int32)
+    n = len(indptr) - 1
+    part = np.empty(n, np.int32)
+    cut = C.c_int64(0)
+    check(lib().apt_partition(n, int(indptr[-1]), indptr.ctypes.data, indices.ctypes.data, n_parts,
+                              PARTITION[method], seed, part.ctypes.data, C.byref(cut)))
+    return part, cut.value
 
 
 def select_strategy(stats: PlanStats, bw: BwProfile):

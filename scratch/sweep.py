@@ -30,6 +30,9 @@ SWEEPS = {
     "papers-gat": ("papers", [dict(dim=128, hidden=h) for h in (32, 128, 512, 1024)], 4),
     "products-fanout": ("products", [dict(fanouts=(10, 5)), dict(fanouts=(15, 10)), dict(fanouts=(20, 15, 10))], 0),
     "tiny-gat": ("tiny", [dict(hidden=32), dict(hidden=128)], 4),
+    # Fig. 11 partition-quality ablation: planted range vs random vs LDG streaming
+    "products-partition": ("products", [dict(partition=p) for p in ("range", "random", "ldg")], 0),
+    "papers-partition": ("papers", [dict(partition=p) for p in ("range", "random", "ldg")], 0),
 }
 
 
@@ -89,7 +92,11 @@ def main():
     bench.GAT_HEADS = heads
     dt = A.DTYPE[args.dtype]
     for v in variants:
+        v = dict(v)
+        bench.PARTITION = v.pop("partition", "range")
         cfg = base.replace(**v)
+        if bench.PARTITION != "range":
+            v["partition"] = bench.PARTITION
         rec = {"sweep": args.sweep, "variant": {k: list(x) if isinstance(x, tuple) else x for k, x in v.items()},
                "config": bench.workload_config(cfg), "dtype": args.dtype, "gat_heads": heads,
                "graph_gen_s": round(t_gen, 1)}
