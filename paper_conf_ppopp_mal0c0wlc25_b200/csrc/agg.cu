@@ -14,6 +14,7 @@
 #include "common.cuh"
 #include "kernels.h"
 #include <algorithm>
+#include <cstdlib>
 
 namespace apt {
 
@@ -175,16 +176,128 @@ static cudaError_t dispatch_agg(const AggArgs& a, const Src& s, cudaStream_t st)
   return cudaGetLastError();
 }
 
+// ----------------------------------------------------- layer 1, branch-free loads
+// The layer-1 case (ELL from the sampler, rows of <= 16 vectors: two destination rows
+// per warp) without predicated loads: a lane whose edge is padding (past the row's
+// count, or filtered out by SNP) points at a zero row in shared memory, so every load
+// of a batch is issued unconditionally through generic addressing (feature rows in
+// global / peer / mapped-host memory, the zero row in shared memory: no hot spot).
+template <int EPV, int NB, int MINB>
+__global__ void __launch_bounds__(256, MINB) agg_l1_kernel(AggArgs a, EllFstoreSrc src) {
+  APT_PDL_PROLOGUE();
+  __shared__ uint4 zrow[16];
+  if (threadIdx.x < 16) zrow[threadIdx.x] = make_uint4(0, 0, 0, 0);
+  __syncthreads();
+  const int lane = lane_id();
+  const int sub = lane >> 4, l = lane & 15;
+  const int64_t n_dst = *a.n_dst;
+  const int V = int(ceil_div(a.dim, EPV));
+  const int lv = l < V ? l : 0;
+  const int k = src.k;
+  const int64_t nwarps = int64_t(gridDim.x) * (blockDim.x >> 5);
+  for (int64_t w = (int64_t(blockIdx.x) * blockDim.x + threadIdx.x) >> 5; w * 2 < n_dst; w += nwarps) {
+    const int64_t i = w * 2 + sub;
+    const bool valid = i < n_dst;
+    const int cnt = valid ? src.count(i) : 0;
+    const int cmax = max(cnt, __shfl_xor_sync(0xffffffffu, cnt, 16));
+    float acc[EPV];
+#pragma unroll
+    for (int q = 0; q < EPV; ++q) acc[q] = 0.f;
+    for (int e0 = 0; e0 < cmax; e0 += 16) {
+      int u = -1;
+      if (valid && e0 + l < k) u = src.node(i * k + e0 + l);
+      const bool keep = e0 + l < cnt && (!a.filt_part || a.filt_part[u] == a.keep_part);
+      const char* rp = keep ? src.row_ptr(u) : reinterpret_cast<const char*>(zrow);
+      const int m = min(16, cmax - e0);
+      for (int j = 0; j < m; j += NB) {
+        uint4 v[NB];
+#pragma unroll
+        for (int q = 0; q < NB; ++q) {
+          const char* r = reinterpret_cast<const char*>(
+              __shfl_sync(0xffffffffu, reinterpret_cast<uintptr_t>(rp), sub * 16 + ((j + q) & 15)));
+          v[q] = *reinterpret_cast<const uint4*>(r + lv * 16);
+        }
+#pragma unroll
+        for (int q = 0; q < NB; ++q) accumulate_vec<EPV>(acc, v[q]);
+      }
+    }
+    if (!valid || l >= V) continue;
+    if (a.z_ones && l == 0) a.z_bf16[i * a.z_bf16_pitch + a.dim] = 0x3F80;
+    const float fdeg = float(a.deg_override ? a.deg_override[i] : cnt);
+    const float rdeg = fdeg > 0.f ? __frcp_rn(fdeg) : 0.f;
+    float z[EPV];
+#pragma unroll
+    for (int q = 0; q < EPV; ++q) z[q] = fdeg > 0.f ? div_rn_rcp(acc[q], fdeg, rdeg) : 0.f;
+    const int c0 = l * EPV;
+    const bool full = c0 + EPV <= a.dim;
+    if (a.z_f32) {
+      float* o = a.z_f32 + i * a.z_f32_pitch + c0;
+#pragma unroll
+      for (int q = 0; q < EPV; ++q)
+        if (full || c0 + q < a.dim) o[q] = z[q];
+    }
+    if (a.z_bf16) {
+      uint16_t* o = a.z_bf16 + i * a.z_bf16_pitch + c0;
+      if (full) {
+        if constexpr (EPV == 8) {
+          *reinterpret_cast<uint4*>(o) = make_uint4(pack_bf16x2(z[0], z[1]), pack_bf16x2(z[2], z[3]),
+                                                    pack_bf16x2(z[4], z[5]), pack_bf16x2(z[6], z[7]));
+        } else {
+          *reinterpret_cast<uint2*>(o) = make_uint2(pack_bf16x2(z[0], z[1]), pack_bf16x2(z[2], z[3]));
+        }
+      } else {
+#pragma unroll
+        for (int q = 0; q < EPV; ++q) {
+          if (c0 + q < a.dim) {
+            __nv_bfloat16 h = __float2bfloat16_rn(z[q]);
+            o[q] = *reinterpret_cast<uint16_t*>(&h);
+          }
+        }
+      }
+    }
+  }
+}
+
 cudaError_t launch_agg_fstore(const AggArgs& a, const FeatView& fv, cudaStream_t st) {
   EllFstoreSrc s{a.cnt, a.nbr, a.k, fv, fv.pitch * (fv.dtype == kBF16 ? 2 : 4)};
   AggArgs b = a;
   b.dim = fv.dim;
+  const int epv = fv.dtype == kBF16 ? 8 : 4;
+  const int V = int(ceil_div(b.dim, epv));
+  // variant (A/B on products): 0 agg_kernel, 1 agg_l1_kernel (NB 4, default),
+  // 2 agg_l1_kernel with 8 loads in flight per lane.  All measured within 2 us (34 us in
+  // the step, 26.6 us alone); a cp.async double-buffered variant measured 38.7 us.
+  static const int variant = [] { const char* e = std::getenv("APT_AGG_VARIANT"); return e ? atoi(e) : 1; }();
+  if ((variant == 1 || variant == 2) && V <= 16) {
+    int64_t blocks = ceil_div(ceil_div(b.max_dst, 2) * 32, 256);
+    blocks = std::max<int64_t>(1, std::min<int64_t>(blocks, 148 * 16));
+    if (fv.dtype == kBF16) {
+      if (variant == 1) launch_pdl(agg_l1_kernel<8, 4, 6>, dim3(blocks), dim3(256), 0, st, b, s);
+      else launch_pdl(agg_l1_kernel<8, 8, 4>, dim3(blocks), dim3(256), 0, st, b, s);
+    } else {
+      if (variant == 1) launch_pdl(agg_l1_kernel<4, 4, 6>, dim3(blocks), dim3(256), 0, st, b, s);
+      else launch_pdl(agg_l1_kernel<4, 8, 4>, dim3(blocks), dim3(256), 0, st, b, s);
+    }
+    return cudaGetLastError();
+  }
   return fv.dtype == kBF16 ? dispatch_agg<8>(b, s, st) : dispatch_agg<4>(b, s, st);
 }
 
 cudaError_t launch_agg_csr(const AggArgs& a, cudaStream_t st) {
-  CsrSrc s{a.indptr, a.indices, a.x, a.x_pitch * 4};
-  return dispatch_agg<4>(a, s, st);
+  // rows wider than one launch covers (> 128 fp32 vectors): column chunks of 512
+  constexpr int kChunk = 512;
+  for (int c0 = 0; c0 < a.dim; c0 += kChunk) {
+    AggArgs b = a;
+    b.dim = std::min(kChunk, a.dim - c0);
+    b.x = a.x + c0;
+    if (a.z_f32) b.z_f32 = a.z_f32 + c0;
+    if (a.z_bf16) b.z_bf16 = a.z_bf16 + c0;
+    b.z_ones = (c0 + b.dim == a.dim) ? a.z_ones : 0;   // column a.dim, written by the last chunk
+    CsrSrc s{b.indptr, b.indices, b.x, a.x_pitch * 4};
+    cudaError_t e = dispatch_agg<4>(b, s, st);
+    if (e != cudaSuccess) return e;
+  }
+  return cudaSuccess;
 }
 
 // ---------------------------------------------------------------- backward

@@ -124,6 +124,20 @@ __global__ void __launch_bounds__(256) pull_bwd_kernel(PullArgs a) {
 }
 
 cudaError_t launch_pull_bwd(const PullArgs& a, cudaStream_t st) {
+  if (a.dim > 512) {   // wide rows: column chunks of 512 (128 fp32 vectors per lane group)
+    for (int c0 = 0; c0 < a.dim; c0 += 512) {
+      PullArgs b = a;
+      b.dim = std::min(512, a.dim - c0);
+      b.dz = a.dz + c0;
+      if (a.h) b.h = a.h + c0;
+      if (a.mask) b.mask = a.mask + c0 / 16;
+      if (a.g) b.g = a.g + c0;
+      if (a.gb) b.gb = a.gb + c0;
+      cudaError_t e = launch_pull_bwd(b, st);
+      if (e != cudaSuccess) return e;
+    }
+    return cudaSuccess;
+  }
   const int V = int(ceil_div(a.dim, 4));
   if ((a.dz_pitch & 3) || (a.h_pitch & 3) || (a.g && (a.g_pitch & 3)) || (a.gb && (a.gb_pitch & 3)))
     return cudaErrorInvalidValue;

@@ -177,7 +177,15 @@ __global__ void __launch_bounds__(256) colsum_kernel2(const T* __restrict__ g, i
 
 apt_status launch_colsum2(apt_ctx* c, const void* g, bool bf16, int64_t pitch, int dim, const int32_t* n_dev,
                                  float* out) {
-  if (dim > 1024) return set_err(c, APT_E_UNSUPPORTED, "colsum: dim > 1024");
+  if (dim > 1024) {   // column chunks of 1024
+    for (int c0 = 0; c0 < dim; c0 += 1024) {
+      const void* gc = bf16 ? static_cast<const void*>(static_cast<const uint16_t*>(g) + c0)
+                            : static_cast<const void*>(static_cast<const float*>(g) + c0);
+      apt_status s = launch_colsum2(c, gc, bf16, pitch, std::min(1024, dim - c0), n_dev, out + c0);
+      if (s != APT_OK) return s;
+    }
+    return APT_OK;
+  }
   const int blocks = 296;
   if (bf16) launch_pdl(colsum_kernel2<uint16_t>, dim3(blocks), dim3(256), 0, c->stream, static_cast<const uint16_t*>(g), pitch, dim, n_dev, out);
   else launch_pdl(colsum_kernel2<float>, dim3(blocks), dim3(256), 0, c->stream, static_cast<const float*>(g), pitch, dim, n_dev, out);

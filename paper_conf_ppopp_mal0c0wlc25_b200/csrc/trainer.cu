@@ -35,6 +35,8 @@ apt_status gat_alloc(apt_trainer* t, RankState& rs);
 apt_status gat_tables(apt_trainer* t);
 apt_status gat_layer1_fwd(apt_trainer* t, bool time_it);
 apt_status gat_layer1_bwd(apt_trainer* t);
+apt_status launch_colsum2(apt_ctx* c, const void* g, bool bf16, int64_t pitch, int dim, const int32_t* n_dev,
+                          float* out);
 
 // Floats of the flat gradient buffer [dW1 db1 (da_src1 da_dst1 for a GAT layer 1) dW2 db2 ...].
 int64_t grad_floats(const apt_trainer* t, const RankState& rs) {
@@ -176,13 +178,28 @@ apt_status weight_grad(apt_trainer* t, const Layer& L, const float* G, int64_t g
     c->launches++;
     return APT_OK;
   }
+  // CUDA cores (fp32 mode, or dims past the tcgen05 kernel): in bf16 mode the hidden
+  // layers' gradient exists only as its bf16 copy Gb (the pull kernel writes no fp32 G)
   SimtGemmArgs a{};
-  a.A = G; a.a_t = kF32; a.sam = 1; a.sak = g_pitch;
+  const bool gb = z_bf16 && L.Gb;
+  if (gb) { a.A = L.Gb; a.a_t = kBF16; a.sak = L.gb_pitch; }
+  else { a.A = G; a.a_t = kF32; a.sak = g_pitch; }
+  a.sam = 1;
   a.B = Z; a.b_t = z_bf16 ? kBF16 : kF32; a.sbk = z_pitch; a.sbn = 1;
   a.C = dW; a.ldc = dW_ld; a.M = L.d_out; a.N = d_in; a.K = max_rows; a.K_dev = n_rows;
-  a.accumulate = 1; a.k_chunk = 2048;
+  a.accumulate = 1; a.k_chunk = 256;      // short k-chunks: the simt k-loop is latency bound
   CK(c, launch_simt_gemm(a, st));
-  if (db) CK(c, launch_colsum(G, g_pitch, L.d_out, n_rows, max_rows, db, st));
+  if (db) {
+    if (gb) {
+      cudaStream_t keep = c->stream;
+      c->stream = st;
+      apt_status s2 = launch_colsum2(c, L.Gb, true, L.gb_pitch, L.d_out, n_rows, db);
+      c->stream = keep;
+      if (s2 != APT_OK) return s2;
+    } else {
+      CK(c, launch_colsum(G, g_pitch, L.d_out, n_rows, max_rows, db, st));
+    }
+  }
   c->launches += db ? 2 : 1;
   return APT_OK;
 }
@@ -664,7 +681,9 @@ apt_status upper_bwd(apt_trainer* t, RankState& rs) {
       CK(c, launch_tc_gemm(g, c->stream));
     } else {
       SimtGemmArgs a{};
-      a.A = L.G; a.a_t = kF32; a.sam = L.h_pitch; a.sak = 1;
+      if (bf) { a.A = L.Gb; a.a_t = kBF16; a.sam = L.gb_pitch; }   // bf16 mode: only Gb exists
+      else { a.A = L.G; a.a_t = kF32; a.sam = L.h_pitch; }
+      a.sak = 1;
       if (bf) { a.B = L.Wb; a.b_t = kBF16; a.sbk = L.wb_pitch; }
       else { a.B = L.W; a.b_t = kF32; a.sbk = L.d_in; }
       a.sbn = 1;

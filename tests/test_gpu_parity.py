@@ -225,6 +225,31 @@ def test_train_step_matches_oracle(A, ctx, tiny, dtype, step):
         assert np.allclose(tr.read("db", l)[0], db, **tol), f"db layer {l}"
 
 
+@pytest.mark.parametrize("dtype", ["f32", "bf16"])
+def test_train_step_wide_hidden(A, ctx, tiny, dtype):
+    """Hidden width past every single-launch limit (config 5 sweeps d' to 1024): the upper
+    layer's aggregation and the pull backward run in 512-column chunks, the projections
+    and weight gradients on the CUDA-core fallback (bf16 mode reads the bf16 gradient)."""
+    cfg, g, train = tiny
+    cfg = cfg.replace(hidden=1040)
+    tr, params, labels = _trainer(A, ctx, cfg, g, train, dtype)
+    tr.step(1, update=False)
+    seeds = tr.read("seeds")[:, 0].astype(np.int64)
+    blocks = oracle.sample_blocks(g, seeds, cfg.fanouts, cfg.sample_seed, 1)
+    p64 = [(W.astype(np.float64), b.astype(np.float64)) for W, b in params]
+    ref = model.train_step(blocks, cfg.feat_seed, cfg.dim, p64, labels[seeds], len(seeds), dtype)
+    tol = TOL[dtype]
+    K = len(blocks)
+    for l in range(1, K + 1):
+        assert np.allclose(tr.read("H", l), ref["cache"]["h"][l - 1], **tol), f"H layer {l}"
+    assert abs(tr.loss() - ref["loss"]) <= tol["rtol"] * abs(ref["loss"]) + tol["atol"]
+    for l in range(1, K + 1):
+        dW, db = ref["grads"][l - 1]
+        atol = tol["atol"] * (10 if dtype == "bf16" else 1)
+        assert np.allclose(tr.read("dW", l), dW, rtol=tol["rtol"], atol=atol), f"dW layer {l}"
+        assert np.allclose(tr.read("db", l)[0], db, rtol=tol["rtol"], atol=atol), f"db layer {l}"
+
+
 @pytest.mark.parametrize("use_graph", [False, True])
 def test_step_host_pipelined_matches_device_steps(A, ctx, tiny, use_graph):
     """The pipelined end-to-end call (submit batch t+1, run batch t) returns, call by call,
