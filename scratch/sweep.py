@@ -29,6 +29,7 @@ SWEEPS = {
     "friendster-h": ("friendster", [dict(hidden=8), dict(hidden=32), dict(hidden=128)], 0),
     "papers-gat": ("papers", [dict(dim=128, hidden=h) for h in (32, 128, 512, 1024)], 4),
     "products-fanout": ("products", [dict(fanouts=(10, 5)), dict(fanouts=(15, 10)), dict(fanouts=(20, 15, 10))], 0),
+    "papers-gat-wide": ("papers", [dict(dim=128, hidden=1024)], 4),
     "tiny-gat": ("tiny", [dict(hidden=32), dict(hidden=128)], 4),
     # Fig. 11 partition-quality ablation: planted range vs random vs LDG streaming
     "products-partition": ("products", [dict(partition=p) for p in ("range", "random", "ldg")], 0),
