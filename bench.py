@@ -336,6 +336,14 @@ def run_apt(args, cfg):
         os.path.join(ROOT, "MEASURED_PEAKS.json")) else None
     hbm_peak = peaks["hbm_gbs"] if peaks else 6650.0
     achieved = sum(agg_bytes) / (sum(agg_ms) * 1e-3) / 1e9
+    # DRAM traffic of the same kernel from one committed `ncu --set full` capture of this
+    # workload (dram__bytes_read + dram__bytes_write per launch), next to the algorithmic bytes
+    traffic, traffic_src = None, None
+    tpath = os.path.join(ROOT, "profiles", "r01_ncu_agg_l1_traffic.json")
+    if not GAT_HEADS and args.dtype == "bf16" and cfg.name == "products" and cfg.fanouts == (10, 10, 10) \
+            and os.path.exists(tpath):
+        tj = json.load(open(tpath))
+        traffic, traffic_src = tj["traffic_bytes_per_launch"], tj["source"]
     mean_agg = sum(agg_ms) / len(agg_ms)
     phase_mean = [sum(p[j] for p in phases) / len(phases) for j in range(6)]
 
@@ -351,7 +359,8 @@ def run_apt(args, cfg):
                 "timing": "host wall clock per call of apt_trainer_step_host_pipelined (syncs), max over ranks"},
         "gpu_launches": int(launches),
         "roofline": {"bound": "hbm", "achieved": achieved, "peak": hbm_peak, "unit": "GB/s",
-                     "frac": (achieved / hbm_peak) if achieved else None, "traffic": None,
+                     "frac": (achieved / hbm_peak) if achieved else None, "traffic": traffic,
+                     "traffic_source": traffic_src, "algorithmic_bytes_per_launch": sum(agg_bytes) / len(agg_bytes),
                      "kernel": "gat_fwd_kernel (layer-1 fused gather+attention+weighted sums)" if GAT_HEADS
                      else "agg_kernel (layer-1 fused gather+mean)",
                      "peak_source": "MEASURED_PEAKS.json hbm_gbs" if peaks else "fallback 6.65 TB/s",
