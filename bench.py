@@ -170,6 +170,19 @@ def oracle_steps(cfg, g, train, labels, n_steps, world=1):
     return times, seeds_done
 
 
+def host_cpu():
+    """The box's host CPU model and core count (the oracle baseline's machine)."""
+    model = "unknown"
+    try:
+        for line in open("/proc/cpuinfo"):
+            if line.startswith("model name"):
+                model = line.split(":", 1)[1].strip()
+                break
+    except OSError:
+        pass
+    return {"model": model, "nproc": os.cpu_count()}
+
+
 def gat_oracle_step(cfg, blocks, params, labels_s, n_global):
     """The oracle's step with a GAT first layer (oracle/gat.py, fp64) and SAGE-mean upper
     layers: forward, CE loss, backward of every layer (test infrastructure timed as a baseline)."""
@@ -219,7 +232,8 @@ def run_reference(args, cfg):
             "steps": args.steps, "warmup": args.warmup, "ms_per_step": ms, "higher_is_better": True,
             "scaling": "weak", "vs_baseline": None, "dtype": "f64", "data": "synthetic",
             "config": workload_config(cfg),
-            "cpu_baseline": {"value": value, "unit": "seeds/s", "cores": 1, "kind": "oracle", "sample": sample},
+            "cpu_baseline": {"value": value, "unit": "seeds/s", "cores": 1, "kind": "oracle", "sample": sample,
+                             "host": host_cpu()},
             "e2e": {"value": value, "unit": "seeds/s", "h2d_bytes_per_step": 0, "d2h_bytes_per_step": 0}}
     print(json.dumps(line), flush=True)
     return 0
@@ -304,6 +318,26 @@ def run_apt(args, cfg):
         dist.all_reduce(tt, op=dist.ReduceOp.MAX)
         ms = float(tt.item())
     value = world * cfg.batch / (ms / 1e3)
+    pct = {f"p{q}": float(np.percentile(step_ms, q)) for q in (10, 50, 90)}
+
+    # ---- one full epoch, timed as a whole (validates epoch = steps x step time);
+    # all steps of epoch 0 back to back through the pipelined graph, no L2 flush in between
+    epoch_measured = None
+    if spe <= 4096:
+        if world > 1:
+            dist.barrier()
+        torch.cuda.synchronize()
+        ee0, ee1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+        ee0.record(stream)
+        for s_ in range(spe):
+            tr.step(s_)
+        ee1.record(stream)
+        torch.cuda.synchronize()
+        epoch_measured = ee0.elapsed_time(ee1) / 1e3
+        if world > 1:
+            tt = torch.tensor([epoch_measured], device="cuda")
+            dist.all_reduce(tt, op=dist.ReduceOp.MAX)
+            epoch_measured = float(tt.item())
 
     # ---- e2e: host global batches in (pinned), host losses out, through the public
     # pipelined call apt_trainer_step_host_pipelined (submit batch t+1, run batch t): each
@@ -351,7 +385,8 @@ def run_apt(args, cfg):
         "metric": METRIC, "value": value, "unit": "seeds/s", "n_gpus": world, "steps": K, "warmup": args.warmup,
         "ms_per_step": ms, "higher_is_better": True, "scaling": "weak", "vs_baseline": None,
         "dtype": args.dtype, "data": "synthetic",
-        "epoch_s": spe * ms / 1e3, "steps_per_epoch": spe,
+        "epoch_s": spe * ms / 1e3, "steps_per_epoch": spe, "epoch_s_measured": epoch_measured,
+        "ms_per_step_pct": pct,
         "config": dict(workload_config(cfg), strategy=args.strategy, parallelism=f"{args.strategy.lower()}{world}",
                        global_batch=B, l2="flushed between timed steps (256 MB write); inputs also > L2",
                        cuda_graph=not args.no_graph),
@@ -374,6 +409,7 @@ def run_apt(args, cfg):
     if rank == 0 and world == 1 and not args.no_cpu_baseline:
         times, nseeds = oracle_steps(cfg, g, train, labels, args.cpu_steps, 1)
         out["cpu_baseline"] = {"value": nseeds / sum(times), "unit": "seeds/s", "cores": 1, "kind": "oracle",
+                               "host": host_cpu(),
                                "sample": f"first {args.cpu_steps} steps of epoch 0 ({cfg.batch} seeds each, "
                                          f"full step: sampling + fp64 {'GAT layer 1 + ' if GAT_HEADS else ''}SAGE "
                                          f"fwd/bwd), one host thread"}

@@ -379,6 +379,38 @@ __global__ void trial_ids_kernel(int32_t* ids, int64_t n, int64_t n_rows, uint32
     ids[t] = int32_t(h % uint32_t(n_rows));
   }
 }
+// Peer-operator trials (one process per GPU): the same row gather reading another
+// rank's table (pull), writing into it (push), rows spread over every peer
+// (all-to-all), whole chunks from every peer (all-gather), chunk sums over the peers
+// (reduce-scatter: the fused Reshuffle's reduce) and full sums (all-reduce).
+__global__ void trial_peer_gather_kernel(const uint4* const* __restrict__ tab, int C, int self, int mode,
+                                         int64_t n_rows, int vec_per_row, const int32_t* __restrict__ ids, int64_t n,
+                                         uint4* __restrict__ out, uint4* const* __restrict__ wtab) {
+  const int64_t total = n * vec_per_row;
+  for (int64_t t = int64_t(blockIdx.x) * blockDim.x + threadIdx.x; t < total; t += int64_t(gridDim.x) * blockDim.x) {
+    const int64_t i = t / vec_per_row;
+    const int j = int(t - i * vec_per_row);
+    const int peer = mode == 2 ? (self + 1 + int(i % (C - 1))) % C : (self + 1) % C;
+    if (mode == 1) wtab[peer][int64_t(ids[i]) * vec_per_row + j] = out[t];               // push
+    else out[t] = ld_nc_v4(tab[peer] + int64_t(ids[i]) * vec_per_row + j);               // pull / all-to-all
+  }
+}
+__global__ void trial_collective_kernel(const float* const* __restrict__ tab, int C, int self, int mode, int64_t n,
+                                        float* __restrict__ out) {
+  // mode 0 all-gather (n floats per rank), 1 reduce-scatter (own chunk of n/C), 2 all-reduce (n)
+  const int64_t chunk = mode == 1 ? n / C : n;
+  const int64_t total = mode == 0 ? n * C : chunk;
+  for (int64_t t = int64_t(blockIdx.x) * blockDim.x + threadIdx.x; t < total; t += int64_t(gridDim.x) * blockDim.x) {
+    if (mode == 0) {
+      out[t] = tab[t / n][t % n];
+    } else {
+      const int64_t j = mode == 1 ? int64_t(self) * chunk + t : t;
+      float s = 0.f;
+      for (int r = 0; r < C; ++r) s += tab[r][j];
+      out[t] = s;
+    }
+  }
+}
 }  // namespace apt
 
 extern "C" apt_status apt_profile_links(apt_ctx* c, apt_bw_profile* out) {
@@ -436,7 +468,7 @@ extern "C" apt_status apt_profile_links(apt_ctx* c, apt_bw_profile* out) {
   CK(c, cudaGetLastError());
   // NVLink operators (peer pull / push, all-to-all, all-gather, reduce-scatter,
   // all-reduce): measured references of this pool (B200_PROFILING.md) when no peer
-  // GPU is attached to this ctx.
+  // GPU is attached to this ctx ...
   const double nvl = 770e9, ar_bus = 725e9, a_peer = 3e-6;
   const int C = std::max(2, c->world);
   for (int op : {APT_OP_PEER_PULL, APT_OP_PEER_PUSH, APT_OP_ALLTOALLV, APT_OP_ALLGATHER, APT_OP_REDUCE_SCATTER,
@@ -444,6 +476,65 @@ extern "C" apt_status apt_profile_links(apt_ctx* c, apt_bw_profile* out) {
     out->alpha_s[op] = a_peer;
     out->beta_Bps[op] = op == APT_OP_ALLREDUCE ? ar_bus * C / (2.0 * (C - 1)) : nvl;
     out->measured[op] = 0;
+  }
+  // ... and timed over the peers' CUDA-IPC-mapped tables in a job of one process per
+  // GPU (collective: every rank runs the same trials between device barriers, so the
+  // links carry all ranks' traffic at once, as in a step)
+  if (multiprocess(c)) {
+    std::vector<void*> opened;
+    std::vector<void*> tv(c->world, nullptr);
+    apt_status st = share_ptr(c, table, tv.data(), &opened);
+    if (st != APT_OK) return st;
+    uint4** tab = A.alloc<uint4*>(c->world, false);
+    if (!tab) return set_err(c, APT_E_OOM, "apt_profile_links: out of device memory");
+    CK(c, cudaMemcpyAsync(tab, tv.data(), sizeof(void*) * c->world, cudaMemcpyHostToDevice, c->stream));
+    cudaEventCreate(&e0);
+    cudaEventCreate(&e1);
+    const int self = c->rank, W = c->world;
+    auto timed = [&](auto&& launch) -> double {   // barrier, then the op on every rank at once
+      float b = 1e30f;
+      for (int it = 0; it < 6; ++it) {
+        if (device_barrier(c) != APT_OK) return -1.0;
+        cudaEventRecord(e0, c->stream);
+        launch();
+        cudaEventRecord(e1, c->stream);
+        cudaEventSynchronize(e1);
+        float ms = 0.f;
+        cudaEventElapsedTime(&ms, e0, e1);
+        if (it) b = std::min(b, ms);
+      }
+      return double(b) * 1e-3;
+    };
+    uint4* const* wtab = tab;
+    const int modes[3] = {0, 1, 2};
+    const int ops[3] = {APT_OP_PEER_PULL, APT_OP_PEER_PUSH, APT_OP_ALLTOALLV};
+    for (int m = 0; m < 3; ++m) {
+      const double ts = timed([&] { trial_peer_gather_kernel<<<blocks, 256, 0, c->stream>>>(tab, W, self, modes[m], table_rows, vec, ids, n_small, outb, wtab); });
+      const double tb = timed([&] { trial_peer_gather_kernel<<<blocks, 256, 0, c->stream>>>(tab, W, self, modes[m], table_rows, vec, ids, n_big, outb, wtab); });
+      if (ts < 0 || tb < 0) return set_err(c, APT_E_DEVICE_ASSERT, "apt_profile_links: barrier failed");
+      fit(ops[m], ts, double(n_small) * vec * 16, tb, double(n_big) * vec * 16);
+    }
+    const float* const* ftab = reinterpret_cast<float* const*>(tab);
+    float* fout = reinterpret_cast<float*>(outb);
+    const int cops[3] = {APT_OP_ALLGATHER, APT_OP_REDUCE_SCATTER, APT_OP_ALLREDUCE};
+    const int64_t f_small = int64_t(1) << 14, f_big = int64_t(1) << 22;   // floats per rank
+    for (int m = 0; m < 3; ++m) {
+      const double ts = timed([&] { trial_collective_kernel<<<blocks, 256, 0, c->stream>>>(ftab, W, self, m, f_small, fout); });
+      const double tb = timed([&] { trial_collective_kernel<<<blocks, 256, 0, c->stream>>>(ftab, W, self, m, f_big, fout); });
+      if (ts < 0 || tb < 0) return set_err(c, APT_E_DEVICE_ASSERT, "apt_profile_links: barrier failed");
+      // bytes each rank receives: all-gather (C-1) n, reduce-scatter (C-1) n / C, all-reduce (C-1) n
+      const double k = m == 1 ? double(W - 1) / W : double(W - 1);
+      fit(cops[m], ts, 4.0 * f_small * k, tb, 4.0 * f_big * k);
+    }
+    cudaEventDestroy(e0);
+    cudaEventDestroy(e1);
+    CK(c, cudaStreamSynchronize(c->stream));
+    if ((st = device_barrier(c)) != APT_OK) return st;
+    CK(c, cudaStreamSynchronize(c->stream));
+    close_peers(opened);
+    char x = 0;
+    std::vector<char> xs(c->world);
+    if ((st = allgather(c, &x, xs.data(), 1)) != APT_OK) return st;   // every mapping closed before any free
   }
   return APT_OK;
 }

@@ -13,6 +13,7 @@
 #include <algorithm>
 #include <cmath>
 #include <cstdlib>
+#include <functional>
 #include <vector>
 #include <cstring>
 #include <cub/device/device_radix_sort.cuh>
@@ -786,22 +787,44 @@ apt_status step_body(apt_trainer* t, int update, bool host_batch, int q = 0) {
   apt_status s = sample_all(t, q, host_batch, c->stream, true);
   if (s != APT_OK) return s;
   activate(t, q);
+  t->deferred_fork = nullptr;   // unpipelined: nothing to fork (a failed earlier call may have left one)
   return compute_body(t, update);
 }
 
 // Pipelined step: compute on set p while the next step (id `next` is the value of the
 // set_step node, patched per replay) is sampled into set p^1 on the sampling stream.
+// Where the next step's sampling branch forks off the step (A/B): 0 at the
+// step's start, 1 after the layer-1 forward (the gather+aggregate then runs alone).
+static int sample_fork_point() {
+  static const int v = [] { const char* e = std::getenv("APT_SAMPLE_FORK"); return e ? atoi(e) : 1; }();
+  return v;
+}
+
+// Run the next-step sampling fork now, or leave it for compute_body to launch right
+// after the layer-1 forward.
+static apt_status fork_or_defer(apt_trainer* t, std::function<apt_status()> fork) {
+  if (sample_fork_point() == 1) {
+    t->deferred_fork = std::move(fork);
+    return APT_OK;
+  }
+  return fork();
+}
+
 apt_status pipelined_body(apt_trainer* t, int p, int update, uint64_t next) {
   apt_ctx* c = t->ctx;
   CK(c, record_ev(t, 0));
-  CK(c, cudaEventRecord(c->ev_pfork, c->stream));
-  CK(c, cudaStreamWaitEvent(c->samp, c->ev_pfork, 0));
-  set_step_kernel<<<1, 1, 0, c->samp>>>(t->step_cells + (p ^ 1), next);
-  CK(c, cudaGetLastError());
-  c->launches++;
-  apt_status s = sample_all(t, p ^ 1, false, c->samp, false);
+  apt_status s = fork_or_defer(t, [t, c, p, next]() -> apt_status {
+    CK(c, cudaEventRecord(c->ev_pfork, c->stream));
+    CK(c, cudaStreamWaitEvent(c->samp, c->ev_pfork, 0));
+    set_step_kernel<<<1, 1, 0, c->samp>>>(t->step_cells + (p ^ 1), next);
+    CK(c, cudaGetLastError());
+    c->launches++;
+    apt_status s2 = sample_all(t, p ^ 1, false, c->samp, false);
+    if (s2 != APT_OK) return s2;
+    CK(c, cudaEventRecord(c->ev_pjoin, c->samp));
+    return APT_OK;
+  });
   if (s != APT_OK) return s;
-  CK(c, cudaEventRecord(c->ev_pjoin, c->samp));
   t->csc_forked = false;
   activate(t, p);
   s = compute_body(t, update);
@@ -826,6 +849,12 @@ apt_status compute_body(apt_trainer* t, int update) {
     }
   } else {
     apt_status s = layer1_fwd_strategy(t);
+    if (s != APT_OK) return s;
+  }
+  if (t->deferred_fork) {   // pipelined: the next step's sampling branch forks here
+    std::function<apt_status()> f = std::move(t->deferred_fork);
+    t->deferred_fork = nullptr;
+    apt_status s = f();
     if (s != APT_OK) return s;
   }
   CK(c, record_ev(t, 2));
@@ -1136,14 +1165,18 @@ apt_status apt_trainer_step_host_pipelined(apt_trainer* t, const int64_t* next_b
   }
   auto body = [&](uint64_t nstep) -> apt_status {
     CK(c, record_ev(t, 0));
-    CK(c, cudaEventRecord(c->ev_pfork, c->stream));
-    CK(c, cudaStreamWaitEvent(c->samp, c->ev_pfork, 0));
-    CK(c, cudaMemcpyAsync(t->hb_dev + q * t->hb_len, stage, hb_bytes, cudaMemcpyHostToDevice, c->samp));
-    set_step_kernel<<<1, 1, 0, c->samp>>>(t->step_cells + q, nstep);
-    CK(c, cudaGetLastError());
-    apt_status s = sample_all(t, q, true, c->samp, false);
+    apt_status s = fork_or_defer(t, [&, nstep]() -> apt_status {
+      CK(c, cudaEventRecord(c->ev_pfork, c->stream));
+      CK(c, cudaStreamWaitEvent(c->samp, c->ev_pfork, 0));
+      CK(c, cudaMemcpyAsync(t->hb_dev + q * t->hb_len, stage, hb_bytes, cudaMemcpyHostToDevice, c->samp));
+      set_step_kernel<<<1, 1, 0, c->samp>>>(t->step_cells + q, nstep);
+      CK(c, cudaGetLastError());
+      apt_status s2 = sample_all(t, q, true, c->samp, false);
+      if (s2 != APT_OK) return s2;
+      CK(c, cudaEventRecord(c->ev_pjoin, c->samp));
+      return APT_OK;
+    });
     if (s != APT_OK) return s;
-    CK(c, cudaEventRecord(c->ev_pjoin, c->samp));
     t->csc_forked = false;
     activate(t, p);
     s = compute_body(t, update);

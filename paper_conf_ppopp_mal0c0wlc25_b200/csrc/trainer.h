@@ -2,6 +2,7 @@
 #pragma once
 #include <cuda_runtime.h>
 
+#include <functional>
 #include <vector>
 
 #include "runtime.h"
@@ -180,6 +181,7 @@ struct apt_trainer {
   int64_t primed = -1;               // step id already sampled into sset[primed_parity]
   int primed_parity = 0;
   bool csc_forked = false;
+  std::function<apt_status()> deferred_fork;   // pipelined: next-step sampling, launched after the layer-1 forward
   bool fused_l1 = false;             // the last layer-1 forward ran as the single fused kernel           // this step's block transposes run on the side branch (wait ev_csc)
   cudaGraphExec_t gexec_p[2][2] = {};   // [parity][update] pipelined step graphs
   cudaGraph_t graph_p[2][2] = {};

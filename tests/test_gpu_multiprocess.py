@@ -35,3 +35,14 @@ def test_multiprocess_gat_layer_matches_oracle(world):
     out = r.stdout + r.stderr
     line = [l for l in out.splitlines() if l.startswith("RESULT")]
     assert r.returncode == 0 and line and line[0] == "RESULT OK", out[-4000:]
+
+
+@pytest.mark.parametrize("world", [2])
+def test_multiprocess_link_trials_measure_peer_ops(world):
+    env = dict(os.environ, APT_TEST_DEVICE="0")
+    cmd = [sys.executable, "-m", "torch.distributed.run", "--nnodes=1", f"--nproc-per-node={world}",
+           "--master-addr", "127.0.0.1", "--master-port", "29535", os.path.join(ROOT, "tests", "mp_links.py")]
+    r = subprocess.run(cmd, capture_output=True, text=True, timeout=600, env=env, cwd=ROOT)
+    out = r.stdout + r.stderr
+    line = [l for l in out.splitlines() if l.startswith("RESULT")]
+    assert r.returncode == 0 and line and line[0] == "RESULT OK", out[-4000:]
