@@ -17,13 +17,20 @@ from oracle import model
 
 
 # ---------------------------------------------------------------- O0 Philox
-@pytest.mark.parametrize("ctr,key,expect", [
-    # Random123 kat_vectors, philox4x32_10 (Salmon et al. SC'11)
-    ([0, 0, 0, 0], [0, 0], [0x6627e8d5, 0xe169c58d, 0xbc57ac4c, 0x9b00dbd8]),
-    ([0xffffffff] * 4, [0xffffffff] * 2, [0x408f276d, 0x41c83b0e, 0xa20bc7c6, 0x6d5451fd]),
-    ([0x243f6a88, 0x85a308d3, 0x13198a2e, 0x03707344], [0xa4093822, 0x299f31d0],
-     [0xd16cfe09, 0x94fdcceb, 0x5001e420, 0x24126ea1]),
-])
+def _philox_kats():
+    """tests/golden/philox4x32_10_kat.txt: Random123 kat_vectors (cited in the file)."""
+    import os
+    path = os.path.join(os.path.dirname(__file__), "golden", "philox4x32_10_kat.txt")
+    out = []
+    for line in open(path):
+        if line.strip() and not line.startswith("#"):
+            ctr, key, exp = (list(int(w, 16) for w in f.split()) for f in line.split("|"))
+            out.append((ctr, key, exp))
+    assert len(out) == 3
+    return out
+
+
+@pytest.mark.parametrize("ctr,key,expect", _philox_kats())
 def test_philox_kat(ctr, key, expect):
     assert [int(x) for x in oracle.philox(ctr, key)] == expect
 

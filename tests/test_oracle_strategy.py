@@ -4,6 +4,8 @@ The worked example of Figs. 2-3 pins the virtual-node / remote-row
 logic; closed-form volumes pin the counters; Table 1's text
  gives directional checks.
 """
+import os
+
 import numpy as np
 import pytest
 
@@ -11,10 +13,30 @@ import aptgen
 import oracle
 from oracle import strategy as S
 
+GOLDEN = os.path.join(os.path.dirname(__file__), "golden", "fig2_fig3_example.txt")
+
+
+def _golden():
+    """tests/golden/fig2_fig3_example.txt: the paper's Fig. 2/3 example."""
+    part, blocks, expect = {}, {}, []
+    for line in open(GOLDEN):
+        w = line.split()
+        if not w or w[0].startswith("#"):
+            continue
+        if w[0] == "partition":
+            part.update({c: int(w[1][3:]) - 1 for c in w[2:]})
+        elif w[0] == "block":
+            blocks.setdefault(int(w[1][3:]) - 1, []).append((w[2], w[4:]))
+        elif w[0] == "expect":
+            expect.append(w[1:])
+    return part, blocks, expect
+
+
 # Fig. 2(a)/3 node names -> ids.  GPU 1 manages A,B,E,G,H; GPU 2 manages C,D,F,M,K.
-NAMES = "ABCDEFGHKM"
+_PART, _BLOCKS, _EXPECT = _golden()
+NAMES = "".join(sorted(_PART))
 ID = {c: i for i, c in enumerate(NAMES)}
-PART = np.array([0 if c in "ABEGH" else 1 for c in NAMES], np.int32)
+PART = np.array([_PART[c] for c in NAMES], np.int32)
 
 
 def hand_block(dst, edges):
@@ -35,9 +57,28 @@ def hand_block(dst, edges):
 @pytest.fixture
 def fig2():
     # seed A on GPU 1: layer-1 destinations B, K; B <- G, H and K <- D, A.
-    b0 = hand_block("BK", {"B": "GH", "K": "DA"})
-    b1 = hand_block("", {})
-    return [b0, b1]
+    out = []
+    for g in range(2):
+        rows = _BLOCKS.get(g, [])
+        out.append(hand_block("".join(v for v, _ in rows), {v: "".join(us) for v, us in rows}))
+    return out
+
+
+def test_fig3_golden_expectations(fig2):
+    """Every `expect` line of the golden file (each cites its passage there)."""
+    assert len(_EXPECT) >= 10
+    for strat, key, *args in _EXPECT:
+        if key == "col_range":
+            assert S.col_range(int(args[0][3:]) - 1, 2, 4) == (int(args[1]), int(args[2]))
+            continue
+        st = S.emulate_layer1(strat, fig2, PART, 2, d=4, d_out=2)
+        g = int(args[0][3:]) - 1
+        if key in ("virtual", "requests", "request"):
+            field = "virtual" if key == "virtual" else "requests"
+            (o, vs), = st[g][field]
+            assert o == int(args[1][3:]) - 1 and "".join(NAMES[v] for v in vs) == args[2], (strat, key)
+        else:
+            assert st[g][key] == int(args[1]), (strat, key, st[g][key])
 
 
 def test_fig3_snp_one_virtual_node(fig2):
