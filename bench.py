@@ -288,7 +288,7 @@ def run_apt(args, cfg):
 
     K = args.steps
     ev = [(torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)) for _ in range(K)]
-    agg_ms, phases, step_ids, agg_bytes = [], [], [], []
+    agg_ms, phases, step_ids, agg_bytes, step_bytes = [], [], [], [], []
     bf = 2 if args.dtype == "bf16" else 4
     if world > 1:
         dist.barrier()
@@ -306,6 +306,8 @@ def run_apt(args, cfg):
             agg_ms.append(ph[5])
             step_ids.append(s)
             agg_bytes.append(layer1_bytes(ctx, gr, tr, cfg, rank, s, bf))   # outside the events
+            if i < 5 and not GAT_HEADS:
+                step_bytes.append(step_phase_bytes(ctx, gr, g, tr, cfg, rank, s, bf))
         torch.cuda.synchronize()
     launches = ctx.launches() - l0
     if world > 1:
@@ -400,6 +402,7 @@ def run_apt(args, cfg):
                      else "agg_kernel (layer-1 fused gather+mean)",
                      "peak_source": "MEASURED_PEAKS.json hbm_gbs" if peaks else "fallback 6.65 TB/s",
                      "share_of_step": mean_agg / ms_local},
+        "step_roofline": step_roofline(step_bytes, hbm_peak, ms) if step_bytes else None,
         "phases_ms": {"sample": phase_mean[0], "layer1_fwd": phase_mean[1], "upper_fwd_loss": phase_mean[2],
                       "backward": phase_mean[3], "allreduce_sgd": phase_mean[4], "agg_kernel": phase_mean[5]},
         "clocks": clk.summary(),
@@ -506,6 +509,61 @@ def layer1_bytes(ctx, gr, tr, cfg, rank, step, bf):
         n += v.n_dst * cfg.dim * bf * (GAT_HEADS - 1) + v.n_edges * GAT_HEADS * 4
     b.close()
     return n
+
+
+def step_phase_bytes(ctx, gr, g, tr, cfg, rank, step, bf):
+    """Algorithmic HBM bytes of one whole GDP step at C = 1, per phase (SURVEY §8(d)'s
+    per-phase table): sampling (indptr sector + neighbour sectors + writes),
+    compaction, the layer-1 gather of unique rows + mean, every projection, the upper
+    layers' means, loss, backward (dZ = G W, the mean's backward, weight gradients) and
+    SGD.  Block sizes come from apt_sample on the same seeds and step."""
+    import torch
+    seeds = torch.as_tensor(tr.read("seeds", rank=rank)[:, 0].astype(np.int64)).cuda()
+    K = len(cfg.fanouts)
+    b = ctx.sample(gr, seeds, len(seeds), cfg.fanouts, cfg.sample_seed, step)
+    dims = [cfg.dim] + [o for _, o in cfg.dims()]
+    bz = bg = bw = bf                    # Z, G and W copies in the compute dtype; H, dZ fp32
+    ph = {"sampling": 0, "compaction": 0, "layer1_gather_mean": 0, "projections": 0, "upper_means": 0,
+          "loss": 0, "backward": 0, "sgd": 0}
+    for h in range(K):
+        dst, src, indptr, _ = b.block_host(h)
+        k = cfg.fanouts[K - 1 - h]
+        deg = (g.indptr[dst.astype(np.int64) + 1] - g.indptr[dst.astype(np.int64)]).astype(np.int64)
+        nb = np.where(deg <= k, (4 * deg + 31) // 32 * 32, k * 32)
+        E = int(indptr[-1]) if len(indptr) else 0
+        N, U = len(dst), len(src)
+        ph["sampling"] += N * 32 + int(nb.sum()) + N * k * 8
+        ph["compaction"] += E * 12 + U * 8
+        layer = K - h
+        din, dout = dims[layer - 1], dims[layer]
+        if layer == 1:
+            ph["layer1_gather_mean"] += U * din * bf + E * 4 + (N + 1) * 4 + N * din * bz
+            ph["backward"] += N * (dout * bg + din * bz)                          # dW1 = G^T Z
+        else:
+            ph["upper_means"] += U * din * 4 + E * 4 + (N + 1) * 4 + N * din * bz
+            ph["backward"] += (N * dout * bg + din * dout * bw + N * din * 4      # dZ = G W
+                               + N * din * 4 + E * 4 + U * din * (4 + bg)         # mean bwd (mask, G)
+                               + N * (dout * bg + din * bz))                      # dW = G^T Z
+        ph["projections"] += N * din * bz + N * dout * 4 + din * dout * bw
+        if layer == K:
+            ph["loss"] += N * dout * 4 * 2
+    nparam = sum(dims[i] * dims[i + 1] + dims[i + 1] for i in range(K))
+    ph["sgd"] = nparam * (4 + 4 + 4 + bw)
+    b.close()
+    return ph
+
+
+def step_roofline(step_bytes, peak_gbs, ms):
+    """T_roof / T_meas of the whole step: T_roof = the step's algorithmic
+    HBM bytes / the measured HBM peak (every phase HBM-bound at C = 1, no NVLink)."""
+    keys = step_bytes[0].keys()
+    mean = {k: sum(s[k] for s in step_bytes) / len(step_bytes) for k in keys}
+    total = sum(mean.values())
+    t_roof_ms = total / (peak_gbs * 1e9) * 1e3
+    return {"bound": "hbm", "bytes_per_step": total, "bytes_by_phase": mean, "peak_gbs": peak_gbs,
+            "t_roof_ms": t_roof_ms, "t_meas_ms": ms, "frac": t_roof_ms / ms,
+            "note": "T_roof = algorithmic bytes (SURVEY 8(d) table, sector-granular random reads, "
+                    "unique rows once) / measured HBM peak; mean over the first timed steps"}
 
 
 def make_trainer(A, ctx, gr, fs, cfg, dt, strat, labels, lr=0.05):

@@ -7,7 +7,9 @@ the aggregation (Z10), W applied after the mean (Z8: W*mean = mean(W*) in
 exact arithmetic).  Loss = sum_s CE(h^K_s, y_s) / |global batch| (Z20).
 
 bf16 mode emulates the CUDA path's rounding points (O5): features are exact
-in bf16 (O4), Z -> fp32 -> bf16 RNE, W -> bf16 RNE, everything else fp64.
+in bf16 (O4), Z -> fp32 -> bf16 RNE, W -> bf16 RNE, hidden activations
+h^l (l < K) -> bf16 RNE after bias + ReLU (reading R11: the next
+layer's mean and the ReLU mask read the stored bf16 copy), everything else fp64.
 """
 from __future__ import annotations
 
@@ -60,6 +62,8 @@ def forward(blocks, feat_seed, dim, params, dtype="f32", x0=None, snp=None):
                 Z = bf16_round(Z)
             pre = Z @ W.T + np.asarray(b, np.float64)
         H = np.maximum(pre, 0.0) if l < K else pre
+        if dtype == "bf16" and l < K:
+            H = bf16_round(H)                  # reading R11
         cache["Z"].append(Z)
         cache["pre"].append(pre)
         cache["h"].append(H)

@@ -46,8 +46,8 @@ struct EllFstoreSrc {            // layer 1: sampler ELL + the feature store (lo
   }
 };
 
-struct CsrSrc {                  // upper layers: block CSR over the previous layer's rows
-  const int32_t* indptr; const int32_t* indices; const float* x; int64_t row_bytes;
+struct CsrSrc {                  // upper layers: block CSR over the previous layer's rows (fp32 or bf16)
+  const int32_t* indptr; const int32_t* indices; const void* x; int64_t row_bytes;
   __device__ __forceinline__ int64_t begin(int64_t i) const { return indptr[i]; }
   __device__ __forceinline__ int count(int64_t i) const { return indptr[i + 1] - indptr[i]; }
   __device__ __forceinline__ int cap(int c) const { return c; }
@@ -284,17 +284,24 @@ cudaError_t launch_agg_fstore(const AggArgs& a, const FeatView& fv, cudaStream_t
 }
 
 cudaError_t launch_agg_csr(const AggArgs& a, cudaStream_t st) {
-  // rows wider than one launch covers (> 128 fp32 vectors): column chunks of 512
-  constexpr int kChunk = 512;
+  // rows wider than one launch covers (> 128 16-B vectors): column chunks of 512 fp32 /
+  // 1024 bf16 columns
+  const bool bf = a.xb != nullptr;
+  const int kChunk = bf ? 1024 : 512;
   for (int c0 = 0; c0 < a.dim; c0 += kChunk) {
     AggArgs b = a;
     b.dim = std::min(kChunk, a.dim - c0);
-    b.x = a.x + c0;
     if (a.z_f32) b.z_f32 = a.z_f32 + c0;
     if (a.z_bf16) b.z_bf16 = a.z_bf16 + c0;
     b.z_ones = (c0 + b.dim == a.dim) ? a.z_ones : 0;   // column a.dim, written by the last chunk
-    CsrSrc s{b.indptr, b.indices, b.x, a.x_pitch * 4};
-    cudaError_t e = dispatch_agg<4>(b, s, st);
+    cudaError_t e;
+    if (bf) {
+      CsrSrc s{b.indptr, b.indices, a.xb + c0, a.x_pitch * 2};
+      e = dispatch_agg<8>(b, s, st);
+    } else {
+      CsrSrc s{b.indptr, b.indices, a.x + c0, a.x_pitch * 4};
+      e = dispatch_agg<4>(b, s, st);
+    }
     if (e != cudaSuccess) return e;
   }
   return cudaSuccess;

@@ -25,16 +25,19 @@ __global__ void csc_count_kernel(const int32_t* __restrict__ indptr, const int32
     atomicAdd(cnt + indices[e], 1);
 }
 
-// csc_dst[csc_ptr[u] + j] = v for the j-th in-edge (v, u); counts return to 0 (ready for the next step)
+// csc_dst[csc_ptr[u] + j] = (v, deg(v)) for the j-th in-edge (v, u): the pull reads the
+// destination and its sampled degree with one 8-B load.  Counts return to 0 (ready for
+// the next step).
 __global__ void csc_fill_kernel(const int32_t* __restrict__ indptr, const int32_t* __restrict__ indices,
                                 const int32_t* __restrict__ n_dst_p, const int32_t* __restrict__ csc_ptr,
-                                int32_t* __restrict__ cnt, int32_t* __restrict__ csc_dst) {
+                                int32_t* __restrict__ cnt, int2* __restrict__ csc_dst) {
   APT_PDL_PROLOGUE();
   const int64_t n = *n_dst_p;
   for (int64_t v = int64_t(blockIdx.x) * blockDim.x + threadIdx.x; v < n; v += int64_t(gridDim.x) * blockDim.x) {
-    for (int e = indptr[v]; e < indptr[v + 1]; ++e) {
+    const int b = indptr[v], e1 = indptr[v + 1];
+    for (int e = b; e < e1; ++e) {
       const int u = indices[e];
-      csc_dst[csc_ptr[u] + atomicSub(cnt + u, 1) - 1] = int32_t(v);
+      csc_dst[csc_ptr[u] + atomicSub(cnt + u, 1) - 1] = make_int2(int32_t(v), e1 - b);
     }
   }
 }
@@ -51,9 +54,43 @@ cudaError_t launch_csc_build(const CscArgs& a, cudaStream_t st) {
   return cudaGetLastError();
 }
 
-// One warp per source row u (VPL float4 vectors per lane): g = sum over in-edges of
-// dZ[v] / deg(v) (correctly rounded per term, reading O5), masked by H[u] > 0.
-template <int VPL>
+// One warp per R source rows u (VPL float4 vectors per lane per row): g = sum over
+// in-edges of dZ[v] / deg(v) (correctly rounded per term, reading O5), masked by
+// H[u] > 0.  Latency design (the layer-1 pull has ~1 in-edge per row, so the kernel is
+// a chain of dependent loads, not a stream): the R rows of a warp are in flight at
+// once; each row's ReLU mask is loaded with its CSC bounds (independent of the edge
+// chain); the in-edges' (v, deg) pairs come with one coalesced 8-B load per lane and
+// are broadcast by shuffles, so a row costs three dependent loads (bounds -> edges ->
+// dZ rows) instead of five.
+// MS = mask source: 0 none, 1 bit mask, 2 fp32 H, 3 bf16 H.  The raw mask words are
+// loaded with the CSC bounds and decoded only after the edge loop (a DRAM-latency H
+// read overlaps the bounds -> edges -> dZ chain instead of stalling it).
+template <int MS> struct MaskRaw { uint32_t w; };
+template <> struct MaskRaw<2> { float4 w; };
+template <> struct MaskRaw<3> { uint2 w; };
+
+template <int MS>
+__device__ __forceinline__ MaskRaw<MS> load_mask(const PullArgs& a, int64_t u, int j) {
+  MaskRaw<MS> m;
+  if constexpr (MS == 0) m.w = 0xFu;
+  if constexpr (MS == 1) m.w = uint32_t(a.mask[u * a.mask_pitch + (j * 4) / 16]) >> ((j * 4) & 15);
+  if constexpr (MS == 2) m.w = __ldg(reinterpret_cast<const float4*>(a.h + u * a.h_pitch + j * 4));
+  if constexpr (MS == 3) m.w = __ldg(reinterpret_cast<const uint2*>(a.hb + u * a.hb_pitch + j * 4));
+  return m;
+}
+__device__ __forceinline__ uint32_t bf16_pos(uint32_t h16) { return (h16 != 0u && !(h16 & 0x8000u)) ? 1u : 0u; }
+template <int MS>
+__device__ __forceinline__ uint32_t decode_mask(const MaskRaw<MS>& m) {
+  if constexpr (MS == 0 || MS == 1) return m.w & 0xFu;
+  if constexpr (MS == 2)
+    return (m.w.x > 0.f ? 1u : 0u) | (m.w.y > 0.f ? 2u : 0u) | (m.w.z > 0.f ? 4u : 0u) | (m.w.w > 0.f ? 8u : 0u);
+  if constexpr (MS == 3)
+    return bf16_pos(m.w.x & 0xFFFFu) | (bf16_pos(m.w.x >> 16) << 1) | (bf16_pos(m.w.y & 0xFFFFu) << 2) |
+           (bf16_pos(m.w.y >> 16) << 3);
+  return 0xFu;
+}
+
+template <int VPL, int R, int MS>
 __global__ void __launch_bounds__(256) pull_bwd_kernel(PullArgs a) {
   APT_PDL_PROLOGUE();
   const int lane = lane_id();
@@ -61,62 +98,86 @@ __global__ void __launch_bounds__(256) pull_bwd_kernel(PullArgs a) {
   const int V = int(ceil_div(a.dim, 4));
   const int64_t nwarps = int64_t(gridDim.x) * (blockDim.x >> 5);
   const int64_t rows_out = a.gb ? std::min<int64_t>(a.max_src, round_up(n, 64)) : n;
-  for (int64_t u = (int64_t(blockIdx.x) * blockDim.x + threadIdx.x) >> 5; u < rows_out; u += nwarps) {
-    float acc[VPL][4];
+  for (int64_t u0 = ((int64_t(blockIdx.x) * blockDim.x + threadIdx.x) >> 5) * R; u0 < rows_out; u0 += nwarps * R) {
+    int e0[R], cnt[R];
+    MaskRaw<MS> mraw[R][VPL];
 #pragma unroll
-    for (int p = 0; p < VPL; ++p) acc[p][0] = acc[p][1] = acc[p][2] = acc[p][3] = 0.f;
-    if (u < n) {
-      const int e0 = a.csc_ptr[u], e1 = a.csc_ptr[u + 1];
-      for (int e = e0; e < e1; ++e) {
-        const int v = a.csc_dst[e];
-        const float fdeg = float(a.indptr[v + 1] - a.indptr[v]);
-        const float r = __frcp_rn(fdeg);
-        const float* zr = a.dz + int64_t(v) * a.dz_pitch;
+    for (int r = 0; r < R; ++r) {
+      const int64_t u = u0 + r;
+      e0[r] = 0; cnt[r] = 0;
+      if (u < n) { e0[r] = a.csc_ptr[u]; cnt[r] = a.csc_ptr[u + 1] - e0[r]; }
 #pragma unroll
-        for (int p = 0; p < VPL; ++p) {
-          const int j = lane + 32 * p;
-          if (j < V) {
-            const float4 z = *reinterpret_cast<const float4*>(zr + j * 4);
-            acc[p][0] += div_rn_rcp(z.x, fdeg, r);
-            acc[p][1] += div_rn_rcp(z.y, fdeg, r);
-            acc[p][2] += div_rn_rcp(z.z, fdeg, r);
-            acc[p][3] += div_rn_rcp(z.w, fdeg, r);
+      for (int p = 0; p < VPL; ++p) {
+        const int j = lane + 32 * p;
+        if (u < n && j < V) mraw[r][p] = load_mask<MS>(a, u, j);
+        else mraw[r][p] = MaskRaw<MS>{};
+      }
+    }
+    float acc[R][VPL][4];
+#pragma unroll
+    for (int r = 0; r < R; ++r)
+#pragma unroll
+      for (int p = 0; p < VPL; ++p) acc[r][p][0] = acc[r][p][1] = acc[r][p][2] = acc[r][p][3] = 0.f;
+    int cmax = cnt[0];
+#pragma unroll
+    for (int r = 1; r < R; ++r) cmax = max(cmax, cnt[r]);
+    for (int c0 = 0; c0 < cmax; c0 += 32) {
+      int2 ed[R];
+#pragma unroll
+      for (int r = 0; r < R; ++r) ed[r] = c0 + lane < cnt[r] ? a.csc_dst[e0[r] + c0 + lane] : make_int2(0, 1);
+      const int m = min(32, cmax - c0);
+      for (int j = 0; j < m; ++j) {
+#pragma unroll
+        for (int r = 0; r < R; ++r) {
+          const int v = __shfl_sync(0xffffffffu, ed[r].x, j);
+          const float fdeg = float(__shfl_sync(0xffffffffu, ed[r].y, j));
+          if (c0 + j >= cnt[r]) continue;
+          const float rc = __frcp_rn(fdeg);
+          const float* zr = a.dz + int64_t(v) * a.dz_pitch;
+#pragma unroll
+          for (int p = 0; p < VPL; ++p) {
+            const int jv = lane + 32 * p;
+            if (jv < V) {
+              const float4 z = *reinterpret_cast<const float4*>(zr + jv * 4);
+              if (a.dz_scaled) {
+                acc[r][p][0] += z.x; acc[r][p][1] += z.y; acc[r][p][2] += z.z; acc[r][p][3] += z.w;
+              } else {
+                acc[r][p][0] += div_rn_rcp(z.x, fdeg, rc);
+                acc[r][p][1] += div_rn_rcp(z.y, fdeg, rc);
+                acc[r][p][2] += div_rn_rcp(z.z, fdeg, rc);
+                acc[r][p][3] += div_rn_rcp(z.w, fdeg, rc);
+              }
+            }
           }
         }
       }
     }
 #pragma unroll
-    for (int p = 0; p < VPL; ++p) {
-      const int j = lane + 32 * p;
-      if (j >= V) continue;
-      float4 g = make_float4(acc[p][0], acc[p][1], acc[p][2], acc[p][3]);
-      if (u < n && a.mask) {
-        const uint32_t mw = uint32_t(a.mask[u * a.mask_pitch + (j * 4) / 16]) >> ((j * 4) & 15);
-        if (!(mw & 1u)) g.x = 0.f;
-        if (!(mw & 2u)) g.y = 0.f;
-        if (!(mw & 4u)) g.z = 0.f;
-        if (!(mw & 8u)) g.w = 0.f;
-      } else if (u < n && a.h) {
-        const float4 h = *reinterpret_cast<const float4*>(a.h + u * a.h_pitch + j * 4);
-        if (!(h.x > 0.f)) g.x = 0.f;
-        if (!(h.y > 0.f)) g.y = 0.f;
-        if (!(h.z > 0.f)) g.z = 0.f;
-        if (!(h.w > 0.f)) g.w = 0.f;
-      }
-      const int c0 = j * 4;
-      if (a.g && u < n) *reinterpret_cast<float4*>(a.g + u * a.g_pitch + c0) = g;
-      if (a.gb) {
-        uint16_t* o = a.gb + u * a.gb_pitch + c0;
-        if (c0 + 4 <= a.dim) {
-          *reinterpret_cast<uint2*>(o) = make_uint2(pack_bf16x2(g.x, g.y), pack_bf16x2(g.z, g.w));
-        } else {
-          const float w[4] = {g.x, g.y, g.z, g.w};
+    for (int r = 0; r < R; ++r) {
+      const int64_t u = u0 + r;
+      if (u >= rows_out) continue;
 #pragma unroll
-          for (int q = 0; q < 4; ++q)
-            if (c0 + q < a.dim) {
-              __nv_bfloat16 hh = __float2bfloat16_rn(w[q]);
-              o[q] = *reinterpret_cast<uint16_t*>(&hh);
-            }
+      for (int p = 0; p < VPL; ++p) {
+        const int j = lane + 32 * p;
+        if (j >= V) continue;
+        const uint32_t kp = (u < n) ? decode_mask<MS>(mraw[r][p]) : 0u;
+        const float4 g = make_float4(kp & 1u ? acc[r][p][0] : 0.f, kp & 2u ? acc[r][p][1] : 0.f,
+                                     kp & 4u ? acc[r][p][2] : 0.f, kp & 8u ? acc[r][p][3] : 0.f);
+        const int c0 = j * 4;
+        if (a.g && u < n) *reinterpret_cast<float4*>(a.g + u * a.g_pitch + c0) = g;
+        if (a.gb) {
+          uint16_t* o = a.gb + u * a.gb_pitch + c0;
+          if (c0 + 4 <= a.dim) {
+            *reinterpret_cast<uint2*>(o) = make_uint2(pack_bf16x2(g.x, g.y), pack_bf16x2(g.z, g.w));
+          } else {
+            const float w[4] = {g.x, g.y, g.z, g.w};
+#pragma unroll
+            for (int q = 0; q < 4; ++q)
+              if (c0 + q < a.dim) {
+                __nv_bfloat16 hh = __float2bfloat16_rn(w[q]);
+                o[q] = *reinterpret_cast<uint16_t*>(&hh);
+              }
+          }
         }
       }
     }
@@ -130,6 +191,7 @@ cudaError_t launch_pull_bwd(const PullArgs& a, cudaStream_t st) {
       b.dim = std::min(512, a.dim - c0);
       b.dz = a.dz + c0;
       if (a.h) b.h = a.h + c0;
+      if (a.hb) b.hb = a.hb + c0;
       if (a.mask) b.mask = a.mask + c0 / 16;
       if (a.g) b.g = a.g + c0;
       if (a.gb) b.gb = a.gb + c0;
@@ -141,10 +203,20 @@ cudaError_t launch_pull_bwd(const PullArgs& a, cudaStream_t st) {
   const int V = int(ceil_div(a.dim, 4));
   if ((a.dz_pitch & 3) || (a.h_pitch & 3) || (a.g && (a.g_pitch & 3)) || (a.gb && (a.gb_pitch & 3)))
     return cudaErrorInvalidValue;
-  const int64_t blocks = std::max<int64_t>(1, std::min<int64_t>(ceil_div(round_up(a.max_src, 64) * 32, 256), 148 * 16));
-  if (V <= 32) launch_pdl(pull_bwd_kernel<1>, dim3(blocks), dim3(256), 0, st, a);
-  else if (V <= 64) launch_pdl(pull_bwd_kernel<2>, dim3(blocks), dim3(256), 0, st, a);
-  else if (V <= 128) launch_pdl(pull_bwd_kernel<4>, dim3(blocks), dim3(256), 0, st, a);
+  constexpr int R = 2;   // rows in flight per warp
+  const int64_t blocks =
+      std::max<int64_t>(1, std::min<int64_t>(ceil_div(ceil_div(round_up(a.max_src, 64), R) * 32, 256), 148 * 16));
+  const int ms = a.mask ? 1 : a.hb ? 3 : a.h ? 2 : 0;
+  auto go = [&](auto vpl) {
+    constexpr int VP = decltype(vpl)::value;
+    if (ms == 0) launch_pdl(pull_bwd_kernel<VP, R, 0>, dim3(blocks), dim3(256), 0, st, a);
+    else if (ms == 1) launch_pdl(pull_bwd_kernel<VP, R, 1>, dim3(blocks), dim3(256), 0, st, a);
+    else if (ms == 2) launch_pdl(pull_bwd_kernel<VP, R, 2>, dim3(blocks), dim3(256), 0, st, a);
+    else launch_pdl(pull_bwd_kernel<VP, R, 3>, dim3(blocks), dim3(256), 0, st, a);
+  };
+  if (V <= 32) go(std::integral_constant<int, 1>{});
+  else if (V <= 64) go(std::integral_constant<int, 2>{});
+  else if (V <= 128) go(std::integral_constant<int, 4>{});
   else return cudaErrorInvalidValue;
   return cudaGetLastError();
 }

@@ -63,6 +63,9 @@ struct RowParams {
   int n_split;              // CTAs share an M tile: CTA b computes columns [(b % n_split) * BN, +BN)
   uint16_t* mask;           // optional ReLU bit mask [M x mask_pitch] (16 columns per word)
   int64_t mask_pitch;
+  const int32_t* row_div;   // optional: divide row m by indptr[m+1] - indptr[m] (RN)
+  uint16_t* Yb;             // optional bf16 output instead of Y (not with routing / accumulation)
+  int64_t yb_pitch;
 };
 
 __global__ void __launch_bounds__(ROW_THREADS, 2)
@@ -95,6 +98,10 @@ __global__ void __launch_bounds__(ROW_THREADS, 2)
     asm volatile("prefetch.tensormap [%0];" ::"l"(reinterpret_cast<uint64_t>(&mapB)) : "memory");
   }
   if (warp == 1) tmem_alloc(tmem_slot, uint32_t(p.tmem_cols));
+  // this CTA's bias slice (zero past N or without bias), read by the epilogue
+  float* sbias = reinterpret_cast<float*>(
+      (reinterpret_cast<uintptr_t>(reinterpret_cast<float*>(tmem_slot + 4) + 8 * 32 * 17) + 15) & ~uintptr_t(15));
+  for (int j = threadIdx.x; j < p.BN; j += blockDim.x) sbias[j] = (p.bias && n0 + j < p.N) ? p.bias[n0 + j] : 0.f;
   fence_before();
   __syncthreads();
   fence_after();
@@ -163,7 +170,10 @@ __global__ void __launch_bounds__(ROW_THREADS, 2)
     // rows is staged in shared memory (row stride 17 floats: conflict-free writes) and
     // written back row-contiguously: 4 lanes cover one 64-B row segment, so a store
     // instruction moves 8 segments instead of 32 scattered 16-B pieces.  Eight
-    // warps keep twice the independent TMEM-load -> store chains in flight.
+    // warps keep twice the independent TMEM-load -> store chains in flight.  The
+    // bias slice sits in shared memory (loaded once per CTA) and the next chunk's TMEM
+    // load is issued before the current chunk is processed, so a chunk's critical path
+    // is shared-memory latency, not a global bias load and a TMEM round trip.
     const int q = warp & 3, h = (warp - 2) >> 2;
     float* stg = reinterpret_cast<float*>(tmem_slot + 4) + (warp - 2) * 32 * 17;
     const int rsub = lane >> 2, cq = (lane & 3) * 4;
@@ -176,25 +186,27 @@ __global__ void __launch_bounds__(ROW_THREADS, 2)
       const int64_t m_own = t * BM + q * 32 + lane;
       float* own = nullptr;
       if (m_own < M) {
-        if (p.out_rank) own = p.out_base[p.out_rank[m_own]] + int64_t(p.out_row[m_own]) * p.y_pitch;
+        if (p.Yb) own = reinterpret_cast<float*>(p.Yb + m_own * p.yb_pitch);   // bf16 row (reading R11)
+        else if (p.out_rank) own = p.out_base[p.out_rank[m_own]] + int64_t(p.out_row[m_own]) * p.y_pitch;
         else own = p.Y + m_own * p.y_pitch;
       }
+      float own_deg = 0.f;
+      if (p.row_div && m_own < M) own_deg = float(p.row_div[m_own + 1] - p.row_div[m_own]);
+      const float own_rdeg = own_deg > 0.f ? __frcp_rn(own_deg) : 0.f;
+      const uint32_t tbase = tmem_base + (uint32_t(q * 32) << 16) + uint32_t(acc * p.BN);
+      uint32_t r[16], rn[16];
+      if (16 * h < p.BN) {
+        tmem_ld16_nowait(tbase + uint32_t(16 * h), r);
+        tmem_wait16(r);
+      }
       for (int c = 16 * h; c < p.BN; c += 32) {
-        uint32_t r[16];
-        tmem_ld16(tmem_base + (uint32_t(q * 32) << 16) + uint32_t(acc * p.BN + c), r);
+        const bool more = c + 32 < p.BN;
+        if (more) tmem_ld16_nowait(tbase + uint32_t(c + 32), rn);
 #pragma unroll
         for (int j = 0; j < 16; ++j) stg[lane * 17 + j] = __uint_as_float(r[j]);
         __syncwarp();
         const int col = n0 + c + cq;
-        float4 bv = make_float4(0.f, 0.f, 0.f, 0.f);
-        if (p.bias) {
-          if (col + 4 <= p.N) bv = *reinterpret_cast<const float4*>(p.bias + col);
-          else {
-            if (col < p.N) bv.x = p.bias[col];
-            if (col + 1 < p.N) bv.y = p.bias[col + 1];
-            if (col + 2 < p.N) bv.z = p.bias[col + 2];
-          }
-        }
+        const float4 bv = *reinterpret_cast<const float4*>(sbias + c + cq);
 #pragma unroll
         for (int it = 0; it < 4; ++it) {
           const int row = it * 8 + rsub;
@@ -202,6 +214,13 @@ __global__ void __launch_bounds__(ROW_THREADS, 2)
           const float* sv = stg + row * 17 + cq;
           float4 v = make_float4(sv[0] + bv.x, sv[1] + bv.y, sv[2] + bv.z, sv[3] + bv.w);
           if (p.relu) { v.x = fmaxf(v.x, 0.f); v.y = fmaxf(v.y, 0.f); v.z = fmaxf(v.z, 0.f); v.w = fmaxf(v.w, 0.f); }
+          if (p.row_div) {   // dZ / deg(v), the same correctly rounded quotient the pull formed per edge
+            const float dg = __shfl_sync(0xffffffffu, own_deg, row), rd = __shfl_sync(0xffffffffu, own_rdeg, row);
+            if (dg > 0.f) {
+              v.x = div_rn_rcp(v.x, dg, rd); v.y = div_rn_rcp(v.y, dg, rd);
+              v.z = div_rn_rcp(v.z, dg, rd); v.w = div_rn_rcp(v.w, dg, rd);
+            }
+          }
           if (p.mask) {   // 16 mask bits of (row, chunk) from the 4 lanes of the row segment
             uint32_t bits = (col < p.N && v.x > 0.f ? 1u : 0u) | (col + 1 < p.N && v.y > 0.f ? 2u : 0u) |
                             (col + 2 < p.N && v.z > 0.f ? 4u : 0u) | (col + 3 < p.N && v.w > 0.f ? 8u : 0u);
@@ -214,6 +233,19 @@ __global__ void __launch_bounds__(ROW_THREADS, 2)
             }
           }
           if (!dst || col >= p.N) continue;
+          if (p.Yb) {
+            uint16_t* db = reinterpret_cast<uint16_t*>(dst) + col;
+            if (col + 4 <= p.N) {
+              *reinterpret_cast<uint2*>(db) = make_uint2(pack_bf16x2(v.x, v.y), pack_bf16x2(v.z, v.w));
+            } else {
+              const float w4[4] = {v.x, v.y, v.z, v.w};
+              for (int qq = 0; qq < 4 && col + qq < p.N; ++qq) {
+                __nv_bfloat16 hh = __float2bfloat16_rn(w4[qq]);
+                db[qq] = *reinterpret_cast<uint16_t*>(&hh);
+              }
+            }
+            continue;
+          }
           if (p.accumulate) {
             if (col + 4 <= p.N) {
               red_add_v4(dst + col, v.x, v.y, v.z, v.w);
@@ -231,6 +263,11 @@ __global__ void __launch_bounds__(ROW_THREADS, 2)
           }
         }
         __syncwarp();
+        if (more) {
+          tmem_wait16(rn);
+#pragma unroll
+          for (int j = 0; j < 16; ++j) r[j] = rn[j];
+        }
       }
       fence_before();
       mbar_arrive(tempty + acc);
@@ -391,6 +428,7 @@ cudaError_t launch_tc_gemm(const TcGemmArgs& a, cudaStream_t st) {
   using namespace tc;
   if (!tc_gemm_supported(a.N, a.K)) return cudaErrorInvalidValue;
   if ((a.z_pitch * 2) % 16 || (a.w_pitch * 2) % 16 || (a.y_pitch * 4) % 16) return cudaErrorInvalidValue;
+  if (a.Yb && ((a.yb_pitch * 2) % 8 || a.out_rank || a.accumulate)) return cudaErrorInvalidValue;
   const int BN_all = int(round_up(a.N, 16));
   const int nkb = int(ceil_div(a.K, BK));
   // few M tiles (small blocks, a requester's own rows): split the columns over CTAs so
@@ -420,7 +458,8 @@ cudaError_t launch_tc_gemm(const TcGemmArgs& a, cudaStream_t st) {
   // loads and MMAs overlap the other's epilogue
   static const int two_cta = [] { const char* v = std::getenv("APT_PROJ_2CTA"); return v ? atoi(v) : 0; }();   // off: measured slower end to end (the overlapped sampling then lands on the backward)
   auto smem_of = [&](int st) {
-    return 1024 + size_t(st) * A_STAGE_BYTES + size_t(nkb) * b_kb_bytes + 16 * 8 + 16 + 8 * 32 * 17 * 4;
+    return 1024 + size_t(st) * A_STAGE_BYTES + size_t(nkb) * b_kb_bytes + 16 * 8 + 16 + 8 * 32 * 17 * 4 +
+           16 + size_t(BN) * 4;
   };
   int stages = STAGES, nacc = 2, per_sm = 1;
   if (two_cta && !a.w_mn && smem_of(2) <= 113 * 1024 && BN <= 256 && tiles * n_split > sm_count()) {
@@ -431,7 +470,8 @@ cudaError_t launch_tc_gemm(const TcGemmArgs& a, cudaStream_t st) {
   int cols = 32;
   while (cols < nacc * BN) cols <<= 1;
   RowParams p{a.M_max, a.M_dev, a.N, BN, nkb, cols, a.w_mn, stages, nacc, b_kb_bytes, a.bias, a.relu, a.Y, a.y_pitch,
-              a.out_base, a.out_rank, a.out_row, a.accumulate, n_split, a.mask, a.mask_pitch};
+              a.out_base, a.out_rank, a.out_row, a.accumulate, n_split, a.mask, a.mask_pitch, a.row_div_indptr,
+              a.Yb, a.yb_pitch};
   const size_t smem = smem_of(stages);   // + epilogue staging
   if (smem > 227 * 1024) return cudaErrorInvalidValue;
   static bool attr_set = false;

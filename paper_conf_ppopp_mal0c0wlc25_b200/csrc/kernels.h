@@ -87,8 +87,9 @@ struct AggArgs {
   // CSR form (upper layers)
   const int32_t* indptr;
   const int32_t* indices;
-  const float* x;              // [n_src x x_pitch] fp32 (CSR form)
+  const float* x;              // [n_src x x_pitch] fp32 (CSR form) ...
   int64_t x_pitch;
+  const uint16_t* xb;          // ... or bf16 rows (bf16 mode's hidden activations, reading R11), pitch x_pitch
   // optional per-edge filter (SNP partial sums): only sources u with part[u] == keep_part
   const int32_t* filt_part;
   int keep_part;
@@ -145,7 +146,7 @@ struct CscArgs {
   int32_t* cnt;        // [max_src], zero on entry and exit
   int32_t* csc_ptr;    // [max_src + 1]
   int32_t* csc_total;  // [1]
-  int32_t* csc_dst;    // [max_edges]
+  int2* csc_dst;       // [max_edges] (v, deg(v)) per in-edge
   int32_t* ws;         // scan workspace, >= 2*ceil(max_src/2048) + 8
   int64_t grid_cap;    // max blocks of the grid-stride kernels (0: default)
 };
@@ -154,7 +155,7 @@ cudaError_t launch_csc_build(const CscArgs& a, cudaStream_t st);
 // G[u] = mask(H[u] > 0) * sum_{(v,u)} dZ[v] / deg(v) over rows u < *n_src; fp32 G and/or
 // bf16 Gb (whose 64-row-block tail is zeroed).
 struct PullArgs {
-  const int32_t* csc_ptr; const int32_t* csc_dst; const int32_t* indptr;
+  const int32_t* csc_ptr; const int2* csc_dst; const int32_t* indptr;
   const float* dz; int64_t dz_pitch;
   const float* h; int64_t h_pitch;        // null: no mask
   const uint16_t* mask; int64_t mask_pitch;   // if set: the ReLU mask as bits (replaces reading h)
@@ -162,6 +163,8 @@ struct PullArgs {
   uint16_t* gb; int64_t gb_pitch;          // may be null
   const int32_t* n_src; int64_t max_src;
   int dim;
+  int dz_scaled;                           // dz rows already divided by deg (tcgen05 epilogue)
+  const uint16_t* hb; int64_t hb_pitch;    // if set: the ReLU mask from bf16 H (bf16 mode, reading R11)
 };
 cudaError_t launch_pull_bwd(const PullArgs& a, cudaStream_t st);
 
@@ -199,6 +202,12 @@ struct TcGemmArgs {
   int w_mn;                            // B stored N-contiguous (dZ = G W uses W [d_out x d_in] as is)
   int accumulate;                      // add into Y with vector reductions (partial sums of SNP / NFP)
   uint16_t* mask; int64_t mask_pitch;  // optional: bit c%16 of mask[m][c/16] = (Y[m][c] > 0) (ReLU mask for the backward)
+  // optional: row m is divided (RN) by its block degree indptr[m+1] - indptr[m] (the
+  // mean's backward pre-scales dZ / deg once per row instead of once per in-edge)
+  const int32_t* row_div_indptr;
+  // optional bf16 output instead of Y (hidden activations in bf16 mode, reading R11):
+  // row m -> Yb + m * yb_pitch (not with routing / accumulation)
+  uint16_t* Yb; int64_t yb_pitch;
 };
 int tc_gemm_supported(int N, int K);
 cudaError_t launch_tc_gemm(const TcGemmArgs& a, cudaStream_t st);
@@ -220,7 +229,8 @@ cudaError_t launch_tc_wgrad(const TcWgradArgs& a, cudaStream_t st);
 // Gb = bf16(G * (H > 0)) over rows < n (relu != 0) or bf16(G); rows in
 // [n, round_up(n, 64)) of Gb are zeroed (tail of the tcgen05 row blocks).
 cudaError_t launch_grad_finish(const float* G, int64_t g_pitch, const float* H, int64_t h_pitch, int dim, int relu,
-                               uint16_t* Gb, int64_t gb_pitch, const int32_t* n_dev, int64_t max_n, cudaStream_t st);
+                               uint16_t* Gb, int64_t gb_pitch, const int32_t* n_dev, int64_t max_n, cudaStream_t st,
+                               const uint16_t* Hb = nullptr, int64_t hb_pitch = 0);   // Hb: mask from bf16 H
 
 // ---------------------------------------------------------------- misc.cu
 cudaError_t launch_ce_loss(const float* logits, int64_t pitch, int n_classes, const int32_t* seeds,

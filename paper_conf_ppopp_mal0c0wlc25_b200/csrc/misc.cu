@@ -83,7 +83,8 @@ cudaError_t launch_relu_bwd(float* g, const float* h, int64_t pitch, int dim, co
 // One thread per 4 columns (16-B G / H loads, 8-B Gb stores).
 __global__ void grad_finish_kernel(const float* __restrict__ G, int64_t gp, const float* __restrict__ H, int64_t hp,
                                    int dim, int relu, uint16_t* __restrict__ Gb, int64_t gbp,
-                                   const int32_t* __restrict__ n_p, int64_t max_n) {
+                                   const int32_t* __restrict__ n_p, int64_t max_n,
+                                   const uint16_t* __restrict__ Hb, int64_t hbp) {
   APT_PDL_PROLOGUE();
   const int64_t n = *n_p;
   const int64_t rows = std::min<int64_t>(max_n, round_up(n, 64));
@@ -98,7 +99,13 @@ __global__ void grad_finish_kernel(const float* __restrict__ G, int64_t gp, cons
       continue;
     }
     float4 g = *reinterpret_cast<const float4*>(G + r * gp + c);
-    if (relu) {
+    if (relu && Hb) {   // bf16 H: positive <=> sign bit clear and not zero
+      const uint16_t* hb = Hb + r * hbp + c;
+      if (!(hb[0] != 0 && !(hb[0] & 0x8000u))) g.x = 0.f;
+      if (!(c + 1 < dim && hb[1] != 0 && !(hb[1] & 0x8000u))) g.y = 0.f;
+      if (!(c + 2 < dim && hb[2] != 0 && !(hb[2] & 0x8000u))) g.z = 0.f;
+      if (!(c + 3 < dim && hb[3] != 0 && !(hb[3] & 0x8000u))) g.w = 0.f;
+    } else if (relu) {
       const float4 h = *reinterpret_cast<const float4*>(H + r * hp + c);
       if (!(h.x > 0.f)) g.x = 0.f;
       if (!(h.y > 0.f)) g.y = 0.f;
@@ -118,10 +125,11 @@ __global__ void grad_finish_kernel(const float* __restrict__ G, int64_t gp, cons
 }
 
 cudaError_t launch_grad_finish(const float* G, int64_t g_pitch, const float* H, int64_t h_pitch, int dim, int relu,
-                               uint16_t* Gb, int64_t gb_pitch, const int32_t* n_dev, int64_t max_n, cudaStream_t st) {
+                               uint16_t* Gb, int64_t gb_pitch, const int32_t* n_dev, int64_t max_n, cudaStream_t st,
+                               const uint16_t* Hb, int64_t hb_pitch) {
   if ((g_pitch & 3) || (h_pitch & 3)) return cudaErrorInvalidValue;
   launch_pdl(grad_finish_kernel, dim3(grid_of(max_n * ceil_div(dim, 4))), dim3(256), 0, st, G, g_pitch, H, h_pitch, dim, relu, Gb,
-                                                                          gb_pitch, n_dev, max_n);
+                                                                          gb_pitch, n_dev, max_n, Hb, hb_pitch);
   return cudaGetLastError();
 }
 

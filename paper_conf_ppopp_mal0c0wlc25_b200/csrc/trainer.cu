@@ -151,6 +151,7 @@ apt_status project(apt_trainer* t, const Layer& L, const void* Zb, const float* 
     TcGemmArgs a{static_cast<const uint16_t*>(Zb), z_pitch_b, Wb, L.wb_pitch, max_rows, n_rows, L.d_out, K,
                  bias, relu, Y, L.h_pitch, out_base, out_rank, out_row, 0};
     if (relu && L.Mk && !out_rank) { a.mask = L.Mk; a.mask_pitch = L.mk_pitch; }   // ReLU bits for the backward
+    if (Y == L.H && L.Hb && !out_rank) { a.Yb = L.Hb; a.yb_pitch = L.hb_pitch; }   // R11: bf16 only
     CK(c, launch_tc_gemm(a, c->stream));
   } else {
     if (out_rank) return set_err(c, APT_E_UNSUPPORTED, "routed epilogue needs the tcgen05 path");
@@ -160,8 +161,25 @@ apt_status project(apt_trainer* t, const Layer& L, const void* Zb, const float* 
     a.sak = 1; a.sbk = 1;
     a.C = Y; a.ldc = L.h_pitch; a.bias = bias; a.M_dev = n_rows; a.M = max_rows; a.N = L.d_out; a.K = K; a.relu = relu;
     CK(c, launch_simt_gemm(a, c->stream));
+    if (Y == L.H && L.Hb) {   // R11: the bf16 copy the next layer and the backward read
+      CK(c, launch_to_bf16(L.H, L.h_pitch, L.Hb, L.hb_pitch, L.d_out, n_rows, max_rows, c->stream));
+      c->launches++;
+    }
   }
   c->launches++;
+  return APT_OK;
+}
+
+// Reading R11: layer-1 producers that write fp32 H (the strategies' Reshuffle, GAT, the
+// fused opt-in kernel) hand the next layer its bf16 copy.
+apt_status hidden1_to_bf16(apt_trainer* t) {
+  apt_ctx* c = t->ctx;
+  for (auto& rs : t->R) {
+    Layer& L = rs.L[0];
+    if (!L.Hb) continue;
+    CK(c, launch_to_bf16(L.H, L.h_pitch, L.Hb, L.hb_pitch, L.d_out, L.n_rows, L.max_rows, c->stream));
+    c->launches++;
+  }
   return APT_OK;
 }
 
@@ -285,7 +303,7 @@ apt_status apt_trainer_create(apt_ctx* c, const apt_graph* g, const apt_fstore* 
           hp.indices = A.alloc<int32_t>(maxF * hp.k, false);
           hp.csc_cnt = A.alloc<int32_t>(hp.max_src, true);
           hp.csc_ptr = A.alloc<int32_t>(hp.max_src + 1, true);
-          hp.csc_dst = A.alloc<int32_t>(maxF * hp.k, false);
+          hp.csc_dst = A.alloc<int2>(maxF * hp.k, false);
           hp.csc_ws = A.alloc<int32_t>(2 * ceil_div(hp.max_src, 2048) + 8, false);
         }
         dst = hp.src;
@@ -312,6 +330,10 @@ apt_status apt_trainer_create(apt_ctx* c, const apt_graph* g, const apt_fstore* 
       if (m->dtype == APT_BF16) L.Zb = A.alloc<uint16_t>(L.max_rows * L.zb_pitch, true);
       else L.Zf = A.alloc<float>(L.max_rows * L.zf_pitch, true);
       L.H = A.alloc<float>(L.max_rows * L.h_pitch, true);
+      if (m->dtype == APT_BF16 && l < K) {   // reading R11: hidden activations stored in bf16
+        L.hb_pitch = round_up(L.d_out, 8);
+        L.Hb = A.alloc<uint16_t>(L.max_rows * L.hb_pitch, true);
+      }
       L.G = A.alloc<float>(L.max_rows * L.h_pitch, true);
       if (m->dtype == APT_BF16) L.Gb = A.alloc<uint16_t>(L.max_rows * L.gb_pitch, true);
       // (ReLU bit masks, L.Mk, are supported by the epilogue and the pull kernel but not
@@ -614,6 +636,10 @@ apt_status layer1_fwd_gdp(apt_trainer* t, RankState& rs, bool time_it) {
       if (time_it) CK(c, record_ev(t, 7));
       c->launches++;
       t->fused_l1 = true;
+      if (L.Hb) {
+        CK(c, launch_to_bf16(L.H, L.h_pitch, L.Hb, L.hb_pitch, L.d_out, L.n_rows, L.max_rows, c->stream));
+        c->launches++;
+      }
       return APT_OK;
     }
     if (e != cudaErrorNotSupported) return check_cuda(c, e, "launch_sage_l1");
@@ -642,6 +668,7 @@ apt_status upper_fwd_loss(apt_trainer* t, RankState& rs) {
     const Hop& hp = rs.hops[t->K - l];
     AggArgs a{};
     a.indptr = hp.indptr; a.indices = hp.indices; a.x = P.H; a.x_pitch = P.h_pitch;
+    if (P.Hb) { a.x = nullptr; a.xb = P.Hb; a.x_pitch = P.hb_pitch; }   // R11
     a.n_dst = hp.n_dst; a.max_dst = hp.max_dst; a.dim = L.d_in;
     if (t->m.dtype == APT_BF16) { a.z_bf16 = L.Zb; a.z_bf16_pitch = L.zb_pitch; a.z_ones = 1; }
     // fp32 Z is kept in both modes for the upper layers' weight gradient in fp32 mode
@@ -675,11 +702,14 @@ apt_status upper_bwd(apt_trainer* t, RankState& rs) {
     apt_status s = weight_grad(t, L, L.G, L.h_pitch, bf ? static_cast<const void*>(L.Zb) : L.Zf, bf,
                                bf ? L.zb_pitch : L.zf_pitch, L.n_rows, L.max_rows, L.d_in, L.dW, L.db, L.d_in, c->side);
     if (s != APT_OK) return s;
+    int dz_scaled = 0;
     // dZ = G W  (bf16 mode: tcgen05 with the bf16 weights of the forward, W read N-major as stored)
     if (bf && tc_gemm_supported(L.d_in, L.d_out)) {
       TcGemmArgs g{L.Gb, L.gb_pitch, L.Wb, L.wb_pitch, L.max_rows, L.n_rows, L.d_in, L.d_out, nullptr, 0,
                    L.dZ, L.zf_pitch, nullptr, nullptr, nullptr, 1};
+      g.row_div_indptr = hp.indptr;   // dZ / deg once per row (the pull then only sums)
       CK(c, launch_tc_gemm(g, c->stream));
+      dz_scaled = 1;
     } else {
       SimtGemmArgs a{};
       if (bf) { a.A = L.Gb; a.a_t = kBF16; a.sam = L.gb_pitch; }   // bf16 mode: only Gb exists
@@ -699,7 +729,9 @@ apt_status upper_bwd(apt_trainer* t, RankState& rs) {
     const bool l1_local = l - 1 > 1 || t->world == 1 || t->s == APT_GDP;
     const uint16_t* mk = (bf && P.Mk && l1_local && tc_gemm_supported(P.d_out, P.d_in)) ? P.Mk : nullptr;
     PullArgs pa{hp.csc_ptr, hp.csc_dst, hp.indptr, L.dZ, L.zf_pitch, P.H, P.h_pitch, mk, P.mk_pitch,
-                bf ? nullptr : P.G, P.h_pitch, bf ? P.Gb : nullptr, P.gb_pitch, hp.counts, P.max_rows, L.d_in};
+                bf ? nullptr : P.G, P.h_pitch, bf ? P.Gb : nullptr, P.gb_pitch, hp.counts, P.max_rows, L.d_in,
+                dz_scaled};
+    if (P.Hb && !mk) { pa.h = nullptr; pa.hb = P.Hb; pa.hb_pitch = P.hb_pitch; }   // R11: mask from bf16 H
     CK(c, launch_pull_bwd(pa, c->stream));
     c->launches += 2;
   }
@@ -840,6 +872,7 @@ apt_status compute_body(apt_trainer* t, int update) {
   CK(c, record_ev(t, 1));
   if (t->gat_heads) {
     apt_status s = gat_layer1_fwd(t, true);
+    if (s == APT_OK) s = hidden1_to_bf16(t);
     if (s != APT_OK) return s;
   } else if (gdp) {
     bool first = true;
@@ -850,6 +883,7 @@ apt_status compute_body(apt_trainer* t, int update) {
     }
   } else {
     apt_status s = layer1_fwd_strategy(t);
+    if (s == APT_OK) s = hidden1_to_bf16(t);
     if (s != APT_OK) return s;
   }
   if (t->deferred_fork) {   // pipelined: the next step's sampling branch forks here
@@ -916,7 +950,8 @@ apt_status apt_layer_fwd(apt_trainer* t, int64_t step) {
   activate(t, 0);
   apt_status s = APT_OK;
   if (t->gat_heads) {
-    return gat_layer1_fwd(t, false);
+    s = gat_layer1_fwd(t, false);
+    return s == APT_OK ? hidden1_to_bf16(t) : s;
   } else if (t->world == 1 || t->s == APT_GDP) {
     bool first = true;
     for (auto& rs : t->R) {
@@ -926,6 +961,7 @@ apt_status apt_layer_fwd(apt_trainer* t, int64_t step) {
     }
   } else {
     s = layer1_fwd_strategy(t);
+    if (s == APT_OK) s = hidden1_to_bf16(t);
     if (s != APT_OK) return s;
   }
   return APT_OK;
@@ -948,7 +984,7 @@ apt_status apt_layer_bwd(apt_trainer* t, const float* const* dh1, int64_t pitch)
                                                                              L.n_rows);
     CK(c, cudaGetLastError());
     if (bf) CK(c, launch_grad_finish(L.G, L.h_pitch, L.H, L.h_pitch, L.d_out, relu, L.Gb, L.gb_pitch, L.n_rows,
-                                     L.max_rows, c->stream));
+                                     L.max_rows, c->stream, L.Hb, L.hb_pitch));
     else if (relu) CK(c, launch_relu_bwd(L.G, L.H, L.h_pitch, L.d_out, L.n_rows, L.max_rows, c->stream));
     CK(c, cudaMemsetAsync(L.dW, 0, sizeof(float) * grad_floats_l1(t), c->stream));
     c->launches++;
@@ -1300,7 +1336,11 @@ apt_status apt_trainer_read(apt_trainer* t, int rank, int what, int layer, void*
       if (L.Zb) return copy_rows(L.Zb, nr, L.d_in, L.zb_pitch, 2, true);
       return copy_rows(L.Zf, nr, L.d_in, L.zf_pitch, 4, false);
     }
-    case 3: { const Layer& L = rs->L[layer - 1]; return copy_rows(L.H, count(L.n_rows), L.d_out, L.h_pitch, 4, false); }
+    case 3: {   // bf16 mode, hidden layers: the stored bf16 activation (reading R11)
+      const Layer& L = rs->L[layer - 1];
+      if (L.Hb) return copy_rows(L.Hb, count(L.n_rows), L.d_out, L.hb_pitch, 2, true);
+      return copy_rows(L.H, count(L.n_rows), L.d_out, L.h_pitch, 4, false);
+    }
     case 4: {
       const Layer& L = rs->L[layer - 1];
       if (layer == 1 && rs->x.dW1s) {   // NFP: concatenate the column-owned slices of the hosted ranks

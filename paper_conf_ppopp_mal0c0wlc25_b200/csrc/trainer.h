@@ -24,7 +24,7 @@ struct Hop {
   // transpose of the block (upper hops only): in-edges of every local source
   int32_t* csc_cnt = nullptr;       // [max_src] (zero between uses)
   int32_t* csc_ptr = nullptr;       // [max_src + 1]
-  int32_t* csc_dst = nullptr;       // [max_dst * k]
+  int2* csc_dst = nullptr;          // [max_dst * k]
   int32_t* csc_ws = nullptr;        // scan workspace
 };
 
@@ -36,6 +36,8 @@ struct Layer {
   float* Zf = nullptr;              // [max_rows x zf_pitch] (fp32 mode)
   uint16_t* Zb = nullptr;           // [max_rows x zb_pitch] (bf16 mode)
   float* H = nullptr;               // post-activation (or logits)
+  uint16_t* Hb = nullptr;           // bf16 mode, hidden layers: the activation as the next layer and the
+  int64_t hb_pitch = 0;             //   backward read it (reading R11); GDP projections write only Hb
   float* G = nullptr;               // dL/dpre
   uint16_t* Gb = nullptr;           // bf16 copy of G (tcgen05 backward, bf16 mode)
   uint16_t* Mk = nullptr;           // ReLU mask bits of H (bf16 mode, hidden layers) [max_rows x mk_pitch]

@@ -192,6 +192,39 @@ def test_forward_matches_explicit_tree_recursion(tiny_graph, tiny_cfg):
         assert np.allclose(cache["logits"][i], h_of(int(s), K), rtol=1e-12, atol=1e-12)
 
 
+def test_bf16_forward_matches_tree_recursion_with_torch_rounding(tiny_graph, tiny_cfg):
+    """bf16 mode's rounding points (O5, reading R11) by an independent recursion: the
+    mean in fp64 -> fp32 -> bf16, W in bf16, hidden activations rounded to bf16 after
+    bias + ReLU, every rounding done by torch's bfloat16 conversion."""
+    import torch
+
+    def rb(x):
+        return torch.tensor(np.asarray(x, np.float64)).float().bfloat16().double().numpy()
+
+    cfg, seeds, blocks, params, _ = _tiny_setup(tiny_graph, tiny_cfg, 6, dict(dim=8, hidden=5, n_classes=3))
+    K = len(blocks)
+    nbrs = [dict() for _ in range(K)]
+    for h, blk in enumerate(blocks):
+        for i, v in enumerate(blk.dst):
+            nbrs[h][int(v)] = [int(u) for u in blk.nbr[i * blk.k:i * blk.k + blk.cnt[i]]]
+
+    def h_of(v, layer):
+        if layer == 0:
+            return oracle.features(cfg.feat_seed, np.array([v]), cfg.dim)[0]
+        us = nbrs[K - layer][v]
+        z = np.mean([h_of(u, layer - 1) for u in us], axis=0) if us else np.zeros(
+            cfg.dim if layer == 1 else cfg.hidden)
+        W, b = params[layer - 1]
+        pre = rb(W) @ rb(z) + b
+        return rb(np.maximum(pre, 0)) if layer < K else pre
+
+    cache = model.forward(blocks, cfg.feat_seed, cfg.dim, params, "bf16")
+    for i, s in enumerate(seeds):
+        assert np.allclose(cache["logits"][i], h_of(int(s), K), rtol=1e-12, atol=1e-12)
+    for h in cache["h"][:-1]:                    # hidden activations are bf16 values
+        assert np.array_equal(rb(h), h)
+
+
 def test_ce_loss_matches_torch(tiny_graph, tiny_cfg):
     import torch
     rng = np.random.default_rng(3)
