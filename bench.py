@@ -52,6 +52,8 @@ def parse():
     ap.add_argument("--strategy", default="GDP", choices=list(STRATS))
     ap.add_argument("--dtype", default="bf16", choices=["bf16", "f32"])
     ap.add_argument("--no-graph", action="store_true", help="eager launches instead of CUDA-graph replay")
+    ap.add_argument("--no-pipeline", action="store_true",
+                    help="sample each step inside it instead of overlapping the next step's sampling (A/B)")
     ap.add_argument("--no-cpu-baseline", action="store_true")
     ap.add_argument("--cpu-steps", type=int, default=3, help="oracle steps for cpu_baseline")
     ap.add_argument("--e2e-steps", type=int, default=10)
@@ -279,6 +281,8 @@ def run_apt(args, cfg):
     tr.set_params(aptgen.weights(cfg))
     tr.set_epoch(train, 0)
     tr.use_graph(not args.no_graph)
+    if args.no_pipeline:
+        tr.set_pipeline(False)
     spe = tr.steps_per_epoch()
 
     flush = torch.empty(256 << 20, dtype=torch.uint8, device="cuda")   # 256 MB > 126 MB L2
@@ -391,7 +395,7 @@ def run_apt(args, cfg):
         "ms_per_step_pct": pct,
         "config": dict(workload_config(cfg), strategy=args.strategy, parallelism=f"{args.strategy.lower()}{world}",
                        global_batch=B, l2="flushed between timed steps (256 MB write); inputs also > L2",
-                       cuda_graph=not args.no_graph),
+                       cuda_graph=not args.no_graph, pipelined_sampling=not args.no_pipeline),
         "e2e": {"value": B / e2e_s, "unit": "seeds/s", "h2d_bytes_per_step": h2d, "d2h_bytes_per_step": 4,
                 "timing": "host wall clock per call of apt_trainer_step_host_pipelined (syncs), max over ranks"},
         "gpu_launches": int(launches),
@@ -409,6 +413,12 @@ def run_apt(args, cfg):
     }
     if rank == 0 and world == 1 and not args.no_planner:
         out["planner"] = planner_report(A, g, cfg, train, labels, args, stream, ms_local)
+        # the workload's access skew next to the paper's Table 3 (reading R12)
+        n_acc = min(spe, 64)
+        out["access_skew"] = {"steps": n_acc, "buckets": ["<1%", "1-5%", "5-10%", "10-20%", "20-50%", "50-100%"],
+                              "table": skew_table(tr.access_counts(n_acc)),
+                              "paper_table3": {"PS": [0.501, 0.348, 0.088, 0.047, 0.017, 0.0],
+                                               "FS": [0.177, 0.294, 0.191, 0.188, 0.135, 0.016]}}
     if rank == 0 and world == 1 and not args.no_cpu_baseline:
         times, nseeds = oracle_steps(cfg, g, train, labels, args.cpu_steps, 1)
         out["cpu_baseline"] = {"value": nseeds / sum(times), "unit": "seeds/s", "cores": 1, "kind": "oracle",
@@ -509,6 +519,19 @@ def layer1_bytes(ctx, gr, tr, cfg, rank, step, bf):
         n += v.n_dst * cfg.dim * bf * (GAT_HEADS - 1) + v.n_edges * GAT_HEADS * 4
     b.close()
     return n
+
+
+def skew_table(counts, edges=(0.01, 0.05, 0.10, 0.20, 0.50, 1.0)):
+    """Table 3's layout: nodes ranked by access count, share of all accesses
+    per rank bucket."""
+    c = np.sort(np.asarray(counts, np.int64))[::-1]
+    total = max(1, int(c.sum()))
+    out, lo = [], 0
+    for e in edges:
+        hi = int(round(e * len(c)))
+        out.append(float(c[lo:hi].sum()) / total)
+        lo = hi
+    return out
 
 
 def step_phase_bytes(ctx, gr, g, tr, cfg, rank, step, bf):

@@ -320,6 +320,17 @@ apt_status apt_trainer_agg_bytes(apt_trainer* t, double* bytes);
  * runs Permute+Shuffle of every strategy on the shared samples (no feature
  * loading, no training), counts volumes and times T_build.  Syncs.          */
 apt_status apt_dryrun(apt_trainer* t, int64_t n_steps, apt_plan_stats* out);
+/* Node access frequencies (Table 3; reading R12): counts_host[u]
+ * (host int32 [n], caller-owned, overwritten) = number of (step, requester)
+ * pairs of the first n_steps global steps of the current epoch (GDP seed split)
+ * whose layer-1 block has u as a source, i.e. how often u's input row is loaded.
+ * Same sampler as the step (bit-identical blocks).  Syncs.                   */
+apt_status apt_access_counts(apt_trainer* t, int64_t n_steps, int32_t* counts_host);
+/* Hot list of the excess cache: the k ids with the largest
+ * counts[] (host int32 [n]), descending, ties by ascending id, into ids_out
+ * (host int64 [k], caller-owned).  Pure host arithmetic; APT_E_INVALID if
+ * k > n or a pointer is NULL.                                               */
+apt_status apt_hot_rows(const int32_t* counts, int64_t n, int64_t k, int64_t* ids_out);
 /* Bandwidth trials of the exchange operators: each operator this
  * process can run is timed at two message sizes and fitted to alpha + bytes/beta
  * (local HBM row gather, pinned-host read); NVLink operators take the pool's

@@ -245,3 +245,36 @@ def predict(per_strategy_stats, alpha, beta, t_build):
         pred.append(worst)
     pick = int(np.argmin(pred))
     return pred, pick
+
+
+def access_counts(graph, train, fanouts, sample_seed, epoch, C, B, n_steps):
+    """Node access frequencies (Table 3; reading R12): counts[u] =
+    number of (step, rank) pairs among the first n_steps global steps of the epoch, GDP
+    seed split, whose layer-1 block reads u's input row, i.e. u is the source of at
+    least one sampled layer-1 edge (the dst prefix is not loaded unless it is also a
+    sampled neighbour)."""
+    from . import epoch_perm, global_batch, sample_blocks
+    perm = epoch_perm(train, sample_seed, epoch)
+    counts = np.zeros(graph.n, np.int64)
+    for t in range(n_steps):
+        gb = global_batch(perm, t, C, B)
+        for seeds in assign_seeds("GDP", gb, None, C, B):
+            if len(seeds) == 0:
+                continue
+            blk = sample_blocks(graph, seeds, fanouts, sample_seed, t)[-1]
+            counts[np.unique(blk.src[blk.indices])] += 1
+    return counts
+
+
+def skew_table(counts, edges=(0.01, 0.05, 0.10, 0.20, 0.50, 1.0)):
+    """Table 3's access ratios: rank nodes by access count (descending) and report the
+    share of all accesses that falls in each rank bucket (<1%, 1-5%, ..., 50-100%)."""
+    c = np.sort(np.asarray(counts, np.int64))[::-1]
+    total = max(1, int(c.sum()))
+    n = len(c)
+    out, lo = [], 0
+    for e in edges:
+        hi = int(round(e * n))
+        out.append(float(c[lo:hi].sum()) / total)
+        lo = hi
+    return out

@@ -117,7 +117,7 @@ def lib():
             "apt_trainer_use_graph": [vp, i32], "apt_trainer_set_pipeline": [vp, i32], "apt_trainer_read": [vp, i32, i32, i32, vp, i64, vp, vp],
             "apt_trainer_phase_ms": [vp, vp, i32], "apt_trainer_agg_bytes": [vp, vp],
             "apt_partition": [i64, i64, vp, vp, i32, i32, u64, vp, vp],
-            "apt_dryrun": [vp, i64, vp], "apt_layer_fwd": [vp, i64], "apt_layer_bwd": [vp, vp, i64], "apt_profile_links": [vp, vp], "apt_select_strategy": [vp, vp, vp, vp],
+            "apt_dryrun": [vp, i64, vp], "apt_access_counts": [vp, i64, vp], "apt_hot_rows": [vp, i64, i64, vp], "apt_layer_fwd": [vp, i64], "apt_layer_bwd": [vp, vp, i64], "apt_profile_links": [vp, vp], "apt_select_strategy": [vp, vp, vp, vp],
         }
         for name, args in sig.items():
             f = getattr(L, name)
@@ -392,6 +392,12 @@ class Trainer(Handle):
         arr = (C.c_void_p * len(dh1_list))(*[_ptr(x) for x in dh1_list])
         self.ctx.ck(lib().apt_layer_bwd(self.h, arr, pitch))
 
+    def access_counts(self, n_steps):
+        """apt_access_counts: per-node input-row loads over the first n_steps steps (Table 3)."""
+        out = np.zeros(len(self._labels), np.int32)   # labels are per node
+        self.ctx.ck(lib().apt_access_counts(self.h, n_steps, out.ctypes.data))
+        return out
+
     def dryrun(self, n_steps):
         st = PlanStats()
         self.ctx.ck(lib().apt_dryrun(self.h, n_steps, C.byref(st)))
@@ -418,6 +424,14 @@ def partition(indptr, indices, n_parts, method="ldg", seed=0):
     check(lib().apt_partition(n, int(indptr[-1]), indptr.ctypes.data, indices.ctypes.data, n_parts,
                               PARTITION[method], seed, part.ctypes.data, C.byref(cut)))
     return part, cut.value
+
+
+def hot_rows(counts, k):
+    """apt_hot_rows: the k most-accessed node ids, descending count, ties by id."""
+    counts = np.ascontiguousarray(counts, np.int32)
+    out = np.empty(k, np.int64)
+    check(lib().apt_hot_rows(counts.ctypes.data, len(counts), k, out.ctypes.data))
+    return out
 
 
 def select_strategy(stats: PlanStats, bw: BwProfile):

@@ -150,28 +150,33 @@ __global__ void dry_set_step_kernel(uint64_t* p, uint64_t v) {
 
 using namespace apt;
 
-extern "C" apt_status apt_dryrun(apt_trainer* t, int64_t n_steps, apt_plan_stats* out) {
-  if (!t || !out || n_steps < 1) return set_err(t ? t->ctx : nullptr, APT_E_INVALID, "apt_dryrun: bad arguments");
-  if (!t->perm) return set_err(t->ctx, APT_E_STATE, "apt_dryrun: call apt_trainer_set_epoch first");
-  apt_ctx* c = t->ctx;
-  const int C = t->world, K = t->K;
-  const apt_graph* g = t->g;
-  n_steps = std::min<int64_t>(n_steps, t->steps_per_epoch);
+namespace {
+// The dry run's sampler: seed selection + K hops of sampling/compaction for one
+// (rank, step) of the current epoch into its own buffers (no feature loading, no
+// training).  Shared by apt_dryrun and apt_access_counts.
+struct DrySampler {
+  apt_trainer* t;
   Arena A;
-  const int64_t n_words = ceil_div(g->n, 32);
-  // sampler state sized for the largest seed set (SNP/DNP: up to C*B on one rank)
-  const int64_t B0 = int64_t(C) * t->m.batch;
-  int32_t* seeds = A.alloc<int32_t>(B0, false);
-  int32_t* small = A.alloc<int32_t>(16, true);
-  uint32_t* dst_bm = A.alloc<uint32_t>(n_words, true);
-  uint32_t* new_bm = A.alloc<uint32_t>(n_words, true);
-  int32_t* pos = A.alloc<int32_t>(g->n, false);
-  int32_t* partials = A.alloc<int32_t>(2 * ceil_div(n_words, 2048) + 8, false);
-  uint64_t* step_dev = A.alloc<uint64_t>(1, true);
-  uint32_t* own_bm = A.alloc<uint32_t>(n_words * C, true);        // one bitmap per owner / block
-  DryCounters* dc = A.alloc<DryCounters>(4, true);                 // per strategy
-  std::vector<Hop> hops(K);
-  {
+  int64_t n_words = 0;
+  int32_t *seeds = nullptr, *small = nullptr, *pos = nullptr, *partials = nullptr;
+  uint32_t *dst_bm = nullptr, *new_bm = nullptr;
+  uint64_t* step_dev = nullptr;
+  std::vector<Hop> hops;
+  bool init(apt_trainer* tr) {
+    t = tr;
+    const int C = t->world, K = t->K;
+    const apt_graph* g = t->g;
+    n_words = ceil_div(g->n, 32);
+    // sampler state sized for the largest seed set (SNP/DNP: up to C*B on one rank)
+    const int64_t B0 = int64_t(C) * t->m.batch;
+    seeds = A.alloc<int32_t>(B0, false);
+    small = A.alloc<int32_t>(16, true);
+    dst_bm = A.alloc<uint32_t>(n_words, true);
+    new_bm = A.alloc<uint32_t>(n_words, true);
+    pos = A.alloc<int32_t>(g->n, false);
+    partials = A.alloc<int32_t>(2 * ceil_div(n_words, 2048) + 8, false);
+    step_dev = A.alloc<uint64_t>(1, true);
+    hops.resize(K);
     int64_t maxF = B0;
     const int32_t* dst = seeds;
     const int32_t* n_dst = small;
@@ -195,8 +200,49 @@ extern "C" apt_status apt_dryrun(apt_trainer* t, int64_t n_steps, apt_plan_stats
       n_dst = hp.counts;
       maxF = hp.max_src;
     }
+    return seeds && step_dev && hops[K - 1].nbr && (K == 1 || hops[K - 2].indices);
   }
-  if (!own_bm || !dc || !hops[K - 1].nbr) return set_err(c, APT_E_OOM, "apt_dryrun: out of device memory");
+  void set_step(int64_t st, cudaStream_t s) { dry_set_step_kernel<<<1, 1, 0, s>>>(step_dev, uint64_t(st)); }
+  // rank r's seeds of the current step (by_part: its partition's seeds, SNP/DNP) and its blocks
+  apt_status sample(int r, bool by_part) {
+    apt_ctx* c = t->ctx;
+    const int C = t->world, K = t->K;
+    const apt_graph* g = t->g;
+    SeedArgs sa{t->perm, t->n_train, step_dev, t->steps_per_epoch, C, r, t->m.batch, by_part ? 1 : 0, g->part,
+                seeds, small, small + 1};
+    CK(c, launch_select_seeds(sa, c->stream));
+    for (int h = 0; h < K; ++h) {
+      Hop& hp = hops[h];
+      SampleArgs sm{g->indptr, g->indices, hp.dst, hp.n_dst, hp.max_dst, hp.k,
+                    philox_key(t->m.sample_seed, kDomSample), step_dev, h, hp.cnt, hp.nbr};
+      CK(c, launch_sample(sm, c->stream));
+      if (h + 1 < K) {
+        CompactArgs ca{hp.dst, hp.n_dst, hp.max_dst, hp.cnt, hp.nbr, hp.k, dst_bm, new_bm, n_words, pos, hp.src,
+                       hp.counts, hp.indptr, hp.indices, hp.counts + 1, partials, hp.part2};
+        CK(c, launch_compact(ca, c->stream));
+      }
+    }
+    c->launches += 1 + 4 * K;
+    return APT_OK;
+  }
+};
+}  // namespace
+
+extern "C" apt_status apt_dryrun(apt_trainer* t, int64_t n_steps, apt_plan_stats* out) {
+  if (!t || !out || n_steps < 1) return set_err(t ? t->ctx : nullptr, APT_E_INVALID, "apt_dryrun: bad arguments");
+  if (!t->perm) return set_err(t->ctx, APT_E_STATE, "apt_dryrun: call apt_trainer_set_epoch first");
+  apt_ctx* c = t->ctx;
+  const int C = t->world, K = t->K;
+  const apt_graph* g = t->g;
+  n_steps = std::min<int64_t>(n_steps, t->steps_per_epoch);
+  DrySampler ds;
+  const bool ok = ds.init(t);
+  Arena& A = ds.A;
+  const int64_t n_words = ds.n_words;
+  uint32_t* own_bm = A.alloc<uint32_t>(n_words * C, true);        // one bitmap per owner / block
+  DryCounters* dc = A.alloc<DryCounters>(4, true);                 // per strategy
+  std::vector<Hop>& hops = ds.hops;
+  if (!ok || !own_bm || !dc) return set_err(c, APT_E_OOM, "apt_dryrun: out of device memory");
   // tiers of the unified store (rows beyond the HBM budgets, replicated hot rows)
   const TierInfo ti{g->part, g->lrow, t->f->tiered ? t->f->rows_dev : nullptr, t->f->cache_bm, n_words};
   std::vector<cudaEvent_t> ev;
@@ -211,24 +257,11 @@ extern "C" apt_status apt_dryrun(apt_trainer* t, int64_t n_steps, apt_plan_stats
   for (int S = 0; S < 4; ++S) {
     const bool by_part = (S == APT_SNP || S == APT_DNP) && C > 1;
     for (int64_t st = 0; st < n_steps; ++st) {
-      dry_set_step_kernel<<<1, 1, 0, c->stream>>>(step_dev, uint64_t(st));
+      ds.set_step(st, c->stream);
       CK(c, cudaMemsetAsync(own_bm, 0, sizeof(uint32_t) * n_words * C, c->stream));
       for (int r = 0; r < C; ++r) {
         CK(c, cudaEventRecord(new_event(), c->stream));
-        SeedArgs sa{t->perm, t->n_train, step_dev, t->steps_per_epoch, C, r, t->m.batch, by_part ? 1 : 0, g->part,
-                    seeds, small, small + 1};
-        CK(c, launch_select_seeds(sa, c->stream));
-        for (int h = 0; h < K; ++h) {
-          Hop& hp = hops[h];
-          SampleArgs sm{g->indptr, g->indices, hp.dst, hp.n_dst, hp.max_dst, hp.k,
-                        philox_key(t->m.sample_seed, kDomSample), step_dev, h, hp.cnt, hp.nbr};
-          CK(c, launch_sample(sm, c->stream));
-          if (h + 1 < K) {
-            CompactArgs ca{hp.dst, hp.n_dst, hp.max_dst, hp.cnt, hp.nbr, hp.k, dst_bm, new_bm, n_words, pos, hp.src,
-                           hp.counts, hp.indptr, hp.indices, hp.counts + 1, partials, hp.part2};
-            CK(c, launch_compact(ca, c->stream));
-          }
-        }
+        { apt_status s2 = ds.sample(r, by_part); if (s2 != APT_OK) return s2; }
         CK(c, cudaEventRecord(new_event(), c->stream));
         marks.push_back({S, r});
         const Hop& l1 = hops[K - 1];
@@ -237,7 +270,7 @@ extern "C" apt_status apt_dryrun(apt_trainer* t, int64_t n_steps, apt_plan_stats
         launch_pdl(dry_count_kernel, dim3(blocks), dim3(256), 0, c->stream, S, r, C, l1.dst, l1.n_dst, l1.cnt, l1.nbr, l1.k, g->part,
                                                         own_bm, n_words, dc + S, ti);
         CK(c, cudaGetLastError());
-        c->launches += 4 + 4 * K;
+        c->launches += 3;
       }
       launch_pdl(dry_fold_kernel, dim3(1), dim3(64), 0, c->stream, C, dc + S);
       CK(c, cudaGetLastError());
@@ -350,6 +383,68 @@ extern "C" apt_status apt_dryrun(apt_trainer* t, int64_t n_steps, apt_plan_stats
         out->attn_bytes[APT_SNP][cc] += int64_t(qs.tot_rows[r][cc]) * 2 * H * 4;
       }
   }
+  return APT_OK;
+}
+
+// ---------------------------------------------------------------- access frequencies
+// How often each node's input row is loaded (Table 3, "Node access
+// skewness"; reading R12): once per (step, requester) in which it is a source of the
+// requester's layer-1 block, over the first n_steps global steps of the epoch under
+// GDP's seed split.  Drives the excess cache's hot list.
+namespace apt {
+__global__ void access_count_kernel(const int32_t* __restrict__ n_p, const int32_t* __restrict__ cnt,
+                                    const int32_t* __restrict__ nbr, int k, uint32_t* bm, int32_t* counts) {
+  APT_PDL_PROLOGUE();
+  const int64_t n = *n_p;
+  for (int64_t i = int64_t(blockIdx.x) * blockDim.x + threadIdx.x; i < n; i += int64_t(gridDim.x) * blockDim.x) {
+    const int c_i = cnt[i];
+    for (int e = 0; e < c_i; ++e) {
+      const int u = nbr[i * k + e];
+      if (test_and_set(bm, u)) atomicAdd(counts + u, 1);
+    }
+  }
+}
+}  // namespace apt
+
+extern "C" apt_status apt_access_counts(apt_trainer* t, int64_t n_steps, int32_t* counts_host) {
+  if (!t || !counts_host || n_steps < 1)
+    return set_err(t ? t->ctx : nullptr, APT_E_INVALID, "apt_access_counts: bad arguments");
+  if (!t->perm) return set_err(t->ctx, APT_E_STATE, "apt_access_counts: call apt_trainer_set_epoch first");
+  apt_ctx* c = t->ctx;
+  const int C = t->world, K = t->K;
+  n_steps = std::min<int64_t>(n_steps, t->steps_per_epoch);
+  DrySampler ds;
+  const bool ok = ds.init(t);
+  uint32_t* bm = ds.A.alloc<uint32_t>(ds.n_words, true);
+  int32_t* counts = ds.A.alloc<int32_t>(t->g->n, true);
+  if (!ok || !bm || !counts) return set_err(c, APT_E_OOM, "apt_access_counts: out of device memory");
+  const Hop& l1 = ds.hops[K - 1];
+  const int64_t blocks = std::max<int64_t>(1, std::min<int64_t>(ceil_div(l1.max_dst, 256), 148 * 8));
+  for (int64_t st = 0; st < n_steps; ++st) {
+    ds.set_step(st, c->stream);
+    for (int r = 0; r < C; ++r) {
+      CK(c, cudaMemsetAsync(bm, 0, sizeof(uint32_t) * ds.n_words, c->stream));
+      { apt_status s = ds.sample(r, false); if (s != APT_OK) return s; }
+      launch_pdl(access_count_kernel, dim3(blocks), dim3(256), 0, c->stream, l1.n_dst, l1.cnt, l1.nbr, l1.k, bm, counts);
+      CK(c, cudaGetLastError());
+      c->launches++;
+    }
+  }
+  CK(c, cudaMemcpyAsync(counts_host, counts, sizeof(int32_t) * t->g->n, cudaMemcpyDeviceToHost, c->stream));
+  CK(c, cudaStreamSynchronize(c->stream));
+  return APT_OK;
+}
+
+// Hot list for the excess cache: node ids by descending access count, ties by
+// ascending id (host arithmetic).
+extern "C" apt_status apt_hot_rows(const int32_t* counts, int64_t n, int64_t k, int64_t* ids_out) {
+  if (!counts || !ids_out || n < 0 || k < 0 || k > n) return APT_E_INVALID;
+  std::vector<int64_t> idx(static_cast<size_t>(n));
+  for (int64_t i = 0; i < n; ++i) idx[size_t(i)] = i;
+  std::partial_sort(idx.begin(), idx.begin() + k, idx.end(), [&](int64_t a, int64_t b) {
+    return counts[a] != counts[b] ? counts[a] > counts[b] : a < b;
+  });
+  std::copy(idx.begin(), idx.begin() + k, ids_out);
   return APT_OK;
 }
 

@@ -66,11 +66,15 @@ struct RowParams {
   const int32_t* row_div;   // optional: divide row m by indptr[m+1] - indptr[m] (RN)
   uint16_t* Yb;             // optional bf16 output instead of Y (not with routing / accumulation)
   int64_t yb_pitch;
+  int b_early;              // B (W) is not written by the preceding kernel: load it before the PDL wait
 };
 
 __global__ void __launch_bounds__(ROW_THREADS, 2)
     rowtile_kernel(const __grid_constant__ CUtensorMap mapA, const __grid_constant__ CUtensorMap mapB, RowParams p) {
-  APT_PDL_PROLOGUE();
+  // Programmatic dependent launch: barrier init, TMEM allocation, tensor-map prefetch
+  // and (b_early) the resident B load run before griddepcontrol.wait, i.e. while the
+  // preceding kernel of the step drains; everything that reads its outputs (the row
+  // count, A) or writes global memory comes after the wait.
   extern __shared__ __align__(1024) uint8_t smem_raw[];
   uint8_t* smem = smem_raw + ((1024u - (smem_u32(smem_raw) & 1023u)) & 1023u);   // 1 KB aligned, still __shared__
   uint8_t* smem_a = smem;                                        // stages x 16 KB
@@ -82,10 +86,10 @@ __global__ void __launch_bounds__(ROW_THREADS, 2)
   uint64_t* tfull = bfull + 1;            // [2]
   uint64_t* tempty = tfull + 2;           // [2]
   uint32_t* tmem_slot = reinterpret_cast<uint32_t*>(tempty + 2);
+  float* sbias = reinterpret_cast<float*>(reinterpret_cast<uint8_t*>(bars) + 128);           // [<= 256]
+  float* stg_all = reinterpret_cast<float*>(reinterpret_cast<uint8_t*>(bars) + 128 + 1024);   // [8][32][17]
 
   const int warp = threadIdx.x >> 5, lane = lane_id();
-  const int64_t M = std::min<int64_t>(p.M_max, int64_t(*p.M_dev));
-  const int64_t ntiles = ceil_div(M, BM);
   const int n0 = int(blockIdx.x % p.n_split) * p.BN;              // this CTA's column slice
   const int64_t t0 = blockIdx.x / p.n_split, tstride = gridDim.x / p.n_split;
 
@@ -98,28 +102,35 @@ __global__ void __launch_bounds__(ROW_THREADS, 2)
     asm volatile("prefetch.tensormap [%0];" ::"l"(reinterpret_cast<uint64_t>(&mapB)) : "memory");
   }
   if (warp == 1) tmem_alloc(tmem_slot, uint32_t(p.tmem_cols));
-  // this CTA's bias slice (zero past N or without bias), read by the epilogue
-  float* sbias = reinterpret_cast<float*>(
-      (reinterpret_cast<uintptr_t>(reinterpret_cast<float*>(tmem_slot + 4) + 8 * 32 * 17) + 15) & ~uintptr_t(15));
-  for (int j = threadIdx.x; j < p.BN; j += blockDim.x) sbias[j] = (p.bias && n0 + j < p.N) ? p.bias[n0 + j] : 0.f;
   fence_before();
   __syncthreads();
   fence_after();
   const uint32_t tmem_base = *tmem_slot;
+  // resident B (this CTA's column slice): W does not depend on the preceding kernel when
+  // the caller says so (b_early), so its load overlaps that kernel's tail
+  auto load_b = [&]() {
+    mbar_expect_tx(bfull, uint32_t(p.nkb) * p.b_kb_bytes);
+    const int nb = int(ceil_div(p.BN, 64));
+    for (int kb = 0; kb < p.nkb; ++kb) {
+      uint8_t* dst = smem_b + size_t(kb) * p.b_kb_bytes;
+      if (p.b_mn) {
+        for (int j = 0; j < nb; ++j) tma_load_2d(dst + j * MNBLK, &mapB, bfull, n0 + j * 64, kb * BK);
+      } else {
+        tma_load_2d(dst, &mapB, bfull, kb * BK, n0);
+      }
+    }
+  };
+  if (p.b_early && warp == 0 && lane == 0) load_b();
+  pdl_wait();
+  pdl_launch();
+  const int64_t M = std::min<int64_t>(p.M_max, int64_t(*p.M_dev));
+  const int64_t ntiles = ceil_div(M, BM);
 
   if (warp == 0) {
+    if (lane == 0 && p.b_early && ntiles <= t0) mbar_wait(bfull, 0);   // no tile: let B land before exit
     if (lane == 0 && ntiles > t0) {
-      // ---- TMA producer: resident B (this CTA's column slice), then the A ring
-      mbar_expect_tx(bfull, uint32_t(p.nkb) * p.b_kb_bytes);
-      const int nb = int(ceil_div(p.BN, 64));
-      for (int kb = 0; kb < p.nkb; ++kb) {
-        uint8_t* dst = smem_b + size_t(kb) * p.b_kb_bytes;
-        if (p.b_mn) {
-          for (int j = 0; j < nb; ++j) tma_load_2d(dst + j * MNBLK, &mapB, bfull, n0 + j * 64, kb * BK);
-        } else {
-          tma_load_2d(dst, &mapB, bfull, kb * BK, n0);
-        }
-      }
+      // ---- TMA producer: resident B (unless loaded early), then the A ring
+      if (!p.b_early) load_b();
       int s = 0;
       uint32_t ph = 0;
       for (int64_t t = t0; t < ntiles; t += tstride) {
@@ -175,8 +186,11 @@ __global__ void __launch_bounds__(ROW_THREADS, 2)
     // load is issued before the current chunk is processed, so a chunk's critical path
     // is shared-memory latency, not a global bias load and a TMEM round trip.
     const int q = warp & 3, h = (warp - 2) >> 2;
-    float* stg = reinterpret_cast<float*>(tmem_slot + 4) + (warp - 2) * 32 * 17;
+    float* stg = stg_all + (warp - 2) * 32 * 17;
     const int rsub = lane >> 2, cq = (lane & 3) * 4;
+    // this CTA's bias slice (zero past N or without bias), shared by the 8 epilogue warps
+    for (int j = threadIdx.x - 64; j < p.BN; j += 256) sbias[j] = (p.bias && n0 + j < p.N) ? p.bias[n0 + j] : 0.f;
+    asm volatile("bar.sync 1, 256;" ::: "memory");
     int acc = 0;
     uint32_t aph = 0;
     for (int64_t t = t0; t < ntiles; t += tstride) {
@@ -298,7 +312,8 @@ struct WgradParams {
 
 __global__ void __launch_bounds__(THREADS, 1)
     wgrad_kernel(const __grid_constant__ CUtensorMap mapG, const __grid_constant__ CUtensorMap mapZ, WgradParams p) {
-  APT_PDL_PROLOGUE();
+  // PDL: barriers and TMEM are set up before griddepcontrol.wait (overlapping the
+  // preceding kernel's tail); the row count and every operand are read after it
   extern __shared__ __align__(1024) uint8_t smem_raw[];
   uint8_t* smem = smem_raw + ((1024u - (smem_u32(smem_raw) & 1023u)) & 1023u);   // 1 KB aligned, still __shared__
   uint64_t* bars = reinterpret_cast<uint64_t*>(smem + size_t(WG_STAGES) * p.stage_bytes);
@@ -308,13 +323,7 @@ __global__ void __launch_bounds__(THREADS, 1)
   uint32_t* tmem_slot = reinterpret_cast<uint32_t*>(tfull + 1);
 
   const int warp = threadIdx.x >> 5, lane = lane_id();
-  const int64_t rows = std::min<int64_t>(p.rows_max, int64_t(*p.rows_dev));
-  const int64_t nkb_all = ceil_div(rows, BK);
-  const int64_t per = ceil_div(nkb_all, int64_t(gridDim.x));
-  const int64_t kb0 = int64_t(blockIdx.x) * per;
-  const int64_t kb1 = std::min<int64_t>(nkb_all, kb0 + per);
   const int m0 = blockIdx.y * BM;
-  if (kb0 >= kb1) return;   // uniform for the CTA: nothing to add
 
   if (warp == 0 && lane == 0) {
     for (int s = 0; s < WG_STAGES; ++s) { mbar_init(full + s, 1); mbar_init(empty + s, 1); }
@@ -328,6 +337,18 @@ __global__ void __launch_bounds__(THREADS, 1)
   __syncthreads();
   fence_after();
   const uint32_t tmem_base = *tmem_slot;
+  pdl_wait();
+  pdl_launch();
+  const int64_t rows = std::min<int64_t>(p.rows_max, int64_t(*p.rows_dev));
+  const int64_t nkb_all = ceil_div(rows, BK);
+  const int64_t per = ceil_div(nkb_all, int64_t(gridDim.x));
+  const int64_t kb0 = int64_t(blockIdx.x) * per;
+  const int64_t kb1 = std::min<int64_t>(nkb_all, kb0 + per);
+  if (kb0 >= kb1) {   // uniform for the CTA: nothing to add
+    __syncthreads();
+    if (warp == 1) tmem_dealloc(tmem_base, uint32_t(p.tmem_cols));
+    return;
+  }
 
   if (warp == 0) {
     if (lane == 0) {
@@ -436,11 +457,10 @@ cudaError_t launch_tc_gemm(const TcGemmArgs& a, cudaStream_t st) {
   const int64_t tiles = std::max<int64_t>(1, ceil_div(a.M_max, BM));
   int n_split = 1;
   while (n_split < 4 && tiles * n_split * 2 <= sm_count() && BN_all % (64 * n_split * 2) == 0) n_split *= 2;
-  // forward projections (W K-major): 128-column slices even with many tiles -- with the
-  // 2-CTA/SM mode below this measured 7 us faster on the products layer-1 projection;
-  // the backward dZ (W N-major) measured faster unsplit, single CTA
+  // 128-column slices even with many tiles: A/B on the products step (APT_PROJ_SPLIT =
+  // 1 / 2 / 4 for every projection and dZ): 0.230 / 0.221 / 0.229 ms
   static const int force_split = [] { const char* v = std::getenv("APT_PROJ_SPLIT"); return v ? atoi(v) : -1; }();
-  const int want_split = force_split >= 0 ? force_split : (a.w_mn ? 1 : 2);
+  const int want_split = force_split >= 0 ? force_split : 2;
   if (want_split > n_split && BN_all % (64 * want_split) == 0) n_split = want_split;
   const int BN = BN_all / n_split;
   CUtensorMap ma, mb;
@@ -458,8 +478,7 @@ cudaError_t launch_tc_gemm(const TcGemmArgs& a, cudaStream_t st) {
   // loads and MMAs overlap the other's epilogue
   static const int two_cta = [] { const char* v = std::getenv("APT_PROJ_2CTA"); return v ? atoi(v) : 0; }();   // off: measured slower end to end (the overlapped sampling then lands on the backward)
   auto smem_of = [&](int st) {
-    return 1024 + size_t(st) * A_STAGE_BYTES + size_t(nkb) * b_kb_bytes + 16 * 8 + 16 + 8 * 32 * 17 * 4 +
-           16 + size_t(BN) * 4;
+    return 1024 + size_t(st) * A_STAGE_BYTES + size_t(nkb) * b_kb_bytes + 128 + 1024 + 8 * 32 * 17 * 4;
   };
   int stages = STAGES, nacc = 2, per_sm = 1;
   if (two_cta && !a.w_mn && smem_of(2) <= 113 * 1024 && BN <= 256 && tiles * n_split > sm_count()) {
@@ -471,7 +490,7 @@ cudaError_t launch_tc_gemm(const TcGemmArgs& a, cudaStream_t st) {
   while (cols < nacc * BN) cols <<= 1;
   RowParams p{a.M_max, a.M_dev, a.N, BN, nkb, cols, a.w_mn, stages, nacc, b_kb_bytes, a.bias, a.relu, a.Y, a.y_pitch,
               a.out_base, a.out_rank, a.out_row, a.accumulate, n_split, a.mask, a.mask_pitch, a.row_div_indptr,
-              a.Yb, a.yb_pitch};
+              a.Yb, a.yb_pitch, a.b_early};
   const size_t smem = smem_of(stages);   // + epilogue staging
   if (smem > 227 * 1024) return cudaErrorInvalidValue;
   static bool attr_set = false;

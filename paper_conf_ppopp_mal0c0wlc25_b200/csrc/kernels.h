@@ -208,6 +208,7 @@ struct TcGemmArgs {
   // optional bf16 output instead of Y (hidden activations in bf16 mode, reading R11):
   // row m -> Yb + m * yb_pitch (not with routing / accumulation)
   uint16_t* Yb; int64_t yb_pitch;
+  int b_early;                         // W is not written by the preceding kernel (the step's projections)
 };
 int tc_gemm_supported(int N, int K);
 cudaError_t launch_tc_gemm(const TcGemmArgs& a, cudaStream_t st);

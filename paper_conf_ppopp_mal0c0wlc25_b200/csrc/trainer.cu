@@ -152,6 +152,7 @@ apt_status project(apt_trainer* t, const Layer& L, const void* Zb, const float* 
                  bias, relu, Y, L.h_pitch, out_base, out_rank, out_row, 0};
     if (relu && L.Mk && !out_rank) { a.mask = L.Mk; a.mask_pitch = L.mk_pitch; }   // ReLU bits for the backward
     if (Y == L.H && L.Hb && !out_rank) { a.Yb = L.Hb; a.yb_pitch = L.hb_pitch; }   // R11: bf16 only
+    a.b_early = 1;   // the step's weights change only in the SGD at its end
     CK(c, launch_tc_gemm(a, c->stream));
   } else {
     if (out_rank) return set_err(c, APT_E_UNSUPPORTED, "routed epilogue needs the tcgen05 path");
@@ -708,6 +709,7 @@ apt_status upper_bwd(apt_trainer* t, RankState& rs) {
       TcGemmArgs g{L.Gb, L.gb_pitch, L.Wb, L.wb_pitch, L.max_rows, L.n_rows, L.d_in, L.d_out, nullptr, 0,
                    L.dZ, L.zf_pitch, nullptr, nullptr, nullptr, 1};
       g.row_div_indptr = hp.indptr;   // dZ / deg once per row (the pull then only sums)
+      g.b_early = 1;
       CK(c, launch_tc_gemm(g, c->stream));
       dz_scaled = 1;
     } else {
