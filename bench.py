@@ -45,8 +45,8 @@ STRATS = ("GDP", "NFP", "SNP", "DNP")
 def parse():
     ap = argparse.ArgumentParser()
     ap.add_argument("--gpus", type=int, default=1)
-    ap.add_argument("--steps", type=int, default=30)
-    ap.add_argument("--warmup", type=int, default=5)
+    ap.add_argument("--steps", type=int, default=100)
+    ap.add_argument("--warmup", type=int, default=20)
     ap.add_argument("--impl", default="apt", choices=["apt", "reference"])
     ap.add_argument("--config", default="products", choices=sorted(aptgen.CONFIGS))
     ap.add_argument("--strategy", default="GDP", choices=list(STRATS))

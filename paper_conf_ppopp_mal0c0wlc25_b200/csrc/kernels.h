@@ -107,6 +107,25 @@ struct AggArgs {
 };
 cudaError_t launch_agg_fstore(const AggArgs& a, const FeatView& fv, cudaStream_t st);
 cudaError_t launch_agg_csr(const AggArgs& a, cudaStream_t st);
+// Output layer K fused (outlayer.cu, bf16 mode): mean of H_{K-1} bf16 rows over the
+// block CSR, logits on CUDA cores, CE loss, G / Gb, dZ = (Gb W) / deg.
+struct OutLayerArgs {
+  const int32_t* indptr; const int32_t* indices;   // block of layer K (hop 0)
+  const int32_t* n_dst; int64_t max_dst;
+  const uint16_t* xb; int64_t x_pitch;             // H_{K-1} bf16 [n_src x x_pitch]
+  int d_in, d_out;
+  const uint16_t* Wb; int64_t wb_pitch; const float* bias;
+  const int32_t* seeds; const int32_t* labels; const int32_t* n_global;
+  uint16_t* Zb; int64_t zb_pitch;                  // Z_K bf16 + ones column d_in
+  float* H; int64_t h_pitch;                       // logits
+  float* loss;
+  float* G; int64_t g_pitch;
+  uint16_t* Gb; int64_t gb_pitch;                  // zero-padded to the 64-row block
+  float* dZ; int64_t dz_pitch;                     // (G W) / deg
+};
+int outlayer_supported(int d_in, int d_out);
+cudaError_t launch_outlayer(const OutLayerArgs& a, cudaStream_t st);
+
 
 // dX[src_e] += dZ[v] / deg(v)  (O5 backward), fp32 atomics.
 cudaError_t launch_agg_bwd(const int32_t* indptr, const int32_t* indices, const int32_t* n_dst, int64_t max_dst,

@@ -660,13 +660,35 @@ apt_status layer1_fwd_gdp(apt_trainer* t, RankState& rs, bool time_it) {
                  t->K > 1 ? 1 : 0, L.H, nullptr, nullptr, nullptr);
 }
 
+// The output layer as one kernel (outlayer.cu): bf16 mode, K >= 2, <= 64 classes,
+// input width <= 256, opt-in with APT_FUSED_OUT=1 (read when the step is built).
+// Measured on products: faster alone (0.266 vs 0.272 ms with the
+// step's sampling inline) but slower next to the overlapped sampling of the next
+// step (0.243 vs 0.221 ms), so the pipelined default keeps the unfused kernels.
+static bool fused_out(const apt_trainer* t, const RankState& rs) {
+  const char* e = std::getenv("APT_FUSED_OUT");
+  if (!e || atoi(e) != 1 || t->m.dtype != APT_BF16 || t->K < 2) return false;
+  const Layer& LK = rs.L[t->K - 1];
+  return rs.L[t->K - 2].Hb && outlayer_supported(LK.d_in, LK.d_out);
+}
+
 // Upper layers l = 2..K (data parallel) + CE loss on one rank.
 apt_status upper_fwd_loss(apt_trainer* t, RankState& rs) {
   apt_ctx* c = t->ctx;
+  const bool fo = fused_out(t, rs);
   for (int l = 2; l <= t->K; ++l) {
     Layer& L = rs.L[l - 1];
     const Layer& P = rs.L[l - 2];
     const Hop& hp = rs.hops[t->K - l];
+    if (l == t->K && fo) {   // mean + logits + CE + G + dZ of the output layer in one kernel
+      CK(c, cudaMemsetAsync(rs.loss, 0, sizeof(float), c->stream));
+      OutLayerArgs o{hp.indptr, hp.indices, hp.n_dst, hp.max_dst, P.Hb, P.hb_pitch, L.d_in, L.d_out,
+                     L.Wb, L.wb_pitch, L.b, rs.seeds, t->labels, rs.small + 1, L.Zb, L.zb_pitch,
+                     L.H, L.h_pitch, rs.loss, L.G, L.h_pitch, L.Gb, L.gb_pitch, L.dZ, L.zf_pitch};
+      CK(c, launch_outlayer(o, c->stream));
+      c->launches++;
+      return APT_OK;
+    }
     AggArgs a{};
     a.indptr = hp.indptr; a.indices = hp.indices; a.x = P.H; a.x_pitch = P.h_pitch;
     if (P.Hb) { a.x = nullptr; a.xb = P.Hb; a.x_pitch = P.hb_pitch; }   // R11
@@ -704,6 +726,9 @@ apt_status upper_bwd(apt_trainer* t, RankState& rs) {
                                bf ? L.zb_pitch : L.zf_pitch, L.n_rows, L.max_rows, L.d_in, L.dW, L.db, L.d_in, c->side);
     if (s != APT_OK) return s;
     int dz_scaled = 0;
+    if (l == t->K && fused_out(t, rs)) {
+      dz_scaled = 1;   // dZ / deg came with the fused output layer
+    } else
     // dZ = G W  (bf16 mode: tcgen05 with the bf16 weights of the forward, W read N-major as stored)
     if (bf && tc_gemm_supported(L.d_in, L.d_out)) {
       TcGemmArgs g{L.Gb, L.gb_pitch, L.Wb, L.wb_pitch, L.max_rows, L.n_rows, L.d_in, L.d_out, nullptr, 0,

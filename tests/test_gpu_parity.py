@@ -225,6 +225,29 @@ def test_train_step_matches_oracle(A, ctx, tiny, dtype, step):
         assert np.allclose(tr.read("db", l)[0], db, **tol), f"db layer {l}"
 
 
+@pytest.mark.parametrize("step", [0, 2])
+def test_train_step_fused_output_layer(A, ctx, tiny, step, monkeypatch):
+    """The opt-in fused output layer (outlayer.cu: mean + logits + CE + G + dZ/deg in one
+    kernel, APT_FUSED_OUT=1) against the oracle: logits, loss, every layer's gradients."""
+    monkeypatch.setenv("APT_FUSED_OUT", "1")
+    cfg, g, train = tiny
+    tr, params, labels = _trainer(A, ctx, cfg, g, train, "bf16")
+    tr.step(step, update=False)
+    seeds = tr.read("seeds")[:, 0].astype(np.int64)
+    blocks = oracle.sample_blocks(g, seeds, cfg.fanouts, cfg.sample_seed, step)
+    p64 = [(W.astype(np.float64), b.astype(np.float64)) for W, b in params]
+    ref = model.train_step(blocks, cfg.feat_seed, cfg.dim, p64, labels[seeds], len(seeds), "bf16")
+    tol = TOL["bf16"]
+    K = len(blocks)
+    assert np.allclose(tr.read("Z", K), ref["cache"]["Z"][K - 1], **tol)
+    assert np.allclose(tr.read("H", K), ref["cache"]["h"][K - 1], **tol)
+    assert abs(tr.loss() - ref["loss"]) <= tol["rtol"] * abs(ref["loss"]) + tol["atol"]
+    for l in range(1, K + 1):
+        dW, db = ref["grads"][l - 1]
+        assert np.allclose(tr.read("dW", l), dW, **tol), f"dW layer {l}"
+        assert np.allclose(tr.read("db", l)[0], db, **tol), f"db layer {l}"
+
+
 @pytest.mark.parametrize("dtype", ["f32", "bf16"])
 def test_train_step_wide_hidden(A, ctx, tiny, dtype):
     """Hidden width past every single-launch limit (config 5 sweeps d' to 1024): the upper
