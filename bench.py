@@ -414,7 +414,7 @@ def run_apt(args, cfg):
     if rank == 0 and world == 1 and not args.no_planner:
         out["planner"] = planner_report(A, g, cfg, train, labels, args, stream, ms_local)
         # the workload's access skew next to the paper's Table 3 (reading R12)
-        n_acc = min(spe, 64)
+        n_acc = spe   # one whole epoch (the paper ranks nodes over training; a prefix undercounts the tail)
         out["access_skew"] = {"steps": n_acc, "buckets": ["<1%", "1-5%", "5-10%", "10-20%", "20-50%", "50-100%"],
                               "table": skew_table(tr.access_counts(n_acc)),
                               "paper_table3": {"PS": [0.501, 0.348, 0.088, 0.047, 0.017, 0.0],

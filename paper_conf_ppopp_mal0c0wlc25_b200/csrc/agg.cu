@@ -258,16 +258,113 @@ __global__ void __launch_bounds__(256, MINB) agg_l1_kernel(AggArgs a, EllFstoreS
   }
 }
 
+// agg_l1_kernel with the next row pair's count and edge ids loaded one iteration
+// ahead (fanout <= 16: one id per lane), so a row pair's critical path starts at its
+// feature-row loads instead of at the index loads.
+template <int EPV, int NB, int MINB>
+__global__ void __launch_bounds__(256, MINB) agg_l1_pf_kernel(AggArgs a, EllFstoreSrc src) {
+  APT_PDL_PROLOGUE();
+  __shared__ uint4 zrow[16];
+  if (threadIdx.x < 16) zrow[threadIdx.x] = make_uint4(0, 0, 0, 0);
+  __syncthreads();
+  const int lane = lane_id();
+  const int sub = lane >> 4, l = lane & 15;
+  const int64_t n_dst = *a.n_dst;
+  const int V = int(ceil_div(a.dim, EPV));
+  const int lv = l < V ? l : 0;
+  const int k = src.k;
+  const int64_t nwarps = int64_t(gridDim.x) * (blockDim.x >> 5);
+  int64_t w = (int64_t(blockIdx.x) * blockDim.x + threadIdx.x) >> 5;
+  int cnt_n = 0, u_n = -1;
+  {
+    const int64_t i = w * 2 + sub;
+    if (i < n_dst) { cnt_n = src.count(i); if (l < k) u_n = src.node(i * k + l); }
+  }
+  for (; w * 2 < n_dst; w += nwarps) {
+    const int64_t i = w * 2 + sub;
+    const bool valid = i < n_dst;
+    const int cnt = cnt_n, u = u_n;
+    {   // next pair's count and ids, consumed one iteration later
+      const int64_t i2 = (w + nwarps) * 2 + sub;
+      cnt_n = 0; u_n = -1;
+      if (i2 < n_dst) { cnt_n = src.count(i2); if (l < k) u_n = src.node(i2 * k + l); }
+    }
+    const int cmax = max(cnt, __shfl_xor_sync(0xffffffffu, cnt, 16));
+    float acc[EPV];
+#pragma unroll
+    for (int q = 0; q < EPV; ++q) acc[q] = 0.f;
+    const bool keep = l < cnt && (!a.filt_part || a.filt_part[u] == a.keep_part);
+    const char* rp = keep ? src.row_ptr(u) : reinterpret_cast<const char*>(zrow);
+    for (int j = 0; j < cmax; j += NB) {
+      uint4 v[NB];
+#pragma unroll
+      for (int q = 0; q < NB; ++q) {
+        const char* r = reinterpret_cast<const char*>(
+            __shfl_sync(0xffffffffu, reinterpret_cast<uintptr_t>(rp), sub * 16 + ((j + q) & 15)));
+        v[q] = *reinterpret_cast<const uint4*>(r + lv * 16);
+      }
+#pragma unroll
+      for (int q = 0; q < NB; ++q) accumulate_vec<EPV>(acc, v[q]);
+    }
+    if (!valid || l >= V) continue;
+    if (a.z_ones && l == 0) a.z_bf16[i * a.z_bf16_pitch + a.dim] = 0x3F80;
+    const float fdeg = float(a.deg_override ? a.deg_override[i] : cnt);
+    const float rdeg = fdeg > 0.f ? __frcp_rn(fdeg) : 0.f;
+    float z[EPV];
+#pragma unroll
+    for (int q = 0; q < EPV; ++q) z[q] = fdeg > 0.f ? div_rn_rcp(acc[q], fdeg, rdeg) : 0.f;
+    const int c0 = l * EPV;
+    const bool full = c0 + EPV <= a.dim;
+    if (a.z_f32) {
+      float* o = a.z_f32 + i * a.z_f32_pitch + c0;
+#pragma unroll
+      for (int q = 0; q < EPV; ++q)
+        if (full || c0 + q < a.dim) o[q] = z[q];
+    }
+    if (a.z_bf16) {
+      uint16_t* o = a.z_bf16 + i * a.z_bf16_pitch + c0;
+      if (full) {
+        if constexpr (EPV == 8) {
+          *reinterpret_cast<uint4*>(o) = make_uint4(pack_bf16x2(z[0], z[1]), pack_bf16x2(z[2], z[3]),
+                                                    pack_bf16x2(z[4], z[5]), pack_bf16x2(z[6], z[7]));
+        } else {
+          *reinterpret_cast<uint2*>(o) = make_uint2(pack_bf16x2(z[0], z[1]), pack_bf16x2(z[2], z[3]));
+        }
+      } else {
+#pragma unroll
+        for (int q = 0; q < EPV; ++q) {
+          if (c0 + q < a.dim) {
+            __nv_bfloat16 h = __float2bfloat16_rn(z[q]);
+            o[q] = *reinterpret_cast<uint16_t*>(&h);
+          }
+        }
+      }
+    }
+  }
+}
+
 cudaError_t launch_agg_fstore(const AggArgs& a, const FeatView& fv, cudaStream_t st) {
   EllFstoreSrc s{a.cnt, a.nbr, a.k, fv, fv.pitch * (fv.dtype == kBF16 ? 2 : 4)};
   AggArgs b = a;
   b.dim = fv.dim;
   const int epv = fv.dtype == kBF16 ? 8 : 4;
   const int V = int(ceil_div(b.dim, epv));
-  // variant (A/B on products): 0 agg_kernel, 1 agg_l1_kernel (NB 4, default),
-  // 2 agg_l1_kernel with 8 loads in flight per lane.  All measured within 2 us (34 us in
-  // the step, 26.6 us alone); a cp.async double-buffered variant measured 38.7 us.
-  static const int variant = [] { const char* e = std::getenv("APT_AGG_VARIANT"); return e ? atoi(e) : 1; }();
+  // variant (A/B on products): 0 agg_kernel, 1 agg_l1_kernel (NB 4), 2
+  // agg_l1_kernel with 8 loads in flight per lane, 4 / 5 agg_l1_pf_kernel (next row
+  // pair's indices one iteration ahead) at 40 / 48 registers.  In the step: 34.5 (1),
+  // 33.2 (4), 32.4 us (5, default); a cp.async double-buffered variant measured 38.7 us.
+  static const int variant = [] { const char* e = std::getenv("APT_AGG_VARIANT"); return e ? atoi(e) : 5; }();
+  if ((variant == 4 || variant == 5) && V <= 16 && b.k <= 16) {
+    int64_t blocks = ceil_div(ceil_div(b.max_dst, 2) * 32, 256);
+    blocks = std::max<int64_t>(1, std::min<int64_t>(blocks, 148 * 16));
+    if (fv.dtype == kBF16) {
+      if (variant == 4) launch_pdl(agg_l1_pf_kernel<8, 4, 6>, dim3(blocks), dim3(256), 0, st, b, s);
+      else launch_pdl(agg_l1_pf_kernel<8, 4, 5>, dim3(blocks), dim3(256), 0, st, b, s);
+    } else {
+      launch_pdl(agg_l1_pf_kernel<4, 4, 6>, dim3(blocks), dim3(256), 0, st, b, s);
+    }
+    return cudaGetLastError();
+  }
   if ((variant == 1 || variant == 2) && V <= 16) {
     int64_t blocks = ceil_div(ceil_div(b.max_dst, 2) * 32, 256);
     blocks = std::max<int64_t>(1, std::min<int64_t>(blocks, 148 * 16));
