@@ -67,6 +67,7 @@ struct RowParams {
   uint16_t* Yb;             // optional bf16 output instead of Y (not with routing / accumulation)
   int64_t yb_pitch;
   int b_early;              // B (W) is not written by the preceding kernel: load it before the PDL wait
+  int staged;               // force the staged epilogue for plain rows too (APT_EPI_STAGED=1, A/B)
 };
 
 __global__ void __launch_bounds__(ROW_THREADS, 2)
@@ -186,6 +187,8 @@ __global__ void __launch_bounds__(ROW_THREADS, 2)
     // load is issued before the current chunk is processed, so a chunk's critical path
     // is shared-memory latency, not a global bias load and a TMEM round trip.
     const int q = warp & 3, h = (warp - 2) >> 2;
+    // staged: 0 direct for every plain output, 1 never (A/B), 2 only for bf16 rows
+    const bool direct = !p.out_rank && !p.accumulate && !p.mask && (p.staged == 0 || (p.staged == 2 && p.Yb));
     float* stg = stg_all + (warp - 2) * 32 * 17;
     const int rsub = lane >> 2, cq = (lane & 3) * 4;
     // this CTA's bias slice (zero past N or without bias), shared by the 8 epilogue warps
@@ -212,6 +215,67 @@ __global__ void __launch_bounds__(ROW_THREADS, 2)
       if (16 * h < p.BN) {
         tmem_ld16_nowait(tbase + uint32_t(16 * h), r);
         tmem_wait16(r);
+      }
+      if (direct) {
+        // Direct path (plain rows: no routing, reduction or mask): the lane owns its row
+        // (its TMEM lane) and writes the chunk's 16 values straight from registers as
+        // whole 32-B sectors -- no staging, shuffles or per-element branches; the
+        // epilogue was instruction-bound (~275 warp instructions per chunk staged)
+        for (int c = 16 * h; c < p.BN; c += 32) {
+          const bool more = c + 32 < p.BN;
+          if (more) tmem_ld16_nowait(tbase + uint32_t(c + 32), rn);
+          if (own) {
+            float v[16];
+#pragma unroll
+            for (int j = 0; j < 16; j += 4) {
+              const float4 bv = *reinterpret_cast<const float4*>(sbias + c + j);
+              v[j] = __uint_as_float(r[j]) + bv.x; v[j + 1] = __uint_as_float(r[j + 1]) + bv.y;
+              v[j + 2] = __uint_as_float(r[j + 2]) + bv.z; v[j + 3] = __uint_as_float(r[j + 3]) + bv.w;
+            }
+            if (p.relu) {
+#pragma unroll
+              for (int j = 0; j < 16; ++j) v[j] = fmaxf(v[j], 0.f);
+            }
+            if (p.row_div && own_deg > 0.f) {
+#pragma unroll
+              for (int j = 0; j < 16; ++j) v[j] = div_rn_rcp(v[j], own_deg, own_rdeg);
+            }
+            const int col = n0 + c;
+            if (p.Yb) {
+              uint16_t* d = reinterpret_cast<uint16_t*>(own) + col;
+              if (col + 16 <= p.N) {
+                reinterpret_cast<uint4*>(d)[0] = make_uint4(pack_bf16x2(v[0], v[1]), pack_bf16x2(v[2], v[3]),
+                                                            pack_bf16x2(v[4], v[5]), pack_bf16x2(v[6], v[7]));
+                reinterpret_cast<uint4*>(d)[1] = make_uint4(pack_bf16x2(v[8], v[9]), pack_bf16x2(v[10], v[11]),
+                                                            pack_bf16x2(v[12], v[13]), pack_bf16x2(v[14], v[15]));
+              } else {
+#pragma unroll
+                for (int j = 0; j < 16; ++j)
+                  if (col + j < p.N) d[j] = bf16_bits(v[j]);
+              }
+            } else {
+              float* d = own + col;
+              if (col + 16 <= p.N) {
+#pragma unroll
+                for (int j = 0; j < 16; j += 4)
+                  *reinterpret_cast<float4*>(d + j) = make_float4(v[j], v[j + 1], v[j + 2], v[j + 3]);
+              } else {
+#pragma unroll
+                for (int j = 0; j < 16; ++j)
+                  if (col + j < p.N) d[j] = v[j];
+              }
+            }
+          }
+          if (more) {
+            tmem_wait16(rn);
+#pragma unroll
+            for (int j = 0; j < 16; ++j) r[j] = rn[j];
+          }
+        }
+        fence_before();
+        mbar_arrive(tempty + acc);
+        if (++acc == p.nacc) { acc = 0; aph ^= 1; }
+        continue;
       }
       for (int c = 16 * h; c < p.BN; c += 32) {
         const bool more = c + 32 < p.BN;
@@ -297,7 +361,7 @@ __global__ void __launch_bounds__(ROW_THREADS, 2)
 }
 
 // ------------------------------------------------------------ weight-gradient kernel
-constexpr int WG_STAGES = 3;
+constexpr int WG_MAX_STAGES = 8;   // ring depth: as many stages as shared memory holds (runtime p.stages)
 
 struct WgradParams {
   const int32_t* rows_dev;  // number of valid rows (device)
@@ -305,6 +369,7 @@ struct WgradParams {
   int d_out, d_in, BN, nbz, tmem_cols;
   int ones_col;             // Z column d_in holds 1.0: output column d_in is db
   uint32_t stage_bytes;     // A (2 x 8 KB) + B (nbz x 8 KB)
+  int stages;               // ring depth (<= WG_MAX_STAGES)
   float* dW;                // [d_out x ldw] (accumulated)
   float* db;                // [d_out] (accumulated) or null
   int64_t ldw;
@@ -316,17 +381,17 @@ __global__ void __launch_bounds__(THREADS, 1)
   // preceding kernel's tail); the row count and every operand are read after it
   extern __shared__ __align__(1024) uint8_t smem_raw[];
   uint8_t* smem = smem_raw + ((1024u - (smem_u32(smem_raw) & 1023u)) & 1023u);   // 1 KB aligned, still __shared__
-  uint64_t* bars = reinterpret_cast<uint64_t*>(smem + size_t(WG_STAGES) * p.stage_bytes);
+  uint64_t* bars = reinterpret_cast<uint64_t*>(smem + size_t(p.stages) * p.stage_bytes);
   uint64_t* full = bars;
-  uint64_t* empty = bars + WG_STAGES;
-  uint64_t* tfull = bars + 2 * WG_STAGES;
+  uint64_t* empty = bars + WG_MAX_STAGES;
+  uint64_t* tfull = bars + 2 * WG_MAX_STAGES;
   uint32_t* tmem_slot = reinterpret_cast<uint32_t*>(tfull + 1);
 
   const int warp = threadIdx.x >> 5, lane = lane_id();
   const int m0 = blockIdx.y * BM;
 
   if (warp == 0 && lane == 0) {
-    for (int s = 0; s < WG_STAGES; ++s) { mbar_init(full + s, 1); mbar_init(empty + s, 1); }
+    for (int s = 0; s < p.stages; ++s) { mbar_init(full + s, 1); mbar_init(empty + s, 1); }
     mbar_init(tfull, 1);
     asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
     asm volatile("prefetch.tensormap [%0];" ::"l"(reinterpret_cast<uint64_t>(&mapG)) : "memory");
@@ -366,7 +431,7 @@ __global__ void __launch_bounds__(THREADS, 1)
         const int y = int(kb * BK);
         for (int j = 0; j < na; ++j) tma_load_2d(st + j * MNBLK, &mapG, full + s, m0 + 64 * j, y);
         for (int j = 0; j < nz; ++j) tma_load_2d(st + 2 * MNBLK + j * MNBLK, &mapZ, full + s, j * 64, y);
-        if (++s == WG_STAGES) { s = 0; ph ^= 1; }
+        if (++s == p.stages) { s = 0; ph ^= 1; }
       }
     }
   } else if (warp == 1) {
@@ -389,7 +454,7 @@ __global__ void __launch_bounds__(THREADS, 1)
         mma_commit(empty + s);
       }
       __syncwarp();
-      if (++s == WG_STAGES) { s = 0; ph ^= 1; }
+      if (++s == p.stages) { s = 0; ph ^= 1; }
     }
     if (lane == 0) mma_commit(tfull);
     __syncwarp();
@@ -463,6 +528,7 @@ cudaError_t launch_tc_gemm(const TcGemmArgs& a, cudaStream_t st) {
   const int want_split = force_split >= 0 ? force_split : 2;
   if (want_split > n_split && BN_all % (64 * want_split) == 0) n_split = want_split;
   const int BN = BN_all / n_split;
+  static const int epi_staged = [] { const char* v = std::getenv("APT_EPI_STAGED"); return v ? atoi(v) : 0; }();
   CUtensorMap ma, mb;
   if (!make_map(&ma, a.Z, a.K, std::max<int64_t>(a.M_max, 1), a.z_pitch, BK, BM)) return cudaErrorInvalidValue;
   uint32_t b_kb_bytes;
@@ -490,7 +556,7 @@ cudaError_t launch_tc_gemm(const TcGemmArgs& a, cudaStream_t st) {
   while (cols < nacc * BN) cols <<= 1;
   RowParams p{a.M_max, a.M_dev, a.N, BN, nkb, cols, a.w_mn, stages, nacc, b_kb_bytes, a.bias, a.relu, a.Y, a.y_pitch,
               a.out_base, a.out_rank, a.out_row, a.accumulate, n_split, a.mask, a.mask_pitch, a.row_div_indptr,
-              a.Yb, a.yb_pitch, a.b_early};
+              a.Yb, a.yb_pitch, a.b_early, epi_staged};
   const size_t smem = smem_of(stages);   // + epilogue staging
   if (smem > 227 * 1024) return cudaErrorInvalidValue;
   static bool attr_set = false;
@@ -520,9 +586,16 @@ cudaError_t launch_tc_wgrad(const TcWgradArgs& a, cudaStream_t st) {
   if (!make_map(&mg, a.G, a.d_out, rows, a.g_pitch, 64, BK)) return cudaErrorInvalidValue;
   if (!make_map(&mz, a.Z, zcols, rows, a.z_pitch, 64, BK)) return cudaErrorInvalidValue;
   const uint32_t stage = uint32_t(2 + nbz) * MNBLK;
-  WgradParams p{a.rows_dev, a.rows_max, a.d_out, a.d_in, BN, nbz, cols, a.db ? 1 : 0, stage, a.dW, a.db,
+  WgradParams p{a.rows_dev, a.rows_max, a.d_out, a.d_in, BN, nbz, cols, a.db ? 1 : 0, stage, 0, a.dW, a.db,
                 a.ldw > 0 ? a.ldw : a.d_in};
-  const size_t smem = 1024 + size_t(WG_STAGES) * stage + 8 * 8 + 16 + 4 * 32 * 33 * 4;
+  // ring depth: as many stages as fit (more bytes in flight per SM: the loads are the
+  // latency of this kernel), A/B via APT_WG_STAGES
+  static const int want = [] { const char* v = std::getenv("APT_WG_STAGES"); return v ? atoi(v) : 3; }();   // 3 / 8: 0.2199 / 0.2205 ms
+  const size_t fixed = 1024 + size_t(2 * WG_MAX_STAGES + 1) * 8 + 16 + 4 * 32 * 33 * 4;
+  int stages = std::max(2, std::min<int>(want, int((227 * 1024 - fixed) / stage)));
+  stages = std::min(stages, WG_MAX_STAGES);
+  p.stages = stages;
+  const size_t smem = fixed + size_t(stages) * stage;
   if (smem > 227 * 1024) return cudaErrorInvalidValue;
   static bool attr_set = false;
   if (!attr_set) {
