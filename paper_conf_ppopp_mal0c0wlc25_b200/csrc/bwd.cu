@@ -184,6 +184,83 @@ __global__ void __launch_bounds__(256) pull_bwd_kernel(PullArgs a) {
   }
 }
 
+// bf16 dZ / deg rows (reading R13), bf16 G, ReLU mask from bf16 H: a lane owns 8
+// columns (one 16-B load per in-edge), R source rows in flight per warp; the mask is
+// applied to the packed bf16 pairs with one AND against a per-half compare of H's bits
+// (bf16 > 0 <=> its 16-bit pattern is a positive signed integer).
+template <int VP, int R>
+__global__ void __launch_bounds__(256) pull_bwd_b8_kernel(PullArgs a) {
+  APT_PDL_PROLOGUE();
+  const int lane = lane_id();
+  const int64_t n = *a.n_src;
+  const int V8 = a.dim >> 3;                      // dim % 8 == 0 (checked at launch)
+  const int64_t nwarps = int64_t(gridDim.x) * (blockDim.x >> 5);
+  const int64_t rows_out = std::min<int64_t>(a.max_src, round_up(n, 64));
+  for (int64_t u0 = ((int64_t(blockIdx.x) * blockDim.x + threadIdx.x) >> 5) * R; u0 < rows_out; u0 += nwarps * R) {
+    int e0[R], cnt[R];
+    uint4 hm[R][VP];
+#pragma unroll
+    for (int r = 0; r < R; ++r) {
+      const int64_t u = u0 + r;
+      e0[r] = 0; cnt[r] = 0;
+      if (u < n) { e0[r] = a.csc_ptr[u]; cnt[r] = a.csc_ptr[u + 1] - e0[r]; }
+#pragma unroll
+      for (int p = 0; p < VP; ++p) {
+        const int j = lane + 32 * p;
+        hm[r][p] = (u < n && j < V8) ? __ldg(reinterpret_cast<const uint4*>(a.hb + u * a.hb_pitch + j * 8))
+                                     : make_uint4(0, 0, 0, 0);
+      }
+    }
+    float acc[R][VP][8];
+#pragma unroll
+    for (int r = 0; r < R; ++r)
+#pragma unroll
+      for (int p = 0; p < VP; ++p)
+#pragma unroll
+        for (int q = 0; q < 8; ++q) acc[r][p][q] = 0.f;
+    int cmax = cnt[0];
+#pragma unroll
+    for (int r = 1; r < R; ++r) cmax = max(cmax, cnt[r]);
+    for (int c0 = 0; c0 < cmax; c0 += 32) {
+      int v[R];
+#pragma unroll
+      for (int r = 0; r < R; ++r) v[r] = c0 + lane < cnt[r] ? a.csc_dst[e0[r] + c0 + lane].x : 0;
+      const int m = min(32, cmax - c0);
+      for (int e = 0; e < m; ++e) {
+#pragma unroll
+        for (int r = 0; r < R; ++r) {
+          const int w = __shfl_sync(0xffffffffu, v[r], e);
+          if (c0 + e >= cnt[r]) continue;
+#pragma unroll
+          for (int p = 0; p < VP; ++p) {
+            const int j = lane + 32 * p;
+            if (j < V8) {
+              const uint4 z = *reinterpret_cast<const uint4*>(a.dzb + int64_t(w) * a.dzb_pitch + j * 8);
+              accumulate_bf16x8(acc[r][p], z);
+            }
+          }
+        }
+      }
+    }
+#pragma unroll
+    for (int r = 0; r < R; ++r) {
+      const int64_t u = u0 + r;
+      if (u >= rows_out) continue;
+#pragma unroll
+      for (int p = 0; p < VP; ++p) {
+        const int j = lane + 32 * p;
+        if (j >= V8) continue;
+        const float* x = acc[r][p];
+        const uint4 o = make_uint4(pack_bf16x2(x[0], x[1]) & __vcmpgts2(hm[r][p].x, 0u),
+                                   pack_bf16x2(x[2], x[3]) & __vcmpgts2(hm[r][p].y, 0u),
+                                   pack_bf16x2(x[4], x[5]) & __vcmpgts2(hm[r][p].z, 0u),
+                                   pack_bf16x2(x[6], x[7]) & __vcmpgts2(hm[r][p].w, 0u));
+        *reinterpret_cast<uint4*>(a.gb + u * a.gb_pitch + j * 8) = o;
+      }
+    }
+  }
+}
+
 cudaError_t launch_pull_bwd(const PullArgs& a, cudaStream_t st) {
   if (a.dim > 512) {   // wide rows: column chunks of 512 (128 fp32 vectors per lane group)
     for (int c0 = 0; c0 < a.dim; c0 += 512) {
@@ -192,6 +269,7 @@ cudaError_t launch_pull_bwd(const PullArgs& a, cudaStream_t st) {
       b.dz = a.dz + c0;
       if (a.h) b.h = a.h + c0;
       if (a.hb) b.hb = a.hb + c0;
+      if (a.dzb) b.dzb = a.dzb + c0;
       if (a.mask) b.mask = a.mask + c0 / 16;
       if (a.g) b.g = a.g + c0;
       if (a.gb) b.gb = a.gb + c0;
@@ -204,6 +282,23 @@ cudaError_t launch_pull_bwd(const PullArgs& a, cudaStream_t st) {
   if ((a.dz_pitch & 3) || (a.h_pitch & 3) || (a.g && (a.g_pitch & 3)) || (a.gb && (a.gb_pitch & 3)))
     return cudaErrorInvalidValue;
   constexpr int R = 2;   // rows in flight per warp
+  if (a.dzb) {            // reading R13 (bf16 mode): bf16 dZ, bf16 G, mask from bf16 H
+    if (!a.gb || a.g || !a.hb || (a.dim & 7) || (a.dzb_pitch & 7) || (a.hb_pitch & 7) || (a.gb_pitch & 7))
+      return cudaErrorInvalidValue;
+    static const int rr = [] { const char* e = std::getenv("APT_PULL_ROWS"); return e ? atoi(e) : 2; }();
+    const int Rr = rr == 4 ? 4 : 2;
+    const int64_t blocks =
+        std::max<int64_t>(1, std::min<int64_t>(ceil_div(ceil_div(round_up(a.max_src, 64), Rr) * 32, 256), 148 * 16));
+    const int V8 = a.dim >> 3;
+    if (Rr == 4) {
+      if (V8 <= 32) launch_pdl(pull_bwd_b8_kernel<1, 4>, dim3(blocks), dim3(256), 0, st, a);
+      else launch_pdl(pull_bwd_b8_kernel<2, 4>, dim3(blocks), dim3(256), 0, st, a);
+    } else {
+      if (V8 <= 32) launch_pdl(pull_bwd_b8_kernel<1, 2>, dim3(blocks), dim3(256), 0, st, a);
+      else launch_pdl(pull_bwd_b8_kernel<2, 2>, dim3(blocks), dim3(256), 0, st, a);
+    }
+    return cudaGetLastError();
+  }
   const int64_t blocks =
       std::max<int64_t>(1, std::min<int64_t>(ceil_div(ceil_div(round_up(a.max_src, 64), R) * 32, 256), 148 * 16));
   const int ms = a.mask ? 1 : a.hb ? 3 : a.h ? 2 : 0;

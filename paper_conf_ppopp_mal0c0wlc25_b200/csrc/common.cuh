@@ -99,6 +99,12 @@ __device__ __forceinline__ T warp_sum(T v) {
 
 __device__ __forceinline__ float bf16_lo(uint32_t v) { return __uint_as_float(v << 16); }
 __device__ __forceinline__ float bf16_bits_to_float(uint16_t b) { return __uint_as_float(uint32_t(b) << 16); }
+__device__ __forceinline__ void accumulate_bf16x8(float* acc, uint4 raw) {
+  acc[0] += __uint_as_float(raw.x << 16); acc[1] += __uint_as_float(raw.x & 0xFFFF0000u);
+  acc[2] += __uint_as_float(raw.y << 16); acc[3] += __uint_as_float(raw.y & 0xFFFF0000u);
+  acc[4] += __uint_as_float(raw.z << 16); acc[5] += __uint_as_float(raw.z & 0xFFFF0000u);
+  acc[6] += __uint_as_float(raw.w << 16); acc[7] += __uint_as_float(raw.w & 0xFFFF0000u);
+}
 __device__ __forceinline__ uint16_t bf16_bits(float x) {
   __nv_bfloat16 h = __float2bfloat16_rn(x);
   return *reinterpret_cast<uint16_t*>(&h);

@@ -184,6 +184,7 @@ struct PullArgs {
   int dim;
   int dz_scaled;                           // dz rows already divided by deg (tcgen05 epilogue)
   const uint16_t* hb; int64_t hb_pitch;    // if set: the ReLU mask from bf16 H (bf16 mode, reading R11)
+  const uint16_t* dzb; int64_t dzb_pitch;  // if set: dZ / deg as bf16 rows instead of dz (reading R13)
 };
 cudaError_t launch_pull_bwd(const PullArgs& a, cudaStream_t st);
 

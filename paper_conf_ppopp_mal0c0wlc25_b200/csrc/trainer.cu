@@ -341,6 +341,10 @@ apt_status apt_trainer_create(apt_ctx* c, const apt_graph* g, const apt_fstore* 
       //  allocated: measured on products, the 2-byte mask stores cost the projection more
       //  than the pull saves by not reading H -- 78 vs 66 us forward, 72 vs 74 us backward)
       if (l > 1) L.dZ = A.alloc<float>(L.max_rows * L.zf_pitch, true);
+      if (l > 1 && m->dtype == APT_BF16) {   // reading R13: the mean's backward reads dZ / deg in bf16
+        L.dzb_pitch = round_up(L.d_in, 8);
+        L.dZb = A.alloc<uint16_t>(L.max_rows * L.dzb_pitch, true);
+      }
       L.W = A.alloc<float>(int64_t(L.d_out) * L.d_in, true);
       L.b = A.alloc<float>(L.d_out, true);
       L.Wb = A.alloc<uint16_t>(int64_t(L.d_out) * L.wb_pitch, true);
@@ -660,6 +664,13 @@ apt_status layer1_fwd_gdp(apt_trainer* t, RankState& rs, bool time_it) {
                  t->K > 1 ? 1 : 0, L.H, nullptr, nullptr, nullptr);
 }
 
+// Reading R13 (bf16 mode): the projection's backward writes dZ / deg as bf16 rows for
+// the mean's backward.  APT_BF16_DZ=0 keeps fp32 rows (A/B).
+static bool bf16_dz_enabled() {
+  const char* e = std::getenv("APT_BF16_DZ");
+  return !e || atoi(e) != 0;
+}
+
 // The output layer as one kernel (outlayer.cu): bf16 mode, K >= 2, <= 64 classes,
 // input width <= 256, opt-in with APT_FUSED_OUT=1 (read when the step is built).
 // Measured on products: faster alone (0.266 vs 0.272 ms with the
@@ -726,6 +737,7 @@ apt_status upper_bwd(apt_trainer* t, RankState& rs) {
                                bf ? L.zb_pitch : L.zf_pitch, L.n_rows, L.max_rows, L.d_in, L.dW, L.db, L.d_in, c->side);
     if (s != APT_OK) return s;
     int dz_scaled = 0;
+    const uint16_t* dzb = nullptr;
     if (l == t->K && fused_out(t, rs)) {
       dz_scaled = 1;   // dZ / deg came with the fused output layer
     } else
@@ -735,6 +747,7 @@ apt_status upper_bwd(apt_trainer* t, RankState& rs) {
                    L.dZ, L.zf_pitch, nullptr, nullptr, nullptr, 1};
       g.row_div_indptr = hp.indptr;   // dZ / deg once per row (the pull then only sums)
       g.b_early = 1;
+      if (L.dZb && bf16_dz_enabled()) { g.Yb = L.dZb; g.yb_pitch = L.dzb_pitch; dzb = L.dZb; }   // R13
       CK(c, launch_tc_gemm(g, c->stream));
       dz_scaled = 1;
     } else {
@@ -759,6 +772,7 @@ apt_status upper_bwd(apt_trainer* t, RankState& rs) {
                 bf ? nullptr : P.G, P.h_pitch, bf ? P.Gb : nullptr, P.gb_pitch, hp.counts, P.max_rows, L.d_in,
                 dz_scaled};
     if (P.Hb && !mk) { pa.h = nullptr; pa.hb = P.Hb; pa.hb_pitch = P.hb_pitch; }   // R11: mask from bf16 H
+    if (dzb) { pa.dzb = dzb; pa.dzb_pitch = L.dzb_pitch; }                            // R13: bf16 dZ / deg
     CK(c, launch_pull_bwd(pa, c->stream));
     c->launches += 2;
   }

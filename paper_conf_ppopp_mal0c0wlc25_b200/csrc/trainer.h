@@ -45,6 +45,8 @@ struct Layer {
   bool mk_valid = false;            // the last forward wrote Mk (tcgen05 epilogue on this rank)
   int64_t gb_pitch = 0;
   float* dZ = nullptr;              // [max_rows x zf_pitch] scratch (l > 1)
+  uint16_t* dZb = nullptr;          // bf16 mode: (G W) / deg in bf16 [max_rows x dzb_pitch] (reading R13)
+  int64_t dzb_pitch = 0;
   float* W = nullptr;               // [d_out x d_in] fp32 master
   float* b = nullptr;
   uint16_t* Wb = nullptr;           // [d_out x wb_pitch] bf16 copy (tensor cores)

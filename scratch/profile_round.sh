@@ -11,6 +11,6 @@ timeout 600 python bench.py --impl reference --steps 3 --warmup 3 > gpurun_out/f
 timeout 400 ncu --metrics gpu__time_duration.sum --clock-control none --csv --log-file gpurun_out/final_launches.csv \
   python bench.py --steps 5 --warmup 3 --no-cpu-baseline --no-planner > /dev/null 2>&1
 timeout 600 ncu --set full --clock-control none --import-source on \
-  -k regex:'agg_l1_kernel|rowtile_kernel|pull_bwd_kernel|wgrad_kernel|sample_kernel|compact_scan|outlayer_kernel|agg_kernel' \
+  -k regex:'agg_l1|rowtile_kernel|pull_bwd_kernel|wgrad_kernel|sample_kernel|compact_scan|outlayer_kernel|agg_kernel' \
   --launch-skip 40 -c 24 -o gpurun_out/final_full python bench.py --steps 3 --warmup 3 --no-cpu-baseline --no-planner \
   > gpurun_out/final_ncu_full.log 2>&1
