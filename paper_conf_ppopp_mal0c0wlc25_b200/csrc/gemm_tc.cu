@@ -604,7 +604,9 @@ cudaError_t launch_tc_wgrad(const TcWgradArgs& a, cudaStream_t st) {
   }
   const int mt = int(ceil_div(a.d_out, BM));
   const int64_t kbs = std::max<int64_t>(1, ceil_div(a.rows_max, BK));
-  const int splits = int(std::max<int64_t>(1, std::min<int64_t>(kbs, sm_count() / mt)));
+  // row splits: one CTA per SM (A/B APT_WG_SPLITS_PER_SM = 1 / 2: 0.207 / 0.224 ms; ring depth 3 / 6: same)
+  static const int per_sm = [] { const char* v = std::getenv("APT_WG_SPLITS_PER_SM"); return v ? std::max(1, atoi(v)) : 1; }();
+  const int splits = int(std::max<int64_t>(1, std::min<int64_t>(kbs, int64_t(per_sm) * sm_count() / mt)));
   launch_pdl(wgrad_kernel, dim3(dim3(splits, mt)), dim3(THREADS), smem, st, mg, mz, p);
   return cudaGetLastError();
 }
