@@ -42,6 +42,23 @@ __global__ void csc_fill_kernel(const int32_t* __restrict__ indptr, const int32_
   }
 }
 
+// The same fill with one thread per (row, slot) of the sampler's fixed fanout k: no
+// per-row loop of dependent atomics (A/B: APT_CSC_SLOTS=0 keeps the row loop).
+__global__ void csc_fill_slots_kernel(const int32_t* __restrict__ indptr, const int32_t* __restrict__ indices,
+                                      const int32_t* __restrict__ n_dst_p, int k, const int32_t* __restrict__ csc_ptr,
+                                      int32_t* __restrict__ cnt, int2* __restrict__ csc_dst) {
+  APT_PDL_PROLOGUE();
+  const int64_t slots = int64_t(*n_dst_p) * k;
+  for (int64_t s = int64_t(blockIdx.x) * blockDim.x + threadIdx.x; s < slots; s += int64_t(gridDim.x) * blockDim.x) {
+    const int64_t v = s / k;
+    const int q = int(s - v * k);
+    const int b = indptr[v], deg = indptr[v + 1] - b;
+    if (q >= deg) continue;
+    const int u = indices[b + q];
+    csc_dst[csc_ptr[u] + atomicSub(cnt + u, 1) - 1] = make_int2(int32_t(v), deg);
+  }
+}
+
 cudaError_t launch_csc_build(const CscArgs& a, cudaStream_t st) {
   const int64_t T = 256;
   const int64_t cap = a.grid_cap > 0 ? a.grid_cap : 148 * 16;
@@ -49,6 +66,13 @@ cudaError_t launch_csc_build(const CscArgs& a, cudaStream_t st) {
   launch_pdl(csc_count_kernel, dim3(ge), dim3(T), 0, st, a.indptr, a.indices, a.n_edges, a.cnt);
   cudaError_t e = launch_scan_counts(a.cnt, a.n_src, a.max_src, a.csc_ptr, a.csc_total, a.ws, st);
   if (e != cudaSuccess) return e;
+  static const int slots = [] { const char* v = std::getenv("APT_CSC_SLOTS"); return v ? atoi(v) : 1; }();
+  if (slots && a.k > 0) {
+    const int64_t gs = std::max<int64_t>(1, std::min<int64_t>(ceil_div(a.max_dst * a.k, T), cap));
+    launch_pdl(csc_fill_slots_kernel, dim3(gs), dim3(T), 0, st, a.indptr, a.indices, a.n_dst, a.k, a.csc_ptr, a.cnt,
+               a.csc_dst);
+    return cudaGetLastError();
+  }
   const int64_t gd = std::max<int64_t>(1, std::min<int64_t>(ceil_div(a.max_dst, T), cap));
   launch_pdl(csc_fill_kernel, dim3(gd), dim3(T), 0, st, a.indptr, a.indices, a.n_dst, a.csc_ptr, a.cnt, a.csc_dst);
   return cudaGetLastError();

@@ -168,6 +168,7 @@ struct CscArgs {
   int2* csc_dst;       // [max_edges] (v, deg(v)) per in-edge
   int32_t* ws;         // scan workspace, >= 2*ceil(max_src/2048) + 8
   int64_t grid_cap;    // max blocks of the grid-stride kernels (0: default)
+  int k;               // > 0: rows have at most k edges (sampler fanout): fill by (row, slot) in parallel
 };
 cudaError_t launch_csc_build(const CscArgs& a, cudaStream_t st);
 

@@ -584,7 +584,7 @@ apt_status phase_sample(apt_trainer* t, RankState& rs, SampleSet& ss, bool from_
         cs_st = c->side;
       }
       CscArgs cs{hp.indptr, hp.indices, hp.n_dst, hp.max_dst, hp.counts + 1, hp.max_dst * hp.k, hp.counts,
-                 hp.max_src, hp.csc_cnt, hp.csc_ptr, hp.counts + 2, hp.csc_dst, hp.csc_ws, cap};
+                 hp.max_src, hp.csc_cnt, hp.csc_ptr, hp.counts + 2, hp.csc_dst, hp.csc_ws, cap, hp.k};
       CK(c, launch_csc_build(cs, cs_st));
       c->launches += 4;
     }
