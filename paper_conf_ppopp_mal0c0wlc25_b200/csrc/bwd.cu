@@ -15,11 +15,22 @@ namespace apt {
 
 cudaError_t launch_scan_counts(const int32_t* cnt, const int32_t* n_dev, int64_t max_n, int32_t* out, int32_t* total,
                                int32_t* ws, cudaStream_t st);
+int scan_tiles(int64_t max_n);
+cudaError_t launch_scan_counts_prereset(const int32_t* cnt, const int32_t* n_dev, int64_t max_n, int32_t* out,
+                                        int32_t* total, int32_t* ws, cudaStream_t st);
 
-// in-degree of every local source of the block
+// in-degree of every local source of the block; also zeroes the next scan's status
+// words and ticket (one launch fewer on the sampling branch)
 __global__ void csc_count_kernel(const int32_t* __restrict__ indptr, const int32_t* __restrict__ indices,
-                                 const int32_t* __restrict__ n_edges_p, int32_t* __restrict__ cnt) {
+                                 const int32_t* __restrict__ n_edges_p, int32_t* __restrict__ cnt,
+                                 uint64_t* __restrict__ scan_st, int scan_nb, int32_t* __restrict__ scan_ticket) {
   APT_PDL_PROLOGUE();
+  if (scan_st) {
+    for (int64_t i = int64_t(blockIdx.x) * blockDim.x + threadIdx.x; i <= scan_nb; i += int64_t(gridDim.x) * blockDim.x) {
+      if (i < scan_nb) scan_st[i] = 0;
+      else *scan_ticket = 0;
+    }
+  }
   const int64_t E = *n_edges_p;
   for (int64_t e = int64_t(blockIdx.x) * blockDim.x + threadIdx.x; e < E; e += int64_t(gridDim.x) * blockDim.x)
     atomicAdd(cnt + indices[e], 1);
@@ -63,8 +74,10 @@ cudaError_t launch_csc_build(const CscArgs& a, cudaStream_t st) {
   const int64_t T = 256;
   const int64_t cap = a.grid_cap > 0 ? a.grid_cap : 148 * 16;
   const int64_t ge = std::max<int64_t>(1, std::min<int64_t>(ceil_div(a.max_edges, T), cap));
-  launch_pdl(csc_count_kernel, dim3(ge), dim3(T), 0, st, a.indptr, a.indices, a.n_edges, a.cnt);
-  cudaError_t e = launch_scan_counts(a.cnt, a.n_src, a.max_src, a.csc_ptr, a.csc_total, a.ws, st);
+  const int nb = scan_tiles(a.max_src);
+  launch_pdl(csc_count_kernel, dim3(ge), dim3(T), 0, st, a.indptr, a.indices, a.n_edges, a.cnt,
+             reinterpret_cast<uint64_t*>(a.ws), nb, a.ws + 2 * nb + 2);
+  cudaError_t e = launch_scan_counts_prereset(a.cnt, a.n_src, a.max_src, a.csc_ptr, a.csc_total, a.ws, st);
   if (e != cudaSuccess) return e;
   static const int slots = [] { const char* v = std::getenv("APT_CSC_SLOTS"); return v ? atoi(v) : 1; }();
   if (slots && a.k > 0) {

@@ -174,7 +174,7 @@ struct DrySampler {
     dst_bm = A.alloc<uint32_t>(n_words, true);
     new_bm = A.alloc<uint32_t>(n_words, true);
     pos = A.alloc<int32_t>(g->n, false);
-    partials = A.alloc<int32_t>(2 * ceil_div(n_words, 2048) + 8, false);
+    partials = A.alloc<int32_t>(2 * ceil_div(n_words, kScanWsTile) + 8, false);
     step_dev = A.alloc<uint64_t>(1, true);
     hops.resize(K);
     int64_t maxF = B0;
@@ -190,7 +190,7 @@ struct DrySampler {
       hp.cnt = A.alloc<int32_t>(maxF, true);
       hp.nbr = A.alloc<int32_t>(maxF * hp.k, false);
       hp.counts = A.alloc<int32_t>(4, true);
-      hp.part2 = A.alloc<int32_t>(2 * ceil_div(maxF, 2048) + 8, false);
+      hp.part2 = A.alloc<int32_t>(2 * ceil_div(maxF, kScanWsTile) + 8, false);
       if (h + 1 < K) {
         hp.src = A.alloc<int32_t>(hp.max_src, false);
         hp.indptr = A.alloc<int32_t>(maxF + 1, true);

@@ -5,6 +5,10 @@
 
 namespace apt {
 
+// Workspace granularity of the single-pass scans (sample.cu): one status word pair per
+// tile; the scans' tile (kScanThreads * kScanItems) must be a multiple of it.
+constexpr int kScanWsTile = 512;
+
 // ---------------------------------------------------------------- sample.cu
 struct SampleArgs {
   const int64_t* indptr;
@@ -38,8 +42,8 @@ struct CompactArgs {
   int32_t* indptr;             // [max_dst + 1]
   int32_t* indices;            // [max_dst * k]
   int32_t* n_edges;
-  int32_t* partials;           // scan workspace (>= n_words/2048 + 2)
-  int32_t* partials2;          // scan workspace (>= max_dst/2048 + 2)
+  int32_t* partials;           // scan workspace (>= 2 * n_words / kScanWsTile + 8)
+  int32_t* partials2;          // scan workspace (>= 2 * max_dst / kScanWsTile + 8)
   int64_t grid_cap;            // max blocks of the grid-stride kernels (0: default)
 };
 cudaError_t launch_compact(const CompactArgs& a, cudaStream_t st);
@@ -166,7 +170,7 @@ struct CscArgs {
   int32_t* csc_ptr;    // [max_src + 1]
   int32_t* csc_total;  // [1]
   int2* csc_dst;       // [max_edges] (v, deg(v)) per in-edge
-  int32_t* ws;         // scan workspace, >= 2*ceil(max_src/2048) + 8
+  int32_t* ws;         // scan workspace, >= 2*ceil(max_src/kScanWsTile) + 8
   int64_t grid_cap;    // max blocks of the grid-stride kernels (0: default)
   int k;               // > 0: rows have at most k edges (sampler fanout): fill by (row, slot) in parallel
 };

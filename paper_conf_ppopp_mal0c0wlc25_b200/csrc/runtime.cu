@@ -446,7 +446,7 @@ apt_status apt_sample(apt_ctx* c, const apt_graph* g, const int64_t* seeds_dev, 
   uint32_t* new_bm = b->arena.alloc<uint32_t>(n_words, true);
   int32_t* pos = b->arena.alloc<int32_t>(g->n, false);
   int64_t maxF = n_seeds;
-  int64_t max_part = 2 * ceil_div(n_words, 2048) + 8;
+  int64_t max_part = 2 * ceil_div(n_words, kScanWsTile) + 8;
   int32_t* counts = b->arena.alloc<int32_t>(4 * K + 4, true);
   uint64_t* step_dev = b->arena.alloc<uint64_t>(1, false);
   int32_t* seeds32 = b->arena.alloc<int32_t>(n_seeds, false);
@@ -483,7 +483,7 @@ apt_status apt_sample(apt_ctx* c, const apt_graph* g, const int64_t* seeds_dev, 
     int32_t* src = b->arena.alloc<int32_t>(maxS, false);
     int32_t* indptr = b->arena.alloc<int32_t>(maxF + 1, true);
     int32_t* indices = b->arena.alloc<int32_t>(maxF * k, false);
-    int32_t* part2 = b->arena.alloc<int32_t>(2 * ceil_div(maxF, 2048) + 8, false);
+    int32_t* part2 = b->arena.alloc<int32_t>(2 * ceil_div(maxF, kScanWsTile) + 8, false);
     if (!cnt || !nbr || !src || !indptr || !indices || !partials || !part2) {
       apt_batch_destroy(b);
       return set_err(c, APT_E_OOM, "apt_sample: out of device memory");

@@ -25,7 +25,7 @@ namespace apt {
 //  Philox_SAMPLE(seed; {v_lo, v_hi, step, (h<<24)|(t>>2)}), r = (w*(j+1))>>32,
 //  insert (r already chosen ? j : r); positions ascending.
 template <int KS>  // KS = ceil(k/32) slots per lane
-__global__ void __launch_bounds__(256) sample_kernel(const int64_t* __restrict__ indptr,
+__global__ void __launch_bounds__(256, (KS <= 2 ? 8 : 4)) sample_kernel(const int64_t* __restrict__ indptr,
                                                      const int32_t* __restrict__ indices,
                                                      const int32_t* __restrict__ frontier,
                                                      const int32_t* __restrict__ n_frontier, int k,
@@ -37,10 +37,20 @@ __global__ void __launch_bounds__(256) sample_kernel(const int64_t* __restrict__
   const int64_t F = *n_frontier;
   const uint32_t step = uint32_t(*step_ptr);
   const int64_t nwarps = int64_t(gridDim.x) * (blockDim.x >> 5);
-  for (int64_t i = (int64_t(blockIdx.x) * blockDim.x + threadIdx.x) >> 5; i < F; i += nwarps) {
-    const int v = frontier[i];
-    const int64_t base = indptr[v];
-    const int64_t deg = indptr[v + 1] - base;
+  // software pipeline over the warp's frontier nodes: the next node's CSR bounds and
+  // the id after it are loaded while the current node draws and gathers, so a node's
+  // chain starts at its neighbour loads (frontier -> indptr -> indices was 3 deep)
+  int64_t i = (int64_t(blockIdx.x) * blockDim.x + threadIdx.x) >> 5;
+  int v_cur = i < F ? frontier[i] : 0;
+  int64_t b0 = i < F ? indptr[v_cur] : 0, b1 = i < F ? indptr[v_cur + 1] : 0;
+  int v_nxt = i + nwarps < F ? frontier[i + nwarps] : 0;
+  for (; i < F; i += nwarps) {
+    const int v = v_cur;
+    const int64_t base = b0;
+    const int64_t deg = b1 - b0;
+    if (i + nwarps < F) { b0 = indptr[v_nxt]; b1 = indptr[v_nxt + 1]; }
+    v_cur = v_nxt;
+    v_nxt = i + 2 * nwarps < F ? frontier[i + 2 * nwarps] : 0;
     int32_t* out = nbr + i * k;
     if (deg <= k) {
       for (int q = lane; q < deg; q += 32) out[q] = indices[base + q];
@@ -119,7 +129,8 @@ cudaError_t launch_sample(const SampleArgs& a, cudaStream_t st) {
 // ------------------------------------------------------ device-wide scan ----
 // Three-kernel reduce-then-scan over int32 values: partials -> spine -> emit.
 constexpr int kScanThreads = 256;
-constexpr int kScanItems = 8;
+constexpr int kScanItems = 4;   // 1 024-word tiles: 8 -> 4 doubles the CTAs of the look-back scans
+static_assert((kScanThreads * kScanItems) % kScanWsTile == 0, "scan workspace granularity");
 constexpr int kScanTile = kScanThreads * kScanItems;
 
 template <typename T>
@@ -350,6 +361,18 @@ __global__ void __launch_bounds__(kScanThreads) count_scan_kernel(CntScanOp c, u
   if (threadIdx.x == 0) tk = atomicAdd(ticket, 1);
   __syncthreads();
   scan_tile(c, st, tk, nb);
+}
+
+// The same scan when the preceding kernel already zeroed the status words and the
+// ticket (ws: nb = scan_tiles(max_n) status pairs, ticket at ws + 2 nb + 2).
+int scan_tiles(int64_t max_n) { return int(std::max<int64_t>(1, ceil_div(max_n, kScanTile))); }
+cudaError_t launch_scan_counts_prereset(const int32_t* cnt, const int32_t* n_dev, int64_t max_n, int32_t* out,
+                                        int32_t* total, int32_t* ws, cudaStream_t st) {
+  const int nb = scan_tiles(max_n);
+  CntScanOp cop{cnt, n_dev, out, total};
+  launch_pdl(count_scan_kernel, dim3(nb), dim3(kScanThreads), 0, st, cop, reinterpret_cast<uint64_t*>(ws), nb,
+             ws + 2 * nb + 2);
+  return cudaGetLastError();
 }
 
 cudaError_t launch_scan_counts(const int32_t* cnt, const int32_t* n_dev, int64_t max_n, int32_t* out, int32_t* total,

@@ -277,7 +277,7 @@ apt_status apt_trainer_create(apt_ctx* c, const apt_graph* g, const apt_fstore* 
     rs.dst_bm = A.alloc<uint32_t>(n_words, true);
     rs.new_bm = A.alloc<uint32_t>(n_words, true);
     rs.pos = A.alloc<int32_t>(g->n, false);
-    rs.partials = A.alloc<int32_t>(2 * ceil_div(n_words, 2048) + 8, false);
+    rs.partials = A.alloc<int32_t>(2 * ceil_div(n_words, kScanWsTile) + 8, false);
     for (int q = 0; q < 2; ++q) {
       SampleSet& ss = rs.sset[q];
       ss.seeds = A.alloc<int32_t>(std::max<int64_t>(B0, int64_t(C) * m->batch), false);
@@ -297,7 +297,7 @@ apt_status apt_trainer_create(apt_ctx* c, const apt_graph* g, const apt_fstore* 
         hp.cnt = A.alloc<int32_t>(maxF, true);
         hp.nbr = A.alloc<int32_t>(maxF * hp.k, false);
         hp.counts = A.alloc<int32_t>(4, true);
-        hp.part2 = A.alloc<int32_t>(2 * ceil_div(maxF, 2048) + 8, false);
+        hp.part2 = A.alloc<int32_t>(2 * ceil_div(maxF, kScanWsTile) + 8, false);
         if (h + 1 < K) {   // the layer-1 hop is consumed in ELL form (fused gather), no CSR needed
           hp.src = A.alloc<int32_t>(hp.max_src, false);
           hp.indptr = A.alloc<int32_t>(maxF + 1, true);
@@ -305,7 +305,7 @@ apt_status apt_trainer_create(apt_ctx* c, const apt_graph* g, const apt_fstore* 
           hp.csc_cnt = A.alloc<int32_t>(hp.max_src, true);
           hp.csc_ptr = A.alloc<int32_t>(hp.max_src + 1, true);
           hp.csc_dst = A.alloc<int2>(maxF * hp.k, false);
-          hp.csc_ws = A.alloc<int32_t>(2 * ceil_div(hp.max_src, 2048) + 8, false);
+          hp.csc_ws = A.alloc<int32_t>(2 * ceil_div(hp.max_src, kScanWsTile) + 8, false);
         }
         dst = hp.src;
         n_dst = hp.counts;
@@ -586,7 +586,7 @@ apt_status phase_sample(apt_trainer* t, RankState& rs, SampleSet& ss, bool from_
       CscArgs cs{hp.indptr, hp.indices, hp.n_dst, hp.max_dst, hp.counts + 1, hp.max_dst * hp.k, hp.counts,
                  hp.max_src, hp.csc_cnt, hp.csc_ptr, hp.counts + 2, hp.csc_dst, hp.csc_ws, cap, hp.k};
       CK(c, launch_csc_build(cs, cs_st));
-      c->launches += 4;
+      c->launches += 3;   // count (+ scan reset), scan, fill
     }
   }
   if (fork_csc && t->K > 1) {
