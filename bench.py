@@ -403,7 +403,7 @@ def run_apt(args, cfg):
                      "frac": (achieved / hbm_peak) if achieved else None, "traffic": traffic,
                      "traffic_source": traffic_src, "algorithmic_bytes_per_launch": sum(agg_bytes) / len(agg_bytes),
                      "kernel": "gat_fwd_kernel (layer-1 fused gather+attention+weighted sums)" if GAT_HEADS
-                     else "agg_kernel (layer-1 fused gather+mean)",
+                     else "agg_l1_pf_kernel (layer-1 fused gather+mean)",
                      "peak_source": "MEASURED_PEAKS.json hbm_gbs" if peaks else "fallback 6.65 TB/s",
                      "share_of_step": mean_agg / ms_local},
         "step_roofline": step_roofline(step_bytes, hbm_peak, ms) if step_bytes else None,

@@ -75,8 +75,9 @@ cudaError_t launch_csc_build(const CscArgs& a, cudaStream_t st) {
   const int64_t cap = a.grid_cap > 0 ? a.grid_cap : 148 * 16;
   const int64_t ge = std::max<int64_t>(1, std::min<int64_t>(ceil_div(a.max_edges, T), cap));
   const int nb = scan_tiles(a.max_src);
-  launch_pdl(csc_count_kernel, dim3(ge), dim3(T), 0, st, a.indptr, a.indices, a.n_edges, a.cnt,
-             reinterpret_cast<uint64_t*>(a.ws), nb, a.ws + 2 * nb + 2);
+  if (!a.counted)
+    launch_pdl(csc_count_kernel, dim3(ge), dim3(T), 0, st, a.indptr, a.indices, a.n_edges, a.cnt,
+               reinterpret_cast<uint64_t*>(a.ws), nb, a.ws + 2 * nb + 2);
   cudaError_t e = launch_scan_counts_prereset(a.cnt, a.n_src, a.max_src, a.csc_ptr, a.csc_total, a.ws, st);
   if (e != cudaSuccess) return e;
   static const int slots = [] { const char* v = std::getenv("APT_CSC_SLOTS"); return v ? atoi(v) : 1; }();

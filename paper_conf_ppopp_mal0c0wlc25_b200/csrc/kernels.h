@@ -45,8 +45,12 @@ struct CompactArgs {
   int32_t* partials;           // scan workspace (>= 2 * n_words / kScanWsTile + 8)
   int32_t* partials2;          // scan workspace (>= 2 * max_dst / kScanWsTile + 8)
   int64_t grid_cap;            // max blocks of the grid-stride kernels (0: default)
+  // optional: the block transpose's in-degree count, done while the indices are mapped
+  // (csc_cnt zero on entry), and the reset of its scan's status words / ticket
+  int32_t* csc_cnt; uint64_t* csc_st; int csc_nb; int32_t* csc_ticket;
 };
 cudaError_t launch_compact(const CompactArgs& a, cudaStream_t st);
+int scan_tiles(int64_t max_n);   // status pairs of a look-back scan over max_n items
 
 struct SeedArgs {
   const int32_t* perm;
@@ -173,6 +177,7 @@ struct CscArgs {
   int32_t* ws;         // scan workspace, >= 2*ceil(max_src/kScanWsTile) + 8
   int64_t grid_cap;    // max blocks of the grid-stride kernels (0: default)
   int k;               // > 0: rows have at most k edges (sampler fanout): fill by (row, slot) in parallel
+  int counted;         // cnt already holds the in-degrees and the scan workspace is reset (launch_compact)
 };
 cudaError_t launch_csc_build(const CscArgs& a, cudaStream_t st);
 

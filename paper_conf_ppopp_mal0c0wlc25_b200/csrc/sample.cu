@@ -184,8 +184,15 @@ __global__ void map_indices_kernel(const int32_t* __restrict__ dst, const int32_
                                    const int32_t* __restrict__ nbr, const int32_t* __restrict__ n_dst,
                                    int k, const int32_t* __restrict__ indptr,
                                    const int32_t* __restrict__ pos, int32_t* __restrict__ indices,
-                                   uint32_t* __restrict__ dst_bm) {
+                                   uint32_t* __restrict__ dst_bm, int32_t* __restrict__ csc_cnt,
+                                   uint64_t* __restrict__ csc_st, int csc_nb, int32_t* __restrict__ csc_ticket) {
   APT_PDL_PROLOGUE();
+  if (csc_st) {
+    for (int64_t i = int64_t(blockIdx.x) * blockDim.x + threadIdx.x; i <= csc_nb; i += int64_t(gridDim.x) * blockDim.x) {
+      if (i < csc_nb) csc_st[i] = 0;
+      else *csc_ticket = 0;
+    }
+  }
   const int64_t slots = int64_t(*n_dst) * k;
   for (int64_t s = int64_t(blockIdx.x) * blockDim.x + threadIdx.x; s < slots; s += int64_t(gridDim.x) * blockDim.x) {
     const int64_t i = s / k;
@@ -195,7 +202,9 @@ __global__ void map_indices_kernel(const int32_t* __restrict__ dst, const int32_
       atomicAnd(dst_bm + (v >> 5), ~(1u << (v & 31)));
     }
     if (q >= cnt[i]) continue;
-    indices[indptr[i] + q] = pos[nbr[s]];
+    const int u = pos[nbr[s]];
+    indices[indptr[i] + q] = u;
+    if (csc_cnt) atomicAdd(csc_cnt + u, 1);   // in-degree of local source u (block transpose)
   }
 }
 
@@ -400,7 +409,8 @@ cudaError_t launch_compact(const CompactArgs& a, cudaStream_t st) {
   CntScanOp cop{a.cnt, a.n_dst, a.indptr, a.n_edges};
   launch_pdl(compact_scan_kernel, dim3(nbA + nbB), dim3(kScanThreads), 0, st, bop, stA, nbA, cop, stB, nbB, ticket);
   launch_pdl(map_indices_kernel, dim3(gm), dim3(T), 0, st, a.dst, a.cnt, a.nbr, a.n_dst, a.k, a.indptr,
-                                                                  a.pos, a.indices, a.dst_bm);
+                                                                  a.pos, a.indices, a.dst_bm, a.csc_cnt, a.csc_st, a.csc_nb,
+                                                                  a.csc_ticket);
   return cudaGetLastError();
 }
 

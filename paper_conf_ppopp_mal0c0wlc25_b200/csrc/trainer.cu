@@ -574,6 +574,12 @@ apt_status phase_sample(apt_trainer* t, RankState& rs, SampleSet& ss, bool from_
     if (h + 1 < t->K) {
       CompactArgs ca{hp.dst, hp.n_dst, hp.max_dst, hp.cnt, hp.nbr, hp.k, rs.dst_bm, rs.new_bm, n_words, rs.pos, hp.src,
                      hp.counts, hp.indptr, hp.indices, hp.counts + 1, rs.partials, hp.part2, cap};
+      static const int count_in_map = [] { const char* v = std::getenv("APT_CSC_COUNT_IN_MAP"); return v ? atoi(v) : 1; }();
+      if (count_in_map) {   // the transpose's in-degrees counted while the indices are mapped
+        const int nb = scan_tiles(hp.max_src);
+        ca.csc_cnt = hp.csc_cnt; ca.csc_st = reinterpret_cast<uint64_t*>(hp.csc_ws); ca.csc_nb = nb;
+        ca.csc_ticket = hp.csc_ws + 2 * nb + 2;
+      }
       CK(c, launch_compact(ca, st));
       c->launches += 3;
       // transpose of this block for the pull-form mean backward
@@ -584,9 +590,10 @@ apt_status phase_sample(apt_trainer* t, RankState& rs, SampleSet& ss, bool from_
         cs_st = c->side;
       }
       CscArgs cs{hp.indptr, hp.indices, hp.n_dst, hp.max_dst, hp.counts + 1, hp.max_dst * hp.k, hp.counts,
-                 hp.max_src, hp.csc_cnt, hp.csc_ptr, hp.counts + 2, hp.csc_dst, hp.csc_ws, cap, hp.k};
+                 hp.max_src, hp.csc_cnt, hp.csc_ptr, hp.counts + 2, hp.csc_dst, hp.csc_ws, cap, hp.k,
+                 ca.csc_cnt ? 1 : 0};
       CK(c, launch_csc_build(cs, cs_st));
-      c->launches += 3;   // count (+ scan reset), scan, fill
+      c->launches += ca.csc_cnt ? 2 : 3;   // (count + scan reset,) scan, fill
     }
   }
   if (fork_csc && t->K > 1) {
