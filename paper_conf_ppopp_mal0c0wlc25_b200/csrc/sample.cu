@@ -98,12 +98,84 @@ __global__ void __launch_bounds__(256, (KS <= 2 ? 8 : 4)) sample_kernel(const in
   }
 }
 
+// Fanout <= 16: two frontier nodes per warp, one per 16-lane half (k of 16 lanes busy
+// instead of k of 32), the same draws and the same Floyd / ranking steps as
+// sample_kernel with every shuffle confined to the half (bit-identical output).
+__global__ void __launch_bounds__(256, 6) sample_g16_kernel(const int64_t* __restrict__ indptr,
+                                                            const int32_t* __restrict__ indices,
+                                                            const int32_t* __restrict__ frontier,
+                                                            const int32_t* __restrict__ n_frontier, int k,
+                                                            uint2 key, const uint64_t* __restrict__ step_ptr,
+                                                            int hop, int32_t* __restrict__ cnt,
+                                                            int32_t* __restrict__ nbr) {
+  APT_PDL_PROLOGUE();
+  const int lane = lane_id();
+  const int g = lane >> 4, l = lane & 15;
+  const uint32_t gmask = g ? 0xFFFF0000u : 0x0000FFFFu;
+  const int64_t F = *n_frontier;
+  const uint32_t step = uint32_t(*step_ptr);
+  const int64_t nwarps = int64_t(gridDim.x) * (blockDim.x >> 5);
+  const int64_t stride = 2 * nwarps;
+  // node of this half: i = 2 * warp + g; the next node's CSR bounds and the id after
+  // it are loaded one iteration ahead (as in sample_kernel)
+  int64_t i = ((int64_t(blockIdx.x) * blockDim.x + threadIdx.x) >> 5) * 2 + g;
+  int v_cur = i < F ? frontier[i] : 0;
+  int64_t b0 = i < F ? indptr[v_cur] : 0, b1 = i < F ? indptr[v_cur + 1] : 0;
+  int v_nxt = i + stride < F ? frontier[i + stride] : 0;
+  for (int64_t i0 = i - g; i0 < F; i0 += stride, i += stride) {   // warp-uniform loop
+    const bool valid = i < F;
+    const int v = v_cur;
+    const int64_t base = b0;
+    const int64_t deg = valid ? b1 - b0 : 0;
+    if (i + stride < F) { b0 = indptr[v_nxt]; b1 = indptr[v_nxt + 1]; }
+    v_cur = v_nxt;
+    v_nxt = i + 2 * stride < F ? frontier[i + 2 * stride] : 0;
+    int32_t* out = nbr + i * k;
+    const bool small = deg <= k;
+    // draws (only the halves that sample use them)
+    uint32_t r_me = 0;
+    if (valid && !small && l < k) {
+      const uint4 w = philox(make_uint4(uint32_t(v), 0u, step, (uint32_t(hop) << 24) | uint32_t(l >> 2)), key);
+      const uint64_t j = uint64_t(deg - k + l);
+      r_me = uint32_t((uint64_t(word_of(w, l & 3)) * (j + 1)) >> 32);
+    }
+    uint32_t chosen = 0xFFFFFFFFu;
+    for (int tt = 0; tt < k; ++tt) {   // Floyd's membership step, one draw at a time
+      const uint32_t r = __shfl_sync(0xffffffffu, r_me, tt, 16);
+      const bool hit = l < tt && chosen == r;
+      const bool member = (__ballot_sync(0xffffffffu, hit) & gmask) != 0u;
+      if (l == tt) chosen = member ? uint32_t(deg - k + tt) : r;
+    }
+    int rank = 0;
+    for (int tt = 0; tt < k; ++tt) {
+      const uint32_t o = __shfl_sync(0xffffffffu, chosen, tt, 16);
+      rank += (o < chosen) ? 1 : 0;
+    }
+    if (!valid) continue;
+    if (small) {
+      for (int q = l; q < deg; q += 16) out[q] = indices[base + q];
+      if (l == 0) cnt[i] = int32_t(deg);
+    } else {
+      if (l < k) out[rank] = indices[base + chosen];
+      if (l == 0) cnt[i] = k;
+    }
+  }
+}
+
 cudaError_t launch_sample(const SampleArgs& a, cudaStream_t st) {
   const int threads = 256;
   const int64_t warps = a.max_frontier;
   int64_t blocks = ceil_div(warps * 32, threads);
   blocks = std::max<int64_t>(1, std::min<int64_t>(blocks, a.grid_cap > 0 ? a.grid_cap : 148 * 16));
   const int ks = int(ceil_div(a.k, 32));
+  static const int g16 = [] { const char* v = std::getenv("APT_SAMPLE_G16"); return v ? atoi(v) : 1; }();
+  if (g16 && a.k <= 16) {
+    int64_t b2 = ceil_div(ceil_div(a.max_frontier, 2) * 32, threads);
+    b2 = std::max<int64_t>(1, std::min<int64_t>(b2, a.grid_cap > 0 ? a.grid_cap : 148 * 16));
+    launch_pdl(sample_g16_kernel, dim3(b2), dim3(threads), 0, st, a.indptr, a.indices, a.frontier, a.n_frontier, a.k,
+               a.key, a.step, a.hop, a.cnt, a.nbr);
+    return cudaGetLastError();
+  }
 #define APT_SAMPLE_CASE(KS)                                                                      \
   case KS:                                                                                       \
     launch_pdl(sample_kernel<KS>, dim3(blocks), dim3(threads), 0, st, a.indptr, a.indices, a.frontier, a.n_frontier, \
