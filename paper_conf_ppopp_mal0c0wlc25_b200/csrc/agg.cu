@@ -301,6 +301,9 @@ __global__ void __launch_bounds__(256, MINB) agg_l1_pf_kernel(AggArgs a, EllFsto
       for (int q = 0; q < NB; ++q) {
         const char* r = reinterpret_cast<const char*>(
             __shfl_sync(0xffffffffu, reinterpret_cast<uintptr_t>(rp), sub * 16 + ((j + q) & 15)));
+        // NB not dividing 16: slots past the 16 edge lanes wrap onto real edges, read
+        // the zero row instead (cnt <= k <= 16, so every such slot is padding)
+        if constexpr ((16 % NB) != 0) if (j + q >= 16) r = reinterpret_cast<const char*>(zrow);
         v[q] = *reinterpret_cast<const uint4*>(r + lv * 16);
       }
 #pragma unroll
@@ -349,16 +352,27 @@ cudaError_t launch_agg_fstore(const AggArgs& a, const FeatView& fv, cudaStream_t
   b.dim = fv.dim;
   const int epv = fv.dtype == kBF16 ? 8 : 4;
   const int V = int(ceil_div(b.dim, epv));
-  // variant (A/B on products, DESIGN §7): 0 agg_kernel, 1 agg_l1_kernel (NB 4), 2
+  // variant (A/B on products, DESIGN §8): 0 agg_kernel, 1 agg_l1_kernel (NB 4), 2
   // agg_l1_kernel with 8 loads in flight per lane, 4 / 5 agg_l1_pf_kernel (next row
-  // pair's indices one iteration ahead) at 40 / 48 registers.  In the step: 34.5 (1),
-  // 33.2 (4), 32.4 us (5, default); a cp.async double-buffered variant measured 38.7 us.
-  static const int variant = [] { const char* e = std::getenv("APT_AGG_VARIANT"); return e ? atoi(e) : 5; }();
-  if ((variant == 4 || variant == 5) && V <= 16 && b.k <= 16) {
+  // pair's indices one iteration ahead) at 40 / 48 registers, 6 / 7 agg_l1_pf_kernel with
+  // 5 loads in flight per lane (a fanout-10 row in two rounds) at 48 / 64 registers.
+  // In the step, grid at 16 blocks per SM: 34.5 (1), 33.2 (4), 33.2 (5), 34.5 (6),
+  // 32.4 us (7); at one resident wave: 30.5 (5), 30.2 us (7, default).
+  static const int variant = [] { const char* e = std::getenv("APT_AGG_VARIANT"); return e ? atoi(e) : 7; }();
+  // APT_AGG_BPSM: grid cap in blocks per SM; default = the instantiation's resident
+  // blocks per SM (one wave: every warp streams several row pairs, so the one-ahead
+  // index prefetch pays and there is no partial last wave)
+  static const int bpsm_env = [] { const char* e = std::getenv("APT_AGG_BPSM"); return e ? atoi(e) : 0; }();
+  if ((variant >= 4 && variant <= 7) && V <= 16 && b.k <= 16) {
+    const bool bf = fv.dtype == kBF16;
+    const int minb = !bf ? 6 : variant == 4 ? 6 : variant == 7 ? 4 : 5;
+    const int bpsm = bpsm_env > 0 ? bpsm_env : minb;
     int64_t blocks = ceil_div(ceil_div(b.max_dst, 2) * 32, 256);
-    blocks = std::max<int64_t>(1, std::min<int64_t>(blocks, 148 * 16));
-    if (fv.dtype == kBF16) {
-      if (variant == 4) launch_pdl(agg_l1_pf_kernel<8, 4, 6>, dim3(blocks), dim3(256), 0, st, b, s);
+    blocks = std::max<int64_t>(1, std::min<int64_t>(blocks, 148 * int64_t(bpsm)));
+    if (bf) {
+      if (variant == 6) launch_pdl(agg_l1_pf_kernel<8, 5, 5>, dim3(blocks), dim3(256), 0, st, b, s);
+      else if (variant == 7) launch_pdl(agg_l1_pf_kernel<8, 5, 4>, dim3(blocks), dim3(256), 0, st, b, s);
+      else if (variant == 4) launch_pdl(agg_l1_pf_kernel<8, 4, 6>, dim3(blocks), dim3(256), 0, st, b, s);
       else launch_pdl(agg_l1_pf_kernel<8, 4, 5>, dim3(blocks), dim3(256), 0, st, b, s);
     } else {
       launch_pdl(agg_l1_pf_kernel<4, 4, 6>, dim3(blocks), dim3(256), 0, st, b, s);
