@@ -166,8 +166,12 @@ static cudaError_t dispatch_agg(const AggArgs& a, const Src& s, cudaStream_t st)
   const int V = int(ceil_div(a.dim, EPV));
   const int threads = 256;
   const int rpw = V <= 16 ? 2 : 1;
+  // APT_AGGU_BPSM: grid cap in blocks per SM (A/B: 16 / 6 / 4 -> upper
+  // layers' forward 50.5 / 50.5 / 49.7 us in the step; 4 leaves room for the sampling
+  // branch and every warp streams several rows)
+  static const int bpsm = [] { const char* e = std::getenv("APT_AGGU_BPSM"); return e ? atoi(e) : 4; }();
   int64_t blocks = ceil_div(ceil_div(a.max_dst, rpw) * 32, threads);
-  blocks = std::max<int64_t>(1, std::min<int64_t>(blocks, 148 * 16));
+  blocks = std::max<int64_t>(1, std::min<int64_t>(blocks, 148 * int64_t(bpsm)));
   if (V <= 16) launch_pdl(agg_kernel<EPV, 1, 16, Src>, dim3(blocks), dim3(threads), 0, st, a, s);
   else if (V <= 32) launch_pdl(agg_kernel<EPV, 1, 32, Src>, dim3(blocks), dim3(threads), 0, st, a, s);
   else if (V <= 64) launch_pdl(agg_kernel<EPV, 2, 32, Src>, dim3(blocks), dim3(threads), 0, st, a, s);

@@ -325,8 +325,10 @@ cudaError_t launch_pull_bwd(const PullArgs& a, cudaStream_t st) {
       return cudaErrorInvalidValue;
     static const int rr = [] { const char* e = std::getenv("APT_PULL_ROWS"); return e ? atoi(e) : 2; }();
     const int Rr = rr == 4 ? 4 : 2;
-    const int64_t blocks =
-        std::max<int64_t>(1, std::min<int64_t>(ceil_div(ceil_div(round_up(a.max_src, 64), Rr) * 32, 256), 148 * 16));
+    // APT_PULL_BPSM: grid cap in blocks per SM (A/B knob)
+    static const int bpsm = [] { const char* e = std::getenv("APT_PULL_BPSM"); return e ? atoi(e) : 16; }();
+    const int64_t blocks = std::max<int64_t>(
+        1, std::min<int64_t>(ceil_div(ceil_div(round_up(a.max_src, 64), Rr) * 32, 256), 148 * int64_t(bpsm)));
     const int V8 = a.dim >> 3;
     if (Rr == 4) {
       if (V8 <= 32) launch_pdl(pull_bwd_b8_kernel<1, 4>, dim3(blocks), dim3(256), 0, st, a);
