@@ -161,17 +161,15 @@ __global__ void __launch_bounds__(256, (VPL == 1 ? 6 : 4)) agg_kernel(AggArgs a,
   }
 }
 
+// bpsm: grid cap in blocks per SM.  The upper layers' mean uses 4 (A/B: 16 /
+// 6 / 4 -> upper forward 50.5 / 50.5 / 49.7 us in the step: room for the sampling branch,
+// every warp streams several rows); the layer-1 gather from the store keeps 16.
 template <int EPV, class Src>
-static cudaError_t dispatch_agg(const AggArgs& a, const Src& s, cudaStream_t st) {
+static cudaError_t dispatch_agg(const AggArgs& a, const Src& s, int bpsm, cudaStream_t st) {
   const int V = int(ceil_div(a.dim, EPV));
   const int threads = 256;
   const int rpw = V <= 16 ? 2 : 1;
-  // APT_AGGU_BPSM: grid cap in blocks per SM (A/B: 16 / 6 / 4 -> upper
-  // layers' forward 50.5 / 50.5 / 49.7 us in the step; 4 leaves room for the sampling
-  // branch and every warp streams several rows)
-  static const int bpsm = [] { const char* e = std::getenv("APT_AGGU_BPSM"); return e ? atoi(e) : 4; }();
-  int64_t blocks = ceil_div(ceil_div(a.max_dst, rpw) * 32, threads);
-  blocks = std::max<int64_t>(1, std::min<int64_t>(blocks, 148 * int64_t(bpsm)));
+  const int64_t blocks = grid_cap(ceil_div(ceil_div(a.max_dst, rpw) * 32, threads), bpsm);
   if (V <= 16) launch_pdl(agg_kernel<EPV, 1, 16, Src>, dim3(blocks), dim3(threads), 0, st, a, s);
   else if (V <= 32) launch_pdl(agg_kernel<EPV, 1, 32, Src>, dim3(blocks), dim3(threads), 0, st, a, s);
   else if (V <= 64) launch_pdl(agg_kernel<EPV, 2, 32, Src>, dim3(blocks), dim3(threads), 0, st, a, s);
@@ -181,90 +179,13 @@ static cudaError_t dispatch_agg(const AggArgs& a, const Src& s, cudaStream_t st)
 }
 
 // ----------------------------------------------------- layer 1, branch-free loads
-// The layer-1 case (ELL from the sampler, rows of <= 16 vectors: two destination rows
-// per warp) without predicated loads: a lane whose edge is padding (past the row's
-// count, or filtered out by SNP) points at a zero row in shared memory, so every load
-// of a batch is issued unconditionally through generic addressing (feature rows in
-// global / peer / mapped-host memory, the zero row in shared memory: no hot spot).
-template <int EPV, int NB, int MINB>
-__global__ void __launch_bounds__(256, MINB) agg_l1_kernel(AggArgs a, EllFstoreSrc src) {
-  APT_PDL_PROLOGUE();
-  __shared__ uint4 zrow[16];
-  if (threadIdx.x < 16) zrow[threadIdx.x] = make_uint4(0, 0, 0, 0);
-  __syncthreads();
-  const int lane = lane_id();
-  const int sub = lane >> 4, l = lane & 15;
-  const int64_t n_dst = *a.n_dst;
-  const int V = int(ceil_div(a.dim, EPV));
-  const int lv = l < V ? l : 0;
-  const int k = src.k;
-  const int64_t nwarps = int64_t(gridDim.x) * (blockDim.x >> 5);
-  for (int64_t w = (int64_t(blockIdx.x) * blockDim.x + threadIdx.x) >> 5; w * 2 < n_dst; w += nwarps) {
-    const int64_t i = w * 2 + sub;
-    const bool valid = i < n_dst;
-    const int cnt = valid ? src.count(i) : 0;
-    const int cmax = max(cnt, __shfl_xor_sync(0xffffffffu, cnt, 16));
-    float acc[EPV];
-#pragma unroll
-    for (int q = 0; q < EPV; ++q) acc[q] = 0.f;
-    for (int e0 = 0; e0 < cmax; e0 += 16) {
-      int u = -1;
-      if (valid && e0 + l < k) u = src.node(i * k + e0 + l);
-      const bool keep = e0 + l < cnt && (!a.filt_part || a.filt_part[u] == a.keep_part);
-      const char* rp = keep ? src.row_ptr(u) : reinterpret_cast<const char*>(zrow);
-      const int m = min(16, cmax - e0);
-      for (int j = 0; j < m; j += NB) {
-        uint4 v[NB];
-#pragma unroll
-        for (int q = 0; q < NB; ++q) {
-          const char* r = reinterpret_cast<const char*>(
-              __shfl_sync(0xffffffffu, reinterpret_cast<uintptr_t>(rp), sub * 16 + ((j + q) & 15)));
-          v[q] = *reinterpret_cast<const uint4*>(r + lv * 16);
-        }
-#pragma unroll
-        for (int q = 0; q < NB; ++q) accumulate_vec<EPV>(acc, v[q]);
-      }
-    }
-    if (!valid || l >= V) continue;
-    if (a.z_ones && l == 0) a.z_bf16[i * a.z_bf16_pitch + a.dim] = 0x3F80;
-    const float fdeg = float(a.deg_override ? a.deg_override[i] : cnt);
-    const float rdeg = fdeg > 0.f ? __frcp_rn(fdeg) : 0.f;
-    float z[EPV];
-#pragma unroll
-    for (int q = 0; q < EPV; ++q) z[q] = fdeg > 0.f ? div_rn_rcp(acc[q], fdeg, rdeg) : 0.f;
-    const int c0 = l * EPV;
-    const bool full = c0 + EPV <= a.dim;
-    if (a.z_f32) {
-      float* o = a.z_f32 + i * a.z_f32_pitch + c0;
-#pragma unroll
-      for (int q = 0; q < EPV; ++q)
-        if (full || c0 + q < a.dim) o[q] = z[q];
-    }
-    if (a.z_bf16) {
-      uint16_t* o = a.z_bf16 + i * a.z_bf16_pitch + c0;
-      if (full) {
-        if constexpr (EPV == 8) {
-          *reinterpret_cast<uint4*>(o) = make_uint4(pack_bf16x2(z[0], z[1]), pack_bf16x2(z[2], z[3]),
-                                                    pack_bf16x2(z[4], z[5]), pack_bf16x2(z[6], z[7]));
-        } else {
-          *reinterpret_cast<uint2*>(o) = make_uint2(pack_bf16x2(z[0], z[1]), pack_bf16x2(z[2], z[3]));
-        }
-      } else {
-#pragma unroll
-        for (int q = 0; q < EPV; ++q) {
-          if (c0 + q < a.dim) {
-            __nv_bfloat16 h = __float2bfloat16_rn(z[q]);
-            o[q] = *reinterpret_cast<uint16_t*>(&h);
-          }
-        }
-      }
-    }
-  }
-}
-
-// agg_l1_kernel with the next row pair's count and edge ids loaded one iteration
-// ahead (fanout <= 16: one id per lane), so a row pair's critical path starts at its
-// feature-row loads instead of at the index loads.
+// The layer-1 case (ELL from the sampler, fanout <= 16, rows of <= 16 vectors: two
+// destination rows per warp, one edge id per lane) without predicated loads: a lane
+// whose edge is padding (past the row's count, or filtered out by SNP) points at a zero
+// row in shared memory, so every load of a batch is issued unconditionally through
+// generic addressing (feature rows in global / peer / mapped-host memory, the zero row
+// in shared memory: no hot spot).  The next row pair's count and edge ids are loaded
+// one iteration ahead, so a row pair's critical path starts at its feature-row loads.
 template <int EPV, int NB, int MINB>
 __global__ void __launch_bounds__(256, MINB) agg_l1_pf_kernel(AggArgs a, EllFstoreSrc src) {
   APT_PDL_PROLOGUE();
@@ -356,46 +277,23 @@ cudaError_t launch_agg_fstore(const AggArgs& a, const FeatView& fv, cudaStream_t
   b.dim = fv.dim;
   const int epv = fv.dtype == kBF16 ? 8 : 4;
   const int V = int(ceil_div(b.dim, epv));
-  // variant (A/B on products): 0 agg_kernel, 1 agg_l1_kernel (NB 4), 2
-  // agg_l1_kernel with 8 loads in flight per lane, 4 / 5 agg_l1_pf_kernel (next row
-  // pair's indices one iteration ahead) at 40 / 48 registers, 6 / 7 agg_l1_pf_kernel with
-  // 5 loads in flight per lane (a fanout-10 row in two rounds) at 48 / 64 registers.
-  // In the step, grid at 16 blocks per SM: 34.5 (1), 33.2 (4), 33.2 (5), 34.5 (6),
-  // 32.4 us (7); at one resident wave: 30.5 (5), 30.2 us (7, default).
-  static const int variant = [] { const char* e = std::getenv("APT_AGG_VARIANT"); return e ? atoi(e) : 7; }();
-  // APT_AGG_BPSM: grid cap in blocks per SM; default = the instantiation's resident
-  // blocks per SM (one wave: every warp streams several row pairs, so the one-ahead
-  // index prefetch pays and there is no partial last wave)
-  static const int bpsm_env = [] { const char* e = std::getenv("APT_AGG_BPSM"); return e ? atoi(e) : 0; }();
-  if ((variant >= 4 && variant <= 7) && V <= 16 && b.k <= 16) {
-    const bool bf = fv.dtype == kBF16;
-    const int minb = !bf ? 6 : variant == 4 ? 6 : variant == 7 ? 4 : 5;
-    const int bpsm = bpsm_env > 0 ? bpsm_env : minb;
-    int64_t blocks = ceil_div(ceil_div(b.max_dst, 2) * 32, 256);
-    blocks = std::max<int64_t>(1, std::min<int64_t>(blocks, 148 * int64_t(bpsm)));
-    if (bf) {
-      if (variant == 6) launch_pdl(agg_l1_pf_kernel<8, 5, 5>, dim3(blocks), dim3(256), 0, st, b, s);
-      else if (variant == 7) launch_pdl(agg_l1_pf_kernel<8, 5, 4>, dim3(blocks), dim3(256), 0, st, b, s);
-      else if (variant == 4) launch_pdl(agg_l1_pf_kernel<8, 4, 6>, dim3(blocks), dim3(256), 0, st, b, s);
-      else launch_pdl(agg_l1_pf_kernel<8, 4, 5>, dim3(blocks), dim3(256), 0, st, b, s);
-    } else {
-      launch_pdl(agg_l1_pf_kernel<4, 4, 6>, dim3(blocks), dim3(256), 0, st, b, s);
-    }
-    return cudaGetLastError();
-  }
-  if ((variant == 1 || variant == 2) && V <= 16) {
-    int64_t blocks = ceil_div(ceil_div(b.max_dst, 2) * 32, 256);
-    blocks = std::max<int64_t>(1, std::min<int64_t>(blocks, 148 * 16));
+  // NB 5 loads in flight per lane (a fanout-10 row in two rounds) at 64 registers, the
+  // grid one resident wave: every warp streams several row pairs, so the one-ahead index
+  // prefetch pays and there is no partial last wave (A/B in DESIGN §8: 30.2 us in the
+  // step vs 32.4 at 16 blocks per SM and 33.2-34.5 for NB 4 / 8 and 48 registers)
+  if (V <= 16 && b.k <= 16) {
     if (fv.dtype == kBF16) {
-      if (variant == 1) launch_pdl(agg_l1_kernel<8, 4, 6>, dim3(blocks), dim3(256), 0, st, b, s);
-      else launch_pdl(agg_l1_kernel<8, 8, 4>, dim3(blocks), dim3(256), 0, st, b, s);
+      auto kern = agg_l1_pf_kernel<8, 5, 4>;
+      const int64_t blocks = grid_cap(ceil_div(ceil_div(b.max_dst, 2) * 32, 256), resident_blocks(kern, 256));
+      launch_pdl(kern, dim3(blocks), dim3(256), 0, st, b, s);
     } else {
-      if (variant == 1) launch_pdl(agg_l1_kernel<4, 4, 6>, dim3(blocks), dim3(256), 0, st, b, s);
-      else launch_pdl(agg_l1_kernel<4, 8, 4>, dim3(blocks), dim3(256), 0, st, b, s);
+      auto kern = agg_l1_pf_kernel<4, 4, 6>;
+      const int64_t blocks = grid_cap(ceil_div(ceil_div(b.max_dst, 2) * 32, 256), resident_blocks(kern, 256));
+      launch_pdl(kern, dim3(blocks), dim3(256), 0, st, b, s);
     }
     return cudaGetLastError();
   }
-  return fv.dtype == kBF16 ? dispatch_agg<8>(b, s, st) : dispatch_agg<4>(b, s, st);
+  return fv.dtype == kBF16 ? dispatch_agg<8>(b, s, 16, st) : dispatch_agg<4>(b, s, 16, st);
 }
 
 cudaError_t launch_agg_csr(const AggArgs& a, cudaStream_t st) {
@@ -412,10 +310,10 @@ cudaError_t launch_agg_csr(const AggArgs& a, cudaStream_t st) {
     cudaError_t e;
     if (bf) {
       CsrSrc s{b.indptr, b.indices, a.xb + c0, a.x_pitch * 2};
-      e = dispatch_agg<8>(b, s, st);
+      e = dispatch_agg<8>(b, s, 4, st);
     } else {
       CsrSrc s{b.indptr, b.indices, a.x + c0, a.x_pitch * 4};
-      e = dispatch_agg<4>(b, s, st);
+      e = dispatch_agg<4>(b, s, 4, st);
     }
     if (e != cudaSuccess) return e;
   }
@@ -449,7 +347,7 @@ __global__ void __launch_bounds__(256) agg_bwd_kernel(const int32_t* __restrict_
 
 cudaError_t launch_agg_bwd(const int32_t* indptr, const int32_t* indices, const int32_t* n_dst, int64_t max_dst,
                            const float* dz, int64_t dz_pitch, int dim, float* dx, int64_t dx_pitch, cudaStream_t st) {
-  int64_t blocks = std::max<int64_t>(1, std::min<int64_t>(ceil_div(max_dst * 32, 256), 148 * 16));
+  int64_t blocks = grid_cap(ceil_div(max_dst * 32, 256), 16);
   launch_pdl(agg_bwd_kernel, dim3(blocks), dim3(256), 0, st, indptr, indices, n_dst, dz, dz_pitch, dim, dx, dx_pitch);
   return cudaGetLastError();
 }
@@ -474,7 +372,7 @@ __global__ void gather_kernel(FeatView fv, const int32_t* __restrict__ ids, cons
 
 cudaError_t launch_gather(const FeatView& fv, const int32_t* ids, const int32_t* n_dev, int64_t max_n, void* out,
                           int64_t out_pitch, cudaStream_t st) {
-  int64_t blocks = std::max<int64_t>(1, std::min<int64_t>(ceil_div(max_n * 32, 256), 148 * 16));
+  int64_t blocks = grid_cap(ceil_div(max_n * 32, 256), 16);
   const int esz = fv.dtype == kBF16 ? 2 : 4;
   launch_pdl(gather_kernel, dim3(blocks), dim3(256), 0, st, fv, ids, n_dev, max_n, reinterpret_cast<char*>(out), out_pitch * esz);
   return cudaGetLastError();
@@ -499,7 +397,7 @@ __global__ void fill_features_kernel(void* shard, int bf16, int64_t pitch, int c
 
 cudaError_t launch_fill_features(void* shard, DType dt, int64_t pitch, int col0, int ncols, const int32_t* ids,
                                  int64_t n, uint64_t seed, cudaStream_t st) {
-  int64_t blocks = std::max<int64_t>(1, std::min<int64_t>(ceil_div(n * pitch, 256), 148 * 64));
+  int64_t blocks = grid_cap(ceil_div(n * pitch, 256), 64);
   fill_features_kernel<<<blocks, 256, 0, st>>>(shard, dt == kBF16, pitch, col0, ncols, ids, n,
                                                philox_key(seed, kDomFeat));
   return cudaGetLastError();
@@ -537,7 +435,7 @@ extern "C" int64_t apt_selftest_div(void) {
   unsigned long long* d = nullptr;
   if (cudaMalloc(&d, 8) != cudaSuccess) return -1;
   cudaMemset(d, 0, 8);
-  apt::selftest_div_kernel<<<148 * 8, 256>>>(d);
+  apt::selftest_div_kernel<<<apt::num_sms() * 8, 256>>>(d);
   unsigned long long h = 0;
   if (cudaMemcpy(&h, d, 8, cudaMemcpyDeviceToHost) != cudaSuccess) h = ~0ull;
   cudaFree(d);

@@ -6,7 +6,9 @@
 // the side stream while the forward runs) and every source row pulls its in-edges:
 // one pass reads dZ (L2-resident), the ReLU mask from H, and writes G (fp32) and/or
 // its bf16 copy directly; no atomics, no zeroing.  Within a row the in-edges are
-// summed in a fixed (CSC) order.
+// summed in their CSC order, which the fill's atomic slot counters make
+// scheduling-dependent: G is not bitwise reproducible run to run (fp32 sums of the same
+// terms in another order; the parity tests' T1 allowance covers it).
 #include "common.cuh"
 #include "kernels.h"
 #include <algorithm>
@@ -54,7 +56,8 @@ __global__ void csc_fill_kernel(const int32_t* __restrict__ indptr, const int32_
 }
 
 // The same fill with one thread per (row, slot) of the sampler's fixed fanout k: no
-// per-row loop of dependent atomics (A/B: APT_CSC_SLOTS=0 keeps the row loop).
+// per-row loop of dependent atomics (A/B: APT_CSC_SLOTS=0 keeps the row loop).  Either
+// fill orders a row's in-edges by the order its atomicSub calls land.
 __global__ void csc_fill_slots_kernel(const int32_t* __restrict__ indptr, const int32_t* __restrict__ indices,
                                       const int32_t* __restrict__ n_dst_p, int k, const int32_t* __restrict__ csc_ptr,
                                       int32_t* __restrict__ cnt, int2* __restrict__ csc_dst) {
@@ -72,7 +75,7 @@ __global__ void csc_fill_slots_kernel(const int32_t* __restrict__ indptr, const 
 
 cudaError_t launch_csc_build(const CscArgs& a, cudaStream_t st) {
   const int64_t T = 256;
-  const int64_t cap = a.grid_cap > 0 ? a.grid_cap : 148 * 16;
+  const int64_t cap = a.grid_cap > 0 ? a.grid_cap : int64_t(num_sms()) * 16;
   const int64_t ge = std::max<int64_t>(1, std::min<int64_t>(ceil_div(a.max_edges, T), cap));
   const int nb = scan_tiles(a.max_src);
   if (!a.counted)
@@ -328,7 +331,7 @@ cudaError_t launch_pull_bwd(const PullArgs& a, cudaStream_t st) {
     // APT_PULL_BPSM: grid cap in blocks per SM (A/B knob)
     static const int bpsm = [] { const char* e = std::getenv("APT_PULL_BPSM"); return e ? atoi(e) : 16; }();
     const int64_t blocks = std::max<int64_t>(
-        1, std::min<int64_t>(ceil_div(ceil_div(round_up(a.max_src, 64), Rr) * 32, 256), 148 * int64_t(bpsm)));
+        1, std::min<int64_t>(ceil_div(ceil_div(round_up(a.max_src, 64), Rr) * 32, 256), int64_t(num_sms()) * bpsm));
     const int V8 = a.dim >> 3;
     if (Rr == 4) {
       if (V8 <= 32) launch_pdl(pull_bwd_b8_kernel<1, 4>, dim3(blocks), dim3(256), 0, st, a);
@@ -340,7 +343,7 @@ cudaError_t launch_pull_bwd(const PullArgs& a, cudaStream_t st) {
     return cudaGetLastError();
   }
   const int64_t blocks =
-      std::max<int64_t>(1, std::min<int64_t>(ceil_div(ceil_div(round_up(a.max_src, 64), R) * 32, 256), 148 * 16));
+      std::max<int64_t>(1, std::min<int64_t>(ceil_div(ceil_div(round_up(a.max_src, 64), R) * 32, 256), int64_t(num_sms()) * 16));
   const int ms = a.mask ? 1 : a.hb ? 3 : a.h ? 2 : 0;
   auto go = [&](auto vpl) {
     constexpr int VP = decltype(vpl)::value;

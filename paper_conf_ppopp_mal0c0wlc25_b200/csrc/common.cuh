@@ -6,6 +6,10 @@
 #include <cuda_bf16.h>
 #include <stdint.h>
 
+#include <map>
+#include <mutex>
+#include <tuple>
+
 #ifndef __CUDACC__
 #error "compile with nvcc -gencode arch=compute_100a,code=sm_100a"
 #endif
@@ -82,6 +86,41 @@ inline cudaError_t launch_pdl(void (*kern)(KArgs...), dim3 grid, dim3 block, siz
   cfg.attrs = at;
   cfg.numAttrs = 1;
   return cudaLaunchKernelEx(&cfg, kern, static_cast<KArgs>(args)...);
+}
+
+// ------------------------------------------------------- grid sizing ----
+// SM count of the current device (148 on B200), queried once per process (one process
+// drives one device; an emulated job uses one device too).
+inline int num_sms() {
+  static const int n = [] {
+    int d = 0, v = 0;
+    if (cudaGetDevice(&d) != cudaSuccess || cudaDeviceGetAttribute(&v, cudaDevAttrMultiProcessorCount, d) != cudaSuccess ||
+        v <= 0)
+      v = 148;
+    return v;
+  }();
+  return n;
+}
+// Resident blocks per SM the hardware grants this kernel (registers, shared memory,
+// launch bounds), queried once per instantiation: a "one resident wave" grid is
+// num_sms() * resident_blocks(kernel, threads).
+template <typename K>
+inline int resident_blocks(K kernel, int threads, size_t smem = 0) {
+  static std::mutex mu;
+  static std::map<std::tuple<const void*, int, size_t>, int> cache;
+  const auto key = std::make_tuple(reinterpret_cast<const void*>(kernel), threads, smem);
+  std::lock_guard<std::mutex> lk(mu);
+  auto it = cache.find(key);
+  if (it != cache.end()) return it->second;
+  int b = 0;
+  if (cudaOccupancyMaxActiveBlocksPerMultiprocessor(&b, kernel, threads, smem) != cudaSuccess || b <= 0) b = 1;
+  cache.emplace(key, b);
+  return b;
+}
+// Grid of ceil(n / per_block) blocks capped at `per_sm` blocks on every SM.
+inline int64_t grid_cap(int64_t want, int64_t per_sm) {
+  const int64_t cap = int64_t(num_sms()) * per_sm;
+  return want < 1 ? 1 : (want < cap ? want : cap);
 }
 
 // ---------------------------------------------------------------- misc ----

@@ -266,7 +266,7 @@ extern "C" apt_status apt_dryrun(apt_trainer* t, int64_t n_steps, apt_plan_stats
         marks.push_back({S, r});
         const Hop& l1 = hops[K - 1];
         launch_pdl(dry_nd_kernel, dim3(1), dim3(32), 0, c->stream, r, l1.n_dst, dc + S);
-        const int64_t blocks = std::max<int64_t>(1, std::min<int64_t>(ceil_div(l1.max_dst, 256), 148 * 8));
+        const int64_t blocks = grid_cap(ceil_div(l1.max_dst, 256), 8);
         launch_pdl(dry_count_kernel, dim3(blocks), dim3(256), 0, c->stream, S, r, C, l1.dst, l1.n_dst, l1.cnt, l1.nbr, l1.k, g->part,
                                                         own_bm, n_words, dc + S, ti);
         CK(c, cudaGetLastError());
@@ -419,7 +419,7 @@ extern "C" apt_status apt_access_counts(apt_trainer* t, int64_t n_steps, int32_t
   int32_t* counts = ds.A.alloc<int32_t>(t->g->n, true);
   if (!ok || !bm || !counts) return set_err(c, APT_E_OOM, "apt_access_counts: out of device memory");
   const Hop& l1 = ds.hops[K - 1];
-  const int64_t blocks = std::max<int64_t>(1, std::min<int64_t>(ceil_div(l1.max_dst, 256), 148 * 8));
+  const int64_t blocks = grid_cap(ceil_div(l1.max_dst, 256), 8);
   for (int64_t st = 0; st < n_steps; ++st) {
     ds.set_step(st, c->stream);
     for (int r = 0; r < C; ++r) {
@@ -543,7 +543,7 @@ extern "C" apt_status apt_profile_links(apt_ctx* c, apt_bw_profile* out) {
     out->beta_Bps[op] = beta;
     out->measured[op] = 1;
   };
-  const int blocks = 148 * 8;
+  const int blocks = num_sms() * 8;
   // local HBM gather: random rows of the table (the store's local tier)
   const double tg_s = best([&] { trial_gather_kernel<<<blocks, 256, 0, c->stream>>>(table, table_rows, vec, ids, n_small, outb); });
   const double tg_b = best([&] { trial_gather_kernel<<<blocks, 256, 0, c->stream>>>(table, table_rows, vec, ids, n_big, outb); });

@@ -60,7 +60,7 @@ constexpr float kSlope = 0.2f;     // LeakyReLU slope of GAT [45]
 
 __device__ __align__(16) uint4 g_gat_zero_row[64];
 
-static int64_t gridn(int64_t n, int t = 256) { return std::max<int64_t>(1, std::min<int64_t>(ceil_div(n, t), 148 * 16)); }
+static int64_t gridn(int64_t n, int t = 256) { return grid_cap(ceil_div(n, t), 16); }
 
 struct GatItems {
   const int32_t* n;       // device item count
@@ -655,7 +655,7 @@ static GatKArgs kargs(apt_trainer* t, RankState& rs) {
 template <int EPV, int LG, int H>
 static cudaError_t launch_one(const GatKArgs& a, bool bwd, int64_t max_items, cudaStream_t st) {
   constexpr int RPW = 32 / LG;
-  const int64_t blocks = std::max<int64_t>(1, std::min<int64_t>(ceil_div(ceil_div(max_items, RPW) * 32, 256), 148 * 8));
+  const int64_t blocks = grid_cap(ceil_div(ceil_div(max_items, RPW) * 32, 256), 8);
   const size_t smem = size_t(2) * H * a.cpad * sizeof(float);
   if (bwd) return launch_pdl(gat_bwd_kernel<EPV, LG, H>, dim3(blocks), dim3(256), smem, st, a);
   return launch_pdl(gat_fwd_kernel<EPV, LG, H>, dim3(blocks), dim3(256), smem, st, a);

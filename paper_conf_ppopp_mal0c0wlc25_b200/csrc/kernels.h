@@ -115,25 +115,6 @@ struct AggArgs {
 };
 cudaError_t launch_agg_fstore(const AggArgs& a, const FeatView& fv, cudaStream_t st);
 cudaError_t launch_agg_csr(const AggArgs& a, cudaStream_t st);
-// Output layer K fused (outlayer.cu, bf16 mode): mean of H_{K-1} bf16 rows over the
-// block CSR, logits on CUDA cores, CE loss, G / Gb, dZ = (Gb W) / deg.
-struct OutLayerArgs {
-  const int32_t* indptr; const int32_t* indices;   // block of layer K (hop 0)
-  const int32_t* n_dst; int64_t max_dst;
-  const uint16_t* xb; int64_t x_pitch;             // H_{K-1} bf16 [n_src x x_pitch]
-  int d_in, d_out;
-  const uint16_t* Wb; int64_t wb_pitch; const float* bias;
-  const int32_t* seeds; const int32_t* labels; const int32_t* n_global;
-  uint16_t* Zb; int64_t zb_pitch;                  // Z_K bf16 + ones column d_in
-  float* H; int64_t h_pitch;                       // logits
-  float* loss;
-  float* G; int64_t g_pitch;
-  uint16_t* Gb; int64_t gb_pitch;                  // zero-padded to the 64-row block
-  float* dZ; int64_t dz_pitch;                     // (G W) / deg
-};
-int outlayer_supported(int d_in, int d_out);
-cudaError_t launch_outlayer(const OutLayerArgs& a, cudaStream_t st);
-
 
 // dX[src_e] += dZ[v] / deg(v)  (O5 backward), fp32 atomics.
 cudaError_t launch_agg_bwd(const int32_t* indptr, const int32_t* indices, const int32_t* n_dst, int64_t max_dst,
@@ -147,21 +128,6 @@ cudaError_t launch_gather(const FeatView& fv, const int32_t* ids, const int32_t*
 // Fill a shard with the synthetic O4 features of the listed global ids.
 cudaError_t launch_fill_features(void* shard, DType dt, int64_t pitch, int col0, int ncols, const int32_t* ids,
                                  int64_t n, uint64_t seed, cudaStream_t st);
-
-// ---------------------------------------------------------------- fused.cu
-// Layer-1 forward in one kernel: TMA gather4 of the sampled rows, mean, tcgen05
-// projection, bias + ReLU.  Single-shard bf16 store; cudaErrorNotSupported otherwise.
-struct FusedL1Args {
-  const int32_t* cnt; const int32_t* nbr; int k;        // sampler ELL
-  const int32_t* n_dev; int64_t M_max;                  // destination rows
-  const uint16_t* feat; int64_t n_rows_table; int row_elems;   // bf16 store [rows x row_elems]
-  int d;                                                // features aggregated
-  const uint16_t* Wb; int64_t w_pitch; int N;           // bf16 W [N x w_pitch]
-  const float* bias; int relu;
-  float* Y; int64_t y_pitch;                            // fp32 h1
-  uint16_t* Z; int64_t z_pitch; int z_ones;             // bf16 Z (weight gradient)
-};
-cudaError_t launch_sage_l1(const FusedL1Args& a, cudaStream_t st);
 
 // ---------------------------------------------------------------- bwd.cu
 // Transpose of a sampled block (counting sort): csc_ptr [n_src+1], csc_dst [E].

@@ -8,7 +8,7 @@
 namespace apt {
 
 static int64_t grid_of(int64_t n, int t = 256) {
-  return std::max<int64_t>(1, std::min<int64_t>(ceil_div(n, t), 148 * 32));
+  return grid_cap(ceil_div(n, t), 32);
 }
 
 // loss = sum_s CE(logits_s, y_s) / n_global  (reading Z20);  g = (softmax - onehot) / n_global.
@@ -209,7 +209,7 @@ cudaError_t launch_sgd_multi(const SgdBatch& b, float lr, cudaStream_t st) {
   if (b.n <= 0) return cudaSuccess;
   int64_t mx = 1;
   for (int i = 0; i < b.n; ++i) mx = std::max<int64_t>(mx, b.seg[i].n);
-  dim3 grid(unsigned(std::min<int64_t>(ceil_div(mx, 256), 148 * 4)), unsigned(b.n));
+  dim3 grid(unsigned(grid_cap(ceil_div(mx, 256), 4)), unsigned(b.n));
   launch_pdl(sgd_multi_kernel, dim3(grid), dim3(256), 0, st, b, lr);
   return cudaGetLastError();
 }

@@ -166,12 +166,12 @@ cudaError_t launch_sample(const SampleArgs& a, cudaStream_t st) {
   const int threads = 256;
   const int64_t warps = a.max_frontier;
   int64_t blocks = ceil_div(warps * 32, threads);
-  blocks = std::max<int64_t>(1, std::min<int64_t>(blocks, a.grid_cap > 0 ? a.grid_cap : 148 * 16));
+  blocks = std::max<int64_t>(1, std::min<int64_t>(blocks, a.grid_cap > 0 ? a.grid_cap : int64_t(num_sms()) * 16));
   const int ks = int(ceil_div(a.k, 32));
   static const int g16 = [] { const char* v = std::getenv("APT_SAMPLE_G16"); return v ? atoi(v) : 1; }();
   if (g16 && a.k <= 16) {
     int64_t b2 = ceil_div(ceil_div(a.max_frontier, 2) * 32, threads);
-    b2 = std::max<int64_t>(1, std::min<int64_t>(b2, a.grid_cap > 0 ? a.grid_cap : 148 * 16));
+    b2 = std::max<int64_t>(1, std::min<int64_t>(b2, a.grid_cap > 0 ? a.grid_cap : int64_t(num_sms()) * 16));
     launch_pdl(sample_g16_kernel, dim3(b2), dim3(threads), 0, st, a.indptr, a.indices, a.frontier, a.n_frontier, a.k,
                a.key, a.step, a.hop, a.cnt, a.nbr);
     return cudaGetLastError();
@@ -281,7 +281,7 @@ __global__ void map_indices_kernel(const int32_t* __restrict__ dst, const int32_
 }
 
 static int64_t grid_for(int64_t n, int threads) {
-  return std::max<int64_t>(1, std::min<int64_t>(ceil_div(n, threads), 148 * 32));
+  return grid_cap(ceil_div(n, threads), 32);
 }
 
 // Fused compaction, three launches per hop:

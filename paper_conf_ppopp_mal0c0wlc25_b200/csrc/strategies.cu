@@ -49,7 +49,7 @@ FeatView feat_view(const apt_fstore* f, int r);
 
 namespace apt {
 
-static int64_t grid_n(int64_t n, int t = 256) { return std::max<int64_t>(1, std::min<int64_t>(ceil_div(n, t), 148 * 16)); }
+static int64_t grid_n(int64_t n, int t = 256) { return grid_cap(ceil_div(n, t), 16); }
 
 struct WorkTab {
   int32_t* const* n;

@@ -139,7 +139,7 @@ __global__ void zero_rows_kernel(float* p, int64_t pitch, const int32_t* n_p) {
     q[t] = make_float4(0.f, 0.f, 0.f, 0.f);
 }
 
-static int64_t blocks_for(int64_t n) { return std::max<int64_t>(1, std::min<int64_t>(ceil_div(n, 256), 148 * 16)); }
+static int64_t blocks_for(int64_t n) { return grid_cap(ceil_div(n, 256), 16); }
 
 // Projection dispatch: tcgen05 (bf16 mode) or exact fp32 CUDA cores.
 apt_status project(apt_trainer* t, const Layer& L, const void* Zb, const float* Zf, int64_t z_pitch_b,
@@ -550,7 +550,7 @@ apt_status phase_sample(apt_trainer* t, RankState& rs, SampleSet& ss, bool from_
   // that it fills gaps instead of competing with the step's chain for every SM
   static const int64_t bg_cap = [] {
     const char* v = std::getenv("APT_BG_BLOCKS_PER_SM");
-    return int64_t(148) * (v ? std::max(1, atoi(v)) : 4);
+    return int64_t(num_sms()) * (v ? std::max(1, atoi(v)) : 4);
   }();
   const int64_t cap = st == c->samp ? bg_cap : 0;
   {
@@ -626,38 +626,12 @@ void activate(apt_trainer* t, int q) {
 }
 
 // GDP layer-1 forward on one rank: the fused gather+mean (local + peer rows), then the
-// projection.  APT_FUSED_L1=1 selects the single-kernel layer (fused.cu: gather warps ->
-// UMMA tile in shared memory -> tcgen05 -> epilogue) for a single-shard bf16 store --
-// correct (tested) but measured slower on products (78 us vs 34 + 30 us): the gather
-// needs the parallelism of thousands of short-lived warps more than it gains from not
-// writing and re-reading the 10 MB Z.
+// projection.
 apt_status layer1_fwd_gdp(apt_trainer* t, RankState& rs, bool time_it) {
   apt_ctx* c = t->ctx;
   Layer& L = rs.L[0];
   const Hop& hp = rs.hops[t->K - 1];
   const FeatView fv = feat_view(t->f, rs.rank);
-  const char* fz = std::getenv("APT_FUSED_L1");
-  const bool want_fused = fz && *fz == '1';
-  if (t->m.dtype == APT_BF16 && !fv.part && want_fused && tc_gemm_supported(L.d_out, L.d_in)) {
-    FusedL1Args fa{hp.cnt, hp.nbr, hp.k, hp.n_dst, hp.max_dst, static_cast<const uint16_t*>(fv.base[0]),
-                   t->g->n, int(fv.pitch), fv.dim, L.Wb, L.wb_pitch, L.d_out, L.b, t->K > 1 ? 1 : 0,
-                   L.H, L.h_pitch, L.Zb, L.zb_pitch, 1};
-    if (time_it) CK(c, record_ev(t, 6));
-    cudaError_t e = launch_sage_l1(fa, c->stream);
-    if (e == cudaSuccess) {
-      if (time_it) CK(c, record_ev(t, 7));
-      c->launches++;
-      t->fused_l1 = true;
-      if (L.Hb) {
-        CK(c, launch_to_bf16(L.H, L.h_pitch, L.Hb, L.hb_pitch, L.d_out, L.n_rows, L.max_rows, c->stream));
-        c->launches++;
-      }
-      return APT_OK;
-    }
-    if (e != cudaErrorNotSupported) return check_cuda(c, e, "launch_sage_l1");
-    cudaGetLastError();   // clear the sticky not-supported status; take the two-kernel path
-  }
-  t->fused_l1 = false;
   AggArgs a{};
   a.cnt = hp.cnt; a.nbr = hp.nbr; a.k = hp.k;
   a.n_dst = hp.n_dst; a.max_dst = hp.max_dst; a.dim = L.d_in;
@@ -678,35 +652,13 @@ static bool bf16_dz_enabled() {
   return !e || atoi(e) != 0;
 }
 
-// The output layer as one kernel (outlayer.cu): bf16 mode, K >= 2, <= 64 classes,
-// input width <= 256, opt-in with APT_FUSED_OUT=1 (read when the step is built).
-// Measured on products: faster alone (0.266 vs 0.272 ms with the
-// step's sampling inline) but slower next to the overlapped sampling of the next
-// step (0.243 vs 0.221 ms), so the pipelined default keeps the unfused kernels.
-static bool fused_out(const apt_trainer* t, const RankState& rs) {
-  const char* e = std::getenv("APT_FUSED_OUT");
-  if (!e || atoi(e) != 1 || t->m.dtype != APT_BF16 || t->K < 2) return false;
-  const Layer& LK = rs.L[t->K - 1];
-  return rs.L[t->K - 2].Hb && outlayer_supported(LK.d_in, LK.d_out);
-}
-
 // Upper layers l = 2..K (data parallel) + CE loss on one rank.
 apt_status upper_fwd_loss(apt_trainer* t, RankState& rs) {
   apt_ctx* c = t->ctx;
-  const bool fo = fused_out(t, rs);
   for (int l = 2; l <= t->K; ++l) {
     Layer& L = rs.L[l - 1];
     const Layer& P = rs.L[l - 2];
     const Hop& hp = rs.hops[t->K - l];
-    if (l == t->K && fo) {   // mean + logits + CE + G + dZ of the output layer in one kernel
-      CK(c, cudaMemsetAsync(rs.loss, 0, sizeof(float), c->stream));
-      OutLayerArgs o{hp.indptr, hp.indices, hp.n_dst, hp.max_dst, P.Hb, P.hb_pitch, L.d_in, L.d_out,
-                     L.Wb, L.wb_pitch, L.b, rs.seeds, t->labels, rs.small + 1, L.Zb, L.zb_pitch,
-                     L.H, L.h_pitch, rs.loss, L.G, L.h_pitch, L.Gb, L.gb_pitch, L.dZ, L.zf_pitch};
-      CK(c, launch_outlayer(o, c->stream));
-      c->launches++;
-      return APT_OK;
-    }
     AggArgs a{};
     a.indptr = hp.indptr; a.indices = hp.indices; a.x = P.H; a.x_pitch = P.h_pitch;
     if (P.Hb) { a.x = nullptr; a.xb = P.Hb; a.x_pitch = P.hb_pitch; }   // R11
@@ -745,9 +697,6 @@ apt_status upper_bwd(apt_trainer* t, RankState& rs) {
     if (s != APT_OK) return s;
     int dz_scaled = 0;
     const uint16_t* dzb = nullptr;
-    if (l == t->K && fused_out(t, rs)) {
-      dz_scaled = 1;   // dZ / deg came with the fused output layer
-    } else
     // dZ = G W  (bf16 mode: tcgen05 with the bf16 weights of the forward, W read N-major as stored)
     if (bf && tc_gemm_supported(L.d_in, L.d_out)) {
       TcGemmArgs g{L.Gb, L.gb_pitch, L.Wb, L.wb_pitch, L.max_rows, L.n_rows, L.d_in, L.d_out, nullptr, 0,

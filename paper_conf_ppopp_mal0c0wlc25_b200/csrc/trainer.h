@@ -186,7 +186,6 @@ struct apt_trainer {
   int primed_parity = 0;
   bool csc_forked = false;
   std::function<apt_status()> deferred_fork;   // pipelined: next-step sampling, launched after the layer-1 forward
-  bool fused_l1 = false;             // the last layer-1 forward ran as the single fused kernel           // this step's block transposes run on the side branch (wait ev_csc)
   cudaGraphExec_t gexec_p[2][2] = {};   // [parity][update] pipelined step graphs
   cudaGraph_t graph_p[2][2] = {};
   cudaGraphNode_t step_node_p[2][2] = {};

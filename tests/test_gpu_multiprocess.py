@@ -18,8 +18,8 @@ def test_multiprocess_strategies_match_oracle(world):
     env = dict(os.environ, APT_TEST_DEVICE="0")
     cmd = [sys.executable, "-m", "torch.distributed.run", "--nnodes=1", f"--nproc-per-node={world}",
            "--master-addr", "127.0.0.1", "--master-port", "29533", os.path.join(ROOT, "tests", "mp_step.py"),
-           "f32,bf16", "GDP,NFP,SNP,DNP"]
-    r = subprocess.run(cmd, capture_output=True, text=True, timeout=600, env=env, cwd=ROOT)
+           "f32,bf16", "GDP,NFP,SNP,DNP", "5,5;5,5,5"]
+    r = subprocess.run(cmd, capture_output=True, text=True, timeout=900, env=env, cwd=ROOT)
     out = r.stdout + r.stderr
     line = [l for l in out.splitlines() if l.startswith("RESULT")]
     assert r.returncode == 0 and line and line[0] == "RESULT OK", out[-4000:]

@@ -10,8 +10,10 @@ import pytest
 import aptgen
 import oracle
 from oracle import model
+from parity_util import assert_close, reconcile, sum_bounds, t1
 
 pytestmark = pytest.mark.gpu
+LAMBDA_U = 6 * 2.0 ** -24       # one fp32 rounding of the bias add, at LAMBDA
 
 torch = pytest.importorskip("torch")
 
@@ -161,9 +163,11 @@ def test_project_tcgen05_bf16(A, ctx, M, N, K):
     Y = torch.zeros((M, yp), dtype=torch.float32, device="cuda")
     ctx.project(torch.as_tensor(Zb.view(np.int16)).cuda(), kp, A.BF16, torch.as_tensor(W).cuda(),
                 torch.as_tensor(bias).cuda(), M, N, K, 1, Y, yp)
-    ref = np.maximum(Z @ oracle.bf16_round(W).T + bias, 0)
+    Wr = oracle.bf16_round(W)
+    ref = np.maximum(Z @ Wr.T + bias, 0)
     got = Y.cpu().numpy()[:, :N]
-    assert np.allclose(got, ref, rtol=1e-5, atol=1e-5), np.abs(got - ref).max()
+    # fp32 accumulation of bf16 products: the fp32 bar with the T1 allowance
+    assert_close(got, ref, "f32", "Y", t1(np.abs(Z), np.abs(Wr).T, K) + LAMBDA_U * np.abs(bias))
 
 
 @pytest.mark.parametrize("M,N,K", [(1, 5, 3), (130, 47, 100), (2000, 256, 100)])
@@ -176,7 +180,7 @@ def test_project_fp32(A, ctx, M, N, K):
     ctx.project(torch.as_tensor(Z).cuda(), K, A.F32, torch.as_tensor(W).cuda(), torch.as_tensor(bias).cuda(),
                 M, N, K, 0, Y, N)
     ref = Z.astype(np.float64) @ W.T.astype(np.float64) + bias
-    assert np.allclose(Y.cpu().numpy(), ref, rtol=1e-5, atol=1e-5)
+    assert_close(Y.cpu().numpy(), ref, "f32", "Y", t1(np.abs(Z), np.abs(W).T, K) + LAMBDA_U * np.abs(bias))
 
 
 # ------------------------------------------------------------------ the training step (C = 1)
@@ -197,10 +201,25 @@ def _trainer(A, ctx, cfg, g, train, dtype, strategy="GDP", lr=0.1):
 TOL = {"f32": dict(rtol=1e-5, atol=1e-6), "bf16": dict(rtol=2e-2, atol=2e-3)}
 
 
+def _check_grads(tr, ref, bd, dtype, K, rank=0, what=""):
+    for l in range(1, K + 1):
+        dW, db = ref["grads"][l - 1]
+        assert_close(tr.read("dW", l, rank=rank), dW, dtype, f"{what}dW layer {l}", bd["dW"][l - 1])
+        assert_close(tr.read("db", l, rank=rank)[0], db, dtype, f"{what}db layer {l}", bd["db"][l - 1])
+
+
+# fanouts: tiny's [5,5]; 3 layers like the benchmarked model; layer-1 fanouts 16 and
+# 12 (the two-nodes-per-warp sampler at its k = 16 limit, the layer-1 gather's 5-load rounds
+# with a ragged last round, k in 11..16)
+FANOUTS = [(5, 5), (5, 5, 5), (16, 12), (12, 16)]
+
+
 @pytest.mark.parametrize("dtype", ["f32", "bf16"])
 @pytest.mark.parametrize("step", [0, 3])
-def test_train_step_matches_oracle(A, ctx, tiny, dtype, step):
+@pytest.mark.parametrize("fanouts", FANOUTS)
+def test_train_step_matches_oracle(A, ctx, tiny, dtype, step, fanouts):
     cfg, g, train = tiny
+    cfg = cfg.replace(fanouts=fanouts)
     tr, params, labels = _trainer(A, ctx, cfg, g, train, dtype)
     tr.step(step, update=False)
     loss = tr.loss()
@@ -215,37 +234,11 @@ def test_train_step_matches_oracle(A, ctx, tiny, dtype, step):
         assert np.array_equal(tr.read("dst", l)[:, 0], blocks[K - l].dst)
     # layer-1 Z is bit-exact under O4 features (exact sums, IEEE division)
     assert np.array_equal(tr.read("Z", 1), ref["cache"]["Z"][0].astype(np.float32))
-    tol = TOL[dtype]
+    ref, bd = reconcile(blocks, p64, ref, dtype, len(seeds), [tr.read("H", l) for l in range(1, K)])
     for l in range(1, K + 1):
-        assert np.allclose(tr.read("H", l), ref["cache"]["h"][l - 1], **tol), f"H layer {l}"
-    assert abs(loss - ref["loss"]) <= tol["rtol"] * abs(ref["loss"]) + tol["atol"]
-    for l in range(1, K + 1):
-        dW, db = ref["grads"][l - 1]
-        assert np.allclose(tr.read("dW", l), dW, **tol), f"dW layer {l}"
-        assert np.allclose(tr.read("db", l)[0], db, **tol), f"db layer {l}"
-
-
-@pytest.mark.parametrize("step", [0, 2])
-def test_train_step_fused_output_layer(A, ctx, tiny, step, monkeypatch):
-    """The opt-in fused output layer (outlayer.cu: mean + logits + CE + G + dZ/deg in one
-    kernel, APT_FUSED_OUT=1) against the oracle: logits, loss, every layer's gradients."""
-    monkeypatch.setenv("APT_FUSED_OUT", "1")
-    cfg, g, train = tiny
-    tr, params, labels = _trainer(A, ctx, cfg, g, train, "bf16")
-    tr.step(step, update=False)
-    seeds = tr.read("seeds")[:, 0].astype(np.int64)
-    blocks = oracle.sample_blocks(g, seeds, cfg.fanouts, cfg.sample_seed, step)
-    p64 = [(W.astype(np.float64), b.astype(np.float64)) for W, b in params]
-    ref = model.train_step(blocks, cfg.feat_seed, cfg.dim, p64, labels[seeds], len(seeds), "bf16")
-    tol = TOL["bf16"]
-    K = len(blocks)
-    assert np.allclose(tr.read("Z", K), ref["cache"]["Z"][K - 1], **tol)
-    assert np.allclose(tr.read("H", K), ref["cache"]["h"][K - 1], **tol)
-    assert abs(tr.loss() - ref["loss"]) <= tol["rtol"] * abs(ref["loss"]) + tol["atol"]
-    for l in range(1, K + 1):
-        dW, db = ref["grads"][l - 1]
-        assert np.allclose(tr.read("dW", l), dW, **tol), f"dW layer {l}"
-        assert np.allclose(tr.read("db", l)[0], db, **tol), f"db layer {l}"
+        assert_close(tr.read("H", l), ref["cache"]["h"][l - 1], dtype, f"H layer {l}", bd["H"][l - 1])
+    assert abs(loss - ref["loss"]) <= (1e-5 if dtype == "f32" else 2e-2) * abs(ref["loss"])
+    _check_grads(tr, ref, bd, dtype, K)
 
 
 @pytest.mark.parametrize("dtype", ["f32", "bf16"])
@@ -261,16 +254,12 @@ def test_train_step_wide_hidden(A, ctx, tiny, dtype):
     blocks = oracle.sample_blocks(g, seeds, cfg.fanouts, cfg.sample_seed, 1)
     p64 = [(W.astype(np.float64), b.astype(np.float64)) for W, b in params]
     ref = model.train_step(blocks, cfg.feat_seed, cfg.dim, p64, labels[seeds], len(seeds), dtype)
-    tol = TOL[dtype]
     K = len(blocks)
+    ref, bd = reconcile(blocks, p64, ref, dtype, len(seeds), [tr.read("H", l) for l in range(1, K)])
     for l in range(1, K + 1):
-        assert np.allclose(tr.read("H", l), ref["cache"]["h"][l - 1], **tol), f"H layer {l}"
-    assert abs(tr.loss() - ref["loss"]) <= tol["rtol"] * abs(ref["loss"]) + tol["atol"]
-    for l in range(1, K + 1):
-        dW, db = ref["grads"][l - 1]
-        atol = tol["atol"] * (10 if dtype == "bf16" else 1)
-        assert np.allclose(tr.read("dW", l), dW, rtol=tol["rtol"], atol=atol), f"dW layer {l}"
-        assert np.allclose(tr.read("db", l)[0], db, rtol=tol["rtol"], atol=atol), f"db layer {l}"
+        assert_close(tr.read("H", l), ref["cache"]["h"][l - 1], dtype, f"H layer {l}", bd["H"][l - 1])
+    assert abs(tr.loss() - ref["loss"]) <= (1e-5 if dtype == "f32" else 2e-2) * abs(ref["loss"])
+    _check_grads(tr, ref, bd, dtype, K)
 
 
 @pytest.mark.parametrize("use_graph", [False, True])
@@ -324,25 +313,6 @@ def test_pipelined_steps_equal_unpipelined(A, tiny, strategy, C):
         assert np.array_equal(seeds, outs[0][1])
         for (W0, b0), (W1, b1) in zip(outs[0][0], params):
             assert np.allclose(W0, W1, rtol=1e-5, atol=1e-6) and np.allclose(b0, b1, rtol=1e-5, atol=1e-6)
-
-
-@pytest.mark.parametrize("dtype", ["bf16"])
-def test_fused_layer1_kernel_matches_oracle(A, ctx, tiny, dtype, monkeypatch):
-    """The opt-in single-kernel layer 1 (gather -> UMMA tile in smem -> tcgen05 -> epilogue):
-    Z bit-exact, h1 / logits / gradients against the oracle, like the two-kernel path."""
-    monkeypatch.setenv("APT_FUSED_L1", "1")
-    cfg, g, train = tiny
-    tr, params, labels = _trainer(A, ctx, cfg, g, train, dtype)
-    tr.step(1, update=False)
-    seeds = tr.read("seeds")[:, 0].astype(np.int64)
-    blocks = oracle.sample_blocks(g, seeds, cfg.fanouts, cfg.sample_seed, 1)
-    p64 = [(W.astype(np.float64), b.astype(np.float64)) for W, b in params]
-    ref = model.train_step(blocks, cfg.feat_seed, cfg.dim, p64, labels[seeds], len(seeds), dtype)
-    assert np.array_equal(tr.read("Z", 1), ref["cache"]["Z"][0].astype(np.float32))
-    tol = TOL[dtype]
-    assert np.allclose(tr.read("H", 1), ref["cache"]["h"][0], **tol)
-    for l in range(1, len(blocks) + 1):
-        assert np.allclose(tr.read("dW", l), ref["grads"][l - 1][0], **tol)
 
 
 def test_sgd_update_and_graph_replay(A, ctx, tiny):
@@ -406,7 +376,6 @@ def test_weight_grad(A, ctx, rows, d_out, d_in, dtype):
         Zh[:, :d_in] = (Zr.astype(np.float32).view(np.uint32) >> 16).astype(np.uint16)
         Zt = torch.as_tensor(Zh.view(np.int16)).cuda()
         Gr = oracle.bf16_round(G)
-        tol = dict(rtol=1e-4, atol=1e-5 * np.sqrt(rows))
     else:
         Zr = Z.astype(np.float32).astype(np.float64)
         zp = (d_in + 3) // 4 * 4
@@ -414,16 +383,16 @@ def test_weight_grad(A, ctx, rows, d_out, d_in, dtype):
         Zf[:, :d_in] = Zr
         Zt = torch.as_tensor(Zf).cuda()
         Gr = G.astype(np.float64)
-        tol = dict(rtol=1e-5, atol=1e-5 * np.sqrt(rows))   # fp32 accumulation-order error grows ~ sqrt(rows)
     dW = torch.zeros((d_out, d_in), dtype=torch.float32, device="cuda")
     db = torch.zeros(d_out, dtype=torch.float32, device="cuda")
     ctx.weight_grad(torch.as_tensor(Gd).cuda(), gp, Zt, zp, A.DTYPE[dtype], rows, d_out, d_in, dW, db)
-    assert np.allclose(dW.cpu().numpy(), Gr.T @ Zr, **tol), np.abs(dW.cpu().numpy() - Gr.T @ Zr).max()
-    assert np.allclose(db.cpu().numpy(), Gr.sum(0), **tol)
+    # fp32 accumulation over `rows` products of the (emulated) operands: the fp32 bar with T1
+    assert_close(dW.cpu().numpy(), Gr.T @ Zr, "f32", "dW", t1(np.abs(Gr).T, np.abs(Zr), rows))
+    assert_close(db.cpu().numpy(), Gr.sum(0), "f32", "db", t1(np.abs(Gr).T, np.ones(rows), rows))
 
 
 # ------------------------------------------------------------------ strategies (C ranks emulated on one B200)
-def _strategy_ref(cfg, g, train, labels, params, strategy, C, step, dtype):
+def _strategy_ref(cfg, g, train, labels, params, strategy, C, step, dtype, bounds=None):
     """Oracle: every rank's own blocks through the fp64 model, loss over the global batch (Z20);
     the strategies must reproduce it (P:59, P:279 'semantically equivalent')."""
     from oracle import strategy as S
@@ -432,19 +401,24 @@ def _strategy_ref(cfg, g, train, labels, params, strategy, C, step, dtype):
     part = aptgen.partition(g.n, C)
     seeds = S.assign_seeds(strategy, gb, part, C, cfg.batch)
     p64 = [(W.astype(np.float64), b.astype(np.float64)) for W, b in params]
-    refs = []
+    refs, bds = [], []
     for r in range(C):
         blocks = oracle.sample_blocks(g, seeds[r], cfg.fanouts, cfg.sample_seed, step)
         snp = (part, C) if strategy == "SNP" else None     # SNP's own rounding points (partials)
         refs.append(model.train_step(blocks, cfg.feat_seed, cfg.dim, p64, labels[seeds[r]], len(gb), dtype, snp=snp))
-    return seeds, refs
+        if bounds is not None:     # bounds = the trainer: reconcile with rank r's mask bits (T3)
+            refs[-1], bd = reconcile(blocks, p64, refs[-1], dtype, len(gb),
+                                     [bounds.read("H", l, rank=r) for l in range(1, len(cfg.fanouts))])
+            bds.append(bd)
+    return (seeds, refs, bds) if bounds is not None else (seeds, refs)
 
 
 @pytest.mark.parametrize("dtype", ["f32", "bf16"])
-@pytest.mark.parametrize("C", [2, 4, 8])
+@pytest.mark.parametrize("C,fanouts", [(2, (5, 5)), (4, (5, 5)), (8, (5, 5)), (2, (5, 5, 5)), (4, (5, 5, 5))])
 @pytest.mark.parametrize("strategy", ["GDP", "NFP", "SNP", "DNP"])
-def test_strategy_step_matches_oracle(A, tiny, strategy, C, dtype):
+def test_strategy_step_matches_oracle(A, tiny, strategy, C, fanouts, dtype):
     cfg, g, train = tiny
+    cfg = cfg.replace(fanouts=fanouts)
     ctx = A.Ctx(-1, C, 0)                      # all C ranks on this device
     gr = ctx.graph_load(g.indptr, g.indices, aptgen.partition(g.n, C))
     dt = A.DTYPE[dtype]
@@ -457,22 +431,23 @@ def test_strategy_step_matches_oracle(A, tiny, strategy, C, dtype):
     tr.set_params(params)
     tr.set_epoch(train, 0)
     tr.step(0, update=False)
-    seeds, refs = _strategy_ref(cfg, g, train, labels, params, strategy, C, 0, dtype)
-    tol = TOL[dtype]
+    seeds, refs, bds = _strategy_ref(cfg, g, train, labels, params, strategy, C, 0, dtype, bounds=tr)
     K = len(cfg.fanouts)
     for r in range(C):
         assert np.array_equal(tr.read("seeds", rank=r)[:, 0], seeds[r])
-        assert np.allclose(tr.read("H", 1, rank=r), refs[r]["cache"]["h"][0], **tol), f"h1 rank {r}"
-        assert np.allclose(tr.read("H", K, rank=r), refs[r]["cache"]["h"][K - 1], **tol), f"logits rank {r}"
+        for l in range(1, K + 1):
+            assert_close(tr.read("H", l, rank=r), refs[r]["cache"]["h"][l - 1], dtype, f"H layer {l} rank {r}",
+                         bds[r]["H"][l - 1])
     loss = tr.loss()
     ref_loss = sum(x["loss"] for x in refs)
-    assert abs(loss - ref_loss) <= tol["rtol"] * abs(ref_loss) + tol["atol"]
+    assert abs(loss - ref_loss) <= (1e-5 if dtype == "f32" else 2e-2) * abs(ref_loss)
     for l in range(1, K + 1):
         dW = sum(x["grads"][l - 1][0] for x in refs)
         db = sum(x["grads"][l - 1][1] for x in refs)
+        sb = sum_bounds(bds)
         for r in (0, C - 1):
-            assert np.allclose(tr.read("dW", l, rank=r), dW, **tol), f"dW layer {l} rank {r}"
-            assert np.allclose(tr.read("db", l, rank=r)[0], db, **tol), f"db layer {l} rank {r}"
+            assert_close(tr.read("dW", l, rank=r), dW, dtype, f"dW layer {l} rank {r}", sb["dW"][l - 1])
+            assert_close(tr.read("db", l, rank=r)[0], db, dtype, f"db layer {l} rank {r}", sb["db"][l - 1])
 
 
 # ------------------------------------------------------------------ S12/S13 planner
@@ -622,7 +597,8 @@ def test_products_full_size_layer1_rows_vs_oracle(A, ctx):
         zb = oracle.bf16_round(z)                   # bf16 mode stores Z at its bf16 rounding point (O5)
         assert np.array_equal(Z[i], zb.astype(np.float32)), v
         h = np.maximum(zb @ W1.T + b1, 0)
-        assert np.allclose(H[i], h, rtol=2e-2, atol=2e-3), v
+        # same bf16 operands: fp32 accumulation (T1) and one bf16 rounding of h (2^-9, flip-wide)
+        assert_close(H[i], h, "bf16", f"h1 of {v}", t1(np.abs(zb), np.abs(W1).T, cfg.dim) + 2.0 ** -8 * np.abs(h))
 
 
 # ------------------------------------------------------------------ unified feature store tiers (NEXT #2)
@@ -659,9 +635,11 @@ def test_tiered_store_rows_and_step(A, tiny, dtype, frac, n_hot):
         tr.set_params(params)
         tr.set_epoch(train, 0)
         tr.step(0, update=False)
-        seeds, refs = _strategy_ref(cfg, g, train, labels, params, strategy, C, 0, dtype)
-        tol = TOL[dtype]
+        seeds, refs, bds = _strategy_ref(cfg, g, train, labels, params, strategy, C, 0, dtype, bounds=tr)
         for r in range(C):
-            assert np.allclose(tr.read("H", 1, rank=r), refs[r]["cache"]["h"][0], **tol), (strategy, C, r)
-        dW = sum(x["grads"][0][0] for x in refs)
-        assert np.allclose(tr.read("dW", 1, rank=0), dW, **tol), (strategy, C)
+            assert_close(tr.read("H", 1, rank=r), refs[r]["cache"]["h"][0], dtype, f"{strategy} C{C} H1 rank {r}",
+                         bds[r]["H"][0])
+        sb = sum_bounds(bds)
+        for l in range(1, len(cfg.fanouts) + 1):
+            assert_close(tr.read("dW", l, rank=0), sum(x["grads"][l - 1][0] for x in refs), dtype,
+                         f"{strategy} C{C} dW{l}", sb["dW"][l - 1])

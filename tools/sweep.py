@@ -4,10 +4,10 @@ line with the measured 1-GPU step (GDP, CUDA graph, L2 flushed), the Planner's E
 prediction per strategy at C = 2, 4, 8 and every strategy's step with C ranks emulated
 on this GPU (C <= --emulate-max-c).  Uses bench.py's trainer / planner code.
 
-  python scratch/sweep.py papers-d         # config 3: papers, d in {64, 256}
-  python scratch/sweep.py friendster-h     # config 4: friendster d=256, hidden {8, 32, 128}
-  python scratch/sweep.py papers-gat       # config 5: papers d=128, GAT 4 heads, hidden 32..1024
-  python scratch/sweep.py products-fanout  # fanouts [10,5], [15,10], [20,15,10]
+  python tools/sweep.py papers-d         # config 3: papers, d in {64, 256}
+  python tools/sweep.py friendster-h     # config 4: friendster d=256, hidden {8, 32, 128}
+  python tools/sweep.py papers-gat       # config 5: papers d=128, GAT 4 heads, hidden 32..1024
+  python tools/sweep.py products-fanout  # fanouts [10,5], [15,10], [20,15,10]
 """
 import argparse
 import json
