@@ -233,3 +233,71 @@ def test_tiered_store_classification_invariants(tiny_graph):
         assert newly_local.sum() == int((t(r, hot) != 0).sum()) > 0
         assert np.all(np.isin(ids[newly_local], hot))
         assert np.array_equal(tc(r, ids)[~newly_local], t(r, ids)[~newly_local])
+
+
+@pytest.mark.parametrize("C", [2, 4])
+def test_predict_prices_each_term_with_its_operator(tiny_graph, tiny_cfg, C):
+    """Eq. 2 branch by branch.  (1) alpha = 0, T_build = 0 and a DIFFERENT beta
+    for every operator: each strategy's prediction is exactly its own byte terms, each over
+    its own operator -- feature rows local / peer; NFP's graph all-gather,
+    forward reduce-scatter and backward all-gather (Z15); SNP / DNP's all-to-alls (Z16)
+    -- maximised over ranks (Z13).  (2) beta -> infinity, a DIFFERENT alpha per operator:
+    exactly its calls x alpha (Z23).  (3) the hidden bytes priced are the paper's volumes
+    (P:147 NFP 2d'CN_d of which (C-1)/C crosses the wire, P:148 SNP 2d'N_vs, P:161 DNP
+    2d'N_vd), written out here from N_d, N_vs, N_vd.  A mis-assigned beta or alpha fails."""
+    d, dd, hb = tiny_cfg.dim, tiny_cfg.hidden, 4
+    beta = [1.0e9 * (i + 2) for i in range(8)]            # all distinct
+    alpha = [1.0e-6 * (i + 3) for i in range(8)]
+    stats, exp_b, exp_a = [], [], []
+    for s in S.STRATEGIES:
+        blocks, part, gb, seeds = _rank_blocks(tiny_graph, tiny_cfg, C, s)
+        st = S.emulate_layer1(s, blocks, part, C, d, dd)
+        for x in st:
+            x["steps"] = 1
+        stats.append(st)
+        tb, ta = [], []
+        for x in st:
+            t = x["feat_bytes_local"] / beta[S.OP_LOCAL_GATHER] + x["feat_bytes_peer"] / beta[S.OP_PEER_PULL]
+            a = alpha[S.OP_LOCAL_GATHER] + (alpha[S.OP_PEER_PULL] if x["feat_bytes_peer"] else 0.0)
+            if s == "NFP":
+                t += (x["graph_bytes"] + x["hidden_bytes_bwd"]) / beta[S.OP_ALLGATHER] \
+                    + x["hidden_bytes_fwd"] / beta[S.OP_REDUCE_SCATTER]
+                a += 2 * alpha[S.OP_ALLGATHER] + alpha[S.OP_REDUCE_SCATTER]
+            elif s in ("SNP", "DNP"):
+                t += (x["graph_bytes"] + x["hidden_bytes_fwd"] + x["hidden_bytes_bwd"]) / beta[S.OP_ALLTOALLV]
+                a += 3 * alpha[S.OP_ALLTOALLV]
+            tb.append(t)
+            ta.append(a)
+        exp_b.append(max(tb))
+        exp_a.append(max(ta))
+        hidden = sum(x["hidden_bytes_fwd"] + x["hidden_bytes_bwd"] for x in st)
+        if s == "NFP":
+            assert hidden * C == 2 * dd * C * sum(x["n_d"] for x in st) * hb * (C - 1)
+        elif s == "SNP":
+            assert hidden == 2 * dd * sum(x["n_vs"] for x in st) * hb
+        elif s == "DNP":
+            assert hidden == 2 * dd * sum(x["n_vd"] for x in st) * hb
+        else:
+            assert hidden == 0
+    zero = [[0.0] * C for _ in range(4)]
+    pred, pick = S.predict(stats, [0.0] * 8, beta, zero)
+    assert pred == pytest.approx(exp_b, rel=1e-12) and pick == int(np.argmin(exp_b))
+    pred_a, _ = S.predict(stats, alpha, [1e300] * 8, zero)
+    assert pred_a == pytest.approx(exp_a, rel=1e-12)
+
+
+def test_epoch_perm_is_sorted_by_philox_key_then_id():
+    """O1 exactly: perm = train ascending by (key, u), key(u) = word0 | word1 << 32 of
+    Philox_PERM(seed; {u_lo, u_hi, epoch, 0}) -- keys recomputed here from the KAT-pinned
+    Philox block function (oracle.philox), not from orc_perm_key.  Ties (none expected
+    among 64-bit keys) break by u; checked on the full order."""
+    train = np.arange(7, 40000, 5, dtype=np.int64)
+    seed, epoch = 0x1234_5678_9ABC, 3
+    perm = oracle.epoch_perm(train, seed, epoch)
+    key = (seed & 0xFFFFFFFF, ((seed >> 32) & 0xFFFFFFFF) ^ oracle.DOMAIN["PERM"])
+    keys = {}
+    for u in train:
+        w = oracle.philox([u & 0xFFFFFFFF, u >> 32, epoch, 0], key)
+        keys[int(u)] = int(w[0]) | (int(w[1]) << 32)
+    expect = sorted(train.tolist(), key=lambda u: (keys[u], u))
+    assert perm.tolist() == expect
