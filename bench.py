@@ -470,8 +470,12 @@ def planner_report(A, g, cfg, train, labels, args, stream, gdp_ms):
         for h in (tr, fs, gr):
             h.close()
         ctx.close()
-    rep["C1"] = {"measured_ms_per_step": {s: gdp_ms for s in STRATS}, "pick": "GDP",
-                 "note": "at C = 1 every strategy degenerates to GDP (SURVEY §8(d))"}
+    # C = 1: every strategy through its own driver (identity exchanges), timed
+    em1 = emulated_strategy_times(A, g, cfg, train, labels, 1, dt, stream)
+    rep["C1"] = {"measured_ms_per_step": em1, "bench_gdp_ms_per_step": gdp_ms, "pick": "GDP",
+                 "fastest": min(em1, key=em1.get),
+                 "note": "at C = 1 every strategy degenerates to GDP's arithmetic; each ran through its own "
+                         "driver (5 steps, CUDA graph, no L2 flush); GDP is also the timed bench step"}
     return rep
 
 
@@ -483,7 +487,7 @@ def emulated_strategy_times(A, g, cfg, train, labels, C, dt, stream, steps=5):
     import torch
     out = {}
     for s in STRATS:
-        ctx = A.Ctx(-1, C, 0, stream.cuda_stream)
+        ctx = A.Ctx(-1, C, 0, stream.cuda_stream) if C > 1 else A.Ctx(0, 1, 0, stream.cuda_stream)
         gr = ctx.graph_load(g.indptr, g.indices, partition(A, g, C))
         fs = ctx.fstore_create(gr, A.NFP if s == "NFP" else A.GDP, dt, cfg.dim, None, cfg.feat_seed)
         tr = make_trainer(A, ctx, gr, fs, cfg, dt, A.STRATEGY[s], labels)
@@ -536,16 +540,26 @@ def skew_table(counts, edges=(0.01, 0.05, 0.10, 0.20, 0.50, 1.0)):
 
 def step_phase_bytes(ctx, gr, g, tr, cfg, rank, step, bf):
     """Algorithmic HBM bytes of one whole GDP step at C = 1, per phase (SURVEY §8(d)'s
-    per-phase table): sampling (indptr sector + neighbour sectors + writes),
-    compaction, the layer-1 gather of unique rows + mean, every projection, the upper
-    layers' means, loss, backward (dZ = G W, the mean's backward, weight gradients) and
-    SGD.  Block sizes come from apt_sample on the same seeds and step."""
+    per-phase table), every tensor counted at the width the path stores
+    it: bf16 mode keeps Z, the hidden activations (R11), the backward's G (R4) and
+    dZ / deg (R13) and the weights' copies in bf16, the logits and their gradient in
+    fp32; fp32 mode keeps everything in fp32.  Phases: sampling (indptr sector +
+    neighbour sectors + writes), compaction (+ the block transposes of the upper hops),
+    the layer-1 gather of unique rows + mean, every projection, the upper layers'
+    means, loss, backward (dZ = G W, the mean's backward reading the mask and writing
+    G, every dW = G^T Z) and SGD.  Block sizes come from apt_sample on the same seeds
+    and step."""
+    seeds_h = tr.read("seeds", rank=rank)[:, 0].astype(np.int64)
     import torch
-    seeds = torch.as_tensor(tr.read("seeds", rank=rank)[:, 0].astype(np.int64)).cuda()
+    seeds = torch.as_tensor(seeds_h).cuda()
     K = len(cfg.fanouts)
     b = ctx.sample(gr, seeds, len(seeds), cfg.fanouts, cfg.sample_seed, step)
     dims = [cfg.dim] + [o for _, o in cfg.dims()]
-    bz = bg = bw = bf                    # Z, G and W copies in the compute dtype; H, dZ fp32
+    half = bf == 2
+    b_z = b_w = 2 if half else 4      # Z, bf16 weight copies (tensor-core operands)
+    b_h = 2 if half else 4            # hidden activations as stored (R11)
+    b_g = 2 if half else 4            # G read by the contractions / written by the pull (R4)
+    b_dz = 2 if half else 4           # dZ / deg rows (R13)
     ph = {"sampling": 0, "compaction": 0, "layer1_gather_mean": 0, "projections": 0, "upper_means": 0,
           "loss": 0, "backward": 0, "sgd": 0}
     for h in range(K):
@@ -555,23 +569,25 @@ def step_phase_bytes(ctx, gr, g, tr, cfg, rank, step, bf):
         nb = np.where(deg <= k, (4 * deg + 31) // 32 * 32, k * 32)
         E = int(indptr[-1]) if len(indptr) else 0
         N, U = len(dst), len(src)
-        ph["sampling"] += N * 32 + int(nb.sum()) + N * k * 8
-        ph["compaction"] += E * 12 + U * 8
         layer = K - h
         din, dout = dims[layer - 1], dims[layer]
+        ph["sampling"] += N * 32 + int(nb.sum()) + N * k * 8
+        ph["compaction"] += E * 12 + U * 8 + (E * 12 if layer > 1 else 0)     # + block transpose
         if layer == 1:
-            ph["layer1_gather_mean"] += U * din * bf + E * 4 + (N + 1) * 4 + N * din * bz
-            ph["backward"] += N * (dout * bg + din * bz)                          # dW1 = G^T Z
+            ph["layer1_gather_mean"] += U * din * bf + E * 4 + (N + 1) * 4 + N * din * b_z
+            ph["backward"] += N * (dout * b_g + din * b_z)                      # dW1 = G^T Z
         else:
-            ph["upper_means"] += U * din * 4 + E * 4 + (N + 1) * 4 + N * din * bz
-            ph["backward"] += (N * dout * bg + din * dout * bw + N * din * 4      # dZ = G W
-                               + N * din * 4 + E * 4 + U * din * (4 + bg)         # mean bwd (mask, G)
-                               + N * (dout * bg + din * bz))                      # dW = G^T Z
-        ph["projections"] += N * din * bz + N * dout * 4 + din * dout * bw
+            ph["upper_means"] += U * din * b_h + E * 4 + (N + 1) * 4 + N * din * b_z
+            ph["backward"] += (N * dout * b_g + din * dout * b_w + N * din * b_dz   # dZ = (G W) / deg
+                               + N * din * b_dz + E * 8 + U * din * b_h            # pull: dZ, (v, deg), mask
+                               + U * din * b_g                                     # ... writes G_{l-1}
+                               + N * (dout * b_g + din * b_z))                      # dW = G^T Z
+        b_out = 4 if layer == K else b_h                                            # logits fp32
+        ph["projections"] += N * din * b_z + N * dout * b_out + din * dout * b_w
         if layer == K:
-            ph["loss"] += N * dout * 4 * 2
+            ph["loss"] += N * dout * 4 + N * dout * (4 + (2 if half else 0))        # logits -> G (+ bf16 copy)
     nparam = sum(dims[i] * dims[i + 1] + dims[i + 1] for i in range(K))
-    ph["sgd"] = nparam * (4 + 4 + 4 + bw)
+    ph["sgd"] = nparam * (4 + 4 + 4 + b_w)
     b.close()
     return ph
 

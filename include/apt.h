@@ -347,6 +347,13 @@ apt_status apt_select_strategy(const apt_plan_stats* st, const apt_bw_profile* b
  * numerators; 0 expected, < 0 on a CUDA failure.  Uses the current device.      */
 int64_t apt_selftest_div(void);
 
+/* Self-test of the epoch permutation's sort (S1, reading O1; sort.cu): n (key, value)
+ * pairs with Philox keys masked to key_bits bits (equal keys when key_bits is small),
+ * values 0..n-1, sorted on the device by the library's stable LSD radix sort; returns
+ * the number of positions that differ from a host std::stable_sort, < 0 on failure.
+ * Uses the current device; syncs.                                                    */
+int64_t apt_selftest_sort(int64_t n, uint64_t seed, int key_bits);
+
 #ifdef __cplusplus
 }
 #endif

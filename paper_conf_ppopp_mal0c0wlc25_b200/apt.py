@@ -133,6 +133,8 @@ def lib():
         L.apt_exchange_selftest.restype = st
         L.apt_selftest_div.argtypes = []
         L.apt_selftest_div.restype = C.c_int64
+        L.apt_selftest_sort.argtypes = [i64, u64, i32]
+        L.apt_selftest_sort.restype = C.c_int64
         L.apt_trainer_steps_per_epoch.argtypes = [vp]
         L.apt_trainer_steps_per_epoch.restype = C.c_int64
         _lib = L

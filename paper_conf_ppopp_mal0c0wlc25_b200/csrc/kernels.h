@@ -65,6 +65,9 @@ struct SeedArgs {
   const int32_t* n_dev;        // if set: perm is one global batch of *n_dev ids (host-batch path)
 };
 cudaError_t launch_select_seeds(const SeedArgs& a, cudaStream_t st);
+// sort.cu: stable LSD radix sort of (uint64 key, int32 value) pairs in place (S1, O1).
+size_t radix_sort_pairs_scratch(int64_t n);
+cudaError_t launch_radix_sort_pairs(uint64_t* keys, int32_t* vals, int64_t n, void* scratch, cudaStream_t st);
 cudaError_t launch_perm_keys(const int32_t* train, int64_t n, uint64_t seed, uint64_t epoch, uint64_t* keys,
                              cudaStream_t st);
 

@@ -16,7 +16,6 @@
 #include <functional>
 #include <vector>
 #include <cstring>
-#include <cub/device/device_radix_sort.cuh>
 
 #include "common.cuh"
 #include "trainer.h"
@@ -512,24 +511,17 @@ apt_status apt_trainer_set_epoch(apt_trainer* t, const int64_t* train, int64_t n
   t->steps_per_epoch = ceil_div(n_train, int64_t(t->world) * t->m.batch);
   t->primed = -1;   // a prefetched batch belongs to the previous permutation
   t->host_primed = false;
-  int32_t *tr_dev = nullptr, *tmp_vals = nullptr;
-  uint64_t *k_in = nullptr, *k_out = nullptr;
-  void* tmp = nullptr;
-  size_t tmp_bytes = 0;
-  CK(c, cudaMallocAsync(&tr_dev, sizeof(int32_t) * n_train, c->stream));
-  CK(c, cudaMallocAsync(&tmp_vals, sizeof(int32_t) * n_train, c->stream));
-  CK(c, cudaMallocAsync(&k_in, sizeof(uint64_t) * n_train, c->stream));
-  CK(c, cudaMallocAsync(&k_out, sizeof(uint64_t) * n_train, c->stream));
-  CK(c, cudaMemcpyAsync(tr_dev, h.data(), sizeof(int32_t) * n_train, cudaMemcpyHostToDevice, c->stream));
-  CK(c, launch_perm_keys(tr_dev, n_train, t->m.sample_seed, epoch, k_in, c->stream));
-  // stable LSD radix sort by key: ties keep the ascending id order (reading O1)
-  CK(c, cub::DeviceRadixSort::SortPairs(nullptr, tmp_bytes, k_in, k_out, tr_dev, t->perm, int(n_train), 0, 64, c->stream));
-  CK(c, cudaMallocAsync(&tmp, tmp_bytes, c->stream));
-  CK(c, cub::DeviceRadixSort::SortPairs(tmp, tmp_bytes, k_in, k_out, tr_dev, t->perm, int(n_train), 0, 64, c->stream));
-  c->launches += 6;
-  for (void* p : {static_cast<void*>(tr_dev), static_cast<void*>(tmp_vals), static_cast<void*>(k_in),
-                  static_cast<void*>(k_out), tmp})
-    CK(c, cudaFreeAsync(p, c->stream));
+  uint64_t* keys = nullptr;
+  void* scratch = nullptr;
+  CK(c, cudaMallocAsync(&keys, sizeof(uint64_t) * n_train, c->stream));
+  CK(c, cudaMallocAsync(&scratch, radix_sort_pairs_scratch(n_train), c->stream));
+  CK(c, cudaMemcpyAsync(t->perm, h.data(), sizeof(int32_t) * n_train, cudaMemcpyHostToDevice, c->stream));
+  CK(c, launch_perm_keys(t->perm, n_train, t->m.sample_seed, epoch, keys, c->stream));
+  // stable LSD radix sort by key (sort.cu): ties keep the ascending id order (reading O1)
+  CK(c, launch_radix_sort_pairs(keys, t->perm, n_train, scratch, c->stream));
+  c->launches += 1 + 24;
+  CK(c, cudaFreeAsync(keys, c->stream));
+  CK(c, cudaFreeAsync(scratch, c->stream));
   CK(c, cudaStreamSynchronize(c->stream));
   return APT_OK;
 }

@@ -121,3 +121,21 @@ def test_products_bench_step_bf16_vs_unrounded_fp64(A, products):
         assert_close(tr.read("db", l)[0], db, "bf16u", f"db layer {l} (unrounded ref)", bd["db"][l - 1])
     tr.close()
     ctx.close()
+
+
+def test_products_epoch_permutation_full_train(A, products):
+    """S1 at full size: the device permutation (Philox keys + the library's radix sort) of a
+    1.2 M-id train set equals oracle.epoch_perm, read back through the seeds of the first,
+    a middle and the short last step (O1, R6)."""
+    cfg, g, _, labels = products
+    train = np.arange(1, g.n, 2, dtype=np.int64)           # 1.2 M ascending ids
+    ctx, tr = _bench_trainer(A, cfg, g, train, labels, "bf16")
+    tr.set_epoch(train, 5)
+    perm = oracle.epoch_perm(train, cfg.sample_seed, 5)
+    spe = tr.steps_per_epoch()
+    assert spe == -(-len(train) // cfg.batch)
+    for s in (0, spe // 2, spe - 1):
+        tr.step(s, update=False)
+        assert np.array_equal(tr.read("seeds")[:, 0], perm[s * cfg.batch:(s + 1) * cfg.batch]), s
+    tr.close()
+    ctx.close()

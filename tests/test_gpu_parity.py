@@ -127,6 +127,13 @@ def test_mean_division_is_ieee_exhaustive(A, ctx):
     agree bit for bit with IEEE x/d on every O4 mean (O5) -- 67M operands."""
     assert A.lib().apt_selftest_div() == 0
 
+@pytest.mark.parametrize("n,bits", [(1, 64), (2049, 3), (300001, 12), (1200000, 64), (65536, 1)])
+def test_epoch_sort_stable_radix(A, ctx, n, bits):
+    """S1's own radix sort (sort.cu) is a STABLE sort by the 64-bit key (equal keys keep the
+    input order, reading O1's tie rule): against a host stable sort, with many equal keys."""
+    assert A.lib().apt_selftest_sort(n, 77, bits) == 0
+
+
 def test_aggregate_bit_exact_and_bwd(A, ctx, tiny):
     cfg, g, train = tiny
     gr = ctx.graph_load(g.indptr, g.indices)
