@@ -68,14 +68,18 @@ typedef struct apt_trainer apt_trainer;
 
 /* A sampled bipartite block: dst ids are the prefix of src ids;
  * CSR over local source positions.  Device pointers, borrowed from the
- * owning apt_batch; int32 node ids.                                         */
+ * owning apt_batch (valid until it is destroyed); node ids int64 (ABI rule),
+ * local positions int32.                                                    */
 typedef struct {
   int64_t n_dst, n_src, n_edges;
-  const int32_t* dst_ids;  /* [n_dst]   global ids (device)                 */
-  const int32_t* src_ids;  /* [n_src]   global ids, dst prefix (device)     */
+  const int64_t* dst_ids;  /* [n_dst]   global ids (device)                 */
+  const int64_t* src_ids;  /* [n_src]   global ids, dst prefix (device)     */
   const int32_t* indptr;   /* [n_dst+1] (device)                            */
   const int32_t* indices;  /* [n_edges] positions into src_ids (device)     */
 } apt_block_view;
+
+/* State the standalone first-layer forward keeps for its backward (apt_layer_fwd). */
+typedef struct apt_layer_saved apt_layer_saved;
 
 /* Model + sampler of the training task (the user's "specifics"). */
 typedef struct {
@@ -220,11 +224,18 @@ apt_status apt_sample(apt_ctx* ctx, const apt_graph* g, const int64_t* seeds_dev
                       apt_batch** out);
 apt_status apt_batch_block(const apt_batch* b, int hop, apt_block_view* out);
 apt_status apt_batch_destroy(apt_batch* b);
+/* A ctx hosting several ranks (rank = -1 emulation) runs the layer API on one batch
+ * per hosted rank: per_rank[i] is hosted rank i's batch (same graph, K, fanouts,
+ * rng_seed and step).  The group borrows the batches: keep them alive until the group
+ * is destroyed (apt_batch_destroy).  apt_batch_block on a group -> APT_E_INVALID.    */
+apt_status apt_batch_group(apt_ctx* ctx, const apt_batch* const* per_rank, int n, apt_batch** out);
 
 /* ------------------------------------------------------------ single ops */
-/* Gather rows of ids_dev (device int32[n]) from rank-0's view of the store
- * into out_dev (device, rows of the store's padded pitch, store dtype).     */
-apt_status apt_gather(apt_ctx* ctx, const apt_fstore* f, const int32_t* ids_dev, int64_t n, void* out_dev);
+/* Gather rows of ids_dev (device int64[n], node ids) from this rank's view of the
+ * store (own shard, NVLink peers, host tier, cache) into out_dev
+ * (device, rows of the store's padded pitch, store dtype).  An id outside
+ * [0, n_nodes) -> APT_E_DEVICE_ASSERT at the next sync (its row is node 0's).  */
+apt_status apt_gather(apt_ctx* ctx, const apt_fstore* f, const int64_t* ids_dev, int64_t n, void* out_dev);
 /* Segmented mean (O5): z[v] = mean_{e in row v} x[indices[e]].  x_src device
  * [n_src x x_pitch] of dtype; z_dst device fp32 [n_dst x z_pitch].          */
 apt_status apt_aggregate(apt_ctx* ctx, const apt_block_view* blk, const void* x_src, apt_dtype dtype,
@@ -290,17 +301,41 @@ apt_status apt_trainer_use_graph(apt_trainer* t, int enable);
  * P:299 "sampling" overlapped).  Results are identical with it off.          */
 apt_status apt_trainer_set_pipeline(apt_trainer* t, int enable);
 
-/* The first GNN layer alone under the trainer's strategy -- the layer APT
- * parallelises (upper layers are data parallel and may be the
- * caller's own).  apt_layer_fwd: seeds of `step`, K-hop sampling and the layer-1
- * Permute/Shuffle/Execute/Reshuffle for every hosted rank; h^1 is read
- * with apt_trainer_read(H, layer 1).  Async.
- * apt_layer_bwd: dh1[i] = device fp32 dL/dh^1 of hosted rank i (rows = its layer-1
- * destinations, `pitch` floats apart); computes dL/dpre^1 (ReLU mask when K > 1)
- * and dW^1, db^1 of the strategy (owners' g^T Z, requester db), all-reduced over
- * the ranks (NFP: column-owned slices, read back concatenated).  Async.        */
-apt_status apt_layer_fwd(apt_trainer* t, int64_t step);
-apt_status apt_layer_bwd(apt_trainer* t, const float* const* dh1, int64_t pitch);
+/* The first GNN layer alone -- the layer APT parallelises (the
+ * sampler and the upper layers are the user's black boxes).
+ *
+ * apt_layer_fwd: h1 = ReLU(mean-aggregate(x) W^T + bias) of the layer-1 block of
+ *   `batch` (hop K-1 of apt_sample's output; Eq. 1 with W after the mean, Z8; ReLU
+ *   because layer 1 is a hidden layer, Z9) under `strategy`'s Permute / Shuffle /
+ *   Execute / Reshuffle.  Collective for a multi-process job.
+ *   batch: this rank's batch, or for an emulated ctx an apt_batch_group of every
+ *   hosted rank's batch.  fstore: laid out for the strategy (NFP: column-sharded),
+ *   its dtype = `dtype`.  W: device fp32 [d_out x d] row-major, bias: device fp32
+ *   [d_out] (replicated: every rank passes the same values).  h1_out: device fp32
+ *   [rows x d_out], the hosted ranks' layer-1 destinations concatenated in rank
+ *   order (rows = sum of n_dst of each batch's layer-1 block); bf16 mode writes the
+ *   stored bf16 activation (R11) widened to fp32.  *saved: library-owned, needed by
+ *   apt_layer_bwd, released with apt_layer_saved_destroy.  Async (one host sync while
+ *   staging the blocks).
+ * apt_layer_bwd: dh1 = device fp32 dL/dh1 in h1_out's layout; computes g = dh1 *
+ *   ReLU'(pre) and dW = g^T Z (owners' partial sums, NFP column-owned slices), db = g^T 1
+ *   at the requester (R3), all-reduced over the ranks.  dW: device fp32
+ *   [d_out x d]: the full gradient (NFP: the hosted ranks' column slices, other columns
+ *   untouched); dbias: device fp32 [d_out].  Collective; async.                      */
+apt_status apt_layer_fwd(apt_ctx* ctx, apt_strategy strategy, const apt_batch* batch, const apt_fstore* fstore,
+                         const float* W, const float* bias, int d_out, apt_dtype dtype, float* h1_out,
+                         apt_layer_saved** saved);
+apt_status apt_layer_bwd(apt_ctx* ctx, apt_layer_saved* saved, const float* dh1, float* dW, float* dbias);
+apt_status apt_layer_saved_destroy(apt_layer_saved* saved);
+
+/* The same first layer bound to a trainer (its model, epoch and strategy):
+ * apt_trainer_layer_fwd samples step `step` of the epoch for every hosted rank and runs
+ * the layer-1 forward (SAGE or GAT); h^1 is read with apt_trainer_read(H, layer 1).
+ * apt_trainer_layer_bwd: dh1[i] = device fp32 dL/dh^1 of hosted rank i (rows = its
+ * layer-1 destinations, `pitch` floats apart); dW^1, db^1 (GAT: also da_src, da_dst)
+ * of the strategy, all-reduced (NFP: column-owned slices).  Async.                   */
+apt_status apt_trainer_layer_fwd(apt_trainer* t, int64_t step);
+apt_status apt_trainer_layer_bwd(apt_trainer* t, const float* const* dh1, int64_t pitch);
 
 /* Readouts for tests (syncs).  what: 0 seeds, 1 layer-l dst ids, 2 Z_l (fp32),
  * 3 H_l (post-activation / logits), 4 dW_l, 5 db_l, 6 G_l (dL/dpre),

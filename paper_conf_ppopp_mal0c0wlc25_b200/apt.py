@@ -117,7 +117,9 @@ def lib():
             "apt_trainer_use_graph": [vp, i32], "apt_trainer_set_pipeline": [vp, i32], "apt_trainer_read": [vp, i32, i32, i32, vp, i64, vp, vp],
             "apt_trainer_phase_ms": [vp, vp, i32], "apt_trainer_agg_bytes": [vp, vp],
             "apt_partition": [i64, i64, vp, vp, i32, i32, u64, vp, vp],
-            "apt_dryrun": [vp, i64, vp], "apt_access_counts": [vp, i64, vp], "apt_hot_rows": [vp, i64, i64, vp], "apt_layer_fwd": [vp, i64], "apt_layer_bwd": [vp, vp, i64], "apt_profile_links": [vp, vp], "apt_select_strategy": [vp, vp, vp, vp],
+            "apt_dryrun": [vp, i64, vp], "apt_access_counts": [vp, i64, vp], "apt_hot_rows": [vp, i64, i64, vp], "apt_trainer_layer_fwd": [vp, i64], "apt_trainer_layer_bwd": [vp, vp, i64],
+            "apt_layer_fwd": [vp, i32, vp, vp, vp, vp, i32, i32, vp, vp], "apt_layer_bwd": [vp, vp, vp, vp, vp],
+            "apt_layer_saved_destroy": [vp], "apt_batch_group": [vp, vp, i32, vp], "apt_profile_links": [vp, vp], "apt_select_strategy": [vp, vp, vp, vp],
         }
         for name, args in sig.items():
             f = getattr(L, name)
@@ -226,6 +228,9 @@ class Ctx:
         return Batch(self, h)
 
     def gather(self, fstore, ids_dev, n, out_dev):
+        """apt_gather: ids_dev int64 node ids (ABI rule)."""
+        if hasattr(ids_dev, "dtype") and str(ids_dev.dtype) not in ("torch.int64", "int64"):
+            raise AptError(1, f"apt_gather: ids must be int64, got {ids_dev.dtype}")
         self.ck(lib().apt_gather(self.h, fstore.h, _ptr(ids_dev), n, _ptr(out_dev)))
 
     def aggregate(self, view, x_dev, dtype, dim, x_pitch, z_dev, z_pitch):
@@ -241,6 +246,27 @@ class Ctx:
     def weight_grad(self, G_dev, g_pitch, Z_dev, z_pitch, dtype, rows, d_out, d_in, dW_dev, db_dev=None):
         self.ck(lib().apt_weight_grad(self.h, _ptr(G_dev), g_pitch, _ptr(Z_dev), z_pitch, dtype, rows, d_out, d_in,
                                       _ptr(dW_dev), _ptr(db_dev)))
+
+    def batch_group(self, batches):
+        """apt_batch_group: one batch per hosted rank (emulated ctx) -> a group batch."""
+        arr = (C.c_void_p * len(batches))(*[b.h for b in batches])
+        h = C.c_void_p()
+        self.ck(lib().apt_batch_group(self.h, arr, len(batches), C.byref(h)))
+        g = Batch(self, h)
+        g._keep = (self,) + tuple(batches)          # the group borrows its members
+        return g
+
+    def layer_fwd(self, strategy, batch, fstore, W_dev, bias_dev, d_out, dtype, h1_dev):
+        """apt_layer_fwd: the first layer of `batch` under `strategy`; returns
+        the saved state for layer_bwd.  h1_dev: fp32 [rows x d_out], ranks concatenated."""
+        h = C.c_void_p()
+        self.ck(lib().apt_layer_fwd(self.h, strategy, batch.h, fstore.h, _ptr(W_dev), _ptr(bias_dev), d_out, dtype,
+                                    _ptr(h1_dev), C.byref(h)))
+        return Handle(h, lib().apt_layer_saved_destroy, keep=(self, batch, fstore))
+
+    def layer_bwd(self, saved, dh1_dev, dW_dev, db_dev):
+        """apt_layer_bwd: dW [d_out x d] and db [d_out] (device fp32) of the strategy."""
+        self.ck(lib().apt_layer_bwd(self.h, saved.h, _ptr(dh1_dev), _ptr(dW_dev), _ptr(db_dev)))
 
     def profile_links(self):
         bw = BwProfile()
@@ -275,11 +301,12 @@ class Batch(Handle):
         return v
 
     def block_host(self, hop):
-        """Copy a block to host numpy arrays (dst, src, indptr, indices)."""
+        """Copy a block to host numpy arrays (dst, src int64 node ids; indptr, indices int32)."""
         v = self.block(hop)
         out = []
-        for ptr, n in ((v.dst_ids, v.n_dst), (v.src_ids, v.n_src), (v.indptr, v.n_dst + 1), (v.indices, v.n_edges)):
-            a = np.empty(n, np.int32)
+        for ptr, n, dt in ((v.dst_ids, v.n_dst, np.int64), (v.src_ids, v.n_src, np.int64),
+                           (v.indptr, v.n_dst + 1, np.int32), (v.indices, v.n_edges, np.int32)):
+            a = np.empty(n, dt)
             if n:
                 self.ctx.d2h(a, ptr)
             out.append(a)
@@ -387,12 +414,13 @@ class Trainer(Handle):
         return list(ms)
 
     def layer_fwd(self, step):
-        self.ctx.ck(lib().apt_layer_fwd(self.h, step))
+        """apt_trainer_layer_fwd: sample step `step` of the epoch, run layer 1."""
+        self.ctx.ck(lib().apt_trainer_layer_fwd(self.h, step))
 
     def layer_bwd(self, dh1_list, pitch):
-        """dh1_list: one device tensor per hosted rank (fp32 [rows x pitch])."""
+        """apt_trainer_layer_bwd.  dh1_list: one device tensor per hosted rank (fp32 [rows x pitch])."""
         arr = (C.c_void_p * len(dh1_list))(*[_ptr(x) for x in dh1_list])
-        self.ctx.ck(lib().apt_layer_bwd(self.h, arr, pitch))
+        self.ctx.ck(lib().apt_trainer_layer_bwd(self.h, arr, pitch))
 
     def access_counts(self, n_steps):
         """apt_access_counts: per-node input-row loads over the first n_steps steps (Table 3)."""

@@ -65,6 +65,9 @@ struct SeedArgs {
   const int32_t* n_dev;        // if set: perm is one global batch of *n_dev ids (host-batch path)
 };
 cudaError_t launch_select_seeds(const SeedArgs& a, cudaStream_t st);
+// layer_api.cu: int32 <-> int64 node ids at the ABI.
+cudaError_t launch_widen_ids(const int32_t* a, int64_t n, int64_t* b, cudaStream_t st);
+cudaError_t launch_narrow_ids(const int64_t* a, int64_t n, int64_t n_nodes, int32_t* b, uint32_t* err, cudaStream_t st);
 // sort.cu: stable LSD radix sort of (uint64 key, int32 value) pairs in place (S1, O1).
 size_t radix_sort_pairs_scratch(int64_t n);
 cudaError_t launch_radix_sort_pairs(uint64_t* keys, int32_t* vals, int64_t n, void* scratch, cudaStream_t st);

@@ -255,3 +255,32 @@ cudaError_t launch_transpose(const float* src, int rows, int cols, float* dst, c
 }
 
 }  // namespace apt
+
+namespace apt {
+// Node ids are int64 at the ABI and int32 inside (n_nodes < 2^31).
+__global__ void widen_ids_kernel(const int32_t* __restrict__ a, int64_t n, int64_t* __restrict__ b) {
+  for (int64_t i = int64_t(blockIdx.x) * blockDim.x + threadIdx.x; i < n; i += int64_t(gridDim.x) * blockDim.x) b[i] = a[i];
+}
+__global__ void narrow_ids_kernel(const int64_t* __restrict__ a, int64_t n, int64_t n_nodes, int32_t* __restrict__ b,
+                                  uint32_t* err) {
+  for (int64_t i = int64_t(blockIdx.x) * blockDim.x + threadIdx.x; i < n; i += int64_t(gridDim.x) * blockDim.x) {
+    const int64_t v = a[i];
+    if (v < 0 || v >= n_nodes) {
+      atomicOr(err, kDevErrBadId);
+      b[i] = 0;
+    } else {
+      b[i] = int32_t(v);
+    }
+  }
+}
+cudaError_t launch_widen_ids(const int32_t* a, int64_t n, int64_t* b, cudaStream_t st) {
+  if (n <= 0) return cudaSuccess;
+  widen_ids_kernel<<<unsigned(grid_cap(ceil_div(n, 256), 16)), 256, 0, st>>>(a, n, b);
+  return cudaGetLastError();
+}
+cudaError_t launch_narrow_ids(const int64_t* a, int64_t n, int64_t n_nodes, int32_t* b, uint32_t* err, cudaStream_t st) {
+  if (n <= 0) return cudaSuccess;
+  narrow_ids_kernel<<<unsigned(grid_cap(ceil_div(n, 256), 16)), 256, 0, st>>>(a, n, n_nodes, b, err);
+  return cudaGetLastError();
+}
+}  // namespace apt

@@ -441,6 +441,10 @@ apt_status apt_sample(apt_ctx* c, const apt_graph* g, const int64_t* seeds_dev, 
   b->ctx = c;
   ctx_retain(c);
   b->K = K;
+  b->g = g;
+  b->rng_seed = rng_seed;
+  b->step = step;
+  for (int l = 0; l < K; ++l) b->fanouts[l] = fanouts[l];
   const int64_t n_words = ceil_div(g->n, 32);
   uint32_t* dst_bm = b->arena.alloc<uint32_t>(n_words, true);
   uint32_t* new_bm = b->arena.alloc<uint32_t>(n_words, true);
@@ -498,6 +502,8 @@ apt_status apt_sample(apt_ctx* c, const apt_graph* g, const int64_t* seeds_dev, 
     b->src[h] = src;
     b->indptr[h] = indptr;
     b->indices[h] = indices;
+    b->cnt[h] = cnt;
+    b->nbr[h] = nbr;
     dst = src;
     n_dst = counts + 1 + 2 * h;
     maxF = maxS;
@@ -506,23 +512,61 @@ apt_status apt_sample(apt_ctx* c, const apt_graph* g, const int64_t* seeds_dev, 
   CK(c, cudaMemcpyAsync(hc.data(), counts, sizeof(int32_t) * hc.size(), cudaMemcpyDeviceToHost, c->stream));
   CK(c, cudaStreamSynchronize(c->stream));
   int64_t nd = n_seeds;
+  b->counts = counts;
   for (int h = 0; h < K; ++h) {
     b->n_dst[h] = nd;
     b->n_src[h] = hc[1 + 2 * h];
     b->n_edges[h] = hc[2 + 2 * h];
     nd = b->n_src[h];
+    // int64 ids at the ABI (apt_block_view): widened once here
+    b->dst64[h] = b->arena.alloc<int64_t>(b->n_dst[h], false);
+    b->src64[h] = b->arena.alloc<int64_t>(b->n_src[h], false);
+    if (!b->dst64[h] || !b->src64[h]) {
+      apt_batch_destroy(b);
+      return set_err(c, APT_E_OOM, "apt_sample: out of device memory");
+    }
+    CK(c, launch_widen_ids(b->dst[h], b->n_dst[h], b->dst64[h], c->stream));
+    CK(c, launch_widen_ids(b->src[h], b->n_src[h], b->src64[h], c->stream));
+    c->launches += 2;
   }
+  CK(c, cudaStreamSynchronize(c->stream));
+  *out = b;
+  return APT_OK;
+}
+
+apt_status apt_batch_group(apt_ctx* c, const apt_batch* const* per_rank, int n, apt_batch** out) {
+  if (!c || !per_rank || !out || n < 1 || n > APT_MAX_RANKS || n != c->n_local)
+    return set_err(c, APT_E_INVALID, "apt_batch_group: need one batch per hosted rank (%d)", c ? c->n_local : 0);
+  for (int i = 0; i < n; ++i) {
+    const apt_batch* m = per_rank[i];
+    if (!m || m->ctx != c || !m->members.empty() || m->K != per_rank[0]->K || m->g != per_rank[0]->g ||
+        m->rng_seed != per_rank[0]->rng_seed || m->step != per_rank[0]->step)
+      return set_err(c, APT_E_INVALID, "apt_batch_group: batch %d is not a plain batch of this ctx with the same "
+                                       "graph, K, rng_seed and step", i);
+    for (int l = 0; l < m->K; ++l)
+      if (m->fanouts[l] != per_rank[0]->fanouts[l]) return set_err(c, APT_E_INVALID, "apt_batch_group: fanouts differ");
+  }
+  auto* b = new apt_batch();
+  b->ctx = c;
+  ctx_retain(c);
+  b->g = per_rank[0]->g;
+  b->K = per_rank[0]->K;
+  b->rng_seed = per_rank[0]->rng_seed;
+  b->step = per_rank[0]->step;
+  for (int l = 0; l < b->K; ++l) b->fanouts[l] = per_rank[0]->fanouts[l];
+  b->members.assign(per_rank, per_rank + n);
   *out = b;
   return APT_OK;
 }
 
 apt_status apt_batch_block(const apt_batch* b, int hop, apt_block_view* out) {
   if (!b || !out || hop < 0 || hop >= b->K) return set_err(nullptr, APT_E_INVALID, "apt_batch_block: bad hop");
+  if (!b->members.empty()) return set_err(b->ctx, APT_E_INVALID, "apt_batch_block: a batch group has no single block");
   out->n_dst = b->n_dst[hop];
   out->n_src = b->n_src[hop];
   out->n_edges = b->n_edges[hop];
-  out->dst_ids = b->dst[hop];
-  out->src_ids = b->src[hop];
+  out->dst_ids = b->dst64[hop];
+  out->src_ids = b->src64[hop];
   out->indptr = b->indptr[hop];
   out->indices = b->indices[hop];
   return APT_OK;
@@ -537,11 +581,18 @@ apt_status apt_batch_destroy(apt_batch* b) {
 }
 
 // ------------------------------------------------------------- single ops
-apt_status apt_gather(apt_ctx* c, const apt_fstore* f, const int32_t* ids, int64_t n, void* out) {
+apt_status apt_gather(apt_ctx* c, const apt_fstore* f, const int64_t* ids, int64_t n, void* out) {
   if (!c || !f || (n && (!ids || !out)) || n < 0) return set_err(c, APT_E_INVALID, "apt_gather: bad arguments");
+  if (!n) return APT_OK;
   FeatView v = feat_view(f, c->rank);
-  CK(c, launch_gather(v, ids, nullptr, n, out, v.pitch, c->stream));
-  c->launches++;
+  // int64 ids at the ABI, int32 inside: narrowed on the device, an id
+  // outside [0, n_nodes) sets the device error word (APT_E_DEVICE_ASSERT at the next sync)
+  int32_t* ids32 = nullptr;
+  CK(c, cudaMallocAsync(&ids32, sizeof(int32_t) * n, c->stream));
+  CK(c, launch_narrow_ids(ids, n, f->g->n, ids32, c->dev_err, c->stream));
+  CK(c, launch_gather(v, ids32, nullptr, n, out, v.pitch, c->stream));
+  CK(c, cudaFreeAsync(ids32, c->stream));
+  c->launches += 2;
   return APT_OK;
 }
 

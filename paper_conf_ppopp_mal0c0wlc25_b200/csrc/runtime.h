@@ -144,11 +144,20 @@ struct apt_fstore {
 
 struct apt_batch {
   apt_ctx* ctx = nullptr;
+  const apt_graph* g = nullptr;
   int K = 0;
+  uint64_t rng_seed = 0, step = 0;             // the sampler's Philox key and step id (O2)
+  int fanouts[APT_MAX_LAYERS] = {};            // fanouts[l-1] of layer l
   int64_t n_dst[APT_MAX_LAYERS] = {}, n_src[APT_MAX_LAYERS] = {}, n_edges[APT_MAX_LAYERS] = {};
   int32_t* dst[APT_MAX_LAYERS] = {};
   int32_t* src[APT_MAX_LAYERS] = {};
   int32_t* indptr[APT_MAX_LAYERS] = {};
   int32_t* indices[APT_MAX_LAYERS] = {};
+  int32_t* cnt[APT_MAX_LAYERS] = {};           // the sampler's ELL form of every hop (fixed stride k)
+  int32_t* nbr[APT_MAX_LAYERS] = {};
+  int32_t* counts = nullptr;                   // device: [0] n_seeds, [1 + 2h] n_src(h), [2 + 2h] n_edges(h)
+  int64_t* dst64[APT_MAX_LAYERS] = {};         // int64 copies of the ids for apt_block_view (ABI rule)
+  int64_t* src64[APT_MAX_LAYERS] = {};
+  std::vector<const apt_batch*> members;       // apt_batch_group: one borrowed batch per hosted rank
   apt::Arena arena;
 };

@@ -229,9 +229,21 @@ extern "C" {
 
 apt_status apt_trainer_destroy(apt_trainer* t);
 
+namespace apt {
+// layer_only: a first-layer session of apt_layer_fwd (no labels, no loss)
+apt_status trainer_create(apt_ctx* c, const apt_graph* g, const apt_fstore* f, const apt_model_desc* m,
+                          apt_strategy s, const int32_t* labels, apt_trainer** out, bool layer_only);
+}
+
 apt_status apt_trainer_create(apt_ctx* c, const apt_graph* g, const apt_fstore* f, const apt_model_desc* m,
                               apt_strategy s, const int32_t* labels, apt_trainer** out) {
-  if (!c || !g || !f || !m || !labels || !out || m->n_layers < 1 || m->n_layers > APT_MAX_LAYERS || m->batch < 1 ||
+  if (!labels) return set_err(c, APT_E_INVALID, "apt_trainer_create: labels is null");
+  return apt::trainer_create(c, g, f, m, s, labels, out, false);
+}
+
+apt_status apt::trainer_create(apt_ctx* c, const apt_graph* g, const apt_fstore* f, const apt_model_desc* m,
+                               apt_strategy s, const int32_t* labels, apt_trainer** out, bool layer_only) {
+  if (!c || !g || !f || !m || (!labels && !layer_only) || !out || m->n_layers < 1 || m->n_layers > APT_MAX_LAYERS || m->batch < 1 ||
       s < APT_GDP || s > APT_DNP)
     return set_err(c, APT_E_INVALID, "apt_trainer_create: bad arguments");
   if (m->dims[0] != f->dim) return set_err(c, APT_E_INVALID, "apt_trainer_create: dims[0]=%d != store dim %d", m->dims[0], f->dim);
@@ -257,14 +269,14 @@ apt_status apt_trainer_create(apt_ctx* c, const apt_graph* g, const apt_fstore* 
   t->world = c->world;
   Arena& A = t->arena;
   const int K = t->K, C = t->world;
-  t->labels = A.alloc<int32_t>(g->n, false);
+  t->labels = labels ? A.alloc<int32_t>(g->n, false) : nullptr;
   t->step_cells = A.alloc<uint64_t>(2, true);   // step id of sample set 0 / 1
   t->step_dev = t->step_cells;
   t->hb_len = 1 + int64_t(C) * m->batch;
   t->hb_dev = A.alloc<int32_t>(2 * t->hb_len, true);
   CK(c, cudaMallocHost(reinterpret_cast<void**>(&t->hb_pinned), sizeof(int32_t) * 2 * t->hb_len));
   CK(c, cudaMallocHost(reinterpret_cast<void**>(&t->loss_pinned), sizeof(float) * APT_MAX_RANKS));
-  CK(c, cudaMemcpyAsync(t->labels, labels, sizeof(int32_t) * g->n, cudaMemcpyHostToDevice, c->stream));
+  if (labels) CK(c, cudaMemcpyAsync(t->labels, labels, sizeof(int32_t) * g->n, cudaMemcpyHostToDevice, c->stream));
   const int64_t n_words = ceil_div(g->n, 32);
   // upper bounds per hop.  SNP/DNP seeds follow the partition: up to C*B on one rank.
   const int64_t B0 = (s == APT_SNP || s == APT_DNP) ? int64_t(C) * m->batch : m->batch;
@@ -434,15 +446,15 @@ apt_status apt_trainer_set_params(apt_trainer* t, int layer, const float* W, con
   apt_ctx* c = t->ctx;
   for (auto& rs : t->R) {
     Layer& L = rs.L[layer - 1];
-    CK(c, cudaMemcpyAsync(L.W, W, sizeof(float) * L.d_out * L.d_in, cudaMemcpyHostToDevice, c->stream));
-    CK(c, cudaMemcpyAsync(L.b, b, sizeof(float) * L.d_out, cudaMemcpyHostToDevice, c->stream));
+    CK(c, cudaMemcpyAsync(L.W, W, sizeof(float) * L.d_out * L.d_in, cudaMemcpyDefault, c->stream));   // host or device
+    CK(c, cudaMemcpyAsync(L.b, b, sizeof(float) * L.d_out, cudaMemcpyDefault, c->stream));
     CK(c, launch_to_bf16(L.W, L.d_in, L.Wb, L.wb_pitch, L.d_in, nullptr, L.d_out, c->stream));
     c->launches++;
     if (layer == 1 && rs.x.W1s) {   // NFP: the rank's column slice of W^1 (column-owned)
       const int w = rs.x.w_cols;
       if (w > 0) {
         CK(c, cudaMemcpy2DAsync(rs.x.W1s, sizeof(float) * w, W + rs.x.col_lo, sizeof(float) * L.d_in, sizeof(float) * w,
-                                L.d_out, cudaMemcpyHostToDevice, c->stream));
+                                L.d_out, cudaMemcpyDefault, c->stream));
         CK(c, launch_to_bf16(rs.x.W1s, w, rs.x.Wb1s, rs.x.ws_pitch, w, nullptr, L.d_out, c->stream));
         c->launches++;
       }
@@ -917,13 +929,159 @@ apt_status compute_body(apt_trainer* t, int update) {
   return APT_OK;
 }
 
+// The layer-1 forward on the active sample set (every hosted rank): GAT, GDP, or the
+// strategy's Permute/Shuffle/Execute/Reshuffle; h^1 left in L[0].H / Hb.
+apt_status layer1_forward(apt_trainer* t) {
+  apt_status s = APT_OK;
+  if (t->gat_heads) {
+    s = gat_layer1_fwd(t, false);
+    return s == APT_OK ? hidden1_to_bf16(t) : s;
+  }
+  if (t->world == 1 || t->s == APT_GDP) {
+    bool first = true;
+    for (auto& rs : t->R) {
+      s = layer1_fwd_gdp(t, rs, first);
+      first = false;
+      if (s != APT_OK) return s;
+    }
+    return APT_OK;
+  }
+  s = layer1_fwd_strategy(t);
+  return s == APT_OK ? hidden1_to_bf16(t) : s;
+}
+
+// rows [0, n) of a bf16 or fp32 matrix -> fp32 rows of `dp` floats (layer API outputs)
+__global__ void rows_to_f32_kernel(float* __restrict__ dst, int64_t dp, const float* __restrict__ src,
+                                   const uint16_t* __restrict__ srcb, int64_t sp, int cols, int64_t n) {
+  const int64_t total = n * cols;
+  for (int64_t i = int64_t(blockIdx.x) * blockDim.x + threadIdx.x; i < total; i += int64_t(gridDim.x) * blockDim.x) {
+    const int64_t r = i / cols;
+    const int c = int(i - r * cols);
+    dst[r * dp + c] = srcb ? bf16_bits_to_float(srcb[r * sp + c]) : src[r * sp + c];
+  }
+}
+
 }  // namespace apt
+
+// A first-layer session of the standalone layer API (apt_layer_fwd / apt_layer_bwd,
+// SURVEY §8(b)): an internal layer-only trainer whose layer-1 hop holds the caller's
+// sampled blocks, and the row layout of h1 / dh1 (hosted ranks concatenated in order).
+struct apt_layer_saved {
+  apt_ctx* ctx = nullptr;
+  apt_trainer* t = nullptr;
+  int n_local = 0;
+  int64_t rows[APT_MAX_RANKS] = {};
+  int64_t off[APT_MAX_RANKS + 1] = {};
+  int d_in = 0, d_out = 0;
+};
 
 extern "C" {
 
-// ---- the first layer alone (the part APT parallelises): forward ...
-apt_status apt_layer_fwd(apt_trainer* t, int64_t step) {
-  if (!t || !t->perm) return set_err(t ? t->ctx : nullptr, APT_E_STATE, "apt_layer_fwd: call apt_trainer_set_epoch first");
+apt_status apt_layer_saved_destroy(apt_layer_saved* sv) {
+  if (!sv) return APT_OK;
+  apt_ctx* c = sv->ctx;
+  if (sv->t) apt_trainer_destroy(sv->t);
+  delete sv;
+  if (c) ctx_release(c);
+  return APT_OK;
+}
+
+apt_status apt_layer_fwd(apt_ctx* c, apt_strategy s, const apt_batch* batch, const apt_fstore* f, const float* W,
+                         const float* bias, int d_out, apt_dtype dtype, float* h1_out, apt_layer_saved** saved) {
+  if (!c || !batch || !f || !W || !bias || !h1_out || !saved || d_out < 1 || s < APT_GDP || s > APT_DNP)
+    return set_err(c, APT_E_INVALID, "apt_layer_fwd: bad arguments (batch %p store %p W %p bias %p h1 %p saved %p "
+                                     "d_out %d strategy %d)", (const void*)batch, (const void*)f, (const void*)W,
+                   (const void*)bias, (const void*)h1_out, (const void*)saved, d_out, int(s));
+  if (c->broken) return set_err(c, APT_E_STATE, "ctx is broken by an earlier CUDA error");
+  if (batch->ctx != c || f->ctx != c) return set_err(c, APT_E_INVALID, "apt_layer_fwd: batch / store of another ctx");
+  if ((dtype == APT_BF16) != (f->dtype == kBF16)) return set_err(c, APT_E_INVALID, "apt_layer_fwd: dtype != store dtype");
+  std::vector<const apt_batch*> per;
+  if (batch->members.empty()) per.push_back(batch);
+  else per = batch->members;
+  if (int(per.size()) != c->n_local)
+    return set_err(c, APT_E_INVALID, "apt_layer_fwd: %zu batches for %d hosted ranks (apt_batch_group)", per.size(),
+                   c->n_local);
+  if (batch->g != f->g) return set_err(c, APT_E_INVALID, "apt_layer_fwd: batch and store are on different graphs");
+  const int K = batch->K;
+  apt_model_desc m{};
+  m.n_layers = K;
+  m.dims[0] = f->dim;
+  m.dims[1] = d_out;
+  for (int l = 2; l <= K; ++l) m.dims[l] = 8;          // upper layers unused by a layer session
+  int64_t B = 1;
+  for (auto* b : per) B = std::max<int64_t>(B, b->n_dst[0]);
+  for (int l = 0; l < K; ++l) m.fanouts[l] = batch->fanouts[l];
+  m.batch = int(B);
+  m.dtype = dtype;
+  m.sample_seed = batch->rng_seed;                      // owners re-sample with the batch's key (R1)
+  auto* sv = new apt_layer_saved();
+  sv->ctx = c;
+  ctx_retain(c);
+  sv->n_local = c->n_local;
+  sv->d_in = f->dim;
+  sv->d_out = d_out;
+  apt_status st = trainer_create(c, batch->g, f, &m, s, nullptr, &sv->t, true);
+  if (st != APT_OK) { apt_layer_saved_destroy(sv); return st; }
+  apt_trainer* t = sv->t;
+  if ((st = apt_trainer_set_params(t, 1, W, bias)) != APT_OK) { apt_layer_saved_destroy(sv); return st; }
+  const uint64_t step = batch->step;
+  CK(c, cudaMemcpyAsync(t->step_cells, &step, sizeof(step), cudaMemcpyHostToDevice, c->stream));
+  // the caller's layer-1 blocks (hop K-1, sampler ELL form) into sample set 0 of every rank
+  for (int li = 0; li < c->n_local; ++li) {
+    const apt_batch* b = per[li];
+    Hop& hp = t->R[li].sset[0].hops[K - 1];
+    const int64_t n = b->n_dst[K - 1];
+    if (n > hp.max_dst) { apt_layer_saved_destroy(sv); return set_err(c, APT_E_INVALID, "apt_layer_fwd: block too large"); }
+    CK(c, cudaMemcpyAsync(const_cast<int32_t*>(hp.dst), b->dst[K - 1], sizeof(int32_t) * n, cudaMemcpyDeviceToDevice,
+                          c->stream));
+    const int32_t n32 = int32_t(n);
+    CK(c, cudaMemcpyAsync(const_cast<int32_t*>(hp.n_dst), &n32, 4, cudaMemcpyHostToDevice, c->stream));
+    CK(c, cudaMemcpyAsync(hp.cnt, b->cnt[K - 1], sizeof(int32_t) * n, cudaMemcpyDeviceToDevice, c->stream));
+    CK(c, cudaMemcpyAsync(hp.nbr, b->nbr[K - 1], sizeof(int32_t) * n * hp.k, cudaMemcpyDeviceToDevice, c->stream));
+    sv->rows[li] = n;
+    sv->off[li + 1] = sv->off[li] + n;
+  }
+  CK(c, cudaStreamSynchronize(c->stream));   // host staging of the counts above
+  t->primed = -1;
+  activate(t, 0);
+  if ((st = layer1_forward(t)) != APT_OK) { apt_layer_saved_destroy(sv); return st; }
+  for (int li = 0; li < c->n_local; ++li) {
+    const Layer& L = t->R[li].L[0];
+    if (!sv->rows[li]) continue;
+    rows_to_f32_kernel<<<unsigned(blocks_for(sv->rows[li] * d_out)), 256, 0, c->stream>>>(
+        h1_out + sv->off[li] * d_out, d_out, L.H, L.Hb, L.Hb ? L.hb_pitch : L.h_pitch, d_out, sv->rows[li]);
+    CK(c, cudaGetLastError());
+    c->launches++;
+  }
+  *saved = sv;
+  return APT_OK;
+}
+
+apt_status apt_layer_bwd(apt_ctx* c, apt_layer_saved* sv, const float* dh1, float* dW, float* dbias) {
+  if (!c || !sv || sv->ctx != c || !dh1 || !dW || !dbias) return set_err(c, APT_E_INVALID, "apt_layer_bwd: bad arguments");
+  apt_trainer* t = sv->t;
+  std::vector<const float*> ptr(sv->n_local);
+  for (int li = 0; li < sv->n_local; ++li) ptr[li] = dh1 + sv->off[li] * sv->d_out;
+  apt_status st = apt_trainer_layer_bwd(t, ptr.data(), sv->d_out);
+  if (st != APT_OK) return st;
+  const RankState& r0 = t->R[0];
+  const Layer& L = r0.L[0];
+  if (r0.x.dW1s) {   // NFP: W^1 is column-owned -- the hosted ranks' slices into their columns
+    for (auto& rs : t->R)
+      if (rs.x.w_cols > 0)
+        CK(c, cudaMemcpy2DAsync(dW + rs.x.col_lo, sizeof(float) * L.d_in, rs.x.dW1s, sizeof(float) * rs.x.w_cols,
+                                sizeof(float) * rs.x.w_cols, L.d_out, cudaMemcpyDeviceToDevice, c->stream));
+  } else {
+    CK(c, cudaMemcpyAsync(dW, L.dW, sizeof(float) * L.d_out * L.d_in, cudaMemcpyDeviceToDevice, c->stream));
+  }
+  CK(c, cudaMemcpyAsync(dbias, L.db, sizeof(float) * L.d_out, cudaMemcpyDeviceToDevice, c->stream));
+  return APT_OK;
+}
+
+// ---- the first layer alone (the part APT parallelises), bound to a trainer:
+// the trainer samples step `step` of its epoch, then runs the layer-1 forward ...
+apt_status apt_trainer_layer_fwd(apt_trainer* t, int64_t step) {
+  if (!t || !t->perm) return set_err(t ? t->ctx : nullptr, APT_E_STATE, "apt_trainer_layer_fwd: call apt_trainer_set_epoch first");
   apt_ctx* c = t->ctx;
   if (c->broken) return set_err(c, APT_E_STATE, "ctx is broken by an earlier CUDA error");
   t->primed = -1;   // sample set 0 is overwritten
@@ -937,37 +1095,21 @@ apt_status apt_layer_fwd(apt_trainer* t, int64_t step) {
     if (s != APT_OK) return s;
   }
   activate(t, 0);
-  apt_status s = APT_OK;
-  if (t->gat_heads) {
-    s = gat_layer1_fwd(t, false);
-    return s == APT_OK ? hidden1_to_bf16(t) : s;
-  } else if (t->world == 1 || t->s == APT_GDP) {
-    bool first = true;
-    for (auto& rs : t->R) {
-      s = layer1_fwd_gdp(t, rs, first);
-      first = false;
-      if (s != APT_OK) return s;
-    }
-  } else {
-    s = layer1_fwd_strategy(t);
-    if (s == APT_OK) s = hidden1_to_bf16(t);
-    if (s != APT_OK) return s;
-  }
-  return APT_OK;
+  return layer1_forward(t);
 }
 
 // ... and backward from dL/dh1 (one device pointer per hosted rank, rows of the
 // rank's layer-1 destinations, fp32, `pitch` floats apart): dW1/db1 of the
 // strategy, all-reduced over the ranks (NFP: column-owned slices).
-apt_status apt_layer_bwd(apt_trainer* t, const float* const* dh1, int64_t pitch) {
-  if (!t || !dh1 || pitch < t->m.dims[1]) return set_err(t ? t->ctx : nullptr, APT_E_INVALID, "apt_layer_bwd: bad arguments");
+apt_status apt_trainer_layer_bwd(apt_trainer* t, const float* const* dh1, int64_t pitch) {
+  if (!t || !dh1 || pitch < t->m.dims[1]) return set_err(t ? t->ctx : nullptr, APT_E_INVALID, "apt_trainer_layer_bwd: bad arguments");
   apt_ctx* c = t->ctx;
   const bool bf = t->m.dtype == APT_BF16;
   const int relu = t->K > 1 ? 1 : 0;
   for (size_t li = 0; li < t->R.size(); ++li) {
     RankState& rs = t->R[li];
     Layer& L = rs.L[0];
-    if (!dh1[li]) return set_err(c, APT_E_INVALID, "apt_layer_bwd: dh1[%zu] is null", li);
+    if (!dh1[li]) return set_err(c, APT_E_INVALID, "apt_trainer_layer_bwd: dh1[%zu] is null", li);
     // G = dh1 (copied over the rows the step produced; the count stays on the device)
     launch_pdl(copy_rows_kernel, dim3(blocks_for(L.max_rows * L.d_out)), dim3(256), 0, c->stream, L.G, L.h_pitch, dh1[li], pitch, L.d_out,
                                                                              L.n_rows);

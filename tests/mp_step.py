@@ -36,8 +36,8 @@ def main():
     torch.cuda.set_device(dev)
     fanout_sets = [tuple(int(x) for x in f.split(",")) for f in (sys.argv[3] if len(sys.argv) > 3 else "5,5").split(";")]
     g = aptgen.make_graph(aptgen.CONFIGS["tiny"])
-    train = aptgen.train_nodes(g, cfg)
-    labels = aptgen.labels(cfg, g.n)
+    train = aptgen.train_nodes(g, aptgen.CONFIGS["tiny"])
+    labels = aptgen.labels(aptgen.CONFIGS["tiny"], g.n)
     part = aptgen.partition(g.n, world)
     errors = []
     for fanouts, dtype, strategy in [(f, d, s) for f in fanout_sets for d in sys.argv[1].split(",")
@@ -58,7 +58,7 @@ def main():
                 pitch = (cfg.dim + 7) // 8 * 8 if dtype == "bf16" else (cfg.dim + 3) // 4 * 4
                 buf = torch.zeros(len(ids) * pitch * esz, dtype=torch.uint8, device="cuda")
                 torch.cuda.synchronize()            # torch's zero-fill runs on another stream than the library's
-                ctx.gather(fs, torch.as_tensor(ids).cuda(), len(ids), buf)
+                ctx.gather(fs, torch.as_tensor(ids.astype(np.int64)).cuda(), len(ids), buf)
                 torch.cuda.synchronize()
                 raw = buf.cpu().numpy()
                 if dtype == "bf16":

@@ -110,7 +110,7 @@ def test_feature_store_bit_exact(A, ctx, tiny, dtype, dim):
     pitch = ((dim + 7) // 8 * 8) if dtype == "bf16" else ((dim + 3) // 4 * 4)
     esz = 2 if dtype == "bf16" else 4
     out = torch.zeros(len(ids) * pitch * esz, dtype=torch.uint8, device="cuda")
-    ctx.gather(fs, torch.as_tensor(ids).cuda(), len(ids), out)
+    ctx.gather(fs, torch.as_tensor(ids.astype(np.int64)).cuda(), len(ids), out)
     torch.cuda.synchronize()
     raw = out.cpu().numpy()
     if dtype == "bf16":
@@ -205,7 +205,6 @@ def _trainer(A, ctx, cfg, g, train, dtype, strategy="GDP", lr=0.1):
     return tr, params, labels
 
 
-TOL = {"f32": dict(rtol=1e-5, atol=1e-6), "bf16": dict(rtol=2e-2, atol=2e-3)}
 
 
 def _check_grads(tr, ref, bd, dtype, K, rank=0, what=""):
@@ -515,53 +514,79 @@ def test_dryrun_counts_match_oracle_and_pick(A, tiny, C, frac, n_hot, heads):
 
 
 @pytest.mark.parametrize("dtype", ["f32", "bf16"])
-@pytest.mark.parametrize("strategy,C", [("GDP", 1), ("GDP", 2), ("NFP", 2), ("SNP", 4), ("DNP", 4)])
-def test_layer_fwd_bwd_api(A, tiny, strategy, C, dtype):
-    """apt_layer_fwd / apt_layer_bwd: the first layer alone under each strategy, with the
-    upstream gradient supplied by the caller (upper layers may be the user's own)."""
+@pytest.mark.parametrize("strategy,C,fanouts", [("GDP", 1, (5, 5)), ("GDP", 2, (5, 5)), ("NFP", 2, (5, 5)),
+                                                ("SNP", 4, (5, 5)), ("DNP", 4, (5, 5)), ("SNP", 2, (5, 5, 5)),
+                                                ("NFP", 4, (12, 16))])
+def test_layer_fwd_bwd_api(A, tiny, strategy, C, fanouts, dtype):
+    """The standalone layer API of SURVEY §8(b) (sampler and upper layers are the
+    user's black boxes): the caller samples each rank's batch with apt_sample, runs
+    apt_layer_fwd(strategy, batch, store, W, bias) and feeds its own dL/dh1 to apt_layer_bwd
+    -- h1 of every rank, dW1 and db1 (all-reduced; NFP assembled from the column-owned
+    slices) against the oracle."""
+    from oracle import strategy as S
     cfg, g, train = tiny
+    cfg = cfg.replace(fanouts=fanouts)
     ctx = A.Ctx(-1, C, 0) if C > 1 else A.Ctx(0, 1, 0)
     part = aptgen.partition(g.n, C)
     gr = ctx.graph_load(g.indptr, g.indices, part)
     dt = A.DTYPE[dtype]
     fs = ctx.fstore_create(gr, A.NFP if strategy == "NFP" else A.GDP, dt, cfg.dim, None, cfg.feat_seed)
-    dims = [cfg.dim] + [d for _, d in cfg.dims()]
-    labels = aptgen.labels(cfg, g.n)
-    tr = A.Trainer(ctx, gr, fs, dims, cfg.fanouts, cfg.batch, dt, 0.1, cfg.sample_seed, cfg.feat_seed,
-                   A.STRATEGY[strategy], labels)
-    params = aptgen.weights(cfg)
-    tr.set_params(params)
-    tr.set_epoch(train, 0)
-    tr.layer_fwd(0)
-    from oracle import strategy as S
+    step = min(3, oracle.steps_per_epoch(len(train), C, cfg.batch) - 1)   # the last global batch is short
     perm = oracle.epoch_perm(train, cfg.sample_seed, 0)
-    gb = oracle.global_batch(perm, 0, C, cfg.batch)
+    gb = oracle.global_batch(perm, step, C, cfg.batch)
     seeds = S.assign_seeds(strategy, gb, part, C, cfg.batch)
-    p64 = [(W.astype(np.float64), b.astype(np.float64)) for W, b in params]
+    batches = [ctx.sample(gr, dev_i64(sd), len(sd), cfg.fanouts, cfg.sample_seed, step) for sd in seeds]
+    batch = ctx.batch_group(batches) if C > 1 else batches[0]
+    W, b = aptgen.weights(cfg)[0]
+    d1 = W.shape[0]
+    K = len(cfg.fanouts)
+    rows = [len(oracle.sample_blocks(g, sd, cfg.fanouts, cfg.sample_seed, step)[K - 1].dst) for sd in seeds]
+    h1 = torch.zeros((sum(rows), d1), dtype=torch.float32, device="cuda")
+    saved = ctx.layer_fwd(A.STRATEGY[strategy], batch, fs, torch.as_tensor(W).cuda(), torch.as_tensor(b).cuda(), d1,
+                          dt, h1)
+    torch.cuda.synchronize()
+    H = h1.cpu().numpy()
+    Wr = oracle.bf16_round(W.astype(np.float64)) if dtype == "bf16" else W.astype(np.float64)
     rng = np.random.default_rng(C)
-    dW = 0.0
-    db = 0.0
-    dh_dev = []
-    tol = TOL[dtype]
+    dh = rng.normal(size=(sum(rows), d1)).astype(np.float32)
+    dW = db = 0.0
+    bW = bb = 0.0
+    off = 0
     for r in range(C):
-        blocks = oracle.sample_blocks(g, seeds[r], cfg.fanouts, cfg.sample_seed, 0)
-        cache = model.forward(blocks, cfg.feat_seed, cfg.dim, p64, dtype,
-                              snp=(part, C) if strategy == "SNP" else None)
-        assert np.allclose(tr.read("H", 1, rank=r), cache["h"][0], **tol)
-        n1, d1 = cache["h"][0].shape
-        dh = rng.normal(size=(n1, d1)).astype(np.float32)
-        gpre = dh.astype(np.float64) * (cache["pre"][0] > 0)
+        blk = oracle.sample_blocks(g, seeds[r], cfg.fanouts, cfg.sample_seed, step)[K - 1]
+        x = oracle.features(cfg.feat_seed, blk.src, cfg.dim)
+        Zs = model.snp_partials(blk, x, part, C) if strategy == "SNP" else [oracle.aggregate(blk.indptr, blk.indices, x)]
         if dtype == "bf16":
-            gpre = oracle.bf16_round(gpre)                     # reading R4: g rounded for tcgen05
-        Zs = cache["Zparts"] if cache["Zparts"] is not None else [cache["Z"][0]]
-        dW = dW + sum(gpre.T @ Z for Z in Zs)
+            Zs = [oracle.bf16_round(z) for z in Zs]     # the bf16 rounding point of Z (SNP: of each partial, R5)
+        pre = sum(z @ Wr.T for z in Zs) + b
+        h = np.maximum(pre, 0.0)
+        if dtype == "bf16":
+            h = oracle.bf16_round(h)                      # the stored activation (R11)
+        got = H[off:off + rows[r]]
+        # T1 for the pre-activation (same operands on both sides), plus one bf16 flip of h
+        Zabs = sum(np.abs(z) for z in Zs)
+        sig = np.sqrt(Zs[0].shape[1]) * 2.0 ** -24 * (Zabs @ np.abs(Wr).T + np.abs(b))
+        bound = 6 * sig + (2.0 ** -8 * np.abs(h) if dtype == "bf16" else 0.0)
+        assert_close(got, h, dtype, f"h1 rank {r}", bound)
+        # T3: the ReLU bit the GPU took where the pre-activation is within the band of zero
+        on = got > 0
+        amb = np.abs(pre) <= 6 * sig + (2.0 ** -8 * np.abs(pre) if dtype == "bf16" else 0.0)
+        assert not ((on != (pre > 0)) & ~amb).any(), f"rank {r}: mask differs outside the ambiguity band"
+        gpre = dh[off:off + rows[r]].astype(np.float64) * on
+        if dtype == "bf16":
+            gpre = oracle.bf16_round(gpre)                # reading R4: g rounded for tcgen05
+        dW = dW + sum(gpre.T @ z for z in Zs)
         db = db + gpre.sum(0)
-        dh_dev.append(torch.as_tensor(dh).cuda())
-    tr.layer_bwd(dh_dev, d1)
-    atol = tol["atol"] * 100                                   # unit-scale g: sums of ~1e4 products
-    for r in (0, C - 1):
-        assert np.allclose(tr.read("dW", 1, rank=r), dW, rtol=tol["rtol"], atol=atol)
-        assert np.allclose(tr.read("db", 1, rank=r)[0], db, rtol=tol["rtol"], atol=atol)
+        bW = bW + t1(np.abs(gpre).T, Zabs, rows[r])
+        bb = bb + t1(np.abs(gpre).T, np.ones(rows[r]), rows[r])
+        off += rows[r]
+    dW_dev = torch.zeros((d1, cfg.dim), dtype=torch.float32, device="cuda")
+    db_dev = torch.zeros(d1, dtype=torch.float32, device="cuda")
+    ctx.layer_bwd(saved, torch.as_tensor(dh).cuda(), dW_dev, db_dev)
+    torch.cuda.synchronize()
+    assert_close(dW_dev.cpu().numpy(), dW, "f32", "dW1", bW)     # emulated operands: fp32 bar + T1
+    assert_close(db_dev.cpu().numpy(), db, "f32", "db1", bb)
+    saved.close()
 
 
 @pytest.mark.slow
@@ -628,7 +653,7 @@ def test_tiered_store_rows_and_step(A, tiny, dtype, frac, n_hot):
             esz = 2 if dtype == "bf16" else 4
             out = torch.zeros(g.n * pitch * esz, dtype=torch.uint8, device="cuda")
             torch.cuda.synchronize()
-            ctx.gather(fs, torch.as_tensor(ids).cuda(), g.n, out)
+            ctx.gather(fs, torch.as_tensor(ids.astype(np.int64)).cuda(), g.n, out)
             torch.cuda.synchronize()
             raw = out.cpu().numpy()
             got = ((raw.view(np.uint16).astype(np.uint32) << 16).view(np.float32) if dtype == "bf16"
