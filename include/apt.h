@@ -243,9 +243,12 @@ apt_status apt_aggregate(apt_ctx* ctx, const apt_block_view* blk, const void* x_
 /* Backward of the mean: dx[indices[e]] += dz[v]/deg(v) (accumulates).       */
 apt_status apt_aggregate_bwd(apt_ctx* ctx, const apt_block_view* blk, const float* dz, int dim, int64_t dz_pitch,
                              float* dx_src, int64_t dx_pitch);
-/* Projection Y = Z W^T + b (+ReLU) (Eq. 1).  dtype APT_BF16: Z is
- * bf16 [M x z_pitch], tcgen05 path (N, K <= 256); APT_F32: Z fp32, CUDA-core
- * fp32.  W host-independent device fp32 [N x K]; Y device fp32 [M x y_pitch]. */
+/* Projection Y = Z W^T + b (+ReLU) (Eq. 1) on the tensor cores.  dtype
+ * APT_BF16: Z is bf16 [M x z_pitch], W rounded to bf16, kind::f16 with fp32
+ * accumulation (N, K <= 256: the row-tile kernel with W resident; wider: the general
+ * kernel, N tiled and K streamed); APT_F32: Z fp32, 3xTF32 on kind::tf32 (each product
+ * carried to ~2^-21, reading P1), falling back to exact fp32 CUDA cores when a pitch is
+ * not a 16-byte multiple.  W device fp32 [N x K]; Y device fp32 [M x y_pitch].  Syncs. */
 apt_status apt_project(apt_ctx* ctx, const void* Z, int64_t z_pitch, apt_dtype dtype, const float* W,
                        const float* bias, int64_t M, int N, int K, int relu, float* Y, int64_t y_pitch);
 
@@ -253,8 +256,9 @@ apt_status apt_project(apt_ctx* ctx, const void* Z, int64_t z_pitch, apt_dtype d
  * G[r][o] Z[r][i] and db[o] += sum_r G[r][o] over rows r < rows (accumulates
  * into dW [d_out x d_in] and db [d_out], device fp32; db may be NULL).  G device
  * fp32 [rows x g_pitch]; Z device [rows x z_pitch] of dtype.  APT_BF16: G is
- * rounded to bf16 and the contraction runs on tcgen05 (d_out <= 256, d_in < 320);
- * APT_F32: exact fp32 CUDA cores.  Syncs.                                    */
+ * rounded to bf16 and the contraction runs on tcgen05 kind::f16 (any d_out, d_in);
+ * APT_F32: 3xTF32 on kind::tf32 (CUDA cores if a pitch is not a 16-byte multiple).
+ * Syncs.                                                                    */
 apt_status apt_weight_grad(apt_ctx* ctx, const float* G, int64_t g_pitch, const void* Z, int64_t z_pitch,
                            apt_dtype dtype, int64_t rows, int d_out, int d_in, float* dW, float* db);
 
@@ -388,6 +392,12 @@ int64_t apt_selftest_div(void);
  * the number of positions that differ from a host std::stable_sort, < 0 on failure.
  * Uses the current device; syncs.                                                    */
 int64_t apt_selftest_sort(int64_t n, uint64_t seed, int key_bits);
+
+/* Self-test of the general tensor-core contraction (gemm_tc_gen.cu): C = A B + bias for
+ * fp32 (3xTF32, f32 = 1) or bf16 operands, A / B K-major or M/N-major, M x N x K, split-K
+ * accumulating when `accumulate`; returns max |C - ref| / (sum_k |A||B| + |bias|) against
+ * an fp64 host product, < 0 on failure.  Uses the current device; syncs.             */
+double apt_selftest_gemm(int f32, int a_mn, int b_mn, int64_t M, int N, int64_t K, int accumulate);
 
 #ifdef __cplusplus
 }

@@ -137,6 +137,8 @@ def lib():
         L.apt_selftest_div.restype = C.c_int64
         L.apt_selftest_sort.argtypes = [i64, u64, i32]
         L.apt_selftest_sort.restype = C.c_int64
+        L.apt_selftest_gemm.argtypes = [i32, i32, i32, i64, i32, i64, i32]
+        L.apt_selftest_gemm.restype = C.c_double
         L.apt_trainer_steps_per_epoch.argtypes = [vp]
         L.apt_trainer_steps_per_epoch.restype = C.c_int64
         _lib = L

@@ -115,7 +115,10 @@ __global__ void __launch_bounds__(256, (VPL == 1 ? 6 : 4)) agg_kernel(AggArgs a,
       }
     }
     if (!valid) continue;
-    if (a.z_ones && l == 0) a.z_bf16[i * a.z_bf16_pitch + a.dim] = 0x3F80;   // bf16 1.0: bias-gradient column
+    if (a.z_ones && l == 0) {   // 1.0 in column dim: the bias-gradient column of the weight-gradient GEMM
+      if (a.z_bf16) a.z_bf16[i * a.z_bf16_pitch + a.dim] = 0x3F80;
+      else if (a.z_f32) a.z_f32[i * a.z_f32_pitch + a.dim] = 1.f;
+    }
     const float fdeg = float(a.deg_override ? a.deg_override[i] : cnt);
     const float rdeg = fdeg > 0.f ? __frcp_rn(fdeg) : 0.f;   // one reciprocal per row (O5 division below)
 #pragma unroll
@@ -235,7 +238,10 @@ __global__ void __launch_bounds__(256, MINB) agg_l1_pf_kernel(AggArgs a, EllFsto
       for (int q = 0; q < NB; ++q) accumulate_vec<EPV>(acc, v[q]);
     }
     if (!valid || l >= V) continue;
-    if (a.z_ones && l == 0) a.z_bf16[i * a.z_bf16_pitch + a.dim] = 0x3F80;
+    if (a.z_ones && l == 0) {
+      if (a.z_bf16) a.z_bf16[i * a.z_bf16_pitch + a.dim] = 0x3F80;
+      else if (a.z_f32) a.z_f32[i * a.z_f32_pitch + a.dim] = 1.f;
+    }
     const float fdeg = float(a.deg_override ? a.deg_override[i] : cnt);
     const float rdeg = fdeg > 0.f ? __frcp_rn(fdeg) : 0.f;
     float z[EPV];

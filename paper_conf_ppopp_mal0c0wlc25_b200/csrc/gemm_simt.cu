@@ -1,7 +1,9 @@
-// gemm_simt.cu -- exact-fp32 CUDA-core GEMM used where the tensor-core path
-// does not apply: the fp32 parity mode of the projection (S8, rtol 1e-5 needs
-// fp32 products, TF32 alone misses it) and the weight-gradient / input-gradient
-// contractions of the backward pass (S10/S11: dW = g^T Z, dZ = g W).
+// gemm_simt.cu -- the generic contraction entry (launch_simt_gemm) and its CUDA-core
+// fallback.  Operands that TMA can address go to the tensor cores (gemm_tc_gen.cu:
+// 3xTF32 for the fp32 parity mode, kind::f16 for bf16 past the row-tile kernel's
+// limits); what remains (mixed operand types, strides that are not 16-byte multiples)
+// runs here in exact fp32 FMA: the projection (S8) and the backward contractions
+// (S10/S11: dW = g^T Z, dZ = g W).
 //
 // C[m][n] (+)= sum_k A(m,k) B(k,n) (+bias[n]) (relu) with arbitrary element
 // strides, 64x64 tiles, 16-deep k slabs in shared memory, 4x4 outputs per
@@ -9,6 +11,7 @@
 #include "common.cuh"
 #include "kernels.h"
 #include <algorithm>
+#include <cstdlib>
 
 namespace apt {
 
@@ -96,6 +99,10 @@ __global__ void __launch_bounds__(256) simt_gemm_kernel(SimtGemmArgs a) {
 
 cudaError_t launch_simt_gemm(const SimtGemmArgs& a, cudaStream_t st) {
   if (a.relu && a.accumulate) return cudaErrorInvalidValue;
+  // tensor cores whenever the operands are TMA-addressable (gemm_tc_gen.cu: 3xTF32 for
+  // fp32, kind::f16 for bf16); APT_SIMT_GEMM=1 keeps these CUDA cores (A/B)
+  static const int simt_only = [] { const char* v = std::getenv("APT_SIMT_GEMM"); return v ? atoi(v) : 0; }();
+  if (!simt_only && tc_gen_supported(a)) return launch_tc_gen_gemm(a, -1, nullptr, st);
   const int64_t kc = a.k_chunk > 0 ? a.k_chunk : a.K;
   dim3 grid(unsigned(std::max<int64_t>(1, ceil_div(a.M, BM))), unsigned(ceil_div(a.N, BN)),
             unsigned(std::max<int64_t>(1, ceil_div(a.K, kc))));

@@ -188,6 +188,11 @@ struct SimtGemmArgs {
   float* const* out_base; const int32_t* out_rank; const int32_t* out_row;
 };
 cudaError_t launch_simt_gemm(const SimtGemmArgs& a, cudaStream_t st);
+// gemm_tc_gen.cu: the same contract on tcgen05 (fp32: 3xTF32 on kind::tf32; bf16:
+// kind::f16), any M, N, K; ones_col >= 0 routes output column ones_col to ones_out[m]
+// (the bias gradient from an all-ones column of B).  tc_gen_supported: TMA-addressable.
+int tc_gen_supported(const SimtGemmArgs& a);
+cudaError_t launch_tc_gen_gemm(const SimtGemmArgs& a, int ones_col, float* ones_out, cudaStream_t st);
 
 // ---------------------------------------------------------------- gemm_tc.cu
 // tcgen05 projection: Y[m][n] = sum_k Z[m][k] W[n][k] + bias[n] (relu), bf16 in,

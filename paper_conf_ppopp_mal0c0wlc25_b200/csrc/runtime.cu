@@ -641,15 +641,22 @@ apt_status apt_project(apt_ctx* c, const void* Z, int64_t z_pitch, apt_dtype dt,
   int32_t mh = int32_t(M);
   CK(c, cudaMemcpyAsync(md, &mh, 4, cudaMemcpyHostToDevice, c->stream));
   if (dt == APT_BF16) {
-    if (!tc_gemm_supported(N, K)) return set_err(c, APT_E_UNSUPPORTED, "apt_project: tcgen05 path needs N,K <= 256");
     const int64_t wp = round_up(K, 8);
     uint16_t* Wb = nullptr;
     CK(c, cudaMallocAsync(reinterpret_cast<void**>(&Wb), sizeof(uint16_t) * N * wp, c->stream));
     CK(c, cudaMemsetAsync(Wb, 0, sizeof(uint16_t) * N * wp, c->stream));
     CK(c, launch_to_bf16(W, K, Wb, wp, K, nullptr, N, c->stream));
-    TcGemmArgs a{static_cast<const uint16_t*>(Z), z_pitch, Wb, wp, M, md, N, K, bias, relu, Y, y_pitch,
-                 nullptr, nullptr, nullptr, 0};
-    CK(c, launch_tc_gemm(a, c->stream));
+    if (tc_gemm_supported(N, K)) {   // the row-tile kernel (resident W)
+      TcGemmArgs a{static_cast<const uint16_t*>(Z), z_pitch, Wb, wp, M, md, N, K, bias, relu, Y, y_pitch,
+                   nullptr, nullptr, nullptr, 0};
+      CK(c, launch_tc_gemm(a, c->stream));
+    } else {                         // wider: the general tcgen05 kernel (N tiled, K streamed)
+      SimtGemmArgs a{};
+      a.A = Z; a.a_t = kBF16; a.sam = z_pitch; a.sak = 1;
+      a.B = Wb; a.b_t = kBF16; a.sbk = 1; a.sbn = wp;
+      a.C = Y; a.ldc = y_pitch; a.bias = bias; a.M_dev = md; a.M = M; a.N = N; a.K = K; a.relu = relu;
+      CK(c, launch_simt_gemm(a, c->stream));
+    }
     CK(c, cudaFreeAsync(Wb, c->stream));
     c->launches += 2;
   } else {
@@ -673,7 +680,6 @@ apt_status apt_weight_grad(apt_ctx* c, const float* G, int64_t g_pitch, const vo
   int32_t rh = int32_t(rows);
   CK(c, cudaMemcpyAsync(rd, &rh, 4, cudaMemcpyHostToDevice, c->stream));
   if (dt == APT_BF16) {
-    if (!tc_wgrad_supported(d_out, d_in)) return set_err(c, APT_E_UNSUPPORTED, "apt_weight_grad: tcgen05 path needs d_out <= 256, d_in < 320");
     // G -> bf16 (tail of the last 64-row block zeroed); Z -> a copy with the all-ones column d_in
     const int64_t gbp = round_up(d_out, 8), zbp = round_up(d_in + 1, 8);
     const int64_t rr = std::max<int64_t>(rows, 1);
@@ -684,8 +690,16 @@ apt_status apt_weight_grad(apt_ctx* c, const float* G, int64_t g_pitch, const vo
     CK(c, launch_bf16_pad_ones(static_cast<const uint16_t*>(Z), z_pitch, Zb, zbp, d_in, rd, rr, c->stream));
     float* dbw = db;
     if (!dbw) CK(c, cudaMallocAsync(reinterpret_cast<void**>(&dbw), sizeof(float) * d_out, c->stream));
-    TcWgradArgs w{Gb, gbp, Zb, zbp, rd, rr, d_out, d_in, dW, dbw};
-    CK(c, launch_tc_wgrad(w, c->stream));
+    if (tc_wgrad_supported(d_out, d_in)) {
+      TcWgradArgs w{Gb, gbp, Zb, zbp, rd, rr, d_out, d_in, dW, dbw};
+      CK(c, launch_tc_wgrad(w, c->stream));
+    } else {   // wider: the general tcgen05 kernel, db from Z's all-ones column
+      SimtGemmArgs a{};
+      a.A = Gb; a.a_t = kBF16; a.sam = 1; a.sak = gbp;
+      a.B = Zb; a.b_t = kBF16; a.sbk = zbp; a.sbn = 1;
+      a.C = dW; a.ldc = d_in; a.M = d_out; a.N = d_in + 1; a.K = rr; a.K_dev = rd; a.accumulate = 1;
+      CK(c, launch_tc_gen_gemm(a, d_in, dbw, c->stream));
+    }
     if (!db) CK(c, cudaFreeAsync(dbw, c->stream));
     CK(c, cudaFreeAsync(Gb, c->stream));
     CK(c, cudaFreeAsync(Zb, c->stream));
@@ -696,7 +710,7 @@ apt_status apt_weight_grad(apt_ctx* c, const float* G, int64_t g_pitch, const vo
     a.B = Z; a.b_t = kF32; a.sbk = z_pitch; a.sbn = 1;
     a.C = dW; a.ldc = d_in; a.M = d_out; a.N = d_in; a.K = std::max<int64_t>(rows, 1); a.K_dev = rd;
     a.accumulate = 1; a.k_chunk = 2048;
-    CK(c, launch_simt_gemm(a, c->stream));
+    CK(c, launch_simt_gemm(a, c->stream));   // 3xTF32 tensor cores when TMA-addressable
     if (db) CK(c, launch_colsum(G, g_pitch, d_out, rd, std::max<int64_t>(rows, 1), db, c->stream));
     c->launches += db ? 2 : 1;
   }

@@ -197,7 +197,20 @@ apt_status weight_grad(apt_trainer* t, const Layer& L, const float* G, int64_t g
     c->launches++;
     return APT_OK;
   }
-  // CUDA cores (fp32 mode, or dims past the tcgen05 kernel): in bf16 mode the hidden
+  // fp32 mode: 3xTF32 tensor cores (gemm_tc_gen.cu), db from Z's all-ones column d_in
+  if (!z_bf16 && z_pitch > d_in) {
+    SimtGemmArgs a{};
+    a.A = G; a.a_t = kF32; a.sam = 1; a.sak = g_pitch;
+    a.B = Z; a.b_t = kF32; a.sbk = z_pitch; a.sbn = 1;
+    a.C = dW; a.ldc = dW_ld; a.M = L.d_out; a.N = d_in + (db ? 1 : 0); a.K = max_rows; a.K_dev = n_rows;
+    a.accumulate = 1;
+    if (tc_gen_supported(a)) {
+      CK(c, launch_tc_gen_gemm(a, db ? d_in : -1, db, st));
+      c->launches++;
+      return APT_OK;
+    }
+  }
+  // CUDA cores (dims or strides past the tensor-core kernels): in bf16 mode the hidden
   // layers' gradient exists only as its bf16 copy Gb (the pull kernel writes no fp32 G)
   SimtGemmArgs a{};
   const bool gb = z_bf16 && L.Gb;
@@ -332,7 +345,7 @@ apt_status apt::trainer_create(apt_ctx* c, const apt_graph* g, const apt_fstore*
       const Hop& hp = rs.hops[K - l];
       L.d_in = m->dims[l - 1];
       L.d_out = m->dims[l];
-      L.zf_pitch = round_up(L.d_in, 4);
+      L.zf_pitch = round_up(L.d_in + 1, 4);    // + the all-ones bias-gradient column (fp32 mode)
       L.zb_pitch = round_up(L.d_in + 1, 8);   // + the all-ones bias-gradient column
       L.gb_pitch = round_up(L.d_out, 8);
       L.h_pitch = round_up(L.d_out, 4);
@@ -640,7 +653,7 @@ apt_status layer1_fwd_gdp(apt_trainer* t, RankState& rs, bool time_it) {
   a.cnt = hp.cnt; a.nbr = hp.nbr; a.k = hp.k;
   a.n_dst = hp.n_dst; a.max_dst = hp.max_dst; a.dim = L.d_in;
   if (t->m.dtype == APT_BF16) { a.z_bf16 = L.Zb; a.z_bf16_pitch = L.zb_pitch; a.z_ones = 1; }
-  else { a.z_f32 = L.Zf; a.z_f32_pitch = L.zf_pitch; }
+  else { a.z_f32 = L.Zf; a.z_f32_pitch = L.zf_pitch; a.z_ones = 1; }
   if (time_it) CK(c, record_ev(t, 6));
   CK(c, launch_agg_fstore(a, fv, c->stream));
   c->launches++;
@@ -669,7 +682,7 @@ apt_status upper_fwd_loss(apt_trainer* t, RankState& rs) {
     a.n_dst = hp.n_dst; a.max_dst = hp.max_dst; a.dim = L.d_in;
     if (t->m.dtype == APT_BF16) { a.z_bf16 = L.Zb; a.z_bf16_pitch = L.zb_pitch; a.z_ones = 1; }
     // fp32 Z is kept in both modes for the upper layers' weight gradient in fp32 mode
-    if (t->m.dtype != APT_BF16) { a.z_f32 = L.Zf; a.z_f32_pitch = L.zf_pitch; }
+    if (t->m.dtype != APT_BF16) { a.z_f32 = L.Zf; a.z_f32_pitch = L.zf_pitch; a.z_ones = 1; }
     CK(c, launch_agg_csr(a, c->stream));
     c->launches++;
     apt_status s = project(t, L, L.Zb, L.Zf, L.zb_pitch, L.zf_pitch, L.n_rows, L.max_rows, L.d_in, L.W, L.Wb, L.b,

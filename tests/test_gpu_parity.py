@@ -157,7 +157,8 @@ def test_aggregate_bit_exact_and_bwd(A, ctx, tiny):
 
 # ------------------------------------------------------------------ S8 projection
 @pytest.mark.parametrize("M,N,K", [(1, 16, 64), (127, 32, 64), (128, 47, 100), (1000, 256, 100),
-                                   (5000, 256, 256), (333, 48, 256), (4099, 8, 16)])
+                                   (5000, 256, 256), (333, 48, 256), (4099, 8, 16), (1000, 512, 384),
+                                   (300, 1040, 64)])
 def test_project_tcgen05_bf16(A, ctx, M, N, K):
     rng = np.random.default_rng(M + N + K)
     kp = (K + 7) // 8 * 8
@@ -177,8 +178,24 @@ def test_project_tcgen05_bf16(A, ctx, M, N, K):
     assert_close(got, ref, "f32", "Y", t1(np.abs(Z), np.abs(Wr).T, K) + LAMBDA_U * np.abs(bias))
 
 
-@pytest.mark.parametrize("M,N,K", [(1, 5, 3), (130, 47, 100), (2000, 256, 100)])
+@pytest.mark.parametrize("f32", [1, 0])
+@pytest.mark.parametrize("a_mn,b_mn", [(0, 0), (0, 1), (1, 0), (1, 1)])
+@pytest.mark.parametrize("M,N,K,acc", [(64, 32, 32, 0), (64, 32, 64, 1), (300, 70, 100, 0), (130, 300, 1000, 1),
+                                       (1, 8, 8, 0), (4099, 264, 72, 1)])
+def test_general_tensor_core_gemm(A, ctx, f32, a_mn, b_mn, M, N, K, acc):
+    """The general tcgen05 contraction (gemm_tc_gen.cu) in every operand layout: fp32 as
+    3xTF32 (each product carried to ~2^-21 of its magnitude: reading P1), bf16 exact
+    operands with fp32 accumulation; N tiled past 256, K streamed, split-K accumulating.
+    Error relative to sum_k |A||B| + |b| (the T1 scale of the sum)."""
+    err = A.lib().apt_selftest_gemm(f32, a_mn, b_mn, M, N, K, acc)
+    assert 0 <= err < (2e-6 if f32 else 5e-7), err
+
+
+@pytest.mark.parametrize("M,N,K", [(1, 5, 3), (1, 8, 4), (130, 47, 100), (2000, 256, 100), (49537, 256, 100),
+                                   (3001, 300, 520), (700, 1024, 256), (257, 40, 1030)])
 def test_project_fp32(A, ctx, M, N, K):
+    """fp32 mode on the tensor cores (3xTF32, kind::tf32; K = 3 / N = 5 fall back to CUDA
+    cores: pitches not 16-byte multiples), N tiled past 256 and K streamed past 256."""
     rng = np.random.default_rng(7)
     Z = rng.normal(size=(M, K)).astype(np.float32)
     W = rng.normal(size=(N, K)).astype(np.float32)
@@ -364,7 +381,8 @@ def test_step_host_e2e_matches_device_step(A, ctx, tiny, use_graph):
 
 # ------------------------------------------------------------------ S11 weight gradient
 @pytest.mark.parametrize("rows,d_out,d_in", [(1, 16, 64), (63, 47, 256), (64, 256, 100), (1000, 256, 256),
-                                             (49537, 256, 100), (5000, 32, 64), (300, 200, 8)])
+                                             (49537, 256, 100), (5000, 32, 64), (300, 200, 8), (2000, 1040, 256),
+                                             (777, 300, 1024)])
 @pytest.mark.parametrize("dtype", ["bf16", "f32"])
 def test_weight_grad(A, ctx, rows, d_out, d_in, dtype):
     """dW = G^T Z, db = colsum(G): tcgen05 (MN-major operands, all-ones bias column) in bf16
