@@ -58,7 +58,7 @@ def parse():
     ap.add_argument("--cpu-steps", type=int, default=3, help="oracle steps for cpu_baseline")
     ap.add_argument("--e2e-steps", type=int, default=10)
     ap.add_argument("--no-planner", action="store_true")
-    ap.add_argument("--dryrun-steps", type=int, default=8)
+    ap.add_argument("--dryrun-steps", type=int, default=0, help="dry-run steps (0: one full epoch, P:142)")
     ap.add_argument("--emulate-max-c", type=int, default=4,
                     help="also time every strategy with C ranks emulated on the GPU, for C up to this")
     ap.add_argument("--verbose", action="store_true")
@@ -415,8 +415,20 @@ def run_apt(args, cfg):
         out["planner"] = planner_report(A, g, cfg, train, labels, args, stream, ms_local)
         # the workload's access skew next to the paper's Table 3 (reading R12)
         n_acc = spe   # one whole epoch (the paper ranks nodes over training; a prefix undercounts the tail)
+        counts0 = tr.access_counts(n_acc)
+        # "the top-1% nodes of two epochs overlap by 94.77%": the same statistic here
+        tr.set_epoch(train, 1)
+        counts1 = tr.access_counts(n_acc)
+        tr.set_epoch(train, 0)
+        k1 = max(1, g.n // 100)
+        top0 = np.argsort(-counts0.astype(np.int64), kind="stable")[:k1]
+        top1 = np.argsort(-counts1.astype(np.int64), kind="stable")[:k1]
+        out["planner"]["epoch_top1pct_overlap"] = len(np.intersect1d(top0, top1)) / k1
+        out["planner"]["dryrun_vs_epoch"] = {
+            f"C{C}": {"dryrun_wall_s": out["planner"][f"C{C}"]["dryrun_wall_s"], "epoch_s_measured_C1": epoch_measured,
+                      "note": "paper P:279: 25 s dry-run vs 449 s of GDP training (T4s)"} for C in (2, 4, 8)}
         out["access_skew"] = {"steps": n_acc, "buckets": ["<1%", "1-5%", "5-10%", "10-20%", "20-50%", "50-100%"],
-                              "table": skew_table(tr.access_counts(n_acc)),
+                              "table": skew_table(counts0),
                               "paper_table3": {"PS": [0.501, 0.348, 0.088, 0.047, 0.017, 0.0],
                                                "FS": [0.177, 0.294, 0.191, 0.188, 0.135, 0.016]}}
     if rank == 0 and world == 1 and not args.no_cpu_baseline:
@@ -448,11 +460,17 @@ def planner_report(A, g, cfg, train, labels, args, stream, gdp_ms):
         fs = ctx.fstore_create(gr, A.GDP, dt, cfg.dim, None, cfg.feat_seed)
         tr = make_trainer(A, ctx, gr, fs, cfg, dt, A.GDP, labels)
         tr.set_epoch(train, 0)
-        st = tr.dryrun(args.dryrun_steps)
+        st = tr.dryrun(args.dryrun_steps or tr.steps_per_epoch())
         bw = ctx.profile_links()
         pick, pred = A.select_strategy(st, bw)
         steps = max(1, st.steps)
-        rep[f"C{C}"] = {"dryrun_steps": st.steps, "pred_ms_per_step": {s: 1e3 * p / steps for s, p in zip(STRATS, pred)},
+        rep[f"C{C}"] = {"dryrun_steps": st.steps, "dryrun_wall_s": st.t_dryrun_s,
+                        "steps_per_epoch": tr.steps_per_epoch(),
+                        "t_build_ms_per_step": {s: 1e3 * max(st.t_build_s[i][r] for r in range(C)) / steps
+                                                for i, s in enumerate(STRATS)},
+                        "t_resample_ms_per_step": {s: 1e3 * max(st.t_resample_s[i][r] for r in range(C)) / steps
+                                                   for i, s in enumerate(STRATS)},
+                        "pred_ms_per_step": {s: 1e3 * p / steps for s, p in zip(STRATS, pred)},
                         "partition": PARTITION, "edge_cut_frac": _partition(A, g, C)[1] / max(1, g.nnz),
                         "pick": STRATS[pick],
                         "n_vs_per_step": sum(st.n_vs[r] for r in range(C)) / steps,

@@ -126,6 +126,11 @@ typedef struct {
   int gat_heads;
   int64_t attn_bytes[4][APT_MAX_RANKS];
   int64_t attn_feat_bytes[4][APT_MAX_RANKS];
+  /* Reading R1: owners re-sample the rows requesters route to them with the same Philox
+   * key; that time (measured layer-1 sampling cost per row x rows re-sampled) is
+   * included in t_build_s and reported here.                                        */
+  double t_resample_s[4][APT_MAX_RANKS];
+  double t_dryrun_s;                         /* host wall time of the whole dry run */
 } apt_plan_stats;
 
 /* Operator slots of the bandwidth profile ("trials").          */
@@ -191,9 +196,27 @@ typedef struct {
                                rest form the host tier (pinned, mapped; read over PCIe / C2C)          */
   int64_t cache_rows;       /* excess cache: rows replicated into every GPU's spare HBM */
   const int64_t* hot_ids;   /* host, >= cache_rows candidate ids, hottest first (apt_hot_rows)        */
+  /* P:163 "Cache configuration" (cache_rule = APT_CACHE_P163; hbm_frac / cache_rows unused):
+   * every GPU's HBM holds only its cache set -- the cache_budget_rows most popular nodes
+   * under the store layout's strategy rule (apt_cache_sets, from the dry-run counts) --
+   * and the host tier holds every row; a row is read from the own cache, else from a
+   * peer GPU's cache over NVLink, else from the host (the feature map of P:241-247).   */
+  int cache_rule;
+  const int32_t* counts;    /* host int32[n]: access frequencies (apt_access_counts)                   */
+  int64_t cache_budget_rows;
 } apt_fstore_opts;
+enum { APT_CACHE_NONE = 0, APT_CACHE_P163 = 1 };
+/* The per-GPU cache sets of P:163: GDP / NFP the most popular nodes of the graph, SNP
+ * of the GPU's partition, DNP of its partition and their 1-hop neighbours; popularity =
+ * counts descending, ties by ascending id; at most `budget` ids per GPU.  Host CSR
+ * (symmetric), part host int32[n]; ids_out host int64 [C x budget] (rank r's ids,
+ * hottest first, at ids_out + r * budget), n_out host int64 [C].  Host only.           */
+apt_status apt_cache_sets(int64_t n, const int64_t* indptr, const int32_t* indices, const int32_t* part, int C,
+                          apt_strategy strategy, const int32_t* counts, int64_t budget, int64_t* ids_out,
+                          int64_t* n_out);
 /* apt_fstore_create with tiers (opts NULL: everything in HBM).  Row-sharded
- * layouts only (NFP: APT_E_UNSUPPORTED).  Kernels see one view per rank: own
+ * layouts only (NFP: APT_E_UNSUPPORTED: NFP keeps its 1/C column slice of every row,
+ * with that much memory it reads nothing from the host).  Kernels see one view per rank: own
  * HBM rows, NVLink peer rows, host rows, own cached rows.  Syncs.            */
 apt_status apt_fstore_create_tiered(apt_ctx* ctx, const apt_graph* g, apt_strategy layout, apt_dtype dtype,
                                     int dim, const float* host_feats, uint64_t feat_seed, const apt_fstore_opts* opts,

@@ -97,6 +97,52 @@ def tiered_store(part, C, hbm_frac, hot_ids=None, cache_rows=0):
     return tier
 
 
+def cache_sets(strategy, counts, part, C, budget, indptr=None, indices=None):
+    """P:163 "Cache configuration": the node ids each GPU keeps in its memory, from the
+    dry-run access frequencies `counts` (apt_access_counts, reading R12):
+      GDP, NFP -- "the most popular nodes" (of the whole graph);
+      SNP      -- "the most popular nodes in its assigned graph partition";
+      DNP      -- the most popular among "the nodes in its partition and their 1-hop
+                  neighbors" (needs the CSR).
+    Popularity order: count descending, then id ascending (reading C1); at most `budget`
+    ids per GPU.  Returns [ids of rank r, hottest first] for r in 0..C-1."""
+    counts = np.asarray(counts, np.int64)
+    part = np.asarray(part)
+    n = len(counts)
+    order = np.lexsort((np.arange(n), -counts))            # count desc, id asc
+    out = []
+    for r in range(C):
+        if strategy in ("GDP", "NFP"):
+            cand = np.ones(n, bool)
+        elif strategy == "SNP":
+            cand = part == r
+        elif strategy == "DNP":
+            own = part == r
+            cand = own.copy()
+            for u in np.nonzero(own)[0]:
+                cand[indices[indptr[u]:indptr[u + 1]]] = True
+        else:
+            raise ValueError(strategy)
+        out.append(order[cand[order]][:budget].astype(np.int64))
+    return out
+
+
+def cached_store(sets, n):
+    """The unified store of P:163 caches (P:241-247 feature map): rank r reads u from
+    its own cache if u is in sets[r], else from the lowest peer whose cache holds it
+    (NVLink), else from the host.  Returns tier(r, ids) -> 0 local, 1 peer, 2 host."""
+    C = len(sets)
+    mine = [np.zeros(n, bool) for _ in range(C)]
+    for r in range(C):
+        mine[r][np.asarray(sets[r], np.int64)] = True
+    anyc = np.any(mine, axis=0) if C else np.zeros(n, bool)
+
+    def tier(r, ids):
+        ids = np.asarray(ids, np.int64)
+        return np.where(mine[r][ids], 0, np.where(anyc[ids], 1, 2))
+    return tier
+
+
 def emulate_layer1(strategy, l1_blocks, part, C, d, d_out, feat_bytes=4, hidden_bytes=4, tier=None, heads=0):
     """l1_blocks[r] = rank r's layer-1 Block (dst, src, indptr, indices).  tier(r, ids):
     where rank r reads each row (0 local HBM, 1 NVLink peer, 2 host; default: own

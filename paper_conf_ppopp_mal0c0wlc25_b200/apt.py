@@ -50,11 +50,13 @@ class PlanStats(C.Structure):
                 ("feat_bytes_local", _A4), ("feat_bytes_peer", _A4), ("graph_bytes", _A4),
                 ("hidden_bytes_fwd", _A4), ("hidden_bytes_bwd", _A4), ("n_calls", _A4),
                 ("t_build_s", _D4), ("t_train_s", C.c_double), ("rows_host", _A4), ("feat_bytes_host", _A4),
-                ("gat_heads", C.c_int), ("attn_bytes", _A4), ("attn_feat_bytes", _A4)]
+                ("gat_heads", C.c_int), ("attn_bytes", _A4), ("attn_feat_bytes", _A4), ("t_resample_s", _D4),
+                ("t_dryrun_s", C.c_double)]
 
 
 class FstoreOpts(C.Structure):
-    _fields_ = [("hbm_frac", C.c_double), ("cache_rows", C.c_int64), ("hot_ids", C.c_void_p)]
+    _fields_ = [("hbm_frac", C.c_double), ("cache_rows", C.c_int64), ("hot_ids", C.c_void_p),
+                ("cache_rule", C.c_int), ("counts", C.c_void_p), ("cache_budget_rows", C.c_int64)]
 
 
 class BwProfile(C.Structure):
@@ -117,6 +119,7 @@ def lib():
             "apt_trainer_use_graph": [vp, i32], "apt_trainer_set_pipeline": [vp, i32], "apt_trainer_read": [vp, i32, i32, i32, vp, i64, vp, vp],
             "apt_trainer_phase_ms": [vp, vp, i32], "apt_trainer_agg_bytes": [vp, vp],
             "apt_partition": [i64, i64, vp, vp, i32, i32, u64, vp, vp],
+            "apt_cache_sets": [i64, vp, vp, vp, i32, i32, vp, i64, vp, vp],
             "apt_dryrun": [vp, i64, vp], "apt_access_counts": [vp, i64, vp], "apt_hot_rows": [vp, i64, i64, vp], "apt_trainer_layer_fwd": [vp, i64], "apt_trainer_layer_bwd": [vp, vp, i64],
             "apt_layer_fwd": [vp, i32, vp, vp, vp, vp, i32, i32, vp, vp], "apt_layer_bwd": [vp, vp, vp, vp, vp],
             "apt_layer_saved_destroy": [vp], "apt_batch_group": [vp, vp, i32, vp], "apt_profile_links": [vp, vp], "apt_select_strategy": [vp, vp, vp, vp],
@@ -208,11 +211,19 @@ class Ctx:
                                      indices.ctypes.data, _ptr(part), C.byref(h)))
         return Handle(h, lib().apt_graph_destroy, keep=(self,))
 
-    def fstore_create(self, graph, layout, dtype, dim, host_feats=None, feat_seed=0, hbm_frac=1.0, hot_ids=None):
+    def fstore_create(self, graph, layout, dtype, dim, host_feats=None, feat_seed=0, hbm_frac=1.0, hot_ids=None,
+                      counts=None, cache_budget_rows=None):
         """hbm_frac < 1: the rows beyond every shard's HBM budget form the pinned host tier;
-        hot_ids: rows replicated into every GPU's spare HBM (excess cache), hottest first."""
+        hot_ids: rows replicated into every GPU's spare HBM (excess cache), hottest first.
+        counts + cache_budget_rows: P:163's per-strategy GPU caches (APT_CACHE_P163)."""
         h = C.c_void_p()
         hf = None if host_feats is None else np.ascontiguousarray(host_feats, np.float32)
+        if counts is not None:
+            cnt = np.ascontiguousarray(counts, np.int32)
+            o = FstoreOpts(0.0, 0, None, CACHE_P163, cnt.ctypes.data, int(cache_budget_rows))
+            self.ck(lib().apt_fstore_create_tiered(self.h, graph.h, layout, dtype, dim, _ptr(hf), feat_seed,
+                                                   C.byref(o), C.byref(h)))
+            return Handle(h, lib().apt_fstore_destroy, keep=(self, graph, cnt))
         if hbm_frac == 1.0 and hot_ids is None:
             self.ck(lib().apt_fstore_create(self.h, graph.h, layout, dtype, dim, _ptr(hf), feat_seed, C.byref(h)))
             return Handle(h, lib().apt_fstore_destroy, keep=(self, graph))
@@ -456,6 +467,23 @@ def partition(indptr, indices, n_parts, method="ldg", seed=0):
     check(lib().apt_partition(n, int(indptr[-1]), indptr.ctypes.data, indices.ctypes.data, n_parts,
                               PARTITION[method], seed, part.ctypes.data, C.byref(cut)))
     return part, cut.value
+
+
+CACHE_P163 = 1
+
+
+def cache_sets(indptr, indices, part, n_parts, strategy, counts, budget):
+    """apt_cache_sets: every GPU's cache ids, hottest first."""
+    indptr = np.ascontiguousarray(indptr, np.int64)
+    indices = np.ascontiguousarray(indices, np.int32)
+    part = np.ascontiguousarray(part, np.int32)
+    counts = np.ascontiguousarray(counts, np.int32)
+    n = len(indptr) - 1
+    ids = np.zeros((n_parts, max(budget, 1)), np.int64)
+    cnt = np.zeros(n_parts, np.int64)
+    check(lib().apt_cache_sets(n, indptr.ctypes.data, indices.ctypes.data, part.ctypes.data, n_parts, strategy,
+                               counts.ctypes.data, budget, ids.ctypes.data, cnt.ctypes.data))
+    return [ids[r, :cnt[r]].copy() for r in range(n_parts)]
 
 
 def hot_rows(counts, k):

@@ -16,6 +16,7 @@
 // Counting is set-based: "unique rows read by owner c" is a bitmap per owner,
 // test-and-set with atomicOr, counted the moment a bit flips.
 #include <algorithm>
+#include <chrono>
 #include <cstring>
 #include <vector>
 
@@ -55,8 +56,10 @@ struct DryCounters {
 // own cache), 1 NVLink peer, 2 host tier.
 struct TierInfo {
   const int32_t* part; const int32_t* lrow; const int64_t* rows; const uint32_t* cache_bm; int64_t n_words;
+  const uint32_t* any_bm;   // P:163 caches: cached by some GPU (else the row is on the host only)
   __device__ __forceinline__ int of(int u, int r) const {
     if (cache_bm && (cache_bm[int64_t(r) * n_words + (u >> 5)] >> (u & 31) & 1u)) return 0;
+    if (any_bm) return (any_bm[u >> 5] >> (u & 31) & 1u) ? 1 : 2;
     const int o = part[u];
     if (rows && lrow[u] >= rows[o]) return 2;
     return o == r ? 0 : 1;
@@ -204,7 +207,8 @@ struct DrySampler {
   }
   void set_step(int64_t st, cudaStream_t s) { dry_set_step_kernel<<<1, 1, 0, s>>>(step_dev, uint64_t(st)); }
   // rank r's seeds of the current step (by_part: its partition's seeds, SNP/DNP) and its blocks
-  apt_status sample(int r, bool by_part) {
+  // e0 / e1 (optional): recorded around the layer-1 hop's sampling
+  apt_status sample(int r, bool by_part, cudaEvent_t e0 = nullptr, cudaEvent_t e1 = nullptr) {
     apt_ctx* c = t->ctx;
     const int C = t->world, K = t->K;
     const apt_graph* g = t->g;
@@ -215,7 +219,9 @@ struct DrySampler {
       Hop& hp = hops[h];
       SampleArgs sm{g->indptr, g->indices, hp.dst, hp.n_dst, hp.max_dst, hp.k,
                     philox_key(t->m.sample_seed, kDomSample), step_dev, h, hp.cnt, hp.nbr};
+      if (h == K - 1 && e0) CK(c, cudaEventRecord(e0, c->stream));
       CK(c, launch_sample(sm, c->stream));
+      if (h == K - 1 && e1) CK(c, cudaEventRecord(e1, c->stream));
       if (h + 1 < K) {
         CompactArgs ca{hp.dst, hp.n_dst, hp.max_dst, hp.cnt, hp.nbr, hp.k, dst_bm, new_bm, n_words, pos, hp.src,
                        hp.counts, hp.indptr, hp.indices, hp.counts + 1, partials, hp.part2};
@@ -244,10 +250,12 @@ extern "C" apt_status apt_dryrun(apt_trainer* t, int64_t n_steps, apt_plan_stats
   std::vector<Hop>& hops = ds.hops;
   if (!ok || !own_bm || !dc) return set_err(c, APT_E_OOM, "apt_dryrun: out of device memory");
   // tiers of the unified store (rows beyond the HBM budgets, replicated hot rows)
-  const TierInfo ti{g->part, g->lrow, t->f->tiered ? t->f->rows_dev : nullptr, t->f->cache_bm, n_words};
-  std::vector<cudaEvent_t> ev;
+  const TierInfo ti{g->part, g->lrow, t->f->tiered ? t->f->rows_dev : nullptr, t->f->cache_bm, n_words,
+                    t->f->p163 ? t->f->any_bm : nullptr};
+  std::vector<cudaEvent_t> ev, ev1;   // per (strategy, step, rank): whole sampling / the layer-1 hop
   struct Mark { int s, r; };
   std::vector<Mark> marks;
+  const auto wall0 = std::chrono::steady_clock::now();
   auto new_event = [&]() {
     cudaEvent_t e;
     cudaEventCreate(&e);
@@ -261,7 +269,12 @@ extern "C" apt_status apt_dryrun(apt_trainer* t, int64_t n_steps, apt_plan_stats
       CK(c, cudaMemsetAsync(own_bm, 0, sizeof(uint32_t) * n_words * C, c->stream));
       for (int r = 0; r < C; ++r) {
         CK(c, cudaEventRecord(new_event(), c->stream));
-        { apt_status s2 = ds.sample(r, by_part); if (s2 != APT_OK) return s2; }
+        cudaEvent_t h0, h1;
+        cudaEventCreate(&h0);
+        cudaEventCreate(&h1);
+        ev1.push_back(h0);
+        ev1.push_back(h1);
+        { apt_status s2 = ds.sample(r, by_part, h0, h1); if (s2 != APT_OK) return s2; }
         CK(c, cudaEventRecord(new_event(), c->stream));
         marks.push_back({S, r});
         const Hop& l1 = hops[K - 1];
@@ -281,12 +294,32 @@ extern "C" apt_status apt_dryrun(apt_trainer* t, int64_t n_steps, apt_plan_stats
   CK(c, cudaMemcpy(h, dc, sizeof h, cudaMemcpyDeviceToHost));
   // T_build per (strategy, rank): device time of the rank's seed selection + sampling
   double tb[4][APT_MAX_RANKS] = {};
+  double t_l1 = 0.0;   // layer-1 hop sampling, summed over every (strategy, step, rank)
   for (size_t i = 0; i < marks.size(); ++i) {
-    float ms = 0.f;
+    float ms = 0.f, ms1 = 0.f;
     cudaEventElapsedTime(&ms, ev[2 * i], ev[2 * i + 1]);
+    cudaEventElapsedTime(&ms1, ev1[2 * i], ev1[2 * i + 1]);
     tb[marks[i].s][marks[i].r] += ms * 1e-3;
+    t_l1 += ms1 * 1e-3;
   }
   for (auto e : ev) cudaEventDestroy(e);
+  for (auto e : ev1) cudaEventDestroy(e);
+  unsigned long long rows_l1 = 0;
+  for (int S = 0; S < 4; ++S)
+    for (int r = 0; r < C; ++r) rows_l1 += h[S].n_d[r];
+  // reading R1: an owner RE-SAMPLES the layer-1 rows other requesters send it (NFP: every
+  // other block; SNP / DNP: the items routed to it), at the measured layer-1 sampling
+  // cost per row -- part of its T_build ("sending part of their computation graphs")
+  const double per_row = rows_l1 ? t_l1 / double(rows_l1) : 0.0;
+  double tr[4][APT_MAX_RANKS] = {};
+  for (int cc = 0; cc < C && C > 1; ++cc) {
+    for (int b = 0; b < C; ++b)
+      if (b != cc) {
+        tr[APT_NFP][cc] += per_row * double(h[APT_NFP].n_d[b]);
+        tr[APT_SNP][cc] += per_row * double(h[APT_SNP].tot_rows[b][cc]);
+        tr[APT_DNP][cc] += per_row * double(h[APT_DNP].tot_rows[b][cc]);
+      }
+  }
 
   // ---- assemble the Planner statistics (message formats: oracle/strategy.py)
   memset(out, 0, sizeof *out);
@@ -298,7 +331,8 @@ extern "C" apt_status apt_dryrun(apt_trainer* t, int64_t n_steps, apt_plan_stats
   for (int S = 0; S < 4; ++S)
     for (int r = 0; r < C; ++r) {
       out->n_d[S][r] = h[S].n_d[r];
-      out->t_build_s[S][r] = tb[S][r];
+      out->t_resample_s[S][r] = tr[S][r];
+      out->t_build_s[S][r] = tb[S][r] + tr[S][r];
     }
   // GDP: local / peer / host rows of each requester's own block
   for (int r = 0; r < C; ++r) {
@@ -383,6 +417,7 @@ extern "C" apt_status apt_dryrun(apt_trainer* t, int64_t n_steps, apt_plan_stats
         out->attn_bytes[APT_SNP][cc] += int64_t(qs.tot_rows[r][cc]) * 2 * H * 4;
       }
   }
+  out->t_dryrun_s = std::chrono::duration<double>(std::chrono::steady_clock::now() - wall0).count();
   return APT_OK;
 }
 

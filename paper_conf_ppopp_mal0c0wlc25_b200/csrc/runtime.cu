@@ -61,6 +61,11 @@ apt_status check_cuda(apt_ctx* c, cudaError_t e, const char* what) {
     if (_s != APT_OK) return _s;                                    \
   } while (0)
 
+namespace apt {
+apt_status fstore_create_p163(apt_ctx* c, const apt_graph* g, apt_strategy layout, apt_dtype dtype, int dim,
+                              const float* host_feats, uint64_t feat_seed, const apt_fstore_opts* opts, apt_fstore** out);
+}
+
 extern "C" {
 
 apt_status apt_ctx_create(int rank, int world, int device, void* stream, apt_ctx** out) {
@@ -205,6 +210,8 @@ apt_status apt_fstore_create_tiered(apt_ctx* c, const apt_graph* g, apt_strategy
                                     apt_fstore** out) {
   if (!c || !g || !out || dim <= 0 || (dtype != APT_F32 && dtype != APT_BF16) || layout < APT_GDP || layout > APT_AUTO)
     return set_err(c, APT_E_INVALID, "apt_fstore_create: bad arguments");
+  if (opts && opts->cache_rule == APT_CACHE_P163) return apt::fstore_create_p163(c, g, layout, dtype, dim, host_feats,
+                                                                                  feat_seed, opts, out);
   const double frac = opts ? opts->hbm_frac : 1.0;
   const int64_t want_cache = opts ? opts->cache_rows : 0;
   if (!(frac > 0.0 && frac <= 1.0) || want_cache < 0 || (want_cache > 0 && !opts->hot_ids))
@@ -719,3 +726,174 @@ apt_status apt_weight_grad(apt_ctx* c, const float* G, int64_t g_pitch, const vo
 }
 
 }  // extern "C"
+
+// ---------------------------------------------------------------- P:163 caches
+extern "C" apt_status apt_cache_sets(int64_t n, const int64_t* indptr, const int32_t* indices, const int32_t* part,
+                                     int C, apt_strategy strategy, const int32_t* counts, int64_t budget,
+                                     int64_t* ids_out, int64_t* n_out) {
+  if (n < 1 || !counts || !ids_out || !n_out || C < 1 || C > APT_MAX_RANKS || budget < 0 ||
+      ((strategy == APT_SNP || strategy == APT_DNP) && !part) || (strategy == APT_DNP && (!indptr || !indices)) ||
+      strategy < APT_GDP || strategy > APT_DNP)
+    return set_err(nullptr, APT_E_INVALID, "apt_cache_sets: bad arguments");
+  // popularity order: count descending, id ascending (reading C1)
+  std::vector<int32_t> order(n);
+  for (int64_t u = 0; u < n; ++u) order[u] = int32_t(u);
+  std::stable_sort(order.begin(), order.end(), [&](int32_t a, int32_t b) { return counts[a] > counts[b]; });
+  std::vector<uint8_t> cand(n);
+  for (int r = 0; r < C; ++r) {
+    if (strategy == APT_GDP || strategy == APT_NFP) {
+      std::fill(cand.begin(), cand.end(), 1);
+    } else {
+      for (int64_t u = 0; u < n; ++u) cand[u] = part[u] == r;
+      if (strategy == APT_DNP)
+        for (int64_t u = 0; u < n; ++u)
+          if (part[u] == r)
+            for (int64_t e = indptr[u]; e < indptr[u + 1]; ++e) cand[indices[e]] = 1;
+    }
+    int64_t k = 0;
+    for (int64_t i = 0; i < n && k < budget; ++i)
+      if (cand[order[i]]) ids_out[int64_t(r) * budget + k++] = order[i];
+    n_out[r] = k;
+  }
+  return APT_OK;
+}
+
+namespace apt {
+// The store of P:163 caches: shard r = rank r's cache set (hottest first); the host tier
+// holds every row (pinned, mapped, row u at u); rank r's feature map: own cache, else
+// the lowest peer whose cache holds the row (NVLink), else the host.
+apt_status fstore_create_p163(apt_ctx* c, const apt_graph* g, apt_strategy layout, apt_dtype dtype, int dim,
+                              const float* host_feats, uint64_t feat_seed, const apt_fstore_opts* opts,
+                              apt_fstore** out) {
+  const int C = c->world;
+  if (!opts->counts || opts->cache_budget_rows < 0 || dim <= 0 || (dtype != APT_F32 && dtype != APT_BF16))
+    return set_err(c, APT_E_INVALID, "apt_fstore_create: P:163 caches need counts and a budget >= 0");
+  if (layout == APT_NFP && C > 1)
+    return set_err(c, APT_E_UNSUPPORTED, "apt_fstore_create: NFP keeps its column slice of every row (P:171)");
+  const apt_strategy s = layout == APT_AUTO ? APT_GDP : layout;
+  const int64_t B = std::min<int64_t>(opts->cache_budget_rows, g->n);
+  std::vector<int64_t> ids(size_t(C) * std::max<int64_t>(B, 1)), nr(C);
+  std::vector<int64_t> indptr_h;
+  std::vector<int32_t> indices_h;
+  if (s == APT_DNP) {
+    indptr_h.resize(g->n + 1);
+    indices_h.resize(g->nnz);
+    CK(c, cudaMemcpy(indptr_h.data(), g->indptr, sizeof(int64_t) * (g->n + 1), cudaMemcpyDeviceToHost));
+    CK(c, cudaMemcpy(indices_h.data(), g->indices, sizeof(int32_t) * g->nnz, cudaMemcpyDeviceToHost));
+  }
+  apt_status st = apt_cache_sets(g->n, s == APT_DNP ? indptr_h.data() : nullptr, s == APT_DNP ? indices_h.data() : nullptr,
+                                 g->part_h.data(), C, s, opts->counts, B, ids.data(), nr.data());
+  if (st != APT_OK) return st;
+  auto* f = new apt_fstore();
+  f->ctx = c;
+  ctx_retain(c);
+  f->g = g;
+  f->layout = s;
+  f->dtype = dtype == APT_BF16 ? kBF16 : kF32;
+  f->dim = dim;
+  f->world = C;
+  f->tiered = true;
+  f->p163 = true;
+  f->hbm_frac = 0.0;
+  const int align = dtype == APT_BF16 ? 8 : 4;
+  const size_t esz = dtype == APT_BF16 ? 2 : 4;
+  const int64_t pitch = round_up(dim, align);
+  for (int r = 0; r < C; ++r) {
+    f->col_lo[r] = 0;
+    f->col_hi[r] = dim;
+    f->pitch[r] = pitch;
+    f->rows[r] = nr[r];
+  }
+  int32_t* ids_dev = f->arena.alloc<int32_t>(std::max<int64_t>(g->n, 1), false);
+  auto fill = [&](void* dst, const int32_t* ids_h, int64_t n_rows) -> apt_status {
+    if (n_rows <= 0) return APT_OK;
+    if (host_feats) {
+      std::vector<uint8_t> buf(size_t(n_rows * pitch) * esz, 0);
+      for (int64_t i = 0; i < n_rows; ++i) {
+        const int64_t u = ids_h ? ids_h[i] : i;
+        for (int j = 0; j < dim; ++j) {
+          const float v = host_feats[u * dim + j];
+          if (esz == 4) {
+            reinterpret_cast<float*>(buf.data())[i * pitch + j] = v;
+          } else {
+            uint32_t bits;
+            memcpy(&bits, &v, 4);
+            reinterpret_cast<uint16_t*>(buf.data())[i * pitch + j] = uint16_t((bits + 0x7FFFu + ((bits >> 16) & 1u)) >> 16);
+          }
+        }
+      }
+      CK(c, cudaMemcpyAsync(dst, buf.data(), buf.size(), cudaMemcpyDefault, c->stream));
+    } else {
+      const int32_t* idp = nullptr;
+      if (ids_h) {
+        CK(c, cudaMemcpyAsync(ids_dev, ids_h, sizeof(int32_t) * n_rows, cudaMemcpyHostToDevice, c->stream));
+        idp = ids_dev;
+      }
+      CK(c, launch_fill_features(dst, f->dtype, pitch, 0, dim, idp, n_rows, feat_seed, c->stream));
+      c->launches++;
+    }
+    CK(c, cudaStreamSynchronize(c->stream));
+    return APT_OK;
+  };
+  // feature maps: holder[u] = the lowest rank caching u (-1: host only); rows inside each cache
+  const int64_t n_words = ceil_div(g->n, 32);
+  std::vector<int32_t> holder(g->n, -1), hrow(g->n, -1);
+  std::vector<uint32_t> bm(size_t(C) * n_words, 0u), any(n_words, 0u);
+  std::vector<std::vector<int32_t>> set32(C);
+  for (int r = 0; r < C; ++r) {
+    set32[r].resize(nr[r]);
+    for (int64_t i = 0; i < nr[r]; ++i) {
+      const int32_t u = int32_t(ids[size_t(r) * std::max<int64_t>(B, 1) + i]);
+      set32[r][i] = u;
+      bm[size_t(r) * n_words + (u >> 5)] |= 1u << (u & 31);
+      any[u >> 5] |= 1u << (u & 31);
+      if (holder[u] < 0) { holder[u] = r; hrow[u] = int32_t(i); }
+    }
+  }
+  for (int r = 0; r < C; ++r) {
+    if (!c->emulated && r != c->rank) continue;
+    f->shard[r] = f->arena.alloc<uint8_t>(std::max<int64_t>(nr[r], 1) * pitch * int64_t(esz), true);
+    if (!f->shard[r]) { apt_fstore_destroy(f); return set_err(c, APT_E_OOM, "apt_fstore_create: cache"); }
+    if ((st = fill(f->shard[r], set32[r].data(), nr[r])) != APT_OK) { apt_fstore_destroy(f); return st; }
+  }
+  f->host_rows = g->n;
+  if (cudaHostAlloc(&f->host, size_t(g->n * pitch) * esz, cudaHostAllocMapped | cudaHostAllocPortable) != cudaSuccess) {
+    apt_fstore_destroy(f);
+    return set_err(c, APT_E_OOM, "apt_fstore_create: pinned host tier of %lld rows", (long long)g->n);
+  }
+  if ((st = fill(f->host, nullptr, g->n)) != APT_OK) { apt_fstore_destroy(f); return st; }
+  f->rows_dev = f->arena.alloc<int64_t>(C, false);
+  f->cache_bm = f->arena.alloc<uint32_t>(int64_t(C) * n_words, false);
+  f->any_bm = f->arena.alloc<uint32_t>(n_words, false);
+  if (!f->rows_dev || !f->cache_bm || !f->any_bm) { apt_fstore_destroy(f); return set_err(c, APT_E_OOM, "cache maps"); }
+  CK(c, cudaMemcpyAsync(f->rows_dev, f->rows, sizeof(int64_t) * C, cudaMemcpyHostToDevice, c->stream));
+  CK(c, cudaMemcpyAsync(f->cache_bm, bm.data(), sizeof(uint32_t) * bm.size(), cudaMemcpyHostToDevice, c->stream));
+  CK(c, cudaMemcpyAsync(f->any_bm, any.data(), sizeof(uint32_t) * any.size(), cudaMemcpyHostToDevice, c->stream));
+  for (int r = 0; r < C; ++r) {
+    if (!c->emulated && r != c->rank) continue;
+    std::vector<int32_t> tier(g->n), trow(g->n);
+    std::vector<int32_t> own(g->n, -1);
+    for (int64_t i = 0; i < nr[r]; ++i) own[set32[r][i]] = int32_t(i);
+    for (int64_t u = 0; u < g->n; ++u) {
+      if (own[u] >= 0) { tier[u] = r; trow[u] = own[u]; }
+      else if (holder[u] >= 0) { tier[u] = holder[u]; trow[u] = hrow[u]; }
+      else { tier[u] = C; trow[u] = int32_t(u); }
+    }
+    f->tier_map[r] = f->arena.alloc<int32_t>(g->n, false);
+    f->trow_map[r] = f->arena.alloc<int32_t>(g->n, false);
+    if (!f->tier_map[r] || !f->trow_map[r]) { apt_fstore_destroy(f); return set_err(c, APT_E_OOM, "feature map"); }
+    CK(c, cudaMemcpyAsync(f->tier_map[r], tier.data(), sizeof(int32_t) * g->n, cudaMemcpyHostToDevice, c->stream));
+    CK(c, cudaMemcpyAsync(f->trow_map[r], trow.data(), sizeof(int32_t) * g->n, cudaMemcpyHostToDevice, c->stream));
+    CK(c, cudaStreamSynchronize(c->stream));
+    f->tier_h[r] = std::move(tier);
+  }
+  if (multiprocess(c)) {   // every rank maps every peer's cache (NVLink reads of peer-cached rows)
+    void* tab[APT_MAX_RANKS] = {};
+    apt_status s2 = share_ptr(c, f->shard[c->rank], tab, &f->peer_opened);
+    if (s2 != APT_OK) { apt_fstore_destroy(f); return s2; }
+    for (int r = 0; r < C; ++r) f->shard[r] = tab[r];
+  }
+  *out = f;
+  return APT_OK;
+}
+}  // namespace apt

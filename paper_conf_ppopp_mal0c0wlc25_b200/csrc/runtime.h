@@ -133,6 +133,8 @@ struct apt_fstore {
   // lrow[u] >= rows[part[u]] and not cached by r
   int64_t* rows_dev = nullptr;           // [C] HBM rows per shard
   uint32_t* cache_bm = nullptr;          // [C x ceil(n/32)] cached-by-rank bitmaps (null: no caches)
+  bool p163 = false;                     // APT_CACHE_P163: shards are the per-GPU cache sets
+  uint32_t* any_bm = nullptr;            // ... cached by some rank (NVLink-readable)
   std::vector<void*> peer_opened;   // IPC-mapped peer shards (multi-process)
   apt::Arena arena;
   ~apt_fstore() {

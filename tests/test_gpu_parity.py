@@ -693,3 +693,65 @@ def test_tiered_store_rows_and_step(A, tiny, dtype, frac, n_hot):
         for l in range(1, len(cfg.fanouts) + 1):
             assert_close(tr.read("dW", l, rank=0), sum(x["grads"][l - 1][0] for x in refs), dtype,
                          f"{strategy} C{C} dW{l}", sb["dW"][l - 1])
+
+
+# ------------------------------------------------------------------ P:163 per-strategy caches (NEXT #2)
+@pytest.mark.parametrize("dtype", ["f32", "bf16"])
+@pytest.mark.parametrize("strategy,C,frac", [("GDP", 2, 0.1), ("SNP", 2, 0.3), ("DNP", 2, 0.2), ("DNP", 4, 0.05),
+                                             ("GDP", 1, 0.02)])
+def test_p163_cache_store(A, tiny, strategy, C, frac, dtype):
+    """APT_CACHE_P163: every GPU's HBM holds its P:163 cache set (from the oracle's access
+    counts), every row also on the pinned host; rows read back bit-exact through the view,
+    the dry-run's per-tier counts equal the oracle's emulation under the same feature map
+    (own cache / peer cache over NVLink / host), and the strategy's step still
+    matches the oracle (the store only moves features)."""
+    from oracle import strategy as S
+    cfg, g, train = tiny
+    part = aptgen.partition(g.n, C)
+    counts = S.access_counts(g, train, cfg.fanouts, cfg.sample_seed, 0, C, cfg.batch, 2)
+    budget = int(frac * g.n)
+    ctx = A.Ctx(-1, C, 0) if C > 1 else A.Ctx(0, 1, 0)
+    gr = ctx.graph_load(g.indptr, g.indices, part)
+    fs = ctx.fstore_create(gr, A.STRATEGY[strategy], A.DTYPE[dtype], cfg.dim, None, cfg.feat_seed, counts=counts,
+                           cache_budget_rows=budget)
+    ids = np.arange(g.n, dtype=np.int64)
+    pitch = ((cfg.dim + 7) // 8 * 8) if dtype == "bf16" else ((cfg.dim + 3) // 4 * 4)
+    esz = 2 if dtype == "bf16" else 4
+    out = torch.zeros(g.n * pitch * esz, dtype=torch.uint8, device="cuda")
+    torch.cuda.synchronize()
+    ctx.gather(fs, torch.as_tensor(ids).cuda(), g.n, out)
+    torch.cuda.synchronize()
+    raw = out.cpu().numpy()
+    got = ((raw.view(np.uint16).astype(np.uint32) << 16).view(np.float32) if dtype == "bf16"
+           else raw.view(np.float32)).reshape(g.n, pitch)[:, :cfg.dim]
+    assert np.array_equal(got.astype(np.float64), oracle.features(cfg.feat_seed, ids, cfg.dim))
+    dims = [cfg.dim] + [d for _, d in cfg.dims()]
+    labels = aptgen.labels(cfg, g.n)
+    tr = A.Trainer(ctx, gr, fs, dims, cfg.fanouts, cfg.batch, A.DTYPE[dtype], 0.1, cfg.sample_seed, cfg.feat_seed,
+                   A.STRATEGY[strategy], labels)
+    params = aptgen.weights(cfg)
+    tr.set_params(params)
+    tr.set_epoch(train, 0)
+    # dry-run tiers vs the oracle's feature map of the same caches
+    st = tr.dryrun(2)
+    sets = S.cache_sets(strategy, counts, part, C, budget, g.indptr, g.indices)
+    tier = S.cached_store(sets, g.n)
+    perm = oracle.epoch_perm(train, cfg.sample_seed, 0)
+    si = S.STRATEGIES.index(strategy)
+    tot = [dict(rows_local=0, rows_peer=0, rows_host=0) for _ in range(C)]
+    for step in range(st.steps):
+        gb = oracle.global_batch(perm, step, C, cfg.batch)
+        seeds = S.assign_seeds(strategy, gb, part, C, cfg.batch)
+        blocks = [oracle.sample_blocks(g, sd, cfg.fanouts, cfg.sample_seed, step)[-1] for sd in seeds]
+        for r, e in enumerate(S.emulate_layer1(strategy, blocks, part, C, cfg.dim, cfg.hidden, 4, 4, tier=tier)):
+            for k in tot[r]:
+                tot[r][k] += e[k]
+    for r in range(C):
+        for k in tot[r]:
+            assert getattr(st, k)[si][r] == tot[r][k], (k, r, getattr(st, k)[si][r], tot[r][k])
+    tr.step(0, update=False)
+    seeds, refs, bds = _strategy_ref(cfg, g, train, labels, params, strategy, C, 0, dtype, bounds=tr)
+    for r in range(C):
+        assert_close(tr.read("H", 1, rank=r), refs[r]["cache"]["h"][0], dtype, f"H1 rank {r}", bds[r]["H"][0])
+    sb = sum_bounds(bds)
+    assert_close(tr.read("dW", 1, rank=0), sum(x["grads"][0][0] for x in refs), dtype, "dW1", sb["dW"][0])

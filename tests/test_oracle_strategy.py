@@ -301,3 +301,43 @@ def test_epoch_perm_is_sorted_by_philox_key_then_id():
         keys[int(u)] = int(w[0]) | (int(w[1]) << 32)
     expect = sorted(train.tolist(), key=lambda u: (keys[u], u))
     assert perm.tolist() == expect
+
+
+@pytest.mark.parametrize("strategy", ["GDP", "NFP", "SNP", "DNP"])
+def test_cache_sets_follow_p163(tiny_graph, tiny_cfg, strategy):
+    """P:163's cache rules, checked by brute force against their text: every cached node
+    is a candidate of the rule (SNP: own partition; DNP: partition + 1-hop neighbours;
+    GDP/NFP: any node), the set has min(budget, #candidates) nodes, and no uncached
+    candidate is more popular than a cached one (ties: the smaller id is cached)."""
+    g, C, budget = tiny_graph, 4, 700
+    part = aptgen.partition(g.n, C)
+    counts = S.access_counts(g, aptgen.train_nodes(g, tiny_cfg), tiny_cfg.fanouts, tiny_cfg.sample_seed, 0, C,
+                             tiny_cfg.batch, 2)
+    sets = S.cache_sets(strategy, counts, part, C, budget, g.indptr, g.indices)
+    for r in range(C):
+        if strategy in ("GDP", "NFP"):
+            cand = set(range(g.n))
+        elif strategy == "SNP":
+            cand = {u for u in range(g.n) if part[u] == r}
+        else:
+            own = [u for u in range(g.n) if part[u] == r]
+            cand = set(own) | {int(v) for u in own for v in g.indices[g.indptr[u]:g.indptr[u + 1]]}
+        got = [int(u) for u in sets[r]]
+        assert len(got) == len(set(got)) == min(budget, len(cand))
+        assert set(got) <= cand
+        rest = cand - set(got)
+        key = lambda u: (-int(counts[u]), u)
+        if rest:
+            assert max(key(u) for u in got) < min(key(u) for u in rest)
+        assert got == sorted(got, key=key)                 # hottest first
+    if strategy in ("GDP", "NFP"):
+        assert all(np.array_equal(sets[0], x) for x in sets)
+
+
+def test_cached_store_feature_map():
+    """own cache first, else a peer GPU's cache (NVLink), else the host."""
+    sets = [np.array([0, 1]), np.array([1, 2]), np.array([], np.int64)]
+    tier = S.cached_store(sets, 5)
+    assert tier(0, [0, 1, 2, 3]).tolist() == [0, 0, 1, 2]
+    assert tier(1, [0, 1, 2, 4]).tolist() == [1, 0, 0, 2]
+    assert tier(2, [0, 1, 2, 3]).tolist() == [1, 1, 1, 2]
