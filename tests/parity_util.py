@@ -219,3 +219,51 @@ def assert_close(got, ref, dtype, what, bound=None):
         raise AssertionError(f"{what}: {int(bad.sum())}/{ref.size} elements outside the bar (worst at {i}: got "
                              f"{got[i]!r} ref {ref[i]!r} allowed {np.broadcast_to(lim, ref.shape)[i]!r}; max abs "
                              f"err {err.max():.3e}, ref rms {rms(ref):.3e})")
+
+
+def gat_bounds(indptr, indices, x_src, n_dst, W, a_src, a_dst, b, cache, g, heads, dtype):
+    """atol of the GAT layer's h, dW, db, da_src, da_dst (reading T5): the
+    layer's forward and backward (oracle/gat.py) re-evaluated on MAGNITUDES -- every
+    signed sum replaced by the sum of the absolute values of its terms, the softmax
+    Jacobian by its absolute bound alpha (|d| + sum alpha |d|) -- gives M, the size of
+    the terms behind every output; a first-order bound is then c u M: fp32 (T1, the
+    longest sum is over the n_src sources) c = LAMBDA (sqrt(n_src) + 8), u = 2^-24; bf16
+    (T2: W, Z, g, gamma rounded along the chain) c = 4, u = 2^-8."""
+    W = np.abs(np.asarray(W, np.float64))
+    H = heads
+    dp, d = W.shape
+    F = dp // H
+    x = np.abs(np.asarray(x_src, np.float64))
+    n_src = x.shape[0]
+    rows = np.repeat(np.arange(n_dst), np.diff(indptr))
+    alpha = cache["alpha"]
+    Ya = (x @ W.T).reshape(n_src, H, F)
+    As = np.abs(np.asarray(a_src, np.float64)).reshape(H, F)
+    Ad = np.abs(np.asarray(a_dst, np.float64)).reshape(H, F)
+    el = np.einsum("uhf,hf->uh", Ya, As)
+    er = np.einsum("uhf,hf->uh", Ya[:n_dst], Ad)
+    sm = el[indices] + er[rows]                                  # |score| terms per edge
+    smax = np.zeros((n_dst, H))
+    np.maximum.at(smax, rows, sm)
+    agg = np.zeros((n_dst, H, F))
+    np.add.at(agg, rows, alpha[:, :, None] * Ya[indices])
+    Mh = (agg * (1.0 + 2.0 * smax[:, :, None])).reshape(n_dst, dp) + np.abs(np.asarray(b, np.float64))
+    gm = np.abs(np.asarray(g, np.float64)).reshape(n_dst, H, F)
+    dal = np.einsum("ehf,ehf->eh", gm[rows], Ya[indices])
+    t = np.zeros((n_dst, H))
+    np.add.at(t, rows, alpha * dal)
+    de = alpha * (dal + t[rows])
+    dY = np.zeros((n_src, H, F))
+    np.add.at(dY, indices, alpha[:, :, None] * gm[rows])
+    dl = np.zeros((n_src, H))
+    np.add.at(dl, indices, de)
+    dr = np.zeros((n_dst, H))
+    np.add.at(dr, rows, de)
+    dY += dl[:, :, None] * As[None]
+    dY[:n_dst] += dr[:, :, None] * Ad[None]
+    Mda_s = np.einsum("uh,uhf->hf", dl, Ya).reshape(-1)
+    Mda_d = np.einsum("vh,vhf->hf", dr, Ya[:n_dst]).reshape(-1)
+    MdW = dY.reshape(n_src, dp).T @ x
+    Mdb = gm.reshape(n_dst, dp).sum(axis=0)
+    cu = LAMBDA * (np.sqrt(n_src) + 8) * U32 if dtype == "f32" else 4 * 2.0 ** -8
+    return {"h": cu * Mh, "dW": cu * MdW, "db": cu * Mdb, "da_src": cu * Mda_s, "da_dst": cu * Mda_d}
