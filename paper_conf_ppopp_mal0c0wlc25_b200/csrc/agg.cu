@@ -41,7 +41,10 @@ struct EllFstoreSrc {            // layer 1: sampler ELL + the feature store (lo
   __device__ __forceinline__ int cap(int c) const { return k; }
   __device__ __forceinline__ int node(int64_t e) const { return nbr[e]; }
   __device__ __forceinline__ const char* row_ptr(int u) const {
-    if (fv.part) return reinterpret_cast<const char*>(fv.base[fv.part[u]]) + int64_t(fv.lrow[u]) * row_bytes;
+    if (fv.loc) {   // one 8-byte (tier, row) load: local shard, NVLink peer, host tier or cache
+      const int2 l = __ldg(fv.loc + u);
+      return reinterpret_cast<const char*>(fv.base[l.x]) + int64_t(l.y) * row_bytes;
+    }
     return reinterpret_cast<const char*>(fv.base[0]) + int64_t(u) * row_bytes;
   }
 };
@@ -369,7 +372,8 @@ __global__ void gather_kernel(FeatView fv, const int32_t* __restrict__ ids, cons
   const int64_t nwarps = int64_t(gridDim.x) * (blockDim.x >> 5);
   for (int64_t i = (int64_t(blockIdx.x) * blockDim.x + threadIdx.x) >> 5; i < n; i += nwarps) {
     const int u = ids[i];
-    const char* row = fv.part ? reinterpret_cast<const char*>(fv.base[fv.part[u]]) + int64_t(fv.lrow[u]) * fv.pitch * esz
+    const int2 l = fv.loc ? __ldg(fv.loc + u) : make_int2(0, u);
+    const char* row = fv.loc ? reinterpret_cast<const char*>(fv.base[l.x]) + int64_t(l.y) * fv.pitch * esz
                               : reinterpret_cast<const char*>(fv.base[0]) + int64_t(u) * fv.pitch * esz;
     for (int j = lane; j < V; j += 32)
       *reinterpret_cast<uint4*>(out + i * out_pitch_bytes + j * 16) = ld_nc_v4(row + j * 16);

@@ -98,7 +98,10 @@ struct GatKArgs {
 };
 
 __device__ __forceinline__ const char* gat_row(const GatKArgs& a, int u) {
-  if (a.fv.part) return reinterpret_cast<const char*>(a.fv.base[a.fv.part[u]]) + int64_t(a.fv.lrow[u]) * a.row_bytes;
+  if (a.fv.loc) {
+    const int2 l = __ldg(a.fv.loc + u);
+    return reinterpret_cast<const char*>(a.fv.base[l.x]) + int64_t(l.y) * a.row_bytes;
+  }
   return reinterpret_cast<const char*>(a.fv.base[0]) + int64_t(u) * a.row_bytes;
 }
 

@@ -83,8 +83,8 @@ enum DType : int { kF32 = 0, kBF16 = 1 };
 // (pinned, mapped), C+1 = this rank's cache of replicated hot rows.
 struct FeatView {
   const void* base[10];        // per-tier base (local / NVLink peer / mapped host / own cache)
-  const int32_t* part;         // tier of node u (nullptr => single shard, row = u)
-  const int32_t* lrow;         // row of u inside its tier
+  const int2* loc;             // (tier, row inside the tier) of node u: ONE 8-byte load per edge
+                               // (nullptr => single shard, row = u)
   int64_t pitch;               // elements per stored row (padded to 16 B)
   int dim;                     // logical columns to aggregate
   int col0;                    // first column inside the stored row

@@ -166,7 +166,8 @@ apt_status apt_graph_load(apt_ctx* c, int64_t n, int64_t nnz, const int64_t* ind
   g->indices = g->arena.alloc<int32_t>(nnz, false);
   g->part = g->arena.alloc<int32_t>(n, false);
   g->lrow = g->arena.alloc<int32_t>(n, false);
-  if (!g->indptr || !g->indices || !g->part || !g->lrow) {
+  g->loc = g->arena.alloc<int2>(n, false);
+  if (!g->indptr || !g->indices || !g->part || !g->lrow || !g->loc) {
     apt_graph_destroy(g);
     return set_err(c, APT_E_OOM, "apt_graph_load: out of device memory (n=%lld nnz=%lld)", (long long)n, (long long)nnz);
   }
@@ -186,6 +187,12 @@ apt_status apt_graph_load(apt_ctx* c, int64_t n, int64_t nnz, const int64_t* ind
   if (nnz) CK(c, cudaMemcpyAsync(g->indices, indices, sizeof(int32_t) * nnz, cudaMemcpyHostToDevice, c->stream));
   CK(c, cudaMemcpyAsync(g->part, g->part_h.data(), sizeof(int32_t) * n, cudaMemcpyHostToDevice, c->stream));
   CK(c, cudaMemcpyAsync(g->lrow, lrow.data(), sizeof(int32_t) * n, cudaMemcpyHostToDevice, c->stream));
+  {
+    std::vector<int2> loc(n);
+    for (int64_t u = 0; u < n; ++u) loc[u] = make_int2(g->part_h[u], lrow[u]);
+    CK(c, cudaMemcpyAsync(g->loc, loc.data(), sizeof(int2) * n, cudaMemcpyHostToDevice, c->stream));
+    CK(c, cudaStreamSynchronize(c->stream));
+  }
   CK(c, cudaStreamSynchronize(c->stream));
   *out = g;
   return APT_OK;
@@ -371,12 +378,14 @@ apt_status apt_fstore_create_tiered(apt_ctx* c, const apt_graph* g, apt_strategy
         apt_status st = fill_rows(f->cache[r], cached.data(), f->cache_rows[r], 0, dim, pitch);
         if (st != APT_OK) { apt_fstore_destroy(f); return st; }
       }
-      f->tier_map[r] = f->arena.alloc<int32_t>(g->n, false);
-      f->trow_map[r] = f->arena.alloc<int32_t>(g->n, false);
-      if (!f->tier_map[r] || !f->trow_map[r]) { apt_fstore_destroy(f); return set_err(c, APT_E_OOM, "feature map"); }
-      CK(c, cudaMemcpyAsync(f->tier_map[r], tier.data(), sizeof(int32_t) * g->n, cudaMemcpyHostToDevice, c->stream));
-      CK(c, cudaMemcpyAsync(f->trow_map[r], trow.data(), sizeof(int32_t) * g->n, cudaMemcpyHostToDevice, c->stream));
-      CK(c, cudaStreamSynchronize(c->stream));
+      f->loc_map[r] = f->arena.alloc<int2>(g->n, false);
+      if (!f->loc_map[r]) { apt_fstore_destroy(f); return set_err(c, APT_E_OOM, "feature map"); }
+      {
+        std::vector<int2> loc(g->n);
+        for (int64_t u = 0; u < g->n; ++u) loc[u] = make_int2(tier[u], trow[u]);
+        CK(c, cudaMemcpyAsync(f->loc_map[r], loc.data(), sizeof(int2) * g->n, cudaMemcpyHostToDevice, c->stream));
+        CK(c, cudaStreamSynchronize(c->stream));
+      }
       f->tier_h[r] = std::move(tier);
     }
   }
@@ -412,20 +421,17 @@ FeatView feat_view(const apt_fstore* f, int r) {
     const int rr = f->world > 1 ? r : 0;
     v.base[f->world] = f->host;
     v.base[f->world + 1] = f->cache[rr];
-    v.part = f->tier_map[rr];
-    v.lrow = f->trow_map[rr];
+    v.loc = f->loc_map[rr];
     v.pitch = f->pitch[0];
     v.dim = f->dim;
   } else if (rows_sharded) {
-    v.part = f->g->part;
-    v.lrow = f->g->lrow;
+    v.loc = f->g->loc;
     v.pitch = f->pitch[0];
     v.dim = f->dim;
   } else {
     const int s = f->world > 1 ? r : 0;
     v.base[0] = f->shard[s];
-    v.part = nullptr;
-    v.lrow = nullptr;
+    v.loc = nullptr;
     v.pitch = f->pitch[s];
     v.dim = f->col_hi[s] - f->col_lo[s];
   }
@@ -879,12 +885,14 @@ apt_status fstore_create_p163(apt_ctx* c, const apt_graph* g, apt_strategy layou
       else if (holder[u] >= 0) { tier[u] = holder[u]; trow[u] = hrow[u]; }
       else { tier[u] = C; trow[u] = int32_t(u); }
     }
-    f->tier_map[r] = f->arena.alloc<int32_t>(g->n, false);
-    f->trow_map[r] = f->arena.alloc<int32_t>(g->n, false);
-    if (!f->tier_map[r] || !f->trow_map[r]) { apt_fstore_destroy(f); return set_err(c, APT_E_OOM, "feature map"); }
-    CK(c, cudaMemcpyAsync(f->tier_map[r], tier.data(), sizeof(int32_t) * g->n, cudaMemcpyHostToDevice, c->stream));
-    CK(c, cudaMemcpyAsync(f->trow_map[r], trow.data(), sizeof(int32_t) * g->n, cudaMemcpyHostToDevice, c->stream));
-    CK(c, cudaStreamSynchronize(c->stream));
+    f->loc_map[r] = f->arena.alloc<int2>(g->n, false);
+    if (!f->loc_map[r]) { apt_fstore_destroy(f); return set_err(c, APT_E_OOM, "feature map"); }
+    {
+      std::vector<int2> loc(g->n);
+      for (int64_t u = 0; u < g->n; ++u) loc[u] = make_int2(tier[u], trow[u]);
+      CK(c, cudaMemcpyAsync(f->loc_map[r], loc.data(), sizeof(int2) * g->n, cudaMemcpyHostToDevice, c->stream));
+      CK(c, cudaStreamSynchronize(c->stream));
+    }
     f->tier_h[r] = std::move(tier);
   }
   if (multiprocess(c)) {   // every rank maps every peer's cache (NVLink reads of peer-cached rows)

@@ -99,6 +99,7 @@ struct apt_graph {
   int32_t* indices = nullptr;    // device
   int32_t* part = nullptr;       // device owner of every node
   int32_t* lrow = nullptr;       // device row inside the owner's shard
+  int2* loc = nullptr;           // device (part, lrow) of every node: the feature view's one 8-B load
   std::vector<int32_t> part_h;   // host copy
   std::vector<int64_t> shard_rows;   // rows per rank
   int world = 1;
@@ -125,8 +126,7 @@ struct apt_fstore {
   void* host = nullptr;                  // pinned, mapped: rows beyond every shard's HBM budget
   int64_t cache_rows[APT_MAX_RANKS] = {};
   void* cache[APT_MAX_RANKS] = {};       // replicated hot rows (hosted ranks)
-  int32_t* tier_map[APT_MAX_RANKS] = {}; // device [n] per hosted rank
-  int32_t* trow_map[APT_MAX_RANKS] = {};
+  int2* loc_map[APT_MAX_RANKS] = {};     // device [n] per hosted rank: (tier, row) of every node
   std::vector<int32_t> tier_h[APT_MAX_RANKS];   // host copies (tests)
   // for the dry-run's tier classification of every rank's reads (all ranks, any process):
   // u is local to r iff cached by r or (part[u] == r and lrow[u] < rows[r]); host iff
