@@ -375,6 +375,12 @@ def run_apt(args, cfg):
     peaks = json.load(open(os.path.join(ROOT, "MEASURED_PEAKS.json"))) if os.path.exists(
         os.path.join(ROOT, "MEASURED_PEAKS.json")) else None
     hbm_peak = peaks["hbm_gbs"] if peaks else 6650.0
+    # with the pipeline (GDP, SAGE) the layer-1 gather+mean timed inside step i belongs to
+    # the NEXT batch (the sampling branch aggregates it, trainer z_prefetch): pair its time
+    # with the bytes of step i+1 (consecutive steps only)
+    if not args.no_pipeline and not GAT_HEADS and args.strategy == "GDP" and os.environ.get("APT_Z_PREFETCH", "0") == "1":
+        pairs = [(agg_ms[i], agg_bytes[i + 1]) for i in range(len(agg_ms) - 1) if step_ids[i + 1] == step_ids[i] + 1]
+        agg_ms, agg_bytes = [p_[0] for p_ in pairs], [p_[1] for p_ in pairs]
     achieved = sum(agg_bytes) / (sum(agg_ms) * 1e-3) / 1e9
     # DRAM traffic of the same kernel from one committed `ncu --set full` capture of this
     # workload (dram__bytes_read + dram__bytes_write per launch), next to the algorithmic bytes

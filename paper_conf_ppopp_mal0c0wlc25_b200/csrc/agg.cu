@@ -293,11 +293,13 @@ cudaError_t launch_agg_fstore(const AggArgs& a, const FeatView& fv, cudaStream_t
   if (V <= 16 && b.k <= 16) {
     if (fv.dtype == kBF16) {
       auto kern = agg_l1_pf_kernel<8, 5, 4>;
-      const int64_t blocks = grid_cap(ceil_div(ceil_div(b.max_dst, 2) * 32, 256), resident_blocks(kern, 256));
+      const int64_t blocks = grid_cap(ceil_div(ceil_div(b.max_dst, 2) * 32, 256),
+                                      b.bpsm > 0 ? b.bpsm : resident_blocks(kern, 256));
       launch_pdl(kern, dim3(blocks), dim3(256), 0, st, b, s);
     } else {
       auto kern = agg_l1_pf_kernel<4, 4, 6>;
-      const int64_t blocks = grid_cap(ceil_div(ceil_div(b.max_dst, 2) * 32, 256), resident_blocks(kern, 256));
+      const int64_t blocks = grid_cap(ceil_div(ceil_div(b.max_dst, 2) * 32, 256),
+                                      b.bpsm > 0 ? b.bpsm : resident_blocks(kern, 256));
       launch_pdl(kern, dim3(blocks), dim3(256), 0, st, b, s);
     }
     return cudaGetLastError();

@@ -118,6 +118,8 @@ struct AggArgs {
   uint16_t* z_bf16;
   int64_t z_bf16_pitch;
   int z_ones;                  // write 1.0 into bf16 column `dim` (bias-gradient column of the wgrad GEMM)
+  int bpsm;                    // > 0: grid capped at this many blocks per SM (a background launch that
+                               //   leaves registers for the step's chain beside it)
 };
 cudaError_t launch_agg_fstore(const AggArgs& a, const FeatView& fv, cudaStream_t st);
 cudaError_t launch_agg_csr(const AggArgs& a, cudaStream_t st);

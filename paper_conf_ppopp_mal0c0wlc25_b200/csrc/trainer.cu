@@ -373,6 +373,14 @@ apt_status apt::trainer_create(apt_ctx* c, const apt_graph* g, const apt_fstore*
       L.b = A.alloc<float>(L.d_out, true);
       L.Wb = A.alloc<uint16_t>(int64_t(L.d_out) * L.wb_pitch, true);
     }
+    // layer-1 Z per sample set (the pipelined sampling branch aggregates the next batch)
+    {
+      Layer& L1 = rs.L[0];
+      rs.sset[0].z1b = L1.Zb;
+      rs.sset[0].z1f = L1.Zf;
+      if (L1.Zb) rs.sset[1].z1b = A.alloc<uint16_t>(L1.max_rows * L1.zb_pitch, true);
+      if (L1.Zf) rs.sset[1].z1f = A.alloc<float>(L1.max_rows * L1.zf_pitch, true);
+    }
     // flat gradient buffer [dW1 db1 dW2 db2 ...] so one all-reduce covers the model
     const int64_t P = grad_floats(t, rs);
     float* grads = A.alloc<float>(P, true);
@@ -425,6 +433,13 @@ apt_status apt::trainer_create(apt_ctx* c, const apt_graph* g, const apt_fstore*
     CK(c, cudaMemcpyAsync(t->dW_tab, tab.data(), sizeof(float*) * C, cudaMemcpyHostToDevice, c->stream));
   }
   for (int i = 0; i < 8; ++i) cudaEventCreate(&t->ev[i]);
+  {
+    // opt-in (A/B): the next batch's layer-1 gather+mean on the sampling branch.
+    // Step 0.187 -> 0.179 ms, but the gather then runs beside the latency-bound backward
+    // (pull / wgrad: 60 -> 92 us) and its own in-step time rises 30 -> 43 us
+    const char* zp = std::getenv("APT_Z_PREFETCH");
+    t->z_prefetch = (zp && atoi(zp) != 0) && !t->gat_heads && (C == 1 || s == APT_GDP);
+  }
   CK(c, cudaStreamSynchronize(c->stream));
   *out = t;
   return APT_OK;
@@ -637,27 +652,60 @@ void activate(apt_trainer* t, int q) {
     rs.small = ss.small;
     rs.hops = ss.hops;
     for (int l = 1; l <= t->K; ++l) rs.L[l - 1].n_rows = ss.hops[t->K - l].n_dst;
+    if (ss.z1b) rs.L[0].Zb = ss.z1b;
+    if (ss.z1f) rs.L[0].Zf = ss.z1f;
   }
   t->step_dev = t->step_cells + q;
   t->parity = q;
 }
 
-// GDP layer-1 forward on one rank: the fused gather+mean (local + peer rows), then the
-// projection.
-apt_status layer1_fwd_gdp(apt_trainer* t, RankState& rs, bool time_it) {
+// The layer-1 gather+mean of sample set q of one rank (local + peer rows) into the
+// set's Z, on stream st; time_it: bracketed by the phase events 6 / 7 (on st).
+apt_status agg_l1_set(apt_trainer* t, RankState& rs, int q, cudaStream_t st, bool time_it) {
   apt_ctx* c = t->ctx;
-  Layer& L = rs.L[0];
-  const Hop& hp = rs.hops[t->K - 1];
+  const Layer& L = rs.L[0];
+  const SampleSet& ss = rs.sset[q];
+  const Hop& hp = ss.hops[t->K - 1];
   const FeatView fv = feat_view(t->f, rs.rank);
   AggArgs a{};
   a.cnt = hp.cnt; a.nbr = hp.nbr; a.k = hp.k;
   a.n_dst = hp.n_dst; a.max_dst = hp.max_dst; a.dim = L.d_in;
-  if (t->m.dtype == APT_BF16) { a.z_bf16 = L.Zb; a.z_bf16_pitch = L.zb_pitch; a.z_ones = 1; }
-  else { a.z_f32 = L.Zf; a.z_f32_pitch = L.zf_pitch; a.z_ones = 1; }
-  if (time_it) CK(c, record_ev(t, 6));
-  CK(c, launch_agg_fstore(a, fv, c->stream));
+  if (t->m.dtype == APT_BF16) { a.z_bf16 = ss.z1b; a.z_bf16_pitch = L.zb_pitch; a.z_ones = 1; }
+  else { a.z_f32 = ss.z1f; a.z_f32_pitch = L.zf_pitch; a.z_ones = 1; }
+  // beside the step (the sampling branch): a capped grid leaves registers for the chain
+  static const int zbg = [] { const char* v = std::getenv("APT_ZBG_BPSM"); return v ? atoi(v) : 0; }();
+  if (st == c->samp) a.bpsm = zbg;
+  auto rec = [&](int i) {
+    return t->capturing ? cudaEventRecordWithFlags(t->ev[i], st, cudaEventRecordExternal) : cudaEventRecord(t->ev[i], st);
+  };
+  if (time_it) CK(c, rec(6));
+  CK(c, launch_agg_fstore(a, fv, st));
   c->launches++;
-  if (time_it) CK(c, record_ev(t, 7));
+  if (time_it) CK(c, rec(7));
+  return APT_OK;
+}
+
+// The layer-1 aggregation of the batch in set q for every hosted rank on stream st
+// (the pipelined sampling branch: it depends only on the batch and the static store).
+apt_status prefetch_z(apt_trainer* t, int q, cudaStream_t st) {
+  bool first = true;
+  for (auto& rs : t->R) {
+    apt_status s = agg_l1_set(t, rs, q, st, first);
+    first = false;
+    if (s != APT_OK) return s;
+  }
+  return APT_OK;
+}
+
+// GDP layer-1 forward on one rank: the fused gather+mean (local + peer rows) -- unless
+// the pipelined sampling branch already aggregated this batch (z_ready) -- then the
+// projection.
+apt_status layer1_fwd_gdp(apt_trainer* t, RankState& rs, bool time_it) {
+  Layer& L = rs.L[0];
+  if (!t->z_ready) {
+    apt_status s = agg_l1_set(t, rs, t->parity, t->ctx->stream, time_it);
+    if (s != APT_OK) return s;
+  }
   return project(t, L, L.Zb, L.Zf, L.zb_pitch, L.zf_pitch, L.n_rows, L.max_rows, L.d_in, L.W, L.Wb, L.b,
                  t->K > 1 ? 1 : 0, L.H, nullptr, nullptr, nullptr);
 }
@@ -867,6 +915,7 @@ apt_status pipelined_body(apt_trainer* t, int p, int update, uint64_t next) {
     CK(c, cudaGetLastError());
     c->launches++;
     apt_status s2 = sample_all(t, p ^ 1, false, c->samp, false);
+    if (s2 == APT_OK && t->z_prefetch) s2 = prefetch_z(t, p ^ 1, c->samp);   // next batch's layer-1 Z
     if (s2 != APT_OK) return s2;
     CK(c, cudaEventRecord(c->ev_pjoin, c->samp));
     return APT_OK;
@@ -874,7 +923,9 @@ apt_status pipelined_body(apt_trainer* t, int p, int update, uint64_t next) {
   if (s != APT_OK) return s;
   t->csc_forked = false;
   activate(t, p);
+  t->z_ready = t->z_prefetch;   // this batch's Z was aggregated by the previous step's branch (or the prime)
   s = compute_body(t, update);
+  t->z_ready = false;
   if (s != APT_OK) return s;
   CK(c, cudaStreamWaitEvent(c->stream, c->ev_pjoin, 0));   // next step's batch complete
   return APT_OK;
@@ -1201,6 +1252,7 @@ apt_status apt_trainer_step(apt_trainer* t, int64_t step, int update) {
     c->launches++;
     t->csc_forked = false;
     apt_status s = sample_all(t, p, false, c->stream, false);
+    if (s == APT_OK && t->z_prefetch) s = prefetch_z(t, p, c->stream);
     if (s != APT_OK) return s;
   }
   const uint64_t next = uint64_t(step + 1);
@@ -1336,6 +1388,7 @@ apt_status apt_trainer_step_host_pipelined(apt_trainer* t, const int64_t* next_b
     CK(c, cudaGetLastError());
     t->csc_forked = false;
     apt_status s = sample_all(t, 0, true, c->stream, false);
+    if (s == APT_OK && t->z_prefetch) s = prefetch_z(t, 0, c->stream);
     if (s != APT_OK) return s;
     CK(c, cudaStreamSynchronize(c->stream));
     t->host_primed = true;
@@ -1353,6 +1406,7 @@ apt_status apt_trainer_step_host_pipelined(apt_trainer* t, const int64_t* next_b
       set_step_kernel<<<1, 1, 0, c->samp>>>(t->step_cells + q, nstep);
       CK(c, cudaGetLastError());
       apt_status s2 = sample_all(t, q, true, c->samp, false);
+      if (s2 == APT_OK && t->z_prefetch) s2 = prefetch_z(t, q, c->samp);
       if (s2 != APT_OK) return s2;
       CK(c, cudaEventRecord(c->ev_pjoin, c->samp));
       return APT_OK;
@@ -1360,7 +1414,9 @@ apt_status apt_trainer_step_host_pipelined(apt_trainer* t, const int64_t* next_b
     if (s != APT_OK) return s;
     t->csc_forked = false;
     activate(t, p);
+    t->z_ready = t->z_prefetch;
     s = compute_body(t, update);
+    t->z_ready = false;
     if (s != APT_OK) return s;
     for (size_t i = 0; i < t->R.size(); ++i)
       CK(c, cudaMemcpyAsync(t->loss_pinned + i, t->R[i].loss, sizeof(float), cudaMemcpyDeviceToHost, c->stream));

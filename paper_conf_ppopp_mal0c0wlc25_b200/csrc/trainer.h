@@ -120,6 +120,8 @@ struct GatState {
 // The sampled mini-batch of one step (seeds, K hops, block transposes).  Two per
 // rank: step t+1 is sampled into one while step t computes on the other.
 struct SampleSet {
+  uint16_t* z1b = nullptr;          // layer-1 Z of this batch (bf16 / fp32 mode): with the pipeline the
+  float* z1f = nullptr;             //   sampling branch also aggregates it (z_prefetch)
   int32_t* seeds = nullptr;
   int32_t* small = nullptr;         // [0] n_seeds [1] n_global
   uint64_t* step_cell = nullptr;    // step id of the batch held here (Philox key of its samples)
@@ -181,6 +183,9 @@ struct apt_trainer {
   bool capturing = false;
   // pipelining: step t+1 is sampled on ctx->samp while step t computes
   bool pipeline = true;
+  bool z_prefetch = false;           // GDP SAGE layer 1: the next batch's gather+mean runs on the sampling
+                                     //   branch (it reads only the static features), beside this step
+  bool z_ready = false;              // the active set's layer-1 Z is already aggregated
   int parity = 0;                    // sample set the last step computed on
   int64_t primed = -1;               // step id already sampled into sset[primed_parity]
   int primed_parity = 0;
