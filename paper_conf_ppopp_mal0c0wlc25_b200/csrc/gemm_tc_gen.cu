@@ -76,6 +76,7 @@ struct Params {
   float* const* out_base; const int32_t* out_rank; const int32_t* out_row;
   int ones_col; float* ones_out;
   int tmem_cols;
+  uint16_t* Yb; int64_t yb_pitch;   // bf16 rows instead of C (hidden activations, reading R11)
 };
 
 __device__ __forceinline__ void mma_tf32(uint32_t d, uint64_t a, uint64_t b, uint32_t idesc, uint32_t acc) {
@@ -306,7 +307,9 @@ __global__ void __launch_bounds__(THREADS, 1)
       fence_after();
       const int64_t m = ti.mt * BM + q * 32 + lane;
       float* row = nullptr;
-      if (m < M) row = p.out_rank ? p.out_base[p.out_rank[m]] + int64_t(p.out_row[m]) * p.ldc : p.C + m * p.ldc;
+      if (m < M)
+        row = p.Yb ? reinterpret_cast<float*>(p.Yb + m * p.yb_pitch)
+                   : (p.out_rank ? p.out_base[p.out_rank[m]] + int64_t(p.out_row[m]) * p.ldc : p.C + m * p.ldc);
       const bool add_bias = p.bias && ti.ks == 0;
       const uint32_t tbase = tmem_base + (uint32_t(q * 32) << 16) + uint32_t(acc * p.BN);
       uint32_t r[16], rn[16];
@@ -325,7 +328,17 @@ __global__ void __launch_bounds__(THREADS, 1)
             if (p.relu) v[j] = fmaxf(v[j], 0.f);
           }
           const bool plain = p.vec && n0 + 16 <= p.N && !(p.ones_col >= n0 && p.ones_col < n0 + 16);
-          if (plain) {
+          if (p.Yb) {
+            uint16_t* d = reinterpret_cast<uint16_t*>(row) + n0;
+            if (n0 + 16 <= p.N) {
+              reinterpret_cast<uint4*>(d)[0] = make_uint4(pack_bf16x2(v[0], v[1]), pack_bf16x2(v[2], v[3]),
+                                                          pack_bf16x2(v[4], v[5]), pack_bf16x2(v[6], v[7]));
+              reinterpret_cast<uint4*>(d)[1] = make_uint4(pack_bf16x2(v[8], v[9]), pack_bf16x2(v[10], v[11]),
+                                                          pack_bf16x2(v[12], v[13]), pack_bf16x2(v[14], v[15]));
+            } else {
+              for (int j = 0; j < 16 && n0 + j < p.N; ++j) d[j] = bf16_bits(v[j]);
+            }
+          } else if (plain) {
             float* d = row + n0;
 #pragma unroll
             for (int j = 0; j < 16; j += 4) {
@@ -442,6 +455,9 @@ cudaError_t launch_tc_gen_gemm(const SimtGemmArgs& a, int ones_col, float* ones_
   if (a.out_rank) p.vec = a.ldc % 4 == 0 ? 1 : 0;   // peer buffers: 256-B aligned allocations
   p.out_base = a.out_base; p.out_rank = a.out_rank; p.out_row = a.out_row;
   p.ones_col = ones_col; p.ones_out = ones_out;
+  p.Yb = a.Cb; p.yb_pitch = a.ldcb;
+  if (a.Cb && (a.out_rank || a.accumulate || (a.ldcb % 8) || (reinterpret_cast<uintptr_t>(a.Cb) & 15)))
+    return cudaErrorInvalidValue;
   CUtensorMap ma, mb;
   // A(m, k) = A[m * sam + k * sak]
   bool ok = p.a_mn ? make_map2(&ma, a.A, f32, a.M, a.K, a.sak, at, BK) : make_map2(&ma, a.A, f32, a.K, a.M, a.sam, BK, BM);

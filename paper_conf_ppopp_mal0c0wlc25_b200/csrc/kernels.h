@@ -188,6 +188,8 @@ struct SimtGemmArgs {
   const int32_t* K_dev;        // if set, K = *K_dev (<= K)
   // optional row routing: row m goes to out_base[out_rank[m]] + out_row[m] * ldc
   float* const* out_base; const int32_t* out_rank; const int32_t* out_row;
+  // optional bf16 output instead of C (tensor-core path only; the hidden activations, R11)
+  uint16_t* Cb; int64_t ldcb;
 };
 cudaError_t launch_simt_gemm(const SimtGemmArgs& a, cudaStream_t st);
 // gemm_tc_gen.cu: the same contract on tcgen05 (fp32: 3xTF32 on kind::tf32; bf16:

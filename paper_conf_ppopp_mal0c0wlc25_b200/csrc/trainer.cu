@@ -659,6 +659,15 @@ void activate(apt_trainer* t, int q) {
   t->parity = q;
 }
 
+// Where the next step's sampling branch forks off the step (A/B, DESIGN §8): 0 at the
+// step's start (default), 1 after the layer-1 forward (the gather+aggregate then runs
+// alone: 34.6 -> 33.4 us, but the sampling lands on the critical path: step 0.231 -> 0.241 ms),
+// 2 after the layer-1 gather (before its projection).
+static int sample_fork_point() {
+  static const int v = [] { const char* e = std::getenv("APT_SAMPLE_FORK"); return e ? atoi(e) : 0; }();
+  return v;
+}
+
 // The layer-1 gather+mean of sample set q of one rank (local + peer rows) into the
 // set's Z, on stream st; time_it: bracketed by the phase events 6 / 7 (on st).
 apt_status agg_l1_set(apt_trainer* t, RankState& rs, int q, cudaStream_t st, bool time_it) {
@@ -704,6 +713,13 @@ apt_status layer1_fwd_gdp(apt_trainer* t, RankState& rs, bool time_it) {
   Layer& L = rs.L[0];
   if (!t->z_ready) {
     apt_status s = agg_l1_set(t, rs, t->parity, t->ctx->stream, time_it);
+    if (s != APT_OK) return s;
+  }
+  if (t->deferred_fork && sample_fork_point() == 2 && &rs == &t->R.back()) {
+    // the next step's sampling forks after the layer-1 gather (the gather runs alone)
+    std::function<apt_status()> f = std::move(t->deferred_fork);
+    t->deferred_fork = nullptr;
+    apt_status s = f();
     if (s != APT_OK) return s;
   }
   return project(t, L, L.Zb, L.Zf, L.zb_pitch, L.zf_pitch, L.n_rows, L.max_rows, L.d_in, L.W, L.Wb, L.b,
@@ -887,18 +903,10 @@ apt_status step_body(apt_trainer* t, int update, bool host_batch, int q = 0) {
 
 // Pipelined step: compute on set p while the next step (id `next` is the value of the
 // set_step node, patched per replay) is sampled into set p^1 on the sampling stream.
-// Where the next step's sampling branch forks off the step (A/B, DESIGN §8): 0 at the
-// step's start (default), 1 after the layer-1 forward (the gather+aggregate then runs
-// alone: 34.6 -> 33.4 us, but the sampling lands on the critical path: step 0.231 -> 0.241 ms).
-static int sample_fork_point() {
-  static const int v = [] { const char* e = std::getenv("APT_SAMPLE_FORK"); return e ? atoi(e) : 0; }();
-  return v;
-}
-
 // Run the next-step sampling fork now, or leave it for compute_body to launch right
 // after the layer-1 forward.
 static apt_status fork_or_defer(apt_trainer* t, std::function<apt_status()> fork) {
-  if (sample_fork_point() == 1) {
+  if (sample_fork_point() != 0 && (sample_fork_point() == 1 || (!t->gat_heads && (t->world == 1 || t->s == APT_GDP)))) {
     t->deferred_fork = std::move(fork);
     return APT_OK;
   }
