@@ -139,3 +139,58 @@ def test_products_epoch_permutation_full_train(A, products):
         assert np.array_equal(tr.read("seeds")[:, 0], perm[s * cfg.batch:(s + 1) * cfg.batch]), s
     tr.close()
     ctx.close()
+
+
+@pytest.mark.parametrize("strategy,C", [("NFP", 2), ("SNP", 2), ("DNP", 2), ("SNP", 4), ("DNP", 4), ("GDP", 4)])
+def test_products_strategies_match_oracle(A, products, strategy, C):
+    """Every strategy at the benchmark's scale (products shape, 3 layers, B = 1024 per rank,
+    bf16, CUDA graph + pipelined sampling) with C ranks emulated on this B200: every rank's
+    every-layer H, the loss and every all-reduced dW / db against the oracle's per-rank fp64
+    model (the strategies compute the same function), within the derived
+    bounds (T1-T3)."""
+    from oracle import strategy as S
+    from parity_util import sum_bounds
+    cfg, g, train, labels = products
+    torch.cuda.set_device(0)
+    stream = torch.cuda.Stream(priority=-1)
+    ctx = A.Ctx(-1, C, 0, stream.cuda_stream)
+    part = aptgen.partition(g.n, C)
+    gr = ctx.graph_load(g.indptr, g.indices, part)
+    fs = ctx.fstore_create(gr, A.NFP if strategy == "NFP" else A.GDP, A.BF16, cfg.dim, None, cfg.feat_seed)
+    dims = [cfg.dim] + [d for _, d in cfg.dims()]
+    tr = A.Trainer(ctx, gr, fs, dims, cfg.fanouts, cfg.batch, A.BF16, LR, cfg.sample_seed, cfg.feat_seed,
+                   A.STRATEGY[strategy], labels)
+    params = aptgen.weights(cfg)
+    tr.set_params(params)
+    tr.set_epoch(train, 0)
+    tr.use_graph(True)
+    tr.step(0, update=False)
+    step = 1
+    tr.step(step, update=False)
+    perm = oracle.epoch_perm(train, cfg.sample_seed, 0)
+    gb = oracle.global_batch(perm, step, C, cfg.batch)
+    seeds = S.assign_seeds(strategy, gb, part, C, cfg.batch)
+    p64 = [(W.astype(np.float64), b.astype(np.float64)) for W, b in params]
+    K = len(cfg.fanouts)
+    refs, bds = [], []
+    for r in range(C):
+        assert np.array_equal(tr.read("seeds", rank=r)[:, 0], seeds[r])
+        blocks = oracle.sample_blocks(g, seeds[r], cfg.fanouts, cfg.sample_seed, step)
+        ref = model.train_step(blocks, cfg.feat_seed, cfg.dim, p64, labels[seeds[r]], len(gb), "bf16",
+                               snp=(part, C) if strategy == "SNP" else None)
+        ref, bd = reconcile(blocks, p64, ref, "bf16", len(gb), [tr.read("H", l, rank=r) for l in range(1, K)])
+        refs.append(ref)
+        bds.append(bd)
+        for l in range(1, K + 1):
+            assert_close(tr.read("H", l, rank=r), ref["cache"]["h"][l - 1], "bf16", f"H{l} rank {r}", bd["H"][l - 1])
+    loss = sum(x["loss"] for x in refs)
+    assert abs(tr.loss() - loss) <= 2e-2 * abs(loss)
+    sb = sum_bounds(bds)
+    for l in range(1, K + 1):
+        for r in (0, C - 1):
+            assert_close(tr.read("dW", l, rank=r), sum(x["grads"][l - 1][0] for x in refs), "bf16",
+                         f"dW{l} rank {r}", sb["dW"][l - 1])
+            assert_close(tr.read("db", l, rank=r)[0], sum(x["grads"][l - 1][1] for x in refs), "bf16",
+                         f"db{l} rank {r}", sb["db"][l - 1])
+    tr.close()
+    ctx.close()
