@@ -319,6 +319,15 @@ apt_status apt_trainer_step_host(apt_trainer* t, const int64_t* gbatch_host, int
  * primes (*had_step = 0).  Syncs.                                           */
 apt_status apt_trainer_step_host_pipelined(apt_trainer* t, const int64_t* next_batch, int64_t n_next,
                                            int64_t next_step, int update, float* loss_prev, int* had_step);
+/* The same pipelined end-to-end call without waiting for the step it launches: it
+ * writes the next batch into pinned staging, launches this call's step (H2D of the next
+ * batch, the step, D2H of its loss) and then waits only for the step the PREVIOUS call
+ * launched, returning that step's loss (*had_step = 0 on the first two calls) -- the
+ * device always has the next step queued while the host prepares the next call.  Use
+ * apt_trainer_loss (syncs) for the last step's loss.  Device error words surface at the
+ * next synchronising call.                                                          */
+apt_status apt_trainer_step_host_async(apt_trainer* t, const int64_t* next_batch, int64_t n_next, int64_t next_step,
+                                       int update, float* loss_prev, int* had_step);
 /* Loss of the last step (sum over ranks).  Syncs.                           */
 apt_status apt_trainer_loss(apt_trainer* t, float* loss);
 /* Record/replay the device part of apt_trainer_step as a CUDA graph.        */

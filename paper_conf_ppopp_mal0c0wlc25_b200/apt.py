@@ -116,6 +116,7 @@ def lib():
             "apt_trainer_set_epoch": [vp, vp, i64, u64], "apt_trainer_step": [vp, i64, i32],
             "apt_trainer_step_host": [vp, vp, i64, i64, i32, vp], "apt_trainer_loss": [vp, vp],
             "apt_trainer_step_host_pipelined": [vp, vp, i64, i64, i32, vp, vp],
+            "apt_trainer_step_host_async": [vp, vp, i64, i64, i32, vp, vp],
             "apt_trainer_use_graph": [vp, i32], "apt_trainer_set_pipeline": [vp, i32], "apt_trainer_read": [vp, i32, i32, i32, vp, i64, vp, vp],
             "apt_trainer_phase_ms": [vp, vp, i32], "apt_trainer_agg_bytes": [vp, vp],
             "apt_partition": [i64, i64, vp, vp, i32, i32, u64, vp, vp],
@@ -396,6 +397,14 @@ class Trainer(Handle):
         self.ctx.ck(lib().apt_trainer_step_host_pipelined(self.h, _ptr(next_batch_host), len(next_batch_host),
                                                           next_step, 1 if update else 0, C.byref(loss),
                                                           C.byref(had)))
+        return loss.value if had.value else None
+
+    def step_host_async(self, next_batch_host, next_step, update=True):
+        """Submit the next host batch and launch the previously submitted one without waiting
+        for it; returns the loss of the step the previous call launched (None at first)."""
+        loss, had = C.c_float(0), C.c_int(0)
+        self.ctx.ck(lib().apt_trainer_step_host_async(self.h, _ptr(next_batch_host), len(next_batch_host), next_step,
+                                                      1 if update else 0, C.byref(loss), C.byref(had)))
         return loss.value if had.value else None
 
     def loss(self):

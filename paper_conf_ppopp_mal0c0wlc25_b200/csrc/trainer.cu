@@ -288,7 +288,8 @@ apt_status apt::trainer_create(apt_ctx* c, const apt_graph* g, const apt_fstore*
   t->hb_len = 1 + int64_t(C) * m->batch;
   t->hb_dev = A.alloc<int32_t>(2 * t->hb_len, true);
   CK(c, cudaMallocHost(reinterpret_cast<void**>(&t->hb_pinned), sizeof(int32_t) * 2 * t->hb_len));
-  CK(c, cudaMallocHost(reinterpret_cast<void**>(&t->loss_pinned), sizeof(float) * APT_MAX_RANKS));
+  CK(c, cudaMallocHost(reinterpret_cast<void**>(&t->loss_pinned), sizeof(float) * 2 * APT_MAX_RANKS));
+  for (int q = 0; q < 2; ++q) CK(c, cudaEventCreateWithFlags(&t->ev_done[q], cudaEventDisableTiming));
   if (labels) CK(c, cudaMemcpyAsync(t->labels, labels, sizeof(int32_t) * g->n, cudaMemcpyHostToDevice, c->stream));
   const int64_t n_words = ceil_div(g->n, 32);
   // upper bounds per hop.  SNP/DNP seeds follow the partition: up to C*B on one rank.
@@ -461,6 +462,8 @@ apt_status apt_trainer_destroy(apt_trainer* t) {
   if (t->graph_host) cudaGraphDestroy(t->graph_host);
   if (t->hb_pinned) cudaFreeHost(t->hb_pinned);
   if (t->loss_pinned) cudaFreeHost(t->loss_pinned);
+  for (int q = 0; q < 2; ++q)
+    if (t->ev_done[q]) cudaEventDestroy(t->ev_done[q]);
   for (int i = 0; i < 8; ++i)
     if (t->ev[i]) cudaEventDestroy(t->ev[i]);
   apt_ctx* c = t->ctx;
@@ -1372,8 +1375,8 @@ apt_status apt_trainer_step_host(apt_trainer* t, const int64_t* gbatch, int64_t 
 // step's loss.  While the step computes, the next batch is copied in and sampled on
 // the sampling stream (one graph replay per call).  The first call only primes (loss
 // NaN, *had_step = 0).
-apt_status apt_trainer_step_host_pipelined(apt_trainer* t, const int64_t* next_batch, int64_t n_next, int64_t next_step,
-                                           int update, float* loss_prev, int* had_step) {
+static apt_status step_host_pipelined_impl(apt_trainer* t, const int64_t* next_batch, int64_t n_next, int64_t next_step,
+                                           int update, float* loss_prev, int* had_step, bool async) {
   if (!t || !next_batch || !loss_prev || !had_step || n_next < 1 || n_next > int64_t(t->world) * t->m.batch)
     return set_err(t ? t->ctx : nullptr, APT_E_INVALID, "apt_trainer_step_host_pipelined: bad arguments");
   apt_ctx* c = t->ctx;
@@ -1391,6 +1394,7 @@ apt_status apt_trainer_step_host_pipelined(apt_trainer* t, const int64_t* next_b
   }
   const size_t hb_bytes = sizeof(int32_t) * size_t(t->hb_len);
   if (!t->host_primed) {   // prime: copy in and sample the first batch into set 0
+    t->async_pending = false;
     CK(c, cudaMemcpyAsync(t->hb_dev, stage, hb_bytes, cudaMemcpyHostToDevice, c->stream));
     set_step_kernel<<<1, 1, 0, c->stream>>>(t->step_cells, uint64_t(next_step));
     CK(c, cudaGetLastError());
@@ -1427,7 +1431,8 @@ apt_status apt_trainer_step_host_pipelined(apt_trainer* t, const int64_t* next_b
     t->z_ready = false;
     if (s != APT_OK) return s;
     for (size_t i = 0; i < t->R.size(); ++i)
-      CK(c, cudaMemcpyAsync(t->loss_pinned + i, t->R[i].loss, sizeof(float), cudaMemcpyDeviceToHost, c->stream));
+      CK(c, cudaMemcpyAsync(t->loss_pinned + p * APT_MAX_RANKS + i, t->R[i].loss, sizeof(float),
+                            cudaMemcpyDeviceToHost, c->stream));
     CK(c, cudaStreamWaitEvent(c->stream, c->ev_pjoin, 0));
     return APT_OK;
   };
@@ -1458,13 +1463,40 @@ apt_status apt_trainer_step_host_pipelined(apt_trainer* t, const int64_t* next_b
     if (s != APT_OK) return s;
     c->launches++;
   }
+  t->host_parity = q;
+  if (async) {
+    // the step just launched keeps the device busy while the host returns the loss of the
+    // step the PREVIOUS call launched (its loss slot is the other parity)
+    CK(c, cudaEventRecord(t->ev_done[p], c->stream));
+    *had_step = 0;
+    if (t->async_pending) {
+      CK(c, cudaEventSynchronize(t->ev_done[p ^ 1]));
+      float tot = 0.f;
+      for (size_t i = 0; i < t->R.size(); ++i) tot += t->loss_pinned[(p ^ 1) * APT_MAX_RANKS + i];
+      *loss_prev = tot;
+      *had_step = 1;
+    }
+    t->async_pending = true;
+    CK(c, cudaGetLastError());
+    return APT_OK;
+  }
+  t->async_pending = false;
   CK(c, cudaStreamSynchronize(c->stream));
   float tot = 0.f;
-  for (size_t i = 0; i < t->R.size(); ++i) tot += t->loss_pinned[i];
+  for (size_t i = 0; i < t->R.size(); ++i) tot += t->loss_pinned[p * APT_MAX_RANKS + i];
   *loss_prev = tot;
   *had_step = 1;
-  t->host_parity = q;
   return apt_ctx_sync(c);
+}
+
+apt_status apt_trainer_step_host_pipelined(apt_trainer* t, const int64_t* next_batch, int64_t n_next, int64_t next_step,
+                                           int update, float* loss_prev, int* had_step) {
+  return step_host_pipelined_impl(t, next_batch, n_next, next_step, update, loss_prev, had_step, false);
+}
+
+apt_status apt_trainer_step_host_async(apt_trainer* t, const int64_t* next_batch, int64_t n_next, int64_t next_step,
+                                       int update, float* loss_prev, int* had_step) {
+  return step_host_pipelined_impl(t, next_batch, n_next, next_step, update, loss_prev, had_step, true);
 }
 
 apt_status apt_trainer_loss(apt_trainer* t, float* loss) {

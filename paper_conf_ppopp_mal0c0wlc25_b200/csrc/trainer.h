@@ -211,7 +211,9 @@ struct apt_trainer {
   cudaGraph_t graph_hp[2][2] = {};
   cudaGraphNode_t step_node_hp[2][2] = {};
   int64_t launches_hp[2][2] = {};
-  float* loss_pinned = nullptr;       // [APT_MAX_RANKS] per hosted rank
+  float* loss_pinned = nullptr;       // [2][APT_MAX_RANKS] per sample-set parity, per hosted rank
+  cudaEvent_t ev_done[2] = {};        // end of the step graph of each parity (async end-to-end calls)
+  bool async_pending = false;         // an async call launched a step whose loss is not yet returned
   cudaGraph_t graph = nullptr;
   cudaGraphNode_t step_node = nullptr;
   int64_t launches_per_step = 0;

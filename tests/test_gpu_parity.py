@@ -310,6 +310,32 @@ def test_step_host_pipelined_matches_device_steps(A, ctx, tiny, use_graph):
     assert np.allclose(got, ref, rtol=1e-6)
 
 
+@pytest.mark.parametrize("use_graph", [False, True])
+def test_step_host_async_matches_device_steps(A, ctx, tiny, use_graph):
+    """The asynchronous end-to-end call returns, one call late, the losses of the
+    device-resident steps on the same batches (and the last one via apt_trainer_loss)."""
+    cfg, g, train = tiny
+    perm = oracle.epoch_perm(train, cfg.sample_seed, 0)
+    tr, params, labels = _trainer(A, ctx, cfg, g, train, "bf16")
+    tr.use_graph(use_graph)
+    ref = []
+    for step in range(4):
+        tr.step(step % 3, update=False)
+        ref.append(tr.loss())
+    tr2, _, _ = _trainer(A, ctx, cfg, g, train, "bf16")
+    tr2.use_graph(use_graph)
+    got = []
+    for call in range(5):
+        nxt = torch.as_tensor(perm[(call % 3) * cfg.batch:((call % 3) + 1) * cfg.batch]).pin_memory()
+        loss = tr2.step_host_async(nxt, call % 3, update=False)
+        if call < 2:
+            assert loss is None
+        else:
+            got.append(loss)
+    got.append(tr2.loss())             # the last launched step (batch 3 % 3)
+    assert np.allclose(got, ref, rtol=1e-6), (got, ref)
+
+
 @pytest.mark.parametrize("strategy,C", [("GDP", 1), ("SNP", 2), ("NFP", 2), ("DNP", 2)])
 def test_pipelined_steps_equal_unpipelined(A, tiny, strategy, C):
     """Sampling step t+1 during step t (two sample sets, second stream) changes nothing:
