@@ -384,7 +384,7 @@ def run_apt(args, cfg):
     # with the pipeline (GDP, SAGE) the layer-1 gather+mean timed inside step i belongs to
     # the NEXT batch (the sampling branch aggregates it, trainer z_prefetch): pair its time
     # with the bytes of step i+1 (consecutive steps only)
-    if not args.no_pipeline and not GAT_HEADS and args.strategy == "GDP" and os.environ.get("APT_Z_PREFETCH", "0") == "1":
+    if not args.no_pipeline and not GAT_HEADS and args.strategy == "GDP" and os.environ.get("APT_Z_PREFETCH", "0") != "0":
         pairs = [(agg_ms[i], agg_bytes[i + 1]) for i in range(len(agg_ms) - 1) if step_ids[i + 1] == step_ids[i] + 1]
         agg_ms, agg_bytes = [p_[0] for p_ in pairs], [p_[1] for p_ in pairs]
     achieved = sum(agg_bytes) / (sum(agg_ms) * 1e-3) / 1e9

@@ -440,6 +440,9 @@ apt_status apt::trainer_create(apt_ctx* c, const apt_graph* g, const apt_fstore*
     // (pull / wgrad: 60 -> 92 us) and its own in-step time rises 30 -> 43 us
     const char* zp = std::getenv("APT_Z_PREFETCH");
     t->z_prefetch = (zp && atoi(zp) != 0) && !t->gat_heads && (C == 1 || s == APT_GDP);
+    t->z_where = zp ? std::max(1, atoi(zp)) : 1;
+    CK(c, cudaEventCreateWithFlags(&t->ev_zt, cudaEventDisableTiming));
+    CK(c, cudaEventCreateWithFlags(&t->ev_zf, cudaEventDisableTiming));
   }
   CK(c, cudaStreamSynchronize(c->stream));
   *out = t;
@@ -462,6 +465,8 @@ apt_status apt_trainer_destroy(apt_trainer* t) {
   if (t->graph_host) cudaGraphDestroy(t->graph_host);
   if (t->hb_pinned) cudaFreeHost(t->hb_pinned);
   if (t->loss_pinned) cudaFreeHost(t->loss_pinned);
+  if (t->ev_zt) cudaEventDestroy(t->ev_zt);
+  if (t->ev_zf) cudaEventDestroy(t->ev_zf);
   for (int q = 0; q < 2; ++q)
     if (t->ev_done[q]) cudaEventDestroy(t->ev_done[q]);
   for (int i = 0; i < 8; ++i)
@@ -926,7 +931,7 @@ apt_status pipelined_body(apt_trainer* t, int p, int update, uint64_t next) {
     CK(c, cudaGetLastError());
     c->launches++;
     apt_status s2 = sample_all(t, p ^ 1, false, c->samp, false);
-    if (s2 == APT_OK && t->z_prefetch) s2 = prefetch_z(t, p ^ 1, c->samp);   // next batch's layer-1 Z
+    if (s2 == APT_OK && t->z_prefetch && t->z_where == 1) s2 = prefetch_z(t, p ^ 1, c->samp);   // next batch's layer-1 Z
     if (s2 != APT_OK) return s2;
     CK(c, cudaEventRecord(c->ev_pjoin, c->samp));
     return APT_OK;
@@ -935,8 +940,10 @@ apt_status pipelined_body(apt_trainer* t, int p, int update, uint64_t next) {
   t->csc_forked = false;
   activate(t, p);
   t->z_ready = t->z_prefetch;   // this batch's Z was aggregated by the previous step's branch (or the prime)
+  t->z_next = (t->z_prefetch && t->z_where == 2) ? (p ^ 1) : -1;
   s = compute_body(t, update);
   t->z_ready = false;
+  t->z_next = -1;
   if (s != APT_OK) return s;
   CK(c, cudaStreamWaitEvent(c->stream, c->ev_pjoin, 0));   // next step's batch complete
   return APT_OK;
@@ -980,6 +987,16 @@ apt_status compute_body(apt_trainer* t, int update) {
     apt_status s = upper_bwd(t, rs);
     if (s != APT_OK) return s;
   }
+  if (t->z_next >= 0) {
+    // the next batch's layer-1 gather+mean beside this step's tail (weight gradient of
+    // layer 1, SGD): it needs the next batch's sampling (ev_pjoin) and nothing of this step
+    CK(c, cudaEventRecord(t->ev_zt, c->stream));
+    CK(c, cudaStreamWaitEvent(c->samp, t->ev_zt, 0));
+    CK(c, cudaStreamWaitEvent(c->samp, c->ev_pjoin, 0));
+    apt_status s = prefetch_z(t, t->z_next, c->samp);
+    if (s != APT_OK) return s;
+    CK(c, cudaEventRecord(t->ev_zf, c->samp));
+  }
   if (t->gat_heads) {
     apt_status s = gat_layer1_bwd(t);
     if (s != APT_OK) return s;
@@ -999,6 +1016,7 @@ apt_status compute_body(apt_trainer* t, int update) {
   CK(c, record_ev(t, 4));
   apt_status s = allreduce_sgd(t, update);
   if (s != APT_OK) return s;
+  if (t->z_next >= 0) CK(c, cudaStreamWaitEvent(c->stream, t->ev_zf, 0));   // the next step's Z is ready
   CK(c, record_ev(t, 5));
   t->ev_ok = true;
   return APT_OK;
@@ -1418,7 +1436,7 @@ static apt_status step_host_pipelined_impl(apt_trainer* t, const int64_t* next_b
       set_step_kernel<<<1, 1, 0, c->samp>>>(t->step_cells + q, nstep);
       CK(c, cudaGetLastError());
       apt_status s2 = sample_all(t, q, true, c->samp, false);
-      if (s2 == APT_OK && t->z_prefetch) s2 = prefetch_z(t, q, c->samp);
+      if (s2 == APT_OK && t->z_prefetch && t->z_where == 1) s2 = prefetch_z(t, q, c->samp);
       if (s2 != APT_OK) return s2;
       CK(c, cudaEventRecord(c->ev_pjoin, c->samp));
       return APT_OK;
@@ -1427,8 +1445,10 @@ static apt_status step_host_pipelined_impl(apt_trainer* t, const int64_t* next_b
     t->csc_forked = false;
     activate(t, p);
     t->z_ready = t->z_prefetch;
+    t->z_next = (t->z_prefetch && t->z_where == 2) ? q : -1;
     s = compute_body(t, update);
     t->z_ready = false;
+    t->z_next = -1;
     if (s != APT_OK) return s;
     for (size_t i = 0; i < t->R.size(); ++i)
       CK(c, cudaMemcpyAsync(t->loss_pinned + p * APT_MAX_RANKS + i, t->R[i].loss, sizeof(float),

@@ -186,6 +186,9 @@ struct apt_trainer {
   bool z_prefetch = false;           // GDP SAGE layer 1: the next batch's gather+mean runs on the sampling
                                      //   branch (it reads only the static features), beside this step
   bool z_ready = false;              // the active set's layer-1 Z is already aggregated
+  int z_where = 1;                   // z_prefetch: 1 on the sampling branch, 2 beside this step's backward tail
+  int z_next = -1;                   // z_where 2: the set whose Z this step aggregates (pipelined bodies)
+  cudaEvent_t ev_zt = nullptr, ev_zf = nullptr;   // tail prefetch: fork point / done
   int parity = 0;                    // sample set the last step computed on
   int64_t primed = -1;               // step id already sampled into sset[primed_parity]
   int primed_parity = 0;
