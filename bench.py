@@ -391,7 +391,7 @@ def run_apt(args, cfg):
     # DRAM traffic of the same kernel from one committed `ncu --set full` capture of this
     # workload (dram__bytes_read + dram__bytes_write per launch), next to the algorithmic bytes
     traffic, traffic_src = None, None
-    tpath = os.path.join(ROOT, "profiles", "r01_ncu_agg_l1_traffic.json")
+    tpath = os.path.join(ROOT, "profiles", "r02_ncu_agg_l1_traffic.json")
     if not GAT_HEADS and args.dtype == "bf16" and cfg.name == "products" and cfg.fanouts == (10, 10, 10) \
             and os.path.exists(tpath):
         tj = json.load(open(tpath))
