@@ -311,6 +311,14 @@ __global__ void __launch_bounds__(256, 2) gat_bwd_kernel(GatKArgs a) {
   const int64_t n = *a.it.n;
   const int k = a.it.k;
   const int64_t nwarps = int64_t(gridDim.x) * (blockDim.x >> 5);
+  // d w~_src accumulates in registers over every item the lane touches (the lane always
+  // owns the same feature columns) and reaches shared memory once per warp at the end;
+  // the destination term (one row per item) is combined across the two half-warps first
+  float dws[H][EPV];
+#pragma unroll
+  for (int h = 0; h < H; ++h)
+#pragma unroll
+    for (int q = 0; q < EPV; ++q) dws[h][q] = 0.f;
   for (int64_t w = (int64_t(blockIdx.x) * blockDim.x + threadIdx.x) >> 5; w * RPW < n; w += nwarps) {
     const int64_t i = w * RPW + sub;
     const bool valid = i < n;
@@ -320,14 +328,13 @@ __global__ void __launch_bounds__(256, 2) gat_bwd_kernel(GatKArgs a) {
     const int v = valid ? a.it.gid[i] : 0;
     const int row = valid ? (a.it.row ? a.it.row[i] : int(i)) : 0;
     const int rk = valid ? (a.it.rank ? a.it.rank[i] : a.it.self) : 0;
-    float gm[H][EPV], t[H], Lv[H], der[H], dws[H][EPV];
+    float gm[H][EPV], t[H], Lv[H], der[H];
 #pragma unroll
     for (int h = 0; h < H; ++h) {
 #pragma unroll
       for (int q = 0; q < EPV; ++q) {
         const int c = l * EPV + q;
         gm[h][q] = (valid && a.mode != 2 && l < V && c < a.cols) ? a.gam[(i * H + h) * a.gp + c] : 0.f;
-        dws[h][q] = 0.f;
       }
       t[h] = valid ? a.tb[i * H + h] : 0.f;
       Lv[h] = valid ? a.Lb[i * H + h] : 0.f;
@@ -407,18 +414,27 @@ __global__ void __launch_bounds__(256, 2) gat_bwd_kernel(GatKArgs a) {
         }
       }
     }
-    if (!valid || a.mode == 1) continue;
+    if (a.mode == 1) continue;                                   // uniform
     float xv[EPV];
-    unpack<EPV>(ld_nc_v4(gat_row(a, v) + lv * 16), xv);
-    if (l < V) {
+    unpack<EPV>(valid ? ld_nc_v4(gat_row(a, v) + lv * 16) : make_uint4(0, 0, 0, 0), xv);
 #pragma unroll
-      for (int h = 0; h < H; ++h)
+    for (int h = 0; h < H; ++h)
 #pragma unroll
-        for (int q = 0; q < EPV; ++q) {
-          atomicAdd(&sdw[h * a.cpad + l * EPV + q], dws[h][q]);
-          atomicAdd(&sdw[(H + h) * a.cpad + l * EPV + q], der[h] * xv[q]);
-        }
-    }
+      for (int q = 0; q < EPV; ++q) {
+        float dd = valid ? der[h] * xv[q] : 0.f;
+        if (LG == 16) dd += __shfl_xor_sync(0xffffffffu, dd, 16);   // the warp's two items, same columns
+        if (sub == 0 && l < V && dd != 0.f) atomicAdd(&sdw[(H + h) * a.cpad + l * EPV + q], dd);
+      }
+  }
+  if (a.mode != 1) {
+#pragma unroll
+    for (int h = 0; h < H; ++h)
+#pragma unroll
+      for (int q = 0; q < EPV; ++q) {
+        float v = dws[h][q];
+        if (LG == 16) v += __shfl_xor_sync(0xffffffffu, v, 16);
+        if (sub == 0 && l < V && v != 0.f) atomicAdd(&sdw[h * a.cpad + l * EPV + q], v);
+      }
   }
   __syncthreads();
   if (a.mode == 1) return;
@@ -435,10 +451,20 @@ __global__ void gat_wt_kernel(const float* __restrict__ W, int64_t ldw, const fl
   const int total = 2 * H * cols;
   for (int t = blockIdx.x * blockDim.x + threadIdx.x; t < total; t += gridDim.x * blockDim.x) {
     const int c = t % cols, h = (t / cols) % H, which = t / (cols * H);
-    const float* a = which ? ad : as;
-    float s = 0.f;
-    for (int f = 0; f < F; ++f) s = fmaf(a[h * F + f], W[int64_t(h * F + f) * ldw + c], s);
-    wt[t] = s;
+    const float* __restrict__ a = (which ? ad : as) + h * F;
+    const float* __restrict__ w = W + int64_t(h * F) * ldw + c;
+    // independent partial sums: the F row loads of W are in flight together (a chain of
+    // F dependent FMAs made this tiny kernel a 20-us latency chain)
+    float s0 = 0.f, s1 = 0.f, s2 = 0.f, s3 = 0.f;
+    int f = 0;
+    for (; f + 4 <= F; f += 4) {
+      s0 = fmaf(__ldg(a + f), __ldg(w + int64_t(f) * ldw), s0);
+      s1 = fmaf(__ldg(a + f + 1), __ldg(w + int64_t(f + 1) * ldw), s1);
+      s2 = fmaf(__ldg(a + f + 2), __ldg(w + int64_t(f + 2) * ldw), s2);
+      s3 = fmaf(__ldg(a + f + 3), __ldg(w + int64_t(f + 3) * ldw), s3);
+    }
+    for (; f < F; ++f) s0 = fmaf(__ldg(a + f), __ldg(w + int64_t(f) * ldw), s0);
+    wt[t] = (s0 + s1) + (s2 + s3);
   }
 }
 
@@ -489,6 +515,37 @@ __global__ void gat_t_kernel(const T* __restrict__ g, int64_t gp, const float* _
   const int64_t n = *n_p;
   const int lane = lane_id();
   const int64_t nw = int64_t(gridDim.x) * (blockDim.x >> 5);
+  if constexpr (sizeof(T) == 2) {
+    if (F % 8 == 0 && gp % 8 == 0 && hp % 4 == 0 && H <= 8) {
+      // 8 columns of one head per lane and chunk: 16-byte g loads, 2 x 16-byte h loads
+      const int nv = H * F / 8;
+      for (int64_t r = (int64_t(blockIdx.x) * blockDim.x + threadIdx.x) >> 5; r < n; r += nw) {
+        float s[8] = {0.f, 0.f, 0.f, 0.f, 0.f, 0.f, 0.f, 0.f};
+        for (int v = lane; v < nv; v += 32) {
+          const int c = v * 8, h = c / F;
+          const uint4 gr = *reinterpret_cast<const uint4*>(g + r * gp + c);
+          const float4 h0 = *reinterpret_cast<const float4*>(h1 + r * hp + c);
+          const float4 h4 = *reinterpret_cast<const float4*>(h1 + r * hp + c + 4);
+          const float4 b0 = *reinterpret_cast<const float4*>(b + c);
+          const float4 b4 = *reinterpret_cast<const float4*>(b + c + 4);
+          float acc = 0.f;
+          acc = fmaf(bf16_lo(gr.x), h0.x - b0.x, acc); acc = fmaf(bf16_hi(gr.x), h0.y - b0.y, acc);
+          acc = fmaf(bf16_lo(gr.y), h0.z - b0.z, acc); acc = fmaf(bf16_hi(gr.y), h0.w - b0.w, acc);
+          acc = fmaf(bf16_lo(gr.z), h4.x - b4.x, acc); acc = fmaf(bf16_hi(gr.z), h4.y - b4.y, acc);
+          acc = fmaf(bf16_lo(gr.w), h4.z - b4.z, acc); acc = fmaf(bf16_hi(gr.w), h4.w - b4.w, acc);
+#pragma unroll
+          for (int q = 0; q < 8; ++q) if (q == h) s[q] += acc;
+        }
+#pragma unroll
+        for (int q = 0; q < 8; ++q) {
+          if (q >= H) break;
+          const float tot = warp_sum(s[q]);
+          if (lane == 0) t[r * H + q] = tot;
+        }
+      }
+      return;
+    }
+  }
   for (int64_t r = (int64_t(blockIdx.x) * blockDim.x + threadIdx.x) >> 5; r < n; r += nw) {   // warp per row
     for (int h = 0; h < H; ++h) {
       float s = 0.f;
@@ -520,6 +577,42 @@ __global__ void gat_gather_kernel(T* const* __restrict__ gtab, int64_t gp, float
   const int64_t n = *it.n;
   const int64_t rows = sizeof(T) == 2 ? std::min<int64_t>(icap, round_up(n, 64)) : n;
   const int d_out = H * F;
+  if constexpr (sizeof(T) == 2) {
+    if (F % 8 == 0 && gp % 8 == 0 && wpb % 8 == 0) {
+      // bf16 rows in 16-byte vectors (8 columns of one head per thread)
+      const int nv = d_out / 8;
+      for (int64_t x = int64_t(blockIdx.x) * blockDim.x + threadIdx.x; x < rows * nv; x += int64_t(gridDim.x) * blockDim.x) {
+        const int64_t i = x / nv;
+        const int c = int(x - i * nv) * 8;
+        uint4* dst = reinterpret_cast<uint4*>(wGb + i * wpb + c);
+        uint4* dsts = snp ? reinterpret_cast<uint4*>(wGsb + i * wpb + c) : nullptr;
+        if (i >= n) {
+          *dst = make_uint4(0, 0, 0, 0);
+          if (dsts) *dsts = make_uint4(0, 0, 0, 0);
+          continue;
+        }
+        const int h = c / F;
+        const int rk = it.rank ? it.rank[i] : it.self;
+        const int row = it.row ? it.row[i] : int(i);
+        const uint4 graw = *reinterpret_cast<const uint4*>(gtab[rk] + int64_t(row) * gp + c);
+        *dst = graw;
+        const float L = snp ? Ltab[rk][int64_t(row) * H + h] : Lm[i * H + h];
+        if (dsts) {
+          const float om = Ss[i * H + h] > 0.f ? Ss[i * H + h] * expf(Lm[i * H + h] - L) : 0.f;
+          const uint32_t w4[4] = {graw.x, graw.y, graw.z, graw.w};
+          uint32_t o4[4];
+#pragma unroll
+          for (int q = 0; q < 4; ++q) o4[q] = pack_bf16x2(bf16_lo(w4[q]) * om, bf16_hi(w4[q]) * om);
+          *dsts = make_uint4(o4[0], o4[1], o4[2], o4[3]);
+        }
+        if (c % F == 0) {
+          tb[i * H + h] = ttab[rk][int64_t(row) * H + h];
+          Lb[i * H + h] = L;
+        }
+      }
+      return;
+    }
+  }
   for (int64_t x = int64_t(blockIdx.x) * blockDim.x + threadIdx.x; x < rows * d_out; x += int64_t(gridDim.x) * blockDim.x) {
     const int64_t i = x / d_out;
     const int c = int(x - i * d_out);
