@@ -926,13 +926,11 @@ apt_status gat_layer1_fwd(apt_trainer* t, bool time_it) {
     GatKArgs a = kargs(t, rs);
     a.mode = mode;
     a.tab = t->ssum_tab;
-    if (first && mode != 1) CK(c, t->capturing ? cudaEventRecordWithFlags(t->ev[6], c->stream, cudaEventRecordExternal)
-                                               : cudaEventRecord(t->ev[6], c->stream));
+    if (first && mode != 1) CK(c, tap_event(t, t->ev[6], c->stream));
     apt_status s = launch_gat(t, a, false, rs.ga.icap);
     if (s != APT_OK) return s;
     if (first && mode != 1) {
-      CK(c, t->capturing ? cudaEventRecordWithFlags(t->ev[7], c->stream, cudaEventRecordExternal)
-                         : cudaEventRecord(t->ev[7], c->stream));
+      CK(c, tap_event(t, t->ev[7], c->stream));
       first = false;
     }
     return APT_OK;

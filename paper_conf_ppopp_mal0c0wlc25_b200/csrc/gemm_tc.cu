@@ -70,7 +70,7 @@ struct RowParams {
   int staged;               // force the staged epilogue for plain rows too (APT_EPI_STAGED=1, A/B)
 };
 
-__global__ void __launch_bounds__(ROW_THREADS, 2)
+__global__ void __launch_bounds__(ROW_THREADS, 1)
     rowtile_kernel(const __grid_constant__ CUtensorMap mapA, const __grid_constant__ CUtensorMap mapB, RowParams p) {
   // Programmatic dependent launch: barrier init, TMEM allocation, tensor-map prefetch
   // and (b_early) the resident B load run before griddepcontrol.wait, i.e. while the
@@ -211,71 +211,82 @@ __global__ void __launch_bounds__(ROW_THREADS, 2)
       if (p.row_div && m_own < M) own_deg = float(p.row_div[m_own + 1] - p.row_div[m_own]);
       const float own_rdeg = own_deg > 0.f ? __frcp_rn(own_deg) : 0.f;
       const uint32_t tbase = tmem_base + (uint32_t(q * 32) << 16) + uint32_t(acc * p.BN);
-      uint32_t r[16], rn[16];
-      if (16 * h < p.BN) {
-        tmem_ld16_nowait(tbase + uint32_t(16 * h), r);
-        tmem_wait16(r);
-      }
       if (direct) {
         // Direct path (plain rows: no routing, reduction or mask): the lane owns its row
-        // (its TMEM lane) and writes the chunk's 16 values straight from registers as
-        // whole 32-B sectors -- no staging, shuffles or per-element branches; the
-        // epilogue was instruction-bound (~275 warp instructions per chunk staged)
-        for (int c = 16 * h; c < p.BN; c += 32) {
-          const bool more = c + 32 < p.BN;
-          if (more) tmem_ld16_nowait(tbase + uint32_t(c + 32), rn);
+        // (its TMEM lane) and writes straight from registers -- no staging, shuffles or
+        // per-element branches.  The warp owns a contiguous half of the tile's 16-column
+        // chunks and loads up to four of them (64 columns) before ONE wait, so a lane
+        // writes up to 128 contiguous bytes of its row per group and the TMEM round trip
+        // is paid once per group, not per chunk (ncu: the one-chunk-in-flight loop was
+        // latency-bound at ~10 cycles per issued instruction with 2 warps per scheduler).
+        const int nch = p.BN / 16, half = (nch + 1) / 2;
+        const int cb0 = h * half, cb1 = min(nch, cb0 + half);
+        for (int cb = cb0; cb < cb1; cb += 4) {
+          const int ng = min(4, cb1 - cb);
+          uint32_t r4[4][16];
+#pragma unroll
+          for (int i = 0; i < 4; ++i)
+            if (i < ng) tmem_ld16_nowait(tbase + uint32_t(16 * (cb + i)), r4[i]);
+#pragma unroll
+          for (int i = 0; i < 4; ++i)
+            if (i < ng) tmem_wait16(r4[i]);
           if (own) {
-            float v[16];
 #pragma unroll
-            for (int j = 0; j < 16; j += 4) {
-              const float4 bv = *reinterpret_cast<const float4*>(sbias + c + j);
-              v[j] = __uint_as_float(r[j]) + bv.x; v[j + 1] = __uint_as_float(r[j + 1]) + bv.y;
-              v[j + 2] = __uint_as_float(r[j + 2]) + bv.z; v[j + 3] = __uint_as_float(r[j + 3]) + bv.w;
-            }
-            if (p.relu) {
+            for (int i = 0; i < 4; ++i) {
+              if (i >= ng) break;
+              const int c = 16 * (cb + i);
+              float v[16];
 #pragma unroll
-              for (int j = 0; j < 16; ++j) v[j] = fmaxf(v[j], 0.f);
-            }
-            if (p.row_div && own_deg > 0.f) {
-#pragma unroll
-              for (int j = 0; j < 16; ++j) v[j] = div_rn_rcp(v[j], own_deg, own_rdeg);
-            }
-            const int col = n0 + c;
-            if (p.Yb) {
-              uint16_t* d = reinterpret_cast<uint16_t*>(own) + col;
-              if (col + 16 <= p.N) {
-                reinterpret_cast<uint4*>(d)[0] = make_uint4(pack_bf16x2(v[0], v[1]), pack_bf16x2(v[2], v[3]),
-                                                            pack_bf16x2(v[4], v[5]), pack_bf16x2(v[6], v[7]));
-                reinterpret_cast<uint4*>(d)[1] = make_uint4(pack_bf16x2(v[8], v[9]), pack_bf16x2(v[10], v[11]),
-                                                            pack_bf16x2(v[12], v[13]), pack_bf16x2(v[14], v[15]));
-              } else {
-#pragma unroll
-                for (int j = 0; j < 16; ++j)
-                  if (col + j < p.N) d[j] = bf16_bits(v[j]);
+              for (int j = 0; j < 16; j += 4) {
+                const float4 bv = *reinterpret_cast<const float4*>(sbias + c + j);
+                v[j] = __uint_as_float(r4[i][j]) + bv.x; v[j + 1] = __uint_as_float(r4[i][j + 1]) + bv.y;
+                v[j + 2] = __uint_as_float(r4[i][j + 2]) + bv.z; v[j + 3] = __uint_as_float(r4[i][j + 3]) + bv.w;
               }
-            } else {
-              float* d = own + col;
-              if (col + 16 <= p.N) {
+              if (p.relu) {
 #pragma unroll
-                for (int j = 0; j < 16; j += 4)
-                  *reinterpret_cast<float4*>(d + j) = make_float4(v[j], v[j + 1], v[j + 2], v[j + 3]);
+                for (int j = 0; j < 16; ++j) v[j] = fmaxf(v[j], 0.f);
+              }
+              if (p.row_div && own_deg > 0.f) {
+#pragma unroll
+                for (int j = 0; j < 16; ++j) v[j] = div_rn_rcp(v[j], own_deg, own_rdeg);
+              }
+              const int col = n0 + c;
+              if (p.Yb) {
+                uint16_t* d = reinterpret_cast<uint16_t*>(own) + col;
+                if (col + 16 <= p.N) {
+                  reinterpret_cast<uint4*>(d)[0] = make_uint4(pack_bf16x2(v[0], v[1]), pack_bf16x2(v[2], v[3]),
+                                                              pack_bf16x2(v[4], v[5]), pack_bf16x2(v[6], v[7]));
+                  reinterpret_cast<uint4*>(d)[1] = make_uint4(pack_bf16x2(v[8], v[9]), pack_bf16x2(v[10], v[11]),
+                                                              pack_bf16x2(v[12], v[13]), pack_bf16x2(v[14], v[15]));
+                } else {
+#pragma unroll
+                  for (int j = 0; j < 16; ++j)
+                    if (col + j < p.N) d[j] = bf16_bits(v[j]);
+                }
               } else {
+                float* d = own + col;
+                if (col + 16 <= p.N) {
 #pragma unroll
-                for (int j = 0; j < 16; ++j)
-                  if (col + j < p.N) d[j] = v[j];
+                  for (int j = 0; j < 16; j += 4)
+                    *reinterpret_cast<float4*>(d + j) = make_float4(v[j], v[j + 1], v[j + 2], v[j + 3]);
+                } else {
+#pragma unroll
+                  for (int j = 0; j < 16; ++j)
+                    if (col + j < p.N) d[j] = v[j];
+                }
               }
             }
-          }
-          if (more) {
-            tmem_wait16(rn);
-#pragma unroll
-            for (int j = 0; j < 16; ++j) r[j] = rn[j];
           }
         }
         fence_before();
         mbar_arrive(tempty + acc);
         if (++acc == p.nacc) { acc = 0; aph ^= 1; }
         continue;
+      }
+      uint32_t r[16], rn[16];
+      if (16 * h < p.BN) {
+        tmem_ld16_nowait(tbase + uint32_t(16 * h), r);
+        tmem_wait16(r);
       }
       for (int c = 16 * h; c < p.BN; c += 32) {
         const bool more = c + 32 < p.BN;

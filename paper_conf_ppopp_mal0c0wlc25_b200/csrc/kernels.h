@@ -248,7 +248,9 @@ cudaError_t launch_grad_finish(const float* G, int64_t g_pitch, const float* H, 
 cudaError_t launch_ce_loss(const float* logits, int64_t pitch, int n_classes, const int32_t* seeds,
                            const int32_t* n_seeds, int64_t max_seeds, const int32_t* labels,
                            const int32_t* n_global, float* loss, float* g, int64_t g_pitch, uint16_t* gb,
-                           int64_t gb_pitch, cudaStream_t st);
+                           int64_t gb_pitch, float* zero, int64_t zero_n, int32_t* ws, cudaStream_t st);
+// ce_loss workspace: [ticket, partial sums of up to kCeMaxBlocks blocks], zero-initialised once
+constexpr int kCeMaxBlocks = 1024;
 cudaError_t launch_relu_bwd(float* g, const float* h, int64_t pitch, int dim, const int32_t* n_dev, int64_t max_n,
                             cudaStream_t st);
 cudaError_t launch_colsum(const float* g, int64_t pitch, int dim, const int32_t* n_dev, int64_t max_n, float* out,

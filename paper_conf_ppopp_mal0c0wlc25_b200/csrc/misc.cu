@@ -16,12 +16,19 @@ __global__ void ce_loss_kernel(const float* __restrict__ logits, int64_t pitch, 
                                const int32_t* __restrict__ seeds, const int32_t* __restrict__ n_seeds_p,
                                const int32_t* __restrict__ labels, const int32_t* __restrict__ n_global_p,
                                float* __restrict__ loss, float* __restrict__ g, int64_t g_pitch,
-                               uint16_t* __restrict__ gb, int64_t gb_pitch, int64_t max_seeds) {
+                               uint16_t* __restrict__ gb, int64_t gb_pitch, int64_t max_seeds,
+                               float* __restrict__ zero, int64_t zero_n, float* __restrict__ part,
+                               int32_t* __restrict__ ticket) {
   APT_PDL_PROLOGUE();
   const int lane = lane_id();
   const int64_t n = *n_seeds_p;
   const float inv_n = 1.0f / float(max(1, *n_global_p));
   const int64_t nwarps = int64_t(gridDim.x) * (blockDim.x >> 5);
+  // the step's gradient accumulators start at zero (the backward's reductions add into
+  // them); done here instead of a memset node, which would break the PDL chain
+  for (int64_t t = int64_t(blockIdx.x) * blockDim.x + threadIdx.x; t < zero_n; t += int64_t(gridDim.x) * blockDim.x)
+    zero[t] = 0.f;
+  float wloss = 0.f;   // this warp's rows (fixed assignment: the loss sum is deterministic)
   for (int64_t i = (int64_t(blockIdx.x) * blockDim.x + threadIdx.x) >> 5; i < n; i += nwarps) {
     const float* row = logits + i * pitch;
     float m = -INFINITY;
@@ -33,7 +40,7 @@ __global__ void ce_loss_kernel(const float* __restrict__ logits, int64_t pitch, 
     s = warp_sum(s);
     const int y = labels[seeds[i]];
     const float lse = m + logf(s);
-    if (lane == 0) atomicAdd(loss, (lse - row[y]) * inv_n);
+    wloss += (lse - row[y]) * inv_n;
     for (int c = lane; c < C; c += 32) {
       const float p = expf(row[c] - lse);
       const float v = (p - (c == y ? 1.f : 0.f)) * inv_n;
@@ -50,14 +57,36 @@ __global__ void ce_loss_kernel(const float* __restrict__ logits, int64_t pitch, 
          t += int64_t(gridDim.x) * blockDim.x)
       gb[n * gb_pitch + t] = 0;
   }
+  // loss = the blocks' partial sums added in block order by the last block to finish
+  // (no zeroed accumulator needed before the kernel, and run-to-run identical)
+  __shared__ float wsum[8];
+  __shared__ bool last;
+  if (lane == 0) wsum[threadIdx.x >> 5] = wloss;
+  __syncthreads();
+  if (threadIdx.x == 0) {
+    float b = 0.f;
+    for (int w = 0; w < int(blockDim.x >> 5); ++w) b += wsum[w];
+    part[blockIdx.x] = b;
+    __threadfence();
+    last = atomicAdd(ticket, 1) == int(gridDim.x) - 1;
+  }
+  __syncthreads();
+  if (last && threadIdx.x == 0) {
+    __threadfence();
+    float tot = 0.f;
+    for (int b = 0; b < int(gridDim.x); ++b) tot += __ldcg(part + b);
+    *loss = tot;
+    *ticket = 0;
+  }
 }
 
 cudaError_t launch_ce_loss(const float* logits, int64_t pitch, int n_classes, const int32_t* seeds,
                            const int32_t* n_seeds, int64_t max_seeds, const int32_t* labels,
                            const int32_t* n_global, float* loss, float* g, int64_t g_pitch, uint16_t* gb,
-                           int64_t gb_pitch, cudaStream_t st) {
-  launch_pdl(ce_loss_kernel, dim3(grid_of(max_seeds * 32)), dim3(256), 0, st, logits, pitch, n_classes, seeds, n_seeds, labels,
-                                                          n_global, loss, g, g_pitch, gb, gb_pitch, max_seeds);
+                           int64_t gb_pitch, float* zero, int64_t zero_n, int32_t* ws, cudaStream_t st) {
+  const int64_t grid = std::min<int64_t>(kCeMaxBlocks, grid_of(max_seeds * 32));
+  launch_pdl(ce_loss_kernel, dim3(grid), dim3(256), 0, st, logits, pitch, n_classes, seeds, n_seeds, labels,
+             n_global, loss, g, g_pitch, gb, gb_pitch, max_seeds, zero, zero_n, reinterpret_cast<float*>(ws + 1), ws);
   return cudaGetLastError();
 }
 

@@ -34,6 +34,9 @@ static void ctx_free(apt_ctx* c) {
   release_exported(c);
   if (c->side) { cudaStreamSynchronize(c->side); cudaStreamDestroy(c->side); }
   if (c->samp) { cudaStreamSynchronize(c->samp); cudaStreamDestroy(c->samp); }
+  if (c->tap) { cudaStreamSynchronize(c->tap); cudaStreamDestroy(c->tap); }
+  if (c->ev_tap) cudaEventDestroy(c->ev_tap);
+  if (c->ev_tapj) cudaEventDestroy(c->ev_tapj);
   if (c->ev_pfork) cudaEventDestroy(c->ev_pfork);
   if (c->ev_pjoin) cudaEventDestroy(c->ev_pjoin);
   if (c->ev_fork) cudaEventDestroy(c->ev_fork);
@@ -102,7 +105,12 @@ apt_status apt_ctx_create(int rank, int world, int device, void* stream, apt_ctx
     c->own_stream = true;
   }
   cudaStreamCreateWithPriority(&c->side, cudaStreamNonBlocking, prio_hi);
-  cudaStreamCreateWithPriority(&c->samp, cudaStreamNonBlocking, prio_lo);
+  // APT_SAMP_PRIO=1: the sampling stream at the chain's priority (A/B)
+  static const int samp_hi = [] { const char* v = std::getenv("APT_SAMP_PRIO"); return v ? atoi(v) : 0; }();
+  cudaStreamCreateWithPriority(&c->samp, cudaStreamNonBlocking, samp_hi ? prio_hi : prio_lo);
+  cudaStreamCreateWithPriority(&c->tap, cudaStreamNonBlocking, prio_hi);
+  cudaEventCreateWithFlags(&c->ev_tap, cudaEventDisableTiming);
+  cudaEventCreateWithFlags(&c->ev_tapj, cudaEventDisableTiming);
   cudaEventCreateWithFlags(&c->ev_pfork, cudaEventDisableTiming);
   cudaEventCreateWithFlags(&c->ev_pjoin, cudaEventDisableTiming);
   cudaEventCreateWithFlags(&c->ev_fork, cudaEventDisableTiming);

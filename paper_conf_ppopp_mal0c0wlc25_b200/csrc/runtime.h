@@ -73,6 +73,8 @@ struct apt_ctx {
   bool own_stream = false;
   cudaStream_t side = nullptr;           // forked branch of a step (weight gradients off the critical path)
   cudaStream_t samp = nullptr;           // sampling of the next step (pipelined trainer)
+  cudaStream_t tap = nullptr;            // captured graphs: timing events hang off the chain here
+  cudaEvent_t ev_tap = nullptr, ev_tapj = nullptr;
   cudaEvent_t ev_pfork = nullptr, ev_pjoin = nullptr;
   cudaEvent_t ev_fork = nullptr, ev_join = nullptr, ev_csc = nullptr;
   bool broken = false;

@@ -319,11 +319,9 @@ static apt_status owner_execute(apt_trainer* t, RankState& rs, bool time_it) {
   if (t->s == APT_SNP) { a.filt_part = t->g->part; a.keep_part = rs.rank; }
   if (bf) { a.z_bf16 = x.wZb; a.z_bf16_pitch = x.wzb_pitch; }
   else { a.z_f32 = x.wZf; a.z_f32_pitch = x.wzf_pitch; }
-  if (time_it) CK(c, t->capturing ? cudaEventRecordWithFlags(t->ev[6], c->stream, cudaEventRecordExternal)
-                                  : cudaEventRecord(t->ev[6], c->stream));
+  if (time_it) CK(c, tap_event(t, t->ev[6], c->stream));
   CK(c, launch_agg_fstore(a, feat_view(t->f, rs.rank), c->stream));
-  if (time_it) CK(c, t->capturing ? cudaEventRecordWithFlags(t->ev[7], c->stream, cudaEventRecordExternal)
-                                  : cudaEventRecord(t->ev[7], c->stream));
+  if (time_it) CK(c, tap_event(t, t->ev[7], c->stream));
   c->launches++;
   // Projection with the Reshuffle fused into its epilogue (S8+S9): rows routed to the
   // requesters' h^1 buffers; DNP stores act(Y + b), SNP/NFP add partial Y.

@@ -83,10 +83,7 @@ __global__ void allreduce_sum_kernel(float* const* tab, int C, int64_t n) {
 
 // Phase events: inside a stream capture they must become external event-record
 // nodes (so replays time the phases); outside a capture a plain record.
-static cudaError_t record_ev(apt_trainer* t, int i) {
-  return t->capturing ? cudaEventRecordWithFlags(t->ev[i], t->ctx->stream, cudaEventRecordExternal)
-                      : cudaEventRecord(t->ev[i], t->ctx->stream);
-}
+static cudaError_t record_ev(apt_trainer* t, int i) { return tap_event(t, t->ev[i], t->ctx->stream); }
 
 // The step id enters the device as a kernel argument (no host cell that a later
 // call could overwrite before the copy runs); graph replays patch the argument.
@@ -299,6 +296,7 @@ apt_status apt::trainer_create(apt_ctx* c, const apt_graph* g, const apt_fstore*
     RankState& rs = t->R[li];
     rs.rank = c->emulated ? li : c->rank;
     rs.loss = A.alloc<float>(4, true);
+    rs.ce_ws = A.alloc<int32_t>(kCeMaxBlocks + 4, true);
     rs.dst_bm = A.alloc<uint32_t>(n_words, true);
     rs.new_bm = A.alloc<uint32_t>(n_words, true);
     rs.pos = A.alloc<int32_t>(g->n, false);
@@ -692,9 +690,7 @@ apt_status agg_l1_set(apt_trainer* t, RankState& rs, int q, cudaStream_t st, boo
   // beside the step (the sampling branch): a capped grid leaves registers for the chain
   static const int zbg = [] { const char* v = std::getenv("APT_ZBG_BPSM"); return v ? atoi(v) : 0; }();
   if (st == c->samp) a.bpsm = zbg;
-  auto rec = [&](int i) {
-    return t->capturing ? cudaEventRecordWithFlags(t->ev[i], st, cudaEventRecordExternal) : cudaEventRecord(t->ev[i], st);
-  };
+  auto rec = [&](int i) { return tap_event(t, t->ev[i], st); };
   if (time_it) CK(c, rec(6));
   CK(c, launch_agg_fstore(a, fv, st));
   c->launches++;
@@ -723,7 +719,7 @@ apt_status layer1_fwd_gdp(apt_trainer* t, RankState& rs, bool time_it) {
     apt_status s = agg_l1_set(t, rs, t->parity, t->ctx->stream, time_it);
     if (s != APT_OK) return s;
   }
-  if (t->deferred_fork && sample_fork_point() == 2 && &rs == &t->R.back()) {
+  if (t->deferred_fork && sample_fork_point() >= 2 && &rs == &t->R.back()) {
     // the next step's sampling forks after the layer-1 gather (the gather runs alone)
     std::function<apt_status()> f = std::move(t->deferred_fork);
     t->deferred_fork = nullptr;
@@ -762,9 +758,10 @@ apt_status upper_fwd_loss(apt_trainer* t, RankState& rs) {
     if (s != APT_OK) return s;
   }
   Layer& LK = rs.L[t->K - 1];
-  CK(c, cudaMemsetAsync(rs.loss, 0, sizeof(float), c->stream));
+  // the loss kernel also zeroes this rank's gradient accumulators [dW1 db1 dW2 ...]
+  // (no memset node between the forward and the backward)
   CK(c, launch_ce_loss(LK.H, LK.h_pitch, LK.d_out, rs.seeds, rs.small, LK.max_rows, t->labels, rs.small + 1, rs.loss,
-                       LK.G, LK.h_pitch, LK.Gb, LK.gb_pitch, c->stream));
+                       LK.G, LK.h_pitch, LK.Gb, LK.gb_pitch, rs.L[0].dW, grad_floats(t, rs), rs.ce_ws, c->stream));
   c->launches++;
   return APT_OK;
 }
@@ -906,6 +903,7 @@ apt_status step_body(apt_trainer* t, int update, bool host_batch, int q = 0) {
   if (s != APT_OK) return s;
   activate(t, q);
   t->deferred_fork = nullptr;   // unpipelined: nothing to fork (a failed earlier call may have left one)
+  t->pfork_recorded = false;
   return compute_body(t, update);
 }
 
@@ -913,19 +911,37 @@ apt_status step_body(apt_trainer* t, int update, bool host_batch, int q = 0) {
 // set_step node, patched per replay) is sampled into set p^1 on the sampling stream.
 // Run the next-step sampling fork now, or leave it for compute_body to launch right
 // after the layer-1 forward.
+// Fork point 3: the branch is captured after the layer-1 gather (like 2) but from the
+// fork event recorded at the step start, so it still depends on nothing of this step.
 static apt_status fork_or_defer(apt_trainer* t, std::function<apt_status()> fork) {
-  if (sample_fork_point() != 0 && (sample_fork_point() == 1 || (!t->gat_heads && (t->world == 1 || t->s == APT_GDP)))) {
+  const int fp = sample_fork_point();
+  if (fp != 0 && (fp == 1 || (!t->gat_heads && (t->world == 1 || t->s == APT_GDP)))) {
+    if (fp == 3) {
+      apt_status s = check_cuda(t->ctx, cudaEventRecord(t->ctx->ev_pfork, t->ctx->stream), "fork event");
+      if (s != APT_OK) return s;
+      t->pfork_recorded = true;
+    }
     t->deferred_fork = std::move(fork);
     return APT_OK;
   }
   return fork();
 }
 
+// The fork event of the next step's sampling branch (recorded here unless fork point 3
+// recorded it at the step start).
+static cudaError_t pfork_record(apt_trainer* t) {
+  if (t->pfork_recorded) {
+    t->pfork_recorded = false;
+    return cudaSuccess;
+  }
+  return cudaEventRecord(t->ctx->ev_pfork, t->ctx->stream);
+}
+
 apt_status pipelined_body(apt_trainer* t, int p, int update, uint64_t next) {
   apt_ctx* c = t->ctx;
   CK(c, record_ev(t, 0));
   apt_status s = fork_or_defer(t, [t, c, p, next]() -> apt_status {
-    CK(c, cudaEventRecord(c->ev_pfork, c->stream));
+    CK(c, pfork_record(t));
     CK(c, cudaStreamWaitEvent(c->samp, c->ev_pfork, 0));
     set_step_kernel<<<1, 1, 0, c->samp>>>(t->step_cells + (p ^ 1), next);
     CK(c, cudaGetLastError());
@@ -981,8 +997,7 @@ apt_status compute_body(apt_trainer* t, int update) {
     if (s != APT_OK) return s;
   }
   CK(c, record_ev(t, 3));
-  // zero the gradient accumulators, then backward
-  for (auto& rs : t->R) CK(c, cudaMemsetAsync(rs.L[0].dW, 0, sizeof(float) * grad_floats(t, rs), c->stream));
+  // backward (the gradient accumulators were zeroed by the loss kernel)
   for (auto& rs : t->R) {
     apt_status s = upper_bwd(t, rs);
     if (s != APT_OK) return s;
@@ -1249,7 +1264,10 @@ apt_status apt_trainer_step(apt_trainer* t, int64_t step, int update) {
         t->capturing = true;
         apt_status s = step_body(t, update, false, 0);
         t->capturing = false;
+        const cudaError_t ej = s == APT_OK ? tap_join(t) : cudaSuccess;
+        t->tapped = false;
         cudaError_t e = cudaStreamEndCapture(c->stream, &graph);
+        if (e == cudaSuccess) e = ej;
         t->launches_per_step = c->launches - l0 + 1;   // counted at replay, not at capture
         c->launches = l0;
         if (s != APT_OK) return s;
@@ -1293,7 +1311,10 @@ apt_status apt_trainer_step(apt_trainer* t, int64_t step, int update) {
       t->capturing = true;
       apt_status s = pipelined_body(t, p, update, next);
       t->capturing = false;
+      const cudaError_t ej = s == APT_OK ? tap_join(t) : cudaSuccess;
+      t->tapped = false;
       cudaError_t e = cudaStreamEndCapture(c->stream, &graph);
+      if (e == cudaSuccess) e = ej;
       t->launches_p[p][update] = c->launches - l0;
       c->launches = l0;
       if (s != APT_OK) return s;
@@ -1361,7 +1382,10 @@ apt_status apt_trainer_step_host(apt_trainer* t, const int64_t* gbatch, int64_t 
       t->capturing = true;
       apt_status s = body();
       t->capturing = false;
+      const cudaError_t ej = s == APT_OK ? tap_join(t) : cudaSuccess;
+      t->tapped = false;
       cudaError_t e = cudaStreamEndCapture(c->stream, &graph);
+      if (e == cudaSuccess) e = ej;
       const int64_t per = c->launches - l0 + 1;
       c->launches = l0;
       if (s != APT_OK) return s;
@@ -1430,7 +1454,7 @@ static apt_status step_host_pipelined_impl(apt_trainer* t, const int64_t* next_b
   auto body = [&](uint64_t nstep) -> apt_status {
     CK(c, record_ev(t, 0));
     apt_status s = fork_or_defer(t, [&, nstep]() -> apt_status {
-      CK(c, cudaEventRecord(c->ev_pfork, c->stream));
+      CK(c, pfork_record(t));
       CK(c, cudaStreamWaitEvent(c->samp, c->ev_pfork, 0));
       CK(c, cudaMemcpyAsync(t->hb_dev + q * t->hb_len, stage, hb_bytes, cudaMemcpyHostToDevice, c->samp));
       set_step_kernel<<<1, 1, 0, c->samp>>>(t->step_cells + q, nstep);
@@ -1464,7 +1488,10 @@ static apt_status step_host_pipelined_impl(apt_trainer* t, const int64_t* next_b
       t->capturing = true;
       apt_status s = body(uint64_t(next_step));
       t->capturing = false;
+      const cudaError_t ej = s == APT_OK ? tap_join(t) : cudaSuccess;
+      t->tapped = false;
       cudaError_t e = cudaStreamEndCapture(c->stream, &graph);
+      if (e == cudaSuccess) e = ej;
       t->launches_hp[p][update] = c->launches - l0 + 1;
       c->launches = l0;
       if (s != APT_OK) return s;

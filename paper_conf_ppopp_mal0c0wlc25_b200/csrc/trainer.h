@@ -141,6 +141,7 @@ struct RankState {
   int32_t* pos = nullptr;
   int32_t* partials = nullptr;
   float* loss = nullptr;
+  int32_t* ce_ws = nullptr;          // ce_loss: block-partial losses + ticket (zeroed once, self-resetting)
   Xchg x;
   GatState ga;
 };
@@ -181,6 +182,8 @@ struct apt_trainer {
   uint16_t** gGb_tab = nullptr;      // requesters' Gb (bf16)
   bool use_graph = false;
   bool capturing = false;
+  bool tapped = false;
+  bool pfork_recorded = false;       // fork point 3: the sampling branch's fork event was recorded at the step start               // a captured timing event hangs off the chain on ctx->tap (join before EndCapture)
   // pipelining: step t+1 is sampled on ctx->samp while step t computes
   bool pipeline = true;
   bool z_prefetch = false;           // GDP SAGE layer 1: the next batch's gather+mean runs on the sampling
@@ -229,3 +232,33 @@ struct apt_trainer {
   apt::Arena arena;
   ~apt_trainer() { apt::close_peers(peer_opened); apt::defer_exported(ctx, arena); }
 };
+
+namespace apt {
+// A timing event at the current point of stream st.  Eagerly: a plain record.  Inside a
+// stream capture the record node hangs off the chain on ctx->tap (an internal fork edge),
+// so the kernel that follows on st keeps its programmatic (PDL) edge to the one before:
+// an external record node placed IN the chain cost the step ~5 us per event (measured
+// with tools/timeline.py: the next kernel waited for the full drain + the node).
+// APT_TAP_EVENTS=0 puts them back in the chain (A/B).
+inline cudaError_t tap_event(apt_trainer* t, cudaEvent_t ev, cudaStream_t st) {
+  static const int tap = [] { const char* v = std::getenv("APT_TAP_EVENTS"); return v ? atoi(v) : 1; }();
+  if (!t->capturing) return cudaEventRecord(ev, st);
+  if (!tap) return cudaEventRecordWithFlags(ev, st, cudaEventRecordExternal);
+  apt_ctx* c = t->ctx;
+  cudaError_t e = cudaEventRecord(c->ev_tap, st);
+  if (e == cudaSuccess) e = cudaStreamWaitEvent(c->tap, c->ev_tap, 0);
+  if (e == cudaSuccess) e = cudaEventRecordWithFlags(ev, c->tap, cudaEventRecordExternal);
+  t->tapped = true;
+  return e;
+}
+// Join the tap branch into the capture origin (every forked stream must rejoin before
+// cudaStreamEndCapture); call right before it.
+inline cudaError_t tap_join(apt_trainer* t) {
+  if (!t->tapped) return cudaSuccess;
+  t->tapped = false;
+  apt_ctx* c = t->ctx;
+  cudaError_t e = cudaEventRecord(c->ev_tapj, c->tap);
+  if (e == cudaSuccess) e = cudaStreamWaitEvent(c->stream, c->ev_tapj, 0);
+  return e;
+}
+}  // namespace apt
