@@ -18,7 +18,7 @@ __global__ void ce_loss_kernel(const float* __restrict__ logits, int64_t pitch, 
                                float* __restrict__ loss, float* __restrict__ g, int64_t g_pitch,
                                uint16_t* __restrict__ gb, int64_t gb_pitch, int64_t max_seeds,
                                float* __restrict__ zero, int64_t zero_n, float* __restrict__ part,
-                               int32_t* __restrict__ ticket) {
+                               int32_t* __restrict__ ticket, int32_t* __restrict__ zero_i, int64_t zero_i_n) {
   APT_PDL_PROLOGUE();
   const int lane = lane_id();
   const int64_t n = *n_seeds_p;
@@ -28,9 +28,14 @@ __global__ void ce_loss_kernel(const float* __restrict__ logits, int64_t pitch, 
   // them); done here instead of a memset node, which would break the PDL chain
   for (int64_t t = int64_t(blockIdx.x) * blockDim.x + threadIdx.x; t < zero_n; t += int64_t(gridDim.x) * blockDim.x)
     zero[t] = 0.f;
+  for (int64_t t = int64_t(blockIdx.x) * blockDim.x + threadIdx.x; t < zero_i_n; t += int64_t(gridDim.x) * blockDim.x)
+    zero_i[t] = 0;
   float wloss = 0.f;   // this warp's rows (fixed assignment: the loss sum is deterministic)
   for (int64_t i = (int64_t(blockIdx.x) * blockDim.x + threadIdx.x) >> 5; i < n; i += nwarps) {
     const float* row = logits + i * pitch;
+    // the label's two dependent loads (seed id, then its label) are issued before the
+    // row's arithmetic so that their latency overlaps it
+    const int y = labels[seeds[i]];
     float m = -INFINITY;
     for (int c = lane; c < C; c += 32) m = fmaxf(m, row[c]);
 #pragma unroll
@@ -38,7 +43,6 @@ __global__ void ce_loss_kernel(const float* __restrict__ logits, int64_t pitch, 
     float s = 0.f;
     for (int c = lane; c < C; c += 32) s += expf(row[c] - m);
     s = warp_sum(s);
-    const int y = labels[seeds[i]];
     const float lse = m + logf(s);
     wloss += (lse - row[y]) * inv_n;
     for (int c = lane; c < C; c += 32) {
@@ -57,8 +61,10 @@ __global__ void ce_loss_kernel(const float* __restrict__ logits, int64_t pitch, 
          t += int64_t(gridDim.x) * blockDim.x)
       gb[n * gb_pitch + t] = 0;
   }
-  // loss = the blocks' partial sums added in block order by the last block to finish
-  // (no zeroed accumulator needed before the kernel, and run-to-run identical)
+  // loss = the blocks' partial sums, reduced by the last block to finish in a fixed order
+  // (lane l adds blocks l, l+32, ... then a fixed shuffle tree): no zeroed accumulator
+  // before the kernel, run-to-run identical, and the partials are read 32 at a time
+  // rather than one dependent L2 round trip after another
   __shared__ float wsum[8];
   __shared__ bool last;
   if (lane == 0) wsum[threadIdx.x >> 5] = wloss;
@@ -71,22 +77,28 @@ __global__ void ce_loss_kernel(const float* __restrict__ logits, int64_t pitch, 
     last = atomicAdd(ticket, 1) == int(gridDim.x) - 1;
   }
   __syncthreads();
-  if (last && threadIdx.x == 0) {
+  if (last && threadIdx.x < 32) {
     __threadfence();
     float tot = 0.f;
-    for (int b = 0; b < int(gridDim.x); ++b) tot += __ldcg(part + b);
-    *loss = tot;
-    *ticket = 0;
+    for (int b = lane; b < int(gridDim.x); b += 32) tot += __ldcg(part + b);
+#pragma unroll
+    for (int o = 16; o > 0; o >>= 1) tot += __shfl_xor_sync(0xffffffffu, tot, o);
+    if (lane == 0) {
+      *loss = tot;
+      *ticket = 0;
+    }
   }
 }
 
 cudaError_t launch_ce_loss(const float* logits, int64_t pitch, int n_classes, const int32_t* seeds,
                            const int32_t* n_seeds, int64_t max_seeds, const int32_t* labels,
                            const int32_t* n_global, float* loss, float* g, int64_t g_pitch, uint16_t* gb,
-                           int64_t gb_pitch, float* zero, int64_t zero_n, int32_t* ws, cudaStream_t st) {
+                           int64_t gb_pitch, float* zero, int64_t zero_n, int32_t* ws, cudaStream_t st,
+                           int32_t* zero_i, int64_t zero_i_n) {
   const int64_t grid = std::min<int64_t>(kCeMaxBlocks, grid_of(max_seeds * 32));
   launch_pdl(ce_loss_kernel, dim3(grid), dim3(256), 0, st, logits, pitch, n_classes, seeds, n_seeds, labels,
-             n_global, loss, g, g_pitch, gb, gb_pitch, max_seeds, zero, zero_n, reinterpret_cast<float*>(ws + 1), ws);
+             n_global, loss, g, g_pitch, gb, gb_pitch, max_seeds, zero, zero_n, reinterpret_cast<float*>(ws + 1), ws,
+             zero_i, zero_i_n);
   return cudaGetLastError();
 }
 

@@ -25,6 +25,9 @@ def main():
     ap.add_argument("--dtype", default="bf16")
     ap.add_argument("--out", default="gpurun_out/timeline.json")
     ap.add_argument("--no-pipeline", action="store_true")
+    ap.add_argument("--sync-flush", action="store_true",
+                    help="synchronize between the L2 flush and the step (exposes the host graph launch); "
+                         "default: like bench.py, the launch overlaps the flush")
     args = ap.parse_args()
     import torch
     from torch.profiler import ProfilerActivity, profile
@@ -57,7 +60,8 @@ def main():
     with profile(activities=[ProfilerActivity.CUDA]) as prof:
         for i in range(args.steps):
             flush.zero_()
-            torch.cuda.synchronize()
+            if args.sync_flush:
+                torch.cuda.synchronize()
             tr.step(10 + i)
             torch.cuda.synchronize()
     os.makedirs(os.path.dirname(args.out) or ".", exist_ok=True)
@@ -65,11 +69,12 @@ def main():
     ev = [e for e in json.load(open(args.out))["traceEvents"] if e.get("cat") == "kernel"]
     ev.sort(key=lambda e: e["ts"])
     # split into steps at the flush kernels (FillFunctor / zero_)
-    steps, cur = [], None
+    steps, cur, fl_end = [], None, []
     for e in ev:
         if "FillFunctor" in e["name"]:
             cur = []
             steps.append(cur)
+            fl_end.append(e["ts"] + e["dur"])
         elif cur is not None:
             cur.append(e)
     for si, st in enumerate(steps[1:3], 1):
@@ -77,7 +82,8 @@ def main():
             continue
         t0 = st[0]["ts"]
         t1 = max(e["ts"] + e["dur"] for e in st)
-        print(f"# step {si}: {len(st)} kernels, first->last end {t1 - t0:.1f} us")
+        print(f"# step {si}: {len(st)} kernels, first->last end {t1 - t0:.1f} us; "
+              f"L2 flush end -> first kernel {t0 - fl_end[si]:.1f} us")
         streams = sorted({e["args"].get("stream", 0) for e in st})
         for e in st:
             s = e["args"].get("stream", 0)
