@@ -253,7 +253,12 @@ __global__ void __launch_bounds__(ROW_THREADS, 1)
               const int col = n0 + c;
               if (p.Yb) {
                 uint16_t* d = reinterpret_cast<uint16_t*>(own) + col;
-                if (col + 16 <= p.N) {
+                if (col + 16 <= p.N && (reinterpret_cast<uintptr_t>(d) & 31) == 0) {
+                  // the chunk's 32 bytes of this row as ONE sector-sized store (STG.256)
+                  st_v8(d, pack_bf16x2(v[0], v[1]), pack_bf16x2(v[2], v[3]), pack_bf16x2(v[4], v[5]),
+                        pack_bf16x2(v[6], v[7]), pack_bf16x2(v[8], v[9]), pack_bf16x2(v[10], v[11]),
+                        pack_bf16x2(v[12], v[13]), pack_bf16x2(v[14], v[15]));
+                } else if (col + 16 <= p.N) {
                   reinterpret_cast<uint4*>(d)[0] = make_uint4(pack_bf16x2(v[0], v[1]), pack_bf16x2(v[2], v[3]),
                                                               pack_bf16x2(v[4], v[5]), pack_bf16x2(v[6], v[7]));
                   reinterpret_cast<uint4*>(d)[1] = make_uint4(pack_bf16x2(v[8], v[9]), pack_bf16x2(v[10], v[11]),
@@ -265,7 +270,13 @@ __global__ void __launch_bounds__(ROW_THREADS, 1)
                 }
               } else {
                 float* d = own + col;
-                if (col + 16 <= p.N) {
+                if (col + 16 <= p.N && (reinterpret_cast<uintptr_t>(d) & 31) == 0) {
+#pragma unroll
+                  for (int j = 0; j < 16; j += 8)
+                    st_v8(d + j, __float_as_uint(v[j]), __float_as_uint(v[j + 1]), __float_as_uint(v[j + 2]),
+                          __float_as_uint(v[j + 3]), __float_as_uint(v[j + 4]), __float_as_uint(v[j + 5]),
+                          __float_as_uint(v[j + 6]), __float_as_uint(v[j + 7]));
+                } else if (col + 16 <= p.N) {
 #pragma unroll
                   for (int j = 0; j < 16; j += 4)
                     *reinterpret_cast<float4*>(d + j) = make_float4(v[j], v[j + 1], v[j + 2], v[j + 3]);
