@@ -229,10 +229,8 @@ __global__ void __launch_bounds__(256) pull_bwd_kernel(PullArgs a) {
 // columns (one 16-B load per in-edge), R source rows in flight per warp; the mask is
 // applied to the packed bf16 pairs with one AND against a per-half compare of H's bits
 // (bf16 > 0 <=> its 16-bit pattern is a positive signed integer).
-// (5 blocks' worth of registers per SM: at 4 resident blocks a 6-warp weight-gradient
-// CTA still fits beside them on every SM sub-partition, see `ready`)
 template <int VP, int R>
-__global__ void __launch_bounds__(256, VP == 1 ? 5 : 1) pull_bwd_b8_kernel(PullArgs a) {
+__global__ void __launch_bounds__(256) pull_bwd_b8_kernel(PullArgs a) {
   APT_PDL_PROLOGUE();
   const int lane = lane_id();
   const int64_t n = *a.n_src;
@@ -301,13 +299,6 @@ __global__ void __launch_bounds__(256, VP == 1 ? 5 : 1) pull_bwd_b8_kernel(PullA
         *reinterpret_cast<uint4*>(a.gb + u * a.gb_pitch + j * 8) = o;
       }
     }
-    if (a.ready) {
-      // publish the finished rows to the weight-gradient kernel consuming this block
-      // (every lane's stores, then one release-ordered count per warp; R divides 64)
-      __threadfence();
-      __syncwarp();
-      if (lane == 0) atomicAdd(a.ready + (u0 >> 6), int(std::min<int64_t>(R, rows_out - u0)));
-    }
   }
 }
 
@@ -338,8 +329,7 @@ cudaError_t launch_pull_bwd(const PullArgs& a, cudaStream_t st) {
     static const int rr = [] { const char* e = std::getenv("APT_PULL_ROWS"); return e ? atoi(e) : 2; }();
     const int Rr = rr == 4 ? 4 : 2;
     // APT_PULL_BPSM: grid cap in blocks per SM (A/B knob)
-    static const int bpsm_env = [] { const char* e = std::getenv("APT_PULL_BPSM"); return e ? atoi(e) : 16; }();
-    const int bpsm = a.bpsm > 0 ? a.bpsm : bpsm_env;
+    static const int bpsm = [] { const char* e = std::getenv("APT_PULL_BPSM"); return e ? atoi(e) : 16; }();
     const int64_t blocks = std::max<int64_t>(
         1, std::min<int64_t>(ceil_div(ceil_div(round_up(a.max_src, 64), Rr) * 32, 256), int64_t(num_sms()) * bpsm));
     const int V8 = a.dim >> 3;

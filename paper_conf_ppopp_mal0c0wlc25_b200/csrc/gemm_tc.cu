@@ -395,8 +395,6 @@ struct WgradParams {
   float* dW;                // [d_out x ldw] (accumulated)
   float* db;                // [d_out] (accumulated) or null
   int64_t ldw;
-  const int32_t* ready;     // per 64-row block: rows of G written so far by the running pull kernel
-  int64_t ready_rows_max;
 };
 
 __global__ void __launch_bounds__(THREADS, 1)
@@ -426,11 +424,7 @@ __global__ void __launch_bounds__(THREADS, 1)
   __syncthreads();
   fence_after();
   const uint32_t tmem_base = *tmem_slot;
-  // with `ready`, G is still being written by the kernel before this one: no wait for its
-  // completion (that kernel passed its own griddepcontrol.wait before this grid could
-  // launch, so every earlier kernel of the step -- Z, the zeroed dW -- is complete), the
-  // producer waits per 64-row block instead
-  if (!p.ready) pdl_wait();
+  pdl_wait();
   pdl_launch();
   const int64_t rows = std::min<int64_t>(p.rows_max, int64_t(*p.rows_dev));
   const int64_t nkb_all = ceil_div(rows, BK);
@@ -452,13 +446,7 @@ __global__ void __launch_bounds__(THREADS, 1)
       const int na = (p.d_out - m0 > 64) ? 2 : 1;
       const int zcols = p.ones_col ? p.d_in + 1 : p.d_in;
       const int nz = int(ceil_div(zcols, 64));
-      const int64_t g_rows = std::min<int64_t>(p.ready_rows_max, round_up(rows, int64_t(BK)));
       for (int64_t kb = kb0; kb < kb1; ++kb) {
-        if (p.ready) {
-          const int want = int(std::min<int64_t>(BK, g_rows - kb * BK));
-          while (ld_acquire_gpu(p.ready + kb) < want) __nanosleep(64);
-          asm volatile("fence.proxy.async.global;" ::: "memory");   // generic-proxy writes -> TMA reads
-        }
         mbar_wait(empty + s, ph ^ 1);
         mbar_expect_tx(full + s, uint32_t(na + nz) * MNBLK);
         uint8_t* st = smem + size_t(s) * p.stage_bytes;
@@ -621,7 +609,7 @@ cudaError_t launch_tc_wgrad(const TcWgradArgs& a, cudaStream_t st) {
   if (!make_map(&mz, a.Z, zcols, rows, a.z_pitch, 64, BK)) return cudaErrorInvalidValue;
   const uint32_t stage = uint32_t(2 + nbz) * MNBLK;
   WgradParams p{a.rows_dev, a.rows_max, a.d_out, a.d_in, BN, nbz, cols, a.db ? 1 : 0, stage, 0, a.dW, a.db,
-                a.ldw > 0 ? a.ldw : a.d_in, a.ready, a.ready_rows_max};
+                a.ldw > 0 ? a.ldw : a.d_in};
   // ring depth: as many stages as fit (more bytes in flight per SM: the loads are the
   // latency of this kernel), A/B via APT_WG_STAGES
   static const int want = [] { const char* v = std::getenv("APT_WG_STAGES"); return v ? atoi(v) : 3; }();   // 3 / 8: 0.2199 / 0.2205 ms

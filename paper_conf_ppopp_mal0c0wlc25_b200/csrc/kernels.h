@@ -169,9 +169,6 @@ struct PullArgs {
   int dz_scaled;                           // dz rows already divided by deg (tcgen05 epilogue)
   const uint16_t* hb; int64_t hb_pitch;    // if set: the ReLU mask from bf16 H (bf16 mode, reading R11)
   const uint16_t* dzb; int64_t dzb_pitch;  // if set: dZ / deg as bf16 rows instead of dz (reading R13)
-  int32_t* ready;                          // if set (bf16 mode): rows of G finished per 64-row block, for a
-                                           //   weight-gradient kernel that consumes the blocks as they complete
-  int bpsm;                                // > 0: grid capped at this many blocks per SM (one resident wave)
 };
 cudaError_t launch_pull_bwd(const PullArgs& a, cudaStream_t st);
 
@@ -237,11 +234,6 @@ struct TcWgradArgs {
   int d_out, d_in;
   float* dW; float* db;
   int64_t ldw;                         // row stride of dW (0 => d_in)
-  // if set: G is being written by the kernel launched just before this one (the pull, PDL);
-  // 64-row block kb is loaded once ready[kb] reaches its row count (rows of the block
-  // below G's extent ready_rows = min(ready_rows_max, round_up(rows, 64))), instead of
-  // waiting for that kernel to finish
-  const int32_t* ready; int64_t ready_rows_max;
 };
 int tc_wgrad_supported(int d_out, int d_in);
 cudaError_t launch_tc_wgrad(const TcWgradArgs& a, cudaStream_t st);
@@ -256,8 +248,7 @@ cudaError_t launch_grad_finish(const float* G, int64_t g_pitch, const float* H, 
 cudaError_t launch_ce_loss(const float* logits, int64_t pitch, int n_classes, const int32_t* seeds,
                            const int32_t* n_seeds, int64_t max_seeds, const int32_t* labels,
                            const int32_t* n_global, float* loss, float* g, int64_t g_pitch, uint16_t* gb,
-                           int64_t gb_pitch, float* zero, int64_t zero_n, int32_t* ws, cudaStream_t st,
-                           int32_t* zero_i = nullptr, int64_t zero_i_n = 0);   // zero_i: also zeroed (counters)
+                           int64_t gb_pitch, float* zero, int64_t zero_n, int32_t* ws, cudaStream_t st);
 // ce_loss workspace: [ticket, partial sums of up to kCeMaxBlocks blocks], zero-initialised once
 constexpr int kCeMaxBlocks = 1024;
 cudaError_t launch_relu_bwd(float* g, const float* h, int64_t pitch, int dim, const int32_t* n_dev, int64_t max_n,

@@ -18,7 +18,7 @@ __global__ void ce_loss_kernel(const float* __restrict__ logits, int64_t pitch, 
                                float* __restrict__ loss, float* __restrict__ g, int64_t g_pitch,
                                uint16_t* __restrict__ gb, int64_t gb_pitch, int64_t max_seeds,
                                float* __restrict__ zero, int64_t zero_n, float* __restrict__ part,
-                               int32_t* __restrict__ ticket, int32_t* __restrict__ zero_i, int64_t zero_i_n) {
+                               int32_t* __restrict__ ticket) {
   APT_PDL_PROLOGUE();
   const int lane = lane_id();
   const int64_t n = *n_seeds_p;
@@ -28,8 +28,6 @@ __global__ void ce_loss_kernel(const float* __restrict__ logits, int64_t pitch, 
   // them); done here instead of a memset node, which would break the PDL chain
   for (int64_t t = int64_t(blockIdx.x) * blockDim.x + threadIdx.x; t < zero_n; t += int64_t(gridDim.x) * blockDim.x)
     zero[t] = 0.f;
-  for (int64_t t = int64_t(blockIdx.x) * blockDim.x + threadIdx.x; t < zero_i_n; t += int64_t(gridDim.x) * blockDim.x)
-    zero_i[t] = 0;
   float wloss = 0.f;   // this warp's rows (fixed assignment: the loss sum is deterministic)
   for (int64_t i = (int64_t(blockIdx.x) * blockDim.x + threadIdx.x) >> 5; i < n; i += nwarps) {
     const float* row = logits + i * pitch;
@@ -93,12 +91,10 @@ __global__ void ce_loss_kernel(const float* __restrict__ logits, int64_t pitch, 
 cudaError_t launch_ce_loss(const float* logits, int64_t pitch, int n_classes, const int32_t* seeds,
                            const int32_t* n_seeds, int64_t max_seeds, const int32_t* labels,
                            const int32_t* n_global, float* loss, float* g, int64_t g_pitch, uint16_t* gb,
-                           int64_t gb_pitch, float* zero, int64_t zero_n, int32_t* ws, cudaStream_t st,
-                           int32_t* zero_i, int64_t zero_i_n) {
+                           int64_t gb_pitch, float* zero, int64_t zero_n, int32_t* ws, cudaStream_t st) {
   const int64_t grid = std::min<int64_t>(kCeMaxBlocks, grid_of(max_seeds * 32));
   launch_pdl(ce_loss_kernel, dim3(grid), dim3(256), 0, st, logits, pitch, n_classes, seeds, n_seeds, labels,
-             n_global, loss, g, g_pitch, gb, gb_pitch, max_seeds, zero, zero_n, reinterpret_cast<float*>(ws + 1), ws,
-             zero_i, zero_i_n);
+             n_global, loss, g, g_pitch, gb, gb_pitch, max_seeds, zero, zero_n, reinterpret_cast<float*>(ws + 1), ws);
   return cudaGetLastError();
 }
 

@@ -183,14 +183,13 @@ apt_status hidden1_to_bf16(apt_trainer* t) {
 // dW (+)= G^T Z over the device-counted rows; db += colsum(G)
 apt_status weight_grad(apt_trainer* t, const Layer& L, const float* G, int64_t g_pitch, const void* Z, bool z_bf16,
                        int64_t z_pitch, const int32_t* n_rows, int64_t max_rows, int d_in, float* dW, float* db,
-                       int64_t dW_ld, cudaStream_t st = nullptr, const int32_t* ready = nullptr) {
+                       int64_t dW_ld, cudaStream_t st = nullptr) {
   apt_ctx* c = t->ctx;
   if (!st) st = c->stream;
   if (z_bf16 && L.Gb && tc_wgrad_supported(L.d_out, d_in)) {
-    // tcgen05: dW = Gb^T Zb with db from Z's all-ones column d_in (ready: Gb's 64-row
-    // blocks are consumed as the mean backward launched just before finishes them)
+    // tcgen05: dW = Gb^T Zb with db from Z's all-ones column d_in
     TcWgradArgs w{L.Gb, L.gb_pitch, static_cast<const uint16_t*>(Z), z_pitch, n_rows, max_rows, L.d_out, d_in,
-                  dW, db, 0, ready, L.max_rows};
+                  dW, db};
     CK(c, launch_tc_wgrad(w, st));
     c->launches++;
     return APT_OK;
@@ -352,10 +351,6 @@ apt_status apt::trainer_create(apt_ctx* c, const apt_graph* g, const apt_fstore*
       L.wb_pitch = round_up(L.d_in, 8);
       L.max_rows = hp.max_dst;
       L.n_rows = hp.n_dst;
-      if (l == 1) {   // per 64-row block of layer 1: rows of G finished by the mean backward
-        rs.l1_ready_n = ceil_div(L.max_rows, 64);
-        rs.l1_ready = A.alloc<int32_t>(rs.l1_ready_n, true);
-      }
       if (m->dtype == APT_BF16) L.Zb = A.alloc<uint16_t>(L.max_rows * L.zb_pitch, true);
       else L.Zf = A.alloc<float>(L.max_rows * L.zf_pitch, true);
       L.H = A.alloc<float>(L.max_rows * L.h_pitch, true);
@@ -766,8 +761,7 @@ apt_status upper_fwd_loss(apt_trainer* t, RankState& rs) {
   // the loss kernel also zeroes this rank's gradient accumulators [dW1 db1 dW2 ...]
   // (no memset node between the forward and the backward)
   CK(c, launch_ce_loss(LK.H, LK.h_pitch, LK.d_out, rs.seeds, rs.small, LK.max_rows, t->labels, rs.small + 1, rs.loss,
-                       LK.G, LK.h_pitch, LK.Gb, LK.gb_pitch, rs.L[0].dW, grad_floats(t, rs), rs.ce_ws, c->stream,
-                       t->l1_overlap ? rs.l1_ready : nullptr, t->l1_overlap ? rs.l1_ready_n : 0));
+                       LK.G, LK.h_pitch, LK.Gb, LK.gb_pitch, rs.L[0].dW, grad_floats(t, rs), rs.ce_ws, c->stream));
   c->launches++;
   return APT_OK;
 }
@@ -840,13 +834,6 @@ apt_status upper_bwd(apt_trainer* t, RankState& rs) {
                 dz_scaled};
     if (P.Hb && !mk) { pa.h = nullptr; pa.hb = P.Hb; pa.hb_pitch = P.hb_pitch; }   // R11: mask from bf16 H
     if (dzb) { pa.dzb = dzb; pa.dzb_pitch = L.dzb_pitch; }                            // R13: bf16 dZ / deg
-    if (l == 2 && t->l1_overlap && dzb && pa.hb && P.d_out <= 256) {
-      // layer 1's weight gradient (launched next) consumes G's 64-row blocks as this
-      // kernel finishes them; one resident wave (4 blocks per SM) leaves room beside it
-      pa.ready = rs.l1_ready;
-      pa.bpsm = 4;
-      rs.l1_overlap = true;
-    }
     CK(c, launch_pull_bwd(pa, c->stream));
     c->launches += 2;
   }
@@ -856,10 +843,8 @@ apt_status upper_bwd(apt_trainer* t, RankState& rs) {
 apt_status layer1_bwd_gdp(apt_trainer* t, RankState& rs) {
   Layer& L = rs.L[0];
   const bool bf = t->m.dtype == APT_BF16;
-  const int32_t* ready = rs.l1_overlap ? rs.l1_ready : nullptr;
-  rs.l1_overlap = false;
   return weight_grad(t, L, L.G, L.h_pitch, bf ? static_cast<const void*>(L.Zb) : L.Zf, bf,
-                     bf ? L.zb_pitch : L.zf_pitch, L.n_rows, L.max_rows, L.d_in, L.dW, L.db, L.d_in, nullptr, ready);
+                     bf ? L.zb_pitch : L.zf_pitch, L.n_rows, L.max_rows, L.d_in, L.dW, L.db, L.d_in);
 }
 
 // Gradient all-reduce over the ranks (DDP) of the first P floats of the
@@ -999,19 +984,9 @@ apt_status pipelined_body(apt_trainer* t, int p, int update, uint64_t next) {
   return APT_OK;
 }
 
-// Layer 1's weight gradient overlapped with layer 2's mean backward (bf16 GDP step;
-// APT_L1_OVERLAP=0: after it, A/B).
-static bool l1_overlap_enabled() {
-  static const int v = [] { const char* e = std::getenv("APT_L1_OVERLAP"); return e ? atoi(e) : 1; }();
-  return v != 0;
-}
-
 apt_status compute_body(apt_trainer* t, int update) {
   apt_ctx* c = t->ctx;
   const bool gdp = t->world == 1 || t->s == APT_GDP;
-  t->l1_overlap = gdp && !t->gat_heads && t->m.dtype == APT_BF16 && t->K > 1 && l1_overlap_enabled() &&
-                  tc_wgrad_supported(t->R[0].L[0].d_out, t->R[0].L[0].d_in);
-  for (auto& rs : t->R) rs.l1_overlap = false;
   CK(c, record_ev(t, 1));
   if (t->gat_heads) {
     apt_status s = gat_layer1_fwd(t, true);

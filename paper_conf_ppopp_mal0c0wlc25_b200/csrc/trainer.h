@@ -130,9 +130,6 @@ struct SampleSet {
 
 struct RankState {
   int rank = 0;
-  int32_t* l1_ready = nullptr;       // per 64-row block of layer 1: rows of G written by the mean backward
-  int64_t l1_ready_n = 0;
-  bool l1_overlap = false;           // this step's layer-1 weight gradient consumes l1_ready
   SampleSet sset[2];
   // the set the current step computes on (copies of sset[active]'s fields)
   int32_t* seeds = nullptr;
@@ -191,7 +188,6 @@ struct apt_trainer {
   bool pipeline = true;
   bool z_prefetch = false;           // GDP SAGE layer 1: the next batch's gather+mean runs on the sampling
                                      //   branch (it reads only the static features), beside this step
-  bool l1_overlap = false;           // bf16 GDP step: layer 1's weight gradient overlaps layer 2's mean backward
   bool z_ready = false;              // the active set's layer-1 Z is already aggregated
   int z_where = 1;                   // z_prefetch: 1 on the sampling branch, 2 beside this step's backward tail
   int z_next = -1;                   // z_where 2: the set whose Z this step aggregates (pipelined bodies)
