@@ -270,9 +270,15 @@ __global__ void __launch_bounds__(256, 2) gat_fwd_kernel(GatKArgs a) {
         const int64_t o = (i * H + h) * a.zp + l * EPV;
         if (a.z_bf16) {
           uint16_t* z = static_cast<uint16_t*>(a.Z) + o;
+          if constexpr (EPV == 8) {   // the lane's 8 columns as one 16-byte store
+            *reinterpret_cast<uint4*>(z) =
+                make_uint4(pack_bf16x2(acc[h][0] * inv, acc[h][1] * inv), pack_bf16x2(acc[h][2] * inv, acc[h][3] * inv),
+                           pack_bf16x2(acc[h][4] * inv, acc[h][5] * inv), pack_bf16x2(acc[h][6] * inv, acc[h][7] * inv));
+          } else {
 #pragma unroll
-          for (int qq = 0; qq < EPV; qq += 2)
-            *reinterpret_cast<uint32_t*>(z + qq) = pack_bf16x2(acc[h][qq] * inv, acc[h][qq + 1] * inv);
+            for (int qq = 0; qq < EPV; qq += 2)
+              *reinterpret_cast<uint32_t*>(z + qq) = pack_bf16x2(acc[h][qq] * inv, acc[h][qq + 1] * inv);
+          }
         } else {
           float* z = static_cast<float*>(a.Z) + o;
 #pragma unroll

@@ -330,7 +330,11 @@ __global__ void __launch_bounds__(THREADS, 1)
           const bool plain = p.vec && n0 + 16 <= p.N && !(p.ones_col >= n0 && p.ones_col < n0 + 16);
           if (p.Yb) {
             uint16_t* d = reinterpret_cast<uint16_t*>(row) + n0;
-            if (n0 + 16 <= p.N) {
+            if (n0 + 16 <= p.N && (reinterpret_cast<uintptr_t>(d) & 31) == 0) {   // one 32-byte sector store
+              st_v8(d, pack_bf16x2(v[0], v[1]), pack_bf16x2(v[2], v[3]), pack_bf16x2(v[4], v[5]),
+                    pack_bf16x2(v[6], v[7]), pack_bf16x2(v[8], v[9]), pack_bf16x2(v[10], v[11]),
+                    pack_bf16x2(v[12], v[13]), pack_bf16x2(v[14], v[15]));
+            } else if (n0 + 16 <= p.N) {
               reinterpret_cast<uint4*>(d)[0] = make_uint4(pack_bf16x2(v[0], v[1]), pack_bf16x2(v[2], v[3]),
                                                           pack_bf16x2(v[4], v[5]), pack_bf16x2(v[6], v[7]));
               reinterpret_cast<uint4*>(d)[1] = make_uint4(pack_bf16x2(v[8], v[9]), pack_bf16x2(v[10], v[11]),
@@ -340,10 +344,18 @@ __global__ void __launch_bounds__(THREADS, 1)
             }
           } else if (plain) {
             float* d = row + n0;
+            if (!p.accumulate && (reinterpret_cast<uintptr_t>(d) & 31) == 0) {   // whole 32-byte sectors
 #pragma unroll
-            for (int j = 0; j < 16; j += 4) {
-              if (p.accumulate) red_add_v4(d + j, v[j], v[j + 1], v[j + 2], v[j + 3]);
-              else *reinterpret_cast<float4*>(d + j) = make_float4(v[j], v[j + 1], v[j + 2], v[j + 3]);
+              for (int j = 0; j < 16; j += 8)
+                st_v8(d + j, __float_as_uint(v[j]), __float_as_uint(v[j + 1]), __float_as_uint(v[j + 2]),
+                      __float_as_uint(v[j + 3]), __float_as_uint(v[j + 4]), __float_as_uint(v[j + 5]),
+                      __float_as_uint(v[j + 6]), __float_as_uint(v[j + 7]));
+            } else {
+#pragma unroll
+              for (int j = 0; j < 16; j += 4) {
+                if (p.accumulate) red_add_v4(d + j, v[j], v[j + 1], v[j + 2], v[j + 3]);
+                else *reinterpret_cast<float4*>(d + j) = make_float4(v[j], v[j + 1], v[j + 2], v[j + 3]);
+              }
             }
           } else {
 #pragma unroll
