@@ -9,6 +9,7 @@ on this GPU (C <= --emulate-max-c).  Uses bench.py's trainer / planner code.
   python tools/sweep.py papers-gat       # config 5: papers d=128, GAT 4 heads, hidden 32..1024
   python tools/sweep.py products-fanout  # fanouts [10,5], [15,10], [20,15,10]
   python tools/sweep.py products-cache   # Fig. 8c: P:163 GPU cache size sweep, C = 4
+  python tools/sweep.py friendster-cache # the same on the friendster shape (FS skew)
 """
 import argparse
 import json
@@ -38,6 +39,7 @@ SWEEPS = {
     # Fig. 8c: per-GPU cache budget (fraction of the nodes) under P:163's rules
     "products-cache": ("products", [dict(cache=f) for f in (0.0, 0.01, 0.05, 0.1, 0.25, 0.5)], 0),
     "papers-cache": ("papers", [dict(cache=f) for f in (0.0, 0.01, 0.05, 0.1, 0.25)], 0),
+    "friendster-cache": ("friendster", [dict(cache=f) for f in (0.0, 0.01, 0.05, 0.1, 0.25)], 0),
 }
 
 
