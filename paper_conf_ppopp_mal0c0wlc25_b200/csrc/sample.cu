@@ -363,6 +363,12 @@ __device__ int32_t chain_prefix(uint64_t* st, int b, int32_t agg) {
 template <class Op>
 __device__ void scan_tile(const Op& op, uint64_t* st, int b, int nb) {
   const int64_t n = op.size();
+  // the grid is sized by the capacity (the count lives on the device): tiles past the
+  // data take no part in the look-back chain, and the last tile WITH data (tile 0 of an
+  // empty scan) publishes the total -- at the products shape the hop-1 count scan has
+  // 7 real tiles out of 121
+  const int nb_real = n > 0 ? int(std::min<int64_t>(nb, ceil_div(n, int64_t(kScanTile)))) : 1;
+  if (b >= nb_real) return;   // uniform for the block
   const int64_t base = int64_t(b) * kScanTile + int64_t(threadIdx.x) * kScanItems;
   int32_t vals[kScanItems];
   int32_t s = 0;
@@ -377,7 +383,7 @@ __device__ void scan_tile(const Op& op, uint64_t* st, int b, int nb) {
     const int32_t pre = chain_prefix(st, b, tot);
     if (threadIdx.x == 0) {
       prefix = pre;
-      if (b == nb - 1) op.finish(pre + tot);
+      if (b == nb_real - 1) op.finish(pre + tot);
     }
   }
   __syncthreads();
