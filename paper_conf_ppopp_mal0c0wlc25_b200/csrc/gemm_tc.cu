@@ -68,10 +68,12 @@ struct RowParams {
   int64_t yb_pitch;
   int b_early;              // B (W) is not written by the preceding kernel: load it before the PDL wait
   int staged;               // force the staged epilogue for plain rows too (APT_EPI_STAGED=1, A/B)
+  int tma_store;            // bf16 rows, BN == 128: each warp's 32 x 64 block leaves through a TMA store
 };
 
 __global__ void __launch_bounds__(ROW_THREADS, 1)
-    rowtile_kernel(const __grid_constant__ CUtensorMap mapA, const __grid_constant__ CUtensorMap mapB, RowParams p) {
+    rowtile_kernel(const __grid_constant__ CUtensorMap mapA, const __grid_constant__ CUtensorMap mapB,
+                   const __grid_constant__ CUtensorMap mapY, RowParams p) {
   // Programmatic dependent launch: barrier init, TMEM allocation, tensor-map prefetch
   // and (b_early) the resident B load run before griddepcontrol.wait, i.e. while the
   // preceding kernel of the step drains; everything that reads its outputs (the row
@@ -89,6 +91,10 @@ __global__ void __launch_bounds__(ROW_THREADS, 1)
   uint32_t* tmem_slot = reinterpret_cast<uint32_t*>(tempty + 2);
   float* sbias = reinterpret_cast<float*>(reinterpret_cast<uint8_t*>(bars) + 128);           // [<= 256]
   float* stg_all = reinterpret_cast<float*>(reinterpret_cast<uint8_t*>(bars) + 128 + 1024);   // [8][32][17]
+  // TMA-store staging (tma_store): per epilogue warp two 4 KB buffers of 32 rows x 128 B,
+  // 1 KB aligned (the 128-byte swizzle of the output map)
+  uint8_t* ystage = reinterpret_cast<uint8_t*>(
+      (reinterpret_cast<uintptr_t>(stg_all + 8 * 32 * 17) + 1023) & ~uintptr_t(1023));
 
   const int warp = threadIdx.x >> 5, lane = lane_id();
   const int n0 = int(blockIdx.x % p.n_split) * p.BN;              // this CTA's column slice
@@ -101,6 +107,7 @@ __global__ void __launch_bounds__(ROW_THREADS, 1)
     asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
     asm volatile("prefetch.tensormap [%0];" ::"l"(reinterpret_cast<uint64_t>(&mapA)) : "memory");
     asm volatile("prefetch.tensormap [%0];" ::"l"(reinterpret_cast<uint64_t>(&mapB)) : "memory");
+    if (p.tma_store) asm volatile("prefetch.tensormap [%0];" ::"l"(reinterpret_cast<uint64_t>(&mapY)) : "memory");
   }
   if (warp == 1) tmem_alloc(tmem_slot, uint32_t(p.tmem_cols));
   fence_before();
@@ -196,6 +203,7 @@ __global__ void __launch_bounds__(ROW_THREADS, 1)
     asm volatile("bar.sync 1, 256;" ::: "memory");
     int acc = 0;
     uint32_t aph = 0;
+    int ybuf = 0;
     for (int64_t t = t0; t < ntiles; t += tstride) {
       mbar_wait(tfull + acc, aph);
       fence_after();
@@ -221,6 +229,16 @@ __global__ void __launch_bounds__(ROW_THREADS, 1)
         // latency-bound at ~10 cycles per issued instruction with 2 warps per scheduler).
         const int nch = p.BN / 16, half = (nch + 1) / 2;
         const int cb0 = h * half, cb1 = min(nch, cb0 + half);
+        // tma_store: the warp's 32 rows x 64 columns go through a shared-memory box in the
+        // output map's 128-byte swizzle (row r's 16-byte unit u at (u ^ (r & 7)) * 16: 8
+        // consecutive rows cover all banks) and leave as ONE bulk tensor store, instead of
+        // 32 rows' scattered 32-byte stores; two buffers per warp, the older store must
+        // have finished reading its buffer before the buffer is refilled
+        uint8_t* ysb = ystage + (size_t(warp - 2) * 2 + ybuf) * 4096;
+        if (p.tma_store) {
+          if (lane == 0) bulk_wait_read<1>();
+          __syncwarp();
+        }
         for (int cb = cb0; cb < cb1; cb += 4) {
           const int ng = min(4, cb1 - cb);
           uint32_t r4[4][16];
@@ -230,7 +248,7 @@ __global__ void __launch_bounds__(ROW_THREADS, 1)
 #pragma unroll
           for (int i = 0; i < 4; ++i)
             if (i < ng) tmem_wait16(r4[i]);
-          if (own) {
+          if (own || p.tma_store) {
 #pragma unroll
             for (int i = 0; i < 4; ++i) {
               if (i >= ng) break;
@@ -251,7 +269,19 @@ __global__ void __launch_bounds__(ROW_THREADS, 1)
                 for (int j = 0; j < 16; ++j) v[j] = div_rn_rcp(v[j], own_deg, own_rdeg);
               }
               const int col = n0 + c;
-              if (p.Yb) {
+              if (p.tma_store) {   // rows past M: zeros (the box still covers them)
+                const int u = 2 * (cb + i - cb0);
+                uint8_t* rp = ysb + lane * 128;
+                const bool ok = own != nullptr;
+                *reinterpret_cast<uint4*>(rp + ((u ^ (lane & 7)) << 4)) =
+                    ok ? make_uint4(pack_bf16x2(v[0], v[1]), pack_bf16x2(v[2], v[3]), pack_bf16x2(v[4], v[5]),
+                                    pack_bf16x2(v[6], v[7]))
+                       : make_uint4(0, 0, 0, 0);
+                *reinterpret_cast<uint4*>(rp + (((u + 1) ^ (lane & 7)) << 4)) =
+                    ok ? make_uint4(pack_bf16x2(v[8], v[9]), pack_bf16x2(v[10], v[11]), pack_bf16x2(v[12], v[13]),
+                                    pack_bf16x2(v[14], v[15]))
+                       : make_uint4(0, 0, 0, 0);
+              } else if (p.Yb) {
                 uint16_t* d = reinterpret_cast<uint16_t*>(own) + col;
                 if (col + 16 <= p.N && (reinterpret_cast<uintptr_t>(d) & 31) == 0) {
                   // the chunk's 32 bytes of this row as ONE sector-sized store (STG.256)
@@ -292,6 +322,15 @@ __global__ void __launch_bounds__(ROW_THREADS, 1)
         fence_before();
         mbar_arrive(tempty + acc);
         if (++acc == p.nacc) { acc = 0; aph ^= 1; }
+        if (p.tma_store) {
+          asm volatile("fence.proxy.async.shared::cta;" ::: "memory");   // st.shared -> the TMA engine
+          __syncwarp();
+          if (lane == 0) {
+            tma_store_2d(&mapY, ysb, n0 + 16 * cb0, int(t * BM + q * 32));
+            bulk_commit();
+          }
+          ybuf ^= 1;
+        }
         continue;
       }
       uint32_t r[16], rn[16];
@@ -374,6 +413,7 @@ __global__ void __launch_bounds__(ROW_THREADS, 1)
       if (++acc == p.nacc) { acc = 0; aph ^= 1; }
     }
   }
+  if (p.tma_store && warp >= 2 && lane == 0) bulk_wait_all();   // the output is written before the grid ends
   fence_before();
   __syncthreads();
   if (warp == 1) {
@@ -565,8 +605,20 @@ cudaError_t launch_tc_gemm(const TcGemmArgs& a, cudaStream_t st) {
   // two CTAs per SM when they fit (2-stage ring, one TMEM accumulator each): one CTA's
   // loads and MMAs overlap the other's epilogue
   static const int two_cta = [] { const char* v = std::getenv("APT_PROJ_2CTA"); return v ? atoi(v) : 0; }();   // off: measured slower end to end (the overlapped sampling then lands on the backward)
+  // bf16 rows in 128-column slices leave through TMA stores (APT_EPI_TMA=0: per-row 32-byte
+  // stores, A/B)
+  static const int epi_tma = [] { const char* v = std::getenv("APT_EPI_TMA"); return v ? atoi(v) : 1; }();
+  CUtensorMap my;
+  int tma_store = 0;
+  if (epi_tma && a.Yb && BN == 128 && !a.out_rank && !a.accumulate && !a.mask && !epi_staged &&
+      (a.yb_pitch * 2) % 16 == 0 && (reinterpret_cast<uintptr_t>(a.Yb) & 15) == 0 &&
+      make_map(&my, a.Yb, a.N, std::max<int64_t>(a.M_max, 1), a.yb_pitch, 64, 32))
+    tma_store = 1;
+  else
+    my = ma;   // unused
   auto smem_of = [&](int st) {
-    return 1024 + size_t(st) * A_STAGE_BYTES + size_t(nkb) * b_kb_bytes + 128 + 1024 + 8 * 32 * 17 * 4;
+    return 1024 + size_t(st) * A_STAGE_BYTES + size_t(nkb) * b_kb_bytes + 128 + 1024 + 8 * 32 * 17 * 4 +
+           (tma_store ? 1024 + 8 * 2 * 4096 : 0);
   };
   int stages = STAGES, nacc = 2, per_sm = 1;
   if (two_cta && !a.w_mn && smem_of(2) <= 113 * 1024 && BN <= 256 && tiles * n_split > sm_count()) {
@@ -578,7 +630,7 @@ cudaError_t launch_tc_gemm(const TcGemmArgs& a, cudaStream_t st) {
   while (cols < nacc * BN) cols <<= 1;
   RowParams p{a.M_max, a.M_dev, a.N, BN, nkb, cols, a.w_mn, stages, nacc, b_kb_bytes, a.bias, a.relu, a.Y, a.y_pitch,
               a.out_base, a.out_rank, a.out_row, a.accumulate, n_split, a.mask, a.mask_pitch, a.row_div_indptr,
-              a.Yb, a.yb_pitch, a.b_early, epi_staged};
+              a.Yb, a.yb_pitch, a.b_early, epi_staged, tma_store};
   const size_t smem = smem_of(stages);   // + epilogue staging
   if (smem > 227 * 1024) return cudaErrorInvalidValue;
   static bool attr_set = false;
@@ -587,7 +639,7 @@ cudaError_t launch_tc_gemm(const TcGemmArgs& a, cudaStream_t st) {
     attr_set = true;
   }
   const int grid = int(std::min<int64_t>(tiles * n_split, ((per_sm * sm_count()) / n_split) * n_split));
-  launch_pdl(rowtile_kernel, dim3(grid), dim3(ROW_THREADS), smem, st, ma, mb, p);
+  launch_pdl(rowtile_kernel, dim3(grid), dim3(ROW_THREADS), smem, st, ma, mb, my, p);
   return cudaGetLastError();
 }
 
