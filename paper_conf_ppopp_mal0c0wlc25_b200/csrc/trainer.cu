@@ -690,7 +690,10 @@ apt_status agg_l1_set(apt_trainer* t, RankState& rs, int q, cudaStream_t st, boo
   // beside the step (the sampling branch): a capped grid leaves registers for the chain
   static const int zbg = [] { const char* v = std::getenv("APT_ZBG_BPSM"); return v ? atoi(v) : 0; }();
   if (st == c->samp) a.bpsm = zbg;
-  auto rec = [&](int i) { return tap_event(t, t->ev[i], st); };
+  // the dominant kernel's own events: on the tap branch (default) or in the chain on the
+  // launching stream (APT_AGG_EV_CHAIN=1: exact bracket, but no PDL edge into the projection)
+  static const int agg_chain = [] { const char* v = std::getenv("APT_AGG_EV_CHAIN"); return v ? atoi(v) : 0; }();
+  auto rec = [&](int i) { return tap_event(t, t->ev[i], st, agg_chain != 0); };
   if (time_it) CK(c, rec(6));
   CK(c, launch_agg_fstore(a, fv, st));
   c->launches++;

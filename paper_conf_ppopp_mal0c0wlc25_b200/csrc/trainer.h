@@ -240,10 +240,10 @@ namespace apt {
 // an external record node placed IN the chain cost the step ~5 us per event (measured
 // with tools/timeline.py: the next kernel waited for the full drain + the node).
 // APT_TAP_EVENTS=0 puts them back in the chain (A/B).
-inline cudaError_t tap_event(apt_trainer* t, cudaEvent_t ev, cudaStream_t st) {
+inline cudaError_t tap_event(apt_trainer* t, cudaEvent_t ev, cudaStream_t st, bool in_chain = false) {
   static const int tap = [] { const char* v = std::getenv("APT_TAP_EVENTS"); return v ? atoi(v) : 1; }();
   if (!t->capturing) return cudaEventRecord(ev, st);
-  if (!tap) return cudaEventRecordWithFlags(ev, st, cudaEventRecordExternal);
+  if (!tap || in_chain) return cudaEventRecordWithFlags(ev, st, cudaEventRecordExternal);
   apt_ctx* c = t->ctx;
   cudaError_t e = cudaEventRecord(c->ev_tap, st);
   if (e == cudaSuccess) e = cudaStreamWaitEvent(c->tap, c->ev_tap, 0);
