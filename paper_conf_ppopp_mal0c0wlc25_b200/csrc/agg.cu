@@ -21,10 +21,8 @@ namespace apt {
 template <int EPV>
 __device__ __forceinline__ void accumulate_vec(float* acc, uint4 raw) {
   if constexpr (EPV == 8) {
-    acc[0] += bf16_lo(raw.x); acc[1] += bf16_hi(raw.x);
-    acc[2] += bf16_lo(raw.y); acc[3] += bf16_hi(raw.y);
-    acc[4] += bf16_lo(raw.z); acc[5] += bf16_hi(raw.z);
-    acc[6] += bf16_lo(raw.w); acc[7] += bf16_hi(raw.w);
+    acc_bf16x2(acc[0], acc[1], raw.x); acc_bf16x2(acc[2], acc[3], raw.y);
+    acc_bf16x2(acc[4], acc[5], raw.z); acc_bf16x2(acc[6], acc[7], raw.w);
   } else {
     acc[0] += __uint_as_float(raw.x); acc[1] += __uint_as_float(raw.y);
     acc[2] += __uint_as_float(raw.z); acc[3] += __uint_as_float(raw.w);
@@ -280,6 +278,102 @@ __global__ void __launch_bounds__(256, MINB) agg_l1_pf_kernel(AggArgs a, EllFsto
   }
 }
 
+// The same gather for a single-shard view (fv.loc == nullptr: GDP at C = 1, NFP's column
+// shard, the benchmark): every row sits in base[0], so a lane broadcasts a 32-bit ROW
+// INDEX (padding edges: the shard's zero row fv.zrow) instead of a 64-bit pointer, and an
+// edge's load address is one IMAD.WIDE off the lane's column base: per edge and lane one
+// shuffle, one address op, one non-coherent 16-B load and 8 mixed-precision adds (the
+// pointer form issued two shuffles, two selects and a 64-bit add, and 16 unpack + add
+// instructions; ncu had the kernel issue-active 68 % of its cycles).
+template <int EPV, int NB, int MINB>
+__global__ void __launch_bounds__(256, MINB) agg_l1_flat_kernel(AggArgs a, EllFstoreSrc src) {
+  APT_PDL_PROLOGUE();
+  const int lane = lane_id();
+  const int sub = lane >> 4, l = lane & 15;
+  const int64_t n_dst = *a.n_dst;
+  const int V = int(ceil_div(a.dim, EPV));
+  const int lv = l < V ? l : 0;
+  const int k = src.k;
+  // the lane's column base as one opaque 64-bit value, so each edge's address is a single
+  // IMAD.WIDE.U32 (row * row_bytes + base) rather than a product plus a separate base add
+  uint64_t cbase;
+  asm("mov.b64 %0, %1;" : "=l"(cbase) : "l"(reinterpret_cast<uint64_t>(src.fv.base[0]) + uint64_t(lv) * 16u));
+  const uint32_t rb = uint32_t(src.row_bytes);
+  const int zr = int(src.fv.zrow);
+  const int64_t nwarps = int64_t(gridDim.x) * (blockDim.x >> 5);
+  int64_t w = (int64_t(blockIdx.x) * blockDim.x + threadIdx.x) >> 5;
+  int cnt_n = 0, u_n = zr;
+  {
+    const int64_t i = w * 2 + sub;
+    if (i < n_dst) { cnt_n = src.count(i); if (l < k) u_n = src.node(i * k + l); }
+  }
+  for (; w * 2 < n_dst; w += nwarps) {
+    const int64_t i = w * 2 + sub;
+    const bool valid = i < n_dst;
+    const int cnt = cnt_n, u = u_n;
+    {   // next pair's count and ids, consumed one iteration later
+      const int64_t i2 = (w + nwarps) * 2 + sub;
+      cnt_n = 0; u_n = zr;
+      if (i2 < n_dst) { cnt_n = src.count(i2); if (l < k) u_n = src.node(i2 * k + l); }
+    }
+    const int cmax = max(cnt, __shfl_xor_sync(0xffffffffu, cnt, 16));
+    float acc[EPV];
+#pragma unroll
+    for (int q = 0; q < EPV; ++q) acc[q] = 0.f;
+    const bool keep = l < cnt && (!a.filt_part || a.filt_part[u] == a.keep_part);
+    const uint32_t ur = uint32_t(keep ? u : zr);
+#pragma unroll 1
+    for (int j = 0; j < cmax; j += NB) {
+      uint4 v[NB];
+#pragma unroll
+      for (int q = 0; q < NB; ++q) {
+        uint32_t uq = __shfl_sync(0xffffffffu, ur, sub * 16 + ((j + q) & 15));
+        if constexpr ((16 % NB) != 0) if (j + q >= 16) uq = uint32_t(zr);
+        v[q] = __ldg(reinterpret_cast<const uint4*>(cbase + uint64_t(uq) * rb));   // L1-allocating: the zero row stays in L1
+      }
+#pragma unroll
+      for (int q = 0; q < NB; ++q) accumulate_vec<EPV>(acc, v[q]);
+    }
+    if (!valid || l >= V) continue;
+    if (a.z_ones && l == 0) {
+      if (a.z_bf16) a.z_bf16[i * a.z_bf16_pitch + a.dim] = 0x3F80;
+      else if (a.z_f32) a.z_f32[i * a.z_f32_pitch + a.dim] = 1.f;
+    }
+    const float fdeg = float(a.deg_override ? a.deg_override[i] : cnt);
+    const float rdeg = fdeg > 0.f ? __frcp_rn(fdeg) : 0.f;
+    float z[EPV];
+#pragma unroll
+    for (int q = 0; q < EPV; ++q) z[q] = fdeg > 0.f ? div_rn_rcp(acc[q], fdeg, rdeg) : 0.f;
+    const int c0 = l * EPV;
+    const bool full = c0 + EPV <= a.dim;
+    if (a.z_f32) {
+      float* o = a.z_f32 + i * a.z_f32_pitch + c0;
+#pragma unroll
+      for (int q = 0; q < EPV; ++q)
+        if (full || c0 + q < a.dim) o[q] = z[q];
+    }
+    if (a.z_bf16) {
+      uint16_t* o = a.z_bf16 + i * a.z_bf16_pitch + c0;
+      if (full) {
+        if constexpr (EPV == 8) {
+          *reinterpret_cast<uint4*>(o) = make_uint4(pack_bf16x2(z[0], z[1]), pack_bf16x2(z[2], z[3]),
+                                                    pack_bf16x2(z[4], z[5]), pack_bf16x2(z[6], z[7]));
+        } else {
+          *reinterpret_cast<uint2*>(o) = make_uint2(pack_bf16x2(z[0], z[1]), pack_bf16x2(z[2], z[3]));
+        }
+      } else {
+#pragma unroll
+        for (int q = 0; q < EPV; ++q) {
+          if (c0 + q < a.dim) {
+            __nv_bfloat16 h = __float2bfloat16_rn(z[q]);
+            o[q] = *reinterpret_cast<uint16_t*>(&h);
+          }
+        }
+      }
+    }
+  }
+}
+
 cudaError_t launch_agg_fstore(const AggArgs& a, const FeatView& fv, cudaStream_t st) {
   EllFstoreSrc s{a.cnt, a.nbr, a.k, fv, fv.pitch * (fv.dtype == kBF16 ? 2 : 4)};
   AggArgs b = a;
@@ -290,6 +384,27 @@ cudaError_t launch_agg_fstore(const AggArgs& a, const FeatView& fv, cudaStream_t
   // grid one resident wave: every warp streams several row pairs, so the one-ahead index
   // prefetch pays and there is no partial last wave (A/B in DESIGN §8: 30.2 us in the
   // step vs 32.4 at 16 blocks per SM and 33.2-34.5 for NB 4 / 8 and 48 registers)
+  static const int flat_ok = [] { const char* v = std::getenv("APT_AGG_FLAT"); return v ? atoi(v) : 1; }();
+  if (V <= 16 && b.k <= 16 && !fv.loc && fv.zrow >= 0 && flat_ok) {
+    if (fv.dtype == kBF16) {
+      // 10 loads in flight per lane (a fanout-10 row in one round) at 3 blocks per SM (75
+      // registers): A/B in the step 27.8 vs 28.9 us for 5 loads at 4 blocks per SM; 10 at 4
+      // (spills) 34.0, 5 at 5 29.5, 4 at 5 29.6 (APT_FLAT_VAR 1-4)
+      static const int var = [] { const char* v = std::getenv("APT_FLAT_VAR"); return v ? atoi(v) : 2; }();
+      auto kern = var == 1 ? agg_l1_flat_kernel<8, 10, 4> : var == 0 ? agg_l1_flat_kernel<8, 5, 4>
+                : var == 3 ? agg_l1_flat_kernel<8, 5, 5> : var == 4 ? agg_l1_flat_kernel<8, 4, 5>
+                : agg_l1_flat_kernel<8, 10, 3>;
+      const int64_t blocks = grid_cap(ceil_div(ceil_div(b.max_dst, 2) * 32, 256),
+                                      b.bpsm > 0 ? b.bpsm : resident_blocks(kern, 256));
+      launch_pdl(kern, dim3(blocks), dim3(256), 0, st, b, s);
+    } else {
+      auto kern = agg_l1_flat_kernel<4, 4, 6>;
+      const int64_t blocks = grid_cap(ceil_div(ceil_div(b.max_dst, 2) * 32, 256),
+                                      b.bpsm > 0 ? b.bpsm : resident_blocks(kern, 256));
+      launch_pdl(kern, dim3(blocks), dim3(256), 0, st, b, s);
+    }
+    return cudaGetLastError();
+  }
   if (V <= 16 && b.k <= 16) {
     if (fv.dtype == kBF16) {
       auto kern = agg_l1_pf_kernel<8, 5, 4>;

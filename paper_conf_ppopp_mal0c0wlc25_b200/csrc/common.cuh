@@ -138,11 +138,19 @@ __device__ __forceinline__ T warp_sum(T v) {
 
 __device__ __forceinline__ float bf16_lo(uint32_t v) { return __uint_as_float(v << 16); }
 __device__ __forceinline__ float bf16_bits_to_float(uint16_t b) { return __uint_as_float(uint32_t(b) << 16); }
+// acc0 += lo(w), acc1 += hi(w) for a packed bf16 pair: the mixed-precision add
+// (add.rn.f32.bf16 -> FHADD.BF16 with an .H0/.H1 operand select) is one instruction per
+// element where the unpack (shift / mask) + FADD form took two; the bf16 value converts to
+// fp32 exactly, so the sums are bit-identical to the unpacked form
+__device__ __forceinline__ void acc_bf16x2(float& a0, float& a1, uint32_t w) {
+  asm("{\n\t.reg .b16 lo, hi;\n\tmov.b32 {lo, hi}, %2;\n\t"
+      "add.rn.f32.bf16 %0, lo, %0;\n\tadd.rn.f32.bf16 %1, hi, %1;\n\t}"
+      : "+f"(a0), "+f"(a1) : "r"(w));
+}
+
 __device__ __forceinline__ void accumulate_bf16x8(float* acc, uint4 raw) {
-  acc[0] += __uint_as_float(raw.x << 16); acc[1] += __uint_as_float(raw.x & 0xFFFF0000u);
-  acc[2] += __uint_as_float(raw.y << 16); acc[3] += __uint_as_float(raw.y & 0xFFFF0000u);
-  acc[4] += __uint_as_float(raw.z << 16); acc[5] += __uint_as_float(raw.z & 0xFFFF0000u);
-  acc[6] += __uint_as_float(raw.w << 16); acc[7] += __uint_as_float(raw.w & 0xFFFF0000u);
+  acc_bf16x2(acc[0], acc[1], raw.x); acc_bf16x2(acc[2], acc[3], raw.y);
+  acc_bf16x2(acc[4], acc[5], raw.z); acc_bf16x2(acc[6], acc[7], raw.w);
 }
 __device__ __forceinline__ uint16_t bf16_bits(float x) {
   __nv_bfloat16 h = __float2bfloat16_rn(x);

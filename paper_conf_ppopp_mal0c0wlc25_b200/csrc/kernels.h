@@ -89,6 +89,8 @@ struct FeatView {
   int dim;                     // logical columns to aggregate
   int col0;                    // first column inside the stored row
   DType dtype;
+  int64_t zrow;                // single-shard view (loc == nullptr): index of an all-zero row
+                               // in base[0] (padding edges read it), -1 if there is none
 };
 
 // Edge source for aggregation: either an ELL (cnt + nbr global ids, fixed stride

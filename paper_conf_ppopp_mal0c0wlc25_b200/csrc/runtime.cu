@@ -310,7 +310,9 @@ apt_status apt_fstore_create_tiered(apt_ctx* c, const apt_graph* g, apt_strategy
   for (int r = 0; r < C; ++r) {
     // emulated: all shards here; multi-process: only the own shard is local
     if (!c->emulated && r != c->rank) continue;
-    f->shard[r] = f->arena.alloc<uint8_t>(std::max<int64_t>(f->rows[r], 1) * f->pitch[r] * int64_t(esz), true);
+    // one zero-filled row past the shard's rows: padding edges of the layer-1 gather read
+    // it (FeatView::zrow), so every load of a batch is a plain global load
+    f->shard[r] = f->arena.alloc<uint8_t>((f->rows[r] + 1) * f->pitch[r] * int64_t(esz), true);
     if (!f->shard[r] || !ids_dev) {
       apt_fstore_destroy(f);
       return set_err(c, APT_E_OOM, "apt_fstore_create: out of device memory");
@@ -423,6 +425,7 @@ namespace apt {
 // locally or through its peer pointer).
 FeatView feat_view(const apt_fstore* f, int r) {
   FeatView v{};
+  v.zrow = -1;
   const bool rows_sharded = f->layout != APT_NFP && f->world > 1;
   for (int o = 0; o < f->world; ++o) v.base[o] = f->shard[o];
   if (f->tiered) {
@@ -442,6 +445,7 @@ FeatView feat_view(const apt_fstore* f, int r) {
     v.loc = nullptr;
     v.pitch = f->pitch[s];
     v.dim = f->col_hi[s] - f->col_lo[s];
+    v.zrow = f->rows[s];
   }
   v.col0 = 0;
   v.dtype = f->dtype;
