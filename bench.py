@@ -417,9 +417,14 @@ def run_apt(args, cfg):
                      "frac": (achieved / hbm_peak) if achieved else None, "traffic": traffic,
                      "traffic_source": traffic_src, "algorithmic_bytes_per_launch": sum(agg_bytes) / len(agg_bytes),
                      "kernel": "gat_fwd_kernel (layer-1 fused gather+attention+weighted sums)" if GAT_HEADS
-                     else "agg_l1_pf_kernel (layer-1 fused gather+mean)",
+                     else "agg_l1_flat_kernel (layer-1 fused gather+mean)",
                      "peak_source": "MEASURED_PEAKS.json hbm_gbs" if peaks else "fallback 6.65 TB/s",
-                     "share_of_step": mean_agg / ms_local},
+                     "share_of_step": mean_agg / ms_local,
+                     # context, not the peak: random 208-B row reads measured alone on one B200
+                     # (tools/micro/gather_ceiling.cu, steady state over a 10x table)
+                     "random_row_ceiling": {"gbs": RANDOM_ROW_CEILING_GBS, "frac": achieved / RANDOM_ROW_CEILING_GBS,
+                                            "source": "profiles/r02_gather_ceiling.txt"}
+                     if not GAT_HEADS and achieved else None},
         "step_roofline": step_roofline(step_bytes, hbm_peak, ms) if step_bytes else None,
         "phases_ms": {"sample": phase_mean[0], "layer1_fwd": phase_mean[1], "upper_fwd_loss": phase_mean[2],
                       "backward": phase_mean[3], "allreduce_sgd": phase_mean[4], "agg_kernel": phase_mean[5]},
@@ -622,6 +627,9 @@ def step_phase_bytes(ctx, gr, g, tr, cfg, rank, step, bf):
     ph["sgd"] = nparam * (4 + 4 + 4 + b_w)
     b.close()
     return ph
+
+
+RANDOM_ROW_CEILING_GBS = 3505.0   # x10 uniq_sorted / uniq_random, unroll 8, bpsm 4 (profiles/r02_gather_ceiling.txt)
 
 
 def step_roofline(step_bytes, peak_gbs, ms):

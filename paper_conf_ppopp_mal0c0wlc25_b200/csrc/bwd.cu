@@ -302,6 +302,101 @@ __global__ void __launch_bounds__(256) pull_bwd_b8_kernel(PullArgs a) {
   }
 }
 
+// The same pull as a resident wave of warps, each streaming row groups with the next
+// group's CSC bounds and its first 32 in-edges loaded one iteration ahead: a row group's
+// dependent chain (CSC pointer -> in-edge -> dZ row) shrinks to the dZ row loads, where the
+// block-per-group form paid all three round trips per group (layer-1 rows have ~1.3
+// in-edges each, so the chain, not the bytes, set the time).
+template <int VP, int R>
+__global__ void __launch_bounds__(256) pull_bwd_b8_pf_kernel(PullArgs a) {
+  APT_PDL_PROLOGUE();
+  const int lane = lane_id();
+  const int64_t n = *a.n_src;
+  const int V8 = a.dim >> 3;
+  const int64_t nwarps = int64_t(gridDim.x) * (blockDim.x >> 5);
+  const int64_t rows_out = std::min<int64_t>(a.max_src, round_up(n, 64));
+  int64_t u0 = ((int64_t(blockIdx.x) * blockDim.x + threadIdx.x) >> 5) * R;
+  int e0[R], cnt[R], vv[R];
+#pragma unroll
+  for (int r = 0; r < R; ++r) {
+    const int64_t u = u0 + r;
+    e0[r] = 0; cnt[r] = 0;
+    if (u < n) { e0[r] = a.csc_ptr[u]; cnt[r] = a.csc_ptr[u + 1] - e0[r]; }
+  }
+#pragma unroll
+  for (int r = 0; r < R; ++r) vv[r] = lane < cnt[r] ? a.csc_dst[e0[r] + lane].x : 0;
+  for (; u0 < rows_out; u0 += nwarps * R) {
+    uint4 hm[R][VP];
+    int e0n[R], cntn[R];
+#pragma unroll
+    for (int r = 0; r < R; ++r) {
+      const int64_t u = u0 + r, un = u0 + nwarps * R + r;
+#pragma unroll
+      for (int p = 0; p < VP; ++p) {
+        const int j = lane + 32 * p;
+        hm[r][p] = (u < n && j < V8) ? __ldg(reinterpret_cast<const uint4*>(a.hb + u * a.hb_pitch + j * 8))
+                                     : make_uint4(0, 0, 0, 0);
+      }
+      e0n[r] = 0; cntn[r] = 0;
+      if (un < n) { e0n[r] = a.csc_ptr[un]; cntn[r] = a.csc_ptr[un + 1] - e0n[r]; }
+    }
+    float acc[R][VP][8];
+#pragma unroll
+    for (int r = 0; r < R; ++r)
+#pragma unroll
+      for (int p = 0; p < VP; ++p)
+#pragma unroll
+        for (int q = 0; q < 8; ++q) acc[r][p][q] = 0.f;
+    int cmax = cnt[0];
+#pragma unroll
+    for (int r = 1; r < R; ++r) cmax = max(cmax, cnt[r]);
+    for (int c0 = 0; c0 < cmax; c0 += 32) {
+      int v[R];
+#pragma unroll
+      for (int r = 0; r < R; ++r)
+        v[r] = c0 == 0 ? vv[r] : (c0 + lane < cnt[r] ? a.csc_dst[e0[r] + c0 + lane].x : 0);
+      const int m = min(32, cmax - c0);
+      for (int e = 0; e < m; ++e) {
+#pragma unroll
+        for (int r = 0; r < R; ++r) {
+          const int w = __shfl_sync(0xffffffffu, v[r], e);
+          if (c0 + e >= cnt[r]) continue;
+#pragma unroll
+          for (int p = 0; p < VP; ++p) {
+            const int j = lane + 32 * p;
+            if (j < V8) {
+              const uint4 z = *reinterpret_cast<const uint4*>(a.dzb + int64_t(w) * a.dzb_pitch + j * 8);
+              accumulate_bf16x8(acc[r][p], z);
+            }
+          }
+        }
+      }
+    }
+    // the next group's first in-edges (its CSC bounds arrived during this group's sums)
+#pragma unroll
+    for (int r = 0; r < R; ++r) {
+      e0[r] = e0n[r]; cnt[r] = cntn[r];
+      vv[r] = lane < cnt[r] ? a.csc_dst[e0[r] + lane].x : 0;
+    }
+#pragma unroll
+    for (int r = 0; r < R; ++r) {
+      const int64_t u = u0 + r;
+      if (u >= rows_out) continue;
+#pragma unroll
+      for (int p = 0; p < VP; ++p) {
+        const int j = lane + 32 * p;
+        if (j >= V8) continue;
+        const float* x = acc[r][p];
+        const uint4 o = make_uint4(pack_bf16x2(x[0], x[1]) & __vcmpgts2(hm[r][p].x, 0u),
+                                   pack_bf16x2(x[2], x[3]) & __vcmpgts2(hm[r][p].y, 0u),
+                                   pack_bf16x2(x[4], x[5]) & __vcmpgts2(hm[r][p].z, 0u),
+                                   pack_bf16x2(x[6], x[7]) & __vcmpgts2(hm[r][p].w, 0u));
+        *reinterpret_cast<uint4*>(a.gb + u * a.gb_pitch + j * 8) = o;
+      }
+    }
+  }
+}
+
 cudaError_t launch_pull_bwd(const PullArgs& a, cudaStream_t st) {
   if (a.dim > 512) {   // wide rows: column chunks of 512 (128 fp32 vectors per lane group)
     for (int c0 = 0; c0 < a.dim; c0 += 512) {
@@ -333,6 +428,16 @@ cudaError_t launch_pull_bwd(const PullArgs& a, cudaStream_t st) {
     const int64_t blocks = std::max<int64_t>(
         1, std::min<int64_t>(ceil_div(ceil_div(round_up(a.max_src, 64), Rr) * 32, 256), int64_t(num_sms()) * bpsm));
     const int V8 = a.dim >> 3;
+    static const int pf = [] { const char* e = std::getenv("APT_PULL_PF"); return e ? atoi(e) : 1; }();
+    if (pf && V8 <= 32) {
+      // one resident wave (APT_PULL_PF_BPSM caps blocks per SM: A/B knob)
+      static const int pbpsm = [] { const char* e = std::getenv("APT_PULL_PF_BPSM"); return e ? atoi(e) : 0; }();
+      auto kern = Rr == 4 ? pull_bwd_b8_pf_kernel<1, 4> : pull_bwd_b8_pf_kernel<1, 2>;
+      const int64_t pblocks = grid_cap(ceil_div(ceil_div(round_up(a.max_src, 64), Rr) * 32, 256),
+                                       pbpsm > 0 ? pbpsm : resident_blocks(kern, 256));
+      launch_pdl(kern, dim3(pblocks), dim3(256), 0, st, a);
+      return cudaGetLastError();
+    }
     if (Rr == 4) {
       if (V8 <= 32) launch_pdl(pull_bwd_b8_kernel<1, 4>, dim3(blocks), dim3(256), 0, st, a);
       else launch_pdl(pull_bwd_b8_kernel<2, 4>, dim3(blocks), dim3(256), 0, st, a);
