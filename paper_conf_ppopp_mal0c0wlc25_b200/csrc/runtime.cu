@@ -34,6 +34,9 @@ static void ctx_free(apt_ctx* c) {
   release_exported(c);
   if (c->side) { cudaStreamSynchronize(c->side); cudaStreamDestroy(c->side); }
   if (c->samp) { cudaStreamSynchronize(c->samp); cudaStreamDestroy(c->samp); }
+  if (c->samp2) { cudaStreamSynchronize(c->samp2); cudaStreamDestroy(c->samp2); }
+  if (c->ev_sfork) cudaEventDestroy(c->ev_sfork);
+  if (c->ev_sjoin) cudaEventDestroy(c->ev_sjoin);
   if (c->tap) { cudaStreamSynchronize(c->tap); cudaStreamDestroy(c->tap); }
   if (c->ev_tap) cudaEventDestroy(c->ev_tap);
   if (c->ev_tapj) cudaEventDestroy(c->ev_tapj);
@@ -109,6 +112,9 @@ apt_status apt_ctx_create(int rank, int world, int device, void* stream, apt_ctx
   static const int samp_hi = [] { const char* v = std::getenv("APT_SAMP_PRIO"); return v ? atoi(v) : 0; }();
   cudaStreamCreateWithPriority(&c->samp, cudaStreamNonBlocking, samp_hi ? prio_hi : prio_lo);
   cudaStreamCreateWithPriority(&c->tap, cudaStreamNonBlocking, prio_hi);
+  cudaStreamCreateWithPriority(&c->samp2, cudaStreamNonBlocking, samp_hi ? prio_hi : prio_lo);
+  cudaEventCreateWithFlags(&c->ev_sfork, cudaEventDisableTiming);
+  cudaEventCreateWithFlags(&c->ev_sjoin, cudaEventDisableTiming);
   cudaEventCreateWithFlags(&c->ev_tap, cudaEventDisableTiming);
   cudaEventCreateWithFlags(&c->ev_tapj, cudaEventDisableTiming);
   cudaEventCreateWithFlags(&c->ev_pfork, cudaEventDisableTiming);

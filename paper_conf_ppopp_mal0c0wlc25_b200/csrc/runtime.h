@@ -73,6 +73,8 @@ struct apt_ctx {
   bool own_stream = false;
   cudaStream_t side = nullptr;           // forked branch of a step (weight gradients off the critical path)
   cudaStream_t samp = nullptr;           // sampling of the next step (pipelined trainer)
+  cudaStream_t samp2 = nullptr;          // its block transposes, off the sampling chain (APT_BG_CSC_FORK)
+  cudaEvent_t ev_sfork = nullptr, ev_sjoin = nullptr;
   cudaStream_t tap = nullptr;            // captured graphs: timing events hang off the chain here
   cudaEvent_t ev_tap = nullptr, ev_tapj = nullptr;
   cudaEvent_t ev_pfork = nullptr, ev_pjoin = nullptr;

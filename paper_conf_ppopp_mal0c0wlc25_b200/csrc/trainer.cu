@@ -622,6 +622,15 @@ apt_status phase_sample(apt_trainer* t, RankState& rs, SampleSet& ss, bool from_
       c->launches += 3;
       // transpose of this block for the pull-form mean backward
       cudaStream_t cs_st = st;
+      // the background (next-step) sampling: the transposes on a second low-priority stream,
+      // so the next hop's sampling does not wait for them (joined at the branch's end)
+      static const int bg_fork = [] { const char* v = std::getenv("APT_BG_CSC_FORK"); return v ? atoi(v) : 0; }();
+      if (!fork_csc && bg_fork && st == c->samp) {
+        CK(c, cudaEventRecord(c->ev_sfork, st));
+        CK(c, cudaStreamWaitEvent(c->samp2, c->ev_sfork, 0));
+        cs_st = c->samp2;
+        t->bg_csc_forked = true;
+      }
       if (fork_csc) {
         CK(c, cudaEventRecord(c->ev_fork, st));
         CK(c, cudaStreamWaitEvent(c->side, c->ev_fork, 0));
@@ -971,6 +980,11 @@ apt_status pipelined_body(apt_trainer* t, int p, int update, uint64_t next) {
     apt_status s2 = sample_all(t, p ^ 1, false, c->samp, false);
     if (s2 == APT_OK && t->z_prefetch && t->z_where == 1) s2 = prefetch_z(t, p ^ 1, c->samp);   // next batch's layer-1 Z
     if (s2 != APT_OK) return s2;
+    if (t->bg_csc_forked) {
+      CK(c, cudaEventRecord(c->ev_sjoin, c->samp2));
+      CK(c, cudaStreamWaitEvent(c->samp, c->ev_sjoin, 0));
+      t->bg_csc_forked = false;
+    }
     CK(c, cudaEventRecord(c->ev_pjoin, c->samp));
     return APT_OK;
   });
@@ -1484,6 +1498,11 @@ static apt_status step_host_pipelined_impl(apt_trainer* t, const int64_t* next_b
       apt_status s2 = sample_all(t, q, true, c->samp, false);
       if (s2 == APT_OK && t->z_prefetch && t->z_where == 1) s2 = prefetch_z(t, q, c->samp);
       if (s2 != APT_OK) return s2;
+      if (t->bg_csc_forked) {
+        CK(c, cudaEventRecord(c->ev_sjoin, c->samp2));
+        CK(c, cudaStreamWaitEvent(c->samp, c->ev_sjoin, 0));
+        t->bg_csc_forked = false;
+      }
       CK(c, cudaEventRecord(c->ev_pjoin, c->samp));
       return APT_OK;
     });

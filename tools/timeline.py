@@ -54,12 +54,15 @@ def main():
     if args.no_pipeline:
         tr.set_pipeline(False)
     flush = torch.empty(256 << 20, dtype=torch.uint8, device="cuda")
+    flush_rd = torch.ones(64 << 20, dtype=torch.int32, device="cuda")   # bench.py --flush write+read
+    flush_out = torch.empty((), dtype=torch.int32, device="cuda")
     for i in range(10):
         tr.step(i)
     torch.cuda.synchronize()
     with profile(activities=[ProfilerActivity.CUDA]) as prof:
         for i in range(args.steps):
             flush.zero_()
+            torch.amax(flush_rd, dim=0, out=flush_out)
             if args.sync_flush:
                 torch.cuda.synchronize()
             tr.step(10 + i)
@@ -75,6 +78,8 @@ def main():
             cur = []
             steps.append(cur)
             fl_end.append(e["ts"] + e["dur"])
+        elif cur is not None and not cur and "reduce_kernel" in e["name"]:   # the flush's read pass
+            fl_end[-1] = e["ts"] + e["dur"]
         elif cur is not None:
             cur.append(e)
     for si, st in enumerate(steps[1:3], 1):
