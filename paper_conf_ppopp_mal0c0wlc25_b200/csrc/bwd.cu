@@ -307,7 +307,7 @@ __global__ void __launch_bounds__(256) pull_bwd_b8_kernel(PullArgs a) {
 // dependent chain (CSC pointer -> in-edge -> dZ row) shrinks to the dZ row loads, where the
 // block-per-group form paid all three round trips per group (layer-1 rows have ~1.3
 // in-edges each, so the chain, not the bytes, set the time).
-template <int VP, int R>
+template <int VP, int R, int EB>
 __global__ void __launch_bounds__(256) pull_bwd_b8_pf_kernel(PullArgs a) {
   APT_PDL_PROLOGUE();
   const int lane = lane_id();
@@ -356,20 +356,33 @@ __global__ void __launch_bounds__(256) pull_bwd_b8_pf_kernel(PullArgs a) {
       for (int r = 0; r < R; ++r)
         v[r] = c0 == 0 ? vv[r] : (c0 + lane < cnt[r] ? a.csc_dst[e0[r] + c0 + lane].x : 0);
       const int m = min(32, cmax - c0);
-      for (int e = 0; e < m; ++e) {
+      // EB in-edges of every row of the group in flight at once (predicated loads; the
+      // rows average ~1.3 in-edges, so one batch usually covers the group)
+      for (int eb = 0; eb < m; eb += EB) {
+        uint4 z[EB][R][VP];
+        bool ok[EB][R];
 #pragma unroll
-        for (int r = 0; r < R; ++r) {
-          const int w = __shfl_sync(0xffffffffu, v[r], e);
-          if (c0 + e >= cnt[r]) continue;
+        for (int q = 0; q < EB; ++q)
 #pragma unroll
-          for (int p = 0; p < VP; ++p) {
-            const int j = lane + 32 * p;
-            if (j < V8) {
-              const uint4 z = *reinterpret_cast<const uint4*>(a.dzb + int64_t(w) * a.dzb_pitch + j * 8);
-              accumulate_bf16x8(acc[r][p], z);
+          for (int r = 0; r < R; ++r) {
+            const int e = eb + q;
+            const int w = __shfl_sync(0xffffffffu, v[r], e & 31);
+            ok[q][r] = e < m && c0 + e < cnt[r];
+            const uint16_t* zr = a.dzb + int64_t(w) * a.dzb_pitch;
+#pragma unroll
+            for (int p = 0; p < VP; ++p) {
+              const int j = lane + 32 * p;
+              z[q][r][p] = (ok[q][r] && j < V8) ? __ldg(reinterpret_cast<const uint4*>(zr + j * 8))
+                                                : make_uint4(0, 0, 0, 0);
             }
           }
-        }
+#pragma unroll
+        for (int q = 0; q < EB; ++q)
+#pragma unroll
+          for (int r = 0; r < R; ++r)
+            if (ok[q][r])
+#pragma unroll
+              for (int p = 0; p < VP; ++p) accumulate_bf16x8(acc[r][p], z[q][r][p]);
       }
     }
     // the next group's first in-edges (its CSC bounds arrived during this group's sums)
@@ -432,8 +445,14 @@ cudaError_t launch_pull_bwd(const PullArgs& a, cudaStream_t st) {
     if (pf && V8 <= 32) {
       // one resident wave (APT_PULL_PF_BPSM caps blocks per SM: A/B knob)
       static const int pbpsm = [] { const char* e = std::getenv("APT_PULL_PF_BPSM"); return e ? atoi(e) : 0; }();
-      auto kern = Rr == 4 ? pull_bwd_b8_pf_kernel<1, 4> : pull_bwd_b8_pf_kernel<1, 2>;
-      const int64_t pblocks = grid_cap(ceil_div(ceil_div(round_up(a.max_src, 64), Rr) * 32, 256),
+      // in-edges in flight per row (APT_PULL_EB) x rows per warp (APT_PULL_ROWS): A/B knobs
+      static const int eb = [] { const char* e = std::getenv("APT_PULL_EB"); return e ? atoi(e) : 1; }();   // 1 / 2 / 4: 0.1627 / 0.1673 / 0.1786 ms (A/B)
+      auto kern = Rr == 4 ? pull_bwd_b8_pf_kernel<1, 4, 1>
+                : (rr == 1 ? (eb >= 4 ? pull_bwd_b8_pf_kernel<1, 1, 4> : pull_bwd_b8_pf_kernel<1, 1, 2>)
+                : (eb >= 4 ? pull_bwd_b8_pf_kernel<1, 2, 4> : eb == 2 ? pull_bwd_b8_pf_kernel<1, 2, 2>
+                : pull_bwd_b8_pf_kernel<1, 2, 1>));
+      const int Rk = rr == 1 ? 1 : Rr;
+      const int64_t pblocks = grid_cap(ceil_div(ceil_div(round_up(a.max_src, 64), Rk) * 32, 256),
                                        pbpsm > 0 ? pbpsm : resident_blocks(kern, 256));
       launch_pdl(kern, dim3(pblocks), dim3(256), 0, st, a);
       return cudaGetLastError();

@@ -680,7 +680,13 @@ cudaError_t launch_tc_wgrad(const TcWgradArgs& a, cudaStream_t st) {
   const int64_t kbs = std::max<int64_t>(1, ceil_div(a.rows_max, BK));
   // row splits: one CTA per SM (A/B APT_WG_SPLITS_PER_SM = 1 / 2: 0.207 / 0.224 ms; ring depth 3 / 6: same)
   static const int per_sm = [] { const char* v = std::getenv("APT_WG_SPLITS_PER_SM"); return v ? std::max(1, atoi(v)) : 1; }();
-  const int splits = int(std::max<int64_t>(1, std::min<int64_t>(kbs, int64_t(per_sm) * sm_count() / mt)));
+  // at least APT_WG_MIN_KB k-blocks per split: a small block (the upper layers' few thousand
+  // rows) over every SM leaves each CTA ~1 k-block and every dW element ~74 contended
+  // reductions; fewer, longer splits pipeline their loads and reduce less
+  // (A/B on the products step, 2 x 2 runs: 1 / 4 / 8 / 16 -> 0.1638 / 0.1630 / 0.1642 / 0.1663 ms)
+  static const int min_kb = [] { const char* v = std::getenv("APT_WG_MIN_KB"); return v ? std::max(1, atoi(v)) : 4; }();
+  const int splits = int(std::max<int64_t>(
+      1, std::min<int64_t>(ceil_div(kbs, int64_t(min_kb)), int64_t(per_sm) * sm_count() / mt)));
   launch_pdl(wgrad_kernel, dim3(dim3(splits, mt)), dim3(THREADS), smem, st, mg, mz, p);
   return cudaGetLastError();
 }
