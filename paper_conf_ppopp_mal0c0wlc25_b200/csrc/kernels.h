@@ -251,6 +251,23 @@ cudaError_t launch_ce_loss(const float* logits, int64_t pitch, int n_classes, co
                            const int32_t* n_seeds, int64_t max_seeds, const int32_t* labels,
                            const int32_t* n_global, float* loss, float* g, int64_t g_pitch, uint16_t* gb,
                            int64_t gb_pitch, float* zero, int64_t zero_n, int32_t* ws, cudaStream_t st);
+// outfused.cu: the output layer's mean + projection + softmax CE in one kernel (bf16 mode)
+struct OutFusedArgs {
+  const int32_t* indptr; const int32_t* indices;       // the hop-0 block (CSR over H^{K-1} rows)
+  const uint16_t* hb; int64_t hb_pitch;                 // H^{K-1} in bf16 (reading R11)
+  const int32_t* n_dst; int64_t max_dst;
+  int d_in, C;
+  uint16_t* zb; int64_t zb_pitch;                       // Z^K (bf16, + the all-ones column d_in)
+  const uint16_t* wb; int64_t wb_pitch;                 // W^K bf16 [C][wb_pitch]
+  const float* bias;
+  float* logits; int64_t l_pitch;                       // H^K (fp32)
+  const int32_t* seeds; const int32_t* labels; const int32_t* n_global;
+  float* loss; float* g; int64_t g_pitch; uint16_t* gb; int64_t gb_pitch;
+  float* zero; int64_t zero_n; float* part; int32_t* ticket;
+};
+int out_fused_supported(int d_in, int C, int64_t max_dst);
+cudaError_t launch_out_fused(const OutFusedArgs& a, cudaStream_t st);
+
 // ce_loss workspace: [ticket, partial sums of up to kCeMaxBlocks blocks], zero-initialised once
 constexpr int kCeMaxBlocks = 1024;
 cudaError_t launch_relu_bwd(float* g, const float* h, int64_t pitch, int dim, const int32_t* n_dev, int64_t max_n,

@@ -588,7 +588,7 @@ apt_status phase_sample(apt_trainer* t, RankState& rs, SampleSet& ss, bool from_
   // that it fills gaps instead of competing with the step's chain for every SM
   static const int64_t bg_cap = [] {
     const char* v = std::getenv("APT_BG_BLOCKS_PER_SM");
-    return int64_t(num_sms()) * (v ? std::max(1, atoi(v)) : 4);
+    return int64_t(num_sms()) * (v ? std::max(1, atoi(v)) : 8);   // 4 -> 8 with the fused output layer (A/B)
   }();
   const int64_t cap = st == c->samp ? bg_cap : 0;
   {
@@ -624,7 +624,7 @@ apt_status phase_sample(apt_trainer* t, RankState& rs, SampleSet& ss, bool from_
       cudaStream_t cs_st = st;
       // the background (next-step) sampling: the transposes on a second low-priority stream,
       // so the next hop's sampling does not wait for them (joined at the branch's end)
-      static const int bg_fork = [] { const char* v = std::getenv("APT_BG_CSC_FORK"); return v ? atoi(v) : 0; }();
+      static const int bg_fork = [] { const char* v = std::getenv("APT_BG_CSC_FORK"); return v ? atoi(v) : 1; }();
       if (!fork_csc && bg_fork && st == c->samp) {
         CK(c, cudaEventRecord(c->ev_sfork, st));
         CK(c, cudaStreamWaitEvent(c->samp2, c->ev_sfork, 0));
@@ -756,6 +756,17 @@ apt_status upper_fwd_loss(apt_trainer* t, RankState& rs) {
     Layer& L = rs.L[l - 1];
     const Layer& P = rs.L[l - 2];
     const Hop& hp = rs.hops[t->K - l];
+    if (l == t->K && t->m.dtype == APT_BF16 && P.Hb && L.Zb && !L.Hb && L.Gb &&
+        out_fused_supported(L.d_in, L.d_out, L.max_rows)) {
+      // the output layer's mean, projection and loss in one kernel (outfused.cu)
+      OutFusedArgs o{hp.indptr, hp.indices, P.Hb, P.hb_pitch, hp.n_dst, hp.max_dst, L.d_in, L.d_out,
+                     L.Zb, L.zb_pitch, L.Wb, L.wb_pitch, L.b, L.H, L.h_pitch,
+                     rs.seeds, t->labels, rs.small + 1, rs.loss, L.G, L.h_pitch, L.Gb, L.gb_pitch,
+                     rs.L[0].dW, grad_floats(t, rs), reinterpret_cast<float*>(rs.ce_ws + 1), rs.ce_ws};
+      CK(c, launch_out_fused(o, c->stream));
+      c->launches++;
+      return APT_OK;
+    }
     AggArgs a{};
     a.indptr = hp.indptr; a.indices = hp.indices; a.x = P.H; a.x_pitch = P.h_pitch;
     if (P.Hb) { a.x = nullptr; a.xb = P.Hb; a.x_pitch = P.hb_pitch; }   // R11
@@ -780,7 +791,9 @@ apt_status upper_fwd_loss(apt_trainer* t, RankState& rs) {
 
 // Where the upper layers' weight gradients fork off the main chain (APT_WG_FORK; A/B).
 static int wg_fork_mode() {
-  static const int m = [] { const char* e = std::getenv("APT_WG_FORK"); return e ? atoi(e) : 2; }();
+  // A/B with the fused output layer and the background transposes off the sampling chain
+  // (0 / 1 / 2): 0.1500 / 0.1514 / 0.1571 ms; before them mode 2 won
+  static const int m = [] { const char* e = std::getenv("APT_WG_FORK"); return e ? atoi(e) : 0; }();
   return m;
 }
 
