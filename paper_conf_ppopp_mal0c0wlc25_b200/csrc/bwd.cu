@@ -307,7 +307,7 @@ __global__ void __launch_bounds__(256) pull_bwd_b8_kernel(PullArgs a) {
 // dependent chain (CSC pointer -> in-edge -> dZ row) shrinks to the dZ row loads, where the
 // block-per-group form paid all three round trips per group (layer-1 rows have ~1.3
 // in-edges each, so the chain, not the bytes, set the time).
-template <int VP, int R, int EB>
+template <int VP, int R, int EB, bool BITS>
 __global__ void __launch_bounds__(256) pull_bwd_b8_pf_kernel(PullArgs a) {
   APT_PDL_PROLOGUE();
   const int lane = lane_id();
@@ -334,8 +334,17 @@ __global__ void __launch_bounds__(256) pull_bwd_b8_pf_kernel(PullArgs a) {
 #pragma unroll
       for (int p = 0; p < VP; ++p) {
         const int j = lane + 32 * p;
-        hm[r][p] = (u < n && j < V8) ? __ldg(reinterpret_cast<const uint4*>(a.hb + u * a.hb_pitch + j * 8))
-                                     : make_uint4(0, 0, 0, 0);
+        if constexpr (BITS) {
+          // the lane's 8 ReLU bits (one byte of the row's mask words) as positive bf16 halves
+          // for the same packed-pair compare below
+          uint32_t b = 0;
+          if (u < n && j < V8) b = uint32_t(__ldg(a.mask + u * a.mask_pitch + (j >> 1))) >> (8 * (j & 1));
+          hm[r][p] = make_uint4((b & 1u) | ((b & 2u) << 15), ((b >> 2) & 1u) | (((b >> 3) & 1u) << 16),
+                                ((b >> 4) & 1u) | (((b >> 5) & 1u) << 16), ((b >> 6) & 1u) | (((b >> 7) & 1u) << 16));
+        } else {
+          hm[r][p] = (u < n && j < V8) ? __ldg(reinterpret_cast<const uint4*>(a.hb + u * a.hb_pitch + j * 8))
+                                       : make_uint4(0, 0, 0, 0);
+        }
       }
       e0n[r] = 0; cntn[r] = 0;
       if (un < n) { e0n[r] = a.csc_ptr[un]; cntn[r] = a.csc_ptr[un + 1] - e0n[r]; }
@@ -447,10 +456,11 @@ cudaError_t launch_pull_bwd(const PullArgs& a, cudaStream_t st) {
       static const int pbpsm = [] { const char* e = std::getenv("APT_PULL_PF_BPSM"); return e ? atoi(e) : 0; }();
       // in-edges in flight per row (APT_PULL_EB) x rows per warp (APT_PULL_ROWS): A/B knobs
       static const int eb = [] { const char* e = std::getenv("APT_PULL_EB"); return e ? atoi(e) : 1; }();   // 1 / 2 / 4: 0.1627 / 0.1673 / 0.1786 ms (A/B)
-      auto kern = Rr == 4 ? pull_bwd_b8_pf_kernel<1, 4, 1>
-                : (rr == 1 ? (eb >= 4 ? pull_bwd_b8_pf_kernel<1, 1, 4> : pull_bwd_b8_pf_kernel<1, 1, 2>)
-                : (eb >= 4 ? pull_bwd_b8_pf_kernel<1, 2, 4> : eb == 2 ? pull_bwd_b8_pf_kernel<1, 2, 2>
-                : pull_bwd_b8_pf_kernel<1, 2, 1>));
+      auto kern = a.mask ? pull_bwd_b8_pf_kernel<1, 2, 1, true>
+                : Rr == 4 ? pull_bwd_b8_pf_kernel<1, 4, 1, false>
+                : (rr == 1 ? (eb >= 4 ? pull_bwd_b8_pf_kernel<1, 1, 4, false> : pull_bwd_b8_pf_kernel<1, 1, 2, false>)
+                : (eb >= 4 ? pull_bwd_b8_pf_kernel<1, 2, 4, false> : eb == 2 ? pull_bwd_b8_pf_kernel<1, 2, 2, false>
+                : pull_bwd_b8_pf_kernel<1, 2, 1, false>));
       const int Rk = rr == 1 ? 1 : Rr;
       const int64_t pblocks = grid_cap(ceil_div(ceil_div(round_up(a.max_src, 64), Rk) * 32, 256),
                                        pbpsm > 0 ? pbpsm : resident_blocks(kern, 256));

@@ -63,6 +63,7 @@ struct RowParams {
   int n_split;              // CTAs share an M tile: CTA b computes columns [(b % n_split) * BN, +BN)
   uint16_t* mask;           // optional ReLU bit mask [M x mask_pitch] (16 columns per word)
   int64_t mask_pitch;
+  int mask_direct;          // the mask comes from the direct (bf16-row) epilogue
   const int32_t* row_div;   // optional: divide row m by indptr[m+1] - indptr[m] (RN)
   uint16_t* Yb;             // optional bf16 output instead of Y (not with routing / accumulation)
   int64_t yb_pitch;
@@ -195,7 +196,9 @@ __global__ void __launch_bounds__(ROW_THREADS, 1)
     // is shared-memory latency, not a global bias load and a TMEM round trip.
     const int q = warp & 3, h = (warp - 2) >> 2;
     // staged: 0 direct for every plain output, 1 never (A/B), 2 only for bf16 rows
-    const bool direct = !p.out_rank && !p.accumulate && !p.mask && (p.staged == 0 || (p.staged == 2 && p.Yb));
+    // (bf16 rows may also emit their ReLU bit mask from the direct path: mask_direct)
+    const bool direct = !p.out_rank && !p.accumulate && (!p.mask || p.mask_direct) &&
+                        (p.staged == 0 || (p.staged == 2 && p.Yb));
     float* stg = stg_all + (warp - 2) * 32 * 17;
     const int rsub = lane >> 2, cq = (lane & 3) * 4;
     // this CTA's bias slice (zero past N or without bias), shared by the 8 epilogue warps
@@ -241,6 +244,7 @@ __global__ void __launch_bounds__(ROW_THREADS, 1)
         }
         for (int cb = cb0; cb < cb1; cb += 4) {
           const int ng = min(4, cb1 - cb);
+          uint64_t mbits = 0;   // mask_direct: bit j of chunk i = (bf16 output > 0), 16 per chunk
           uint32_t r4[4][16];
 #pragma unroll
           for (int i = 0; i < 4; ++i)
@@ -269,6 +273,16 @@ __global__ void __launch_bounds__(ROW_THREADS, 1)
                 for (int j = 0; j < 16; ++j) v[j] = div_rn_rcp(v[j], own_deg, own_rdeg);
               }
               const int col = n0 + c;
+              if (p.mask_direct) {   // the ReLU decision the backward reads: the stored bf16 value > 0
+                uint32_t b16 = 0;
+#pragma unroll
+                for (int j = 0; j < 16; j += 2) {
+                  const uint32_t w = pack_bf16x2(v[j], v[j + 1]);
+                  b16 |= ((w & 0x7FFFu) && col + j < p.N ? 1u : 0u) << j;
+                  b16 |= ((w & 0x7FFF0000u) && col + j + 1 < p.N ? 1u : 0u) << (j + 1);
+                }
+                mbits |= uint64_t(b16) << (16 * i);
+              }
               if (p.tma_store) {   // rows past M: zeros (the box still covers them)
                 const int u = 2 * (cb + i - cb0);
                 uint8_t* rp = ysb + lane * 128;
@@ -316,6 +330,14 @@ __global__ void __launch_bounds__(ROW_THREADS, 1)
                     if (col + j < p.N) d[j] = v[j];
                 }
               }
+            }
+          }
+          if (p.mask_direct && own) {   // the group's <= 64 mask bits of this row: one 8-byte store
+            uint16_t* mrow = p.mask + m_own * p.mask_pitch + (n0 + 16 * cb) / 16;
+            if (ng == 4 && (reinterpret_cast<uintptr_t>(mrow) & 7) == 0) {
+              *reinterpret_cast<uint2*>(mrow) = make_uint2(uint32_t(mbits), uint32_t(mbits >> 32));
+            } else {
+              for (int i = 0; i < ng; ++i) mrow[i] = uint16_t(mbits >> (16 * i));
             }
           }
         }
@@ -610,7 +632,10 @@ cudaError_t launch_tc_gemm(const TcGemmArgs& a, cudaStream_t st) {
   static const int epi_tma = [] { const char* v = std::getenv("APT_EPI_TMA"); return v ? atoi(v) : 1; }();
   CUtensorMap my;
   int tma_store = 0;
-  if (epi_tma && a.Yb && BN == 128 && !a.out_rank && !a.accumulate && !a.mask && !epi_staged &&
+  // ReLU bits of bf16 rows from the direct epilogue (8-byte stores of 64 bits per row and warp)
+  const int mask_direct = (a.mask && a.Yb && !a.out_rank && !a.accumulate && !epi_staged && BN % 64 == 0 &&
+                           (a.mask_pitch % 4) == 0) ? 1 : 0;
+  if (epi_tma && a.Yb && BN == 128 && !a.out_rank && !a.accumulate && (!a.mask || mask_direct) && !epi_staged &&
       (a.yb_pitch * 2) % 16 == 0 && (reinterpret_cast<uintptr_t>(a.Yb) & 15) == 0 &&
       make_map(&my, a.Yb, a.N, std::max<int64_t>(a.M_max, 1), a.yb_pitch, 64, 32))
     tma_store = 1;
@@ -629,7 +654,8 @@ cudaError_t launch_tc_gemm(const TcGemmArgs& a, cudaStream_t st) {
   int cols = 32;
   while (cols < nacc * BN) cols <<= 1;
   RowParams p{a.M_max, a.M_dev, a.N, BN, nkb, cols, a.w_mn, stages, nacc, b_kb_bytes, a.bias, a.relu, a.Y, a.y_pitch,
-              a.out_base, a.out_rank, a.out_row, a.accumulate, n_split, a.mask, a.mask_pitch, a.row_div_indptr,
+              a.out_base, a.out_rank, a.out_row, a.accumulate, n_split, a.mask, a.mask_pitch, mask_direct,
+              a.row_div_indptr,
               a.Yb, a.yb_pitch, a.b_early, epi_staged, tma_store};
   const size_t smem = smem_of(stages);   // + epilogue staging
   if (smem > 227 * 1024) return cudaErrorInvalidValue;

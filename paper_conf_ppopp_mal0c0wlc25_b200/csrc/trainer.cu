@@ -147,6 +147,7 @@ apt_status project(apt_trainer* t, const Layer& L, const void* Zb, const float* 
     TcGemmArgs a{static_cast<const uint16_t*>(Zb), z_pitch_b, Wb, L.wb_pitch, max_rows, n_rows, L.d_out, K,
                  bias, relu, Y, L.h_pitch, out_base, out_rank, out_row, 0};
     if (relu && L.Mk && !out_rank) { a.mask = L.Mk; a.mask_pitch = L.mk_pitch; }   // ReLU bits for the backward
+    if (Y == L.H) L.mk_valid = a.mask != nullptr;
     if (Y == L.H && L.Hb && !out_rank) { a.Yb = L.Hb; a.yb_pitch = L.hb_pitch; }   // R11: bf16 only
     a.b_early = 1;   // the step's weights change only in the SGD at its end
     CK(c, launch_tc_gemm(a, c->stream));
@@ -360,9 +361,18 @@ apt_status apt::trainer_create(apt_ctx* c, const apt_graph* g, const apt_fstore*
       }
       L.G = A.alloc<float>(L.max_rows * L.h_pitch, true);
       if (m->dtype == APT_BF16) L.Gb = A.alloc<uint16_t>(L.max_rows * L.gb_pitch, true);
-      // (ReLU bit masks, L.Mk, are supported by the epilogue and the pull kernel but not
-      //  allocated: measured on products, the 2-byte mask stores cost the projection more
-      //  than the pull saves by not reading H -- 78 vs 66 us forward, 72 vs 74 us backward)
+      // ReLU bit masks of the bf16 hidden layers (APT_RELU_BITS=1, opt-in): the direct
+      // epilogue writes each row's 64 bits per warp as one 8-byte store, and the mean's
+      // backward reads 32 B of bits per row instead of the 512-B bf16 row of H.  (Round 1
+      // measured the staged epilogue's 2-byte mask stores: they cost the projection more
+      // than the pull saved -- 78 vs 66 us forward, 72 vs 74 us backward.  Round 2, bits from
+      // the direct / TMA-store epilogue: layer-1 forward 40.5 -> 45.0 us, backward -1 us,
+      // step 0.1500 -> 0.1550 ms: off by default.)
+      static const int relu_bits = [] { const char* v = std::getenv("APT_RELU_BITS"); return v ? atoi(v) : 0; }();
+      if (m->dtype == APT_BF16 && l < K && relu_bits) {
+        L.mk_pitch = round_up(ceil_div(L.d_out, 16), 4);
+        L.Mk = A.alloc<uint16_t>(L.max_rows * L.mk_pitch, true);
+      }
       if (l > 1) L.dZ = A.alloc<float>(L.max_rows * L.zf_pitch, true);
       if (l > 1 && m->dtype == APT_BF16) {   // reading R13: the mean's backward reads dZ / deg in bf16
         L.dzb_pitch = round_up(L.d_in, 8);
@@ -853,11 +863,13 @@ apt_status upper_bwd(apt_trainer* t, RankState& rs) {
     if (l == t->K && t->csc_forked) CK(c, cudaStreamWaitEvent(c->stream, c->ev_csc, 0));
     // ReLU bits of H_{l-1} exist when its projection ran on this rank's tcgen05 path
     const bool l1_local = l - 1 > 1 || t->world == 1 || t->s == APT_GDP;
-    const uint16_t* mk = (bf && P.Mk && l1_local && tc_gemm_supported(P.d_out, P.d_in)) ? P.Mk : nullptr;
+    const uint16_t* mk = (bf && P.Mk && P.mk_valid && l1_local && tc_gemm_supported(P.d_out, P.d_in)) ? P.Mk : nullptr;
     PullArgs pa{hp.csc_ptr, hp.csc_dst, hp.indptr, L.dZ, L.zf_pitch, P.H, P.h_pitch, mk, P.mk_pitch,
                 bf ? nullptr : P.G, P.h_pitch, bf ? P.Gb : nullptr, P.gb_pitch, hp.counts, P.max_rows, L.d_in,
                 dz_scaled};
-    if (P.Hb && !mk) { pa.h = nullptr; pa.hb = P.Hb; pa.hb_pitch = P.hb_pitch; }   // R11: mask from bf16 H
+    // R11: the mask from bf16 H (bf16 mode always passes H; the pull takes the bits instead
+    // where it can, else H)
+    if (P.Hb) { pa.h = nullptr; pa.hb = P.Hb; pa.hb_pitch = P.hb_pitch; }
     if (dzb) { pa.dzb = dzb; pa.dzb_pitch = L.dzb_pitch; }                            // R13: bf16 dZ / deg
     CK(c, launch_pull_bwd(pa, c->stream));
     c->launches += 2;

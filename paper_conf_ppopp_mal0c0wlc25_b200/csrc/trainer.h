@@ -42,7 +42,7 @@ struct Layer {
   uint16_t* Gb = nullptr;           // bf16 copy of G (tcgen05 backward, bf16 mode)
   uint16_t* Mk = nullptr;           // ReLU mask bits of H (bf16 mode, hidden layers) [max_rows x mk_pitch]
   int64_t mk_pitch = 0;
-  bool mk_valid = false;            // the last forward wrote Mk (tcgen05 epilogue on this rank)
+  mutable bool mk_valid = false;    // the captured forward writes Mk (tcgen05 bf16 epilogue on this rank)
   int64_t gb_pitch = 0;
   float* dZ = nullptr;              // [max_rows x zf_pitch] scratch (l > 1)
   uint16_t* dZb = nullptr;          // bf16 mode: (G W) / deg in bf16 [max_rows x dzb_pitch] (reading R13)
