@@ -264,6 +264,7 @@ struct OutFusedArgs {
   const int32_t* seeds; const int32_t* labels; const int32_t* n_global;
   float* loss; float* g; int64_t g_pitch; uint16_t* gb; int64_t gb_pitch;
   float* zero; int64_t zero_n; float* part; int32_t* ticket;
+  uint16_t* dzb; int64_t dzb_pitch;                     // optional: dZ^K = (G W) / deg in bf16 (R13)
 };
 int out_fused_supported(int d_in, int C, int64_t max_dst);
 cudaError_t launch_out_fused(const OutFusedArgs& a, cudaStream_t st);

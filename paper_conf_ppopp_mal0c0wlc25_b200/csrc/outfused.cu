@@ -30,6 +30,7 @@ constexpr int kWarps = 16;
 constexpr int kKMax = 256;         // d_in (multiple of 8)
 constexpr int kNMax = 64;          // classes
 constexpr int kSP = kKMax + 8;     // shared row stride (bf16): 528 B, conflict-free fragment loads
+constexpr int kGS = kNMax + 8;     // G row stride (bf16): 144 B
 
 __device__ __forceinline__ void mma_bf16_16816(float* c, const uint32_t* a, const uint32_t* b) {
   asm volatile(
@@ -45,8 +46,10 @@ __global__ void __launch_bounds__(kWarps * 32, 1) out_fused_kernel(OutFusedArgs 
   extern __shared__ __align__(16) uint8_t smem[];
   uint16_t* Zs = reinterpret_cast<uint16_t*>(smem);                       // [kRows][kSP]
   uint16_t* Ws = Zs + kRows * kSP;                                         // [Cpad][kSP]
-  const int Cpad = (a.C + 7) & ~7;
+  const int Cpad = (a.C + 15) & ~15;
   float* Ls = reinterpret_cast<float*>(Ws + Cpad * kSP);                   // [kRows][kNMax + 1]
+  __shared__ __align__(16) uint16_t Gs[kRows * kGS];                       // bf16 G (dZ = G W)
+  __shared__ float degs[kRows];
   __shared__ float wsum[kWarps];
   __shared__ bool last;
   const int warp = threadIdx.x >> 5, lane = lane_id();
@@ -99,6 +102,7 @@ __global__ void __launch_bounds__(kWarps * 32, 1) out_fused_kernel(OutFusedArgs 
       }
     }
     uint4 zv = make_uint4(0, 0, 0, 0);
+    if (lane == 0) degs[rl] = float(cnt);
     if (i < n) {
       const float fdeg = float(cnt);
       const float rdeg = fdeg > 0.f ? __frcp_rn(fdeg) : 0.f;
@@ -144,6 +148,7 @@ __global__ void __launch_bounds__(kWarps * 32, 1) out_fused_kernel(OutFusedArgs 
       }
     }
   }
+  for (int t = threadIdx.x; t < kRows * kGS / 2; t += blockDim.x) reinterpret_cast<uint32_t*>(Gs)[t] = 0u;
   __syncthreads();
   // the step's gradient accumulators start at zero (ce_loss_kernel's duty)
   for (int64_t t = int64_t(blockIdx.x) * blockDim.x + threadIdx.x; t < a.zero_n; t += int64_t(gridDim.x) * blockDim.x)
@@ -170,7 +175,49 @@ __global__ void __launch_bounds__(kWarps * 32, 1) out_fused_kernel(OutFusedArgs 
       const float p = expf(row[c] - lse);
       const float v = (p - (c == y[q] ? 1.f : 0.f)) * inv_n;
       a.g[i * a.g_pitch + c] = v;
-      a.gb[i * a.gb_pitch + c] = bf16_bits(v);
+      const uint16_t vb = bf16_bits(v);
+      a.gb[i * a.gb_pitch + c] = vb;
+      Gs[rl * kGS + c] = vb;
+    }
+  }
+  // 4. (a.dzb) dZ = (G W) / deg in bf16 (reading R13) for the mean's backward: the same
+  // bf16 G and W the tcgen05 dZ kernel multiplies, fp32 accumulation, the correctly
+  // rounded division per row, RNE to bf16
+  if (a.dzb) {
+    __syncthreads();
+    const int g = lane >> 2, t4 = lane & 3;
+    for (int tile = warp; tile < (kRows / 16) * (a.d_in / 8); tile += kWarps) {
+      const int mt = tile % (kRows / 16), nt = tile / (kRows / 16);
+      const int ncol = nt * 8 + g;
+      float c[4] = {0.f, 0.f, 0.f, 0.f};
+      const uint16_t* A0 = Gs + (mt * 16 + g) * kGS + 2 * t4;
+      const uint16_t* A1 = A0 + 8 * kGS;
+      for (int k0 = 0; k0 < Cpad; k0 += 16) {
+        uint32_t af[4], bfr[2];
+        af[0] = *reinterpret_cast<const uint32_t*>(A0 + k0);
+        af[1] = *reinterpret_cast<const uint32_t*>(A1 + k0);
+        af[2] = *reinterpret_cast<const uint32_t*>(A0 + k0 + 8);
+        af[3] = *reinterpret_cast<const uint32_t*>(A1 + k0 + 8);
+        const uint16_t* Wc = Ws + (k0 + 2 * t4) * kSP + ncol;   // W[class][col]: classes run down rows
+        bfr[0] = uint32_t(Wc[0]) | (uint32_t(Wc[kSP]) << 16);
+        bfr[1] = uint32_t(Wc[8 * kSP]) | (uint32_t(Wc[9 * kSP]) << 16);
+        mma_bf16_16816(c, af, bfr);
+      }
+      const int col = nt * 8 + 2 * t4;
+#pragma unroll
+      for (int h = 0; h < 2; ++h) {
+        const int rl = mt * 16 + g + 8 * h;
+        const int64_t i = r0 + rl;
+        if (i >= n) continue;
+        float v0 = c[2 * h], v1 = c[2 * h + 1];
+        const float dg = degs[rl];
+        if (dg > 0.f) {
+          const float rd = __frcp_rn(dg);
+          v0 = div_rn_rcp(v0, dg, rd);
+          v1 = div_rn_rcp(v1, dg, rd);
+        }
+        *reinterpret_cast<uint32_t*>(a.dzb + i * a.dzb_pitch + col) = pack_bf16x2(v0, v1);
+      }
     }
   }
   {   // zero the tail of the last 64-row block of Gb (tcgen05 weight gradient reads whole blocks)
@@ -214,7 +261,7 @@ cudaError_t launch_out_fused(const OutFusedArgs& a, cudaStream_t st) {
   // APT_OUT_ROWS: rows per CTA (16: one row per warp, 2x the CTAs; 32: two rows per warp)
   static const int rows = [] { const char* v = std::getenv("APT_OUT_ROWS"); return v ? atoi(v) : 16; }();
   const int R = rows == 32 ? 32 : 16;
-  const int Cpad = (a.C + 7) & ~7;
+  const int Cpad = (a.C + 15) & ~15;
   const size_t smem = size_t(R + Cpad) * kSP * 2 + size_t(R) * (kNMax + 1) * 4;
   static bool attr = false;
   if (!attr) {

@@ -762,6 +762,7 @@ static bool bf16_dz_enabled() {
 // Upper layers l = 2..K (data parallel) + CE loss on one rank.
 apt_status upper_fwd_loss(apt_trainer* t, RankState& rs) {
   apt_ctx* c = t->ctx;
+  t->out_dz_fused = false;
   for (int l = 2; l <= t->K; ++l) {
     Layer& L = rs.L[l - 1];
     const Layer& P = rs.L[l - 2];
@@ -773,6 +774,10 @@ apt_status upper_fwd_loss(apt_trainer* t, RankState& rs) {
                      L.Zb, L.zb_pitch, L.Wb, L.wb_pitch, L.b, L.H, L.h_pitch,
                      rs.seeds, t->labels, rs.small + 1, rs.loss, L.G, L.h_pitch, L.Gb, L.gb_pitch,
                      rs.L[0].dW, grad_floats(t, rs), reinterpret_cast<float*>(rs.ce_ws + 1), rs.ce_ws};
+      // dZ^K = (G W) / deg from the same kernel (APT_OUT_DZ=0: the tcgen05 dZ launch, A/B)
+      static const int out_dz = [] { const char* v = std::getenv("APT_OUT_DZ"); return v ? atoi(v) : 1; }();
+      t->out_dz_fused = out_dz && L.dZb && bf16_dz_enabled() && tc_gemm_supported(L.d_in, L.d_out);
+      if (t->out_dz_fused) { o.dzb = L.dZb; o.dzb_pitch = L.dzb_pitch; }
       CK(c, launch_out_fused(o, c->stream));
       c->launches++;
       return APT_OK;
@@ -833,7 +838,10 @@ apt_status upper_bwd(apt_trainer* t, RankState& rs) {
     int dz_scaled = 0;
     const uint16_t* dzb = nullptr;
     // dZ = G W  (bf16 mode: tcgen05 with the bf16 weights of the forward, W read N-major as stored)
-    if (bf && tc_gemm_supported(L.d_in, L.d_out)) {
+    if (l == t->K && t->out_dz_fused) {   // already written by the fused output-layer kernel
+      dz_scaled = 1;
+      dzb = L.dZb;
+    } else if (bf && tc_gemm_supported(L.d_in, L.d_out)) {
       TcGemmArgs g{L.Gb, L.gb_pitch, L.Wb, L.wb_pitch, L.max_rows, L.n_rows, L.d_in, L.d_out, nullptr, 0,
                    L.dZ, L.zf_pitch, nullptr, nullptr, nullptr, 1};
       g.row_div_indptr = hp.indptr;   // dZ / deg once per row (the pull then only sums)

@@ -196,6 +196,7 @@ struct apt_trainer {
   int64_t primed = -1;               // step id already sampled into sset[primed_parity]
   int primed_parity = 0;
   bool csc_forked = false;
+  bool out_dz_fused = false;    // the fused output-layer kernel also wrote dZ^K (bf16 / deg)
   bool bg_csc_forked = false;   // the background sampling forked its transposes onto ctx->samp2
   std::function<apt_status()> deferred_fork;   // pipelined: next-step sampling, launched after the layer-1 forward
   cudaGraphExec_t gexec_p[2][2] = {};   // [parity][update] pipelined step graphs
