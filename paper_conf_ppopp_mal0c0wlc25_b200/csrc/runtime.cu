@@ -112,7 +112,9 @@ apt_status apt_ctx_create(int rank, int world, int device, void* stream, apt_ctx
   static const int samp_hi = [] { const char* v = std::getenv("APT_SAMP_PRIO"); return v ? atoi(v) : 0; }();
   cudaStreamCreateWithPriority(&c->samp, cudaStreamNonBlocking, samp_hi ? prio_hi : prio_lo);
   cudaStreamCreateWithPriority(&c->tap, cudaStreamNonBlocking, prio_hi);
-  cudaStreamCreateWithPriority(&c->samp2, cudaStreamNonBlocking, samp_hi ? prio_hi : prio_lo);
+  // APT_SAMP2_PRIO=1: the background block transposes at the chain's priority (A/B)
+  static const int samp2_hi = [] { const char* v = std::getenv("APT_SAMP2_PRIO"); return v ? atoi(v) : 0; }();
+  cudaStreamCreateWithPriority(&c->samp2, cudaStreamNonBlocking, (samp_hi || samp2_hi) ? prio_hi : prio_lo);
   cudaEventCreateWithFlags(&c->ev_sfork, cudaEventDisableTiming);
   cudaEventCreateWithFlags(&c->ev_sjoin, cudaEventDisableTiming);
   cudaEventCreateWithFlags(&c->ev_tap, cudaEventDisableTiming);
