@@ -307,8 +307,8 @@ __global__ void __launch_bounds__(256) pull_bwd_b8_kernel(PullArgs a) {
 // dependent chain (CSC pointer -> in-edge -> dZ row) shrinks to the dZ row loads, where the
 // block-per-group form paid all three round trips per group (layer-1 rows have ~1.3
 // in-edges each, so the chain, not the bytes, set the time).
-template <int VP, int R, int EB, bool BITS>
-__global__ void __launch_bounds__(256) pull_bwd_b8_pf_kernel(PullArgs a) {
+template <int VP, int R, int EB, bool BITS, int MINB = 1>
+__global__ void __launch_bounds__(256, MINB) pull_bwd_b8_pf_kernel(PullArgs a) {
   APT_PDL_PROLOGUE();
   const int lane = lane_id();
   const int64_t n = *a.n_src;
@@ -456,7 +456,11 @@ cudaError_t launch_pull_bwd(const PullArgs& a, cudaStream_t st) {
       static const int pbpsm = [] { const char* e = std::getenv("APT_PULL_PF_BPSM"); return e ? atoi(e) : 0; }();
       // in-edges in flight per row (APT_PULL_EB) x rows per warp (APT_PULL_ROWS): A/B knobs
       static const int eb = [] { const char* e = std::getenv("APT_PULL_EB"); return e ? atoi(e) : 1; }();   // 1 / 2 / 4: 0.1627 / 0.1673 / 0.1786 ms (A/B)
-      auto kern = a.mask ? pull_bwd_b8_pf_kernel<1, 2, 1, true>
+      // APT_PULL_MINB: blocks per SM the register allocation must allow (A/B)
+      static const int pminb = [] { const char* e = std::getenv("APT_PULL_MINB"); return e ? atoi(e) : 0; }();
+      auto kern = (!a.mask && Rr == 2 && rr != 1 && eb <= 1 && pminb >= 5)
+                  ? (pminb >= 6 ? pull_bwd_b8_pf_kernel<1, 2, 1, false, 6> : pull_bwd_b8_pf_kernel<1, 2, 1, false, 5>)
+                : a.mask ? pull_bwd_b8_pf_kernel<1, 2, 1, true>
                 : Rr == 4 ? pull_bwd_b8_pf_kernel<1, 4, 1, false>
                 : (rr == 1 ? (eb >= 4 ? pull_bwd_b8_pf_kernel<1, 1, 4, false> : pull_bwd_b8_pf_kernel<1, 1, 2, false>)
                 : (eb >= 4 ? pull_bwd_b8_pf_kernel<1, 2, 4, false> : eb == 2 ? pull_bwd_b8_pf_kernel<1, 2, 2, false>
