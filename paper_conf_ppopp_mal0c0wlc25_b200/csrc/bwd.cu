@@ -307,7 +307,7 @@ __global__ void __launch_bounds__(256) pull_bwd_b8_kernel(PullArgs a) {
 // dependent chain (CSC pointer -> in-edge -> dZ row) shrinks to the dZ row loads, where the
 // block-per-group form paid all three round trips per group (layer-1 rows have ~1.3
 // in-edges each, so the chain, not the bytes, set the time).
-template <int VP, int R, int EB, bool BITS, int MINB = 1>
+template <int VP, int R, int EB, bool BITS, int MINB = 4>
 __global__ void __launch_bounds__(256, MINB) pull_bwd_b8_pf_kernel(PullArgs a) {
   APT_PDL_PROLOGUE();
   const int lane = lane_id();
@@ -316,6 +316,15 @@ __global__ void __launch_bounds__(256, MINB) pull_bwd_b8_pf_kernel(PullArgs a) {
   const int64_t nwarps = int64_t(gridDim.x) * (blockDim.x >> 5);
   const int64_t rows_out = std::min<int64_t>(a.max_src, round_up(n, 64));
   int64_t u0 = ((int64_t(blockIdx.x) * blockDim.x + threadIdx.x) >> 5) * R;
+  // each lane's column base in the dZ rows as an opaque 64-bit value (lanes past the row's
+  // vectors read vector 0: in bounds, never stored)
+  const uint32_t zrb = uint32_t(a.dzb_pitch * 2);
+  uint64_t zb[VP];
+#pragma unroll
+  for (int p = 0; p < VP; ++p) {
+    const int j = lane + 32 * p;
+    asm("mov.b64 %0, %1;" : "=l"(zb[p]) : "l"(reinterpret_cast<uint64_t>(a.dzb) + uint64_t(j < V8 ? j : 0) * 16u));
+  }
   int e0[R], cnt[R], vv[R];
 #pragma unroll
   for (int r = 0; r < R; ++r) {
@@ -367,6 +376,7 @@ __global__ void __launch_bounds__(256, MINB) pull_bwd_b8_pf_kernel(PullArgs a) {
       const int m = min(32, cmax - c0);
       // EB in-edges of every row of the group in flight at once (predicated loads; the
       // rows average ~1.3 in-edges, so one batch usually covers the group)
+#pragma unroll 1
       for (int eb = 0; eb < m; eb += EB) {
         uint4 z[EB][R][VP];
         bool ok[EB][R];
@@ -377,21 +387,21 @@ __global__ void __launch_bounds__(256, MINB) pull_bwd_b8_pf_kernel(PullArgs a) {
             const int e = eb + q;
             const int w = __shfl_sync(0xffffffffu, v[r], e & 31);
             ok[q][r] = e < m && c0 + e < cnt[r];
-            const uint16_t* zr = a.dzb + int64_t(w) * a.dzb_pitch;
+            // the row is always a valid one (lanes past a row's count hold id 0), so the
+            // load is unconditional: one IMAD.WIDE off the lane's column base, the value
+            // zeroed by selects where the edge is padding, the adds unconditional
 #pragma unroll
             for (int p = 0; p < VP; ++p) {
-              const int j = lane + 32 * p;
-              z[q][r][p] = (ok[q][r] && j < V8) ? __ldg(reinterpret_cast<const uint4*>(zr + j * 8))
-                                                : make_uint4(0, 0, 0, 0);
+              const uint4 t = __ldg(reinterpret_cast<const uint4*>(zb[p] + uint64_t(uint32_t(w)) * zrb));
+              z[q][r][p] = ok[q][r] ? t : make_uint4(0, 0, 0, 0);
             }
           }
 #pragma unroll
         for (int q = 0; q < EB; ++q)
 #pragma unroll
           for (int r = 0; r < R; ++r)
-            if (ok[q][r])
 #pragma unroll
-              for (int p = 0; p < VP; ++p) accumulate_bf16x8(acc[r][p], z[q][r][p]);
+            for (int p = 0; p < VP; ++p) accumulate_bf16x8(acc[r][p], z[q][r][p]);
       }
     }
     // the next group's first in-edges (its CSC bounds arrived during this group's sums)
