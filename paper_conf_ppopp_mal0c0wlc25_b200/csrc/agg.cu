@@ -422,6 +422,63 @@ cudaError_t launch_agg_fstore(const AggArgs& a, const FeatView& fv, cudaStream_t
   return fv.dtype == kBF16 ? dispatch_agg<8>(b, s, 16, st) : dispatch_agg<4>(b, s, 16, st);
 }
 
+// Upper-layer mean over bf16 rows of 17..32 16-byte vectors (d' in (128, 256]; reading
+// R11): agg_kernel<8, 1, 32, CsrSrc>'s warp-per-row form with the flat gather's
+// addressing -- the edge's source row broadcast as a 32-bit index, one IMAD.WIDE off the
+// lane's opaque column base, unconditional loads of always-valid rows (lanes past the
+// row's count hold row 0), padding zeroed by selects.  Same edge order, same adds, same
+// division and rounding: Z is bit-identical to agg_kernel's.
+__global__ void __launch_bounds__(256, 4) agg_csr_b8_kernel(AggArgs a, uint32_t rb) {
+  APT_PDL_PROLOGUE();
+  const int lane = lane_id();
+  const int64_t n_dst = *a.n_dst;
+  const int V = int(ceil_div(a.dim, 8));
+  const int lv = lane < V ? lane : 0;
+  uint64_t base;
+  asm("mov.b64 %0, %1;" : "=l"(base) : "l"(reinterpret_cast<uint64_t>(a.xb) + uint64_t(lv) * 16u));
+  const int64_t nwarps = int64_t(gridDim.x) * (blockDim.x >> 5);
+  for (int64_t i = (int64_t(blockIdx.x) * blockDim.x + threadIdx.x) >> 5; i < n_dst; i += nwarps) {
+    const int e0 = a.indptr[i];
+    const int cnt = a.indptr[i + 1] - e0;
+    float acc[8];
+#pragma unroll
+    for (int q = 0; q < 8; ++q) acc[q] = 0.f;
+    for (int c0 = 0; c0 < cnt; c0 += 32) {
+      const uint32_t u = c0 + lane < cnt ? uint32_t(a.indices[e0 + c0 + lane]) : 0u;
+      const int m = min(32, cnt - c0);
+#pragma unroll 1
+      for (int j = 0; j < m; j += 4) {
+        uint4 v[4];
+#pragma unroll
+        for (int q = 0; q < 4; ++q) {
+          const uint32_t uq = __shfl_sync(0xffffffffu, u, (j + q) & 31);
+          const uint4 t = __ldg(reinterpret_cast<const uint4*>(base + uint64_t(uq) * rb));
+          v[q] = j + q < m ? t : make_uint4(0, 0, 0, 0);
+        }
+#pragma unroll
+        for (int q = 0; q < 4; ++q) accumulate_vec<8>(acc, v[q]);
+      }
+    }
+    if (a.z_ones && lane == 0) a.z_bf16[i * a.z_bf16_pitch + a.dim] = 0x3F80;
+    if (lane >= V) continue;
+    const float fdeg = float(cnt);
+    const float rdeg = fdeg > 0.f ? __frcp_rn(fdeg) : 0.f;
+    float z[8];
+#pragma unroll
+    for (int q = 0; q < 8; ++q) z[q] = fdeg > 0.f ? div_rn_rcp(acc[q], fdeg, rdeg) : 0.f;
+    const int c0 = lane * 8;
+    uint16_t* o = a.z_bf16 + i * a.z_bf16_pitch + c0;
+    if (c0 + 8 <= a.dim) {
+      *reinterpret_cast<uint4*>(o) = make_uint4(pack_bf16x2(z[0], z[1]), pack_bf16x2(z[2], z[3]),
+                                                pack_bf16x2(z[4], z[5]), pack_bf16x2(z[6], z[7]));
+    } else {
+#pragma unroll
+      for (int q = 0; q < 8; ++q)
+        if (c0 + q < a.dim) o[q] = bf16_bits(z[q]);
+    }
+  }
+}
+
 cudaError_t launch_agg_csr(const AggArgs& a, cudaStream_t st) {
   // rows wider than one launch covers (> 128 16-B vectors): column chunks of 512 fp32 /
   // 1024 bf16 columns
@@ -434,7 +491,15 @@ cudaError_t launch_agg_csr(const AggArgs& a, cudaStream_t st) {
     if (a.z_bf16) b.z_bf16 = a.z_bf16 + c0;
     b.z_ones = (c0 + b.dim == a.dim) ? a.z_ones : 0;   // column a.dim, written by the last chunk
     cudaError_t e;
-    if (bf) {
+    static const int csr_flat = [] { const char* v = std::getenv("APT_AGG_CSR_FLAT"); return v ? atoi(v) : 1; }();
+    const int Vb = int(ceil_div(b.dim, 8));
+    if (bf && csr_flat && Vb > 16 && Vb <= 32 && !b.deg_override && !b.filt_part && b.z_bf16 && !b.z_f32 &&
+        (a.x_pitch * 2) % 16 == 0 && (reinterpret_cast<uintptr_t>(a.xb) & 15) == 0) {
+      b.xb = a.xb + c0;
+      const int64_t blocks = grid_cap(ceil_div(b.max_dst * 32, 256), 4);
+      launch_pdl(agg_csr_b8_kernel, dim3(blocks), dim3(256), 0, st, b, uint32_t(a.x_pitch * 2));
+      e = cudaGetLastError();
+    } else if (bf) {
       CsrSrc s{b.indptr, b.indices, a.xb + c0, a.x_pitch * 2};
       e = dispatch_agg<8>(b, s, 4, st);
     } else {
