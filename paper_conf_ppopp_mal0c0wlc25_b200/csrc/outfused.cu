@@ -73,6 +73,9 @@ __global__ void __launch_bounds__(kWarps * 32, 1) out_fused_kernel(OutFusedArgs 
     y[q] = i < n ? a.labels[a.seeds[i]] : 0;
   }
   // 1. the mean
+  uint64_t hbase;   // the lane's column base in H^{K-1} (lanes past the row's vectors: vector 0)
+  asm("mov.b64 %0, %1;" : "=l"(hbase) : "l"(reinterpret_cast<uint64_t>(a.hb) + uint64_t(lane < V ? lane : 0) * 16u));
+  const uint32_t hrb = uint32_t(a.hb_pitch * 2);
 #pragma unroll 1
   for (int q = 0; q < kRows / kWarps; ++q) {
     const int rl = warp + q * kWarps;
@@ -91,13 +94,14 @@ __global__ void __launch_bounds__(kWarps * 32, 1) out_fused_kernel(OutFusedArgs 
           uint4 v[4];
 #pragma unroll
           for (int qq = 0; qq < 4; ++qq) {
-            const int uu = __shfl_sync(0xffffffffu, u, (e + qq) & 31);
-            v[qq] = (e + qq < m && lane < V) ? __ldg(reinterpret_cast<const uint4*>(a.hb + int64_t(uu) * a.hb_pitch + lane * 8))
-                                             : make_uint4(0, 0, 0, 0);
+            // always-valid rows (lanes past the count hold row 0): one IMAD.WIDE per edge,
+            // padding zeroed by a select, the adds unconditional
+            const uint32_t uu = __shfl_sync(0xffffffffu, uint32_t(u), (e + qq) & 31);
+            const uint4 t = __ldg(reinterpret_cast<const uint4*>(hbase + uint64_t(uu) * hrb));
+            v[qq] = e + qq < m ? t : make_uint4(0, 0, 0, 0);
           }
 #pragma unroll
-          for (int qq = 0; qq < 4; ++qq)
-            if (e + qq < m) accumulate_bf16x8(acc, v[qq]);
+          for (int qq = 0; qq < 4; ++qq) accumulate_bf16x8(acc, v[qq]);
         }
       }
     }
