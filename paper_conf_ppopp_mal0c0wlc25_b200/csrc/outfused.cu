@@ -10,7 +10,7 @@
 //   0. (before griddepcontrol.wait) W^K (bf16, <= 64 x 256) into shared memory -- the
 //      step's weights change only in the SGD at its end;
 //   1. the mean: a warp per row, lane j owns the row's 16-byte vector j, in-edges summed
-//      in CSR order in fp32 (4 source rows in flight) -- the same order and the same
+//      in CSR order in fp32 (8 source rows in flight) -- the same order and the same
 //      mixed-precision adds as agg_kernel, the same reciprocal division (O5) and bf16
 //      rounding (R5), so Z is bit-identical to the unfused path; Z goes to shared memory
 //      and to global (with the all-ones bias-gradient column) for the weight gradient;
@@ -31,6 +31,7 @@ constexpr int kKMax = 256;         // d_in (multiple of 8)
 constexpr int kNMax = 64;          // classes
 constexpr int kSP = kKMax + 8;     // shared row stride (bf16): 528 B, conflict-free fragment loads
 constexpr int kGS = kNMax + 8;     // G row stride (bf16): 144 B
+constexpr int kEB = 8;             // source rows in flight per warp in the mean (a fanout-10 row: 8 + 2)
 
 __device__ __forceinline__ void mma_bf16_16816(float* c, const uint32_t* a, const uint32_t* b) {
   asm volatile(
@@ -90,10 +91,10 @@ __global__ void __launch_bounds__(kWarps * 32, 1) out_fused_kernel(OutFusedArgs 
       for (int c0 = 0; c0 < cnt; c0 += 32) {
         const int u = c0 + lane < cnt ? a.indices[e0 + c0 + lane] : 0;
         const int m = min(32, cnt - c0);
-        for (int e = 0; e < m; e += 4) {
-          uint4 v[4];
+        for (int e = 0; e < m; e += kEB) {
+          uint4 v[kEB];
 #pragma unroll
-          for (int qq = 0; qq < 4; ++qq) {
+          for (int qq = 0; qq < kEB; ++qq) {
             // always-valid rows (lanes past the count hold row 0): one IMAD.WIDE per edge,
             // padding zeroed by a select, the adds unconditional
             const uint32_t uu = __shfl_sync(0xffffffffu, uint32_t(u), (e + qq) & 31);
@@ -101,7 +102,7 @@ __global__ void __launch_bounds__(kWarps * 32, 1) out_fused_kernel(OutFusedArgs 
             v[qq] = e + qq < m ? t : make_uint4(0, 0, 0, 0);
           }
 #pragma unroll
-          for (int qq = 0; qq < 4; ++qq) accumulate_bf16x8(acc, v[qq]);
+          for (int qq = 0; qq < kEB; ++qq) accumulate_bf16x8(acc, v[qq]);
         }
       }
     }
