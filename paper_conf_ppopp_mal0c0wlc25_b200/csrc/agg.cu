@@ -428,7 +428,8 @@ cudaError_t launch_agg_fstore(const AggArgs& a, const FeatView& fv, cudaStream_t
 // lane's opaque column base, unconditional loads of always-valid rows (lanes past the
 // row's count hold row 0), padding zeroed by selects.  Same edge order, same adds, same
 // division and rounding: Z is bit-identical to agg_kernel's.
-__global__ void __launch_bounds__(256, 4) agg_csr_b8_kernel(AggArgs a, uint32_t rb) {
+template <int NB, int MINB>   // source rows in flight per warp, blocks per SM
+__global__ void __launch_bounds__(256, MINB) agg_csr_b8_kernel(AggArgs a, uint32_t rb) {
   APT_PDL_PROLOGUE();
   const int lane = lane_id();
   const int64_t n_dst = *a.n_dst;
@@ -447,16 +448,16 @@ __global__ void __launch_bounds__(256, 4) agg_csr_b8_kernel(AggArgs a, uint32_t 
       const uint32_t u = c0 + lane < cnt ? uint32_t(a.indices[e0 + c0 + lane]) : 0u;
       const int m = min(32, cnt - c0);
 #pragma unroll 1
-      for (int j = 0; j < m; j += 4) {
-        uint4 v[4];
+      for (int j = 0; j < m; j += NB) {
+        uint4 v[NB];
 #pragma unroll
-        for (int q = 0; q < 4; ++q) {
+        for (int q = 0; q < NB; ++q) {
           const uint32_t uq = __shfl_sync(0xffffffffu, u, (j + q) & 31);
           const uint4 t = __ldg(reinterpret_cast<const uint4*>(base + uint64_t(uq) * rb));
           v[q] = j + q < m ? t : make_uint4(0, 0, 0, 0);
         }
 #pragma unroll
-        for (int q = 0; q < 4; ++q) accumulate_vec<8>(acc, v[q]);
+        for (int q = 0; q < NB; ++q) accumulate_vec<8>(acc, v[q]);
       }
     }
     if (a.z_ones && lane == 0) a.z_bf16[i * a.z_bf16_pitch + a.dim] = 0x3F80;
@@ -496,8 +497,11 @@ cudaError_t launch_agg_csr(const AggArgs& a, cudaStream_t st) {
     if (bf && csr_flat && Vb > 16 && Vb <= 32 && !b.deg_override && !b.filt_part && b.z_bf16 && !b.z_f32 &&
         (a.x_pitch * 2) % 16 == 0 && (reinterpret_cast<uintptr_t>(a.xb) & 15) == 0) {
       b.xb = a.xb + c0;
-      const int64_t blocks = grid_cap(ceil_div(b.max_dst * 32, 256), 4);
-      launch_pdl(agg_csr_b8_kernel, dim3(blocks), dim3(256), 0, st, b, uint32_t(a.x_pitch * 2));
+      // APT_CSR_NB: rows in flight per warp (4 at 4 blocks/SM, 6 at 4, 8 at 3; A/B)
+      static const int nb = [] { const char* v = std::getenv("APT_CSR_NB"); return v ? atoi(v) : 4; }();
+      auto kern = nb >= 8 ? agg_csr_b8_kernel<8, 3> : nb >= 6 ? agg_csr_b8_kernel<6, 4> : agg_csr_b8_kernel<4, 4>;
+      const int64_t blocks = grid_cap(ceil_div(b.max_dst * 32, 256), nb >= 8 ? 3 : 4);
+      launch_pdl(kern, dim3(blocks), dim3(256), 0, st, b, uint32_t(a.x_pitch * 2));
       e = cudaGetLastError();
     } else if (bf) {
       CsrSrc s{b.indptr, b.indices, a.xb + c0, a.x_pitch * 2};
